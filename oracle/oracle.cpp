@@ -1,0 +1,242 @@
+// ORACLE -- test infrastructure only.  Plain, slow, obviously-correct CPU
+// definition of what Medusa's parameter-restoration hot path computes.
+//
+// Only tests/, __graft_entry__.smoke() and bench.py (cpu_baseline / --impl
+// reference) may load this library.  It shares no code, header, table or
+// constant with the CUDA path (paper_conf_asplos_zengxgcl25_b200/csrc); the
+// record layout below is restated here from the paper-derived ABI contract.
+//
+// Paper: Zeng et al., "Medusa: Accelerating Serverless LLM Inference with
+// Materialization", ASPLOS'25 -- /root/reference/PAPER.md, cited as P:<line>.
+//
+// Functions and what pins them (tests/test_oracle_*.py):
+//   oracle_check_trace   -- trace well-formedness (readings R-Q7,
+//                           R-ORDER).  Pinned by brute.py's O(n^2) pair check.
+//   oracle_materialize   -- indirect-index-pointer analysis, §4.1 P:204-212:
+//                           for every 8-byte word of every node, the allocation
+//                           live at the node's launch that holds the word
+//                           ("identical or within the range").  Pinned
+//                           by brute.py's literal backward scan, the
+//                           Fig. 6 example, generator ground
+//                           truth and the round trip.
+//   oracle_pack_slots    -- formats the slot list in the ABI layout (mask bit
+//                           per word, per-2048-word chunk prefix, (id<<40|off)
+//                           records).  Pinned by unpacking tests.
+//   oracle_restore       -- replay-based data pointer restoration, §4.2
+//                           P:214-216 (new address of allocation i + offset),
+//                           with per-slot validation (DESIGN.md R-Q8),
+//                           and the kernel-address fill.
+//                           Pinned by identity, constant shift, untouched
+//                           constants, fault injection (closed forms).
+#include <cstdint>
+#include <cstring>
+#include <map>
+#include <vector>
+#include <algorithm>
+
+namespace {
+
+struct Alloc {           // one allocation of the trace; index = allocation ordinal
+    uint64_t base;
+    uint64_t size;
+    uint32_t t_alloc;    // event position of the allocation call
+    uint32_t t_free;     // event position of the free (0xFFFFFFFF = end of time)
+};
+static_assert(sizeof(Alloc) == 24, "trace record is 24 bytes");
+
+const int OK = 0, ERR_INVALID_ARG = -1, ERR_TRACE = -2;
+
+// Event kinds; at equal positions a FREE happens before a LAUNCH before an
+// ALLOC, which is what the strict inequalities t_alloc < t < t_free say.
+enum { EV_FREE = 0, EV_LAUNCH = 1, EV_ALLOC = 2 };
+struct Event { uint32_t t; int kind; uint64_t who; };
+bool ev_less(const Event& a, const Event& b) {
+    if (a.t != b.t) return a.t < b.t;
+    if (a.kind != b.kind) return a.kind < b.kind;
+    return a.who < b.who;
+}
+
+int check_args(uint64_t n_words, const uint64_t* node_off, uint32_t n_nodes,
+               const uint32_t* node_t, const Alloc* a, uint32_t n_alloc) {
+    // Limits of the slot encoding (id < 2^24, offset < 2^40) and image shape.
+    if (n_alloc > (1u << 24)) return ERR_INVALID_ARG;
+    if (n_words > 0xFFFFFFFFull) return ERR_INVALID_ARG;
+    for (uint32_t i = 0; i < n_alloc; ++i) {
+        if (a[i].size > (1ull << 40)) return ERR_INVALID_ARG;
+        if (a[i].base + a[i].size < a[i].base) return ERR_INVALID_ARG;  // wraps past 2^64
+    }
+    if (node_off[0] != 0) return ERR_INVALID_ARG;
+    for (uint32_t j = 0; j < n_nodes; ++j)
+        if (node_off[j + 1] < node_off[j]) return ERR_INVALID_ARG;
+    if (node_off[n_nodes] != n_words) return ERR_INVALID_ARG;
+    // Nodes are listed in launch order ("the sequence of the allocation
+    // and cudaLaunchKernel()"; reading R-ORDER).
+    for (uint32_t j = 0; j + 1 < n_nodes; ++j)
+        if (!(node_t[j] < node_t[j + 1])) return ERR_INVALID_ARG;
+    return OK;
+}
+
+// Well-formed trace: the i-th allocation is the i-th in time, every
+// allocation is freed after it is made, and two allocations that are live at
+// the same moment never share an address (a real allocator never hands out
+// overlapping live memory; DESIGN.md R-Q7).  Lifetimes are open intervals
+// (t_alloc, t_free).
+int check_trace(const Alloc* a, uint32_t n_alloc) {
+    for (uint32_t i = 0; i < n_alloc; ++i) {
+        if (!(a[i].t_alloc < a[i].t_free)) return ERR_TRACE;
+        if (i + 1 < n_alloc && !(a[i].t_alloc < a[i + 1].t_alloc)) return ERR_TRACE;
+    }
+    std::vector<Event> ev;
+    for (uint32_t i = 0; i < n_alloc; ++i) {
+        ev.push_back({a[i].t_alloc, EV_ALLOC, i});
+        ev.push_back({a[i].t_free, EV_FREE, i});
+    }
+    std::sort(ev.begin(), ev.end(), ev_less);
+    std::map<uint64_t, uint32_t> live;  // base -> allocation index, live and non-empty
+    for (const Event& e : ev) {
+        const Alloc& x = a[e.who];
+        if (x.size == 0) continue;  // an empty range overlaps nothing
+        if (e.kind == EV_FREE) { live.erase(x.base); continue; }
+        uint64_t end = x.base + x.size;
+        auto succ = live.lower_bound(x.base);
+        if (succ != live.end() && succ->first < end) return ERR_TRACE;
+        if (succ != live.begin()) {
+            auto pred = std::prev(succ);
+            if (pred->first + a[pred->second].size > x.base) return ERR_TRACE;
+        }
+        live[x.base] = (uint32_t)e.who;
+    }
+    return OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int oracle_check(uint64_t n_words, const uint64_t* node_off, uint32_t n_nodes,
+                 const uint32_t* node_t, const void* allocs, uint32_t n_alloc) {
+    const Alloc* a = (const Alloc*)allocs;
+    int st = check_args(n_words, node_off, n_nodes, node_t, a, n_alloc);
+    if (st != OK) return st;
+    return check_trace(a, n_alloc);
+}
+
+// MATERIALIZE (§4.1).  For node j (launched at t_j) and word g of j with
+// value w, the indirect index pointer is
+//     cand(g) = the i with t_alloc_i < t_j < t_free_i and base_i <= w < base_i + size_i
+// (unique on a well-formed trace; the paper's backward search from the launch,
+// P:212, with the liveness condition of DESIGN.md R-Q1).  Words with no
+// candidate are constants.  Outputs, per word: is_slot[g], id[g],
+// off[g]; returns the status and *n_slots.
+int oracle_materialize(const uint64_t* words, uint64_t n_words, const uint64_t* node_off,
+                       uint32_t n_nodes, const uint32_t* node_t, const void* allocs,
+                       uint32_t n_alloc, uint8_t* is_slot, uint32_t* slot_id,
+                       uint64_t* slot_off, uint64_t* n_slots) {
+    const Alloc* a = (const Alloc*)allocs;
+    *n_slots = 0;
+    int st = oracle_check(n_words, node_off, n_nodes, node_t, allocs, n_alloc);
+    if (st != OK) return st;
+    for (uint64_t g = 0; g < n_words; ++g) { is_slot[g] = 0; slot_id[g] = 0; slot_off[g] = 0; }
+
+    // Sweep the one total order of allocation, free and launch events.
+    std::vector<Event> ev;
+    for (uint32_t i = 0; i < n_alloc; ++i) {
+        ev.push_back({a[i].t_alloc, EV_ALLOC, i});
+        ev.push_back({a[i].t_free, EV_FREE, i});
+    }
+    for (uint32_t j = 0; j < n_nodes; ++j) ev.push_back({node_t[j], EV_LAUNCH, j});
+    std::sort(ev.begin(), ev.end(), ev_less);
+
+    std::map<uint64_t, uint32_t> live;  // base -> index of the live allocation there
+    for (const Event& e : ev) {
+        if (e.kind == EV_ALLOC) {
+            if (a[e.who].size != 0) live[a[e.who].base] = (uint32_t)e.who;
+        } else if (e.kind == EV_FREE) {
+            if (a[e.who].size != 0) live.erase(a[e.who].base);
+        } else {
+            uint32_t j = (uint32_t)e.who;
+            for (uint64_t g = node_off[j]; g < node_off[j + 1]; ++g) {
+                uint64_t w = words[g];
+                auto it = live.upper_bound(w);      // first live base > w
+                if (it == live.begin()) continue;   // no live allocation starts at or below w
+                --it;                               // the live allocation with the largest base <= w
+                const Alloc& x = a[it->second];
+                if (w - x.base < x.size) {          // base <= w < base + size
+                    is_slot[g] = 1;
+                    slot_id[g] = it->second;
+                    slot_off[g] = w - x.base;
+                }
+            }
+        }
+    }
+    uint64_t n = 0;
+    for (uint64_t g = 0; g < n_words; ++g) n += is_slot[g];
+    *n_slots = n;
+    return OK;
+}
+
+// The ABI layout of the indirect-index-pointer table: bit g%32 of
+// mask[g/32] marks word g; chunk_base[c] = number of slots among words
+// [0, 2048*c); record k (k-th slot in word order) = id << 40 | offset.
+void oracle_pack_slots(const uint8_t* is_slot, const uint32_t* slot_id, const uint64_t* slot_off,
+                       uint64_t n_words, uint32_t* mask, uint32_t* chunk_base, uint64_t* records) {
+    const uint64_t CHUNK = 2048;
+    uint64_t n_mask = (n_words + 31) / 32, n_chunks = (n_words + CHUNK - 1) / CHUNK;
+    for (uint64_t m = 0; m < n_mask; ++m) mask[m] = 0;
+    uint64_t k = 0;
+    for (uint64_t g = 0; g < n_words; ++g) {
+        if (g % CHUNK == 0) chunk_base[g / CHUNK] = (uint32_t)k;
+        if (is_slot[g]) {
+            mask[g / 32] |= 1u << (g % 32);
+            records[k] = ((uint64_t)slot_id[g] << 40) | slot_off[g];
+            ++k;
+        }
+    }
+    chunk_base[n_chunks] = (uint32_t)k;
+}
+
+// RESTORE (§4.2) + kernel address fill (§5).  dst starts as a copy of src
+// (constants are restored as their plain values).  Each slot (g, i, off):
+//   i >= n_alloc                        -> bad id
+//   off >= new_size[i]                  -> bad range
+//   src[g] != old_base[i] + off         -> stale (the image no longer holds the
+//                                          materialized pointer)
+//   otherwise dst[g] = new_base[i] + off   (the i-th replayed allocation)
+// A failing slot keeps src[g] and is counted; first_bad_word is the least g.
+// Gather: func_out[j] = table[f_j] if f_j < K and table[f_j] != 0, else 0 (counted).
+// report = {n_bad_slot, first_bad_word, n_bad_id, n_bad_range, n_stale,
+//           n_bad_func, first_bad_node, 0}; "none" = UINT64_MAX.
+void oracle_restore(const uint64_t* src, uint64_t* dst, uint64_t n_words,
+                    const uint64_t* slot_g, const uint32_t* slot_id, const uint64_t* slot_off,
+                    uint64_t n_slots, const uint64_t* old_base, const uint64_t* new_base,
+                    const uint64_t* new_size, uint32_t n_alloc, const uint32_t* func_id,
+                    uint64_t* func_out, uint32_t n_nodes, const uint64_t* table, uint32_t n_func,
+                    uint64_t* report) {
+    uint64_t r[8] = {0, UINT64_MAX, 0, 0, 0, 0, UINT64_MAX, 0};
+    std::vector<uint64_t> out(src, src + n_words);
+    for (uint64_t k = 0; k < n_slots; ++k) {
+        uint64_t g = slot_g[k], i = slot_id[k], off = slot_off[k];
+        int bad = 0;
+        if (i >= n_alloc) { r[2]++; bad = 1; }
+        else if (off >= new_size[i]) { r[3]++; bad = 1; }
+        else if (src[g] != old_base[i] + off) { r[4]++; bad = 1; }
+        else out[g] = new_base[i] + off;
+        if (bad) { r[0]++; if (g < r[1]) r[1] = g; }
+    }
+    for (uint64_t g = 0; g < n_words; ++g) dst[g] = out[g];
+    if (func_id != nullptr) {
+        for (uint32_t j = 0; j < n_nodes; ++j) {
+            uint32_t f = func_id[j];
+            if (f < n_func && table[f] != 0) {
+                func_out[j] = table[f];
+            } else {
+                func_out[j] = 0;
+                r[5]++;
+                if (j < r[6]) r[6] = j;
+            }
+        }
+    }
+    for (int q = 0; q < 8; ++q) report[q] = r[q];
+}
+
+}  // extern "C"
