@@ -1,0 +1,207 @@
+/*
+ * medusa.h -- C ABI of libmedusa.so, the B200 (sm_100a) implementation of the
+ * data-parallel hot path of Medusa's CUDA-graph state materialization
+ * (Zeng et al., "Medusa: Accelerating Serverless LLM Inference with
+ * Materialization", ASPLOS'25; citations P:<line> are lines of the paper text).
+ *
+ *   medusa_materialize      offline: indirect-index-pointer analysis (§4.1,
+ *                           P:204-212) of every 8-byte word of every captured
+ *                           kernel node's parameter image against the
+ *                           allocation trace -> the indirect index pointer
+ *                           table.
+ *   medusa_kernel_table_set online: install the kernel addresses resolved by the
+ *                           triggering kernels (§5).
+ *   medusa_restore          online: replay-based data pointer restoration
+ *                           (§4.2) with per-slot validation
+ *                           and the kernel-address fill of every node.
+ *
+ * Conventions (all entry points)
+ *   - d_* arguments are DEVICE pointers on the calling thread's current CUDA
+ *     device; h_* are host pointers.  All memory is owned by the caller; the
+ *     library never frees caller memory.  It owns only a per-device kernel
+ *     address table and internal scratch that it allocates itself.
+ *   - 64-bit values are little-endian; pointers to u64 arrays must be 8-byte
+ *     aligned (16-byte alignment of word arrays enables the vectorised path).
+ *   - The return value reports argument, trace and launch errors only.
+ *     Data-dependent validation failures of a restore are not call errors:
+ *     they are counted in the device-side medusa_report (the call is async).
+ *   - Thread-safe: calls may come from several host threads and devices.
+ *   - There is no CPU fallback: without a usable sm_100a device every call
+ *     that would touch the GPU returns MEDUSA_ERR_CUDA.
+ */
+#ifndef MEDUSA_H
+#define MEDUSA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#ifndef __DRIVER_TYPES_H__
+typedef struct CUstream_st *cudaStream_t; /* identical to CUDA's own typedef */
+#endif
+
+typedef enum {
+    MEDUSA_OK = 0,
+    MEDUSA_ERR_INVALID_ARG = -1, /* bad pointer/size/alignment, or an input that breaks
+                                    the contract below (limits, CSR shape, launch order) */
+    MEDUSA_ERR_TRACE = -2,       /* allocation trace is not well-formed (see medusa_materialize) */
+    MEDUSA_ERR_CAPACITY = -3,    /* slot table too small; *h_n_slots holds the size needed */
+    MEDUSA_ERR_NO_TABLE = -4,    /* restore asked for the kernel-address fill before any
+                                    medusa_kernel_table_set on this device */
+    MEDUSA_ERR_CUDA = -5         /* CUDA runtime error; see medusa_last_cuda_error() */
+} medusa_status;
+
+/* One allocation of the trace, 24 bytes.  Its index in the trace array is the
+ * allocation ordinal -- the paper's "indirect index pointer" i: "if a pointer is
+ * returned by the i-th buffer allocation, its corresponding indirect index
+ * pointer is i".  base/size: the returned address and the recorded
+ * extent [base, base+size).  t_alloc/t_free: positions of the allocation and of
+ * its free in the one total order of allocation, free and cudaLaunchKernel
+ * events.  t_free = MEDUSA_T_END: never freed.  The allocation is live
+ * at event position t iff t_alloc < t < t_free. */
+typedef struct {
+    uint64_t base;
+    uint64_t size;
+    uint32_t t_alloc;
+    uint32_t t_free;
+} medusa_alloc;
+
+/* The materialized indirect-index-pointer table, in device memory the
+ * caller owns.  For an image of n_words words:
+ *   d_mask:       u32[ceil(n_words/32)]; bit (g % 32) of d_mask[g / 32] is 1 iff
+ *                 word g is a data pointer slot;
+ *   d_chunk_base: u32[ceil(n_words/MEDUSA_CHUNK_WORDS) + 1]; entry c = number of
+ *                 slots among words [0, c*MEDUSA_CHUNK_WORDS); the last entry is
+ *                 the total;
+ *   d_slot:       u64[capacity]; the k-th slot in word order as
+ *                 (allocation index << MEDUSA_OFF_BITS) | byte offset.        */
+typedef struct {
+    uint32_t *d_mask;
+    uint32_t *d_chunk_base;
+    uint64_t *d_slot;
+    uint64_t capacity;
+} medusa_slots;
+
+/* Restore report (device memory, 64 bytes).  "none" = UINT64_MAX.
+ *   n_bad_slot     slots that failed validation (= n_bad_id + n_bad_range + n_stale);
+ *                  a failing slot leaves the source word in place
+ *   first_bad_word least word index of a failing slot
+ *   n_bad_id       slot's allocation index >= n_alloc of the replay
+ *   n_bad_range    slot's offset >= the replayed allocation's size
+ *   n_stale        source word != old_base[i] + offset (the image no longer holds
+ *                  the pointer that was materialized)
+ *   n_bad_func     nodes whose kernel-name id is >= the table size or maps to 0
+ *                  (unresolved); their func_out is 0
+ *   first_bad_node least such node index
+ *   reserved       0 (used internally while the call is in flight)            */
+typedef struct {
+    uint64_t n_bad_slot, first_bad_word, n_bad_id, n_bad_range, n_stale;
+    uint64_t n_bad_func, first_bad_node, reserved;
+} medusa_report;
+
+#define MEDUSA_CHUNK_WORDS 2048u   /* chunk size of d_chunk_base (fixed; part of the ABI) */
+#define MEDUSA_ID_BITS 24u         /* allocation index < 2^24 */
+#define MEDUSA_OFF_BITS 40u        /* byte offset < 2^40 */
+#define MEDUSA_T_END 0xFFFFFFFFu   /* t_free of an allocation that is never freed */
+
+/* medusa_materialize -- offline analysis stage (§4.1).
+ *
+ * Inputs (device):
+ *   d_words[n_words]          every kernel node's parameter image (the bytes the
+ *                             node's param array points to), each zero-
+ *                             padded to a multiple of 8 bytes and concatenated in
+ *                             node order; word g = the u64 at byte 8*g;
+ *   d_node_word_off[n_nodes+1] CSR: node j owns words [off[j], off[j+1]);
+ *                             off[0] = 0, non-decreasing, off[n_nodes] = n_words;
+ *   d_node_t[n_nodes]         event position of node j's cudaLaunchKernel; nodes
+ *                             are listed in launch order (strictly increasing);
+ *   d_alloc[n_alloc]          the allocation trace.
+ * Output: *slots filled (see medusa_slots), *h_n_slots = number of slots.
+ *
+ * Semantics: word g of node j with value w is a slot (i, w - base_i) iff
+ * allocation i is live at node j's launch and base_i <= w < base_i + size_i
+ * ("identical or within the range of the allocated buffer").  On a
+ * well-formed trace at most one such i exists; it is exactly the first match of
+ * the paper's backward search from the launch among allocations not yet
+ * freed ("kernels would always use the allocated buffers before they have been
+ * deallocated").  Every other word is a constant.
+ *
+ * Errors:
+ *   MEDUSA_ERR_INVALID_ARG: null pointers where data is needed; n_alloc > 2^24;
+ *     n_words >= 2^32; some size > 2^40 or base + size wraps past 2^64; the CSR
+ *     is malformed; node times not strictly increasing.
+ *   MEDUSA_ERR_TRACE: t_alloc not strictly increasing in the index, some
+ *     t_alloc >= t_free, or two allocations live at the same time overlap in
+ *     address (zero-size allocations overlap nothing).
+ *   MEDUSA_ERR_CAPACITY: slots->capacity < number of slots.  d_mask and
+ *     d_chunk_base are complete, d_slot holds the first `capacity` records and
+ *     *h_n_slots the number needed.
+ * On INVALID_ARG / TRACE the outputs are unspecified and *h_n_slots = 0.
+ * Work is ordered on `stream`; the call synchronizes `stream` before returning
+ * (it reads the slot count back).  Scratch is allocated by the library.      */
+medusa_status medusa_materialize(const uint64_t *d_words, uint64_t n_words,
+                                 const uint64_t *d_node_word_off, uint32_t n_nodes,
+                                 const uint32_t *d_node_t,
+                                 const medusa_alloc *d_alloc, uint32_t n_alloc,
+                                 medusa_slots *slots, uint64_t *h_n_slots,
+                                 cudaStream_t stream);
+
+/* medusa_kernel_table_set -- install, for the current device, the kernel
+ * address of every kernel-name id: d_func_addr[n_func] (device),
+ * 0 = unresolved.  In the paper these come from dlsym / cudaGetFuncBySymbol and,
+ * for kernels hidden from the symbol tables, from enumerating the modules that
+ * the triggering kernels (the model's first layer) loaded.
+ * The copy is ordered on `stream`; a later medusa_restore must be ordered after
+ * it (same stream, or an event).  Replaces any previous table of this device. */
+medusa_status medusa_kernel_table_set(const uint64_t *d_func_addr, uint32_t n_func,
+                                      cudaStream_t stream);
+
+/* medusa_restore -- online restoration (§4.2; §5).
+ *
+ *   dst = src; then for every slot k (word g, allocation i, offset off) of the
+ *   table produced by medusa_materialize:
+ *     i >= n_alloc                   -> n_bad_id
+ *     off >= d_new_size[i]           -> n_bad_range
+ *     src[g] != d_old_base[i] + off  -> n_stale          (u64 wrap-around)
+ *     otherwise dst[g] = d_new_base[i] + off              (u64 wrap-around)
+ *   d_new_base[i] is the address the i-th allocation returned when the
+ *   (de)allocation sequence was replayed.  Non-slot words
+ *   are copied unchanged (constants keep their plain values).
+ *   Kernel-address fill: d_func_out[j] = table[d_func_id[j]] if the id is below
+ *   the installed table's size and the entry is non-zero, else 0 (n_bad_func).
+ *   d_func_id, d_func_out, n_nodes: all NULL/0 to skip the fill.
+ *
+ * src/dst: u64[n_words], device; dst == src (in place) is allowed, any other
+ * overlap is MEDUSA_ERR_INVALID_ARG.  slots: as produced by medusa_materialize
+ * for this image (n_slots = *h_n_slots).  d_old_base: the trace's base of each
+ * allocation (the materialization-time addresses).  d_report (device) is
+ * written completely by the call.  Fully asynchronous on `stream`; capturable
+ * into a CUDA graph.                                                         */
+medusa_status medusa_restore(const uint64_t *d_src_words, uint64_t *d_dst_words, uint64_t n_words,
+                             const medusa_slots *slots, uint64_t n_slots,
+                             const uint64_t *d_old_base, const uint64_t *d_new_base,
+                             const uint64_t *d_new_size, uint32_t n_alloc,
+                             const uint32_t *d_func_id, uint64_t *d_func_out, uint32_t n_nodes,
+                             medusa_report *d_report, cudaStream_t stream);
+
+/* cudaError_t value behind the last MEDUSA_ERR_CUDA returned on this thread. */
+int medusa_last_cuda_error(void);
+
+/* Human-readable name of a status code (static storage). */
+const char *medusa_status_string(medusa_status status);
+
+/* ---- instrumentation (optional; off by default) --------------------------
+ * When enabled on a thread, every kernel libmedusa launches from that thread is
+ * bracketed by CUDA events recorded on its launch stream.  medusa_timing_read
+ * waits for those events and returns up to `max` (name, milliseconds) pairs of
+ * the launches since the last read (then forgets them).                      */
+void medusa_timing_enable(int on);
+int medusa_timing_read(const char **names, float *ms, int max);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MEDUSA_H */

@@ -1,0 +1,225 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, bit-exact.
+
+Every comparison is element by element on the same seeded inputs: the
+materialized table (mask, chunk prefix, records), the restored words, the
+kernel-address fill and the report.  Sizes: the toy set and the three
+single-model BASELINE configs in full, the ten-model set (139,364 nodes) in
+full, in the launch configuration bench.py times.
+"""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover - CPU-only hosts
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import oracle  # noqa: E402
+import paper_conf_asplos_zengxgcl25_b200 as medusa  # noqa: E402
+from tests.tiny import tiny_trace  # noqa: E402
+from workloads import ALLOC_DTYPE, T_NEVER  # noqa: E402
+
+DEV = torch.device("cuda:0")
+
+
+def _h(t):
+    return t.detach().cpu().numpy()
+
+
+def _oracle_full(words, node_off, node_t, allocs, new_base, new_size, func_id=None, table=None):
+    m = oracle.materialize(words, node_off, node_t, allocs)
+    if m["status"] != 0:
+        return m, None
+    mask, cb, rec = oracle.pack(m, words.size)
+    dst, fout, rep = oracle.restore(words, m["slot_g"], m["slot_id"], m["slot_off"], allocs["base"], new_base,
+                                    new_size, func_id, table)
+    return m, (mask, cb, rec, dst, fout, rep)
+
+
+def _check_materialize(slots, m, packed, n_words):
+    mask, cb, rec = packed[:3]
+    assert slots.n_slots == m["n_slots"]
+    assert np.array_equal(_h(slots.mask).view(np.uint32), mask)
+    assert np.array_equal(_h(slots.chunk_base).view(np.uint32), cb)
+    assert np.array_equal(_h(slots.slot)[: slots.n_slots].view(np.uint64), rec)
+
+
+@pytest.mark.parametrize("name", ["toy", "qwen1.5-4b", "llama2-7b", "llama2-13b", "all10"])
+def test_full_path_parity(graph_sets, name):
+    gs = graph_sets(name)
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    medusa.kernel_table_set(inp["table"])
+    dst, fout, rep = medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"],
+                                    inp["func_id"])
+    torch.cuda.synchronize()
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size,
+                             gs.func_id, gs.table)
+    assert m["status"] == 0
+    _check_materialize(slots, m, packed, gs.n_words)
+    assert np.array_equal(medusa.to_numpy_u64(dst), packed[3])
+    assert np.array_equal(medusa.to_numpy_u64(fout), packed[4])
+    assert np.array_equal(medusa.report_numpy(rep), packed[5])
+    assert medusa.report_numpy(rep)[0] == 0
+
+
+def test_restore_driven_by_oracle_table(graph_sets):
+    """K3+K4 in isolation: the oracle's packed table fed to the GPU restore."""
+    gs = graph_sets("llama2-7b")
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size,
+                             gs.func_id, gs.table)
+    mask, cb, rec, dst_o, fout_o, rep_o = packed
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.Slots(torch.from_numpy(mask.view(np.int32)).to(DEV), torch.from_numpy(cb.view(np.int32)).to(DEV),
+                         torch.from_numpy(rec.view(np.int64)).to(DEV), m["n_slots"])
+    medusa.kernel_table_set(inp["table"])
+    dst, fout, rep = medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"],
+                                    inp["func_id"])
+    assert np.array_equal(medusa.to_numpy_u64(dst), dst_o)
+    assert np.array_equal(medusa.to_numpy_u64(fout), fout_o)
+    assert np.array_equal(medusa.report_numpy(rep), rep_o)
+
+
+def test_in_place_and_misaligned(graph_sets):
+    gs = graph_sets("qwen1.5-4b")
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size)
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    buf = inp["words"].clone()
+    dst, _, rep = medusa.restore(buf, slots, inp["old_base"], inp["new_base"], inp["new_size"], dst=buf)
+    assert dst.data_ptr() == buf.data_ptr()
+    assert np.array_equal(medusa.to_numpy_u64(buf), packed[3])
+    # 8-byte but not 16-byte aligned image and output: scalar path, same bytes
+    big = torch.zeros(gs.n_words + 1, dtype=torch.int64, device=DEV)
+    big[1:] = inp["words"]
+    out = torch.zeros(gs.n_words + 1, dtype=torch.int64, device=DEV)
+    src_v, dst_v = big[1:], out[1:]
+    slots2 = medusa.materialize(src_v, inp["node_off"], inp["node_t"], inp["allocs"])
+    _check_materialize(slots2, m, packed, gs.n_words)
+    medusa.restore(src_v, slots2, inp["old_base"], inp["new_base"], inp["new_size"], dst=dst_v)
+    assert np.array_equal(medusa.to_numpy_u64(dst_v), packed[3])
+
+
+def test_fault_injection_matches_oracle(graph_sets):
+    gs = graph_sets("toy")
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+    g = m["slot_g"]
+    src = gs.words.copy()
+    src[g[5]] ^= np.uint64(8)  # STALE
+    src[g[33]] ^= np.uint64(16)
+    new_size = gs.new_size.copy()
+    k = int(np.flatnonzero(m["slot_off"] > 0)[2])
+    new_size[m["slot_id"][k]] = m["slot_off"][k]  # OOR for every slot of that allocation at off >= size
+    table = gs.table.copy()
+    table[gs.func_id[7]] = 0  # unresolved kernels
+    fid = gs.func_id.copy()
+    fid[3] = table.size + 5
+    n_alloc_replay = int(m["slot_id"].max())  # the last allocation(s) missing from the replay: BAD_ID
+    ob, nb, ns = gs.allocs["base"][:n_alloc_replay], gs.new_base[:n_alloc_replay], new_size[:n_alloc_replay]
+    dst_o, fout_o, rep_o = oracle.restore(src, m["slot_g"], m["slot_id"], m["slot_off"], ob, nb, ns, fid, table)
+    assert rep_o[2] > 0 and rep_o[3] > 0 and rep_o[4] == 2 and rep_o[5] > 0
+    t = lambda a, dt=torch.int64: torch.from_numpy(np.ascontiguousarray(a).view(np.int64 if dt == torch.int64 else np.int32)).to(DEV)
+    medusa.kernel_table_set(t(table))
+    dst, fout, rep = medusa.restore(t(src), slots, t(ob), t(nb), t(ns), t(fid, torch.int32))
+    assert np.array_equal(medusa.to_numpy_u64(dst), dst_o)
+    assert np.array_equal(medusa.to_numpy_u64(fout), fout_o)
+    assert np.array_equal(medusa.report_numpy(rep), rep_o)
+    # the report is rewritten completely by the next call
+    medusa.kernel_table_set(inp["table"])
+    _, _, rep2 = medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"],
+                                inp["func_id"])
+    r2 = medusa.report_numpy(rep2)
+    assert r2[0] == 0 and r2[1] == np.uint64(2**64 - 1) and r2[5] == 0 and r2[7] == 0
+
+
+def _run_tiny(words, off, node_t, allocs):
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(DEV)
+    aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3) if allocs.size else np.zeros((0, 3), np.int64)
+    try:
+        s = medusa.materialize(t(words, np.int64), t(off, np.int64), t(node_t, np.int32),
+                               torch.from_numpy(aa).to(DEV))
+        return 0, s
+    except medusa.MedusaError as e:
+        return e.status, None
+
+
+@pytest.mark.parametrize("overlap_p", [0.0, 0.2])
+def test_tiny_traces_status_and_slots(overlap_p):
+    """Adversarial tiny traces (reuse, adjacency, zero sizes, equal positions,
+    empty nodes, malformed traces): status and table identical to the oracle."""
+    for seed in range(300):
+        words, off, node_t, allocs = tiny_trace(seed * 7 + int(overlap_p * 1000), overlap_p=overlap_p)
+        st, s = _run_tiny(words, off, node_t, allocs)
+        m = oracle.materialize(words, off, node_t, allocs)
+        assert st == m["status"], (seed, st, m["status"])
+        if st == 0:
+            mask, cb, rec = oracle.pack(m, words.size)
+            assert s.n_slots == m["n_slots"]
+            assert np.array_equal(_h(s.mask).view(np.uint32), mask), seed
+            assert np.array_equal(_h(s.chunk_base).view(np.uint32), cb), seed
+            assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec), seed
+
+
+def test_edge_cases():
+    b = 0x7F00_0000_0000
+    A = lambda rows: np.array(rows, dtype=ALLOC_DTYPE)
+    # empty image, no nodes
+    st, s = _run_tiny(np.zeros(0, np.uint64), np.zeros(1, np.uint64), np.zeros(0, np.uint32), A([]))
+    assert st == 0 and s.n_slots == 0 and _h(s.chunk_base)[0] == 0
+    # nodes but no words; allocations but no words
+    st, s = _run_tiny(np.zeros(0, np.uint64), np.zeros(4, np.uint64), np.array([3, 5, 9], np.uint32),
+                      A([(b, 64, 1, T_NEVER)]))
+    assert st == 0 and s.n_slots == 0
+    # no allocations: everything is a constant
+    w = np.arange(5000, dtype=np.uint64) + np.uint64(b)
+    st, s = _run_tiny(w, np.array([0, 4999, 5000], np.uint64), np.array([1, 2], np.uint32), A([]))
+    assert st == 0 and s.n_slots == 0
+    # one allocation covering a ragged multi-chunk image: every word a slot
+    w = np.uint64(b) + np.arange(5000, dtype=np.uint64) * np.uint64(8)
+    st, s = _run_tiny(w, np.array([0, 1, 4096, 5000], np.uint64), np.array([2, 3, 4], np.uint32),
+                      A([(b, 8 * 5000, 1, T_NEVER)]))
+    assert st == 0 and s.n_slots == 5000
+    assert (_h(s.slot)[:5000] == np.arange(5000) * 8).all()
+    # a single node spanning many chunks with its allocation freed before it launches
+    st, s = _run_tiny(w, np.array([0, 5000], np.uint64), np.array([9], np.uint32), A([(b, 8 * 5000, 1, 9)]))
+    assert st == 0 and s.n_slots == 0
+    # invalid arguments detected on the device
+    st, _ = _run_tiny(w[:4], np.array([0, 3, 2, 4], np.uint64), np.array([1, 2, 3], np.uint32), A([]))
+    assert st == medusa.ERR_INVALID_ARG
+    st, _ = _run_tiny(w[:4], np.array([0, 2, 4], np.uint64), np.array([2, 2], np.uint32), A([]))
+    assert st == medusa.ERR_INVALID_ARG
+    st, _ = _run_tiny(w[:4], np.array([0, 4], np.uint64), np.array([2], np.uint32), A([(b, (1 << 40) + 8, 1, 3)]))
+    assert st == medusa.ERR_INVALID_ARG
+    st, _ = _run_tiny(w[:4], np.array([0, 4], np.uint64), np.array([2], np.uint32), A([(b, 64, 3, 3)]))
+    assert st == medusa.ERR_TRACE
+
+
+def test_capacity_too_small(graph_sets):
+    gs = graph_sets("toy")
+    m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+    inp = medusa.upload(gs, DEV)
+    with pytest.raises(medusa.MedusaError) as ei:
+        medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], capacity=10)
+    assert ei.value.status == medusa.ERR_CAPACITY and ei.value.n_slots == m["n_slots"]
+    s = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], capacity=m["n_slots"])
+    assert s.n_slots == m["n_slots"]
+
+
+def test_multi_chunk_malformed_ten_model_trace(graph_sets):
+    """A single overlapping allocation injected into the full ten-model trace is rejected."""
+    gs = graph_sets("all10")
+    allocs = gs.allocs.copy()
+    i = int(np.flatnonzero(gs.alloc_kind == 5)[5000])  # a capture temporary
+    j = i + 1
+    while allocs["size"][j] == 0 or not (allocs["t_alloc"][j] < allocs["t_free"][i]):
+        j += 1
+    allocs["base"][j] = allocs["base"][i] + np.uint64(8)  # overlaps i while both live
+    assert oracle.check(gs.n_words, gs.node_word_off, gs.node_t, allocs) == oracle.ERR_TRACE
+    inp = medusa.upload(gs, DEV)
+    aa = torch.from_numpy(np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3)).to(DEV)
+    with pytest.raises(medusa.MedusaError) as ei:
+        medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], aa)
+    assert ei.value.status == medusa.ERR_TRACE
