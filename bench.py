@@ -1,0 +1,375 @@
+"""Benchmark of the Medusa restoration hot path on B200 (one JSON line on rank 0).
+
+A step = one pass of the whole hot path over one graph set already resident in
+HBM: medusa_materialize (classify every word + emit the indirect-index-pointer
+table) -> medusa_kernel_table_set -> medusa_restore (relocate + validate every
+slot, fill every node's kernel address).  Metric (BASELINE.json): graph nodes
+restored per second, whole job; plus the relocate pass's HBM GB/s.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload all10] [--impl ours|reference]
+
+N > 1 runs under torchrun: every rank restores its own independent instance
+(seed offset per rank), no data-path collective (weak scaling); NCCL is used
+only for the start/stop barriers and the max-over-ranks of the device time.
+--impl reference times the CPU oracle (oracle/, plain C++) on the same config.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    "all10": ("all10", "ten paper models concatenated (Table 1: 139,364 nodes), one call"),
+    "qwen1.5-4b": ("qwen1.5-4b", "Qwen1.5-4B-shaped graph set, 35 batch sizes (16,150 nodes)"),
+    "llama2-7b": ("llama2-7b", "Llama-2-7B-shaped graph set with kernel table (12,518 nodes)"),
+    "llama2-13b": ("llama2-13b", "Llama-2-13B-shaped instance (16,150 nodes)"),
+    "toy": ("toy", "toy 2-layer decoder, 200 nodes"),
+}
+SEED_STRIDE = 1000  # rank r restores the instance generated with seed + r * SEED_STRIDE
+
+
+def algorithmic_bytes(gs, n_slots, n_func):
+    """Bytes the method itself must move."""
+    W, N, A = gs.n_words, gs.n_nodes, gs.n_alloc
+    n_mask = (W + 31) // 32
+    C = (W + 2047) // 2048
+    restore = (16 * W + 4 * n_mask + 4 * (C + 1) + 8 * n_slots + 24 * A + 12 * N + 8 * n_func + 64)
+    classify = (8 * W + 4 * n_mask + 4 * (C + 1) + 8 * n_slots + 12 * N)
+    return dict(restore=restore, mat_classify=classify)
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def load_traffic():
+    """Per-launch DRAM bytes of each kernel from the committed ncu --set full capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        return json.load(open(p))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.proc = None
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "50",
+                 "-i", str(gpu_index)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out, _ = self.proc.communicate()
+        rows = []
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                rows.append(dict(sm=float(f[1]), max=float(f[2]), power=float(f[3]) if f[3] not in ("[N/A]", "") else 0.0,
+                                 hw=f[5], hwt=f[6], swt=f[7], pcap=f[8]))
+            except ValueError:
+                continue
+        if not rows:
+            return None
+        loaded = [r for r in rows if r["sm"] > 0.5 * r["max"]] or rows
+        reasons = set()
+        for r in rows:
+            for k, nm in (("hw", "hw_slowdown"), ("hwt", "hw_thermal_slowdown"), ("swt", "sw_thermal_slowdown"),
+                          ("pcap", "sw_power_cap")):
+                if r[k].lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(r["sm"] for r in loaded), "sm_max_mhz": max(r["max"] for r in rows),
+                "reasons": sorted(reasons), "samples": len(rows), "samples_under_load": len(loaded)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    return int(os.environ.get("RANK", "0")), ws, int(os.environ.get("LOCAL_RANK", "0"))
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle, as it stands, on this arm's config."""
+    rank, ws, _ = dist_env()
+    if rank != 0:
+        return
+    import __graft_entry__ as ge
+    ge.build_oracle()
+    import oracle
+    from workloads import make_graph_set
+
+    cfg, desc = WORKLOADS[args.workload]
+    gs = make_graph_set(cfg)
+
+    def step():
+        m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+        oracle.restore(gs.words, m["slot_g"], m["slot_id"], m["slot_off"], gs.allocs["base"], gs.new_base,
+                       gs.new_size, gs.func_id, gs.table)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = time.perf_counter() - t0
+    value = gs.n_nodes * args.steps / dt
+    print(json.dumps({
+        "impl": "reference", "metric": "graph nodes restored/sec (materialize + restore, whole hot path)",
+        "value": value, "unit": "nodes/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u64", "data": "synthetic",
+        "config": {"workload": f"{cfg}: {desc}", "nodes": gs.n_nodes, "words": gs.n_words, "allocs": gs.n_alloc},
+        "cpu_baseline": {"value": value, "unit": "nodes/s", "cores": 1, "kind": "oracle",
+                         "sample": f"full {cfg} graph set per step, single-threaded oracle/oracle.cpp (-O2)"},
+        "e2e": {"value": value, "unit": "nodes/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import __graft_entry__ as ge
+    ge.build_medusa()
+    import paper_conf_asplos_zengxgcl25_b200 as medusa
+    from workloads import make_graph_set
+    from workloads.graphset import CONFIGS
+
+    rank, ws, local = dist_env()
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a GPU (there is no CPU fallback)")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    cfg, desc = WORKLOADS[args.workload]
+    seed = CONFIGS[cfg]["seed"] + SEED_STRIDE * rank
+    gs = make_graph_set(cfg, seed=seed)
+    inp = medusa.upload(gs, dev)
+    stream = torch.cuda.current_stream(dev)
+    slots = medusa.alloc_slots(gs.n_words, dev)
+    dst = torch.empty_like(inp["words"])
+    fout = torch.empty(gs.n_nodes, dtype=torch.int64, device=dev)
+    rep = torch.empty(8, dtype=torch.int64, device=dev)
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    scrub = torch.empty(max(2 * l2, 256 << 20) // 4, dtype=torch.int32, device=dev)
+
+    def step():
+        medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots)
+        medusa.kernel_table_set(inp["table"])
+        medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                       dst=dst, func_out=fout, report=rep)
+
+    def barrier():
+        torch.cuda.synchronize(dev)
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    for i in range(max(args.warmup, 3)):
+        scrub.fill_(i)
+        step()
+    torch.cuda.synchronize(dev)
+    assert int(medusa.report_numpy(rep)[0]) == 0, "restore reported validation failures"
+    n_slots = slots.n_slots
+
+    # ---- timed region: K steps, L2 scrubbed (2x L2 write) before each --------------
+    sampler = ClockSampler(local)
+    for i in range(20):  # bring clocks up before the timed steps
+        scrub.fill_(i)
+    medusa.timing_enable(True)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    barrier()
+    for k in range(args.steps):
+        scrub.fill_(k)
+        ev[k][0].record(stream)
+        step()
+        ev[k][1].record(stream)
+    barrier()
+    clocks = sampler.stop()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    launches = medusa.timing_read(1 << 20)
+    medusa.timing_enable(False)
+    total_ms = sum(step_ms)
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if ws > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    max_ms = float(t.item())
+    nodes_total = gs.n_nodes * args.steps * ws
+    value = nodes_total / (max_ms / 1e3)
+
+    # per-kernel device time inside the timed region (events on the launch stream)
+    per = {}
+    for name, ms in launches:
+        d = per.setdefault(name, [0, 0.0])
+        d[0] += 1
+        d[1] += ms
+    alg = algorithmic_bytes(gs, n_slots, gs.table.size)
+    peak, peak_src = measured_peak()
+    traffic = load_traffic()
+    kernels = {}
+    for name, (cnt, ms) in sorted(per.items(), key=lambda kv: -kv[1][1]):
+        avg = ms / cnt
+        entry = {"launches": cnt, "avg_us": 1e3 * avg, "share_of_step": ms / total_ms}
+        if name in alg:
+            entry["alg_bytes"] = alg[name]
+            entry["GB/s"] = alg[name] / (avg / 1e3) / 1e9
+        kernels[name] = entry
+    dom = max((n for n in per if n in alg), key=lambda n: per[n][1])
+    dom_avg_s = per[dom][1] / per[dom][0] / 1e3
+    achieved = alg[dom] / dom_avg_s / 1e9
+    rl = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+          "frac": achieved / peak, "traffic": traffic.get(dom), "peak_source": peak_src,
+          "alg_bytes_per_launch": alg[dom]}
+    rst = per["restore"]
+    restore_avg_s = rst[1] / rst[0] / 1e3
+    relocate = {"kernel": "restore", "GB/s": alg["restore"] / restore_avg_s / 1e9,
+                "frac_of_peak": alg["restore"] / restore_avg_s / 1e9 / peak,
+                "nodes_per_s": gs.n_nodes / restore_avg_s, "avg_us": restore_avg_s * 1e6,
+                "traffic": traffic.get("restore")}
+    mat_s = sum(v[1] for k, v in per.items() if k.startswith("mat_")) / args.steps / 1e3
+
+    # ---- sustained relocate: back-to-back restores of the resident set (no scrub) ----
+    sus = None
+    if args.sustained > 0:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        big = int(args.sustained)
+        e0.record(stream)
+        for _ in range(big):
+            medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                           dst=dst, func_out=fout, report=rep)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        s = e0.elapsed_time(e1) / 1e3 / big
+        sus = {"restores": big, "avg_us": s * 1e6, "GB/s": alg["restore"] / s / 1e9,
+               "note": "back-to-back, L2-warm (set fits in the 126 MB L2): upper bound, not the roofline number"}
+
+    # ---- end to end: pinned host buffers -> H2D -> whole path -> D2H of results ----
+    h = medusa.host_arrays(gs)
+    pinned = {k: torch.from_numpy(v).pin_memory() for k, v in h.items()}
+    out_h = torch.empty(gs.n_words, dtype=torch.int64).pin_memory()
+    fout_h = torch.empty(gs.n_nodes, dtype=torch.int64).pin_memory()
+    rep_h = torch.empty(8, dtype=torch.int64).pin_memory()
+    d_in = {k: torch.empty_like(v, device=dev) for k, v in pinned.items()}
+    h2d = sum(v.numel() * v.element_size() for v in pinned.values())
+    d2h = out_h.numel() * 8 + fout_h.numel() * 8 + 64
+
+    def e2e_step():
+        for k, v in pinned.items():
+            d_in[k].copy_(v, non_blocking=True)
+        medusa.materialize(d_in["words"], d_in["node_off"], d_in["node_t"], d_in["allocs"], out=slots)
+        medusa.kernel_table_set(d_in["table"])
+        medusa.restore(d_in["words"], slots, d_in["old_base"], d_in["new_base"], d_in["new_size"],
+                       d_in["func_id"], dst=dst, func_out=fout, report=rep)
+        out_h.copy_(dst, non_blocking=True)
+        fout_h.copy_(fout, non_blocking=True)
+        rep_h.copy_(rep, non_blocking=True)
+
+    for _ in range(2):
+        e2e_step()
+    barrier()
+    e2e_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for k in range(args.steps):
+        e2e_ev[k][0].record(stream)
+        e2e_step()
+        e2e_ev[k][1].record(stream)
+    barrier()
+    e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_ev)
+    t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+    if ws > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    e2e_value = nodes_total / (float(t.item()) / 1e3)
+    assert np.array_equal(out_h.numpy().view(np.uint64), medusa.to_numpy_u64(dst))
+
+    # ---- CPU baseline: the oracle as it stands, rank 0 at N=1 only ----
+    cpu = None
+    if ws == 1 and not args.no_cpu_baseline:
+        ge.build_oracle()
+        import oracle
+        reps, t_cpu, t0 = 0, 0.0, time.perf_counter()
+        while time.perf_counter() - t0 < args.cpu_seconds:
+            t1 = time.perf_counter()
+            m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+            oracle.restore(gs.words, m["slot_g"], m["slot_id"], m["slot_off"], gs.allocs["base"], gs.new_base,
+                           gs.new_size, gs.func_id, gs.table)
+            t_cpu += time.perf_counter() - t1
+            reps += 1
+        cpu = {"value": gs.n_nodes * reps / t_cpu, "unit": "nodes/s", "cores": 1, "kind": "oracle",
+               "sample": f"the full per-rank {cfg} set, {reps} passes (materialize + restore), "
+                         f"single-threaded oracle/oracle.cpp; host has {os.cpu_count()} cores"}
+
+    if rank == 0:
+        line = {
+            "metric": "graph nodes restored/sec (materialize + restore, whole hot path)",
+            "value": value, "unit": "nodes/s", "n_gpus": ws, "steps": args.steps, "warmup": max(args.warmup, 3),
+            "ms_per_step": max_ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u64", "data": "synthetic",
+            "config": {"workload": f"{cfg} per rank: {desc}", "nodes_per_rank": gs.n_nodes, "words": gs.n_words,
+                       "allocs": gs.n_alloc, "slots": n_slots, "kernel_names": int(gs.table.size),
+                       "l2": f"scrubbed before every timed step ({scrub.numel() * 4 >> 20} MiB write; L2 {l2 >> 20} MiB)",
+                       "seed": seed, "parallelism": f"{ws} independent instances, no collective"},
+            "roofline": rl,
+            "relocate": relocate,
+            "materialize_ms": mat_s * 1e3,
+            "kernels": kernels,
+            "sustained_relocate": sus,
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+            "gpu_launches": len(launches),
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS), default="all10")
+    ap.add_argument("--sustained", type=int, default=200, help="back-to-back restores for the L2-warm figure")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -7,28 +7,33 @@
 // Structure of a well-formed trace that the GPU design exploits:
 //  * I = allocations live at the LAST launch T_last.  All of them are live at
 //    the same instant, so they are pairwise address-disjoint: one global list
-//    sorted by base answers "which I-allocation holds w" with one binary search;
-//    it is live at t <= T_last iff t_alloc < t.  (weights, KV cache, static
-//    inputs, permanent buffers: ~27k entries for the ten-model set.)
+//    sorted by base answers "which I-allocation holds w" with one search; it is
+//    live at t <= T_last iff t_alloc < t.  (Weights, KV cache, static inputs,
+//    permanent buffers: ~27k entries for the ten-model set.)
 //  * M = every other allocation ("mortal": capture temporaries, warm-up and
 //    profiling scratch).  Their lifetimes are short, so each is registered in
 //    the word chunks whose launch-time span its lifetime touches; a chunk's
 //    mortal window (~60-150 entries) is sorted by base in shared memory and
 //    searched with a prefix-max-of-end backward walk plus the time check.
 //  * Well-formedness (no two simultaneously-live allocations overlap) is checked
-//    exactly: I-I by adjacency of the sorted list, M-I by an address-run walk
-//    over the sorted I list, M-M inside blocks of 64 allocation ordinals
-//    against the mortals registered as live there.
+//    exactly: I-I by adjacency of the sorted list, M-I with per-32-entry
+//    min(t_alloc) / max(t_free) summaries of the sorted list over the address
+//    run a mortal meets, M-M inside blocks of 64 allocation ordinals against the
+//    mortals registered as live there.
 // Pipeline (all on `stream`; one host synchronization at the end):
-//   k_nodes_chunks  CSR / launch-order checks, per-chunk launch-time span
+//   k_nodes_chunks  CSR / launch-order checks; per-chunk first/last node
 //   k_allocs        trace checks, I/M split, registration counts, prefilter
 //   k_scan          registration offsets (single CTA)
-//   k_scatter       registration lists
+//   k_scatter       registration lists (32-byte window records)
 //   k_sort_tile + k_merge (x log)   I sorted by (base, index)
-//   k_build_i       I arrays, I-I check, fences
+//   k_build_i       I arrays, I-I check, fences, block summaries
 //   k_check         M-M and M-I overlap checks
-//   k_classify      classify every word + ballot/popc emission with a decoupled
-//                   look-back over chunks (persistent CTAs, ticketed chunks)
+//   k_classify      one CTA per 2048-word chunk: TMA bulk copy of the chunk's
+//                   words to shared memory, mortal-window search, I-list search
+//                   through a shared queue, mask words + warp-dense staging of
+//                   the records + the chunk's slot count (no inter-CTA waits)
+//   k_emit          decoupled look-back over the chunk counts -> chunk_base,
+//                   compaction of the staged records into the slot table
 #include <algorithm>
 #include <mutex>
 #include <vector>
@@ -40,13 +45,15 @@ namespace {
 
 constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kAblk = 64;          // allocation ordinals per overlap-check block
-constexpr int kChkCap = 1024;      // registered mortals staged per check batch
-constexpr int kSortTile = 2048;
+constexpr int kChkCap = 256;       // registered mortals staged per check batch
+constexpr int kSortTile = 8192;    // elements sorted per CTA before the merge passes
+constexpr int kMergeTile = 2048;   // outputs per CTA of a merge pass
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
-constexpr int kWinCap = 512;       // mortal-window entries per batch (power of two)
+constexpr int kWinCap = 256;       // mortal-window entries per batch (power of two)
 constexpr int kClsThreads = 256;
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kClsThreads;  // 8
 constexpr int kWarps = kClsThreads / 32;
+constexpr int kIBlk = 32;          // I-list summary block
 constexpr unsigned long long LB_AGG = 1ull << 62, LB_PRE = 2ull << 62, LB_VAL = (1ull << 62) - 1;
 
 struct Ctl {
@@ -60,10 +67,19 @@ struct Ctl {
     unsigned long long n_slots;
 };
 
-struct IRest {
+struct IRest {  // I-list entry (sorted order), base kept in a separate array
     uint64_t end;
     uint32_t t_alloc;
     uint32_t id;
+};
+
+struct WinRec {  // a registered mortal allocation
+    uint64_t base;
+    uint64_t end;
+    uint32_t t_alloc;
+    uint32_t t_free;
+    uint32_t id;
+    uint32_t pad;
 };
 
 struct Dev {  // scratch of one call (device pointers)
@@ -72,13 +88,17 @@ struct Dev {  // scratch of one call (device pointers)
     uint4* rng;                                  // [n]: c_lo, c_hi, b_lo, b_hi
     uint32_t *cnt_c, *fill_c, *off_c;            // [C+1]
     uint32_t *cnt_b, *fill_b, *off_b;            // [nb+1]
-    uint32_t *list_c, *list_b;
+    WinRec *list_c, *list_b;
     uint64_t cap_c, cap_b;
-    uint64_t *sk0, *sk1;                         // [n] sort keys
-    uint32_t *sv0, *sv1;                         // [n] sort values
+    uint64_t* sk[2];                             // [n] sort keys (ping-pong)
+    uint32_t* sv[2];                             // [n] sort values
     uint64_t* i_base;                            // [n]
     IRest* i_rest;                               // [n]
+    uint32_t* i_tf;                              // [n]
+    uint32_t *blk_min_ta, *blk_max_tf;           // [n/32]
     uint64_t* fence;                             // [kFenceCap]
+    uint32_t* chunk_cnt;                         // [C]
+    uint64_t* staging;                           // [n_words] records, warp-dense per 32 words
     unsigned long long* lookback;                // [C]
 };
 
@@ -89,16 +109,6 @@ struct P {  // kernel parameters
 };
 
 __device__ __forceinline__ void flag(Ctl* c, unsigned int bit) { atomicOr(&c->status, bit); }
-
-// largest j in [0, N-1] with node_off[j] <= g (N >= 1)
-__device__ __forceinline__ uint32_t node_of(const uint64_t* off, uint32_t N, uint64_t g) {
-    uint32_t lo = 0, hi = N;  // count of node_off[1..N] <= g
-    while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (off[mid + 1] <= g) lo = mid + 1; else hi = mid;
-    }
-    return lo < N ? lo : N - 1;
-}
 
 __device__ __forceinline__ bool kv_less(uint64_t ka, uint32_t va, uint64_t kb, uint32_t vb) {
     return ka < kb || (ka == kb && va < vb);
@@ -113,93 +123,142 @@ __device__ __forceinline__ void st_release(unsigned long long* p, unsigned long 
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+__device__ __forceinline__ uint64_t warp_min_u64(uint64_t v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v = min(v, (uint64_t)__shfl_xor_sync(0xffffffffu, v, d));
+    return v;
+}
+__device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v = max(v, (uint64_t)__shfl_xor_sync(0xffffffffu, v, d));
+    return v;
+}
+
+// number of merge passes that do work for nI keys (the tile sort writes buffer 1)
+__device__ __forceinline__ int merge_passes(uint32_t nI) {
+    int e = 0;
+    for (uint64_t w = kSortTile; w < nI; w *= 2) ++e;
+    return e;
+}
+
 // ----------------------------------------------------------------------------
-// 1. nodes and chunks
+// 1. nodes and chunks: CSR / order checks; node j writes the chunks whose first
+//    or last word it holds (no search)
 __global__ void k_nodes_chunks(P p) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const MaterializeArgs& a = p.a;
     const uint32_t N = a.n_nodes;
-    if (i <= N) {
-        if (i == 0 && a.node_off[0] != 0) flag(p.d.ctl, ST_INVALID);
-        if (i == N && a.node_off[N] != a.n_words) flag(p.d.ctl, ST_INVALID);
-        if (i < N && a.node_off[i + 1] < a.node_off[i]) flag(p.d.ctl, ST_INVALID);
-        if (i + 1 < N && !(a.node_t[i] < a.node_t[i + 1])) flag(p.d.ctl, ST_INVALID);
+    if (i > N) return;
+    const uint64_t o0 = a.node_off[i];
+    if (i == 0 && o0 != 0) flag(p.d.ctl, ST_INVALID);
+    if (i == N) {
+        if (o0 != a.n_words) flag(p.d.ctl, ST_INVALID);
+        return;
     }
-    if (i < p.C && N > 0) {
-        const uint64_t cs = i * kChunkWords;
+    const uint64_t o1 = a.node_off[i + 1];
+    const uint32_t t = a.node_t[i];
+    if (o1 < o0) { flag(p.d.ctl, ST_INVALID); return; }
+    if (i + 1 < N && !(t < a.node_t[i + 1])) flag(p.d.ctl, ST_INVALID);
+    if (o1 == o0 || o1 > a.n_words) return;
+    for (uint64_t c = o0 / kChunkWords; c <= (o1 - 1) / kChunkWords; ++c) {
+        const uint64_t cs = c * kChunkWords;
         const uint64_t ce = min(cs + kChunkWords, a.n_words) - 1;
-        const uint32_t jf = node_of(a.node_off, N, cs), jl = node_of(a.node_off, N, ce);
-        p.d.jf[i] = jf;
-        p.d.jl[i] = jl;
-        p.d.tmin[i] = a.node_t[jf];
-        p.d.tmax[i] = a.node_t[jl];
+        if (o0 <= cs) { p.d.jf[c] = (uint32_t)i; p.d.tmin[c] = t; }
+        if (ce < o1) { p.d.jl[c] = (uint32_t)i; p.d.tmax[c] = t; }
     }
 }
 
 // ----------------------------------------------------------------------------
 // 2. allocations: checks, I/M split, registration ranges and counts
-__global__ void k_allocs(P p) {
+__global__ void __launch_bounds__(256) k_allocs(P p) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     const MaterializeArgs& a = p.a;
-    if (i >= a.n_alloc) return;
-    const medusa_alloc x = a.alloc[i];
-    if (x.size > (1ull << MEDUSA_OFF_BITS) || x.base + x.size < x.base) flag(p.d.ctl, ST_INVALID);
-    if (!(x.t_alloc < x.t_free)) flag(p.d.ctl, ST_TRACE);
-    if (i + 1 < a.n_alloc && !(x.t_alloc < a.alloc[i + 1].t_alloc)) flag(p.d.ctl, ST_TRACE);
+    const uint32_t lane = threadIdx.x & 31;
+    const bool valid = i < a.n_alloc;
+    medusa_alloc x{};
+    if (valid) x = a.alloc[i];
+    const uint32_t N = a.n_nodes;
+    const uint32_t t_last = N ? a.node_t[N - 1] : 0;
+    bool isI = false;
     uint4 r = make_uint4(1, 0, 1, 0);  // empty ranges
-    if (x.size != 0) {
-        atomicMax(&p.d.ctl->gmin_c, ~(unsigned long long)x.base);
-        atomicMax(&p.d.ctl->gmax, (unsigned long long)(x.base + x.size));
-        const uint32_t N = a.n_nodes;
-        const uint32_t t_last = N ? a.node_t[N - 1] : 0;
-        if (N && x.t_alloc < t_last && t_last < x.t_free) {
-            const unsigned int pos = atomicAdd(&p.d.ctl->nI, 1u);
-            p.d.sk0[pos] = x.base;
-            p.d.sv0[pos] = i;
-        } else {
-            if (p.C && N) {
-                uint32_t lo = 0, hi = p.C;  // first chunk whose last launch is after t_alloc
-                while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.tmax[m] > x.t_alloc) hi = m; else lo = m + 1; }
-                const uint32_t c_lo = lo;
-                lo = 0; hi = p.C;  // chunks whose first launch is before t_free
-                while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.tmin[m] < x.t_free) lo = m + 1; else hi = m; }
-                if (c_lo < lo) {
-                    r.x = c_lo; r.y = lo - 1;
-                    for (uint32_t c = r.x; c <= r.y; ++c) atomicAdd(&p.d.cnt_c[c], 1u);
+    if (valid) {
+        if (x.size > (1ull << MEDUSA_OFF_BITS) || x.base + x.size < x.base) flag(p.d.ctl, ST_INVALID);
+        if (!(x.t_alloc < x.t_free)) flag(p.d.ctl, ST_TRACE);
+        if (i + 1 < a.n_alloc && !(x.t_alloc < a.alloc[i + 1].t_alloc)) flag(p.d.ctl, ST_TRACE);
+        if (x.size != 0) {
+            isI = N && x.t_alloc < t_last && t_last < x.t_free;
+            if (!isI) {
+                if (p.C && N) {
+                    uint32_t lo = 0, hi = p.C;  // first chunk whose last launch is after t_alloc
+                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.tmax[m] > x.t_alloc) hi = m; else lo = m + 1; }
+                    const uint32_t c_lo = lo;
+                    lo = c_lo; hi = p.C;  // chunks whose first launch is before t_free
+                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.tmin[m] < x.t_free) lo = m + 1; else hi = m; }
+                    if (c_lo < lo) {
+                        r.x = c_lo; r.y = lo - 1;
+                        for (uint32_t c = r.x; c <= r.y; ++c) atomicAdd(&p.d.cnt_c[c], 1u);
+                    }
+                }
+                // ordinals allocated while i is live: (i, u), u = #{k : t_alloc_k < t_free_i}
+                uint32_t lo = i + 1, hi = a.n_alloc;
+                while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.alloc[m].t_alloc < x.t_free) lo = m + 1; else hi = m; }
+                if (i + 1 < lo) {
+                    r.z = (i + 1) / kAblk; r.w = (lo - 1) / kAblk;
+                    for (uint32_t b = r.z; b <= r.w; ++b) atomicAdd(&p.d.cnt_b[b], 1u);
                 }
             }
-            // ordinals allocated while i is live: (i, u) with u = #{k : t_alloc_k < t_free_i}
-            uint32_t lo = i + 1, hi = a.n_alloc;
-            while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.alloc[m].t_alloc < x.t_free) lo = m + 1; else hi = m; }
-            if (i + 1 < lo) {
-                r.z = (i + 1) / kAblk; r.w = (lo - 1) / kAblk;
-                for (uint32_t b = r.z; b <= r.w; ++b) atomicAdd(&p.d.cnt_b[b], 1u);
-            }
         }
+        p.d.rng[i] = r;
     }
-    p.d.rng[i] = r;
+    // warp-aggregated: I positions, global prefilter bounds
+    const uint32_t bal = __ballot_sync(0xffffffffu, isI);
+    uint32_t base_pos = 0;
+    if (lane == 0 && bal) base_pos = atomicAdd(&p.d.ctl->nI, (unsigned)__popc(bal));
+    base_pos = __shfl_sync(0xffffffffu, base_pos, 0);
+    if (isI) {
+        const uint32_t pos = base_pos + __popc(bal & lanemask_lt());
+        p.d.sk[0][pos] = x.base;
+        p.d.sv[0][pos] = i;
+    }
+    const bool live = valid && x.size != 0;
+    const uint64_t mn = warp_min_u64(live ? x.base : ~0ull);
+    const uint64_t mx = warp_max_u64(live ? x.base + x.size : 0ull);
+    if (lane == 0 && mx) {
+        atomicMax(&p.d.ctl->gmin_c, ~(unsigned long long)mn);
+        atomicMax(&p.d.ctl->gmax, (unsigned long long)mx);
+    }
 }
 
 // ----------------------------------------------------------------------------
-// 3. exclusive scans of the registration counts (one CTA)
+// 3. exclusive scans of the registration counts (one CTA of 1024 threads)
 __device__ void block_exclusive_scan(const uint32_t* cnt, uint32_t* off, uint32_t n, unsigned long long* total) {
-    __shared__ unsigned long long s_part[1024];
-    const uint32_t T = blockDim.x, tid = threadIdx.x;
+    __shared__ unsigned long long s_w[32];
+    const uint32_t T = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t per = (n + T - 1) / T;
-    const uint32_t b = tid * per, e = min(b + per, n);
+    const uint32_t b = min(tid * per, n), e = min(b + per, n);
     unsigned long long s = 0;
     for (uint32_t k = b; k < e; ++k) s += cnt[k];
-    s_part[tid] = s;
-    __syncthreads();
-    for (uint32_t d = 1; d < T; d <<= 1) {
-        unsigned long long v = tid >= d ? s_part[tid - d] : 0;
-        __syncthreads();
-        s_part[tid] += v;
-        __syncthreads();
+    unsigned long long incl = s;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += y;
     }
-    unsigned long long run = s_part[tid] - s;
+    if (lane == 31) s_w[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+        unsigned long long v = lane < T / 32 ? s_w[lane] : 0, iv = v;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const unsigned long long y = __shfl_up_sync(0xffffffffu, iv, d);
+            if (lane >= d) iv += y;
+        }
+        s_w[lane] = iv - v;  // exclusive prefix of warp totals
+    }
+    __syncthreads();
+    unsigned long long run = s_w[warp] + incl - s;
     for (uint32_t k = b; k < e; ++k) { off[k] = (uint32_t)min(run, 0xFFFFFFFFull); run += cnt[k]; }
-    if (tid == T - 1) { *total = s_part[T - 1]; off[n] = (uint32_t)min(s_part[T - 1], 0xFFFFFFFFull); }
+    if (tid == T - 1) { *total = run; off[n] = (uint32_t)min(run, 0xFFFFFFFFull); }
     __syncthreads();
 }
 
@@ -210,30 +269,36 @@ __global__ void __launch_bounds__(1024) k_scan(P p) {
         flag(p.d.ctl, ST_OVERFLOW);
 }
 
-// 4. registration lists
+// 4. registration lists (32-byte records, so readers need no second gather)
 __global__ void k_scatter(P p) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= p.a.n_alloc) return;
     const uint4 r = p.d.rng[i];
+    if (r.x > r.y && r.z > r.w) return;
+    const medusa_alloc x = p.a.alloc[i];
+    const WinRec w{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
     for (uint32_t c = r.x; c <= r.y; ++c) {
         const uint64_t pos = (uint64_t)p.d.off_c[c] + atomicAdd(&p.d.fill_c[c], 1u);
-        if (pos < p.d.cap_c) p.d.list_c[pos] = i;
+        if (pos < p.d.cap_c) p.d.list_c[pos] = w;
     }
     for (uint32_t b = r.z; b <= r.w; ++b) {
         const uint64_t pos = (uint64_t)p.d.off_b[b] + atomicAdd(&p.d.fill_b[b], 1u);
-        if (pos < p.d.cap_b) p.d.list_b[pos] = i;
+        if (pos < p.d.cap_b) p.d.list_b[pos] = w;
     }
 }
 
 // ----------------------------------------------------------------------------
-// 5. sort I by (base, index): bitonic tiles of 2048, then merge-path passes
-__global__ void __launch_bounds__(1024) k_sort_tile(const Ctl* ctl, const uint64_t* kin, const uint32_t* vin,
-                                                    uint64_t* kout, uint32_t* vout) {
-    __shared__ uint64_t sk[kSortTile];
-    __shared__ uint32_t sv[kSortTile];
-    const uint32_t n = ctl->nI;
+// 5. sort I by (base, index): bitonic tiles of 8192 in shared memory, then
+//    merge-path passes (only those the device-side count needs do any work)
+__global__ void __launch_bounds__(1024) k_sort_tile(P p) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    uint64_t* sk = reinterpret_cast<uint64_t*>(smem_raw);
+    uint32_t* sv = reinterpret_cast<uint32_t*>(sk + kSortTile);
+    const uint32_t n = p.d.ctl->nI;
     const uint32_t t0 = blockIdx.x * kSortTile;
     if (t0 >= n) return;
+    const uint64_t* kin = p.d.sk[0];
+    const uint32_t* vin = p.d.sv[0];
     for (uint32_t q = threadIdx.x; q < kSortTile; q += blockDim.x) {
         const bool in = t0 + q < n;
         sk[q] = in ? kin[t0 + q] : ~0ull;
@@ -254,36 +319,63 @@ __global__ void __launch_bounds__(1024) k_sort_tile(const Ctl* ctl, const uint64
         }
     }
     for (uint32_t q = threadIdx.x; q < kSortTile && t0 + q < n; q += blockDim.x) {
-        kout[t0 + q] = sk[q];
-        vout[t0 + q] = sv[q];
+        p.d.sk[1][t0 + q] = sk[q];
+        p.d.sv[1][t0 + q] = sv[q];
     }
 }
 
-__global__ void __launch_bounds__(256) k_merge(const Ctl* ctl, const uint64_t* kin, const uint32_t* vin,
-                                               uint64_t* kout, uint32_t* vout, uint32_t width) {
-    __shared__ uint64_t sk[kSortTile];
-    __shared__ uint32_t sv[kSortTile];
+// smallest i in [lo, hi) with less(B[d-1-i], A[i]), else hi -- warp-cooperative
+// 32-ary search (all lanes return the same value)
+__device__ uint32_t merge_path_warp(const uint64_t* ka, const uint32_t* va, const uint64_t* kb, const uint32_t* vb,
+                                    uint32_t d, uint32_t lo, uint32_t hi) {
+    const uint32_t lane = threadIdx.x & 31;
+    while (lo < hi) {
+        const uint32_t span = hi - lo;
+        const uint32_t step = (span + 31) / 32;
+        const uint32_t pi = lo + lane * step;
+        bool pr = false;
+        if (pi < hi) pr = kv_less(kb[d - 1 - pi], vb[d - 1 - pi], ka[pi], va[pi]);
+        const uint32_t b = __ballot_sync(0xffffffffu, pr);
+        if (step == 1) return b ? lo + (__ffs(b) - 1) : hi;
+        if (b == 0) {  // answer lies after the last probe that was inside [lo, hi)
+            lo = lo + min(31u, (span - 1) / step) * step + 1;
+        } else {
+            const uint32_t f = __ffs(b) - 1;
+            const uint32_t nhi = lo + f * step;
+            lo = f ? lo + (f - 1) * step + 1 : lo;
+            hi = nhi;
+            if (f == 0) return lo;
+        }
+    }
+    return lo;
+}
+
+__global__ void __launch_bounds__(256) k_merge(P p, uint32_t width, int pass) {
+    __shared__ uint64_t sk[kMergeTile];
+    __shared__ uint32_t sv[kMergeTile];
     __shared__ uint32_t s_i0, s_i1;
-    const uint32_t n = ctl->nI;
-    const uint32_t o0 = blockIdx.x * kSortTile;
+    const uint32_t n = p.d.ctl->nI;
+    if (width >= n) return;  // one run already: nothing to merge (no-op pass)
+    const int in = (1 + pass) & 1;
+    const uint64_t* kin = p.d.sk[in];
+    const uint32_t* vin = p.d.sv[in];
+    uint64_t* kout = p.d.sk[in ^ 1];
+    uint32_t* vout = p.d.sv[in ^ 1];
+    const uint32_t o0 = blockIdx.x * kMergeTile;
     if (o0 >= n) return;
     const uint32_t ps = o0 / (2 * width) * (2 * width);
     const uint32_t a0 = ps, a1 = min(ps + width, n), b0 = a1, b1 = min(ps + 2 * width, n);
-    const uint32_t o1 = min(o0 + kSortTile, n);
+    const uint32_t o1 = min(o0 + kMergeTile, n);
     if (a1 >= b1) {  // lone run: copy
         for (uint32_t q = o0 + threadIdx.x; q < o1; q += blockDim.x) { kout[q] = kin[q]; vout[q] = vin[q]; }
         return;
     }
     const uint32_t la = a1 - a0, lb = b1 - b0;
-    if (threadIdx.x < 2) {
-        const uint32_t d = (threadIdx.x == 0 ? o0 : o1) - ps;
-        uint32_t lo = d > lb ? d - lb : 0, hi = min(d, la);
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (kv_less(kin[b0 + d - 1 - mid], vin[b0 + d - 1 - mid], kin[a0 + mid], vin[a0 + mid])) hi = mid;
-            else lo = mid + 1;
-        }
-        if (threadIdx.x == 0) s_i0 = lo; else s_i1 = lo;
+    const uint32_t warp = threadIdx.x >> 5;
+    if (warp < 2) {
+        const uint32_t d = (warp == 0 ? o0 : o1) - ps;
+        const uint32_t r = merge_path_warp(kin + a0, vin + a0, kin + b0, vin + b0, d, d > lb ? d - lb : 0, min(d, la));
+        if ((threadIdx.x & 31) == 0) { if (warp == 0) s_i0 = r; else s_i1 = r; }
     }
     __syncthreads();
     const uint32_t i0 = s_i0, i1 = s_i1;
@@ -295,8 +387,7 @@ __global__ void __launch_bounds__(256) k_merge(const Ctl* ctl, const uint64_t* k
         sv[q] = vin[src];
     }
     __syncthreads();
-    // sa = sk[0..na), sb = sk[na..na+nbb); each thread merges 8 outputs
-    const uint32_t per = kSortTile / 256;
+    const uint32_t per = kMergeTile / 256;
     const uint32_t d = threadIdx.x * per;
     if (d < na + nbb) {
         uint32_t lo = d > nbb ? d - nbb : 0, hi = min(d, na);
@@ -307,7 +398,7 @@ __global__ void __launch_bounds__(256) k_merge(const Ctl* ctl, const uint64_t* k
         }
         uint32_t ia = lo, ib = d - lo;
         for (uint32_t q = 0; q < per && d + q < na + nbb; ++q) {
-            bool takeA = ib >= nbb || (ia < na && kv_less(sk[ia], sv[ia], sk[na + ib], sv[na + ib]));
+            const bool takeA = ib >= nbb || (ia < na && kv_less(sk[ia], sv[ia], sk[na + ib], sv[na + ib]));
             const uint32_t s = takeA ? ia++ : na + ib++;
             kout[o0 + d + q] = sk[s];
             vout[o0 + d + q] = sv[s];
@@ -315,18 +406,33 @@ __global__ void __launch_bounds__(256) k_merge(const Ctl* ctl, const uint64_t* k
     }
 }
 
-// 6. I arrays, I-I adjacency check, shared-memory fences
-__global__ void k_build_i(P p, const uint64_t* sk, const uint32_t* sv) {
+// 6. I arrays, I-I adjacency check, shared-memory fences, 32-entry summaries
+__global__ void __launch_bounds__(256) k_build_i(P p) {
     const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
     const uint32_t nI = p.d.ctl->nI;
-    if (k >= nI) return;
-    const uint32_t id = sv[k];
-    const medusa_alloc x = p.a.alloc[id];
-    p.d.i_base[k] = x.base;
-    p.d.i_rest[k] = IRest{x.base + x.size, x.t_alloc, id};
-    if (k + 1 < nI && x.base + x.size > sk[k + 1]) flag(p.d.ctl, ST_TRACE);
-    const uint32_t stride = (nI + kFenceCap - 1) / kFenceCap;
-    if (k % stride == 0) p.d.fence[k / stride] = x.base;
+    if (k - (threadIdx.x & 31) >= nI) return;  // whole warp past the end
+    const int fin = (1 + merge_passes(nI)) & 1;
+    const uint64_t* sk = p.d.sk[fin];
+    const uint32_t* sv = p.d.sv[fin];
+    uint32_t ta = 0xFFFFFFFFu, tf = 0;
+    if (k < nI) {
+        const uint32_t id = sv[k];
+        const medusa_alloc x = p.a.alloc[id];
+        p.d.i_base[k] = x.base;
+        p.d.i_rest[k] = IRest{x.base + x.size, x.t_alloc, id};
+        p.d.i_tf[k] = x.t_free;
+        ta = x.t_alloc;
+        tf = x.t_free;
+        if (k + 1 < nI && x.base + x.size > sk[k + 1]) flag(p.d.ctl, ST_TRACE);
+        const uint32_t stride = (nI + kFenceCap - 1) / kFenceCap;
+        if (k % stride == 0) p.d.fence[k / stride] = x.base;
+    }
+    const uint32_t mn = __reduce_min_sync(0xffffffffu, ta);
+    const uint32_t mx = __reduce_max_sync(0xffffffffu, tf);
+    if ((threadIdx.x & 31) == 0) {
+        p.d.blk_min_ta[k / kIBlk] = mn;
+        p.d.blk_max_tf[k / kIBlk] = mx;
+    }
 }
 
 // ----------------------------------------------------------------------------
@@ -345,6 +451,7 @@ __global__ void __launch_bounds__(kAblk) k_check(P p) {
         x = a.alloc[j];
         mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
     }
+    const uint64_t xe = x.base + x.size;
     bool bad = false;
     // M-M: registered mortals live at some allocation of this block
     const uint64_t r0 = p.d.off_b[b];
@@ -353,274 +460,335 @@ __global__ void __launch_bounds__(kAblk) k_check(P p) {
         const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
         __syncthreads();
         for (uint32_t q = threadIdx.x; q < m; q += blockDim.x) {
-            const uint32_t i = p.d.list_b[bs + q];
-            const medusa_alloc y = a.alloc[i];
+            const WinRec y = p.d.list_b[bs + q];
             s_base[q] = y.base;
-            s_end[q] = y.base + y.size;
+            s_end[q] = y.end;
             s_tf[q] = y.t_free;
-            s_idx[q] = i;
+            s_idx[q] = y.id;
         }
         __syncthreads();
         if (mine && !bad) {
-            const uint64_t xe = x.base + x.size;
             for (uint32_t q = 0; q < m; ++q) {
                 if (s_idx[q] < j && s_tf[q] > x.t_alloc && s_base[q] < xe && x.base < s_end[q]) { bad = true; break; }
             }
         }
     }
-    // M-I: the I entries whose ranges meet [base, end) form one run of the sorted list
-    if (mine && !bad) {
-        const uint32_t nI = p.d.ctl->nI;
-        const uint64_t xe = x.base + x.size;
-        uint32_t lo = 0, hi = nI;  // count of I bases < xe
+    // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
+    const uint32_t nI = p.d.ctl->nI;
+    if (mine && !bad && nI) {
+        uint32_t lo = 0, hi = nI;  // e = count of I bases < end
         while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.i_base[m] < xe) lo = m + 1; else hi = m; }
-        for (int64_t k = (int64_t)lo - 1; k >= 0; --k) {
-            const IRest e = p.d.i_rest[k];
-            if (e.end <= x.base) break;
-            const uint32_t tf_e = a.alloc[e.id].t_free;
-            if (max(e.t_alloc, x.t_alloc) < min(tf_e, x.t_free)) { bad = true; break; }
+        const uint32_t e = lo;
+        lo = 0; hi = e;            // s = count of I ends <= base (ends ascend on a disjoint list)
+        while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.i_rest[m].end <= x.base) lo = m + 1; else hi = m; }
+        const uint32_t s = lo;
+        // overlap with e in I: freed before T_last -> some t_alloc_e < t_free; else some t_free_e > t_alloc
+        const bool freed_early = x.t_free <= t_last;
+        uint32_t k = s;
+        while (k < e && !bad) {
+            if (k % kIBlk == 0 && k + kIBlk <= e) {
+                bad = freed_early ? p.d.blk_min_ta[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
+                k += kIBlk;
+            } else {
+                bad = freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
+                ++k;
+            }
         }
     }
     if (bad) flag(p.d.ctl, ST_TRACE);
 }
 
 // ----------------------------------------------------------------------------
-// 8. classify + emit
+// 8. classify one chunk per CTA
 struct ClsShared {
+    uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     uint64_t fence[kFenceCap];
-    uint32_t tw[MEDUSA_CHUNK_WORDS];
+    uint32_t tw[MEDUSA_CHUNK_WORDS];     // launch position of every word
     uint64_t key[kWinCap];
     uint64_t end[kWinCap];
     uint64_t pmax[kWinCap];
     uint32_t ta[kWinCap], tf[kWinCap], id[kWinCap];
     uint16_t val[kWinCap];
-    uint32_t cnt[kWordsPerThread][kWarps];
-    uint32_t thr_max[kClsThreads];
-    uint32_t chunk;
-    unsigned long long prefix;
+    uint16_t queue[MEDUSA_CHUNK_WORDS];
+    uint32_t hits[MEDUSA_CHUNK_WORDS / 32];
+    uint32_t wmax[kWarps];
+    uint32_t nq, total;
+    unsigned long long mbar;
 };
 
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
 __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
+    extern __shared__ __align__(128) unsigned char smem_raw[];
     ClsShared& S = *reinterpret_cast<ClsShared*>(smem_raw);
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t c = blockIdx.x;
     Ctl* ctl = p.d.ctl;
+    const uint64_t cs = (uint64_t)c * kChunkWords;
+    const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
+    const uint64_t* gsrc = a.words + cs;
+    const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
+    // 1. the chunk's words -> shared memory with one bulk copy (TMA engine)
+    if (tid == 0) {
+        S.nq = 0;
+        S.total = 0;
+        if (tma) {
+            const uint32_t mb = smem_u32(&S.mbar);
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                         ::"r"(smem_u32(S.words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
+        }
+    }
+    if (!tma)
+        for (uint32_t q = tid; q < n; q += kClsThreads) S.words[q] = ld_stream(gsrc + q);
+    // 2. meanwhile: fences, launch positions, the mortal window
     const uint32_t nI = ctl->nI;
     const uint32_t stride = nI ? (nI + kFenceCap - 1) / kFenceCap : 1;
     const uint32_t nf = (nI + stride - 1) / stride;
     for (uint32_t f = tid; f < nf; f += kClsThreads) S.fence[f] = p.d.fence[f];
     const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
     const uint32_t N = a.n_nodes;
-    const uint64_t n_mask = (a.n_words + 31) / 32;
-
-    for (;;) {
-        __syncthreads();
-        if (tid == 0) S.chunk = atomicAdd(&ctl->ticket, 1u);
-        __syncthreads();
-        const uint32_t c = S.chunk;
-        if (c >= p.C) break;
-        const uint64_t cs = (uint64_t)c * kChunkWords;
-        const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
-        // words first: their latency overlaps everything below
-        uint64_t w[kWordsPerThread];
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            const uint32_t q = k * kClsThreads + tid;
-            w[k] = q < n ? ld_stream(a.words + cs + q) : 0;
+    for (uint32_t q = tid; q < kChunkWords; q += kClsThreads) S.tw[q] = 0;
+    if (tid < MEDUSA_CHUNK_WORDS / 32) S.hits[tid] = 0;
+    const uint64_t r0 = p.d.off_c[c];
+    const uint64_t r1 = min((uint64_t)p.d.off_c[c + 1], p.d.cap_c);
+    __syncthreads();
+    if (N) {
+        const uint32_t jf = min(p.d.jf[c], N - 1), jl = min(p.d.jl[c], N - 1);
+        if (tid == 0) atomicMax(&S.tw[0], a.node_t[jf]);
+        for (uint32_t j = jf + 1 + tid; j <= jl; j += kClsThreads) {
+            const uint64_t q = a.node_off[j] - cs;
+            if (q < n) atomicMax(&S.tw[q], a.node_t[j]);
         }
-        // launch position of every word: node starts carry t_j, then a max-scan
-        for (uint32_t q = tid; q < kChunkWords; q += kClsThreads) S.tw[q] = 0;
+    }
+    __syncthreads();
+    {  // running max over the chunk: tw[q] = launch position of the node holding word q
+        uint32_t loc[kWordsPerThread];
+        uint32_t run = 0;
+#pragma unroll
+        for (int k = 0; k < kWordsPerThread; ++k) { run = max(run, S.tw[tid * kWordsPerThread + k]); loc[k] = run; }
+        uint32_t incl = run;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl = max(incl, y);
+        }
+        if (lane == 31) S.wmax[warp] = incl;
+        const uint32_t up = __shfl_up_sync(0xffffffffu, incl, 1);
         __syncthreads();
-        if (N) {
-            const uint32_t jf = p.d.jf[c], jl = p.d.jl[c];
-            if (tid == 0) atomicMax(&S.tw[0], a.node_t[jf]);
-            for (uint32_t j = jf + 1 + tid; j <= jl; j += kClsThreads) {
-                const uint64_t q = a.node_off[j] - cs;
-                if (q < n) atomicMax(&S.tw[q], a.node_t[j]);
+        uint32_t before = lane ? up : 0;
+        for (uint32_t ww = 0; ww < warp; ++ww) before = max(before, S.wmax[ww]);
+#pragma unroll
+        for (int k = 0; k < kWordsPerThread; ++k) S.tw[tid * kWordsPerThread + k] = max(before, loc[k]);
+    }
+    if (tma) {
+        const uint32_t mb = smem_u32(&S.mbar);
+        uint32_t done = 0;
+        while (!done) {
+            asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
+                         : "=r"(done) : "r"(mb) : "memory");
+        }
+    }
+    __syncthreads();
+    // 3. mortal window(s): sorted by base, prefix max of end, backward walk
+    for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
+        const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
+        uint32_t mp = 32;
+        while (mp < m) mp <<= 1;
+        for (uint32_t q = tid; q < mp; q += kClsThreads) {
+            if (q < m) {
+                const WinRec x = p.d.list_c[bs + q];
+                S.key[q] = x.base;
+                S.end[q] = x.end;
+                S.ta[q] = x.t_alloc;
+                S.tf[q] = x.t_free;
+                S.id[q] = x.id;
+            } else {
+                S.key[q] = ~0ull;
+            }
+            S.val[q] = (uint16_t)q;
+        }
+        __syncthreads();
+        for (uint32_t size = 2; size <= mp; size <<= 1) {
+            for (uint32_t st = size >> 1; st > 0; st >>= 1) {
+                for (uint32_t q = tid; q < mp / 2; q += kClsThreads) {
+                    const uint32_t lo = 2 * q - (q & (st - 1)), hi = lo + st;
+                    const bool up = (lo & size) == 0;
+                    const uint64_t ka = S.key[lo], kb = S.key[hi];
+                    const uint16_t va = S.val[lo], vb = S.val[hi];
+                    if (kv_less(kb, vb, ka, va) == up) { S.key[lo] = kb; S.key[hi] = ka; S.val[lo] = vb; S.val[hi] = va; }
+                }
+                __syncthreads();
             }
         }
-        __syncthreads();
-        {
-            uint32_t loc[kWordsPerThread];
-            uint32_t run = 0;
-#pragma unroll
-            for (int k = 0; k < kWordsPerThread; ++k) { run = max(run, S.tw[tid * kWordsPerThread + k]); loc[k] = run; }
-            uint32_t incl = run;
+        if (warp == 0) {  // prefix max of end in sorted order
+            const uint32_t per = (m + 31) / 32;
+            const uint32_t b = min(lane * per, m), e = min(b + per, m);
+            uint64_t run = 0;
+            for (uint32_t q = b; q < e; ++q) run = max(run, S.end[S.val[q]]);
+            uint64_t incl = run;
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                const uint64_t y = __shfl_up_sync(0xffffffffu, incl, d);
                 if (lane >= d) incl = max(incl, y);
             }
-            S.thr_max[tid] = incl;  // inclusive within the warp
-            __syncthreads();
-            const uint32_t up = __shfl_up_sync(0xffffffffu, incl, 1);
-            uint32_t before = lane ? up : 0;
-            for (uint32_t ww = 0; ww < warp; ++ww) before = max(before, S.thr_max[ww * 32 + 31]);
-            __syncthreads();
-#pragma unroll
-            for (int k = 0; k < kWordsPerThread; ++k) S.tw[tid * kWordsPerThread + k] = max(before, loc[k]);
+            uint64_t acc = __shfl_up_sync(0xffffffffu, incl, 1);
+            if (lane == 0) acc = 0;
+            for (uint32_t q = b; q < e; ++q) { acc = max(acc, S.end[S.val[q]]); S.pmax[q] = acc; }
         }
         __syncthreads();
-        uint32_t t[kWordsPerThread];
-        bool cand[kWordsPerThread], hit[kWordsPerThread];
-        uint32_t hid[kWordsPerThread];
-        uint64_t hoff[kWordsPerThread];
-#pragma unroll
+#pragma unroll 2
         for (int k = 0; k < kWordsPerThread; ++k) {
             const uint32_t q = k * kClsThreads + tid;
-            t[k] = S.tw[q];
-            cand[k] = q < n && w[k] >= gmin && w[k] < gmax;
-            hit[k] = false;
-            hid[k] = 0;
-            hoff[k] = 0;
-        }
-        // mortal window(s): sorted by base, prefix max of end, backward walk
-        const uint64_t r0 = p.d.off_c[c];
-        const uint64_t r1 = min((uint64_t)p.d.off_c[c + 1], p.d.cap_c);
-        for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
-            const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
-            uint32_t mp = 32;
-            while (mp < m) mp <<= 1;
-            __syncthreads();
-            for (uint32_t q = tid; q < mp; q += kClsThreads) {
-                if (q < m) {
-                    const uint32_t aid = p.d.list_c[bs + q];
-                    const medusa_alloc x = a.alloc[aid];
-                    S.key[q] = x.base;
-                    S.end[q] = x.base + x.size;
-                    S.ta[q] = x.t_alloc;
-                    S.tf[q] = x.t_free;
-                    S.id[q] = aid;
-                } else {
-                    S.key[q] = ~0ull;
-                }
-                S.val[q] = (uint16_t)q;
-            }
-            __syncthreads();
-            for (uint32_t size = 2; size <= mp; size <<= 1) {
-                for (uint32_t st = size >> 1; st > 0; st >>= 1) {
-                    for (uint32_t q = tid; q < mp / 2; q += kClsThreads) {
-                        const uint32_t lo = 2 * q - (q & (st - 1)), hi = lo + st;
-                        const bool up = (lo & size) == 0;
-                        const uint64_t ka = S.key[lo], kb = S.key[hi];
-                        const uint16_t va = S.val[lo], vb = S.val[hi];
-                        if (kv_less(kb, vb, ka, va) == up) { S.key[lo] = kb; S.key[hi] = ka; S.val[lo] = vb; S.val[hi] = va; }
-                    }
-                    __syncthreads();
-                }
-            }
-            if (warp == 0) {  // prefix max of end in sorted order
-                const uint32_t per = (m + 31) / 32;
-                const uint32_t b = lane * per, e = min(b + per, m);
-                uint64_t run = 0;
-                for (uint32_t q = b; q < e; ++q) run = max(run, S.end[S.val[q]]);
-                uint64_t incl = run;
-                for (int d = 1; d < 32; d <<= 1) {
-                    const uint64_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                    if (lane >= d) incl = max(incl, y);
-                }
-                uint64_t acc = __shfl_up_sync(0xffffffffu, incl, 1);
-                if (lane == 0) acc = 0;
-                for (uint32_t q = b; q < e; ++q) { acc = max(acc, S.end[S.val[q]]); S.pmax[q] = acc; }
-            }
-            __syncthreads();
-#pragma unroll
-            for (int k = 0; k < kWordsPerThread; ++k) {
-                if (!cand[k] || hit[k]) continue;
-                const uint64_t x = w[k];
-                uint32_t lo = 0, hi = m;  // count of keys <= x
-                while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.key[mid] <= x) lo = mid + 1; else hi = mid; }
-                for (int q = (int)lo - 1; q >= 0 && S.pmax[q] > x; --q) {
-                    const uint32_t u = S.val[q];
-                    if (x - S.key[q] < S.end[u] - S.key[q] && S.ta[u] < t[k] && t[k] < S.tf[u]) {
-                        hit[k] = true;
-                        hid[k] = S.id[u];
-                        hoff[k] = x - S.key[q];
-                        break;
+            bool hit = false;
+            if (q < n && !((S.hits[q >> 5] >> (q & 31)) & 1u)) {
+                const uint64_t x = S.words[q];
+                if (x >= gmin && x < gmax) {
+                    const uint32_t t = S.tw[q];
+                    uint32_t lo = 0, hi = m;  // count of keys <= x
+                    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.key[mid] <= x) lo = mid + 1; else hi = mid; }
+                    for (int r = (int)lo - 1; r >= 0 && S.pmax[r] > x; --r) {
+                        const uint32_t u = S.val[r];
+                        if (x < S.end[u] && S.ta[u] < t && t < S.tf[u]) {
+                            hit = true;
+                            S.words[q] = ((uint64_t)S.id[u] << MEDUSA_OFF_BITS) | (x - S.key[r]);
+                            break;
+                        }
                     }
                 }
             }
-        }
-        // I list: fence search in shared memory, then at most log2(stride) probes
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            if (!cand[k] || hit[k] || nI == 0) continue;
-            const uint64_t x = w[k];
-            uint32_t lo = 0, hi = nf;  // count of fences <= x
-            while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.fence[mid] <= x) lo = mid + 1; else hi = mid; }
-            if (lo == 0) continue;
-            uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
-            uint32_t l2 = g0 + 1, h2 = g1;  // count of bases <= x within the group
-            while (l2 < h2) { uint32_t mid = (l2 + h2) >> 1; if (p.d.i_base[mid] <= x) l2 = mid + 1; else h2 = mid; }
-            const uint32_t kk = l2 - 1;
-            const uint64_t base = stride == 1 ? S.fence[lo - 1] : p.d.i_base[kk];
-            const IRest e = p.d.i_rest[kk];
-            if (x < e.end && e.t_alloc < t[k]) {
-                hit[k] = true;
-                hid[k] = e.id;
-                hoff[k] = x - base;
-            }
-        }
-        // emission: mask words, per-(k,warp) counts, chunk prefix by look-back
-        uint32_t bal[kWordsPerThread];
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            bal[k] = __ballot_sync(0xffffffffu, hit[k]);
-            const uint64_t mw = (cs + (uint64_t)k * kClsThreads + warp * 32) / 32;
-            if (lane == 0) {
-                S.cnt[k][warp] = __popc(bal[k]);
-                if (mw < n_mask) a.mask[mw] = bal[k];
-            }
+            const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+            if (lane == 0 && bal) S.hits[q >> 5] |= bal;  // one warp owns this hits word
         }
         __syncthreads();
-        if (warp == 0) {
-            // exclusive scan over (k, warp) in word order; 64 entries, 2 per lane
-            const uint32_t e0 = S.cnt[(2 * lane) / kWarps][(2 * lane) % kWarps];
-            const uint32_t e1 = S.cnt[(2 * lane + 1) / kWarps][(2 * lane + 1) % kWarps];
-            const uint32_t pair = e0 + e1;
-            uint32_t incl = pair;
-            for (int d = 1; d < 32; d <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                if (lane >= d) incl += y;
-            }
-            const uint32_t excl = incl - pair;
-            const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-            __syncwarp();
-            S.cnt[(2 * lane) / kWarps][(2 * lane) % kWarps] = excl;
-            S.cnt[(2 * lane + 1) / kWarps][(2 * lane + 1) % kWarps] = excl + e0;
-            if (lane == 0) {
-                unsigned long long prefix = 0;
-                if (c == 0) {
-                    st_release(&p.d.lookback[0], LB_PRE | total);
-                } else {
-                    st_release(&p.d.lookback[c], LB_AGG | total);
-                    int64_t j = (int64_t)c - 1;
-                    while (j >= 0) {
-                        const unsigned long long v = ld_acquire(&p.d.lookback[j]);
-                        if ((v & ~LB_VAL) == 0) { __nanosleep(20); continue; }
-                        prefix += v & LB_VAL;
-                        if (v & LB_PRE) break;
-                        --j;
-                    }
-                    st_release(&p.d.lookback[c], LB_PRE | (prefix + total));
-                }
-                a.chunk_base[c] = (uint32_t)prefix;
-                if (c + 1 == p.C) {
-                    a.chunk_base[p.C] = (uint32_t)(prefix + total);
-                    ctl->n_slots = prefix + total;
-                }
-                S.prefix = prefix;
-            }
+    }
+    // 4. words still unresolved that could point into memory -> the I-list queue
+#pragma unroll 2
+    for (int k = 0; k < kWordsPerThread; ++k) {
+        const uint32_t q = k * kClsThreads + tid;
+        bool need = false;
+        if (q < n && nI && !((S.hits[q >> 5] >> (q & 31)) & 1u)) {
+            const uint64_t x = S.words[q];
+            need = x >= gmin && x < gmax && x >= S.fence[0];
         }
-        __syncthreads();
-        const unsigned long long prefix = S.prefix;
-        const uint32_t lt = lanemask_lt();
+        const uint32_t bal = __ballot_sync(0xffffffffu, need);
+        uint32_t base = 0;
+        if (lane == 0 && bal) base = atomicAdd(&S.nq, (uint32_t)__popc(bal));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (need) S.queue[base + __popc(bal & lanemask_lt())] = (uint16_t)q;
+    }
+    __syncthreads();
+    // 5. I-list search: fences in shared memory, then one group of <= stride bases
+    const uint32_t nq = S.nq;
+    for (uint32_t i = tid; i < nq; i += kClsThreads) {
+        const uint32_t q = S.queue[i];
+        const uint64_t x = S.words[q];
+        const uint32_t t = S.tw[q];
+        uint32_t lo = 0, hi = nf;  // count of fences <= x (>= 1: x >= fence[0])
+        while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.fence[mid] <= x) lo = mid + 1; else hi = mid; }
+        const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
+        uint32_t kk = g0;
+        uint64_t base = S.fence[lo - 1];
+        for (uint32_t k2 = g0 + 1; k2 < g1; ++k2) {
+            const uint64_t b2 = p.d.i_base[k2];
+            if (b2 > x) break;
+            kk = k2;
+            base = b2;
+        }
+        const IRest e = p.d.i_rest[kk];
+        if (x < e.end && e.t_alloc < t) {
+            S.words[q] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (x - base);
+            atomicOr(&S.hits[q >> 5], 1u << (q & 31));
+        }
+    }
+    __syncthreads();
+    // 6. emission: mask words, warp-dense staging of records, chunk count
+    const uint64_t n_mask = (a.n_words + 31) / 32;
+    uint32_t cnt = 0;
 #pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            if (!hit[k]) continue;
-            const unsigned long long rank = prefix + S.cnt[k][warp] + __popc(bal[k] & lt);
-            if (rank < a.capacity) a.slot[rank] = ((uint64_t)hid[k] << MEDUSA_OFF_BITS) | hoff[k];
+    for (int k = 0; k < kWordsPerThread; ++k) {
+        const uint32_t q = k * kClsThreads + tid;
+        const uint32_t bits = S.hits[q >> 5];
+        const uint64_t mw = (cs + q) >> 5;
+        if (lane == 0 && mw < n_mask) a.mask[mw] = bits;
+        if ((bits >> lane) & 1u) p.d.staging[(cs + q - lane) + __popc(bits & lanemask_lt())] = S.words[q];
+        cnt += __popc(bits);
+    }
+    if (lane == 0) atomicAdd(&S.total, cnt);
+    __syncthreads();
+    if (tid == 0) p.d.chunk_cnt[c] = S.total;
+}
+
+// 9. chunk prefix (decoupled look-back over known counts) + record compaction
+__global__ void __launch_bounds__(256) k_emit(P p) {
+    __shared__ uint32_t s_pre[65];
+    __shared__ uint32_t s_chunk;
+    __shared__ unsigned long long s_prefix;
+    const MaterializeArgs& a = p.a;
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) s_chunk = atomicAdd(&p.d.ctl->ticket, 1u);
+    __syncthreads();
+    const uint32_t c = s_chunk;
+    if (warp == 0) {
+        if (lane == 0) {
+            const uint32_t total = p.d.chunk_cnt[c];
+            unsigned long long prefix = 0;
+            if (c == 0) {
+                st_release(&p.d.lookback[0], LB_PRE | total);
+            } else {
+                st_release(&p.d.lookback[c], LB_AGG | total);
+                int64_t j = (int64_t)c - 1;
+                while (j >= 0) {
+                    const unsigned long long v = ld_acquire(&p.d.lookback[j]);
+                    if ((v & ~LB_VAL) == 0) continue;
+                    prefix += v & LB_VAL;
+                    if (v & LB_PRE) break;
+                    --j;
+                }
+                st_release(&p.d.lookback[c], LB_PRE | (prefix + total));
+            }
+            a.chunk_base[c] = (uint32_t)prefix;
+            if (c + 1 == p.C) {
+                a.chunk_base[p.C] = (uint32_t)(prefix + total);
+                p.d.ctl->n_slots = prefix + total;
+            }
+            s_prefix = prefix;
+        }
+    } else if (warp == 1 || warp == 2) {  // popcounts of the chunk's 64 mask words, exclusive scan
+        const uint64_t n_mask = (a.n_words + 31) / 32;
+        const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
+        const uint32_t h = warp - 1;  // half
+        const uint64_t mw = m0 + h * 32 + lane;
+        const uint32_t pc = mw < n_mask ? __popc(a.mask[mw]) : 0;
+        uint32_t incl = pc;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
+        }
+        s_pre[h * 32 + lane] = incl - pc;
+        if (h == 0 && lane == 31) s_pre[64] = incl;  // first-half total
+    }
+    __syncthreads();
+    const unsigned long long prefix = s_prefix;
+    const uint32_t half0 = s_pre[64];
+    // each warp copies 8 mask-word groups: lane l moves record l of the group
+    const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
+    const uint64_t n_mask = (a.n_words + 31) / 32;
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+        const uint32_t local = warp * 8 + g;
+        const uint64_t mw = m0 + local;
+        if (mw >= n_mask) break;
+        const uint32_t bits = a.mask[mw];
+        if (lane < (uint32_t)__popc(bits)) {
+            const unsigned long long dst = prefix + s_pre[local] + (local >= 32 ? half0 : 0) + lane;
+            if (dst < a.capacity) a.slot[dst] = p.d.staging[mw * 32 + lane];
         }
     }
 }
@@ -628,13 +796,12 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
 // ----------------------------------------------------------------------------
 // host side: per-device scratch, launches
 struct Scratch {
-    size_t cap_n = 0, cap_C = 0, cap_nb = 0, cap_c = 0, cap_b = 0;
+    size_t cap_n = 0, cap_C = 0, cap_nb = 0, cap_c = 0, cap_b = 0, cap_w = 0;
     void* zero_region = nullptr;
     size_t zero_bytes = 0;
     Dev d{};
     std::vector<void*> bufs;
     Ctl* h_ctl = nullptr;
-    int sm_count = 0, cls_blocks_per_sm = 0;
 };
 std::mutex g_mu;
 std::vector<Scratch*> g_scratch;
@@ -654,14 +821,16 @@ void release(Scratch& s) {
     s.bufs.clear();
     if (s.zero_region) cudaFree(s.zero_region);
     s.zero_region = nullptr;
-    s.cap_n = s.cap_C = s.cap_nb = s.cap_c = s.cap_b = 0;
+    s.cap_n = s.cap_C = s.cap_nb = s.cap_c = s.cap_b = s.cap_w = 0;
 }
 
-cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t need_c, size_t need_b) {
-    if (n <= s.cap_n && C <= s.cap_C && nb <= s.cap_nb && need_c <= s.cap_c && need_b <= s.cap_b) return cudaSuccess;
+cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t need_c, size_t need_b) {
+    if (n <= s.cap_n && C <= s.cap_C && nb <= s.cap_nb && W <= s.cap_w && need_c <= s.cap_c && need_b <= s.cap_b)
+        return cudaSuccess;
     cudaDeviceSynchronize();
     release(s);
     const size_t N = std::max<size_t>(n, 1024), CC = std::max<size_t>(C, 64), NB = std::max<size_t>(nb, 64);
+    const size_t WW = std::max<size_t>(W, 2048);
     const size_t RC = std::max<size_t>(need_c, 2 * N + 4 * CC), RB = std::max<size_t>(need_b, 3 * N);
     cudaError_t e;
     // zero region: Ctl | cnt_c fill_c [CC+1] | cnt_b fill_b [NB+1] | lookback [CC]
@@ -679,13 +848,15 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t need_c, siz
     if ((e = grow(s, s.d.tmin, CC)) || (e = grow(s, s.d.tmax, CC)) || (e = grow(s, s.d.jf, CC)) ||
         (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.rng, N)) || (e = grow(s, s.d.off_c, CC + 1)) ||
         (e = grow(s, s.d.off_b, NB + 1)) || (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) ||
-        (e = grow(s, s.d.sk0, N)) || (e = grow(s, s.d.sk1, N)) || (e = grow(s, s.d.sv0, N)) ||
-        (e = grow(s, s.d.sv1, N)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
-        (e = grow(s, s.d.fence, (size_t)kFenceCap)))
+        (e = grow(s, s.d.sk[0], N)) || (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) ||
+        (e = grow(s, s.d.sv[1], N)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
+        (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.blk_min_ta, N / kIBlk + 1)) ||
+        (e = grow(s, s.d.blk_max_tf, N / kIBlk + 1)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
+        (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)))
         return e;
     s.d.cap_c = RC;
     s.d.cap_b = RB;
-    s.cap_n = N; s.cap_C = CC; s.cap_nb = NB; s.cap_c = RC; s.cap_b = RB;
+    s.cap_n = N; s.cap_C = CC; s.cap_nb = NB; s.cap_c = RC; s.cap_b = RB; s.cap_w = WW;
     return cudaSuccess;
 }
 
@@ -703,26 +874,22 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     Scratch& s = *g_scratch[dev];
     if (!s.h_ctl) {
         if ((e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-        cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ClsShared));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s.cls_blocks_per_sm, k_classify, kClsThreads,
-                                                      sizeof(ClsShared));
-        if (s.cls_blocks_per_sm < 1) s.cls_blocks_per_sm = 1;
+        cudaFuncSetAttribute(k_sort_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, kSortTile * 12);
     }
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
     const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
     size_t need_c = 0, need_b = 0;
     for (int attempt = 0; attempt < 3; ++attempt) {
-        if ((e = ensure(s, n, C, nb, need_c, need_b)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+        if ((e = ensure(s, n, C, nb, a.n_words, need_c, need_b)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
         P p{a, s.d, C, nb};
         if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) break;
         if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) break;
         const uint32_t T = 256;
         {
-            const uint64_t work = std::max<uint64_t>((uint64_t)a.n_nodes + 1, C);
             TimedLaunch tl("mat_nodes_chunks", stream);
-            k_nodes_chunks<<<(unsigned)((work + T - 1) / T), T, 0, stream>>>(p);
+            k_nodes_chunks<<<(unsigned)((a.n_nodes + 1 + T - 1) / T), T, 0, stream>>>(p);
         }
         if (n) {
             TimedLaunch tl("mat_allocs", stream);
@@ -733,34 +900,33 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
             k_scan<<<1, 1024, 0, stream>>>(p);
         }
         if (n) {
-            TimedLaunch tl("mat_scatter", stream);
-            k_scatter<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
-        }
-        if (n) {
-            const unsigned tiles = (unsigned)((n + kSortTile - 1) / kSortTile);
+            {
+                TimedLaunch tl("mat_scatter", stream);
+                k_scatter<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
+            }
             {
                 TimedLaunch tl("mat_sort_tile", stream);
-                k_sort_tile<<<tiles, 1024, 0, stream>>>(s.d.ctl, s.d.sk0, s.d.sv0, s.d.sk1, s.d.sv1);
+                k_sort_tile<<<(unsigned)((n + kSortTile - 1) / kSortTile), 1024, kSortTile * 12, stream>>>(p);
             }
-            uint64_t *ki = s.d.sk1, *ko = s.d.sk0;
-            uint32_t *vi = s.d.sv1, *vo = s.d.sv0;
-            for (uint64_t width = kSortTile; width < n; width *= 2) {
+            int pass = 0;
+            for (uint64_t width = kSortTile; width < n; width *= 2, ++pass) {
                 TimedLaunch tl("mat_merge", stream);
-                k_merge<<<tiles, 256, 0, stream>>>(s.d.ctl, ki, vi, ko, vo, (uint32_t)width);
-                std::swap(ki, ko);
-                std::swap(vi, vo);
+                k_merge<<<(unsigned)((n + kMergeTile - 1) / kMergeTile), 256, 0, stream>>>(p, (uint32_t)width, pass);
             }
-            TimedLaunch tl("mat_build_i", stream);
-            k_build_i<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p, ki, vi);
-        }
-        if (n) {
+            {
+                TimedLaunch tl("mat_build_i", stream);
+                k_build_i<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
+            }
             TimedLaunch tl("mat_check", stream);
             k_check<<<nb, kAblk, 0, stream>>>(p);
         }
         if (C) {
-            const unsigned grid = (unsigned)std::min<uint64_t>(C, (uint64_t)s.sm_count * s.cls_blocks_per_sm);
-            TimedLaunch tl("mat_classify", stream);
-            k_classify<<<grid, kClsThreads, sizeof(ClsShared), stream>>>(p);
+            {
+                TimedLaunch tl("mat_classify", stream);
+                k_classify<<<C, kClsThreads, sizeof(ClsShared), stream>>>(p);
+            }
+            TimedLaunch tl("mat_emit", stream);
+            k_emit<<<C, 256, 0, stream>>>(p);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) break;
         if ((e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess) break;
