@@ -45,8 +45,8 @@ namespace {
 
 constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kAblk = 64;          // allocation ordinals per overlap-check block
-constexpr int kChkCap = 256;       // registered mortals staged per check batch
-constexpr int kSortTile = 8192;    // elements sorted per CTA before the merge passes
+constexpr int kChkCap = 128;       // registered mortals staged per check batch (per block)
+constexpr int kSortTile = 2048;    // elements sorted per CTA before the merge passes
 constexpr int kMergeTile = 2048;   // outputs per CTA of a merge pass
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
 constexpr int kWinCap = 256;       // mortal-window entries per batch (power of two)
@@ -170,6 +170,26 @@ __global__ void k_nodes_chunks(P p) {
 
 // ----------------------------------------------------------------------------
 // 2. allocations: checks, I/M split, registration ranges and counts
+// first index k in [lo, n) with t[k] >= x (galloping from lo; t ascending)
+__device__ __forceinline__ uint32_t gallop_ge(const uint32_t* t, uint32_t lo, uint32_t n, uint32_t x) {
+    uint32_t step = 1, prev = lo;
+    uint32_t hi = lo;
+    while (hi < n && t[hi] < x) { prev = hi + 1; hi = hi + step; step <<= 1; }
+    if (hi > n) hi = n;
+    uint32_t l = prev;
+    while (l < hi) { const uint32_t m = (l + hi) >> 1; if (t[m] < x) l = m + 1; else hi = m; }
+    return l;
+}
+__device__ __forceinline__ uint32_t gallop_alloc_ge(const medusa_alloc* al, uint32_t lo, uint32_t n, uint32_t x) {
+    uint32_t step = 1, prev = lo;
+    uint32_t hi = lo;
+    while (hi < n && al[hi].t_alloc < x) { prev = hi + 1; hi = hi + step; step <<= 1; }
+    if (hi > n) hi = n;
+    uint32_t l = prev;
+    while (l < hi) { const uint32_t m = (l + hi) >> 1; if (al[m].t_alloc < x) l = m + 1; else hi = m; }
+    return l;
+}
+
 __global__ void __launch_bounds__(256) k_allocs(P p) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     const MaterializeArgs& a = p.a;
@@ -188,22 +208,26 @@ __global__ void __launch_bounds__(256) k_allocs(P p) {
         if (x.size != 0) {
             isI = N && x.t_alloc < t_last && t_last < x.t_free;
             if (!isI) {
-                if (p.C && N) {
-                    uint32_t lo = 0, hi = p.C;  // first chunk whose last launch is after t_alloc
-                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.tmax[m] > x.t_alloc) hi = m; else lo = m + 1; }
-                    const uint32_t c_lo = lo;
-                    lo = c_lo; hi = p.C;  // chunks whose first launch is before t_free
-                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.tmin[m] < x.t_free) lo = m + 1; else hi = m; }
-                    if (c_lo < lo) {
-                        r.x = c_lo; r.y = lo - 1;
-                        for (uint32_t c = r.x; c <= r.y; ++c) atomicAdd(&p.d.cnt_c[c], 1u);
+                if (p.C && N && x.t_alloc < x.t_free) {
+                    // nodes launched while i is live: [j0, j1) = t in (t_alloc, t_free)
+                    uint32_t lo = 0, hi = N;
+                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.node_t[m] <= x.t_alloc) lo = m + 1; else hi = m; }
+                    const uint32_t j0 = lo;
+                    const uint32_t j1 = gallop_ge(a.node_t, j0, N, x.t_free);
+                    // chunks holding their words (exact: no entry for memory no launch can see)
+                    if (j0 < j1) {
+                        const uint64_t w0 = a.node_off[j0], w1 = a.node_off[j1];
+                        if (w0 < w1 && w1 <= a.n_words) {
+                            r.x = (uint32_t)(w0 / kChunkWords);
+                            r.y = (uint32_t)((w1 - 1) / kChunkWords);
+                            for (uint32_t c = r.x; c <= r.y; ++c) atomicAdd(&p.d.cnt_c[c], 1u);
+                        }
                     }
                 }
                 // ordinals allocated while i is live: (i, u), u = #{k : t_alloc_k < t_free_i}
-                uint32_t lo = i + 1, hi = a.n_alloc;
-                while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.alloc[m].t_alloc < x.t_free) lo = m + 1; else hi = m; }
-                if (i + 1 < lo) {
-                    r.z = (i + 1) / kAblk; r.w = (lo - 1) / kAblk;
+                const uint32_t u = gallop_alloc_ge(a.alloc, i + 1, a.n_alloc, x.t_free);
+                if (i + 1 < u) {
+                    r.z = (i + 1) / kAblk; r.w = (u - 1) / kAblk;
                     for (uint32_t b = r.z; b <= r.w; ++b) atomicAdd(&p.d.cnt_b[b], 1u);
                 }
             }
@@ -288,39 +312,108 @@ __global__ void k_scatter(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 5. sort I by (base, index): bitonic tiles of 8192 in shared memory, then
-//    merge-path passes (only those the device-side count needs do any work)
-__global__ void __launch_bounds__(1024) k_sort_tile(P p) {
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    uint64_t* sk = reinterpret_cast<uint64_t*>(smem_raw);
-    uint32_t* sv = reinterpret_cast<uint32_t*>(sk + kSortTile);
+// 5. sort I by (base, index): each warp sorts 256 keys in registers (bitonic
+//    network over shuffles), the CTA merges its 8 runs to a 2048 tile in shared
+//    memory, then merge-path passes (only those the device-side count needs do
+//    any work)
+__device__ __forceinline__ void cas(uint64_t& ka, uint32_t& va, uint64_t& kb, uint32_t& vb, bool up) {
+    if (kv_less(kb, vb, ka, va) == up) {
+        const uint64_t tk = ka; ka = kb; kb = tk;
+        const uint32_t tv = va; va = vb; vb = tv;
+    }
+}
+
+// merge path inside shared memory: smallest i in [lo, hi) with less(B[d-1-i], A[i]), else hi
+__device__ __forceinline__ uint32_t merge_path_smem(const uint64_t* ka, const uint32_t* va, const uint64_t* kb,
+                                                    const uint32_t* vb, uint32_t d, uint32_t lo, uint32_t hi) {
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (kv_less(kb[d - 1 - mid], vb[d - 1 - mid], ka[mid], va[mid])) hi = mid; else lo = mid + 1;
+    }
+    return lo;
+}
+
+__global__ void __launch_bounds__(256) k_sort_tile(P p) {
+    __shared__ uint64_t sk[2][kSortTile];
+    __shared__ uint32_t sv[2][kSortTile];
     const uint32_t n = p.d.ctl->nI;
     const uint32_t t0 = blockIdx.x * kSortTile;
     if (t0 >= n) return;
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint64_t* kin = p.d.sk[0];
     const uint32_t* vin = p.d.sv[0];
-    for (uint32_t q = threadIdx.x; q < kSortTile; q += blockDim.x) {
-        const bool in = t0 + q < n;
-        sk[q] = in ? kin[t0 + q] : ~0ull;
-        sv[q] = in ? vin[t0 + q] : 0xFFFFFFFFu;
+    // 1. warp run of 256: lane holds elements e = lane*8 + r
+    uint64_t k[8];
+    uint32_t v[8];
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+        const uint32_t g = t0 + warp * 256 + lane * 8 + r;
+        k[r] = g < n ? kin[g] : ~0ull;
+        v[r] = g < n ? vin[g] : 0xFFFFFFFFu;
     }
-    __syncthreads();
-    for (uint32_t size = 2; size <= kSortTile; size <<= 1) {
-        for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
-            for (uint32_t q = threadIdx.x; q < kSortTile / 2; q += blockDim.x) {
-                const uint32_t lo = 2 * q - (q & (stride - 1));
-                const uint32_t hi = lo + stride;
-                const bool up = (lo & size) == 0;
-                const uint64_t ka = sk[lo], kb = sk[hi];
-                const uint32_t va = sv[lo], vb = sv[hi];
-                if (kv_less(kb, vb, ka, va) == up) { sk[lo] = kb; sk[hi] = ka; sv[lo] = vb; sv[hi] = va; }
+#pragma unroll
+    for (uint32_t size = 2; size <= 256; size <<= 1) {
+#pragma unroll
+        for (uint32_t j = size >> 1; j > 0; j >>= 1) {
+            if (j >= 8) {
+                const uint32_t lj = j >> 3;
+#pragma unroll
+                for (int r = 0; r < 8; ++r) {
+                    const uint32_t e = lane * 8 + r;
+                    const uint64_t ok = __shfl_xor_sync(0xffffffffu, k[r], lj);
+                    const uint32_t ov = __shfl_xor_sync(0xffffffffu, v[r], lj);
+                    const bool up = (e & size) == 0;
+                    const bool lower = (e & j) == 0;
+                    const bool other_less = kv_less(ok, ov, k[r], v[r]);
+                    // lower element keeps the min when ascending, the max when descending
+                    const bool take = (lower == up) ? other_less : !other_less;
+                    if (take) { k[r] = ok; v[r] = ov; }
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < 8; ++r) {
+                    const int r2 = r ^ (int)j;
+                    if (r2 > r) {
+                        const uint32_t e = lane * 8 + r;
+                        cas(k[r], v[r], k[r2], v[r2], (e & size) == 0);
+                    }
+                }
             }
-            __syncthreads();
         }
     }
-    for (uint32_t q = threadIdx.x; q < kSortTile && t0 + q < n; q += blockDim.x) {
-        p.d.sk[1][t0 + q] = sk[q];
-        p.d.sv[1][t0 + q] = sv[q];
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+        sk[0][warp * 256 + lane * 8 + r] = k[r];
+        sv[0][warp * 256 + lane * 8 + r] = v[r];
+    }
+    __syncthreads();
+    // 2. merge runs 256 -> 2048 in shared memory (8 outputs per thread per round)
+    int src = 0;
+#pragma unroll
+    for (uint32_t run = 256; run < kSortTile; run <<= 1) {
+        const uint32_t o = tid * 8;
+        const uint32_t pair = o / (2 * run);
+        const uint32_t a0 = pair * 2 * run, b0 = a0 + run;
+        const uint32_t d = o - a0;
+        const uint64_t* ka = sk[src] + a0;
+        const uint32_t* va = sv[src] + a0;
+        const uint64_t* kb = sk[src] + b0;
+        const uint32_t* vb = sv[src] + b0;
+        uint32_t ia = merge_path_smem(ka, va, kb, vb, d, d > run ? d - run : 0, min(d, run));
+        uint32_t ib = d - ia;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const bool takeA = ib >= run || (ia < run && kv_less(ka[ia], va[ia], kb[ib], vb[ib]));
+            sk[src ^ 1][o + q] = takeA ? ka[ia] : kb[ib];
+            sv[src ^ 1][o + q] = takeA ? va[ia] : vb[ib];
+            if (takeA) ++ia; else ++ib;
+        }
+        src ^= 1;
+        __syncthreads();
+    }
+    for (uint32_t q = tid; q < kSortTile && t0 + q < n; q += blockDim.x) {
+        p.d.sk[1][t0 + q] = sk[src][q];
+        p.d.sv[1][t0 + q] = sv[src][q];
     }
 }
 
@@ -436,13 +529,42 @@ __global__ void __launch_bounds__(256) k_build_i(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 7. overlap checks for mortal allocations
-__global__ void __launch_bounds__(kAblk) k_check(P p) {
-    __shared__ uint64_t s_base[kChkCap], s_end[kChkCap];
-    __shared__ uint32_t s_tf[kChkCap], s_idx[kChkCap];
+// 7. overlap checks for mortal allocations.  A CTA of 256 threads covers four
+//    registration blocks of 64 ordinals; the I-list fences sit in shared memory.
+constexpr int kChkThreads = 4 * kAblk;
+
+// count of sorted I bases <= x (fences in shared memory, then one group of <= stride
+// bases read with independent loads)
+__device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t nf, uint32_t stride, uint32_t nI,
+                                               const uint64_t* i_base, uint64_t x) {
+    uint32_t lo = 0, hi = nf;
+    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (fence[mid] <= x) lo = mid + 1; else hi = mid; }
+    if (lo == 0) return 0;
+    const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
+    uint32_t c = g0 + 1;
+    for (uint32_t k = g0 + 1; k < g1; k += 8) {
+        uint64_t b[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) b[u] = (k + u < g1) ? i_base[k + u] : ~0ull;
+#pragma unroll
+        for (int u = 0; u < 8; ++u) c += (k + u < g1 && b[u] <= x) ? 1u : 0u;
+        if (b[7] > x) break;
+    }
+    return c;
+}
+
+__global__ void __launch_bounds__(kChkThreads) k_check(P p) {
+    __shared__ uint64_t s_fence[kFenceCap];
+    __shared__ uint64_t s_base[4][kChkCap], s_end[4][kChkCap];
+    __shared__ uint32_t s_tf[4][kChkCap], s_idx[4][kChkCap];
     const MaterializeArgs& a = p.a;
-    const uint32_t b = blockIdx.x;
-    const uint32_t j = b * kAblk + threadIdx.x;
+    const uint32_t sub = threadIdx.x / kAblk;          // registration block within the CTA
+    const uint32_t b = blockIdx.x * 4 + sub;
+    const uint32_t j = blockIdx.x * kChkThreads + threadIdx.x;
+    const uint32_t nI = p.d.ctl->nI;
+    const uint32_t stride = nI ? (nI + kFenceCap - 1) / kFenceCap : 1;
+    const uint32_t nf = (nI + stride - 1) / stride;
+    for (uint32_t f = threadIdx.x; f < nf; f += kChkThreads) s_fence[f] = p.d.fence[f];
     bool mine = false;
     medusa_alloc x{};
     const uint32_t N = a.n_nodes;
@@ -454,46 +576,53 @@ __global__ void __launch_bounds__(kAblk) k_check(P p) {
     const uint64_t xe = x.base + x.size;
     bool bad = false;
     // M-M: registered mortals live at some allocation of this block
-    const uint64_t r0 = p.d.off_b[b];
-    const uint64_t r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
-    for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
-        const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
+    uint64_t r0 = 0, r1 = 0;
+    if (b < p.nb) {
+        r0 = p.d.off_b[b];
+        r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
+    }
+    uint32_t rounds = (uint32_t)((r1 - r0 + kChkCap - 1) / kChkCap);
+    rounds = __reduce_max_sync(0xffffffffu, rounds);
+    __shared__ uint32_t s_rounds[kChkThreads / 32];
+    if ((threadIdx.x & 31) == 0) s_rounds[threadIdx.x >> 5] = rounds;
+    __syncthreads();
+    uint32_t all_rounds = 0;
+    for (int w = 0; w < kChkThreads / 32; ++w) all_rounds = max(all_rounds, s_rounds[w]);
+    for (uint32_t rd = 0; rd < all_rounds; ++rd) {
+        const uint64_t bs = r0 + (uint64_t)rd * kChkCap;
+        const uint32_t m = bs < r1 ? (uint32_t)min((uint64_t)kChkCap, r1 - bs) : 0;
         __syncthreads();
-        for (uint32_t q = threadIdx.x; q < m; q += blockDim.x) {
+        for (uint32_t q = threadIdx.x % kAblk; q < m; q += kAblk) {
             const WinRec y = p.d.list_b[bs + q];
-            s_base[q] = y.base;
-            s_end[q] = y.end;
-            s_tf[q] = y.t_free;
-            s_idx[q] = y.id;
+            s_base[sub][q] = y.base;
+            s_end[sub][q] = y.end;
+            s_tf[sub][q] = y.t_free;
+            s_idx[sub][q] = y.id;
         }
         __syncthreads();
         if (mine && !bad) {
             for (uint32_t q = 0; q < m; ++q) {
-                if (s_idx[q] < j && s_tf[q] > x.t_alloc && s_base[q] < xe && x.base < s_end[q]) { bad = true; break; }
+                if (s_idx[sub][q] < j && s_tf[sub][q] > x.t_alloc && s_base[sub][q] < xe && x.base < s_end[sub][q]) {
+                    bad = true;
+                    break;
+                }
             }
         }
     }
     // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
-    const uint32_t nI = p.d.ctl->nI;
     if (mine && !bad && nI) {
-        uint32_t lo = 0, hi = nI;  // e = count of I bases < end
-        while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.i_base[m] < xe) lo = m + 1; else hi = m; }
-        const uint32_t e = lo;
-        lo = 0; hi = e;            // s = count of I ends <= base (ends ascend on a disjoint list)
-        while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (p.d.i_rest[m].end <= x.base) lo = m + 1; else hi = m; }
-        const uint32_t s = lo;
-        // overlap with e in I: freed before T_last -> some t_alloc_e < t_free; else some t_free_e > t_alloc
+        const uint32_t e = i_count_le(s_fence, nf, stride, nI, p.d.i_base, xe - 1);  // bases < end
+        const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);
+        const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
+        // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
         const bool freed_early = x.t_free <= t_last;
         uint32_t k = s;
-        while (k < e && !bad) {
-            if (k % kIBlk == 0 && k + kIBlk <= e) {
-                bad = freed_early ? p.d.blk_min_ta[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
-                k += kIBlk;
-            } else {
-                bad = freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
-                ++k;
-            }
-        }
+        for (; k < e && (k % kIBlk) != 0; ++k)
+            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
+        for (; k + kIBlk <= e; k += kIBlk)
+            bad |= freed_early ? p.d.blk_min_ta[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
+        for (; k < e; ++k)
+            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
     }
     if (bad) flag(p.d.ctl, ST_TRACE);
 }
@@ -689,17 +818,8 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
         const uint32_t q = S.queue[i];
         const uint64_t x = S.words[q];
         const uint32_t t = S.tw[q];
-        uint32_t lo = 0, hi = nf;  // count of fences <= x (>= 1: x >= fence[0])
-        while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.fence[mid] <= x) lo = mid + 1; else hi = mid; }
-        const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
-        uint32_t kk = g0;
-        uint64_t base = S.fence[lo - 1];
-        for (uint32_t k2 = g0 + 1; k2 < g1; ++k2) {
-            const uint64_t b2 = p.d.i_base[k2];
-            if (b2 > x) break;
-            kk = k2;
-            base = b2;
-        }
+        const uint32_t kk = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x) - 1;  // >= 0: x >= fence[0]
+        const uint64_t base = p.d.i_base[kk];
         const IRest e = p.d.i_rest[kk];
         if (x < e.end && e.t_alloc < t) {
             S.words[q] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (x - base);
@@ -724,9 +844,11 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     if (tid == 0) p.d.chunk_cnt[c] = S.total;
 }
 
-// 9. chunk prefix (decoupled look-back over known counts) + record compaction
+// 9. chunk prefix (decoupled look-back over known counts, 32 predecessors per
+//    probe) + record compaction
 __global__ void __launch_bounds__(256) k_emit(P p) {
-    __shared__ uint32_t s_pre[65];
+    __shared__ uint32_t s_mask[64];
+    __shared__ uint32_t s_pre[64];
     __shared__ uint32_t s_chunk;
     __shared__ unsigned long long s_prefix;
     const MaterializeArgs& a = p.a;
@@ -734,37 +856,40 @@ __global__ void __launch_bounds__(256) k_emit(P p) {
     if (tid == 0) s_chunk = atomicAdd(&p.d.ctl->ticket, 1u);
     __syncthreads();
     const uint32_t c = s_chunk;
+    const uint64_t n_mask = (a.n_words + 31) / 32;
+    const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
     if (warp == 0) {
-        if (lane == 0) {
-            const uint32_t total = p.d.chunk_cnt[c];
-            unsigned long long prefix = 0;
-            if (c == 0) {
-                st_release(&p.d.lookback[0], LB_PRE | total);
-            } else {
-                st_release(&p.d.lookback[c], LB_AGG | total);
-                int64_t j = (int64_t)c - 1;
-                while (j >= 0) {
-                    const unsigned long long v = ld_acquire(&p.d.lookback[j]);
-                    if ((v & ~LB_VAL) == 0) continue;
-                    prefix += v & LB_VAL;
-                    if (v & LB_PRE) break;
-                    --j;
-                }
-                st_release(&p.d.lookback[c], LB_PRE | (prefix + total));
+        const uint32_t total = p.d.chunk_cnt[c];
+        if (lane == 0) st_release(&p.d.lookback[c], (c == 0 ? LB_PRE : LB_AGG) | total);
+        uint32_t prefix = 0;
+        if (c > 0) {
+            int64_t top = (int64_t)c - 1;
+            for (;;) {
+                const int64_t idx = top - lane;
+                const unsigned long long v = idx >= 0 ? ld_acquire(&p.d.lookback[idx]) : LB_PRE;
+                if (__ballot_sync(0xffffffffu, (v & ~LB_VAL) == 0)) continue;  // a predecessor not published yet
+                const uint32_t pre = __ballot_sync(0xffffffffu, (v & LB_PRE) != 0);
+                const uint32_t upto = pre ? (__ffs(pre) - 1) : 31;  // nearest inclusive prefix
+                prefix += __reduce_add_sync(0xffffffffu, lane <= upto ? (uint32_t)(v & LB_VAL) : 0u);
+                if (pre) break;
+                top -= 32;
             }
-            a.chunk_base[c] = (uint32_t)prefix;
+            if (lane == 0) st_release(&p.d.lookback[c], LB_PRE | (prefix + total));
+        }
+        if (lane == 0) {
+            a.chunk_base[c] = prefix;
             if (c + 1 == p.C) {
-                a.chunk_base[p.C] = (uint32_t)(prefix + total);
-                p.d.ctl->n_slots = prefix + total;
+                a.chunk_base[p.C] = prefix + total;
+                p.d.ctl->n_slots = (unsigned long long)prefix + total;
             }
             s_prefix = prefix;
         }
-    } else if (warp == 1 || warp == 2) {  // popcounts of the chunk's 64 mask words, exclusive scan
-        const uint64_t n_mask = (a.n_words + 31) / 32;
-        const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
-        const uint32_t h = warp - 1;  // half
+    } else if (warp == 1 || warp == 2) {  // the chunk's 64 mask words and their popcount prefix
+        const uint32_t h = warp - 1;
         const uint64_t mw = m0 + h * 32 + lane;
-        const uint32_t pc = mw < n_mask ? __popc(a.mask[mw]) : 0;
+        const uint32_t bits = mw < n_mask ? a.mask[mw] : 0u;
+        s_mask[h * 32 + lane] = bits;
+        const uint32_t pc = __popc(bits);
         uint32_t incl = pc;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
@@ -772,23 +897,19 @@ __global__ void __launch_bounds__(256) k_emit(P p) {
             if (lane >= d) incl += y;
         }
         s_pre[h * 32 + lane] = incl - pc;
-        if (h == 0 && lane == 31) s_pre[64] = incl;  // first-half total
     }
     __syncthreads();
+    if (tid < 32) s_pre[32 + tid] += s_pre[31] + __popc(s_mask[31]);  // second half after the first
+    __syncthreads();
     const unsigned long long prefix = s_prefix;
-    const uint32_t half0 = s_pre[64];
-    // each warp copies 8 mask-word groups: lane l moves record l of the group
-    const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
-    const uint64_t n_mask = (a.n_words + 31) / 32;
+    // each warp moves 8 mask-word groups: lane l copies record l of the group
 #pragma unroll
     for (int g = 0; g < 8; ++g) {
         const uint32_t local = warp * 8 + g;
-        const uint64_t mw = m0 + local;
-        if (mw >= n_mask) break;
-        const uint32_t bits = a.mask[mw];
+        const uint32_t bits = s_mask[local];
         if (lane < (uint32_t)__popc(bits)) {
-            const unsigned long long dst = prefix + s_pre[local] + (local >= 32 ? half0 : 0) + lane;
-            if (dst < a.capacity) a.slot[dst] = p.d.staging[mw * 32 + lane];
+            const unsigned long long dst = prefix + s_pre[local] + lane;
+            if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + local) * 32 + lane];
         }
     }
 }
@@ -875,7 +996,6 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     if (!s.h_ctl) {
         if ((e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ClsShared));
-        cudaFuncSetAttribute(k_sort_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, kSortTile * 12);
     }
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
@@ -906,7 +1026,7 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
             }
             {
                 TimedLaunch tl("mat_sort_tile", stream);
-                k_sort_tile<<<(unsigned)((n + kSortTile - 1) / kSortTile), 1024, kSortTile * 12, stream>>>(p);
+                k_sort_tile<<<(unsigned)((n + kSortTile - 1) / kSortTile), 256, 0, stream>>>(p);
             }
             int pass = 0;
             for (uint64_t width = kSortTile; width < n; width *= 2, ++pass) {
@@ -918,7 +1038,7 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
                 k_build_i<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
             }
             TimedLaunch tl("mat_check", stream);
-            k_check<<<nb, kAblk, 0, stream>>>(p);
+            k_check<<<(nb + 3) / 4, kChkThreads, 0, stream>>>(p);
         }
         if (C) {
             {

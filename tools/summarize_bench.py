@@ -1,0 +1,14 @@
+"""Print the key numbers of a bench JSON line."""
+import json
+import sys
+
+d = json.loads(open(sys.argv[1]).read().strip().splitlines()[-1])
+print(f"value {d['value']/1e6:.1f} M nodes/s  ms/step {d['ms_per_step']:.3f}  e2e {d['e2e']['value']/1e6:.1f} M nodes/s")
+r = d["roofline"]
+print(f"roofline[{r['kernel']}] {r['achieved']:.0f} GB/s = {100*r['frac']:.1f}% of {r['peak']}")
+rl = d["relocate"]
+print(f"relocate {rl['GB/s']:.0f} GB/s ({100*rl['frac_of_peak']:.1f}%) {rl['avg_us']:.1f} us  sustained={d.get('sustained_relocate')}")
+for k, v in d["kernels"].items():
+    print(f"  {k:22s} n={v['launches']:4d} avg {v['avg_us']:8.2f} us  share {100*v['share_of_step']:5.1f}%  " +
+          (f"{v['GB/s']:.0f} GB/s" if 'GB/s' in v else ""))
+print("cpu", d.get("cpu_baseline"), "clocks", d.get("clocks"), "launches", d.get("gpu_launches"))
