@@ -6,34 +6,37 @@
 //
 // Structure of a well-formed trace that the GPU design exploits:
 //  * I = allocations live at the LAST launch T_last.  All of them are live at
-//    the same instant, so they are pairwise address-disjoint: one global list
-//    sorted by base answers "which I-allocation holds w" with one search; it is
-//    live at t <= T_last iff t_alloc < t.  (Weights, KV cache, static inputs,
-//    permanent buffers: ~27k entries for the ten-model set.)
+//    the same instant, so they are pairwise address-disjoint: one list sorted by
+//    base answers "which I-allocation holds w" with one search; it is live at
+//    t <= T_last iff t_alloc < t.  (Weights, KV cache, static inputs, permanent
+//    buffers: ~27k entries for the ten-model set.)
 //  * M = every other allocation ("mortal": capture temporaries, warm-up and
-//    profiling scratch).  Their lifetimes are short, so each is registered in
-//    the word chunks whose launch-time span its lifetime touches; a chunk's
-//    mortal window (~60-150 entries) is sorted by base in shared memory and
+//    profiling scratch).  A mortal is registered in exactly the word chunks that
+//    hold words of nodes launched during its lifetime; a chunk's window (~60
+//    entries for the ten-model set) is sorted by base in shared memory and
 //    searched with a prefix-max-of-end backward walk plus the time check.
 //  * Well-formedness (no two simultaneously-live allocations overlap) is checked
 //    exactly: I-I by adjacency of the sorted list, M-I with per-32-entry
-//    min(t_alloc) / max(t_free) summaries of the sorted list over the address
-//    run a mortal meets, M-M inside blocks of 64 allocation ordinals against the
-//    mortals registered as live there.
+//    min(t_alloc) / max(t_free) summaries over the address run a mortal meets,
+//    M-M inside blocks of 32 allocation ordinals against the mortals registered
+//    as live there.
 // Pipeline (all on `stream`; one host synchronization at the end):
-//   k_nodes_chunks  CSR / launch-order checks; per-chunk first/last node
-//   k_allocs        trace checks, I/M split, registration counts, prefilter
-//   k_scan          registration offsets (single CTA)
+//   k_nodes_chunks  CSR / launch-order checks; per-chunk first/last node; node fences
+//   k_allocs        trace checks, I/M split, registration ranges + counts; the
+//                   last CTA scans the counts into offsets
 //   k_scatter       registration lists (32-byte window records)
-//   k_sort_tile + k_merge (x log)   I sorted by (base, index)
-//   k_build_i       I arrays, I-I check, fences, block summaries
+//   k_sort_tile     I keys sorted in tiles of 2048 (register bitonic per warp +
+//                   shared-memory merges)
+//   k_rank          global rank of every key = sum over the other tiles of a
+//                   binary-search count; the last contribution scatters the key
+//   k_finalize_i    I arrays, I-I check, shared-memory fences, block summaries
 //   k_check         M-M and M-I overlap checks
-//   k_classify      one CTA per 2048-word chunk: TMA bulk copy of the chunk's
-//                   words to shared memory, mortal-window search, I-list search
-//                   through a shared queue, mask words + warp-dense staging of
-//                   the records + the chunk's slot count (no inter-CTA waits)
-//   k_emit          decoupled look-back over the chunk counts -> chunk_base,
-//                   compaction of the staged records into the slot table
+//   k_classify      one CTA per 2048-word chunk: TMA bulk copy of the chunk's words
+//                   to shared memory, candidate compaction, window search, I-list
+//                   search, mask words + warp-dense staging of the records + the
+//                   chunk's slot count; the last CTA scans counts -> chunk_base
+//   k_emit          compaction of the staged records into the slot table
+// (k_merge passes replace k_rank when the trace has more than 64 tiles of I keys.)
 #include <algorithm>
 #include <mutex>
 #include <vector>
@@ -44,23 +47,24 @@ namespace medusa {
 namespace {
 
 constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
-constexpr int kAblk = 64;          // allocation ordinals per overlap-check block
-constexpr int kChkCap = 128;       // registered mortals staged per check batch (per block)
-constexpr int kSortTile = 2048;    // elements sorted per CTA before the merge passes
+constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
+constexpr int kChkCap = 64;        // registered mortals staged per warp batch
+constexpr int kSortTile = 2048;    // keys sorted per CTA before ranking / merging
 constexpr int kMergeTile = 2048;   // outputs per CTA of a merge pass
+constexpr int kRankMaxTiles = 64;  // above this many tiles, merge passes instead of ranks
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
-constexpr int kWinCap = 256;       // mortal-window entries per batch (power of two)
+constexpr int kNodeFenceCap = 4096;
+constexpr int kWinCap = 128;       // mortal-window entries per batch (4 per lane of one warp)
 constexpr int kClsThreads = 256;
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kClsThreads;  // 8
 constexpr int kWarps = kClsThreads / 32;
 constexpr int kIBlk = 32;          // I-list summary block
-constexpr unsigned long long LB_AGG = 1ull << 62, LB_PRE = 2ull << 62, LB_VAL = (1ull << 62) - 1;
 
 struct Ctl {
     unsigned int status;
     unsigned int nI;
-    unsigned int ticket;
-    unsigned int pad;
+    unsigned int done_allocs;
+    unsigned int done_cls;
     unsigned long long gmin_c;  // ~(least base) via atomicMax
     unsigned long long gmax;    // greatest end
     unsigned long long need_c, need_b;
@@ -84,14 +88,16 @@ struct WinRec {  // a registered mortal allocation
 
 struct Dev {  // scratch of one call (device pointers)
     Ctl* ctl;
-    uint32_t *tmin, *tmax, *jf, *jl;             // [C]
+    uint32_t *jf, *jl;                           // [C] first / last node of each chunk
+    uint32_t* node_fence;                        // [kNodeFenceCap] node_t every nstride nodes
     uint4* rng;                                  // [n]: c_lo, c_hi, b_lo, b_hi
-    uint32_t *cnt_c, *fill_c, *off_c;            // [C+1]
-    uint32_t *cnt_b, *fill_b, *off_b;            // [nb+1]
+    uint32_t *cnt_c, *fill_c, *off_c;            // [C+1] (zeroed)
+    uint32_t *cnt_b, *fill_b, *off_b;            // [nb+1] (zeroed)
     WinRec *list_c, *list_b;
     uint64_t cap_c, cap_b;
-    uint64_t* sk[2];                             // [n] sort keys (ping-pong)
+    uint64_t* sk[2];                             // [n] sort keys
     uint32_t* sv[2];                             // [n] sort values
+    unsigned long long* rank;                    // [n] (contributions << 32) | rank
     uint64_t* i_base;                            // [n]
     IRest* i_rest;                               // [n]
     uint32_t* i_tf;                              // [n]
@@ -99,28 +105,19 @@ struct Dev {  // scratch of one call (device pointers)
     uint64_t* fence;                             // [kFenceCap]
     uint32_t* chunk_cnt;                         // [C]
     uint64_t* staging;                           // [n_words] records, warp-dense per 32 words
-    unsigned long long* lookback;                // [C]
 };
 
 struct P {  // kernel parameters
     MaterializeArgs a;
     Dev d;
-    uint32_t C, nb;
+    uint32_t C, nb, nstride;  // chunks, check blocks, node-fence stride
+    int merge_mode;           // 1: I keys merged by passes (very large traces)
 };
 
 __device__ __forceinline__ void flag(Ctl* c, unsigned int bit) { atomicOr(&c->status, bit); }
 
 __device__ __forceinline__ bool kv_less(uint64_t ka, uint32_t va, uint64_t kb, uint32_t vb) {
     return ka < kb || (ka == kb && va < vb);
-}
-
-__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
-    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 __device__ __forceinline__ uint64_t warp_min_u64(uint64_t v) {
@@ -134,16 +131,55 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
     return v;
 }
 
-// number of merge passes that do work for nI keys (the tile sort writes buffer 1)
+__device__ __forceinline__ uint32_t n_tiles(uint32_t nI) { return (nI + kSortTile - 1) / kSortTile; }
+// number of merge passes that do work for nI keys (merge mode; tiles are in buffer 1)
 __device__ __forceinline__ int merge_passes(uint32_t nI) {
     int e = 0;
     for (uint64_t w = kSortTile; w < nI; w *= 2) ++e;
     return e;
 }
+// buffer holding the fully sorted I keys
+__device__ __forceinline__ int final_buffer(const P& p, uint32_t nI) {
+    if (p.merge_mode) return (1 + merge_passes(nI)) & 1;
+    return n_tiles(nI) > 1 ? 0 : 1;
+}
+
+// Exclusive scan of cnt[0..n) into off[0..n] (off[n] = total) by one CTA of any
+// size <= 1024 (multiple of 32); reads through L2 (values written by other CTAs).
+__device__ void block_exclusive_scan(const uint32_t* cnt, uint32_t* off, uint32_t n, unsigned long long* total) {
+    __shared__ unsigned long long s_w[32];
+    const uint32_t T = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t per = (n + T - 1) / T;
+    const uint32_t b = min(tid * per, n), e = min(b + per, n);
+    unsigned long long s = 0;
+    for (uint32_t k = b; k < e; ++k) s += __ldcg(cnt + k);
+    unsigned long long incl = s;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += y;
+    }
+    if (lane == 31) s_w[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+        unsigned long long v = lane < T / 32 ? s_w[lane] : 0, iv = v;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const unsigned long long y = __shfl_up_sync(0xffffffffu, iv, d);
+            if (lane >= d) iv += y;
+        }
+        s_w[lane] = iv - v;  // exclusive prefix of warp totals
+    }
+    __syncthreads();
+    unsigned long long run = s_w[warp] + incl - s;
+    for (uint32_t k = b; k < e; ++k) { off[k] = (uint32_t)min(run, 0xFFFFFFFFull); run += __ldcg(cnt + k); }
+    if (tid == T - 1) { *total = run; off[n] = (uint32_t)min(run, 0xFFFFFFFFull); }
+    __syncthreads();
+}
 
 // ----------------------------------------------------------------------------
 // 1. nodes and chunks: CSR / order checks; node j writes the chunks whose first
-//    or last word it holds (no search)
+//    or last word it holds (no search) and, every nstride nodes, a node fence
 __global__ void k_nodes_chunks(P p) {
     const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const MaterializeArgs& a = p.a;
@@ -157,14 +193,15 @@ __global__ void k_nodes_chunks(P p) {
     }
     const uint64_t o1 = a.node_off[i + 1];
     const uint32_t t = a.node_t[i];
+    if (i % p.nstride == 0) p.d.node_fence[i / p.nstride] = t;
     if (o1 < o0) { flag(p.d.ctl, ST_INVALID); return; }
     if (i + 1 < N && !(t < a.node_t[i + 1])) flag(p.d.ctl, ST_INVALID);
     if (o1 == o0 || o1 > a.n_words) return;
     for (uint64_t c = o0 / kChunkWords; c <= (o1 - 1) / kChunkWords; ++c) {
         const uint64_t cs = c * kChunkWords;
         const uint64_t ce = min(cs + kChunkWords, a.n_words) - 1;
-        if (o0 <= cs) { p.d.jf[c] = (uint32_t)i; p.d.tmin[c] = t; }
-        if (ce < o1) { p.d.jl[c] = (uint32_t)i; p.d.tmax[c] = t; }
+        if (o0 <= cs) p.d.jf[c] = (uint32_t)i;
+        if (ce < o1) p.d.jl[c] = (uint32_t)i;
     }
 }
 
@@ -172,8 +209,7 @@ __global__ void k_nodes_chunks(P p) {
 // 2. allocations: checks, I/M split, registration ranges and counts
 // first index k in [lo, n) with t[k] >= x (galloping from lo; t ascending)
 __device__ __forceinline__ uint32_t gallop_ge(const uint32_t* t, uint32_t lo, uint32_t n, uint32_t x) {
-    uint32_t step = 1, prev = lo;
-    uint32_t hi = lo;
+    uint32_t step = 1, prev = lo, hi = lo;
     while (hi < n && t[hi] < x) { prev = hi + 1; hi = hi + step; step <<= 1; }
     if (hi > n) hi = n;
     uint32_t l = prev;
@@ -181,8 +217,7 @@ __device__ __forceinline__ uint32_t gallop_ge(const uint32_t* t, uint32_t lo, ui
     return l;
 }
 __device__ __forceinline__ uint32_t gallop_alloc_ge(const medusa_alloc* al, uint32_t lo, uint32_t n, uint32_t x) {
-    uint32_t step = 1, prev = lo;
-    uint32_t hi = lo;
+    uint32_t step = 1, prev = lo, hi = lo;
     while (hi < n && al[hi].t_alloc < x) { prev = hi + 1; hi = hi + step; step <<= 1; }
     if (hi > n) hi = n;
     uint32_t l = prev;
@@ -191,13 +226,18 @@ __device__ __forceinline__ uint32_t gallop_alloc_ge(const medusa_alloc* al, uint
 }
 
 __global__ void __launch_bounds__(256) k_allocs(P p) {
+    __shared__ uint32_t s_nf[kNodeFenceCap];
+    __shared__ uint32_t s_last;
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     const MaterializeArgs& a = p.a;
     const uint32_t lane = threadIdx.x & 31;
+    const uint32_t N = a.n_nodes;
+    const uint32_t nnf = (N + p.nstride - 1) / p.nstride;
+    for (uint32_t f = threadIdx.x; f < nnf; f += blockDim.x) s_nf[f] = p.d.node_fence[f];
+    __syncthreads();
     const bool valid = i < a.n_alloc;
     medusa_alloc x{};
     if (valid) x = a.alloc[i];
-    const uint32_t N = a.n_nodes;
     const uint32_t t_last = N ? a.node_t[N - 1] : 0;
     bool isI = false;
     uint4 r = make_uint4(1, 0, 1, 0);  // empty ranges
@@ -210,9 +250,14 @@ __global__ void __launch_bounds__(256) k_allocs(P p) {
             if (!isI) {
                 if (p.C && N && x.t_alloc < x.t_free) {
                     // nodes launched while i is live: [j0, j1) = t in (t_alloc, t_free)
-                    uint32_t lo = 0, hi = N;
-                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.node_t[m] <= x.t_alloc) lo = m + 1; else hi = m; }
-                    const uint32_t j0 = lo;
+                    uint32_t lo = 0, hi = nnf;  // fences <= t_alloc
+                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (s_nf[m] <= x.t_alloc) lo = m + 1; else hi = m; }
+                    uint32_t j0 = 0;
+                    if (lo > 0) {
+                        uint32_t l2 = (lo - 1) * p.nstride + 1, h2 = min(lo * p.nstride, N);
+                        while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (a.node_t[m] <= x.t_alloc) l2 = m + 1; else h2 = m; }
+                        j0 = l2;
+                    }
                     const uint32_t j1 = gallop_ge(a.node_t, j0, N, x.t_free);
                     // chunks holding their words (exact: no entry for memory no launch can see)
                     if (j0 < j1) {
@@ -251,49 +296,23 @@ __global__ void __launch_bounds__(256) k_allocs(P p) {
         atomicMax(&p.d.ctl->gmin_c, ~(unsigned long long)mn);
         atomicMax(&p.d.ctl->gmax, (unsigned long long)mx);
     }
-}
-
-// ----------------------------------------------------------------------------
-// 3. exclusive scans of the registration counts (one CTA of 1024 threads)
-__device__ void block_exclusive_scan(const uint32_t* cnt, uint32_t* off, uint32_t n, unsigned long long* total) {
-    __shared__ unsigned long long s_w[32];
-    const uint32_t T = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t per = (n + T - 1) / T;
-    const uint32_t b = min(tid * per, n), e = min(b + per, n);
-    unsigned long long s = 0;
-    for (uint32_t k = b; k < e; ++k) s += cnt[k];
-    unsigned long long incl = s;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, d);
-        if (lane >= d) incl += y;
-    }
-    if (lane == 31) s_w[warp] = incl;
+    // the last CTA turns the registration counts into offsets
     __syncthreads();
-    if (warp == 0) {
-        unsigned long long v = lane < T / 32 ? s_w[lane] : 0, iv = v;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const unsigned long long y = __shfl_up_sync(0xffffffffu, iv, d);
-            if (lane >= d) iv += y;
-        }
-        s_w[lane] = iv - v;  // exclusive prefix of warp totals
+    if (threadIdx.x == 0) {
+        __threadfence();
+        s_last = atomicAdd(&p.d.ctl->done_allocs, 1u) == gridDim.x - 1;
     }
     __syncthreads();
-    unsigned long long run = s_w[warp] + incl - s;
-    for (uint32_t k = b; k < e; ++k) { off[k] = (uint32_t)min(run, 0xFFFFFFFFull); run += cnt[k]; }
-    if (tid == T - 1) { *total = run; off[n] = (uint32_t)min(run, 0xFFFFFFFFull); }
-    __syncthreads();
+    if (s_last) {
+        __threadfence();
+        block_exclusive_scan(p.d.cnt_c, p.d.off_c, p.C, &p.d.ctl->need_c);
+        block_exclusive_scan(p.d.cnt_b, p.d.off_b, p.nb, &p.d.ctl->need_b);
+        if (threadIdx.x == 0 && (p.d.ctl->need_c > p.d.cap_c || p.d.ctl->need_b > p.d.cap_b))
+            flag(p.d.ctl, ST_OVERFLOW);
+    }
 }
 
-__global__ void __launch_bounds__(1024) k_scan(P p) {
-    block_exclusive_scan(p.d.cnt_c, p.d.off_c, p.C, &p.d.ctl->need_c);
-    block_exclusive_scan(p.d.cnt_b, p.d.off_b, p.nb, &p.d.ctl->need_b);
-    if (threadIdx.x == 0 && (p.d.ctl->need_c > p.d.cap_c || p.d.ctl->need_b > p.d.cap_b))
-        flag(p.d.ctl, ST_OVERFLOW);
-}
-
-// 4. registration lists (32-byte records, so readers need no second gather)
+// 3. registration lists (32-byte records, so readers need no second gather)
 __global__ void k_scatter(P p) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= p.a.n_alloc) return;
@@ -312,14 +331,44 @@ __global__ void k_scatter(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 5. sort I by (base, index): each warp sorts 256 keys in registers (bitonic
-//    network over shuffles), the CTA merges its 8 runs to a 2048 tile in shared
-//    memory, then merge-path passes (only those the device-side count needs do
-//    any work)
+// 4. sort I by (base, index)
 __device__ __forceinline__ void cas(uint64_t& ka, uint32_t& va, uint64_t& kb, uint32_t& vb, bool up) {
     if (kv_less(kb, vb, ka, va) == up) {
         const uint64_t tk = ka; ka = kb; kb = tk;
         const uint32_t tv = va; va = vb; vb = tv;
+    }
+}
+
+// Bitonic sort of 32*E (key, val) pairs held E per lane (element e = lane*E + r),
+// ascending, by shuffles and register compare-exchanges (no shared memory).
+template <int E>
+__device__ __forceinline__ void warp_bitonic(uint64_t (&k)[E], uint32_t (&v)[E]) {
+    const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+    for (uint32_t size = 2; size <= 32u * E; size <<= 1) {
+#pragma unroll
+        for (uint32_t j = size >> 1; j > 0; j >>= 1) {
+            if (j >= (uint32_t)E) {
+                const uint32_t lj = j / E;
+#pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const uint32_t e = lane * E + r;
+                    const uint64_t ok = __shfl_xor_sync(0xffffffffu, k[r], lj);
+                    const uint32_t ov = __shfl_xor_sync(0xffffffffu, v[r], lj);
+                    const bool up = (e & size) == 0;
+                    const bool lower = (e & j) == 0;
+                    const bool other_less = kv_less(ok, ov, k[r], v[r]);
+                    // lower element keeps the min when ascending, the max when descending
+                    if ((lower == up) ? other_less : !other_less) { k[r] = ok; v[r] = ov; }
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const int r2 = r ^ (int)j;
+                    if (r2 > r) cas(k[r], v[r], k[r2], v[r2], ((lane * E + r) & size) == 0);
+                }
+            }
+        }
     }
 }
 
@@ -340,60 +389,26 @@ __global__ void __launch_bounds__(256) k_sort_tile(P p) {
     const uint32_t t0 = blockIdx.x * kSortTile;
     if (t0 >= n) return;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint64_t* kin = p.d.sk[0];
-    const uint32_t* vin = p.d.sv[0];
-    // 1. warp run of 256: lane holds elements e = lane*8 + r
     uint64_t k[8];
     uint32_t v[8];
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
         const uint32_t g = t0 + warp * 256 + lane * 8 + r;
-        k[r] = g < n ? kin[g] : ~0ull;
-        v[r] = g < n ? vin[g] : 0xFFFFFFFFu;
+        k[r] = g < n ? p.d.sk[0][g] : ~0ull;
+        v[r] = g < n ? p.d.sv[0][g] : 0xFFFFFFFFu;
     }
-#pragma unroll
-    for (uint32_t size = 2; size <= 256; size <<= 1) {
-#pragma unroll
-        for (uint32_t j = size >> 1; j > 0; j >>= 1) {
-            if (j >= 8) {
-                const uint32_t lj = j >> 3;
-#pragma unroll
-                for (int r = 0; r < 8; ++r) {
-                    const uint32_t e = lane * 8 + r;
-                    const uint64_t ok = __shfl_xor_sync(0xffffffffu, k[r], lj);
-                    const uint32_t ov = __shfl_xor_sync(0xffffffffu, v[r], lj);
-                    const bool up = (e & size) == 0;
-                    const bool lower = (e & j) == 0;
-                    const bool other_less = kv_less(ok, ov, k[r], v[r]);
-                    // lower element keeps the min when ascending, the max when descending
-                    const bool take = (lower == up) ? other_less : !other_less;
-                    if (take) { k[r] = ok; v[r] = ov; }
-                }
-            } else {
-#pragma unroll
-                for (int r = 0; r < 8; ++r) {
-                    const int r2 = r ^ (int)j;
-                    if (r2 > r) {
-                        const uint32_t e = lane * 8 + r;
-                        cas(k[r], v[r], k[r2], v[r2], (e & size) == 0);
-                    }
-                }
-            }
-        }
-    }
+    warp_bitonic<8>(k, v);
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
         sk[0][warp * 256 + lane * 8 + r] = k[r];
         sv[0][warp * 256 + lane * 8 + r] = v[r];
     }
     __syncthreads();
-    // 2. merge runs 256 -> 2048 in shared memory (8 outputs per thread per round)
     int src = 0;
 #pragma unroll
     for (uint32_t run = 256; run < kSortTile; run <<= 1) {
         const uint32_t o = tid * 8;
-        const uint32_t pair = o / (2 * run);
-        const uint32_t a0 = pair * 2 * run, b0 = a0 + run;
+        const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
         const uint32_t d = o - a0;
         const uint64_t* ka = sk[src] + a0;
         const uint32_t* va = sv[src] + a0;
@@ -414,6 +429,34 @@ __global__ void __launch_bounds__(256) k_sort_tile(P p) {
     for (uint32_t q = tid; q < kSortTile && t0 + q < n; q += blockDim.x) {
         p.d.sk[1][t0 + q] = sk[src][q];
         p.d.sv[1][t0 + q] = sv[src][q];
+        p.d.rank[t0 + q] = q;  // rank within the tile, no contribution yet
+    }
+}
+
+// global rank = own tile index + sum over every other tile of #keys below; the
+// thread adding the last contribution scatters the key to its final position
+__global__ void __launch_bounds__(256) k_rank(P p) {
+    const uint32_t nI = p.d.ctl->nI;
+    const uint32_t T = n_tiles(nI);
+    if (T <= 1) return;
+    const uint64_t pairs = (uint64_t)nI * T;
+    const uint64_t* sk = p.d.sk[1];
+    const uint32_t* sv = p.d.sv[1];
+    for (uint64_t q = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; q < pairs; q += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t t = (uint32_t)(q / nI), k = (uint32_t)(q % nI);
+        if (t == k / kSortTile) continue;
+        const uint64_t kk = sk[k];
+        const uint32_t vk = sv[k];
+        uint32_t lo = t * kSortTile, hi = min(lo + kSortTile, nI);
+        const uint32_t base = lo;
+        while (lo < hi) { const uint32_t m = (lo + hi) >> 1; if (kv_less(sk[m], sv[m], kk, vk)) lo = m + 1; else hi = m; }
+        const uint32_t cnt = lo - base;
+        const unsigned long long old = atomicAdd(&p.d.rank[k], (1ull << 32) | cnt);
+        if ((old >> 32) + 1 == T - 1) {
+            const uint32_t r = (uint32_t)old + cnt;
+            p.d.sk[0][r] = kk;
+            p.d.sv[0][r] = vk;
+        }
     }
 }
 
@@ -435,9 +478,9 @@ __device__ uint32_t merge_path_warp(const uint64_t* ka, const uint32_t* va, cons
         } else {
             const uint32_t f = __ffs(b) - 1;
             const uint32_t nhi = lo + f * step;
-            lo = f ? lo + (f - 1) * step + 1 : lo;
-            hi = nhi;
             if (f == 0) return lo;
+            lo = lo + (f - 1) * step + 1;
+            hi = nhi;
         }
     }
     return lo;
@@ -483,13 +526,8 @@ __global__ void __launch_bounds__(256) k_merge(P p, uint32_t width, int pass) {
     const uint32_t per = kMergeTile / 256;
     const uint32_t d = threadIdx.x * per;
     if (d < na + nbb) {
-        uint32_t lo = d > nbb ? d - nbb : 0, hi = min(d, na);
-        while (lo < hi) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (kv_less(sk[na + d - 1 - mid], sv[na + d - 1 - mid], sk[mid], sv[mid])) hi = mid;
-            else lo = mid + 1;
-        }
-        uint32_t ia = lo, ib = d - lo;
+        uint32_t ia = merge_path_smem(sk, sv, sk + na, sv + na, d, d > nbb ? d - nbb : 0, min(d, na));
+        uint32_t ib = d - ia;
         for (uint32_t q = 0; q < per && d + q < na + nbb; ++q) {
             const bool takeA = ib >= nbb || (ia < na && kv_less(sk[ia], sv[ia], sk[na + ib], sv[na + ib]));
             const uint32_t s = takeA ? ia++ : na + ib++;
@@ -499,12 +537,12 @@ __global__ void __launch_bounds__(256) k_merge(P p, uint32_t width, int pass) {
     }
 }
 
-// 6. I arrays, I-I adjacency check, shared-memory fences, 32-entry summaries
-__global__ void __launch_bounds__(256) k_build_i(P p) {
+// 5. I arrays, I-I adjacency check, shared-memory fences, 32-entry summaries
+__global__ void __launch_bounds__(256) k_finalize_i(P p) {
     const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
     const uint32_t nI = p.d.ctl->nI;
     if (k - (threadIdx.x & 31) >= nI) return;  // whole warp past the end
-    const int fin = (1 + merge_passes(nI)) & 1;
+    const int fin = final_buffer(p, nI);
     const uint64_t* sk = p.d.sk[fin];
     const uint32_t* sv = p.d.sv[fin];
     uint32_t ta = 0xFFFFFFFFu, tf = 0;
@@ -528,11 +566,6 @@ __global__ void __launch_bounds__(256) k_build_i(P p) {
     }
 }
 
-// ----------------------------------------------------------------------------
-// 7. overlap checks for mortal allocations.  A CTA of 256 threads covers four
-//    registration blocks of 64 ordinals; the I-list fences sit in shared memory.
-constexpr int kChkThreads = 4 * kAblk;
-
 // count of sorted I bases <= x (fences in shared memory, then one group of <= stride
 // bases read with independent loads)
 __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t nf, uint32_t stride, uint32_t nI,
@@ -553,18 +586,22 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
     return c;
 }
 
-__global__ void __launch_bounds__(kChkThreads) k_check(P p) {
+// ----------------------------------------------------------------------------
+// 6. overlap checks for mortal allocations: one warp per block of 32 ordinals
+__global__ void __launch_bounds__(256) k_check(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
-    __shared__ uint64_t s_base[4][kChkCap], s_end[4][kChkCap];
-    __shared__ uint32_t s_tf[4][kChkCap], s_idx[4][kChkCap];
+    __shared__ uint64_t s_base[8][kChkCap], s_end[8][kChkCap];
+    __shared__ uint32_t s_tf[8][kChkCap], s_idx[8][kChkCap];
     const MaterializeArgs& a = p.a;
-    const uint32_t sub = threadIdx.x / kAblk;          // registration block within the CTA
-    const uint32_t b = blockIdx.x * 4 + sub;
-    const uint32_t j = blockIdx.x * kChkThreads + threadIdx.x;
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t b = blockIdx.x * 8 + warp;
+    const uint32_t j = b * kAblk + lane;
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t stride = nI ? (nI + kFenceCap - 1) / kFenceCap : 1;
     const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = threadIdx.x; f < nf; f += kChkThreads) s_fence[f] = p.d.fence[f];
+    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = p.d.fence[f];
+    __syncthreads();
+    if (b >= p.nb) return;  // whole warp
     bool mine = false;
     medusa_alloc x{};
     const uint32_t N = a.n_nodes;
@@ -575,34 +612,23 @@ __global__ void __launch_bounds__(kChkThreads) k_check(P p) {
     }
     const uint64_t xe = x.base + x.size;
     bool bad = false;
-    // M-M: registered mortals live at some allocation of this block
-    uint64_t r0 = 0, r1 = 0;
-    if (b < p.nb) {
-        r0 = p.d.off_b[b];
-        r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
-    }
-    uint32_t rounds = (uint32_t)((r1 - r0 + kChkCap - 1) / kChkCap);
-    rounds = __reduce_max_sync(0xffffffffu, rounds);
-    __shared__ uint32_t s_rounds[kChkThreads / 32];
-    if ((threadIdx.x & 31) == 0) s_rounds[threadIdx.x >> 5] = rounds;
-    __syncthreads();
-    uint32_t all_rounds = 0;
-    for (int w = 0; w < kChkThreads / 32; ++w) all_rounds = max(all_rounds, s_rounds[w]);
-    for (uint32_t rd = 0; rd < all_rounds; ++rd) {
-        const uint64_t bs = r0 + (uint64_t)rd * kChkCap;
-        const uint32_t m = bs < r1 ? (uint32_t)min((uint64_t)kChkCap, r1 - bs) : 0;
-        __syncthreads();
-        for (uint32_t q = threadIdx.x % kAblk; q < m; q += kAblk) {
+    // M-M: mortals registered as live at some allocation of this block
+    const uint64_t r0 = p.d.off_b[b];
+    const uint64_t r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
+    for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
+        const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
+        __syncwarp();
+        for (uint32_t q = lane; q < m; q += 32) {
             const WinRec y = p.d.list_b[bs + q];
-            s_base[sub][q] = y.base;
-            s_end[sub][q] = y.end;
-            s_tf[sub][q] = y.t_free;
-            s_idx[sub][q] = y.id;
+            s_base[warp][q] = y.base;
+            s_end[warp][q] = y.end;
+            s_tf[warp][q] = y.t_free;
+            s_idx[warp][q] = y.id;
         }
-        __syncthreads();
+        __syncwarp();
         if (mine && !bad) {
             for (uint32_t q = 0; q < m; ++q) {
-                if (s_idx[sub][q] < j && s_tf[sub][q] > x.t_alloc && s_base[sub][q] < xe && x.base < s_end[sub][q]) {
+                if (s_idx[warp][q] < j && s_tf[warp][q] > x.t_alloc && s_base[warp][q] < xe && x.base < s_end[warp][q]) {
                     bad = true;
                     break;
                 }
@@ -628,25 +654,69 @@ __global__ void __launch_bounds__(kChkThreads) k_check(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 8. classify one chunk per CTA
+// 7. classify one chunk per CTA
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     uint64_t fence[kFenceCap];
     uint32_t tw[MEDUSA_CHUNK_WORDS];     // launch position of every word
-    uint64_t key[kWinCap];
-    uint64_t end[kWinCap];
-    uint64_t pmax[kWinCap];
-    uint32_t ta[kWinCap], tf[kWinCap], id[kWinCap];
-    uint16_t val[kWinCap];
-    uint16_t queue[MEDUSA_CHUNK_WORDS];
+    uint64_t wb[kWinCap], we[kWinCap], wpmax[kWinCap];  // window, physically sorted by base
+    uint32_t wta[kWinCap], wtf[kWinCap], wid[kWinCap];
+    uint16_t cq[MEDUSA_CHUNK_WORDS];     // candidate words (could point into memory)
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32];
     uint32_t wmax[kWarps];
-    uint32_t nq, total;
+    uint32_t nc, total, last;
     unsigned long long mbar;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// warp 0: load a batch of <= kWinCap registered mortals, sort by base, lay them out
+// physically sorted, prefix max of end
+__device__ __forceinline__ void window_prepare(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
+    const uint32_t lane = threadIdx.x & 31;
+    constexpr int E = kWinCap / 32;
+    uint64_t k[E];
+    uint32_t v[E];
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+        const uint32_t e = lane * E + r;
+        k[r] = e < m ? p.d.list_c[bs + e].base : ~0ull;
+        v[r] = e;
+    }
+    warp_bitonic<E>(k, v);
+    uint64_t ends[E];
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+        const uint32_t e = lane * E + r;
+        ends[r] = 0;
+        if (e < m) {
+            const WinRec x = p.d.list_c[bs + v[r]];
+            S.wb[e] = x.base;
+            S.we[e] = x.end;
+            S.wta[e] = x.t_alloc;
+            S.wtf[e] = x.t_free;
+            S.wid[e] = x.id;
+            ends[r] = x.end;
+        }
+    }
+    uint64_t run = 0;
+#pragma unroll
+    for (int r = 0; r < E; ++r) { run = max(run, ends[r]); ends[r] = run; }
+    uint64_t incl = run;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint64_t y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl = max(incl, y);
+    }
+    uint64_t before = __shfl_up_sync(0xffffffffu, incl, 1);
+    if (lane == 0) before = 0;
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+        const uint32_t e = lane * E + r;
+        if (e < m) S.wpmax[e] = max(before, ends[r]);
+    }
 }
 
 __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
@@ -660,9 +730,9 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
     const uint64_t* gsrc = a.words + cs;
     const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
-    // 1. the chunk's words -> shared memory with one bulk copy (TMA engine)
+    // A. the chunk's words -> shared memory with one bulk copy (TMA engine)
     if (tid == 0) {
-        S.nq = 0;
+        S.nc = 0;
         S.total = 0;
         if (tma) {
             const uint32_t mb = smem_u32(&S.mbar);
@@ -675,7 +745,6 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     }
     if (!tma)
         for (uint32_t q = tid; q < n; q += kClsThreads) S.words[q] = ld_stream(gsrc + q);
-    // 2. meanwhile: fences, launch positions, the mortal window
     const uint32_t nI = ctl->nI;
     const uint32_t stride = nI ? (nI + kFenceCap - 1) / kFenceCap : 1;
     const uint32_t nf = (nI + stride - 1) / stride;
@@ -687,10 +756,13 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     const uint64_t r0 = p.d.off_c[c];
     const uint64_t r1 = min((uint64_t)p.d.off_c[c + 1], p.d.cap_c);
     __syncthreads();
-    if (N) {
+    // B. warp 0: first window batch; warps 1..7: node starts -> launch positions
+    if (warp == 0) {
+        if (r0 < r1) window_prepare(p, S, r0, (uint32_t)min((uint64_t)kWinCap, r1 - r0));
+    } else if (N) {
         const uint32_t jf = min(p.d.jf[c], N - 1), jl = min(p.d.jl[c], N - 1);
-        if (tid == 0) atomicMax(&S.tw[0], a.node_t[jf]);
-        for (uint32_t j = jf + 1 + tid; j <= jl; j += kClsThreads) {
+        if (tid == 32) atomicMax(&S.tw[0], a.node_t[jf]);
+        for (uint32_t j = jf + 1 + (tid - 32); j <= jl; j += kClsThreads - 32) {
             const uint64_t q = a.node_off[j] - cs;
             if (q < n) atomicMax(&S.tw[q], a.node_t[j]);
         }
@@ -723,111 +795,69 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
                          : "=r"(done) : "r"(mb) : "memory");
         }
     }
-    __syncthreads();
-    // 3. mortal window(s): sorted by base, prefix max of end, backward walk
-    for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
-        const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
-        uint32_t mp = 32;
-        while (mp < m) mp <<= 1;
-        for (uint32_t q = tid; q < mp; q += kClsThreads) {
-            if (q < m) {
-                const WinRec x = p.d.list_c[bs + q];
-                S.key[q] = x.base;
-                S.end[q] = x.end;
-                S.ta[q] = x.t_alloc;
-                S.tf[q] = x.t_free;
-                S.id[q] = x.id;
-            } else {
-                S.key[q] = ~0ull;
-            }
-            S.val[q] = (uint16_t)q;
-        }
-        __syncthreads();
-        for (uint32_t size = 2; size <= mp; size <<= 1) {
-            for (uint32_t st = size >> 1; st > 0; st >>= 1) {
-                for (uint32_t q = tid; q < mp / 2; q += kClsThreads) {
-                    const uint32_t lo = 2 * q - (q & (st - 1)), hi = lo + st;
-                    const bool up = (lo & size) == 0;
-                    const uint64_t ka = S.key[lo], kb = S.key[hi];
-                    const uint16_t va = S.val[lo], vb = S.val[hi];
-                    if (kv_less(kb, vb, ka, va) == up) { S.key[lo] = kb; S.key[hi] = ka; S.val[lo] = vb; S.val[hi] = va; }
-                }
-                __syncthreads();
-            }
-        }
-        if (warp == 0) {  // prefix max of end in sorted order
-            const uint32_t per = (m + 31) / 32;
-            const uint32_t b = min(lane * per, m), e = min(b + per, m);
-            uint64_t run = 0;
-            for (uint32_t q = b; q < e; ++q) run = max(run, S.end[S.val[q]]);
-            uint64_t incl = run;
+    // C. candidates: words inside [least base, greatest end) of the trace
 #pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const uint64_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                if (lane >= d) incl = max(incl, y);
-            }
-            uint64_t acc = __shfl_up_sync(0xffffffffu, incl, 1);
-            if (lane == 0) acc = 0;
-            for (uint32_t q = b; q < e; ++q) { acc = max(acc, S.end[S.val[q]]); S.pmax[q] = acc; }
-        }
-        __syncthreads();
-#pragma unroll 2
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            const uint32_t q = k * kClsThreads + tid;
-            bool hit = false;
-            if (q < n && !((S.hits[q >> 5] >> (q & 31)) & 1u)) {
-                const uint64_t x = S.words[q];
-                if (x >= gmin && x < gmax) {
-                    const uint32_t t = S.tw[q];
-                    uint32_t lo = 0, hi = m;  // count of keys <= x
-                    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.key[mid] <= x) lo = mid + 1; else hi = mid; }
-                    for (int r = (int)lo - 1; r >= 0 && S.pmax[r] > x; --r) {
-                        const uint32_t u = S.val[r];
-                        if (x < S.end[u] && S.ta[u] < t && t < S.tf[u]) {
-                            hit = true;
-                            S.words[q] = ((uint64_t)S.id[u] << MEDUSA_OFF_BITS) | (x - S.key[r]);
-                            break;
-                        }
-                    }
-                }
-            }
-            const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-            if (lane == 0 && bal) S.hits[q >> 5] |= bal;  // one warp owns this hits word
-        }
-        __syncthreads();
-    }
-    // 4. words still unresolved that could point into memory -> the I-list queue
-#pragma unroll 2
     for (int k = 0; k < kWordsPerThread; ++k) {
         const uint32_t q = k * kClsThreads + tid;
-        bool need = false;
-        if (q < n && nI && !((S.hits[q >> 5] >> (q & 31)) & 1u)) {
+        bool cand = false;
+        if (q < n) {
             const uint64_t x = S.words[q];
-            need = x >= gmin && x < gmax && x >= S.fence[0];
+            cand = x >= gmin && x < gmax;
         }
-        const uint32_t bal = __ballot_sync(0xffffffffu, need);
+        const uint32_t bal = __ballot_sync(0xffffffffu, cand);
         uint32_t base = 0;
-        if (lane == 0 && bal) base = atomicAdd(&S.nq, (uint32_t)__popc(bal));
+        if (lane == 0 && bal) base = atomicAdd(&S.nc, (uint32_t)__popc(bal));
         base = __shfl_sync(0xffffffffu, base, 0);
-        if (need) S.queue[base + __popc(bal & lanemask_lt())] = (uint16_t)q;
+        if (cand) S.cq[base + __popc(bal & lanemask_lt())] = (uint16_t)q;
     }
     __syncthreads();
-    // 5. I-list search: fences in shared memory, then one group of <= stride bases
-    const uint32_t nq = S.nq;
-    for (uint32_t i = tid; i < nq; i += kClsThreads) {
-        const uint32_t q = S.queue[i];
-        const uint64_t x = S.words[q];
-        const uint32_t t = S.tw[q];
-        const uint32_t kk = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x) - 1;  // >= 0: x >= fence[0]
-        const uint64_t base = p.d.i_base[kk];
-        const IRest e = p.d.i_rest[kk];
-        if (x < e.end && e.t_alloc < t) {
-            S.words[q] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (x - base);
-            atomicOr(&S.hits[q >> 5], 1u << (q & 31));
+    const uint32_t nc = S.nc;
+    // D. mortal window(s): binary search by base, backward walk while the prefix
+    //    max of end still reaches the word, time check
+    for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
+        const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
+        if (bs != r0) {
+            __syncthreads();
+            if (warp == 0) window_prepare(p, S, bs, m);
+            __syncthreads();
+        }
+        for (uint32_t i = tid; i < nc; i += kClsThreads) {
+            const uint32_t q = S.cq[i];
+            if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
+            const uint64_t x = S.words[q];
+            const uint32_t t = S.tw[q];
+            uint32_t lo = 0, hi = m;  // count of bases <= x
+            while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
+            for (int r = (int)lo - 1; r >= 0 && S.wpmax[r] > x; --r) {
+                if (x < S.we[r] && S.wta[r] < t && t < S.wtf[r]) {
+                    S.words[q] = ((uint64_t)S.wid[r] << MEDUSA_OFF_BITS) | (x - S.wb[r]);
+                    atomicOr(&S.hits[q >> 5], 1u << (q & 31));
+                    break;
+                }
+            }
         }
     }
     __syncthreads();
-    // 6. emission: mask words, warp-dense staging of records, chunk count
+    // E. I list: fences in shared memory, then one group of <= stride bases
+    if (nI) {
+        const uint64_t f0 = S.fence[0];
+        for (uint32_t i = tid; i < nc; i += kClsThreads) {
+            const uint32_t q = S.cq[i];
+            if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
+            const uint64_t x = S.words[q];
+            if (x < f0) continue;
+            const uint32_t t = S.tw[q];
+            const uint32_t kk = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x) - 1;
+            const uint64_t base = p.d.i_base[kk];
+            const IRest e = p.d.i_rest[kk];
+            if (x < e.end && e.t_alloc < t) {
+                S.words[q] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (x - base);
+                atomicOr(&S.hits[q >> 5], 1u << (q & 31));
+            }
+        }
+    }
+    __syncthreads();
+    // F. emission: mask words, warp-dense staging of records, chunk count
     const uint64_t n_mask = (a.n_words + 31) / 32;
     uint32_t cnt = 0;
 #pragma unroll
@@ -841,54 +871,33 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     }
     if (lane == 0) atomicAdd(&S.total, cnt);
     __syncthreads();
-    if (tid == 0) p.d.chunk_cnt[c] = S.total;
+    // G. the last CTA turns the chunk counts into chunk_base
+    if (tid == 0) {
+        p.d.chunk_cnt[c] = S.total;
+        __threadfence();
+        S.last = atomicAdd(&ctl->done_cls, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (S.last) {
+        __threadfence();
+        block_exclusive_scan(p.d.chunk_cnt, a.chunk_base, p.C, &ctl->n_slots);
+    }
 }
 
-// 9. chunk prefix (decoupled look-back over known counts, 32 predecessors per
-//    probe) + record compaction
+// 8. compaction of the staged records into the slot table (one CTA per chunk)
 __global__ void __launch_bounds__(256) k_emit(P p) {
     __shared__ uint32_t s_mask[64];
     __shared__ uint32_t s_pre[64];
-    __shared__ uint32_t s_chunk;
-    __shared__ unsigned long long s_prefix;
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0) s_chunk = atomicAdd(&p.d.ctl->ticket, 1u);
-    __syncthreads();
-    const uint32_t c = s_chunk;
+    const uint32_t c = blockIdx.x;
     const uint64_t n_mask = (a.n_words + 31) / 32;
     const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
-    if (warp == 0) {
-        const uint32_t total = p.d.chunk_cnt[c];
-        if (lane == 0) st_release(&p.d.lookback[c], (c == 0 ? LB_PRE : LB_AGG) | total);
-        uint32_t prefix = 0;
-        if (c > 0) {
-            int64_t top = (int64_t)c - 1;
-            for (;;) {
-                const int64_t idx = top - lane;
-                const unsigned long long v = idx >= 0 ? ld_acquire(&p.d.lookback[idx]) : LB_PRE;
-                if (__ballot_sync(0xffffffffu, (v & ~LB_VAL) == 0)) continue;  // a predecessor not published yet
-                const uint32_t pre = __ballot_sync(0xffffffffu, (v & LB_PRE) != 0);
-                const uint32_t upto = pre ? (__ffs(pre) - 1) : 31;  // nearest inclusive prefix
-                prefix += __reduce_add_sync(0xffffffffu, lane <= upto ? (uint32_t)(v & LB_VAL) : 0u);
-                if (pre) break;
-                top -= 32;
-            }
-            if (lane == 0) st_release(&p.d.lookback[c], LB_PRE | (prefix + total));
-        }
-        if (lane == 0) {
-            a.chunk_base[c] = prefix;
-            if (c + 1 == p.C) {
-                a.chunk_base[p.C] = prefix + total;
-                p.d.ctl->n_slots = (unsigned long long)prefix + total;
-            }
-            s_prefix = prefix;
-        }
-    } else if (warp == 1 || warp == 2) {  // the chunk's 64 mask words and their popcount prefix
-        const uint32_t h = warp - 1;
-        const uint64_t mw = m0 + h * 32 + lane;
+    const uint64_t prefix = a.chunk_base[c];
+    if (warp < 2) {
+        const uint64_t mw = m0 + warp * 32 + lane;
         const uint32_t bits = mw < n_mask ? a.mask[mw] : 0u;
-        s_mask[h * 32 + lane] = bits;
+        s_mask[warp * 32 + lane] = bits;
         const uint32_t pc = __popc(bits);
         uint32_t incl = pc;
 #pragma unroll
@@ -896,19 +905,17 @@ __global__ void __launch_bounds__(256) k_emit(P p) {
             const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
             if (lane >= d) incl += y;
         }
-        s_pre[h * 32 + lane] = incl - pc;
+        s_pre[warp * 32 + lane] = incl - pc;
     }
     __syncthreads();
     if (tid < 32) s_pre[32 + tid] += s_pre[31] + __popc(s_mask[31]);  // second half after the first
     __syncthreads();
-    const unsigned long long prefix = s_prefix;
-    // each warp moves 8 mask-word groups: lane l copies record l of the group
 #pragma unroll
     for (int g = 0; g < 8; ++g) {
         const uint32_t local = warp * 8 + g;
         const uint32_t bits = s_mask[local];
         if (lane < (uint32_t)__popc(bits)) {
-            const unsigned long long dst = prefix + s_pre[local] + lane;
+            const uint64_t dst = prefix + s_pre[local] + lane;
             if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + local) * 32 + lane];
         }
     }
@@ -923,6 +930,7 @@ struct Scratch {
     Dev d{};
     std::vector<void*> bufs;
     Ctl* h_ctl = nullptr;
+    int sm_count = 0;
 };
 std::mutex g_mu;
 std::vector<Scratch*> g_scratch;
@@ -952,26 +960,25 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
     release(s);
     const size_t N = std::max<size_t>(n, 1024), CC = std::max<size_t>(C, 64), NB = std::max<size_t>(nb, 64);
     const size_t WW = std::max<size_t>(W, 2048);
-    const size_t RC = std::max<size_t>(need_c, 2 * N + 4 * CC), RB = std::max<size_t>(need_b, 3 * N);
+    const size_t RC = std::max<size_t>(need_c, N + 4 * CC), RB = std::max<size_t>(need_b, 3 * N);
     cudaError_t e;
-    // zero region: Ctl | cnt_c fill_c [CC+1] | cnt_b fill_b [NB+1] | lookback [CC]
-    s.zero_bytes = 256 + 2 * (CC + 1) * 4 + 2 * (NB + 1) * 4 + 8 * CC + 64;
+    // zero region: Ctl | cnt_c fill_c off_c [CC+1] | cnt_b fill_b off_b [NB+1]
+    s.zero_bytes = 256 + 3 * (CC + 1) * 4 + 3 * (NB + 1) * 4 + 64;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
     char* z = (char*)s.zero_region;
     s.d.ctl = (Ctl*)z;
     size_t o = 256;
     s.d.cnt_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
     s.d.fill_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
+    s.d.off_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
     s.d.cnt_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
     s.d.fill_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
-    o = (o + 7) & ~size_t(7);
-    s.d.lookback = (unsigned long long*)(z + o);
-    if ((e = grow(s, s.d.tmin, CC)) || (e = grow(s, s.d.tmax, CC)) || (e = grow(s, s.d.jf, CC)) ||
-        (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.rng, N)) || (e = grow(s, s.d.off_c, CC + 1)) ||
-        (e = grow(s, s.d.off_b, NB + 1)) || (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) ||
+    s.d.off_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
+    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.node_fence, (size_t)kNodeFenceCap)) ||
+        (e = grow(s, s.d.rng, N)) || (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) ||
         (e = grow(s, s.d.sk[0], N)) || (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) ||
-        (e = grow(s, s.d.sv[1], N)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
-        (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.blk_min_ta, N / kIBlk + 1)) ||
+        (e = grow(s, s.d.sv[1], N)) || (e = grow(s, s.d.rank, N)) || (e = grow(s, s.d.i_base, N)) ||
+        (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.blk_min_ta, N / kIBlk + 1)) ||
         (e = grow(s, s.d.blk_max_tf, N / kIBlk + 1)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
         (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)))
         return e;
@@ -996,14 +1003,18 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     if (!s.h_ctl) {
         if ((e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ClsShared));
+        cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
     const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
+    const uint32_t nstride = std::max<uint32_t>(1, (a.n_nodes + kNodeFenceCap - 1) / kNodeFenceCap);
+    const uint64_t max_tiles = (n + kSortTile - 1) / kSortTile;
+    const int merge_mode = max_tiles > kRankMaxTiles ? 1 : 0;
     size_t need_c = 0, need_b = 0;
     for (int attempt = 0; attempt < 3; ++attempt) {
         if ((e = ensure(s, n, C, nb, a.n_words, need_c, need_b)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-        P p{a, s.d, C, nb};
+        P p{a, s.d, C, nb, nstride, merge_mode};
         if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) break;
         if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) break;
         const uint32_t T = 256;
@@ -1012,33 +1023,37 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
             k_nodes_chunks<<<(unsigned)((a.n_nodes + 1 + T - 1) / T), T, 0, stream>>>(p);
         }
         if (n) {
-            TimedLaunch tl("mat_allocs", stream);
-            k_allocs<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
-        }
-        {
-            TimedLaunch tl("mat_scan", stream);
-            k_scan<<<1, 1024, 0, stream>>>(p);
-        }
-        if (n) {
+            {
+                TimedLaunch tl("mat_allocs", stream);
+                k_allocs<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
+            }
             {
                 TimedLaunch tl("mat_scatter", stream);
                 k_scatter<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
             }
+            const unsigned tiles = (unsigned)max_tiles;
             {
                 TimedLaunch tl("mat_sort_tile", stream);
-                k_sort_tile<<<(unsigned)((n + kSortTile - 1) / kSortTile), 256, 0, stream>>>(p);
+                k_sort_tile<<<tiles, 256, 0, stream>>>(p);
             }
-            int pass = 0;
-            for (uint64_t width = kSortTile; width < n; width *= 2, ++pass) {
-                TimedLaunch tl("mat_merge", stream);
-                k_merge<<<(unsigned)((n + kMergeTile - 1) / kMergeTile), 256, 0, stream>>>(p, (uint32_t)width, pass);
+            if (!merge_mode) {
+                TimedLaunch tl("mat_rank", stream);
+                const uint64_t pairs = n * max_tiles;
+                const unsigned grid = (unsigned)std::min<uint64_t>((pairs + T - 1) / T, (uint64_t)s.sm_count * 8);
+                k_rank<<<grid, T, 0, stream>>>(p);
+            } else {
+                int pass = 0;
+                for (uint64_t width = kSortTile; width < n; width *= 2, ++pass) {
+                    TimedLaunch tl("mat_merge", stream);
+                    k_merge<<<(unsigned)((n + kMergeTile - 1) / kMergeTile), 256, 0, stream>>>(p, (uint32_t)width, pass);
+                }
             }
             {
-                TimedLaunch tl("mat_build_i", stream);
-                k_build_i<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
+                TimedLaunch tl("mat_finalize_i", stream);
+                k_finalize_i<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
             }
             TimedLaunch tl("mat_check", stream);
-            k_check<<<(nb + 3) / 4, kChkThreads, 0, stream>>>(p);
+            k_check<<<(nb + 7) / 8, 256, 0, stream>>>(p);
         }
         if (C) {
             {
