@@ -13,30 +13,32 @@
 //  * M = every other allocation ("mortal": capture temporaries, warm-up and
 //    profiling scratch).  A mortal is registered in exactly the word chunks that
 //    hold words of nodes launched during its lifetime; a chunk's window (~60
-//    entries for the ten-model set) is sorted by base in shared memory and
-//    searched with a prefix-max-of-end backward walk plus the time check.
+//    entries for the ten-model set) is sorted by (base, t_alloc) in registers of
+//    one warp, laid out in shared memory and searched with an upper bound on
+//    (word, launch position), a backward walk while the prefix max of end still
+//    reaches the word, and the time check.
 //  * Well-formedness (no two simultaneously-live allocations overlap) is checked
 //    exactly: I-I by adjacency of the sorted list, M-I with per-32-entry
 //    min(t_alloc) / max(t_free) summaries over the address run a mortal meets,
 //    M-M inside blocks of 32 allocation ordinals against the mortals registered
 //    as live there.
-// Pipeline (all on `stream`; one host synchronization at the end):
-//   k_nodes_chunks  CSR / launch-order checks; per-chunk first/last node; node fences
-//   k_allocs        trace checks, I/M split, registration ranges + counts; the
-//                   last CTA scans the counts into offsets
-//   k_scatter       registration lists (32-byte window records)
-//   k_sort_tile     I keys sorted in tiles of 2048 (register bitonic per warp +
-//                   shared-memory merges)
-//   k_rank          global rank of every key = sum over the other tiles of a
-//                   binary-search count; the last contribution scatters the key
-//   k_finalize_i    I arrays, I-I check, shared-memory fences, block summaries
-//   k_check         M-M and M-I overlap checks
-//   k_classify      one CTA per 2048-word chunk: TMA bulk copy of the chunk's words
-//                   to shared memory, candidate compaction, window search, I-list
-//                   search, mask words + warp-dense staging of the records + the
-//                   chunk's slot count; the last CTA scans counts -> chunk_base
+// Pipeline: five launches on `stream`, one host synchronization at the end.  Role
+// split by blockIdx where two independent phases share a launch:
+//   k_trace         [nodes] CSR / launch-order checks, first/last node per chunk
+//                   [allocs] trace checks, I/M split, registration ranges and
+//                   counts; the last alloc CTA scans the counts into offsets
+//   k_prepare       [sort] I keys sorted in tiles of 2048 (register bitonic per
+//                   warp + shared-memory merges); [scatter] registration lists
+//   k_rank          global rank of every I key = its index in its tile + the count
+//                   below it in every other tile; the last contribution writes
+//                   the I arrays, the fences and the block summaries
+//   k_scan_words    [classify] one CTA per 2048-word chunk: TMA bulk copy of the
+//                   chunk's words to shared memory, candidate compaction, window
+//                   search, I-list search through a compacted queue, mask words,
+//                   warp-dense staging of the records, the chunk's slot count; the
+//                   last classify CTA scans counts -> chunk_base
+//                   [check] M-M, M-I and I-I overlap checks
 //   k_emit          compaction of the staged records into the slot table
-// (k_merge passes replace k_rank when the trace has more than 64 tiles of I keys.)
 #include <algorithm>
 #include <mutex>
 #include <vector>
@@ -47,17 +49,14 @@ namespace medusa {
 namespace {
 
 constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
+constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
-constexpr int kSortTile = 2048;    // keys sorted per CTA before ranking / merging
-constexpr int kMergeTile = 2048;   // outputs per CTA of a merge pass
-constexpr int kRankMaxTiles = 64;  // above this many tiles, merge passes instead of ranks
+constexpr int kSortTile = 2048;    // keys sorted per CTA before ranking
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
-constexpr int kNodeFenceCap = 4096;
-constexpr int kWinCap = 128;       // mortal-window entries per batch (4 per lane of one warp)
-constexpr int kClsThreads = 256;
-constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kClsThreads;  // 8
-constexpr int kWarps = kClsThreads / 32;
+constexpr int kWinCap = 128;       // mortal-window entries per batch (<= 4 per lane of one warp)
+constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
+constexpr int kWarps = kThreads / 32;
 constexpr int kIBlk = 32;          // I-list summary block
 
 struct Ctl {
@@ -89,19 +88,18 @@ struct WinRec {  // a registered mortal allocation
 struct Dev {  // scratch of one call (device pointers)
     Ctl* ctl;
     uint32_t *jf, *jl;                           // [C] first / last node of each chunk
-    uint32_t* node_fence;                        // [kNodeFenceCap] node_t every nstride nodes
     uint4* rng;                                  // [n]: c_lo, c_hi, b_lo, b_hi
     uint32_t *cnt_c, *fill_c, *off_c;            // [C+1] (zeroed)
     uint32_t *cnt_b, *fill_b, *off_b;            // [nb+1] (zeroed)
+    uint32_t *blk_min_ta_c, *blk_max_tf;         // [n/32+1] (zeroed; min kept as ~max(~t))
     WinRec *list_c, *list_b;
     uint64_t cap_c, cap_b;
-    uint64_t* sk[2];                             // [n] sort keys
-    uint32_t* sv[2];                             // [n] sort values
+    uint64_t* sk[2];                             // [n] sort keys: 0 unsorted, 1 sorted tiles
+    uint32_t* sv[2];                             // [n] sort values (allocation index)
     unsigned long long* rank;                    // [n] (contributions << 32) | rank
     uint64_t* i_base;                            // [n]
     IRest* i_rest;                               // [n]
     uint32_t* i_tf;                              // [n]
-    uint32_t *blk_min_ta, *blk_max_tf;           // [n/32]
     uint64_t* fence;                             // [kFenceCap]
     uint32_t* chunk_cnt;                         // [C]
     uint64_t* staging;                           // [n_words] records, warp-dense per 32 words
@@ -110,8 +108,10 @@ struct Dev {  // scratch of one call (device pointers)
 struct P {  // kernel parameters
     MaterializeArgs a;
     Dev d;
-    uint32_t C, nb, nstride;  // chunks, check blocks, node-fence stride
-    int merge_mode;           // 1: I keys merged by passes (very large traces)
+    uint32_t C, nb;              // chunks, check blocks
+    uint32_t node_ctas;          // k_trace: CTAs with the node role
+    uint32_t sort_ctas;          // k_prepare: CTAs with the sort role
+    uint32_t check_ctas;         // k_scan_words: CTAs with the check role (after the C classify CTAs)
 };
 
 __device__ __forceinline__ void flag(Ctl* c, unsigned int bit) { atomicOr(&c->status, bit); }
@@ -132,17 +132,7 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
 }
 
 __device__ __forceinline__ uint32_t n_tiles(uint32_t nI) { return (nI + kSortTile - 1) / kSortTile; }
-// number of merge passes that do work for nI keys (merge mode; tiles are in buffer 1)
-__device__ __forceinline__ int merge_passes(uint32_t nI) {
-    int e = 0;
-    for (uint64_t w = kSortTile; w < nI; w *= 2) ++e;
-    return e;
-}
-// buffer holding the fully sorted I keys
-__device__ __forceinline__ int final_buffer(const P& p, uint32_t nI) {
-    if (p.merge_mode) return (1 + merge_passes(nI)) & 1;
-    return n_tiles(nI) > 1 ? 0 : 1;
-}
+__device__ __forceinline__ uint32_t fence_stride(uint32_t nI) { return nI ? (nI + kFenceCap - 1) / kFenceCap : 1; }
 
 // Exclusive scan of cnt[0..n) into off[0..n] (off[n] = total) by one CTA of any
 // size <= 1024 (multiple of 32); reads through L2 (values written by other CTAs).
@@ -177,36 +167,6 @@ __device__ void block_exclusive_scan(const uint32_t* cnt, uint32_t* off, uint32_
     __syncthreads();
 }
 
-// ----------------------------------------------------------------------------
-// 1. nodes and chunks: CSR / order checks; node j writes the chunks whose first
-//    or last word it holds (no search) and, every nstride nodes, a node fence
-__global__ void k_nodes_chunks(P p) {
-    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const MaterializeArgs& a = p.a;
-    const uint32_t N = a.n_nodes;
-    if (i > N) return;
-    const uint64_t o0 = a.node_off[i];
-    if (i == 0 && o0 != 0) flag(p.d.ctl, ST_INVALID);
-    if (i == N) {
-        if (o0 != a.n_words) flag(p.d.ctl, ST_INVALID);
-        return;
-    }
-    const uint64_t o1 = a.node_off[i + 1];
-    const uint32_t t = a.node_t[i];
-    if (i % p.nstride == 0) p.d.node_fence[i / p.nstride] = t;
-    if (o1 < o0) { flag(p.d.ctl, ST_INVALID); return; }
-    if (i + 1 < N && !(t < a.node_t[i + 1])) flag(p.d.ctl, ST_INVALID);
-    if (o1 == o0 || o1 > a.n_words) return;
-    for (uint64_t c = o0 / kChunkWords; c <= (o1 - 1) / kChunkWords; ++c) {
-        const uint64_t cs = c * kChunkWords;
-        const uint64_t ce = min(cs + kChunkWords, a.n_words) - 1;
-        if (o0 <= cs) p.d.jf[c] = (uint32_t)i;
-        if (ce < o1) p.d.jl[c] = (uint32_t)i;
-    }
-}
-
-// ----------------------------------------------------------------------------
-// 2. allocations: checks, I/M split, registration ranges and counts
 // first index k in [lo, n) with t[k] >= x (galloping from lo; t ascending)
 __device__ __forceinline__ uint32_t gallop_ge(const uint32_t* t, uint32_t lo, uint32_t n, uint32_t x) {
     uint32_t step = 1, prev = lo, hi = lo;
@@ -225,16 +185,37 @@ __device__ __forceinline__ uint32_t gallop_alloc_ge(const medusa_alloc* al, uint
     return l;
 }
 
-__global__ void __launch_bounds__(256) k_allocs(P p) {
-    __shared__ uint32_t s_nf[kNodeFenceCap];
+// ----------------------------------------------------------------------------
+// 1. k_trace
+__device__ void nodes_role(const P& p, uint64_t i) {
+    const MaterializeArgs& a = p.a;
+    const uint32_t N = a.n_nodes;
+    if (i > N) return;
+    const uint64_t o0 = a.node_off[i];
+    if (i == 0 && o0 != 0) flag(p.d.ctl, ST_INVALID);
+    if (i == N) {
+        if (o0 != a.n_words) flag(p.d.ctl, ST_INVALID);
+        return;
+    }
+    const uint64_t o1 = a.node_off[i + 1];
+    if (o1 < o0) { flag(p.d.ctl, ST_INVALID); return; }
+    if (i + 1 < N && !(a.node_t[i] < a.node_t[i + 1])) flag(p.d.ctl, ST_INVALID);
+    if (o1 == o0 || o1 > a.n_words) return;
+    // node i writes the chunks whose first or last word it holds
+    for (uint64_t c = o0 / kChunkWords; c <= (o1 - 1) / kChunkWords; ++c) {
+        const uint64_t cs = c * kChunkWords;
+        const uint64_t ce = min(cs + kChunkWords, a.n_words) - 1;
+        if (o0 <= cs) p.d.jf[c] = (uint32_t)i;
+        if (ce < o1) p.d.jl[c] = (uint32_t)i;
+    }
+}
+
+__device__ void allocs_role(const P& p, uint32_t cta) {
     __shared__ uint32_t s_last;
-    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    const uint32_t i = cta * blockDim.x + threadIdx.x;
     const MaterializeArgs& a = p.a;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t N = a.n_nodes;
-    const uint32_t nnf = (N + p.nstride - 1) / p.nstride;
-    for (uint32_t f = threadIdx.x; f < nnf; f += blockDim.x) s_nf[f] = p.d.node_fence[f];
-    __syncthreads();
     const bool valid = i < a.n_alloc;
     medusa_alloc x{};
     if (valid) x = a.alloc[i];
@@ -250,14 +231,9 @@ __global__ void __launch_bounds__(256) k_allocs(P p) {
             if (!isI) {
                 if (p.C && N && x.t_alloc < x.t_free) {
                     // nodes launched while i is live: [j0, j1) = t in (t_alloc, t_free)
-                    uint32_t lo = 0, hi = nnf;  // fences <= t_alloc
-                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (s_nf[m] <= x.t_alloc) lo = m + 1; else hi = m; }
-                    uint32_t j0 = 0;
-                    if (lo > 0) {
-                        uint32_t l2 = (lo - 1) * p.nstride + 1, h2 = min(lo * p.nstride, N);
-                        while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (a.node_t[m] <= x.t_alloc) l2 = m + 1; else h2 = m; }
-                        j0 = l2;
-                    }
+                    uint32_t lo = 0, hi = N;
+                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.node_t[m] <= x.t_alloc) lo = m + 1; else hi = m; }
+                    const uint32_t j0 = lo;
                     const uint32_t j1 = gallop_ge(a.node_t, j0, N, x.t_free);
                     // chunks holding their words (exact: no entry for memory no launch can see)
                     if (j0 < j1) {
@@ -296,11 +272,12 @@ __global__ void __launch_bounds__(256) k_allocs(P p) {
         atomicMax(&p.d.ctl->gmin_c, ~(unsigned long long)mn);
         atomicMax(&p.d.ctl->gmax, (unsigned long long)mx);
     }
-    // the last CTA turns the registration counts into offsets
+    // the last alloc CTA turns the registration counts into offsets
     __syncthreads();
     if (threadIdx.x == 0) {
         __threadfence();
-        s_last = atomicAdd(&p.d.ctl->done_allocs, 1u) == gridDim.x - 1;
+        const uint32_t alloc_ctas = (a.n_alloc + blockDim.x - 1) / blockDim.x;
+        s_last = atomicAdd(&p.d.ctl->done_allocs, 1u) == alloc_ctas - 1;
     }
     __syncthreads();
     if (s_last) {
@@ -312,37 +289,19 @@ __global__ void __launch_bounds__(256) k_allocs(P p) {
     }
 }
 
-// 3. registration lists (32-byte records, so readers need no second gather)
-__global__ void k_scatter(P p) {
-    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= p.a.n_alloc) return;
-    const uint4 r = p.d.rng[i];
-    if (r.x > r.y && r.z > r.w) return;
-    const medusa_alloc x = p.a.alloc[i];
-    const WinRec w{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
-    for (uint32_t c = r.x; c <= r.y; ++c) {
-        const uint64_t pos = (uint64_t)p.d.off_c[c] + atomicAdd(&p.d.fill_c[c], 1u);
-        if (pos < p.d.cap_c) p.d.list_c[pos] = w;
-    }
-    for (uint32_t b = r.z; b <= r.w; ++b) {
-        const uint64_t pos = (uint64_t)p.d.off_b[b] + atomicAdd(&p.d.fill_b[b], 1u);
-        if (pos < p.d.cap_b) p.d.list_b[pos] = w;
-    }
+__global__ void __launch_bounds__(kThreads) k_trace(P p) {
+    if (blockIdx.x < p.node_ctas) nodes_role(p, (uint64_t)blockIdx.x * blockDim.x + threadIdx.x);
+    else allocs_role(p, blockIdx.x - p.node_ctas);
 }
 
 // ----------------------------------------------------------------------------
-// 4. sort I by (base, index)
-__device__ __forceinline__ void cas(uint64_t& ka, uint32_t& va, uint64_t& kb, uint32_t& vb, bool up) {
-    if (kv_less(kb, vb, ka, va) == up) {
-        const uint64_t tk = ka; ka = kb; kb = tk;
-        const uint32_t tv = va; va = vb; vb = tv;
-    }
-}
+// 2. k_prepare: sort tiles of I keys by (base, index) | registration lists
 
 // Bitonic sort of 32*E (key, val) pairs held E per lane (element e = lane*E + r),
-// ascending, by shuffles and register compare-exchanges (no shared memory).
+// ascending by (key, val), carrying a payload; shuffles and register
+// compare-exchanges only (no shared memory).
 template <int E>
-__device__ __forceinline__ void warp_bitonic(uint64_t (&k)[E], uint32_t (&v)[E]) {
+__device__ __forceinline__ void warp_bitonic(uint64_t (&k)[E], uint32_t (&v)[E], uint32_t (&pl)[E]) {
     const uint32_t lane = threadIdx.x & 31;
 #pragma unroll
     for (uint32_t size = 2; size <= 32u * E; size <<= 1) {
@@ -355,17 +314,22 @@ __device__ __forceinline__ void warp_bitonic(uint64_t (&k)[E], uint32_t (&v)[E])
                     const uint32_t e = lane * E + r;
                     const uint64_t ok = __shfl_xor_sync(0xffffffffu, k[r], lj);
                     const uint32_t ov = __shfl_xor_sync(0xffffffffu, v[r], lj);
+                    const uint32_t op = __shfl_xor_sync(0xffffffffu, pl[r], lj);
                     const bool up = (e & size) == 0;
                     const bool lower = (e & j) == 0;
                     const bool other_less = kv_less(ok, ov, k[r], v[r]);
                     // lower element keeps the min when ascending, the max when descending
-                    if ((lower == up) ? other_less : !other_less) { k[r] = ok; v[r] = ov; }
+                    if ((lower == up) ? other_less : !other_less) { k[r] = ok; v[r] = ov; pl[r] = op; }
                 }
             } else {
 #pragma unroll
                 for (int r = 0; r < E; ++r) {
                     const int r2 = r ^ (int)j;
-                    if (r2 > r) cas(k[r], v[r], k[r2], v[r2], ((lane * E + r) & size) == 0);
+                    if (r2 > r && kv_less(k[r2], v[r2], k[r], v[r]) == (((lane * E + r) & size) == 0)) {
+                        const uint64_t tk = k[r]; k[r] = k[r2]; k[r2] = tk;
+                        const uint32_t tv = v[r]; v[r] = v[r2]; v[r2] = tv;
+                        const uint32_t tp = pl[r]; pl[r] = pl[r2]; pl[r2] = tp;
+                    }
                 }
             }
         }
@@ -382,26 +346,42 @@ __device__ __forceinline__ uint32_t merge_path_smem(const uint64_t* ka, const ui
     return lo;
 }
 
-__global__ void __launch_bounds__(256) k_sort_tile(P p) {
-    __shared__ uint64_t sk[2][kSortTile];
-    __shared__ uint32_t sv[2][kSortTile];
+// the I entry of sorted position r: arrays, fence, block summaries
+__device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t nI, uint32_t id) {
+    const medusa_alloc x = p.a.alloc[id];
+    p.d.i_base[r] = x.base;
+    p.d.i_rest[r] = IRest{x.base + x.size, x.t_alloc, id};
+    p.d.i_tf[r] = x.t_free;
+    const uint32_t stride = fence_stride(nI);
+    if (r % stride == 0) p.d.fence[r / stride] = x.base;
+    atomicMax(&p.d.blk_min_ta_c[r / kIBlk], ~x.t_alloc);
+    atomicMax(&p.d.blk_max_tf[r / kIBlk], x.t_free);
+}
+
+struct SortShared {
+    uint64_t sk[2][kSortTile];
+    uint32_t sv[2][kSortTile];
+};
+
+__device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
     const uint32_t n = p.d.ctl->nI;
-    const uint32_t t0 = blockIdx.x * kSortTile;
+    const uint32_t t0 = tile * kSortTile;
     if (t0 >= n) return;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     uint64_t k[8];
-    uint32_t v[8];
+    uint32_t v[8], pl[8];
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
         const uint32_t g = t0 + warp * 256 + lane * 8 + r;
         k[r] = g < n ? p.d.sk[0][g] : ~0ull;
         v[r] = g < n ? p.d.sv[0][g] : 0xFFFFFFFFu;
+        pl[r] = 0;
     }
-    warp_bitonic<8>(k, v);
+    warp_bitonic<8>(k, v, pl);
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
-        sk[0][warp * 256 + lane * 8 + r] = k[r];
-        sv[0][warp * 256 + lane * 8 + r] = v[r];
+        S.sk[0][warp * 256 + lane * 8 + r] = k[r];
+        S.sv[0][warp * 256 + lane * 8 + r] = v[r];
     }
     __syncthreads();
     int src = 0;
@@ -410,32 +390,60 @@ __global__ void __launch_bounds__(256) k_sort_tile(P p) {
         const uint32_t o = tid * 8;
         const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
         const uint32_t d = o - a0;
-        const uint64_t* ka = sk[src] + a0;
-        const uint32_t* va = sv[src] + a0;
-        const uint64_t* kb = sk[src] + b0;
-        const uint32_t* vb = sv[src] + b0;
+        const uint64_t* ka = S.sk[src] + a0;
+        const uint32_t* va = S.sv[src] + a0;
+        const uint64_t* kb = S.sk[src] + b0;
+        const uint32_t* vb = S.sv[src] + b0;
         uint32_t ia = merge_path_smem(ka, va, kb, vb, d, d > run ? d - run : 0, min(d, run));
         uint32_t ib = d - ia;
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
             const bool takeA = ib >= run || (ia < run && kv_less(ka[ia], va[ia], kb[ib], vb[ib]));
-            sk[src ^ 1][o + q] = takeA ? ka[ia] : kb[ib];
-            sv[src ^ 1][o + q] = takeA ? va[ia] : vb[ib];
+            S.sk[src ^ 1][o + q] = takeA ? ka[ia] : kb[ib];
+            S.sv[src ^ 1][o + q] = takeA ? va[ia] : vb[ib];
             if (takeA) ++ia; else ++ib;
         }
         src ^= 1;
         __syncthreads();
     }
+    const bool single = n <= kSortTile;  // one tile: its order is final
     for (uint32_t q = tid; q < kSortTile && t0 + q < n; q += blockDim.x) {
-        p.d.sk[1][t0 + q] = sk[src][q];
-        p.d.sv[1][t0 + q] = sv[src][q];
-        p.d.rank[t0 + q] = q;  // rank within the tile, no contribution yet
+        if (single) {
+            write_i_entry(p, q, n, S.sv[src][q]);
+        } else {
+            p.d.sk[1][t0 + q] = S.sk[src][q];
+            p.d.sv[1][t0 + q] = S.sv[src][q];
+            p.d.rank[t0 + q] = q;  // rank within the tile, no contribution yet
+        }
     }
 }
 
-// global rank = own tile index + sum over every other tile of #keys below; the
-// thread adding the last contribution scatters the key to its final position
-__global__ void __launch_bounds__(256) k_rank(P p) {
+__device__ void scatter_role(const P& p, uint32_t i) {
+    if (i >= p.a.n_alloc) return;
+    const uint4 r = p.d.rng[i];
+    if (r.x > r.y && r.z > r.w) return;
+    const medusa_alloc x = p.a.alloc[i];
+    const WinRec w{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
+    for (uint32_t c = r.x; c <= r.y; ++c) {
+        const uint64_t pos = (uint64_t)p.d.off_c[c] + atomicAdd(&p.d.fill_c[c], 1u);
+        if (pos < p.d.cap_c) p.d.list_c[pos] = w;
+    }
+    for (uint32_t b = r.z; b <= r.w; ++b) {
+        const uint64_t pos = (uint64_t)p.d.off_b[b] + atomicAdd(&p.d.fill_b[b], 1u);
+        if (pos < p.d.cap_b) p.d.list_b[pos] = w;
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) k_prepare(P p) {
+    __shared__ SortShared S;
+    if (blockIdx.x < p.sort_ctas) sort_role(p, blockIdx.x, S);
+    else scatter_role(p, (blockIdx.x - p.sort_ctas) * blockDim.x + threadIdx.x);
+}
+
+// ----------------------------------------------------------------------------
+// 3. k_rank: rank = index in own tile + count of keys below it in every other
+//    tile; the thread adding the last contribution writes the entry in place
+__global__ void __launch_bounds__(kThreads) k_rank(P p) {
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t T = n_tiles(nI);
     if (T <= 1) return;
@@ -452,117 +460,7 @@ __global__ void __launch_bounds__(256) k_rank(P p) {
         while (lo < hi) { const uint32_t m = (lo + hi) >> 1; if (kv_less(sk[m], sv[m], kk, vk)) lo = m + 1; else hi = m; }
         const uint32_t cnt = lo - base;
         const unsigned long long old = atomicAdd(&p.d.rank[k], (1ull << 32) | cnt);
-        if ((old >> 32) + 1 == T - 1) {
-            const uint32_t r = (uint32_t)old + cnt;
-            p.d.sk[0][r] = kk;
-            p.d.sv[0][r] = vk;
-        }
-    }
-}
-
-// smallest i in [lo, hi) with less(B[d-1-i], A[i]), else hi -- warp-cooperative
-// 32-ary search (all lanes return the same value)
-__device__ uint32_t merge_path_warp(const uint64_t* ka, const uint32_t* va, const uint64_t* kb, const uint32_t* vb,
-                                    uint32_t d, uint32_t lo, uint32_t hi) {
-    const uint32_t lane = threadIdx.x & 31;
-    while (lo < hi) {
-        const uint32_t span = hi - lo;
-        const uint32_t step = (span + 31) / 32;
-        const uint32_t pi = lo + lane * step;
-        bool pr = false;
-        if (pi < hi) pr = kv_less(kb[d - 1 - pi], vb[d - 1 - pi], ka[pi], va[pi]);
-        const uint32_t b = __ballot_sync(0xffffffffu, pr);
-        if (step == 1) return b ? lo + (__ffs(b) - 1) : hi;
-        if (b == 0) {  // answer lies after the last probe that was inside [lo, hi)
-            lo = lo + min(31u, (span - 1) / step) * step + 1;
-        } else {
-            const uint32_t f = __ffs(b) - 1;
-            const uint32_t nhi = lo + f * step;
-            if (f == 0) return lo;
-            lo = lo + (f - 1) * step + 1;
-            hi = nhi;
-        }
-    }
-    return lo;
-}
-
-__global__ void __launch_bounds__(256) k_merge(P p, uint32_t width, int pass) {
-    __shared__ uint64_t sk[kMergeTile];
-    __shared__ uint32_t sv[kMergeTile];
-    __shared__ uint32_t s_i0, s_i1;
-    const uint32_t n = p.d.ctl->nI;
-    if (width >= n) return;  // one run already: nothing to merge (no-op pass)
-    const int in = (1 + pass) & 1;
-    const uint64_t* kin = p.d.sk[in];
-    const uint32_t* vin = p.d.sv[in];
-    uint64_t* kout = p.d.sk[in ^ 1];
-    uint32_t* vout = p.d.sv[in ^ 1];
-    const uint32_t o0 = blockIdx.x * kMergeTile;
-    if (o0 >= n) return;
-    const uint32_t ps = o0 / (2 * width) * (2 * width);
-    const uint32_t a0 = ps, a1 = min(ps + width, n), b0 = a1, b1 = min(ps + 2 * width, n);
-    const uint32_t o1 = min(o0 + kMergeTile, n);
-    if (a1 >= b1) {  // lone run: copy
-        for (uint32_t q = o0 + threadIdx.x; q < o1; q += blockDim.x) { kout[q] = kin[q]; vout[q] = vin[q]; }
-        return;
-    }
-    const uint32_t la = a1 - a0, lb = b1 - b0;
-    const uint32_t warp = threadIdx.x >> 5;
-    if (warp < 2) {
-        const uint32_t d = (warp == 0 ? o0 : o1) - ps;
-        const uint32_t r = merge_path_warp(kin + a0, vin + a0, kin + b0, vin + b0, d, d > lb ? d - lb : 0, min(d, la));
-        if ((threadIdx.x & 31) == 0) { if (warp == 0) s_i0 = r; else s_i1 = r; }
-    }
-    __syncthreads();
-    const uint32_t i0 = s_i0, i1 = s_i1;
-    const uint32_t j0 = (o0 - ps) - i0, j1 = (o1 - ps) - i1;
-    const uint32_t na = i1 - i0, nbb = j1 - j0;
-    for (uint32_t q = threadIdx.x; q < na + nbb; q += blockDim.x) {
-        const uint32_t src = q < na ? a0 + i0 + q : b0 + j0 + (q - na);
-        sk[q] = kin[src];
-        sv[q] = vin[src];
-    }
-    __syncthreads();
-    const uint32_t per = kMergeTile / 256;
-    const uint32_t d = threadIdx.x * per;
-    if (d < na + nbb) {
-        uint32_t ia = merge_path_smem(sk, sv, sk + na, sv + na, d, d > nbb ? d - nbb : 0, min(d, na));
-        uint32_t ib = d - ia;
-        for (uint32_t q = 0; q < per && d + q < na + nbb; ++q) {
-            const bool takeA = ib >= nbb || (ia < na && kv_less(sk[ia], sv[ia], sk[na + ib], sv[na + ib]));
-            const uint32_t s = takeA ? ia++ : na + ib++;
-            kout[o0 + d + q] = sk[s];
-            vout[o0 + d + q] = sv[s];
-        }
-    }
-}
-
-// 5. I arrays, I-I adjacency check, shared-memory fences, 32-entry summaries
-__global__ void __launch_bounds__(256) k_finalize_i(P p) {
-    const uint32_t k = blockIdx.x * blockDim.x + threadIdx.x;
-    const uint32_t nI = p.d.ctl->nI;
-    if (k - (threadIdx.x & 31) >= nI) return;  // whole warp past the end
-    const int fin = final_buffer(p, nI);
-    const uint64_t* sk = p.d.sk[fin];
-    const uint32_t* sv = p.d.sv[fin];
-    uint32_t ta = 0xFFFFFFFFu, tf = 0;
-    if (k < nI) {
-        const uint32_t id = sv[k];
-        const medusa_alloc x = p.a.alloc[id];
-        p.d.i_base[k] = x.base;
-        p.d.i_rest[k] = IRest{x.base + x.size, x.t_alloc, id};
-        p.d.i_tf[k] = x.t_free;
-        ta = x.t_alloc;
-        tf = x.t_free;
-        if (k + 1 < nI && x.base + x.size > sk[k + 1]) flag(p.d.ctl, ST_TRACE);
-        const uint32_t stride = (nI + kFenceCap - 1) / kFenceCap;
-        if (k % stride == 0) p.d.fence[k / stride] = x.base;
-    }
-    const uint32_t mn = __reduce_min_sync(0xffffffffu, ta);
-    const uint32_t mx = __reduce_max_sync(0xffffffffu, tf);
-    if ((threadIdx.x & 31) == 0) {
-        p.d.blk_min_ta[k / kIBlk] = mn;
-        p.d.blk_max_tf[k / kIBlk] = mx;
+        if ((old >> 32) + 1 == T - 1) write_i_entry(p, (uint32_t)old + cnt, nI, vk);
     }
 }
 
@@ -587,112 +485,58 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 }
 
 // ----------------------------------------------------------------------------
-// 6. overlap checks for mortal allocations: one warp per block of 32 ordinals
-__global__ void __launch_bounds__(256) k_check(P p) {
-    __shared__ uint64_t s_fence[kFenceCap];
-    __shared__ uint64_t s_base[8][kChkCap], s_end[8][kChkCap];
-    __shared__ uint32_t s_tf[8][kChkCap], s_idx[8][kChkCap];
-    const MaterializeArgs& a = p.a;
-    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t b = blockIdx.x * 8 + warp;
-    const uint32_t j = b * kAblk + lane;
-    const uint32_t nI = p.d.ctl->nI;
-    const uint32_t stride = nI ? (nI + kFenceCap - 1) / kFenceCap : 1;
-    const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = p.d.fence[f];
-    __syncthreads();
-    if (b >= p.nb) return;  // whole warp
-    bool mine = false;
-    medusa_alloc x{};
-    const uint32_t N = a.n_nodes;
-    const uint32_t t_last = N ? a.node_t[N - 1] : 0;
-    if (j < a.n_alloc) {
-        x = a.alloc[j];
-        mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
-    }
-    const uint64_t xe = x.base + x.size;
-    bool bad = false;
-    // M-M: mortals registered as live at some allocation of this block
-    const uint64_t r0 = p.d.off_b[b];
-    const uint64_t r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
-    for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
-        const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
-        __syncwarp();
-        for (uint32_t q = lane; q < m; q += 32) {
-            const WinRec y = p.d.list_b[bs + q];
-            s_base[warp][q] = y.base;
-            s_end[warp][q] = y.end;
-            s_tf[warp][q] = y.t_free;
-            s_idx[warp][q] = y.id;
-        }
-        __syncwarp();
-        if (mine && !bad) {
-            for (uint32_t q = 0; q < m; ++q) {
-                if (s_idx[warp][q] < j && s_tf[warp][q] > x.t_alloc && s_base[warp][q] < xe && x.base < s_end[warp][q]) {
-                    bad = true;
-                    break;
-                }
-            }
-        }
-    }
-    // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
-    if (mine && !bad && nI) {
-        const uint32_t e = i_count_le(s_fence, nf, stride, nI, p.d.i_base, xe - 1);  // bases < end
-        const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);
-        const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
-        // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
-        const bool freed_early = x.t_free <= t_last;
-        uint32_t k = s;
-        for (; k < e && (k % kIBlk) != 0; ++k)
-            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
-        for (; k + kIBlk <= e; k += kIBlk)
-            bad |= freed_early ? p.d.blk_min_ta[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
-        for (; k < e; ++k)
-            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
-    }
-    if (bad) flag(p.d.ctl, ST_TRACE);
-}
-
-// ----------------------------------------------------------------------------
-// 7. classify one chunk per CTA
+// 4. k_scan_words: classify CTAs (one per chunk) and check CTAs
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     uint64_t fence[kFenceCap];
     uint32_t tw[MEDUSA_CHUNK_WORDS];     // launch position of every word
-    uint64_t wb[kWinCap], we[kWinCap], wpmax[kWinCap];  // window, physically sorted by base
+    uint64_t wb[kWinCap], we[kWinCap], wpmax[kWinCap];  // window sorted by (base, t_alloc)
     uint32_t wta[kWinCap], wtf[kWinCap], wid[kWinCap];
-    uint16_t cq[MEDUSA_CHUNK_WORDS];     // candidate words (could point into memory)
+    uint16_t cq[MEDUSA_CHUNK_WORDS];     // candidate words, then the I-list queue
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32];
     uint32_t wmax[kWarps];
-    uint32_t nc, total, last;
+    uint32_t nc, nq, total, last;
     unsigned long long mbar;
+};
+
+struct ChkShared {
+    uint64_t fence[kFenceCap];
+    uint64_t base[kWarps][kChkCap], end[kWarps][kChkCap];
+    uint32_t tf[kWarps][kChkCap], idx[kWarps][kChkCap];
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-// warp 0: load a batch of <= kWinCap registered mortals, sort by base, lay them out
-// physically sorted, prefix max of end
-__device__ __forceinline__ void window_prepare(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
+// warp 0: a batch of <= kWinCap registered mortals sorted by (base, t_alloc) in
+// registers, laid out in shared memory, with the prefix max of end
+template <int E>
+__device__ __forceinline__ void window_prepare_e(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
     const uint32_t lane = threadIdx.x & 31;
-    constexpr int E = kWinCap / 32;
     uint64_t k[E];
-    uint32_t v[E];
+    uint32_t v[E], pl[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
         const uint32_t e = lane * E + r;
-        k[r] = e < m ? p.d.list_c[bs + e].base : ~0ull;
-        v[r] = e;
+        if (e < m) {
+            const WinRec& x = p.d.list_c[bs + e];
+            k[r] = x.base;
+            v[r] = x.t_alloc;
+        } else {
+            k[r] = ~0ull;
+            v[r] = 0xFFFFFFFFu;
+        }
+        pl[r] = e;
     }
-    warp_bitonic<E>(k, v);
+    warp_bitonic<E>(k, v, pl);
     uint64_t ends[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
         const uint32_t e = lane * E + r;
         ends[r] = 0;
         if (e < m) {
-            const WinRec x = p.d.list_c[bs + v[r]];
+            const WinRec x = p.d.list_c[bs + pl[r]];
             S.wb[e] = x.base;
             S.we[e] = x.end;
             S.wta[e] = x.t_alloc;
@@ -719,12 +563,15 @@ __device__ __forceinline__ void window_prepare(const P& p, ClsShared& S, uint64_
     }
 }
 
-__global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    ClsShared& S = *reinterpret_cast<ClsShared*>(smem_raw);
+__device__ __forceinline__ void window_prepare(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
+    if (m <= 32) window_prepare_e<1>(p, S, bs, m);
+    else if (m <= 64) window_prepare_e<2>(p, S, bs, m);
+    else window_prepare_e<4>(p, S, bs, m);
+}
+
+__device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t c = blockIdx.x;
     Ctl* ctl = p.d.ctl;
     const uint64_t cs = (uint64_t)c * kChunkWords;
     const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
@@ -733,6 +580,7 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     // A. the chunk's words -> shared memory with one bulk copy (TMA engine)
     if (tid == 0) {
         S.nc = 0;
+        S.nq = 0;
         S.total = 0;
         if (tma) {
             const uint32_t mb = smem_u32(&S.mbar);
@@ -744,14 +592,14 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
         }
     }
     if (!tma)
-        for (uint32_t q = tid; q < n; q += kClsThreads) S.words[q] = ld_stream(gsrc + q);
+        for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
     const uint32_t nI = ctl->nI;
-    const uint32_t stride = nI ? (nI + kFenceCap - 1) / kFenceCap : 1;
+    const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = tid; f < nf; f += kClsThreads) S.fence[f] = p.d.fence[f];
+    for (uint32_t f = tid; f < nf; f += kThreads) S.fence[f] = p.d.fence[f];
     const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
     const uint32_t N = a.n_nodes;
-    for (uint32_t q = tid; q < kChunkWords; q += kClsThreads) S.tw[q] = 0;
+    for (uint32_t q = tid; q < kChunkWords; q += kThreads) S.tw[q] = 0;
     if (tid < MEDUSA_CHUNK_WORDS / 32) S.hits[tid] = 0;
     const uint64_t r0 = p.d.off_c[c];
     const uint64_t r1 = min((uint64_t)p.d.off_c[c + 1], p.d.cap_c);
@@ -762,7 +610,7 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     } else if (N) {
         const uint32_t jf = min(p.d.jf[c], N - 1), jl = min(p.d.jl[c], N - 1);
         if (tid == 32) atomicMax(&S.tw[0], a.node_t[jf]);
-        for (uint32_t j = jf + 1 + (tid - 32); j <= jl; j += kClsThreads - 32) {
+        for (uint32_t j = jf + 1 + (tid - 32); j <= jl; j += kThreads - 32) {
             const uint64_t q = a.node_off[j] - cs;
             if (q < n) atomicMax(&S.tw[q], a.node_t[j]);
         }
@@ -798,7 +646,7 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     // C. candidates: words inside [least base, greatest end) of the trace
 #pragma unroll
     for (int k = 0; k < kWordsPerThread; ++k) {
-        const uint32_t q = k * kClsThreads + tid;
+        const uint32_t q = k * kThreads + tid;
         bool cand = false;
         if (q < n) {
             const uint64_t x = S.words[q];
@@ -812,8 +660,8 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     }
     __syncthreads();
     const uint32_t nc = S.nc;
-    // D. mortal window(s): binary search by base, backward walk while the prefix
-    //    max of end still reaches the word, time check
+    // D. mortal window(s): upper bound of (word, launch position) over (base,
+    //    t_alloc), then walk back while the prefix max of end still reaches the word
     for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
         const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
         if (bs != r0) {
@@ -821,13 +669,13 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
             if (warp == 0) window_prepare(p, S, bs, m);
             __syncthreads();
         }
-        for (uint32_t i = tid; i < nc; i += kClsThreads) {
+        for (uint32_t i = tid; i < nc; i += kThreads) {
             const uint32_t q = S.cq[i];
             if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
             const uint64_t x = S.words[q];
             const uint32_t t = S.tw[q];
-            uint32_t lo = 0, hi = m;  // count of bases <= x
-            while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
+            uint32_t lo = 0, hi = m;  // count of entries (base, t_alloc) < (x, t)
+            while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (kv_less(S.wb[mid], S.wta[mid], x, t)) lo = mid + 1; else hi = mid; }
             for (int r = (int)lo - 1; r >= 0 && S.wpmax[r] > x; --r) {
                 if (x < S.we[r] && S.wta[r] < t && t < S.wtf[r]) {
                     S.words[q] = ((uint64_t)S.wid[r] << MEDUSA_OFF_BITS) | (x - S.wb[r]);
@@ -838,14 +686,36 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
         }
     }
     __syncthreads();
-    // E. I list: fences in shared memory, then one group of <= stride bases
+    // E. I list, for the candidates still unresolved, compacted into a queue first
     if (nI) {
         const uint64_t f0 = S.fence[0];
-        for (uint32_t i = tid; i < nc; i += kClsThreads) {
+        uint32_t qv[kWordsPerThread];
+        bool need[kWordsPerThread];
+#pragma unroll
+        for (int k = 0; k < kWordsPerThread; ++k) {
+            const uint32_t i = k * kThreads + tid;
+            need[k] = false;
+            qv[k] = 0;
+            if (i < nc) {
+                const uint32_t q = S.cq[i];
+                qv[k] = q;
+                need[k] = !((S.hits[q >> 5] >> (q & 31)) & 1u) && S.words[q] >= f0;
+            }
+        }
+        __syncthreads();  // cq is rewritten below
+#pragma unroll
+        for (int k = 0; k < kWordsPerThread; ++k) {
+            const uint32_t bal = __ballot_sync(0xffffffffu, need[k]);
+            uint32_t base = 0;
+            if (lane == 0 && bal) base = atomicAdd(&S.nq, (uint32_t)__popc(bal));
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (need[k]) S.cq[base + __popc(bal & lanemask_lt())] = (uint16_t)qv[k];
+        }
+        __syncthreads();
+        const uint32_t nq = S.nq;
+        for (uint32_t i = tid; i < nq; i += kThreads) {
             const uint32_t q = S.cq[i];
-            if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
             const uint64_t x = S.words[q];
-            if (x < f0) continue;
             const uint32_t t = S.tw[q];
             const uint32_t kk = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x) - 1;
             const uint64_t base = p.d.i_base[kk];
@@ -862,7 +732,7 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     uint32_t cnt = 0;
 #pragma unroll
     for (int k = 0; k < kWordsPerThread; ++k) {
-        const uint32_t q = k * kClsThreads + tid;
+        const uint32_t q = k * kThreads + tid;
         const uint32_t bits = S.hits[q >> 5];
         const uint64_t mw = (cs + q) >> 5;
         if (lane == 0 && mw < n_mask) a.mask[mw] = bits;
@@ -871,11 +741,11 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     }
     if (lane == 0) atomicAdd(&S.total, cnt);
     __syncthreads();
-    // G. the last CTA turns the chunk counts into chunk_base
+    // G. the last classify CTA turns the chunk counts into chunk_base
     if (tid == 0) {
         p.d.chunk_cnt[c] = S.total;
         __threadfence();
-        S.last = atomicAdd(&ctl->done_cls, 1u) == gridDim.x - 1;
+        S.last = atomicAdd(&ctl->done_cls, 1u) == p.C - 1;
     }
     __syncthreads();
     if (S.last) {
@@ -884,8 +754,83 @@ __global__ void __launch_bounds__(kClsThreads) k_classify(P p) {
     }
 }
 
-// 8. compaction of the staged records into the slot table (one CTA per chunk)
-__global__ void __launch_bounds__(256) k_emit(P p) {
+// one warp per block of 32 allocation ordinals; the CTA also checks 256 adjacent
+// pairs of the sorted I list
+__device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
+    const MaterializeArgs& a = p.a;
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t nI = p.d.ctl->nI;
+    {  // I-I: sorted neighbours must not overlap (all of I is live at the last launch)
+        const uint32_t k = cta * blockDim.x + threadIdx.x;
+        if (k + 1 < nI && p.d.i_rest[k].end > p.d.i_base[k + 1]) flag(p.d.ctl, ST_TRACE);
+    }
+    const uint32_t stride = fence_stride(nI);
+    const uint32_t nf = (nI + stride - 1) / stride;
+    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) S.fence[f] = p.d.fence[f];
+    __syncthreads();
+    const uint32_t b = cta * kWarps + warp;
+    if (b >= p.nb) return;  // whole warp
+    const uint32_t j = b * kAblk + lane;
+    bool mine = false;
+    medusa_alloc x{};
+    const uint32_t N = a.n_nodes;
+    const uint32_t t_last = N ? a.node_t[N - 1] : 0;
+    if (j < a.n_alloc) {
+        x = a.alloc[j];
+        mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
+    }
+    const uint64_t xe = x.base + x.size;
+    bool bad = false;
+    // M-M: mortals registered as live at some allocation of this block
+    const uint64_t r0 = p.d.off_b[b];
+    const uint64_t r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
+    for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
+        const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
+        __syncwarp();
+        for (uint32_t q = lane; q < m; q += 32) {
+            const WinRec y = p.d.list_b[bs + q];
+            S.base[warp][q] = y.base;
+            S.end[warp][q] = y.end;
+            S.tf[warp][q] = y.t_free;
+            S.idx[warp][q] = y.id;
+        }
+        __syncwarp();
+        if (mine && !bad) {
+            for (uint32_t q = 0; q < m; ++q) {
+                if (S.idx[warp][q] < j && S.tf[warp][q] > x.t_alloc && S.base[warp][q] < xe && x.base < S.end[warp][q]) {
+                    bad = true;
+                    break;
+                }
+            }
+        }
+    }
+    // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
+    if (mine && !bad && nI) {
+        const uint32_t e = i_count_le(S.fence, nf, stride, nI, p.d.i_base, xe - 1);  // bases < end
+        const uint32_t k0 = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x.base);
+        const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
+        // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
+        const bool freed_early = x.t_free <= t_last;
+        uint32_t k = s;
+        for (; k < e && (k % kIBlk) != 0; ++k)
+            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
+        for (; k + kIBlk <= e; k += kIBlk)
+            bad |= freed_early ? ~p.d.blk_min_ta_c[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
+        for (; k < e; ++k)
+            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
+    }
+    if (bad) flag(p.d.ctl, ST_TRACE);
+}
+
+__global__ void __launch_bounds__(kThreads) k_scan_words(P p) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    if (blockIdx.x < p.C) classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
+    else check_role(p, blockIdx.x - p.C, *reinterpret_cast<ChkShared*>(smem_raw));
+}
+
+// ----------------------------------------------------------------------------
+// 5. k_emit: compaction of the staged records into the slot table (one CTA per chunk)
+__global__ void __launch_bounds__(kThreads) k_emit(P p) {
     __shared__ uint32_t s_mask[64];
     __shared__ uint32_t s_pre[64];
     const MaterializeArgs& a = p.a;
@@ -961,9 +906,10 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
     const size_t N = std::max<size_t>(n, 1024), CC = std::max<size_t>(C, 64), NB = std::max<size_t>(nb, 64);
     const size_t WW = std::max<size_t>(W, 2048);
     const size_t RC = std::max<size_t>(need_c, N + 4 * CC), RB = std::max<size_t>(need_b, 3 * N);
+    const size_t NS = N / kIBlk + 1;
     cudaError_t e;
-    // zero region: Ctl | cnt_c fill_c off_c [CC+1] | cnt_b fill_b off_b [NB+1]
-    s.zero_bytes = 256 + 3 * (CC + 1) * 4 + 3 * (NB + 1) * 4 + 64;
+    // zero region: Ctl | cnt_c fill_c off_c [CC+1] | cnt_b fill_b off_b [NB+1] | blk_min_ta_c blk_max_tf [NS]
+    s.zero_bytes = 256 + 3 * (CC + 1) * 4 + 3 * (NB + 1) * 4 + 2 * NS * 4 + 64;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
     char* z = (char*)s.zero_region;
     s.d.ctl = (Ctl*)z;
@@ -974,12 +920,13 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
     s.d.cnt_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
     s.d.fill_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
     s.d.off_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
-    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.node_fence, (size_t)kNodeFenceCap)) ||
-        (e = grow(s, s.d.rng, N)) || (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) ||
-        (e = grow(s, s.d.sk[0], N)) || (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) ||
-        (e = grow(s, s.d.sv[1], N)) || (e = grow(s, s.d.rank, N)) || (e = grow(s, s.d.i_base, N)) ||
-        (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.blk_min_ta, N / kIBlk + 1)) ||
-        (e = grow(s, s.d.blk_max_tf, N / kIBlk + 1)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
+    s.d.blk_min_ta_c = (uint32_t*)(z + o); o += NS * 4;
+    s.d.blk_max_tf = (uint32_t*)(z + o); o += NS * 4;
+    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.rng, N)) ||
+        (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) || (e = grow(s, s.d.sk[0], N)) ||
+        (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) || (e = grow(s, s.d.sv[1], N)) ||
+        (e = grow(s, s.d.rank, N)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
+        (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
         (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)))
         return e;
     s.d.cap_c = RC;
@@ -1000,68 +947,46 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     if ((int)g_scratch.size() <= dev) g_scratch.resize(dev + 1, nullptr);
     if (!g_scratch[dev]) g_scratch[dev] = new Scratch();
     Scratch& s = *g_scratch[dev];
+    const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
     if (!s.h_ctl) {
         if ((e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-        cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ClsShared));
+        cudaFuncSetAttribute(k_scan_words, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem);
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
     const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
-    const uint32_t nstride = std::max<uint32_t>(1, (a.n_nodes + kNodeFenceCap - 1) / kNodeFenceCap);
-    const uint64_t max_tiles = (n + kSortTile - 1) / kSortTile;
-    const int merge_mode = max_tiles > kRankMaxTiles ? 1 : 0;
+    const uint32_t node_ctas = (a.n_nodes + 1 + kThreads - 1) / kThreads;
+    const uint32_t alloc_ctas = (uint32_t)((n + kThreads - 1) / kThreads);
+    const uint32_t sort_ctas = (uint32_t)((n + kSortTile - 1) / kSortTile);
+    const uint32_t check_ctas = n ? std::max<uint32_t>((nb + kWarps - 1) / kWarps, alloc_ctas) : 0;
     size_t need_c = 0, need_b = 0;
     for (int attempt = 0; attempt < 3; ++attempt) {
         if ((e = ensure(s, n, C, nb, a.n_words, need_c, need_b)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-        P p{a, s.d, C, nb, nstride, merge_mode};
+        P p{a, s.d, C, nb, node_ctas, sort_ctas, check_ctas};
         if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) break;
         if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) break;
-        const uint32_t T = 256;
         {
-            TimedLaunch tl("mat_nodes_chunks", stream);
-            k_nodes_chunks<<<(unsigned)((a.n_nodes + 1 + T - 1) / T), T, 0, stream>>>(p);
+            TimedLaunch tl("mat_trace", stream);
+            k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
         }
         if (n) {
             {
-                TimedLaunch tl("mat_allocs", stream);
-                k_allocs<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
+                TimedLaunch tl("mat_prepare", stream);
+                k_prepare<<<sort_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
             }
-            {
-                TimedLaunch tl("mat_scatter", stream);
-                k_scatter<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
-            }
-            const unsigned tiles = (unsigned)max_tiles;
-            {
-                TimedLaunch tl("mat_sort_tile", stream);
-                k_sort_tile<<<tiles, 256, 0, stream>>>(p);
-            }
-            if (!merge_mode) {
-                TimedLaunch tl("mat_rank", stream);
-                const uint64_t pairs = n * max_tiles;
-                const unsigned grid = (unsigned)std::min<uint64_t>((pairs + T - 1) / T, (uint64_t)s.sm_count * 8);
-                k_rank<<<grid, T, 0, stream>>>(p);
-            } else {
-                int pass = 0;
-                for (uint64_t width = kSortTile; width < n; width *= 2, ++pass) {
-                    TimedLaunch tl("mat_merge", stream);
-                    k_merge<<<(unsigned)((n + kMergeTile - 1) / kMergeTile), 256, 0, stream>>>(p, (uint32_t)width, pass);
-                }
-            }
-            {
-                TimedLaunch tl("mat_finalize_i", stream);
-                k_finalize_i<<<(unsigned)((n + T - 1) / T), T, 0, stream>>>(p);
-            }
-            TimedLaunch tl("mat_check", stream);
-            k_check<<<(nb + 7) / 8, 256, 0, stream>>>(p);
+            TimedLaunch tl("mat_rank", stream);
+            const uint64_t pairs = n * (uint64_t)sort_ctas;
+            const unsigned grid = (unsigned)std::min<uint64_t>((pairs + kThreads - 1) / kThreads, (uint64_t)s.sm_count * 8);
+            k_rank<<<grid, kThreads, 0, stream>>>(p);
+        }
+        if (C + check_ctas) {
+            TimedLaunch tl("mat_classify", stream);
+            k_scan_words<<<C + check_ctas, kThreads, scan_smem, stream>>>(p);
         }
         if (C) {
-            {
-                TimedLaunch tl("mat_classify", stream);
-                k_classify<<<C, kClsThreads, sizeof(ClsShared), stream>>>(p);
-            }
             TimedLaunch tl("mat_emit", stream);
-            k_emit<<<C, 256, 0, stream>>>(p);
+            k_emit<<<C, kThreads, 0, stream>>>(p);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) break;
         if ((e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess) break;
