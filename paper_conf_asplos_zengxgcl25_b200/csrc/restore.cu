@@ -8,18 +8,22 @@
 //
 // The pass is HBM-bound: per word it reads 8 B and writes 8 B; the mask adds
 // 1/8 B, each slot record 8 B (about 18% of words are slots).  Design (B200):
-//   * one CTA of 256 threads per 2048-word chunk; a thread moves four 16-byte
-//     pairs with streaming (L1::no_allocate) vector loads issued first, so
-//     32 KB per CTA is in flight;
+//   * one CTA of 256 threads per 2048-word chunk.  The chunk's 16 KB of words
+//     move HBM -> shared memory -> HBM with the TMA engine (cp.async.bulk load
+//     completing on an mbarrier, cp.async.bulk store from shared memory), so no
+//     thread holds image words in registers and ~17 KB of shared memory and ~30
+//     registers per CTA let 8 CTAs share an SM;
 //   * the chunk's records are the contiguous range [chunk_base[c],
-//     chunk_base[c+1]), known after one load -- fetched coalesced into shared
-//     memory with the three base-table gathers (L2-resident: 24 B per
-//     allocation) done per record, not per word, while the mask's prefix
-//     popcounts are scanned; a word finds its record at
-//     prefix[mask word] + popc(mask & lanemask);
+//     chunk_base[c+1]), known after one load.  Work is per record, not per
+//     word: thread r loads record r (coalesced), gathers old_base / new_base /
+//     new_size of its allocation (L2-resident, 24 B per allocation), finds its
+//     word as the (r - prefix)-th set bit of one mask word (__fns over a 64-entry
+//     shared popcount prefix), validates and rewrites the word in shared memory;
 //   * gather tasks (2048 nodes each) are appended to the same grid;
 //   * validation failures (rare) go to the report with atomics; a one-thread
 //     kernel initializes the report first, so CTAs need no fence or ticket.
+// Images whose base or length break TMA's 16-byte granularity use plain loads and
+// stores through the same shared buffer.
 #include "common.cuh"
 
 namespace medusa {
@@ -27,11 +31,8 @@ namespace {
 
 constexpr int kTaskWords = MEDUSA_CHUNK_WORDS;  // 2048
 constexpr int kThreads = 256;
-constexpr int kPairsPerThread = kTaskWords / 2 / kThreads;  // 4
-constexpr int kMaskPerTask = kTaskWords / 32;                // 64
+constexpr int kMaskPerTask = kTaskWords / 32;   // 64
 constexpr int kNodesPerTask = 2048;
-
-enum : uint8_t { REC_OK = 0, REC_BAD_ID = 1, REC_BAD_RANGE = 2 };
 
 __global__ void report_init(medusa_report* r) {
     r->n_bad_slot = 0;
@@ -44,35 +45,41 @@ __global__ void report_init(medusa_report* r) {
     r->reserved = 0;
 }
 
-__global__ void __launch_bounds__(kThreads)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__global__ void __launch_bounds__(kThreads, 6)
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
+    __shared__ __align__(128) uint64_t s_words[kTaskWords];
     __shared__ uint32_t s_mask[kMaskPerTask];
     __shared__ uint32_t s_pre[kMaskPerTask];
-    __shared__ uint64_t s_expect[kTaskWords];
-    __shared__ uint64_t s_newv[kTaskWords];
-    __shared__ uint8_t s_kind[kTaskWords];
     __shared__ uint32_t s_rec0, s_nrec;
+    __shared__ __align__(8) unsigned long long s_mbar;
 
-    const int tid = threadIdx.x;
+    const uint32_t tid = threadIdx.x;
     const uint32_t task = blockIdx.x;
     unsigned long long* rep = reinterpret_cast<unsigned long long*>(a.report);
 
     if (task < n_word_tasks) {
         const uint64_t ws = (uint64_t)task * kTaskWords;
-        const uint64_t we = min(ws + kTaskWords, a.n_words);
-        // 1. the words first (streaming, 16 B per load), then mask and record range
-        uint64_t v[2 * kPairsPerThread];
-        const bool vec = ((reinterpret_cast<uintptr_t>(a.src) | reinterpret_cast<uintptr_t>(a.dst)) & 15) == 0;
-#pragma unroll
-        for (int k = 0; k < kPairsPerThread; ++k) {
-            const uint64_t g = ws + 2ull * (tid + k * kThreads);
-            if (vec && g + 1 < we) {
-                ld_stream_v2(a.src + g, v[2 * k], v[2 * k + 1]);
-            } else {
-                v[2 * k] = g < we ? ld_stream(a.src + g) : 0;
-                v[2 * k + 1] = g + 1 < we ? ld_stream(a.src + g + 1) : 0;
-            }
+        const uint32_t n = (uint32_t)min((uint64_t)kTaskWords, a.n_words - ws);
+        const uint64_t* gsrc = a.src + ws;
+        uint64_t* gdst = a.dst + ws;
+        const bool tma = (((reinterpret_cast<uintptr_t>(gsrc) | reinterpret_cast<uintptr_t>(gdst)) & 15) == 0) &&
+                         (n % 2 == 0);
+        const uint32_t mb = smem_u32(&s_mbar);
+        // 1. the chunk's words: one bulk copy into shared memory; meanwhile the
+        //    mask words and the record range
+        if (tid == 0 && tma) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                         ::"r"(smem_u32(s_words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
         }
+        if (!tma)
+            for (uint32_t q = tid; q < n; q += kThreads) s_words[q] = ld_stream(gsrc + q);
         const uint64_t n_mask = (a.n_words + 31) / 32;
         const uint64_t mw0 = ws / 32;
         if (tid < kMaskPerTask) {
@@ -83,7 +90,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             s_nrec = r1 > r0 ? r1 - r0 : 0;
         }
         __syncthreads();
-        // 2. warp 0: exclusive scan of the 64 mask popcounts; everyone: records
+        // 2. exclusive prefix of the 64 mask popcounts (warp 0)
         if (tid < 32) {
             const uint32_t p0 = __popc(s_mask[2 * tid]), p1 = __popc(s_mask[2 * tid + 1]);
             uint32_t incl = p0 + p1;
@@ -96,71 +103,88 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             s_pre[2 * tid + 1] = incl - p1;
         }
         const uint64_t rec0 = s_rec0;
-        const uint32_t n_rec = min(s_nrec, (uint32_t)kTaskWords);
-        for (uint32_t r = tid; r < n_rec; r += kThreads) {
-            const uint64_t k = rec0 + r;
-            uint8_t kind = REC_BAD_ID;
-            uint64_t exp = 0, nv = 0;
-            if (k < a.n_slots) {
-                const uint64_t rec = a.slot[k];
-                const uint64_t id = rec >> MEDUSA_OFF_BITS;
-                const uint64_t off = rec & kOffMask;
-                if (id < a.n_alloc) {
-                    const uint64_t sz = __ldg(a.new_size + id);
-                    const uint64_t ob = __ldg(a.old_base + id);
-                    const uint64_t nb = __ldg(a.new_base + id);
-                    if (off < sz) {
-                        kind = REC_OK;
-                        exp = ob + off;
-                        nv = nb + off;
-                    } else {
-                        kind = REC_BAD_RANGE;
-                    }
-                }
-            }
-            s_kind[r] = kind;
-            s_expect[r] = exp;
-            s_newv[r] = nv;
-        }
-        __syncthreads();
-        // 3. rewrite slot words, validate, store
+        const uint32_t n_rec = s_nrec;
+        const uint32_t n_rec_c = min(n_rec, (uint32_t)kTaskWords);
+        // 3. records, two per thread per round: load, gather, (after the prefix is
+        //    ready) locate the word, validate and rewrite it in shared memory
         uint32_t n_id = 0, n_rg = 0, n_st = 0;
         uint64_t first = ~0ull;
+        bool words_ready = !tma;
+        for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += 2 * kThreads) {
+            uint64_t exp[2], nv[2];
+            uint32_t kind[2];  // 0 ok, 1 bad id, 2 bad range, 3 none
 #pragma unroll
-        for (int k = 0; k < kPairsPerThread; ++k) {
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const uint32_t q = 2 * (tid + k * kThreads) + h;  // word within the chunk
-                const uint32_t mw = s_mask[q >> 5];
-                if ((mw >> (q & 31)) & 1u) {
-                    const uint32_t r = s_pre[q >> 5] + __popc(mw & ((1u << (q & 31)) - 1u));
-                    bool bad = true;
-                    if (r < n_rec) {
-                        const uint8_t kind = s_kind[r];
-                        if (kind == REC_OK) {
-                            if (v[2 * k + h] == s_expect[r]) { v[2 * k + h] = s_newv[r]; bad = false; }
-                            else ++n_st;
-                        } else if (kind == REC_BAD_ID) {
-                            ++n_id;
-                        } else {
-                            ++n_rg;
+            for (int u = 0; u < 2; ++u) {
+                const uint32_t r = rb + tid + u * kThreads;
+                kind[u] = 3;
+                exp[u] = nv[u] = 0;
+                if (r < n_rec_c) {
+                    kind[u] = 1;
+                    const uint64_t k = rec0 + r;
+                    if (k < a.n_slots) {
+                        const uint64_t rec = a.slot[k];
+                        const uint64_t id = rec >> MEDUSA_OFF_BITS;
+                        const uint64_t off = rec & kOffMask;
+                        if (id < a.n_alloc) {
+                            const uint64_t sz = __ldg(a.new_size + id);
+                            const uint64_t ob = __ldg(a.old_base + id);
+                            const uint64_t nb = __ldg(a.new_base + id);
+                            if (off < sz) {
+                                kind[u] = 0;
+                                exp[u] = ob + off;
+                                nv[u] = nb + off;
+                            } else {
+                                kind[u] = 2;
+                            }
                         }
-                    } else {
-                        ++n_id;  // table shorter than its mask says: no record to apply
                     }
-                    if (bad) first = min(first, ws + q);
                 }
             }
-        }
-#pragma unroll
-        for (int k = 0; k < kPairsPerThread; ++k) {
-            const uint64_t g = ws + 2ull * (tid + k * kThreads);
-            if (vec && g + 1 < we) {
-                st_stream_v2(a.dst + g, v[2 * k], v[2 * k + 1]);
-            } else {
-                if (g < we) st_stream(a.dst + g, v[2 * k]);
-                if (g + 1 < we) st_stream(a.dst + g + 1, v[2 * k + 1]);
+            if (rb == 0) __syncthreads();  // s_pre ready
+            if (!words_ready) {
+                uint32_t ready = 0;
+                while (!ready) {
+                    asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
+                                 : "=r"(ready) : "r"(mb) : "memory");
+                }
+                words_ready = true;
             }
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+                if (kind[u] == 3) continue;
+                const uint32_t r = rb + tid + u * kThreads;
+                uint32_t lo = 0, hi = kMaskPerTask;  // mask word m with s_pre[m] <= r < s_pre[m] + popc
+                while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
+                const uint32_t bit = __fns(s_mask[lo], 0, r - s_pre[lo] + 1);
+                const uint32_t q = lo * 32 + bit;
+                bool bad = true;
+                if (bit >= 32 || q >= n) {
+                    ++n_id;  // more records than mask bits: nothing to apply
+                } else if (kind[u] == 0) {
+                    if (s_words[q] == exp[u]) { s_words[q] = nv[u]; bad = false; }
+                    else ++n_st;
+                } else if (kind[u] == 1) {
+                    ++n_id;
+                } else {
+                    ++n_rg;
+                }
+                if (bad) first = min(first, ws + (q < n ? q : 0));
+            }
+        }
+        // slots the mask shows beyond the table's records have nothing to apply
+        if (tid == 0 && n_rec > (uint32_t)kTaskWords) n_id += n_rec - kTaskWords;
+        __syncthreads();
+        // 4. the chunk's words back to HBM
+        if (tma) {
+            if (tid == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                             ::"l"(gdst), "r"(smem_u32(s_words)), "r"(n * 8) : "memory");
+                asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+            }
+        } else {
+            for (uint32_t q = tid; q < n; q += kThreads) st_stream(gdst + q, s_words[q]);
         }
         if (n_id | n_rg | n_st) {
             atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));

@@ -11,7 +11,7 @@ vals = [float(r[idx["Metric Value"]]) for r in data]
 unit = data[0][idx["Metric Unit"]] if data else "ns"
 scale = {"ns": 1e-3, "nsecond": 1e-3, "us": 1, "usecond": 1, "ms": 1e3, "msecond": 1e3}[unit]
 # one step = from the last 'k_nodes_chunks' to the following 'restore_kernel'
-starts = [i for i, n in enumerate(names) if n == "k_nodes_chunks"]
+starts = [i for i, n in enumerate(names) if n == "k_trace"]
 s = starts[-3] if len(starts) >= 3 else starts[0]  # the timed step (before the e2e loop)
 e = next(i for i in range(s, len(names)) if names[i] == "restore_kernel")
 tot = 0.0
