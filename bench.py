@@ -266,20 +266,32 @@ def run_ours(args):
                 "traffic": traffic.get("restore")}
     mat_s = sum(v[1] for k, v in per.items() if k.startswith("mat_")) / args.steps / 1e3
 
-    # ---- sustained relocate: back-to-back restores of the resident set (no scrub) ----
+    # ---- sustained relocate: back-to-back restores over R distinct copies of the
+    #      image (working set >> L2, so dirty-line write-back is paid inside) ----
     sus = None
     if args.sustained > 0:
+        R = 8
+        srcs = [inp["words"].clone() for _ in range(R)]
+        dsts = [torch.empty_like(inp["words"]) for _ in range(R)]
+        for r in range(R):  # warm
+            medusa.restore(srcs[r], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                           dst=dsts[r], func_out=fout, report=rep)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        big = int(args.sustained)
+        big = max(int(args.sustained), R)
+        torch.cuda.synchronize(dev)
         e0.record(stream)
-        for _ in range(big):
-            medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
-                           dst=dst, func_out=fout, report=rep)
+        for k in range(big):
+            medusa.restore(srcs[k % R], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                           dst=dsts[k % R], func_out=fout, report=rep)
         e1.record(stream)
         torch.cuda.synchronize(dev)
         s = e0.elapsed_time(e1) / 1e3 / big
-        sus = {"restores": big, "avg_us": s * 1e6, "GB/s": alg["restore"] / s / 1e9,
-               "note": "back-to-back, L2-warm (set fits in the 126 MB L2): upper bound, not the roofline number"}
+        sus = {"restores": big, "replicas": R, "avg_us": s * 1e6, "GB/s": alg["restore"] / s / 1e9,
+               "frac_of_peak": alg["restore"] / s / 1e9 / peak, "nodes_per_s": gs.n_nodes / s,
+               "working_set_MB": R * 2 * gs.n_words * 8 / 1e6,
+               "note": "back-to-back restores cycling through R distinct image copies (inputs > L2); "
+                       "includes report init; algorithmic bytes as in roofline"}
+        del srcs, dsts
 
     # ---- end to end: pinned host buffers -> H2D -> whole path -> D2H of results ----
     h = medusa.host_arrays(gs)
