@@ -51,7 +51,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-struct Stage {
+struct __align__(128) Stage {
     uint64_t words[kTaskWords];  // TMA destination and source (16 KB)
     uint32_t mask[kMaskPerTask];
     uint32_t pre[kMaskPerTask];
