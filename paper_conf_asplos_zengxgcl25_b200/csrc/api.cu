@@ -170,7 +170,7 @@ medusa_status medusa_restore(const uint64_t* d_src_words, uint64_t* d_dst_words,
         n_func = g_tables[dev].n_func;
     }
     RestoreArgs a{d_src_words, d_dst_words, n_words, slots->d_mask, slots->d_chunk_base, slots->d_slot,
-                  n_slots < slots->capacity ? n_slots : slots->capacity, d_old_base, d_new_base, d_new_size,
+                  n_slots < slots->capacity ? n_slots : slots->capacity, slots->capacity, d_old_base, d_new_base, d_new_size,
                   n_alloc, gather ? d_func_id : nullptr, d_func_out, gather ? n_nodes : 0, table, n_func,
                   d_report};
     e = launch_restore(a, stream);

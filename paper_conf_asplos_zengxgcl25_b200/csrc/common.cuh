@@ -55,6 +55,7 @@ struct RestoreArgs {
     const uint32_t* chunk_base;
     const uint64_t* slot;
     uint64_t n_slots;  // records that may be read: min(n_slots, capacity)
+    uint64_t slot_capacity;
     const uint64_t* old_base;
     const uint64_t* new_base;
     const uint64_t* new_size;

@@ -51,11 +51,19 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
+constexpr int kStages = 3;
+constexpr int kRecCap = 1024;                 // records per stage delivered by TMA (else loaded directly)
+constexpr int kConsumers = kThreads;          // 8 consumer warps
+constexpr int kBlock = kConsumers + 32;       // + 1 producer warp
+
 struct __align__(128) Stage {
-    uint64_t words[kTaskWords];  // TMA destination and source (16 KB)
-    uint32_t mask[kMaskPerTask];
+    uint64_t words[kTaskWords];   // TMA in -> rewritten -> TMA out (16 KB)
+    uint64_t recs[kRecCap + 2];   // the chunk's records from an even index (TMA)
+    uint32_t mask[kMaskPerTask];  // TMA
     uint32_t pre[kMaskPerTask];
-    uint32_t rec0, nrec;
+    uint32_t chunk, n, rec0, nrec;
+    uint32_t flags;               // 1: words by TMA, 2: mask by TMA, 4: records by TMA
+    uint32_t rec_skew;            // rec0 - first record delivered
 };
 
 __device__ __forceinline__ void mbar_wait(uint32_t mb, uint32_t parity) {
@@ -65,21 +73,30 @@ __device__ __forceinline__ void mbar_wait(uint32_t mb, uint32_t parity) {
                      : "=r"(ready) : "r"(mb), "r"(parity) : "memory");
     }
 }
+__device__ __forceinline__ void tma_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t mb) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(dst), "l"(src), "r"(bytes), "r"(mb) : "memory");
+}
+__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
 
-// Persistent CTAs over chunks c = blockIdx.x, + gridWords, ...  Two stages: while
-// chunk c is processed from stage b, the TMA engine brings chunk c+G's words into
-// stage b^1, and its mask words, record range and first records arrive in registers.
-__global__ void __launch_bounds__(kThreads, 4)
+// Warp-specialized persistent CTAs.  The producer warp (one lane) owns every TMA
+// transfer: for chunk c = blockIdx.x + k*G it fills stage k % kStages with the
+// chunk's words, mask words and records (one mbarrier with the byte count), and
+// once the consumers signal the stage done it writes the words back with a TMA
+// bulk store and refills the stage.  The 8 consumer warps only gather base-table
+// entries, locate and rewrite slot words in shared memory.
+__global__ void __launch_bounds__(kBlock, 2)
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_t n_node_tasks) {
-    __shared__ __align__(128) Stage st[2];
-    __shared__ __align__(8) unsigned long long s_mbar[2];
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    Stage* st = reinterpret_cast<Stage*>(smem_raw);
+    __shared__ __align__(8) unsigned long long s_full[kStages], s_done[kStages];
 
     const uint32_t tid = threadIdx.x;
     unsigned long long* rep = reinterpret_cast<unsigned long long*>(a.report);
 
     if (blockIdx.x >= word_ctas) {  // kernel-address fill
         const uint32_t task = blockIdx.x - word_ctas;
-        if (task >= n_node_tasks) return;
+        if (task >= n_node_tasks || tid >= kThreads) return;
         const uint64_t j0 = (uint64_t)task * kNodesPerTask;
         uint32_t n_bad = 0;
         uint64_t first = ~0ull;
@@ -104,59 +121,84 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_
         return;
     }
 
-    const uint64_t n_mask = (a.n_words + 31) / 32;
-    const bool aligned = ((reinterpret_cast<uintptr_t>(a.src) | reinterpret_cast<uintptr_t>(a.dst)) & 15) == 0;
-    auto chunk_n = [&](uint32_t c) { return (uint32_t)min((uint64_t)kTaskWords, a.n_words - (uint64_t)c * kTaskWords); };
-    auto chunk_tma = [&](uint32_t c) { return aligned && (chunk_n(c) % 2 == 0); };
-    const uint32_t mb0 = (uint32_t)__cvta_generic_to_shared(&s_mbar[0]);
-    const uint32_t mb1 = (uint32_t)__cvta_generic_to_shared(&s_mbar[1]);
-
-    // prefetch of chunk c into stage b: words by TMA; mask words / record range /
-    // first records into registers (written to shared memory at the next step)
-    uint32_t pf_mask = 0, pf_cb0 = 0, pf_cb1 = 0;
-    auto issue_prefetch = [&](uint32_t c, int b) {
-        if (tid == 0 && chunk_tma(c)) {
-            const uint32_t mb = b ? mb1 : mb0;
-            const uint32_t bytes = chunk_n(c) * 8;
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(bytes) : "memory");
-            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                         ::"r"((uint32_t)__cvta_generic_to_shared(st[b].words)), "l"(a.src + (uint64_t)c * kTaskWords),
-                         "r"(bytes), "r"(mb) : "memory");
-        }
-        const uint64_t mw = (uint64_t)c * kMaskPerTask + tid;
-        if (tid < kMaskPerTask) pf_mask = mw < n_mask ? a.mask[mw] : 0u;
-        if (tid == kMaskPerTask) { pf_cb0 = a.chunk_base[c]; pf_cb1 = a.chunk_base[c + 1]; }
-    };
-    auto commit_prefetch = [&](int b) {
-        if (tid < kMaskPerTask) st[b].mask[tid] = pf_mask;
-        if (tid == kMaskPerTask) { st[b].rec0 = pf_cb0; st[b].nrec = pf_cb1 > pf_cb0 ? pf_cb1 - pf_cb0 : 0; }
-    };
-
     if (tid == 0) {
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb0));
-        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb1));
+        for (int s = 0; s < kStages; ++s) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"((uint32_t)__cvta_generic_to_shared(&s_full[s])));
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"((uint32_t)__cvta_generic_to_shared(&s_done[s])));
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    const uint32_t n_mine = n_word_tasks > blockIdx.x ? (n_word_tasks - blockIdx.x + word_ctas - 1) / word_ctas : 0;
+    const uint64_t n_mask = (a.n_words + 31) / 32;
+    const uint64_t n_rec_total = a.n_slots;
 
+    if (tid >= kConsumers) {
+        // ------------------------------------------------------------ producer
+        if (tid != kConsumers) return;
+        const bool aligned = ((reinterpret_cast<uintptr_t>(a.src) | reinterpret_cast<uintptr_t>(a.dst)) & 15) == 0;
+        auto store_stage = [&](int s) {  // words of the chunk held in stage s back to HBM
+            Stage& S = st[s];
+            if (S.flags & 1) {
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                             ::"l"(a.dst + (uint64_t)S.chunk * kTaskWords),
+                             "r"((uint32_t)__cvta_generic_to_shared(S.words)), "r"(S.n * 8) : "memory");
+                asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+            }
+        };
+        for (uint32_t k = 0; k < n_mine + kStages; ++k) {
+            const int s = k % kStages;
+            Stage& S = st[s];
+            if (k >= kStages) {  // the stage's previous chunk: wait for the consumers, write it back
+                mbar_wait((uint32_t)__cvta_generic_to_shared(&s_done[s]), ((k / kStages) - 1) & 1);
+                store_stage(s);
+                asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+            }
+            if (k >= n_mine) continue;
+            const uint32_t c = blockIdx.x + k * word_ctas;
+            const uint64_t ws = (uint64_t)c * kTaskWords;
+            const uint32_t n = (uint32_t)min((uint64_t)kTaskWords, a.n_words - ws);
+            const uint32_t r0 = a.chunk_base[c], r1 = a.chunk_base[c + 1];
+            const uint32_t nrec = r1 > r0 ? r1 - r0 : 0;
+            uint32_t flags = 0, bytes = 0;
+            if (aligned && n % 2 == 0) { flags |= 1; bytes += n * 8; }
+            const uint64_t m0 = (uint64_t)c * kMaskPerTask;
+            if (m0 + kMaskPerTask <= n_mask && ((reinterpret_cast<uintptr_t>(a.mask + m0) & 15) == 0)) {
+                flags |= 2;
+                bytes += kMaskPerTask * 4;
+            }
+            const uint64_t e0 = r0 & ~1ull, e1 = ((uint64_t)r0 + nrec + 1) & ~1ull;  // even-aligned record span
+            const bool rec_ok = nrec > 0 && nrec <= kRecCap && e1 <= min(n_rec_total, a.slot_capacity) &&
+                                ((reinterpret_cast<uintptr_t>(a.slot) & 15) == 0);
+            if (rec_ok) { flags |= 4; bytes += (uint32_t)(e1 - e0) * 8; }
+            S.chunk = c; S.n = n; S.rec0 = r0; S.nrec = nrec; S.flags = flags; S.rec_skew = (uint32_t)(r0 - e0);
+            const uint32_t mb = (uint32_t)__cvta_generic_to_shared(&s_full[s]);
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(bytes) : "memory");
+            if (flags & 1) tma_load((uint32_t)__cvta_generic_to_shared(S.words), a.src + ws, n * 8, mb);
+            if (flags & 2) tma_load((uint32_t)__cvta_generic_to_shared(S.mask), a.mask + m0, kMaskPerTask * 4, mb);
+            if (flags & 4) tma_load((uint32_t)__cvta_generic_to_shared(S.recs), a.slot + e0, (uint32_t)(e1 - e0) * 8, mb);
+        }
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        return;
+    }
+
+    // -------------------------------------------------------------- consumers
     uint32_t n_id = 0, n_rg = 0, n_st = 0;
     uint64_t first = ~0ull;
-    uint32_t c = blockIdx.x;
-    if (c < n_word_tasks) issue_prefetch(c, 0);
-    for (uint32_t it = 0; c < n_word_tasks; ++it, c += word_ctas) {
-        const int b = it & 1;
-        Stage& S = st[b];
-        const uint32_t n = chunk_n(c);
+    for (uint32_t k = 0; k < n_mine; ++k) {
+        const int s = k % kStages;
+        Stage& S = st[s];
+        mbar_wait((uint32_t)__cvta_generic_to_shared(&s_full[s]), (k / kStages) & 1);
+        const uint32_t c = S.chunk, n = S.n, flags = S.flags, nrec = S.nrec;
         const uint64_t ws = (uint64_t)c * kTaskWords;
-        commit_prefetch(b);
-        __syncthreads();  // stage b's mask / range visible; stage b^1 no longer read
-        const uint32_t next = c + word_ctas;
-        if (next < n_word_tasks) {
-            if (tid == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // stage b^1's store has read its words
-            issue_prefetch(next, b ^ 1);
+        const uint64_t rec0 = S.rec0;
+        if (!(flags & 1))
+            for (uint32_t q = tid; q < n; q += kConsumers) S.words[q] = ld_stream(a.src + ws + q);
+        if (!(flags & 2) && tid < kMaskPerTask) {
+            const uint64_t mw = (uint64_t)c * kMaskPerTask + tid;
+            S.mask[tid] = mw < n_mask ? a.mask[mw] : 0u;
         }
-        if (!chunk_tma(c))
-            for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(a.src + ws + q);
+        if (!(flags & 2)) consumer_sync();
         if (tid < 32) {  // exclusive prefix of the 64 mask popcounts
             const uint32_t p0 = __popc(S.mask[2 * tid]), p1 = __popc(S.mask[2 * tid + 1]);
             uint32_t incl = p0 + p1;
@@ -168,23 +210,21 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_
             S.pre[2 * tid] = incl - p0 - p1;
             S.pre[2 * tid + 1] = incl - p1;
         }
-        const uint64_t rec0 = S.rec0;
-        const uint32_t n_rec = S.nrec;
-        const uint32_t n_rec_c = min(n_rec, (uint32_t)kTaskWords);
-        bool words_ready = !chunk_tma(c);
-        for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += 2 * kThreads) {
+        const uint32_t n_rec_c = min(nrec, (uint32_t)kTaskWords);
+        // records, two per thread per round: gather, (prefix ready) locate, rewrite
+        for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += 2 * kConsumers) {
             uint64_t exp[2], nv[2];
             uint32_t kind[2];  // 0 ok, 1 bad id, 2 bad range, 3 none
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
-                const uint32_t r = rb + tid + u * kThreads;
+                const uint32_t r = rb + tid + u * kConsumers;
                 kind[u] = 3;
                 exp[u] = nv[u] = 0;
                 if (r < n_rec_c) {
                     kind[u] = 1;
-                    const uint64_t k = rec0 + r;
-                    if (k < a.n_slots) {
-                        const uint64_t rec = a.slot[k];
+                    const uint64_t kk = rec0 + r;
+                    if (kk < n_rec_total) {
+                        const uint64_t rec = (flags & 4) ? S.recs[S.rec_skew + r] : a.slot[kk];
                         const uint64_t id = rec >> MEDUSA_OFF_BITS;
                         const uint64_t off = rec & kOffMask;
                         if (id < a.n_alloc) {
@@ -202,15 +242,11 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_
                     }
                 }
             }
-            if (rb == 0) __syncthreads();  // prefix ready (and plain-loaded words)
-            if (!words_ready) {
-                mbar_wait(b ? mb1 : mb0, (it >> 1) & 1);
-                words_ready = true;
-            }
+            if (rb == 0) consumer_sync();  // prefix (and directly loaded words) ready
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 if (kind[u] == 3) continue;
-                const uint32_t r = rb + tid + u * kThreads;
+                const uint32_t r = rb + tid + u * kConsumers;
                 uint32_t lo = 0, hi = kMaskPerTask;  // mask word m with pre[m] <= r < pre[m] + popc
                 while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (S.pre[mid] <= r) lo = mid; else hi = mid; }
                 const uint32_t bit = __fns(S.mask[lo], 0, r - S.pre[lo] + 1);
@@ -230,21 +266,17 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_
             }
         }
         // slots the mask shows beyond the table's records have nothing to apply
-        if (tid == 0 && n_rec > (uint32_t)kTaskWords) n_id += n_rec - kTaskWords;
-        __syncthreads();
-        // the chunk's words back to HBM
-        if (chunk_tma(c)) {
-            if (tid == 0) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
-                             ::"l"(a.dst + ws), "r"((uint32_t)__cvta_generic_to_shared(S.words)), "r"(n * 8) : "memory");
-                asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-            }
-        } else {
-            for (uint32_t q = tid; q < n; q += kThreads) st_stream(a.dst + ws + q, S.words[q]);
+        if (tid == 0 && nrec > (uint32_t)kTaskWords) n_id += nrec - kTaskWords;
+        if (!(flags & 1)) {
+            consumer_sync();
+            for (uint32_t q = tid; q < n; q += kConsumers) st_stream(a.dst + ws + q, S.words[q]);
         }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // rewrites visible to the TMA store
+        consumer_sync();
+        if (tid == 0)
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"((uint32_t)__cvta_generic_to_shared(&s_done[s]))
+                         : "memory");
     }
-    if (tid == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
     if (n_id | n_rg | n_st) {
         atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));
         atomicMin(rep + 1, (unsigned long long)first);
@@ -263,17 +295,19 @@ cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sm_count, cudaDevAttrMultiProcessorCount, dev);
         if (sm_count <= 0) sm_count = 148;
+        cudaFuncSetAttribute(restore_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kStages * (int)sizeof(Stage));
     }
     const uint32_t n_word_tasks = (uint32_t)((a.n_words + kTaskWords - 1) / kTaskWords);
     const uint32_t n_node_tasks = a.func_id ? (a.n_nodes + kNodesPerTask - 1) / kNodesPerTask : 0;
-    const uint32_t word_ctas = std::min<uint32_t>(n_word_tasks, (uint32_t)sm_count * 4);
+    const uint32_t word_ctas = std::min<uint32_t>(n_word_tasks, (uint32_t)sm_count * 2);
     {
         TimedLaunch tl("restore_report_init", stream);
         report_init<<<1, 1, 0, stream>>>(a.report);
     }
     if (word_ctas + n_node_tasks) {
         TimedLaunch tl("restore", stream);
-        restore_kernel<<<word_ctas + n_node_tasks, kThreads, 0, stream>>>(a, n_word_tasks, word_ctas, n_node_tasks);
+        restore_kernel<<<word_ctas + n_node_tasks, kBlock, kStages * sizeof(Stage), stream>>>(a, n_word_tasks, word_ctas,
+                                                                                              n_node_tasks);
     }
     return cudaGetLastError();
 }
