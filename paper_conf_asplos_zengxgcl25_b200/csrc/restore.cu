@@ -52,7 +52,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
 }
 
 constexpr int kStages = 3;
-constexpr int kRecCap = 1024;                 // records per stage delivered by TMA (else loaded directly)
+constexpr int kRecCap = 768;                  // records per stage delivered by TMA (else loaded directly)
 constexpr int kConsumers = kThreads;          // 8 consumer warps
 constexpr int kBlock = kConsumers + 32;       // + 1 producer warp
 
@@ -85,7 +85,7 @@ __device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, %0;"
 // once the consumers signal the stage done it writes the words back with a TMA
 // bulk store and refills the stage.  The 8 consumer warps only gather base-table
 // entries, locate and rewrite slot words in shared memory.
-__global__ void __launch_bounds__(kBlock, 2)
+__global__ void __launch_bounds__(kBlock, 3)
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_t n_node_tasks) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     Stage* st = reinterpret_cast<Stage*>(smem_raw);
@@ -137,6 +137,20 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t word_ctas, uint32_
         // ------------------------------------------------------------ producer
         if (tid != kConsumers) return;
         const bool aligned = ((reinterpret_cast<uintptr_t>(a.src) | reinterpret_cast<uintptr_t>(a.dst)) & 15) == 0;
+        {  // warm L2 with this CTA's share of the replayed base table (gathered per record)
+            const uint64_t bytes = (uint64_t)a.n_alloc * 8;
+            const uint64_t per = ((bytes + word_ctas - 1) / word_ctas + 15) & ~15ull;
+            const uint64_t b0 = (uint64_t)blockIdx.x * per;
+            if (b0 < bytes) {
+                const uint32_t len = (uint32_t)((min(b0 + per, bytes) - b0 + 15) & ~15ull);
+                const uint64_t* arrs[3] = {a.new_size, a.old_base, a.new_base};
+                for (int q = 0; q < 3; ++q) {
+                    const char* base = reinterpret_cast<const char*>(arrs[q]);
+                    if ((reinterpret_cast<uintptr_t>(base) & 15) == 0 && b0 + len <= ((bytes + 15) & ~15ull))
+                        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(base + b0), "r"(len) : "memory");
+                }
+            }
+        }
         auto store_stage = [&](int s) {  // words of the chunk held in stage s back to HBM
             Stage& S = st[s];
             if (S.flags & 1) {
@@ -299,7 +313,7 @@ cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     }
     const uint32_t n_word_tasks = (uint32_t)((a.n_words + kTaskWords - 1) / kTaskWords);
     const uint32_t n_node_tasks = a.func_id ? (a.n_nodes + kNodesPerTask - 1) / kNodesPerTask : 0;
-    const uint32_t word_ctas = std::min<uint32_t>(n_word_tasks, (uint32_t)sm_count * 2);
+    const uint32_t word_ctas = std::min<uint32_t>(n_word_tasks, (uint32_t)sm_count * 3);
     {
         TimedLaunch tl("restore_report_init", stream);
         report_init<<<1, 1, 0, stream>>>(a.report);
