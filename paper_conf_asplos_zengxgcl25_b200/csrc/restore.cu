@@ -8,12 +8,14 @@
 //
 // The pass is HBM-bound: per word it reads 8 B and writes 8 B; the mask adds
 // 1/8 B, each slot record 8 B (about 18% of words are slots).  Design (B200):
-//   * one CTA of 128 threads per 2048-word chunk.  The chunk's 16 KB of words
+//   * one CTA of 256 threads per 2048-word chunk.  The chunk's 16 KB of words
 //     move HBM -> shared memory -> HBM with the TMA engine (cp.async.bulk load
 //     completing on an mbarrier, cp.async.bulk store from shared memory), so no
-//     thread holds image words in registers; ~17 KB of shared memory and 4 warps
-//     per CTA let ~12 CTAs share an SM, i.e. every chunk of the ten-model set
-//     (1,512) is resident at once;
+//     thread holds image words in registers; ~17 KB of shared memory and ~35
+//     registers per CTA let 6-7 CTAs share an SM.  (Measured alternatives --
+//     128-thread CTAs, persistent CTAs with a 2-stage ring, a warp-specialized
+//     TMA producer over a 3-stage ring -- were slower: tools/microbench_restore.cu
+//     and DESIGN.md §5);
 //   * thread 0 also asks the TMA engine to prefetch this CTA's slice of the
 //     three base-table arrays into L2 (cp.async.bulk.prefetch.L2), so the
 //     per-record gathers of every CTA hit L2;
@@ -34,7 +36,7 @@ namespace medusa {
 namespace {
 
 constexpr int kTaskWords = MEDUSA_CHUNK_WORDS;  // 2048
-constexpr int kThreads = 128;
+constexpr int kThreads = 256;
 constexpr int kMaskPerTask = kTaskWords / 32;   // 64
 constexpr int kNodesPerTask = 2048;
 
@@ -53,7 +55,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-__global__ void __launch_bounds__(kThreads, 12)
+__global__ void __launch_bounds__(kThreads, 6)
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     __shared__ __align__(128) uint64_t s_words[kTaskWords];
     __shared__ uint32_t s_mask[kMaskPerTask];

@@ -223,3 +223,21 @@ def test_multi_chunk_malformed_ten_model_trace(graph_sets):
     with pytest.raises(medusa.MedusaError) as ei:
         medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], aa)
     assert ei.value.status == medusa.ERR_TRACE
+
+
+def test_replicated_multi_instance_parity(graph_sets):
+    """Three replicas of the Llama-2-7B-shaped set in one call (ids up to 3 x n_alloc,
+    3x the chunks): bit-exact against the oracle."""
+    from workloads.graphset import replicate
+    gs = replicate(graph_sets("llama2-7b"), 3)
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    medusa.kernel_table_set(inp["table"])
+    dst, fout, rep = medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"],
+                                    inp["func_id"])
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size,
+                             gs.func_id, gs.table)
+    _check_materialize(slots, m, packed, gs.n_words)
+    assert np.array_equal(medusa.to_numpy_u64(dst), packed[3])
+    assert np.array_equal(medusa.to_numpy_u64(fout), packed[4])
+    assert np.array_equal(medusa.report_numpy(rep), packed[5])

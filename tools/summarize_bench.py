@@ -7,7 +7,9 @@ print(f"value {d['value']/1e6:.1f} M nodes/s  ms/step {d['ms_per_step']:.3f}  e2
 r = d["roofline"]
 print(f"roofline[{r['kernel']}] {r['achieved']:.0f} GB/s = {100*r['frac']:.1f}% of {r['peak']}")
 rl = d["relocate"]
-print(f"relocate {rl['GB/s']:.0f} GB/s ({100*rl['frac_of_peak']:.1f}%) {rl['avg_us']:.1f} us  sustained={d.get('sustained_relocate')}")
+print(f"relocate {rl['GB/s']:.0f} GB/s ({100*rl['frac_of_peak']:.1f}%) {rl['avg_us']:.1f} us")
+su = d.get('sustained_relocate')
+if su: print(f"sustained relocate x{su['replicas']}: {su['GB/s']:.0f} GB/s ({100*su['frac_of_peak']:.1f}%) {su['avg_ms']:.3f} ms/call {su['nodes_per_s']/1e9:.2f} G nodes/s")
 for k, v in d["kernels"].items():
     print(f"  {k:22s} n={v['launches']:4d} avg {v['avg_us']:8.2f} us  share {100*v['share_of_step']:5.1f}%  " +
           (f"{v['GB/s']:.0f} GB/s" if 'GB/s' in v else ""))

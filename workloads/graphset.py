@@ -610,3 +610,43 @@ def make_graph_set(config: str, seed: int | None = None, models: list | None = N
         for mi, name in enumerate(mlist):
             _run_model(B, mi, MODELS[name])
     return B.build(config)
+
+
+def replicate(gs: GraphSet, R: int, va_stride: int = 1 << 44) -> GraphSet:
+    """R copies of a graph set as one larger set (SURVEY.md §8(d) sustained mode):
+    replica r lives va_stride*r higher in the address space (every address-valued
+    word moves with it; plain constants do not), after all events of replica r-1
+    in time, with allocation ordinals and kernel-name ids offset by r copies."""
+    assert R >= 1
+    span = int(max(int(gs.node_t.max(initial=0)), int(gs.allocs["t_alloc"].max(initial=0)),
+                   int(np.where(gs.allocs["t_free"] == T_NEVER, 0, gs.allocs["t_free"]).max(initial=0)))) + 1
+    assert span * R < T_NEVER
+    is_addr = gs.tags != TAG_CONST
+    words, tags, tid, toff, offs, nts, fids = [], [], [], [], [np.zeros(1, np.uint64)], [], []
+    allocs, new_base = [], []
+    K = gs.table.size
+    for r in range(R):
+        d = np.uint64(va_stride * r)
+        w = gs.words.copy()
+        w[is_addr] += d
+        words.append(w)
+        tags.append(gs.tags)
+        tid.append(np.where(gs.truth_id >= 0, gs.truth_id + r * gs.n_alloc, -1))
+        toff.append(gs.truth_off)
+        offs.append(gs.node_word_off[1:] + np.uint64(r * gs.n_words))
+        nts.append(gs.node_t + np.uint32(r * span))
+        fids.append(gs.func_id + np.uint32(r * K))
+        a = gs.allocs.copy()
+        a["base"] += d
+        a["t_alloc"] += np.uint32(r * span)
+        never = a["t_free"] == T_NEVER
+        a["t_free"] = np.where(never, T_NEVER, a["t_free"] + np.uint32(r * span))
+        allocs.append(a)
+        new_base.append(gs.new_base + d)
+    return GraphSet(
+        name=f"{gs.name}x{R}", words=np.concatenate(words), node_word_off=np.concatenate(offs),
+        node_t=np.concatenate(nts), func_id=np.concatenate(fids), allocs=np.concatenate(allocs),
+        new_base=np.concatenate(new_base), new_size=np.tile(gs.new_size, R), table=np.tile(gs.table, R),
+        func_kind=np.tile(gs.func_kind, R), tags=np.concatenate(tags), truth_id=np.concatenate(tid),
+        truth_off=np.concatenate(toff), node_model=np.tile(gs.node_model, R), node_bs=np.tile(gs.node_bs, R),
+        node_perm=np.tile(gs.node_perm, R), alloc_kind=np.tile(gs.alloc_kind, R), models=gs.models * R)
