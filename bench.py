@@ -112,6 +112,21 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(rows), "samples_under_load": len(loaded)}
 
 
+def rank_seed(cfg, rank):
+    """Seed of the independent instance rank `rank` restores (weak scaling)."""
+    from workloads.graphset import CONFIGS
+    return CONFIGS[cfg]["seed"] + SEED_STRIDE * rank
+
+
+def max_over_ranks(x, dist, device):
+    """Max of a per-rank scalar over all ranks (the job's time is the slowest rank's)."""
+    import torch
+    t = torch.tensor([float(x)], dtype=torch.float64, device=device)
+    if dist is not None and dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     return int(os.environ.get("RANK", "0")), ws, int(os.environ.get("LOCAL_RANK", "0"))
@@ -162,8 +177,6 @@ def run_ours(args):
     ge.build_medusa()
     import paper_conf_asplos_zengxgcl25_b200 as medusa
     from workloads import make_graph_set
-    from workloads.graphset import CONFIGS
-
     rank, ws, local = dist_env()
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a GPU (there is no CPU fallback)")
@@ -173,7 +186,7 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
 
     cfg, desc = WORKLOADS[args.workload]
-    seed = CONFIGS[cfg]["seed"] + SEED_STRIDE * rank
+    seed = rank_seed(cfg, rank)
     gs = make_graph_set(cfg, seed=seed)
     inp = medusa.upload(gs, dev)
     stream = torch.cuda.current_stream(dev)
@@ -228,10 +241,7 @@ def run_ours(args):
     medusa.timing_enable(False)
     clocks = sampler.stop()
     total_ms = sum(step_ms)
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-    if ws > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    max_ms = float(t.item())
+    max_ms = max_over_ranks(total_ms, dist, dev)
     nodes_total = gs.n_nodes * args.steps * ws
     value = nodes_total / (max_ms / 1e3)
 
@@ -335,10 +345,7 @@ def run_ours(args):
         e2e_ev[k][1].record(stream)
     barrier()
     e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_ev)
-    t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
-    if ws > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    e2e_value = nodes_total / (float(t.item()) / 1e3)
+    e2e_value = nodes_total / (max_over_ranks(e2e_ms, dist, dev) / 1e3)
     assert np.array_equal(out_h.numpy().view(np.uint64), medusa.to_numpy_u64(dst))
 
     # ---- CPU baseline: the oracle as it stands, rank 0 at N=1 only ----
