@@ -185,6 +185,39 @@ __device__ __forceinline__ uint32_t gallop_alloc_ge(const medusa_alloc* al, uint
     return l;
 }
 
+// count of entries <= x in the ascending u32 array t[0, n) (warp-cooperative
+// 32-ary search: ~4 dependent global rounds for 10^5 entries; all lanes agree)
+__device__ __forceinline__ uint32_t warp_count_le(const uint32_t* t, uint32_t n, uint32_t x) {
+    const uint32_t lane = threadIdx.x & 31;
+    uint32_t lo = 0, hi = n;  // the count lies in [lo, hi]
+    while (hi - lo > 32) {
+        const uint32_t step = (hi - lo + 31) / 32;
+        const uint32_t pr = lo + lane * step;
+        const bool le = pr < hi && t[pr] <= x;
+        const uint32_t b = __ballot_sync(0xffffffffu, le);
+        const uint32_t k = __popc(b);  // probes <= x form a prefix
+        if (k == 0) return lo;
+        const uint32_t last_le = lo + (k - 1) * step;
+        const uint32_t next = lo + k * step;
+        lo = last_le + 1;
+        if (next < hi) hi = next;
+    }
+    const uint32_t pr = lo + lane;
+    return lo + __popc(__ballot_sync(0xffffffffu, pr < hi && t[pr] <= x));
+}
+
+// atomicAdd(&ctr[key], 1) for every active lane, one atomic per distinct key in the
+// warp; returns the previous value + this lane's rank among the lanes with its key
+__device__ __forceinline__ uint32_t warp_agg_inc(uint32_t* ctr, uint32_t key, bool active) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t peers = __match_any_sync(0xffffffffu, active ? key : 0xFFFFFFFFu);
+    const uint32_t leader = __ffs(peers) - 1;
+    uint32_t base = 0;
+    if (active && lane == leader) base = atomicAdd(ctr + key, (uint32_t)__popc(peers));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    return base + __popc(peers & lanemask_lt());
+}
+
 // ----------------------------------------------------------------------------
 // 1. k_trace
 __device__ void nodes_role(const P& p, uint64_t i) {
@@ -210,9 +243,15 @@ __device__ void nodes_role(const P& p, uint64_t i) {
     }
 }
 
+constexpr int kTWin = 2048;  // node times / allocation times staged per alloc CTA
+
 __device__ void allocs_role(const P& p, uint32_t cta) {
     __shared__ uint32_t s_last;
-    const uint32_t i = cta * blockDim.x + threadIdx.x;
+    __shared__ uint32_t s_nt[kTWin];  // node_t[nj0, nj0 + nw)
+    __shared__ uint32_t s_at[kTWin];  // t_alloc of allocations [i0, i0 + na)
+    __shared__ uint32_t s_nj0;
+    const uint32_t i0 = cta * blockDim.x;
+    const uint32_t i = i0 + threadIdx.x;
     const MaterializeArgs& a = p.a;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t N = a.n_nodes;
@@ -220,8 +259,22 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     medusa_alloc x{};
     if (valid) x = a.alloc[i];
     const uint32_t t_last = N ? a.node_t[N - 1] : 0;
+    // the node times around this CTA's allocations, and the allocation times after them
+    if (threadIdx.x < 32) {
+        const uint32_t ta0 = a.alloc[i0].t_alloc;
+        const uint32_t nj0 = N ? warp_count_le(a.node_t, N, ta0) : 0;
+        if (lane == 0) s_nj0 = nj0;
+    }
+    __syncthreads();
+    const uint32_t nj0 = s_nj0;
+    const uint32_t nw = min((uint32_t)kTWin, N - nj0);
+    const uint32_t na = (uint32_t)min((uint64_t)kTWin, (uint64_t)a.n_alloc - i0);
+    for (uint32_t k = threadIdx.x; k < nw; k += blockDim.x) s_nt[k] = a.node_t[nj0 + k];
+    for (uint32_t k = threadIdx.x; k < na; k += blockDim.x) s_at[k] = a.alloc[i0 + k].t_alloc;
+    __syncthreads();
     bool isI = false;
     uint4 r = make_uint4(1, 0, 1, 0);  // empty ranges
+    bool reg_c = false, reg_b = false;
     if (valid) {
         if (x.size > (1ull << MEDUSA_OFF_BITS) || x.base + x.size < x.base) flag(p.d.ctl, ST_INVALID);
         if (!(x.t_alloc < x.t_free)) flag(p.d.ctl, ST_TRACE);
@@ -231,29 +284,57 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
             if (!isI) {
                 if (p.C && N && x.t_alloc < x.t_free) {
                     // nodes launched while i is live: [j0, j1) = t in (t_alloc, t_free)
-                    uint32_t lo = 0, hi = N;
-                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (a.node_t[m] <= x.t_alloc) lo = m + 1; else hi = m; }
-                    const uint32_t j0 = lo;
-                    const uint32_t j1 = gallop_ge(a.node_t, j0, N, x.t_free);
+                    uint32_t lo = 0, hi = nw;  // window entries <= t_alloc
+                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (s_nt[m] <= x.t_alloc) lo = m + 1; else hi = m; }
+                    uint32_t j0;
+                    if (lo < nw) {
+                        j0 = nj0 + lo;
+                    } else {  // beyond the staged window (or the trace is not ordered)
+                        uint32_t l2 = nj0 + nw, h2 = N;
+                        while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (a.node_t[m] <= x.t_alloc) l2 = m + 1; else h2 = m; }
+                        j0 = l2;
+                    }
+                    uint32_t j1;
+                    if (j0 < nj0 + nw && nw && x.t_free <= s_nt[nw - 1]) {
+                        uint32_t l2 = j0 - nj0, h2 = nw;  // first entry >= t_free
+                        while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (s_nt[m] < x.t_free) l2 = m + 1; else h2 = m; }
+                        j1 = nj0 + l2;
+                    } else {
+                        j1 = gallop_ge(a.node_t, max(j0, nj0 + nw), N, x.t_free);
+                    }
                     // chunks holding their words (exact: no entry for memory no launch can see)
                     if (j0 < j1) {
                         const uint64_t w0 = a.node_off[j0], w1 = a.node_off[j1];
                         if (w0 < w1 && w1 <= a.n_words) {
                             r.x = (uint32_t)(w0 / kChunkWords);
                             r.y = (uint32_t)((w1 - 1) / kChunkWords);
-                            for (uint32_t c = r.x; c <= r.y; ++c) atomicAdd(&p.d.cnt_c[c], 1u);
+                            reg_c = true;
                         }
                     }
                 }
                 // ordinals allocated while i is live: (i, u), u = #{k : t_alloc_k < t_free_i}
-                const uint32_t u = gallop_alloc_ge(a.alloc, i + 1, a.n_alloc, x.t_free);
+                uint32_t u;
+                if (na && x.t_free <= s_at[na - 1]) {
+                    uint32_t l2 = i - i0 + 1, h2 = na;
+                    while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (s_at[m] < x.t_free) l2 = m + 1; else h2 = m; }
+                    u = i0 + l2;
+                } else {
+                    u = gallop_alloc_ge(a.alloc, max(i + 1, i0 + na), a.n_alloc, x.t_free);
+                }
                 if (i + 1 < u) {
                     r.z = (i + 1) / kAblk; r.w = (u - 1) / kAblk;
-                    for (uint32_t b = r.z; b <= r.w; ++b) atomicAdd(&p.d.cnt_b[b], 1u);
+                    reg_b = true;
                 }
             }
         }
         p.d.rng[i] = r;
+    }
+    // registration counts, one atomic per distinct chunk / block of the warp
+    {
+        const uint32_t lc = reg_c ? r.y - r.x + 1 : 0, lb = reg_b ? r.w - r.z + 1 : 0;
+        const uint32_t mc = __reduce_max_sync(0xffffffffu, lc), mbk = __reduce_max_sync(0xffffffffu, lb);
+        for (uint32_t k = 0; k < mc; ++k) warp_agg_inc(p.d.cnt_c, r.x + k, k < lc);
+        for (uint32_t k = 0; k < mbk; ++k) warp_agg_inc(p.d.cnt_b, r.z + k, k < lb);
     }
     // warp-aggregated: I positions, global prefilter bounds
     const uint32_t bal = __ballot_sync(0xffffffffu, isI);
@@ -419,18 +500,34 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
 }
 
 __device__ void scatter_role(const P& p, uint32_t i) {
-    if (i >= p.a.n_alloc) return;
-    const uint4 r = p.d.rng[i];
-    if (r.x > r.y && r.z > r.w) return;
-    const medusa_alloc x = p.a.alloc[i];
-    const WinRec w{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
-    for (uint32_t c = r.x; c <= r.y; ++c) {
-        const uint64_t pos = (uint64_t)p.d.off_c[c] + atomicAdd(&p.d.fill_c[c], 1u);
-        if (pos < p.d.cap_c) p.d.list_c[pos] = w;
+    const bool valid = i < p.a.n_alloc;
+    uint4 r = make_uint4(1, 0, 1, 0);
+    if (valid) r = p.d.rng[i];
+    const uint32_t lc = r.x <= r.y ? r.y - r.x + 1 : 0, lb = r.z <= r.w ? r.w - r.z + 1 : 0;
+    const uint32_t mc = __reduce_max_sync(0xffffffffu, lc), mbk = __reduce_max_sync(0xffffffffu, lb);
+    if ((mc | mbk) == 0) return;  // whole warp
+    WinRec w{};
+    if (lc | lb) {
+        const medusa_alloc x = p.a.alloc[i];
+        w = WinRec{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
     }
-    for (uint32_t b = r.z; b <= r.w; ++b) {
-        const uint64_t pos = (uint64_t)p.d.off_b[b] + atomicAdd(&p.d.fill_b[b], 1u);
-        if (pos < p.d.cap_b) p.d.list_b[pos] = w;
+    for (uint32_t k = 0; k < mc; ++k) {
+        const bool act = k < lc;
+        const uint32_t c = r.x + k;
+        const uint32_t rank = warp_agg_inc(p.d.fill_c, act ? c : 0, act);
+        if (act) {
+            const uint64_t pos = (uint64_t)p.d.off_c[c] + rank;
+            if (pos < p.d.cap_c) p.d.list_c[pos] = w;
+        }
+    }
+    for (uint32_t k = 0; k < mbk; ++k) {
+        const bool act = k < lb;
+        const uint32_t b = r.z + k;
+        const uint32_t rank = warp_agg_inc(p.d.fill_b, act ? b : 0, act);
+        if (act) {
+            const uint64_t pos = (uint64_t)p.d.off_b[b] + rank;
+            if (pos < p.d.cap_b) p.d.list_b[pos] = w;
+        }
     }
 }
 
@@ -829,10 +926,10 @@ __global__ void __launch_bounds__(kThreads) k_scan_words(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 5. k_emit: compaction of the staged records into the slot table (one CTA per chunk)
+// 5. k_emit: compaction of the staged records into the slot table (one CTA per
+//    chunk, one thread per output record: coalesced stores)
 __global__ void __launch_bounds__(kThreads) k_emit(P p) {
-    __shared__ uint32_t s_mask[64];
-    __shared__ uint32_t s_pre[64];
+    __shared__ uint32_t s_pre[65];
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t c = blockIdx.x;
@@ -841,9 +938,7 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     const uint64_t prefix = a.chunk_base[c];
     if (warp < 2) {
         const uint64_t mw = m0 + warp * 32 + lane;
-        const uint32_t bits = mw < n_mask ? a.mask[mw] : 0u;
-        s_mask[warp * 32 + lane] = bits;
-        const uint32_t pc = __popc(bits);
+        const uint32_t pc = mw < n_mask ? __popc(a.mask[mw]) : 0u;
         uint32_t incl = pc;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
@@ -851,18 +946,18 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
             if (lane >= d) incl += y;
         }
         s_pre[warp * 32 + lane] = incl - pc;
+        if (warp == 0 && lane == 31) s_pre[64] = incl;  // first-half total
     }
     __syncthreads();
-    if (tid < 32) s_pre[32 + tid] += s_pre[31] + __popc(s_mask[31]);  // second half after the first
+    const uint32_t half0 = s_pre[64];
+    if (tid >= 32 && tid < 64) s_pre[tid] += half0;  // second half after the first
     __syncthreads();
-#pragma unroll
-    for (int g = 0; g < 8; ++g) {
-        const uint32_t local = warp * 8 + g;
-        const uint32_t bits = s_mask[local];
-        if (lane < (uint32_t)__popc(bits)) {
-            const uint64_t dst = prefix + s_pre[local] + lane;
-            if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + local) * 32 + lane];
-        }
+    const uint32_t total = (uint32_t)(a.chunk_base[c + 1] - prefix);
+    for (uint32_t r = tid; r < total; r += kThreads) {
+        uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
+        while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
+        const uint64_t dst = prefix + r;
+        if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + (r - s_pre[lo])];
     }
 }
 
