@@ -136,34 +136,53 @@ __device__ __forceinline__ uint32_t fence_stride(uint32_t nI) { return nI ? (nI 
 
 // Exclusive scan of cnt[0..n) into off[0..n] (off[n] = total) by one CTA of any
 // size <= 1024 (multiple of 32); reads through L2 (values written by other CTAs).
+// Tiles of 16 consecutive values per thread are loaded with independent loads
+// (one round trip per tile of 16*blockDim values), scanned in registers.
 __device__ void block_exclusive_scan(const uint32_t* cnt, uint32_t* off, uint32_t n, unsigned long long* total) {
     __shared__ unsigned long long s_w[32];
+    constexpr int V = 16;
     const uint32_t T = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t per = (n + T - 1) / T;
-    const uint32_t b = min(tid * per, n), e = min(b + per, n);
-    unsigned long long s = 0;
-    for (uint32_t k = b; k < e; ++k) s += __ldcg(cnt + k);
-    unsigned long long incl = s;
+    unsigned long long carry = 0;
+    for (uint32_t base = 0; base < n || base == 0; base += V * T) {
+        uint32_t v[V];
+        const uint32_t b = base + tid * V;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, d);
-        if (lane >= d) incl += y;
-    }
-    if (lane == 31) s_w[warp] = incl;
-    __syncthreads();
-    if (warp == 0) {
-        unsigned long long v = lane < T / 32 ? s_w[lane] : 0, iv = v;
+        for (int k = 0; k < V; ++k) v[k] = (b + k < n) ? __ldcg(cnt + b + k) : 0u;
+        unsigned long long s = 0;
+#pragma unroll
+        for (int k = 0; k < V; ++k) s += v[k];
+        unsigned long long incl = s;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
-            const unsigned long long y = __shfl_up_sync(0xffffffffu, iv, d);
-            if (lane >= d) iv += y;
+            const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += y;
         }
-        s_w[lane] = iv - v;  // exclusive prefix of warp totals
+        if (lane == 31) s_w[warp] = incl;
+        __syncthreads();
+        unsigned long long tile_total = 0;
+        if (warp == 0) {
+            unsigned long long wv = lane < T / 32 ? s_w[lane] : 0, iv = wv;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const unsigned long long y = __shfl_up_sync(0xffffffffu, iv, d);
+                if (lane >= d) iv += y;
+            }
+            s_w[lane] = iv - wv;  // exclusive prefix of warp totals
+        }
+        __syncthreads();
+        unsigned long long run = carry + s_w[warp] + incl - s;
+#pragma unroll
+        for (int k = 0; k < V; ++k)
+            if (b + k < n) { off[b + k] = (uint32_t)min(run, 0xFFFFFFFFull); run += v[k]; }
+        // the tile's total = the last thread's inclusive value
+        if (tid == T - 1) s_w[0] = run - carry;
+        __syncthreads();
+        tile_total = s_w[0];
+        __syncthreads();
+        carry += tile_total;
+        if (base + V * T >= n) break;
     }
-    __syncthreads();
-    unsigned long long run = s_w[warp] + incl - s;
-    for (uint32_t k = b; k < e; ++k) { off[k] = (uint32_t)min(run, 0xFFFFFFFFull); run += __ldcg(cnt + k); }
-    if (tid == T - 1) { *total = run; off[n] = (uint32_t)min(run, 0xFFFFFFFFull); }
+    if (tid == 0) { *total = carry; off[n] = (uint32_t)min(carry, 0xFFFFFFFFull); }
     __syncthreads();
 }
 
@@ -539,25 +558,34 @@ __global__ void __launch_bounds__(kThreads) k_prepare(P p) {
 
 // ----------------------------------------------------------------------------
 // 3. k_rank: rank = index in own tile + count of keys below it in every other
-//    tile; the thread adding the last contribution writes the entry in place
+//    tile.  CTA (t, kb) stages sorted tile t in shared memory and counts, for the
+//    2048 keys of tile kb (kb != t), how many of tile t's keys are below; the
+//    thread adding a key's last contribution writes its I entry in place.
 __global__ void __launch_bounds__(kThreads) k_rank(P p) {
+    __shared__ uint64_t sk[kSortTile];
+    __shared__ uint32_t sv[kSortTile];
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t T = n_tiles(nI);
     if (T <= 1) return;
-    const uint64_t pairs = (uint64_t)nI * T;
-    const uint64_t* sk = p.d.sk[1];
-    const uint32_t* sv = p.d.sv[1];
-    for (uint64_t q = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; q < pairs; q += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t t = (uint32_t)(q / nI), k = (uint32_t)(q % nI);
-        if (t == k / kSortTile) continue;
-        const uint64_t kk = sk[k];
-        const uint32_t vk = sv[k];
-        uint32_t lo = t * kSortTile, hi = min(lo + kSortTile, nI);
-        const uint32_t base = lo;
-        while (lo < hi) { const uint32_t m = (lo + hi) >> 1; if (kv_less(sk[m], sv[m], kk, vk)) lo = m + 1; else hi = m; }
-        const uint32_t cnt = lo - base;
-        const unsigned long long old = atomicAdd(&p.d.rank[k], (1ull << 32) | cnt);
-        if ((old >> 32) + 1 == T - 1) write_i_entry(p, (uint32_t)old + cnt, nI, vk);
+    const uint64_t* gk = p.d.sk[1];
+    const uint32_t* gv = p.d.sv[1];
+    for (uint64_t job = blockIdx.x; job < (uint64_t)T * T; job += gridDim.x) {
+        const uint32_t t = (uint32_t)(job / T), kb = (uint32_t)(job % T);
+        if (t == kb) continue;
+        const uint32_t t0 = t * kSortTile, tn = min((uint32_t)kSortTile, nI - t0);
+        __syncthreads();
+        for (uint32_t q = threadIdx.x; q < tn; q += blockDim.x) { sk[q] = gk[t0 + q]; sv[q] = gv[t0 + q]; }
+        __syncthreads();
+        const uint32_t k0 = kb * kSortTile, kn = min((uint32_t)kSortTile, nI - k0);
+        for (uint32_t q = threadIdx.x; q < kn; q += blockDim.x) {
+            const uint32_t k = k0 + q;
+            const uint64_t kk = gk[k];
+            const uint32_t vk = gv[k];
+            uint32_t lo = 0, hi = tn;
+            while (lo < hi) { const uint32_t m = (lo + hi) >> 1; if (kv_less(sk[m], sv[m], kk, vk)) lo = m + 1; else hi = m; }
+            const unsigned long long old = atomicAdd(&p.d.rank[k], (1ull << 32) | lo);
+            if ((old >> 32) + 1 == T - 1) write_i_entry(p, (uint32_t)old + lo, nI, vk);
+        }
     }
 }
 
@@ -1071,8 +1099,8 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
                 k_prepare<<<sort_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
             }
             TimedLaunch tl("mat_rank", stream);
-            const uint64_t pairs = n * (uint64_t)sort_ctas;
-            const unsigned grid = (unsigned)std::min<uint64_t>((pairs + kThreads - 1) / kThreads, (uint64_t)s.sm_count * 8);
+            const uint64_t jobs = (uint64_t)sort_ctas * sort_ctas;
+            const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(jobs, (uint64_t)s.sm_count * 4));
             k_rank<<<grid, kThreads, 0, stream>>>(p);
         }
         if (C + check_ctas) {
