@@ -50,7 +50,10 @@ typedef enum {
     MEDUSA_ERR_CAPACITY = -3,    /* slot table too small; *h_n_slots holds the size needed */
     MEDUSA_ERR_NO_TABLE = -4,    /* restore asked for the kernel-address fill before any
                                     medusa_kernel_table_set on this device */
-    MEDUSA_ERR_CUDA = -5         /* CUDA runtime error; see medusa_last_cuda_error() */
+    MEDUSA_ERR_CUDA = -5,        /* CUDA runtime error; see medusa_last_cuda_error() */
+    MEDUSA_ERR_RETRY = -6        /* (medusa_materialize_async result only) the library's
+                                    scratch was too small for this trace: call
+                                    medusa_materialize once, which sizes it exactly */
 } medusa_status;
 
 /* One allocation of the trace, 24 bytes.  Its index in the trace array is the
@@ -148,6 +151,34 @@ medusa_status medusa_materialize(const uint64_t *d_words, uint64_t n_words,
                                  medusa_slots *slots, uint64_t *h_n_slots,
                                  cudaStream_t stream);
 
+/* Result of medusa_materialize_async, written to device memory (16 bytes):
+ * status = one of medusa_status (OK, INVALID_ARG, TRACE, CAPACITY, RETRY),
+ * n_slots as *h_n_slots of medusa_materialize. */
+typedef struct {
+    int32_t status;
+    uint32_t reserved;
+    uint64_t n_slots;
+} medusa_mat_result;
+
+/* medusa_materialize_async -- the same analysis as medusa_materialize, fully
+ * asynchronous on `stream` (no host synchronization; capturable into a CUDA
+ * graph once the library's scratch has been sized by one medusa_materialize
+ * call on this device for a trace of the same or larger size).  The data-
+ * dependent outcome goes to *d_result (device); host-detectable argument errors
+ * are returned synchronously.  If d_result->status is not MEDUSA_OK, the table
+ * and anything computed from it are unspecified.  Calls on one device must be
+ * ordered (one stream, or events): they share the device's scratch. */
+medusa_status medusa_materialize_async(const uint64_t *d_words, uint64_t n_words,
+                                       const uint64_t *d_node_word_off, uint32_t n_nodes,
+                                       const uint32_t *d_node_t,
+                                       const medusa_alloc *d_alloc, uint32_t n_alloc,
+                                       medusa_slots *slots, medusa_mat_result *d_result,
+                                       cudaStream_t stream);
+
+/* n_slots value for medusa_restore: take the slot count from the table itself
+ * (d_chunk_base), e.g. after medusa_materialize_async with no host round trip. */
+#define MEDUSA_N_SLOTS_FROM_TABLE UINT64_MAX
+
 /* medusa_kernel_table_set -- install, for the current device, the kernel
  * address of every kernel-name id: d_func_addr[n_func] (device),
  * 0 = unresolved.  In the paper these come from dlsym / cudaGetFuncBySymbol and,
@@ -175,7 +206,7 @@ medusa_status medusa_kernel_table_set(const uint64_t *d_func_addr, uint32_t n_fu
  *
  * src/dst: u64[n_words], device; dst == src (in place) is allowed, any other
  * overlap is MEDUSA_ERR_INVALID_ARG.  slots: as produced by medusa_materialize
- * for this image (n_slots = *h_n_slots).  d_old_base: the trace's base of each
+ * for this image (n_slots = *h_n_slots, or MEDUSA_N_SLOTS_FROM_TABLE).  d_old_base: the trace's base of each
  * allocation (the materialization-time addresses).  d_report (device) is
  * written completely by the call.  Fully asynchronous on `stream`; capturable
  * into a CUDA graph.                                                         */

@@ -17,7 +17,8 @@ import torch
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libmedusa.so")
 
-OK, ERR_INVALID_ARG, ERR_TRACE, ERR_CAPACITY, ERR_NO_TABLE, ERR_CUDA = 0, -1, -2, -3, -4, -5
+OK, ERR_INVALID_ARG, ERR_TRACE, ERR_CAPACITY, ERR_NO_TABLE, ERR_CUDA, ERR_RETRY = 0, -1, -2, -3, -4, -5, -6
+N_SLOTS_FROM_TABLE = (1 << 64) - 1
 CHUNK_WORDS = 2048
 OFF_BITS = 40
 T_END = 0xFFFFFFFF
@@ -54,6 +55,8 @@ def lib():
         L.medusa_materialize.argtypes = [P, U64, P, U32, P, P, U32, ctypes.POINTER(_Slots),
                                          ctypes.POINTER(U64), P]
         L.medusa_materialize.restype = I
+        L.medusa_materialize_async.argtypes = [P, U64, P, U32, P, P, U32, ctypes.POINTER(_Slots), P, P]
+        L.medusa_materialize_async.restype = I
         L.medusa_kernel_table_set.argtypes = [P, U32, P]
         L.medusa_kernel_table_set.restype = I
         L.medusa_restore.argtypes = [P, P, U64, ctypes.POINTER(_Slots), U64, P, P, P, U32, P, P, U32, P, P]
@@ -126,6 +129,26 @@ def materialize(words, node_off, node_t, allocs, stream=None, capacity=None, out
     return slots
 
 
+def materialize_async(words, node_off, node_t, allocs, out, result, stream=None):
+    """medusa_materialize_async: enqueue only.  `result` = int64[2] device tensor that
+    receives {status (low 32 bits of [0]), n_slots ([1])}; `out` = a Slots sized for
+    this image (its n_slots is not updated -- read `result` or restore with
+    from_table=True)."""
+    cs = out.c_struct()
+    st = lib().medusa_materialize_async(_ptr(words), words.numel(), _ptr(node_off), node_t.numel(), _ptr(node_t),
+                                        _ptr(allocs), allocs.shape[0] if allocs.dim() else 0, ctypes.byref(cs),
+                                        _ptr(result), _stream(stream))
+    if st != OK:
+        raise MedusaError(st, "medusa_materialize_async")
+    return out
+
+
+def mat_result(result):
+    """(status, n_slots) from a materialize_async result tensor (synchronizes)."""
+    r = result.detach().cpu().numpy()
+    return int(np.int32(r[0] & 0xFFFFFFFF)), int(r[1])
+
+
 def kernel_table_set(table, stream=None):
     """medusa_kernel_table_set.  table: int64[K] device tensor of kernel addresses (0 = unresolved)."""
     st = lib().medusa_kernel_table_set(_ptr(table), table.numel(), _stream(stream))
@@ -134,9 +157,10 @@ def kernel_table_set(table, stream=None):
 
 
 def restore(src, slots, old_base, new_base, new_size, func_id=None, dst=None, func_out=None, report=None,
-            stream=None):
+            stream=None, from_table=False):
     """medusa_restore -> (dst int64[n_words], func_out int64[N] or None, report int64[8]).
-    dst may be src (in place)."""
+    dst may be src (in place).  from_table: slot count taken from the table itself
+    (MEDUSA_N_SLOTS_FROM_TABLE), e.g. after materialize_async."""
     dev = src.device
     if dst is None:
         dst = torch.empty_like(src)
@@ -145,7 +169,8 @@ def restore(src, slots, old_base, new_base, new_size, func_id=None, dst=None, fu
     if report is None:
         report = torch.empty(8, dtype=torch.int64, device=dev)
     cs = slots.c_struct()
-    st = lib().medusa_restore(_ptr(src), _ptr(dst), src.numel(), ctypes.byref(cs), slots.n_slots, _ptr(old_base),
+    n_slots = N_SLOTS_FROM_TABLE if from_table else slots.n_slots
+    st = lib().medusa_restore(_ptr(src), _ptr(dst), src.numel(), ctypes.byref(cs), n_slots, _ptr(old_base),
                               _ptr(new_base), _ptr(new_size), new_base.numel(), _ptr(func_id), _ptr(func_out),
                               func_id.numel() if func_id is not None else 0, _ptr(report), _stream(stream))
     if st != OK:

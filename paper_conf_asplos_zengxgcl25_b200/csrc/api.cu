@@ -67,6 +67,7 @@ const char* medusa_status_string(medusa_status s) {
         case MEDUSA_ERR_CAPACITY: return "MEDUSA_ERR_CAPACITY";
         case MEDUSA_ERR_NO_TABLE: return "MEDUSA_ERR_NO_TABLE";
         case MEDUSA_ERR_CUDA: return "MEDUSA_ERR_CUDA";
+        case MEDUSA_ERR_RETRY: return "MEDUSA_ERR_RETRY";
     }
     return "MEDUSA_UNKNOWN_STATUS";
 }
@@ -91,12 +92,10 @@ int medusa_timing_read(const char** names, float* ms, int max) {
     return n;
 }
 
-medusa_status medusa_materialize(const uint64_t* d_words, uint64_t n_words,
-                                 const uint64_t* d_node_word_off, uint32_t n_nodes,
-                                 const uint32_t* d_node_t, const medusa_alloc* d_alloc, uint32_t n_alloc,
-                                 medusa_slots* slots, uint64_t* h_n_slots, cudaStream_t stream) {
-    if (h_n_slots) *h_n_slots = 0;
-    if (!h_n_slots || !slots || !d_node_word_off || !slots->d_chunk_base) return MEDUSA_ERR_INVALID_ARG;
+static medusa_status materialize_args(const uint64_t* d_words, uint64_t n_words, const uint64_t* d_node_word_off,
+                                      uint32_t n_nodes, const uint32_t* d_node_t, const medusa_alloc* d_alloc,
+                                      uint32_t n_alloc, const medusa_slots* slots) {
+    if (!slots || !d_node_word_off || !slots->d_chunk_base) return MEDUSA_ERR_INVALID_ARG;
     if (n_words > 0 && (!d_words || !slots->d_mask)) return MEDUSA_ERR_INVALID_ARG;
     if (n_nodes > 0 && !d_node_t) return MEDUSA_ERR_INVALID_ARG;
     if (n_alloc > 0 && !d_alloc) return MEDUSA_ERR_INVALID_ARG;
@@ -104,10 +103,36 @@ medusa_status medusa_materialize(const uint64_t* d_words, uint64_t n_words,
     if (n_alloc > (1u << MEDUSA_ID_BITS) || n_words > 0xFFFFFFFFull) return MEDUSA_ERR_INVALID_ARG;
     if (!aligned8(d_words) || !aligned8(d_node_word_off) || !aligned8(d_alloc) || !aligned8(slots->d_slot))
         return MEDUSA_ERR_INVALID_ARG;
+    return MEDUSA_OK;
+}
+
+medusa_status medusa_materialize(const uint64_t* d_words, uint64_t n_words,
+                                 const uint64_t* d_node_word_off, uint32_t n_nodes,
+                                 const uint32_t* d_node_t, const medusa_alloc* d_alloc, uint32_t n_alloc,
+                                 medusa_slots* slots, uint64_t* h_n_slots, cudaStream_t stream) {
+    if (h_n_slots) *h_n_slots = 0;
+    if (!h_n_slots) return MEDUSA_ERR_INVALID_ARG;
+    medusa_status st = materialize_args(d_words, n_words, d_node_word_off, n_nodes, d_node_t, d_alloc, n_alloc, slots);
+    if (st != MEDUSA_OK) return st;
     MaterializeArgs a{d_words, n_words, d_node_word_off, n_nodes, d_node_t, d_alloc, n_alloc,
                       slots->d_mask, slots->d_chunk_base, slots->d_slot, slots->capacity};
     cudaError_t ce = cudaSuccess;
-    medusa_status st = run_materialize(a, h_n_slots, stream, &ce);
+    st = run_materialize(a, h_n_slots, stream, &ce);
+    if (st == MEDUSA_ERR_CUDA) g_last_cuda_error = (int)ce;
+    return st;
+}
+
+medusa_status medusa_materialize_async(const uint64_t* d_words, uint64_t n_words,
+                                       const uint64_t* d_node_word_off, uint32_t n_nodes,
+                                       const uint32_t* d_node_t, const medusa_alloc* d_alloc, uint32_t n_alloc,
+                                       medusa_slots* slots, medusa_mat_result* d_result, cudaStream_t stream) {
+    if (!d_result || !aligned8(d_result)) return MEDUSA_ERR_INVALID_ARG;
+    medusa_status st = materialize_args(d_words, n_words, d_node_word_off, n_nodes, d_node_t, d_alloc, n_alloc, slots);
+    if (st != MEDUSA_OK) return st;
+    MaterializeArgs a{d_words, n_words, d_node_word_off, n_nodes, d_node_t, d_alloc, n_alloc,
+                      slots->d_mask, slots->d_chunk_base, slots->d_slot, slots->capacity};
+    cudaError_t ce = cudaSuccess;
+    st = run_materialize_async(a, d_result, stream, &ce);
     if (st == MEDUSA_ERR_CUDA) g_last_cuda_error = (int)ce;
     return st;
 }
@@ -145,7 +170,8 @@ medusa_status medusa_restore(const uint64_t* d_src_words, uint64_t* d_dst_words,
                              const uint32_t* d_func_id, uint64_t* d_func_out, uint32_t n_nodes,
                              medusa_report* d_report, cudaStream_t stream) {
     if (!d_report || !slots || !aligned8(d_report)) return MEDUSA_ERR_INVALID_ARG;
-    if (n_words > 0xFFFFFFFFull || n_slots > n_words) return MEDUSA_ERR_INVALID_ARG;
+    const bool from_table = n_slots == MEDUSA_N_SLOTS_FROM_TABLE;
+    if (n_words > 0xFFFFFFFFull || (!from_table && n_slots > n_words)) return MEDUSA_ERR_INVALID_ARG;
     if (n_words > 0) {
         if (!d_src_words || !d_dst_words || !slots->d_mask || !slots->d_chunk_base) return MEDUSA_ERR_INVALID_ARG;
         if (!aligned8(d_src_words) || !aligned8(d_dst_words)) return MEDUSA_ERR_INVALID_ARG;
@@ -153,6 +179,7 @@ medusa_status medusa_restore(const uint64_t* d_src_words, uint64_t* d_dst_words,
         const uintptr_t bytes = (uintptr_t)n_words * 8;
         if (s != d && s < d + bytes && d < s + bytes) return MEDUSA_ERR_INVALID_ARG;  // partial overlap
     }
+    if (from_table) n_slots = slots->capacity;  // bound only: the table's chunk prefix gives the ranges
     if (n_slots > 0 && (!slots->d_slot || !aligned8(slots->d_slot))) return MEDUSA_ERR_INVALID_ARG;
     if (n_alloc > 0 && (!d_old_base || !d_new_base || !d_new_size)) return MEDUSA_ERR_INVALID_ARG;
     const bool gather = d_func_id || d_func_out || n_nodes;

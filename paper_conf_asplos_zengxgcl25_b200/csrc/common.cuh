@@ -87,5 +87,8 @@ struct MaterializeArgs {
 // status; *n_slots = slots found (0 on INVALID_ARG / TRACE).
 medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaStream_t stream,
                               cudaError_t* cuda_err);
+// Enqueues the analysis only; the outcome is written to *d_result.
+medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
+                                    cudaError_t* cuda_err);
 
 }  // namespace medusa

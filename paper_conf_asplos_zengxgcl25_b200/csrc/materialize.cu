@@ -53,6 +53,7 @@ constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
 constexpr int kSortTile = 2048;    // keys sorted per CTA before ranking
+constexpr int kRankKeys = 256;     // keys ranked per k_rank job (one per thread)
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
 constexpr int kWinCap = 128;       // mortal-window entries per batch (<= 4 per lane of one warp)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
@@ -237,6 +238,13 @@ __device__ __forceinline__ uint32_t warp_agg_inc(uint32_t* ctr, uint32_t key, bo
     return base + __popc(peers & lanemask_lt());
 }
 
+// ctr[key] += 1 for every active lane, one fire-and-forget atomic per distinct key
+__device__ __forceinline__ void warp_agg_add(uint32_t* ctr, uint32_t key, bool active) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t peers = __match_any_sync(0xffffffffu, active ? key : 0xFFFFFFFFu);
+    if (active && lane == __ffs(peers) - 1) atomicAdd(ctr + key, (uint32_t)__popc(peers));
+}
+
 // ----------------------------------------------------------------------------
 // 1. k_trace
 __device__ void nodes_role(const P& p, uint64_t i) {
@@ -352,8 +360,8 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     {
         const uint32_t lc = reg_c ? r.y - r.x + 1 : 0, lb = reg_b ? r.w - r.z + 1 : 0;
         const uint32_t mc = __reduce_max_sync(0xffffffffu, lc), mbk = __reduce_max_sync(0xffffffffu, lb);
-        for (uint32_t k = 0; k < mc; ++k) warp_agg_inc(p.d.cnt_c, r.x + k, k < lc);
-        for (uint32_t k = 0; k < mbk; ++k) warp_agg_inc(p.d.cnt_b, r.z + k, k < lb);
+        for (uint32_t k = 0; k < mc; ++k) warp_agg_add(p.d.cnt_c, r.x + k, k < lc);
+        for (uint32_t k = 0; k < mbk; ++k) warp_agg_add(p.d.cnt_b, r.z + k, k < lb);
     }
     // warp-aggregated: I positions, global prefilter bounds
     const uint32_t bal = __ballot_sync(0xffffffffu, isI);
@@ -569,14 +577,15 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
     if (T <= 1) return;
     const uint64_t* gk = p.d.sk[1];
     const uint32_t* gv = p.d.sv[1];
-    for (uint64_t job = blockIdx.x; job < (uint64_t)T * T; job += gridDim.x) {
-        const uint32_t t = (uint32_t)(job / T), kb = (uint32_t)(job % T);
-        if (t == kb) continue;
+    const uint32_t KB = (nI + kRankKeys - 1) / kRankKeys;  // key blocks of kRankKeys
+    for (uint64_t job = blockIdx.x; job < (uint64_t)T * KB; job += gridDim.x) {
+        const uint32_t t = (uint32_t)(job / KB), kb = (uint32_t)(job % KB);
+        if (t == kb * kRankKeys / kSortTile) continue;  // a key block lies inside one tile
         const uint32_t t0 = t * kSortTile, tn = min((uint32_t)kSortTile, nI - t0);
         __syncthreads();
         for (uint32_t q = threadIdx.x; q < tn; q += blockDim.x) { sk[q] = gk[t0 + q]; sv[q] = gv[t0 + q]; }
         __syncthreads();
-        const uint32_t k0 = kb * kSortTile, kn = min((uint32_t)kSortTile, nI - k0);
+        const uint32_t k0 = kb * kRankKeys, kn = min((uint32_t)kRankKeys, nI - k0);
         for (uint32_t q = threadIdx.x; q < kn; q += blockDim.x) {
             const uint32_t k = k0 + q;
             const uint64_t kk = gk[k];
@@ -989,6 +998,19 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     }
 }
 
+// 6. k_result (async entry): the outcome as a medusa_mat_result
+__global__ void k_result(P p, medusa_mat_result* r) {
+    const Ctl& c = *p.d.ctl;
+    int32_t st = MEDUSA_OK;
+    if (c.status & ST_INVALID) st = MEDUSA_ERR_INVALID_ARG;
+    else if (c.status & ST_TRACE) st = MEDUSA_ERR_TRACE;
+    else if (c.status & ST_OVERFLOW) st = MEDUSA_ERR_RETRY;
+    else if (c.n_slots > p.a.capacity) st = MEDUSA_ERR_CAPACITY;
+    r->status = st;
+    r->reserved = 0;
+    r->n_slots = (st == MEDUSA_OK || st == MEDUSA_ERR_CAPACITY) ? c.n_slots : 0;
+}
+
 // ----------------------------------------------------------------------------
 // host side: per-device scratch, launches
 struct Scratch {
@@ -1060,22 +1082,26 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
 
 }  // namespace
 
-medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaStream_t stream,
-                              cudaError_t* cuda_err) {
-    *n_slots = 0;
+namespace {
+
+Scratch* device_scratch(cudaError_t* e) {
     int dev = 0;
-    cudaError_t e = cudaGetDevice(&dev);
-    if (e != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-    std::lock_guard<std::mutex> lk(g_mu);
+    *e = cudaGetDevice(&dev);
+    if (*e != cudaSuccess) return nullptr;
     if ((int)g_scratch.size() <= dev) g_scratch.resize(dev + 1, nullptr);
     if (!g_scratch[dev]) g_scratch[dev] = new Scratch();
     Scratch& s = *g_scratch[dev];
-    const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
     if (!s.h_ctl) {
-        if ((e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+        if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
+        const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
         cudaFuncSetAttribute(k_scan_words, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem);
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
+    return &s;
+}
+
+// the whole analysis on `stream` (no synchronization)
+cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P* out) {
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
     const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
@@ -1083,35 +1109,55 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     const uint32_t alloc_ctas = (uint32_t)((n + kThreads - 1) / kThreads);
     const uint32_t sort_ctas = (uint32_t)((n + kSortTile - 1) / kSortTile);
     const uint32_t check_ctas = n ? std::max<uint32_t>((nb + kWarps - 1) / kWarps, alloc_ctas) : 0;
+    const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
+    P p{a, s.d, C, nb, node_ctas, sort_ctas, check_ctas};
+    *out = p;
+    cudaError_t e;
+    if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) return e;
+    if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) return e;
+    {
+        TimedLaunch tl("mat_trace", stream);
+        k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
+    }
+    if (n) {
+        {
+            TimedLaunch tl("mat_prepare", stream);
+            k_prepare<<<sort_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
+        }
+        TimedLaunch tl("mat_rank", stream);
+        const uint64_t jobs = (uint64_t)sort_ctas * ((n + kRankKeys - 1) / kRankKeys);
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(jobs, (uint64_t)s.sm_count * 8));
+        k_rank<<<grid, kThreads, 0, stream>>>(p);
+    }
+    if (C + check_ctas) {
+        TimedLaunch tl("mat_classify", stream);
+        k_scan_words<<<C + check_ctas, kThreads, scan_smem, stream>>>(p);
+    }
+    if (C) {
+        TimedLaunch tl("mat_emit", stream);
+        k_emit<<<C, kThreads, 0, stream>>>(p);
+    }
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaStream_t stream,
+                              cudaError_t* cuda_err) {
+    *n_slots = 0;
+    cudaError_t e;
+    std::lock_guard<std::mutex> lk(g_mu);
+    Scratch* sp = device_scratch(&e);
+    if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    Scratch& s = *sp;
+    const uint64_t n = a.n_alloc;
+    const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
+    const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
     size_t need_c = 0, need_b = 0;
     for (int attempt = 0; attempt < 3; ++attempt) {
         if ((e = ensure(s, n, C, nb, a.n_words, need_c, need_b)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-        P p{a, s.d, C, nb, node_ctas, sort_ctas, check_ctas};
-        if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) break;
-        if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) break;
-        {
-            TimedLaunch tl("mat_trace", stream);
-            k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
-        }
-        if (n) {
-            {
-                TimedLaunch tl("mat_prepare", stream);
-                k_prepare<<<sort_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
-            }
-            TimedLaunch tl("mat_rank", stream);
-            const uint64_t jobs = (uint64_t)sort_ctas * sort_ctas;
-            const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(jobs, (uint64_t)s.sm_count * 4));
-            k_rank<<<grid, kThreads, 0, stream>>>(p);
-        }
-        if (C + check_ctas) {
-            TimedLaunch tl("mat_classify", stream);
-            k_scan_words<<<C + check_ctas, kThreads, scan_smem, stream>>>(p);
-        }
-        if (C) {
-            TimedLaunch tl("mat_emit", stream);
-            k_emit<<<C, kThreads, 0, stream>>>(p);
-        }
-        if ((e = cudaGetLastError()) != cudaSuccess) break;
+        P p;
+        if ((e = enqueue(s, a, stream, &p)) != cudaSuccess) break;
         if ((e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess) break;
         if ((e = cudaStreamSynchronize(stream)) != cudaSuccess) break;
         const Ctl h = *s.h_ctl;
@@ -1128,6 +1174,25 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     if (e != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     *cuda_err = cudaErrorUnknown;
     return MEDUSA_ERR_CUDA;
+}
+
+medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
+                                    cudaError_t* cuda_err) {
+    cudaError_t e;
+    std::lock_guard<std::mutex> lk(g_mu);
+    Scratch* sp = device_scratch(&e);
+    if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    Scratch& s = *sp;
+    const uint64_t n = a.n_alloc;
+    const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
+    const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
+    // never (re)allocates while the caller may be capturing a graph, unless it must grow
+    if ((e = ensure(s, n, C, nb, a.n_words, 0, 0)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    P p;
+    if ((e = enqueue(s, a, stream, &p)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    k_result<<<1, 1, 0, stream>>>(p, d_result);
+    if ((e = cudaGetLastError()) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    return MEDUSA_OK;
 }
 
 }  // namespace medusa

@@ -241,3 +241,75 @@ def test_replicated_multi_instance_parity(graph_sets):
     assert np.array_equal(medusa.to_numpy_u64(dst), packed[3])
     assert np.array_equal(medusa.to_numpy_u64(fout), packed[4])
     assert np.array_equal(medusa.report_numpy(rep), packed[5])
+
+
+@pytest.mark.parametrize("name", ["toy", "all10"])
+def test_async_graph_path_parity(graph_sets, name):
+    """medusa_materialize_async -> kernel_table_set -> restore(MEDUSA_N_SLOTS_FROM_TABLE),
+    captured once into a CUDA graph and replayed (the bench's timed step), against the oracle."""
+    gs = graph_sets(name)
+    inp = medusa.upload(gs, DEV)
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size,
+                             gs.func_id, gs.table)
+    slots = medusa.alloc_slots(gs.n_words, DEV)
+    res = torch.full((2,), -7, dtype=torch.int64, device=DEV)
+    dst = torch.empty_like(inp["words"])
+    fout = torch.empty(gs.n_nodes, dtype=torch.int64, device=DEV)
+    rep = torch.empty(8, dtype=torch.int64, device=DEV)
+
+    def step():
+        medusa.materialize_async(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots, result=res)
+        medusa.kernel_table_set(inp["table"])
+        medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                       dst=dst, func_out=fout, report=rep, from_table=True)
+
+    # eager async first (also sizes the library's scratch outside capture)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        step()
+    torch.cuda.synchronize()
+    assert medusa.mat_result(res) == (0, m["n_slots"])
+    slots.n_slots = m["n_slots"]
+    _check_materialize(slots, m, packed, gs.n_words)
+    assert np.array_equal(medusa.to_numpy_u64(dst), packed[3])
+
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        step()
+    for _ in range(2):
+        dst.zero_()
+        fout.zero_()
+        res.fill_(-7)
+        slots.slot.fill_(-1)
+        g.replay()
+        torch.cuda.synchronize()
+        assert medusa.mat_result(res) == (0, m["n_slots"])
+        _check_materialize(slots, m, packed, gs.n_words)
+        assert np.array_equal(medusa.to_numpy_u64(dst), packed[3])
+        assert np.array_equal(medusa.to_numpy_u64(fout), packed[4])
+        assert np.array_equal(medusa.report_numpy(rep), packed[5])
+
+
+def test_async_reports_trace_error_and_capacity():
+    """The async entry point reports what the synchronous one raises, in the result word."""
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(DEV)
+    res = torch.zeros(2, dtype=torch.int64, device=DEV)
+    seen_bad = seen_cap = False
+    for seed in range(60):
+        words, off, node_t, allocs = tiny_trace(seed * 11 + 3, overlap_p=0.2)
+        o = oracle.materialize(words, off, node_t, allocs)
+        aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3) if allocs.size else np.zeros((0, 3), np.int64)
+        inp = dict(words=t(words, np.int64), node_off=t(off, np.int64), node_t=t(node_t, np.int32),
+                   allocs=torch.from_numpy(aa).to(DEV))
+        medusa.materialize_async(**inp, out=medusa.alloc_slots(words.size, DEV), result=res)
+        st, n = medusa.mat_result(res)
+        assert st == o["status"], seed
+        if st != 0:
+            seen_bad = True
+            continue
+        assert n == o["n_slots"], seed
+        if n > 0:
+            medusa.materialize_async(**inp, out=medusa.alloc_slots(words.size, DEV, capacity=n - 1), result=res)
+            assert medusa.mat_result(res) == (medusa.ERR_CAPACITY, n), seed
+            seen_cap = True
+    assert seen_bad and seen_cap
