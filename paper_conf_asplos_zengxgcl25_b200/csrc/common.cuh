@@ -2,6 +2,7 @@
 #pragma once
 
 #include <cstdint>
+#include <utility>
 #include <cuda_runtime.h>
 
 #include "medusa.h"
@@ -36,6 +37,33 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
     return m;
 }
 
+// ---- programmatic dependent launch (PDL) --------------------------------------
+// Kernels after the first of a call are launched with programmatic stream
+// serialization: a grid may start while its predecessor drains.  Every kernel
+// executes pdl_wait() (full completion + memory flush of the predecessor) before
+// it touches anything the predecessor writes, and pdl_trigger() only after its
+// own pdl_wait(), so "my predecessor has triggered" implies "everything before my
+// predecessor is complete": a kernel may read the outputs of kernels two or more
+// launches back before it waits.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned block, size_t smem,
+                              cudaStream_t stream, Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
 // ---- instrumentation (api.cu) -------------------------------------------------
 // Brackets one launch with events when the calling thread enabled timing.
 struct TimedLaunch {
@@ -45,6 +73,43 @@ struct TimedLaunch {
     cudaStream_t stream;
     void* slot;
 };
+
+// ---- timeline instrumentation (diagnostic builds only: -DMEDUSA_TIMELINE) ------
+// Thread 0 of a CTA appends {start, end, kernel, cta, sm, tag} to a per-TU device
+// buffer (tools/timeline.py builds libmedusa_tl.so and reads it back).
+#ifdef MEDUSA_TIMELINE
+struct TlRec {
+    unsigned long long t0, t1;
+    unsigned int kernel, cta, sm, tag;
+};
+__device__ __forceinline__ unsigned long long tl_now() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+#define MEDUSA_TL_DEFINE                                                                         \
+    __device__ TlRec* g_tl = nullptr;                                                            \
+    __device__ unsigned int g_tl_n = 0, g_tl_cap = 0;                                            \
+    __device__ __forceinline__ void tl_rec(unsigned k, unsigned tag, unsigned long long t0) {    \
+        if (threadIdx.x != 0 || !g_tl) return;                                                   \
+        const unsigned i = atomicAdd(&g_tl_n, 1u);                                               \
+        unsigned sm;                                                                             \
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));                                          \
+        if (i < g_tl_cap) g_tl[i] = TlRec{t0, tl_now(), k, blockIdx.x, sm, tag};                 \
+    }
+#define TL_NOW() tl_now()
+#define TL_REC(k, tag, t0) tl_rec((k), (tag), (t0))
+#else
+#pragma nv_diag_suppress 550  // timeline stamps are set but unused without MEDUSA_TIMELINE
+#define MEDUSA_TL_DEFINE
+#define TL_NOW() 0ull
+#define TL_REC(k, tag, t0) ((void)(t0))
+#endif
+#define TL_PHASE(k, tag, var) \
+    do {                      \
+        TL_REC(k, tag, var);  \
+        var = TL_NOW();       \
+    } while (0)
 
 // ---- restore (restore.cu) ------------------------------------------------------
 struct RestoreArgs {

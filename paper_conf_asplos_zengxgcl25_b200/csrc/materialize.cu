@@ -48,6 +48,8 @@
 namespace medusa {
 namespace {
 
+MEDUSA_TL_DEFINE
+
 constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
@@ -59,15 +61,16 @@ constexpr int kWinCap = 128;       // mortal-window entries per batch (<= 4 per 
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
 constexpr int kWarps = kThreads / 32;
 constexpr int kIBlk = 32;          // I-list summary block
+constexpr int kNodeGrp = 128;      // nodes per live-mask group (a chunk holds ~90 nodes in the BASELINE sets)
 
 struct Ctl {
     unsigned int status;
     unsigned int nI;
-    unsigned int done_allocs;
-    unsigned int done_cls;
+    unsigned int pad0;
+    unsigned int pad1;
     unsigned long long gmin_c;  // ~(least base) via atomicMax
     unsigned long long gmax;    // greatest end
-    unsigned long long need_c, need_b;
+    unsigned long long need_c, need_b;  // set (exactly) only when a registration list overflowed
     unsigned long long n_slots;
 };
 
@@ -90,8 +93,13 @@ struct Dev {  // scratch of one call (device pointers)
     Ctl* ctl;
     uint32_t *jf, *jl;                           // [C] first / last node of each chunk
     uint4* rng;                                  // [n]: c_lo, c_hi, b_lo, b_hi
-    uint32_t *cnt_c, *fill_c, *off_c;            // [C+1] (zeroed)
-    uint32_t *cnt_b, *fill_b, *off_b;            // [nb+1] (zeroed)
+    // two-level registration counters (zeroed): cnt[k] per chunk / check block,
+    // sup[g] = sum of cnt over the 256 keys of group g, so any prefix sum is one
+    // CTA-wide reduction (block_prefix) and no serial scan is needed
+    uint32_t *cnt_c, *fill_c;                    // [C+1]
+    uint32_t *cnt_b, *fill_b;                    // [nb+1]
+    unsigned long long *sup_c, *sup_b;           // [C/256+1], [nb/256+1]
+    unsigned long long* chunk_sup;               // [C/256+1] slots per 256 chunks
     uint32_t *blk_min_ta_c, *blk_max_tf;         // [n/32+1] (zeroed; min kept as ~max(~t))
     WinRec *list_c, *list_b;
     uint64_t cap_c, cap_b;
@@ -102,7 +110,7 @@ struct Dev {  // scratch of one call (device pointers)
     IRest* i_rest;                               // [n]
     uint32_t* i_tf;                              // [n]
     uint64_t* fence;                             // [kFenceCap]
-    uint32_t* chunk_cnt;                         // [C]
+    uint32_t* chunk_cnt;                         // [C] slots per chunk
     uint64_t* staging;                           // [n_words] records, warp-dense per 32 words
 };
 
@@ -135,56 +143,53 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
 __device__ __forceinline__ uint32_t n_tiles(uint32_t nI) { return (nI + kSortTile - 1) / kSortTile; }
 __device__ __forceinline__ uint32_t fence_stride(uint32_t nI) { return nI ? (nI + kFenceCap - 1) / kFenceCap : 1; }
 
-// Exclusive scan of cnt[0..n) into off[0..n] (off[n] = total) by one CTA of any
-// size <= 1024 (multiple of 32); reads through L2 (values written by other CTAs).
-// Tiles of 16 consecutive values per thread are loaded with independent loads
-// (one round trip per tile of 16*blockDim values), scanned in registers.
-__device__ void block_exclusive_scan(const uint32_t* cnt, uint32_t* off, uint32_t n, unsigned long long* total) {
-    __shared__ unsigned long long s_w[32];
-    constexpr int V = 16;
-    const uint32_t T = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    unsigned long long carry = 0;
-    for (uint32_t base = 0; base < n || base == 0; base += V * T) {
-        uint32_t v[V];
-        const uint32_t b = base + tid * V;
+// Exclusive scan of one value per thread over the CTA (blockDim.x == kThreads);
+// *total = the sum.  Call with the whole CTA.
+__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* total) {
+    __shared__ uint32_t s_w[kWarps];
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t x = v;
 #pragma unroll
-        for (int k = 0; k < V; ++k) v[k] = (b + k < n) ? __ldcg(cnt + b + k) : 0u;
-        unsigned long long s = 0;
-#pragma unroll
-        for (int k = 0; k < V; ++k) s += v[k];
-        unsigned long long incl = s;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const unsigned long long y = __shfl_up_sync(0xffffffffu, incl, d);
-            if (lane >= d) incl += y;
-        }
-        if (lane == 31) s_w[warp] = incl;
-        __syncthreads();
-        unsigned long long tile_total = 0;
-        if (warp == 0) {
-            unsigned long long wv = lane < T / 32 ? s_w[lane] : 0, iv = wv;
-#pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const unsigned long long y = __shfl_up_sync(0xffffffffu, iv, d);
-                if (lane >= d) iv += y;
-            }
-            s_w[lane] = iv - wv;  // exclusive prefix of warp totals
-        }
-        __syncthreads();
-        unsigned long long run = carry + s_w[warp] + incl - s;
-#pragma unroll
-        for (int k = 0; k < V; ++k)
-            if (b + k < n) { off[b + k] = (uint32_t)min(run, 0xFFFFFFFFull); run += v[k]; }
-        // the tile's total = the last thread's inclusive value
-        if (tid == T - 1) s_w[0] = run - carry;
-        __syncthreads();
-        tile_total = s_w[0];
-        __syncthreads();
-        carry += tile_total;
-        if (base + V * T >= n) break;
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= (uint32_t)d) x += y;
     }
-    if (tid == 0) { *total = carry; off[n] = (uint32_t)min(carry, 0xFFFFFFFFull); }
+    if (lane == 31) s_w[warp] = x;
     __syncthreads();
+    uint32_t before = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) {
+        const uint32_t t = s_w[w];
+        if ((uint32_t)w < warp) before += t;
+        tot += t;
+    }
+    __syncthreads();  // s_w may be rewritten by the next call
+    *total = tot;
+    return before + x - v;
+}
+
+// Sum of cnt[0, k) of a two-level counter (sup[g] = sum of cnt[256g, 256g + 256)):
+// at most k/256 + 255 loads, spread over the CTA, and one reduction; every thread
+// receives the value.  Call with the whole CTA (blockDim.x == kThreads == 256).
+static_assert(kThreads == 256, "block_prefix covers one 256-key group per pass");
+__device__ __forceinline__ unsigned long long block_prefix(const uint32_t* cnt, const unsigned long long* sup,
+                                                           uint32_t k) {
+    __shared__ unsigned long long s_r[kWarps];
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t g = k >> 8;
+    unsigned long long acc = 0;
+    for (uint32_t q = threadIdx.x; q < g; q += kThreads) acc += __ldcg(sup + q);
+    const uint32_t j = (g << 8) + threadIdx.x;
+    if (j < k) acc += __ldcg(cnt + j);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, d);
+    if (lane == 0) s_r[warp] = acc;
+    __syncthreads();
+    unsigned long long t = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) t += s_r[w];
+    __syncthreads();
+    return t;
 }
 
 // first index k in [lo, n) with t[k] >= x (galloping from lo; t ascending)
@@ -245,6 +250,26 @@ __device__ __forceinline__ void warp_agg_add(uint32_t* ctr, uint32_t key, bool a
     if (active && lane == __ffs(peers) - 1) atomicAdd(ctr + key, (uint32_t)__popc(peers));
 }
 
+// sup[g] += |[lo, hi] ∩ group g| for every 256-key group g the active lanes'
+// ranges meet; one atomic per distinct group of the warp (full-warp call)
+__device__ __forceinline__ void warp_group_add_range(unsigned long long* sup, uint32_t lo, uint32_t hi, bool active) {
+    const uint32_t g0 = active ? lo >> 8 : 0, g1 = active ? hi >> 8 : 0;
+    const uint32_t ng = __reduce_max_sync(0xffffffffu, active ? g1 - g0 + 1 : 0u);
+    for (uint32_t k = 0; k < ng; ++k) {
+        const uint32_t g = g0 + k;
+        const bool act = active && g <= g1;
+        const uint32_t n = act ? min(hi, g * 256 + 255) - max(lo, g * 256) + 1 : 0u;
+        uint32_t key = act ? g : 0xFFFFFFFFu;
+        while (true) {
+            const uint32_t gm = __reduce_min_sync(0xffffffffu, key);
+            if (gm == 0xFFFFFFFFu) break;
+            const uint32_t sum = __reduce_add_sync(0xffffffffu, key == gm ? n : 0u);
+            if ((threadIdx.x & 31) == 0) atomicAdd(sup + gm, (unsigned long long)sum);
+            if (key == gm) key = 0xFFFFFFFFu;
+        }
+    }
+}
+
 // ----------------------------------------------------------------------------
 // 1. k_trace
 __device__ void nodes_role(const P& p, uint64_t i) {
@@ -273,7 +298,6 @@ __device__ void nodes_role(const P& p, uint64_t i) {
 constexpr int kTWin = 2048;  // node times / allocation times staged per alloc CTA
 
 __device__ void allocs_role(const P& p, uint32_t cta) {
-    __shared__ uint32_t s_last;
     __shared__ uint32_t s_nt[kTWin];  // node_t[nj0, nj0 + nw)
     __shared__ uint32_t s_at[kTWin];  // t_alloc of allocations [i0, i0 + na)
     __shared__ uint32_t s_nj0;
@@ -283,6 +307,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t N = a.n_nodes;
     const bool valid = i < a.n_alloc;
+    unsigned long long tl_p = TL_NOW();
     medusa_alloc x{};
     if (valid) x = a.alloc[i];
     const uint32_t t_last = N ? a.node_t[N - 1] : 0;
@@ -293,12 +318,14 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         if (lane == 0) s_nj0 = nj0;
     }
     __syncthreads();
+    TL_PHASE(1, 20, tl_p);  // record load, node-window start
     const uint32_t nj0 = s_nj0;
     const uint32_t nw = min((uint32_t)kTWin, N - nj0);
     const uint32_t na = (uint32_t)min((uint64_t)kTWin, (uint64_t)a.n_alloc - i0);
     for (uint32_t k = threadIdx.x; k < nw; k += blockDim.x) s_nt[k] = a.node_t[nj0 + k];
     for (uint32_t k = threadIdx.x; k < na; k += blockDim.x) s_at[k] = a.alloc[i0 + k].t_alloc;
     __syncthreads();
+    TL_PHASE(1, 21, tl_p);  // time windows staged
     bool isI = false;
     uint4 r = make_uint4(1, 0, 1, 0);  // empty ranges
     bool reg_c = false, reg_b = false;
@@ -356,12 +383,15 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         }
         p.d.rng[i] = r;
     }
-    // registration counts, one atomic per distinct chunk / block of the warp
+    // registration counts (one atomic per distinct key of the warp) and their
+    // 256-key group sums
     {
         const uint32_t lc = reg_c ? r.y - r.x + 1 : 0, lb = reg_b ? r.w - r.z + 1 : 0;
         const uint32_t mc = __reduce_max_sync(0xffffffffu, lc), mbk = __reduce_max_sync(0xffffffffu, lb);
         for (uint32_t k = 0; k < mc; ++k) warp_agg_add(p.d.cnt_c, r.x + k, k < lc);
         for (uint32_t k = 0; k < mbk; ++k) warp_agg_add(p.d.cnt_b, r.z + k, k < lb);
+        warp_group_add_range(p.d.sup_c, r.x, r.y, reg_c);
+        warp_group_add_range(p.d.sup_b, r.z, r.w, reg_b);
     }
     // warp-aggregated: I positions, global prefilter bounds
     const uint32_t bal = __ballot_sync(0xffffffffu, isI);
@@ -380,26 +410,20 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         atomicMax(&p.d.ctl->gmin_c, ~(unsigned long long)mn);
         atomicMax(&p.d.ctl->gmax, (unsigned long long)mx);
     }
-    // the last alloc CTA turns the registration counts into offsets
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        const uint32_t alloc_ctas = (a.n_alloc + blockDim.x - 1) / blockDim.x;
-        s_last = atomicAdd(&p.d.ctl->done_allocs, 1u) == alloc_ctas - 1;
-    }
-    __syncthreads();
-    if (s_last) {
-        __threadfence();
-        block_exclusive_scan(p.d.cnt_c, p.d.off_c, p.C, &p.d.ctl->need_c);
-        block_exclusive_scan(p.d.cnt_b, p.d.off_b, p.nb, &p.d.ctl->need_b);
-        if (threadIdx.x == 0 && (p.d.ctl->need_c > p.d.cap_c || p.d.ctl->need_b > p.d.cap_b))
-            flag(p.d.ctl, ST_OVERFLOW);
-    }
+    TL_PHASE(1, 22, tl_p);  // searches, registration counts, I compaction
 }
 
-__global__ void __launch_bounds__(kThreads) k_trace(P p) {
-    if (blockIdx.x < p.node_ctas) nodes_role(p, (uint64_t)blockIdx.x * blockDim.x + threadIdx.x);
-    else allocs_role(p, blockIdx.x - p.node_ctas);
+__global__ void __launch_bounds__(kThreads, 4) k_trace(P p) {
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
+    if (blockIdx.x < p.node_ctas) {
+        nodes_role(p, (uint64_t)blockIdx.x * blockDim.x + threadIdx.x);
+        TL_REC(1, 0, tl0);
+    } else {
+        allocs_role(p, blockIdx.x - p.node_ctas);
+        TL_REC(1, 1, tl0);
+    }
+    pdl_trigger();
 }
 
 // ----------------------------------------------------------------------------
@@ -476,6 +500,7 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
     const uint32_t t0 = tile * kSortTile;
     if (t0 >= n) return;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    unsigned long long tl_p = TL_NOW();
     uint64_t k[8];
     uint32_t v[8], pl[8];
 #pragma unroll
@@ -492,6 +517,7 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
         S.sv[0][warp * 256 + lane * 8 + r] = v[r];
     }
     __syncthreads();
+    TL_PHASE(2, 30, tl_p);  // load + warp bitonic
     int src = 0;
 #pragma unroll
     for (uint32_t run = 256; run < kSortTile; run <<= 1) {
@@ -514,6 +540,7 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
         src ^= 1;
         __syncthreads();
     }
+    TL_PHASE(2, 31, tl_p);  // shared-memory merges
     const bool single = n <= kSortTile;  // one tile: its order is final
     for (uint32_t q = tid; q < kSortTile && t0 + q < n; q += blockDim.x) {
         if (single) {
@@ -526,42 +553,109 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
     }
 }
 
-__device__ void scatter_role(const P& p, uint32_t i) {
-    const bool valid = i < p.a.n_alloc;
-    uint4 r = make_uint4(1, 0, 1, 0);
-    if (valid) r = p.d.rng[i];
-    const uint32_t lc = r.x <= r.y ? r.y - r.x + 1 : 0, lb = r.z <= r.w ? r.w - r.z + 1 : 0;
-    const uint32_t mc = __reduce_max_sync(0xffffffffu, lc), mbk = __reduce_max_sync(0xffffffffu, lb);
-    if ((mc | mbk) == 0) return;  // whole warp
-    WinRec w{};
-    if (lc | lb) {
-        const medusa_alloc x = p.a.alloc[i];
-        w = WinRec{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
+// One registration list (chunks or check blocks): the CTA's 256 allocations
+// register in keys [lo_i, hi_i] (empty when lo_i > hi_i).  Keys are handled in
+// tiles of 256: a tile's list offsets = block_prefix + a CTA scan of the counts;
+// the tile's (allocation, key) pairs are dealt out evenly over the CTA, so one
+// long-lived allocation does not serialize its warp.
+__device__ void scatter_list(const P& p, const uint32_t* cnt, const unsigned long long* sup, uint32_t* fill,
+                             WinRec* list, uint64_t cap, unsigned long long* need, uint32_t lo_i, uint32_t hi_i,
+                             const WinRec& w, uint32_t* s_off, uint32_t* s_pre, uint32_t* s_first, WinRec* s_w,
+                             uint32_t* s_range) {
+    const uint32_t tid = threadIdx.x;
+    const bool has = lo_i <= hi_i;
+    if (tid == 0) { s_range[0] = 0xFFFFFFFFu; s_range[1] = 0; }
+    __syncthreads();
+    {
+        const uint32_t mn = __reduce_min_sync(0xffffffffu, has ? lo_i : 0xFFFFFFFFu);
+        const uint32_t mx = __reduce_max_sync(0xffffffffu, has ? hi_i : 0u);
+        if ((tid & 31) == 0 && mn <= mx) { atomicMin(&s_range[0], mn); atomicMax(&s_range[1], mx); }
     }
-    for (uint32_t k = 0; k < mc; ++k) {
-        const bool act = k < lc;
-        const uint32_t c = r.x + k;
-        const uint32_t rank = warp_agg_inc(p.d.fill_c, act ? c : 0, act);
-        if (act) {
-            const uint64_t pos = (uint64_t)p.d.off_c[c] + rank;
-            if (pos < p.d.cap_c) p.d.list_c[pos] = w;
+    s_w[tid] = w;
+    __syncthreads();
+    const uint32_t lo = s_range[0], hi = s_range[1];
+    if (lo > hi) return;  // whole CTA
+    unsigned long long base = block_prefix(cnt, sup, lo);
+    for (uint32_t t0 = lo; t0 <= hi; t0 += kThreads) {
+        // list offset of every key of the tile
+        const uint32_t key = t0 + tid;
+        uint32_t tile_total;
+        const uint32_t ex = block_excl_scan(key <= hi ? __ldcg(cnt + key) : 0u, &tile_total);
+        s_off[tid] = (uint32_t)min(base + ex, 0xFFFFFFFFull);
+        base += tile_total;
+        // this thread's pairs inside the tile, dealt out over the CTA
+        const uint32_t a = max(lo_i, t0), b = min(hi_i, t0 + kThreads - 1);
+        const uint32_t len = (has && a <= b && a <= hi_i) ? b - a + 1 : 0u;
+        uint32_t n_pairs;
+        const uint32_t pre = block_excl_scan(len, &n_pairs);
+        s_pre[tid] = pre;
+        s_first[tid] = a;
+        __syncthreads();
+        for (uint32_t q0 = 0; q0 < n_pairs; q0 += kThreads) {
+            const uint32_t q = q0 + tid;
+            const bool act = q < n_pairs;
+            uint32_t own = 0, k = 0;
+            if (act) {  // owner: last thread whose pair range starts at or before q
+                uint32_t l = 0, h = kThreads;
+                while (h - l > 1) { const uint32_t m = (l + h) >> 1; if (s_pre[m] <= q) l = m; else h = m; }
+                own = l;
+                k = s_first[own] + (q - s_pre[own]);
+            }
+            const uint32_t rank = warp_agg_inc(fill, act ? k : 0, act);
+            if (act) {
+                const uint64_t pos = (uint64_t)s_off[k - t0] + rank;
+                if (pos < cap) {
+                    list[pos] = s_w[own];
+                } else {
+                    atomicMax(need, (unsigned long long)pos + 1);
+                    flag(p.d.ctl, ST_OVERFLOW);
+                }
+            }
         }
-    }
-    for (uint32_t k = 0; k < mbk; ++k) {
-        const bool act = k < lb;
-        const uint32_t b = r.z + k;
-        const uint32_t rank = warp_agg_inc(p.d.fill_b, act ? b : 0, act);
-        if (act) {
-            const uint64_t pos = (uint64_t)p.d.off_b[b] + rank;
-            if (pos < p.d.cap_b) p.d.list_b[pos] = w;
-        }
+        __syncthreads();  // s_off / s_pre / s_first are rewritten by the next tile
     }
 }
 
+struct ScatterShared {
+    uint32_t off[kThreads], pre[kThreads], first[kThreads], range[2];
+    WinRec w[kThreads];
+};
+
+__device__ void scatter_role(const P& p, uint32_t cta, ScatterShared& S) {
+    const uint32_t i = cta * kThreads + threadIdx.x;
+    const bool valid = i < p.a.n_alloc;
+    uint4 r = make_uint4(1, 0, 1, 0);
+    if (valid) r = p.d.rng[i];
+    WinRec w{};
+    if (r.x <= r.y || r.z <= r.w) {
+        const medusa_alloc x = p.a.alloc[i];
+        w = WinRec{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
+    }
+    scatter_list(p, p.d.cnt_c, p.d.sup_c, p.d.fill_c, p.d.list_c, p.d.cap_c, &p.d.ctl->need_c, r.x, r.y, w, S.off,
+                 S.pre, S.first, S.w, S.range);
+    __syncthreads();
+    scatter_list(p, p.d.cnt_b, p.d.sup_b, p.d.fill_b, p.d.list_b, p.d.cap_b, &p.d.ctl->need_b, r.z, r.w, w, S.off,
+                 S.pre, S.first, S.w, S.range);
+}
+
+union PrepShared {
+    SortShared sort;
+    ScatterShared scatter;
+};
+
 __global__ void __launch_bounds__(kThreads) k_prepare(P p) {
-    __shared__ SortShared S;
-    if (blockIdx.x < p.sort_ctas) sort_role(p, blockIdx.x, S);
-    else scatter_role(p, (blockIdx.x - p.sort_ctas) * blockDim.x + threadIdx.x);
+    extern __shared__ __align__(16) unsigned char prep_raw[];
+    PrepShared& U = *reinterpret_cast<PrepShared*>(prep_raw);
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
+    if (blockIdx.x < p.sort_ctas) {
+        sort_role(p, blockIdx.x, U.sort);
+        TL_REC(2, 0, tl0);
+    } else {
+        scatter_role(p, blockIdx.x - p.sort_ctas, U.scatter);
+        TL_REC(2, 1, tl0);
+    }
+    pdl_trigger();
 }
 
 // ----------------------------------------------------------------------------
@@ -572,6 +666,8 @@ __global__ void __launch_bounds__(kThreads) k_prepare(P p) {
 __global__ void __launch_bounds__(kThreads) k_rank(P p) {
     __shared__ uint64_t sk[kSortTile];
     __shared__ uint32_t sv[kSortTile];
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t T = n_tiles(nI);
     if (T <= 1) return;
@@ -596,6 +692,8 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
             if ((old >> 32) + 1 == T - 1) write_i_entry(p, (uint32_t)old + lo, nI, vk);
         }
     }
+    pdl_trigger();
+    TL_REC(3, 0, tl0);
 }
 
 // count of sorted I bases <= x (fences in shared memory, then one group of <= stride
@@ -623,13 +721,16 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     uint64_t fence[kFenceCap];
-    uint32_t tw[MEDUSA_CHUNK_WORDS];     // launch position of every word
-    uint64_t wb[kWinCap], we[kWinCap], wpmax[kWinCap];  // window sorted by (base, t_alloc)
+    uint32_t tw[MEDUSA_CHUNK_WORDS];     // node of every word, as an index from the chunk's first node
+    uint64_t wb[kWinCap], we[kWinCap];   // window sorted by (base, t_alloc)
     uint32_t wta[kWinCap], wtf[kWinCap], wid[kWinCap];
+    uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
+    uint32_t nt[kNodeGrp];                  // launch positions of nodes g0 .. g0 + kNodeGrp
+    uint32_t gnext;
     uint16_t cq[MEDUSA_CHUNK_WORDS];     // candidate words, then the I-list queue
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32];
     uint32_t wmax[kWarps];
-    uint32_t nc, nq, total, last;
+    uint32_t nc, nq, total;
     unsigned long long mbar;
 };
 
@@ -644,7 +745,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
 }
 
 // warp 0: a batch of <= kWinCap registered mortals sorted by (base, t_alloc) in
-// registers, laid out in shared memory, with the prefix max of end
+// registers, laid out in shared memory
 template <int E>
 __device__ __forceinline__ void window_prepare_e(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
     const uint32_t lane = threadIdx.x & 31;
@@ -664,11 +765,9 @@ __device__ __forceinline__ void window_prepare_e(const P& p, ClsShared& S, uint6
         pl[r] = e;
     }
     warp_bitonic<E>(k, v, pl);
-    uint64_t ends[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
         const uint32_t e = lane * E + r;
-        ends[r] = 0;
         if (e < m) {
             const WinRec x = p.d.list_c[bs + pl[r]];
             S.wb[e] = x.base;
@@ -676,24 +775,7 @@ __device__ __forceinline__ void window_prepare_e(const P& p, ClsShared& S, uint6
             S.wta[e] = x.t_alloc;
             S.wtf[e] = x.t_free;
             S.wid[e] = x.id;
-            ends[r] = x.end;
         }
-    }
-    uint64_t run = 0;
-#pragma unroll
-    for (int r = 0; r < E; ++r) { run = max(run, ends[r]); ends[r] = run; }
-    uint64_t incl = run;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint64_t y = __shfl_up_sync(0xffffffffu, incl, d);
-        if (lane >= d) incl = max(incl, y);
-    }
-    uint64_t before = __shfl_up_sync(0xffffffffu, incl, 1);
-    if (lane == 0) before = 0;
-#pragma unroll
-    for (int r = 0; r < E; ++r) {
-        const uint32_t e = lane * E + r;
-        if (e < m) S.wpmax[e] = max(before, ends[r]);
     }
 }
 
@@ -707,6 +789,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     Ctl* ctl = p.d.ctl;
+    unsigned long long tl_p = TL_NOW();
     const uint64_t cs = (uint64_t)c * kChunkWords;
     const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
     const uint64_t* gsrc = a.words + cs;
@@ -730,27 +813,27 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const uint32_t nI = ctl->nI;
     const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = tid; f < nf; f += kThreads) S.fence[f] = p.d.fence[f];
     const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
     const uint32_t N = a.n_nodes;
     for (uint32_t q = tid; q < kChunkWords; q += kThreads) S.tw[q] = 0;
     if (tid < MEDUSA_CHUNK_WORDS / 32) S.hits[tid] = 0;
-    const uint64_t r0 = p.d.off_c[c];
-    const uint64_t r1 = min((uint64_t)p.d.off_c[c + 1], p.d.cap_c);
+    const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);
+    const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
     __syncthreads();
-    // B. warp 0: first window batch; warps 1..7: node starts -> launch positions
+    TL_PHASE(4, 10, tl_p);  // A: setup, fences
+    // B. warp 0: first window batch; warps 1..7: node starts -> node index per word
+    const uint32_t jf = N ? min(p.d.jf[c], N - 1) : 0, jl = N ? min(p.d.jl[c], N - 1) : 0;
     if (warp == 0) {
         if (r0 < r1) window_prepare(p, S, r0, (uint32_t)min((uint64_t)kWinCap, r1 - r0));
     } else if (N) {
-        const uint32_t jf = min(p.d.jf[c], N - 1), jl = min(p.d.jl[c], N - 1);
-        if (tid == 32) atomicMax(&S.tw[0], a.node_t[jf]);
         for (uint32_t j = jf + 1 + (tid - 32); j <= jl; j += kThreads - 32) {
             const uint64_t q = a.node_off[j] - cs;
-            if (q < n) atomicMax(&S.tw[q], a.node_t[j]);
+            if (q < n) atomicMax(&S.tw[q], j - jf);
         }
     }
     __syncthreads();
-    {  // running max over the chunk: tw[q] = launch position of the node holding word q
+    TL_PHASE(4, 11, tl_p);  // B: first window, node starts
+    {  // running max over the chunk: tw[q] = index (from jf) of the node holding word q
         uint32_t loc[kWordsPerThread];
         uint32_t run = 0;
 #pragma unroll
@@ -793,9 +876,15 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         if (cand) S.cq[base + __popc(bal & lanemask_lt())] = (uint16_t)q;
     }
     __syncthreads();
+    TL_PHASE(4, 12, tl_p);  // C: launch positions, TMA wait, candidates
     const uint32_t nc = S.nc;
-    // D. mortal window(s): upper bound of (word, launch position) over (base,
-    //    t_alloc), then walk back while the prefix max of end still reaches the word
+    // D. mortal window(s).  The entries live at one launch are pairwise disjoint,
+    //    so the only possible container of word x of node u is the live entry
+    //    with the greatest base <= x: one upper bound over the bases sorted in
+    //    shared memory, one AND with node u's live mask (bit e = entry e live at
+    //    u's launch), one leading-zero count, one end check.  Masks are built per
+    //    batch of <= kWinCap entries and group of kNodeGrp nodes.
+    const uint32_t nn = N ? jl - jf + 1 : 0;
     for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
         const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
         if (bs != r0) {
@@ -803,22 +892,61 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
             if (warp == 0) window_prepare(p, S, bs, m);
             __syncthreads();
         }
-        for (uint32_t i = tid; i < nc; i += kThreads) {
-            const uint32_t q = S.cq[i];
-            if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
-            const uint64_t x = S.words[q];
-            const uint32_t t = S.tw[q];
-            uint32_t lo = 0, hi = m;  // count of entries (base, t_alloc) < (x, t)
-            while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (kv_less(S.wb[mid], S.wta[mid], x, t)) lo = mid + 1; else hi = mid; }
-            for (int r = (int)lo - 1; r >= 0 && S.wpmax[r] > x; --r) {
-                if (x < S.we[r] && S.wta[r] < t && t < S.wtf[r]) {
-                    S.words[q] = ((uint64_t)S.wid[r] << MEDUSA_OFF_BITS) | (x - S.wb[r]);
+        const uint32_t mw = (m + 31) / 32;
+        for (uint32_t g0 = 0; g0 < nn;) {
+            const uint32_t ng = min((uint32_t)kNodeGrp, nn - g0);
+            for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
+            if (tid == 0) S.gnext = 0xFFFFFFFFu;
+            __syncthreads();
+            for (uint32_t pr = tid; pr < ng * mw; pr += kThreads) {
+                const uint32_t u = pr / mw, w = pr % mw;
+                const uint32_t t = S.nt[u];
+                uint32_t bits = 0;
+#pragma unroll 8
+                for (uint32_t b = 0; b < 32; ++b) {
+                    const uint32_t e = w * 32 + b;
+                    bits |= (e < m && S.wta[e] < t && t < S.wtf[e]) ? 1u << b : 0u;
+                }
+                S.live[u][w] = bits;
+            }
+            __syncthreads();
+            uint32_t gnext = 0xFFFFFFFFu;
+            for (uint32_t i = tid; i < nc; i += kThreads) {
+                const uint32_t q = S.cq[i];
+                if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
+                const uint32_t u = S.tw[q];
+                if (u < g0) continue;
+                if (u >= g0 + ng) { gnext = min(gnext, u); continue; }
+                const uint64_t x = S.words[q];
+                uint32_t lo = 0, hi = m;  // entries with base <= x
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
+                int e = -1;
+                for (int w = ((int)lo - 1) >> 5; w >= 0; --w) {
+                    uint32_t bits = S.live[u - g0][w];
+                    const uint32_t top = lo - (uint32_t)w * 32;  // entries of word w below lo
+                    if (top < 32) bits &= (1u << top) - 1u;
+                    if (bits) { e = w * 32 + 31 - __clz(bits); break; }
+                }
+                if (e >= 0 && x < S.we[e]) {
+                    S.words[q] = ((uint64_t)S.wid[e] << MEDUSA_OFF_BITS) | (x - S.wb[e]);
                     atomicOr(&S.hits[q >> 5], 1u << (q & 31));
-                    break;
                 }
             }
+            gnext = __reduce_min_sync(0xffffffffu, gnext);
+            if (lane == 0 && gnext != 0xFFFFFFFFu) atomicMin(&S.gnext, gnext);
+            __syncthreads();
+            const uint32_t gn = S.gnext;  // next group holding an unresolved candidate
+            __syncthreads();
+            if (gn == 0xFFFFFFFFu) break;
+            g0 = gn;
         }
     }
+    __syncthreads();
+    TL_PHASE(4, 13, tl_p);  // D: window search
+    // (phases A-D read only what k_trace / k_prepare wrote; the I list, fences
+    //  and summaries come from k_rank, this launch's PDL predecessor)
+    pdl_wait();
+    for (uint32_t f = tid; f < nf; f += kThreads) S.fence[f] = p.d.fence[f];
     __syncthreads();
     // E. I list, for the candidates still unresolved, compacted into a queue first
     if (nI) {
@@ -850,7 +978,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         for (uint32_t i = tid; i < nq; i += kThreads) {
             const uint32_t q = S.cq[i];
             const uint64_t x = S.words[q];
-            const uint32_t t = S.tw[q];
+            const uint32_t t = __ldg(a.node_t + jf + S.tw[q]);  // launch position of the word's node
             const uint32_t kk = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x) - 1;
             const uint64_t base = p.d.i_base[kk];
             const IRest e = p.d.i_rest[kk];
@@ -861,6 +989,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         }
     }
     __syncthreads();
+    TL_PHASE(4, 14, tl_p);  // E: I-list search
     // F. emission: mask words, warp-dense staging of records, chunk count
     const uint64_t n_mask = (a.n_words + 31) / 32;
     uint32_t cnt = 0;
@@ -875,17 +1004,14 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     }
     if (lane == 0) atomicAdd(&S.total, cnt);
     __syncthreads();
-    // G. the last classify CTA turns the chunk counts into chunk_base
+    TL_PHASE(4, 15, tl_p);  // F: emission
+    // G. the chunk's slot count and its 256-chunk group sum (k_emit turns them
+    //    into chunk_base)
     if (tid == 0) {
         p.d.chunk_cnt[c] = S.total;
-        __threadfence();
-        S.last = atomicAdd(&ctl->done_cls, 1u) == p.C - 1;
+        if (S.total) atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)S.total);
     }
-    __syncthreads();
-    if (S.last) {
-        __threadfence();
-        block_exclusive_scan(p.d.chunk_cnt, a.chunk_base, p.C, &ctl->n_slots);
-    }
+    pdl_trigger();
 }
 
 // one warp per block of 32 allocation ordinals; the CTA also checks 256 adjacent
@@ -893,6 +1019,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
     const MaterializeArgs& a = p.a;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
     {  // I-I: sorted neighbours must not overlap (all of I is live at the last launch)
         const uint32_t k = cta * blockDim.x + threadIdx.x;
@@ -901,9 +1028,13 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
     const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
     for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) S.fence[f] = p.d.fence[f];
-    __syncthreads();
-    const uint32_t b = cta * kWarps + warp;
+    // list offsets of this CTA's kWarps check blocks
+    const uint32_t b0 = cta * kWarps;
+    const unsigned long long base = block_prefix(p.d.cnt_b, p.d.sup_b, min(b0, p.nb));
+    const uint32_t b = b0 + warp;
     if (b >= p.nb) return;  // whole warp
+    const uint32_t cb = (lane <= warp && b0 + lane < p.nb) ? __ldcg(p.d.cnt_b + b0 + lane) : 0u;
+    const uint32_t before = __reduce_add_sync(0xffffffffu, lane < warp ? cb : 0u);
     const uint32_t j = b * kAblk + lane;
     bool mine = false;
     medusa_alloc x{};
@@ -916,8 +1047,8 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
     const uint64_t xe = x.base + x.size;
     bool bad = false;
     // M-M: mortals registered as live at some allocation of this block
-    const uint64_t r0 = p.d.off_b[b];
-    const uint64_t r1 = min((uint64_t)p.d.off_b[b + 1], p.d.cap_b);
+    const uint64_t r0 = base + before;
+    const uint64_t r1 = min(r0 + __shfl_sync(0xffffffffu, cb, warp), p.d.cap_b);
     for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
         const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
         __syncwarp();
@@ -954,12 +1085,19 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
             bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
     }
     if (bad) flag(p.d.ctl, ST_TRACE);
+    pdl_trigger();
 }
 
-__global__ void __launch_bounds__(kThreads) k_scan_words(P p) {
+__global__ void __launch_bounds__(kThreads, 4) k_scan_words(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    if (blockIdx.x < p.C) classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
-    else check_role(p, blockIdx.x - p.C, *reinterpret_cast<ChkShared*>(smem_raw));
+    const unsigned long long tl0 = TL_NOW();
+    if (blockIdx.x < p.C) {
+        classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
+        TL_REC(4, 0, tl0);
+    } else {
+        check_role(p, blockIdx.x - p.C, *reinterpret_cast<ChkShared*>(smem_raw));
+        TL_REC(4, 1, tl0);
+    }
 }
 
 // ----------------------------------------------------------------------------
@@ -967,12 +1105,23 @@ __global__ void __launch_bounds__(kThreads) k_scan_words(P p) {
 //    chunk, one thread per output record: coalesced stores)
 __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     __shared__ uint32_t s_pre[65];
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t c = blockIdx.x;
     const uint64_t n_mask = (a.n_words + 31) / 32;
     const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
-    const uint64_t prefix = a.chunk_base[c];
+    // this chunk's first slot: the sum of the slot counts of all earlier chunks
+    const uint64_t prefix = block_prefix(p.d.chunk_cnt, p.d.chunk_sup, c);
+    const uint32_t total = __ldcg(p.d.chunk_cnt + c);
+    if (tid == 0) {
+        a.chunk_base[c] = (uint32_t)prefix;
+        if (c + 1 == p.C) {
+            a.chunk_base[c + 1] = (uint32_t)(prefix + total);
+            p.d.ctl->n_slots = prefix + total;
+        }
+    }
     if (warp < 2) {
         const uint64_t mw = m0 + warp * 32 + lane;
         const uint32_t pc = mw < n_mask ? __popc(a.mask[mw]) : 0u;
@@ -989,17 +1138,20 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     const uint32_t half0 = s_pre[64];
     if (tid >= 32 && tid < 64) s_pre[tid] += half0;  // second half after the first
     __syncthreads();
-    const uint32_t total = (uint32_t)(a.chunk_base[c + 1] - prefix);
     for (uint32_t r = tid; r < total; r += kThreads) {
         uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
         while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
         const uint64_t dst = prefix + r;
         if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + (r - s_pre[lo])];
     }
+    pdl_trigger();
+    TL_REC(5, 0, tl0);
 }
 
 // 6. k_result (async entry): the outcome as a medusa_mat_result
 __global__ void k_result(P p, medusa_mat_result* r) {
+    pdl_wait();
+    pdl_trigger();
     const Ctl& c = *p.d.ctl;
     int32_t st = MEDUSA_OK;
     if (c.status & ST_INVALID) st = MEDUSA_ERR_INVALID_ARG;
@@ -1053,18 +1205,21 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
     const size_t RC = std::max<size_t>(need_c, N + 4 * CC), RB = std::max<size_t>(need_b, 3 * N);
     const size_t NS = N / kIBlk + 1;
     cudaError_t e;
-    // zero region: Ctl | cnt_c fill_c off_c [CC+1] | cnt_b fill_b off_b [NB+1] | blk_min_ta_c blk_max_tf [NS]
-    s.zero_bytes = 256 + 3 * (CC + 1) * 4 + 3 * (NB + 1) * 4 + 2 * NS * 4 + 64;
+    // zero region: Ctl | sup_c chunk_sup [CC/256+1] sup_b [NB/256+1] (u64) | cnt_c fill_c [CC+1] |
+    //              cnt_b fill_b [NB+1] | blk_min_ta_c blk_max_tf [NS]
+    const size_t GC = CC / 256 + 1, GB = NB / 256 + 1;
+    s.zero_bytes = 256 + (2 * GC + GB) * 8 + 2 * (CC + 1) * 4 + 2 * (NB + 1) * 4 + 2 * NS * 4 + 64;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
     char* z = (char*)s.zero_region;
     s.d.ctl = (Ctl*)z;
     size_t o = 256;
+    s.d.sup_c = (unsigned long long*)(z + o); o += GC * 8;
+    s.d.chunk_sup = (unsigned long long*)(z + o); o += GC * 8;
+    s.d.sup_b = (unsigned long long*)(z + o); o += GB * 8;
     s.d.cnt_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
     s.d.fill_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
-    s.d.off_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
     s.d.cnt_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
     s.d.fill_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
-    s.d.off_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
     s.d.blk_min_ta_c = (uint32_t*)(z + o); o += NS * 4;
     s.d.blk_max_tf = (uint32_t*)(z + o); o += NS * 4;
     if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.rng, N)) ||
@@ -1095,6 +1250,7 @@ Scratch* device_scratch(cudaError_t* e) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
         const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
         cudaFuncSetAttribute(k_scan_words, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem);
+        cudaFuncSetAttribute(k_prepare, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(PrepShared));
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
     return &s;
@@ -1122,20 +1278,20 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     if (n) {
         {
             TimedLaunch tl("mat_prepare", stream);
-            k_prepare<<<sort_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
+            if ((e = launch_pdl(k_prepare, sort_ctas + alloc_ctas, kThreads, sizeof(PrepShared), stream, p))) return e;
         }
         TimedLaunch tl("mat_rank", stream);
         const uint64_t jobs = (uint64_t)sort_ctas * ((n + kRankKeys - 1) / kRankKeys);
         const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(jobs, (uint64_t)s.sm_count * 8));
-        k_rank<<<grid, kThreads, 0, stream>>>(p);
+        if ((e = launch_pdl(k_rank, grid, kThreads, 0, stream, p))) return e;
     }
     if (C + check_ctas) {
         TimedLaunch tl("mat_classify", stream);
-        k_scan_words<<<C + check_ctas, kThreads, scan_smem, stream>>>(p);
+        if ((e = launch_pdl(k_scan_words, C + check_ctas, kThreads, scan_smem, stream, p))) return e;
     }
     if (C) {
         TimedLaunch tl("mat_emit", stream);
-        k_emit<<<C, kThreads, 0, stream>>>(p);
+        if ((e = launch_pdl(k_emit, C, kThreads, 0, stream, p))) return e;
     }
     return cudaGetLastError();
 }
@@ -1164,8 +1320,8 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
         if (h.status & ST_INVALID) return MEDUSA_ERR_INVALID_ARG;
         if (h.status & ST_TRACE) return MEDUSA_ERR_TRACE;
         if (h.status & ST_OVERFLOW) {  // registration lists larger than guessed: size exactly, rerun
-            need_c = h.need_c;
-            need_b = h.need_b;
+            need_c = std::max<size_t>(need_c, h.need_c);
+            need_b = std::max<size_t>(need_b, h.need_b);
             continue;
         }
         *n_slots = h.n_slots;
@@ -1190,9 +1346,24 @@ medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result*
     if ((e = ensure(s, n, C, nb, a.n_words, 0, 0)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     P p;
     if ((e = enqueue(s, a, stream, &p)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-    k_result<<<1, 1, 0, stream>>>(p, d_result);
+    if ((e = launch_pdl(k_result, 1, 1, 0, stream, p, d_result))) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     if ((e = cudaGetLastError()) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     return MEDUSA_OK;
 }
 
 }  // namespace medusa
+
+#ifdef MEDUSA_TIMELINE
+extern "C" int medusa_tl_attach_mat(void* buf, unsigned cap) {
+    unsigned zero = 0;
+    medusa::TlRec* b = static_cast<medusa::TlRec*>(buf);
+    if (cudaMemcpyToSymbol(medusa::g_tl, &b, sizeof(b)) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(medusa::g_tl_cap, &cap, sizeof(cap)) != cudaSuccess) return -1;
+    return cudaMemcpyToSymbol(medusa::g_tl_n, &zero, sizeof(zero)) == cudaSuccess ? 0 : -1;
+}
+extern "C" unsigned medusa_tl_count_mat() {
+    unsigned n = 0;
+    cudaMemcpyFromSymbol(&n, medusa::g_tl_n, sizeof(n));
+    return n;
+}
+#endif

@@ -40,7 +40,12 @@ constexpr int kThreads = 256;
 constexpr int kMaskPerTask = kTaskWords / 32;   // 64
 constexpr int kNodesPerTask = 2048;
 
+MEDUSA_TL_DEFINE
+
 __global__ void report_init(medusa_report* r) {
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();  // the previous user of the report may still read it
+    pdl_trigger();
     r->n_bad_slot = 0;
     r->first_bad_word = ~0ull;
     r->n_bad_id = 0;
@@ -49,6 +54,7 @@ __global__ void report_init(medusa_report* r) {
     r->n_bad_func = 0;
     r->first_bad_node = ~0ull;
     r->reserved = 0;
+    TL_REC(6, 0, tl0);
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -66,6 +72,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     const uint32_t tid = threadIdx.x;
     const uint32_t task = blockIdx.x;
     unsigned long long* rep = reinterpret_cast<unsigned long long*>(a.report);
+    const unsigned long long tl0 = TL_NOW();
 
     if (task < n_word_tasks) {
         const uint64_t ws = (uint64_t)task * kTaskWords;
@@ -207,6 +214,8 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         } else {
             for (uint32_t q = tid; q < n; q += kThreads) st_stream(gdst + q, s_words[q]);
         }
+        pdl_wait();  // report_init (this launch's PDL predecessor) has run
+        pdl_trigger();
         if (n_id | n_rg | n_st) {
             atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));
             atomicMin(rep + 1, (unsigned long long)first);
@@ -214,6 +223,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             if (n_rg) atomicAdd(rep + 3, (unsigned long long)n_rg);
             if (n_st) atomicAdd(rep + 4, (unsigned long long)n_st);
         }
+        TL_REC(7, 0, tl0);
     } else if (task < n_tasks) {
         const uint64_t j0 = (uint64_t)(task - n_word_tasks) * kNodesPerTask;
         uint32_t n_bad = 0;
@@ -232,10 +242,13 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 a.func_out[j] = addr;
             }
         }
+        pdl_wait();
+        pdl_trigger();
         if (n_bad) {
             atomicAdd(rep + 5, (unsigned long long)n_bad);
             atomicMin(rep + 6, (unsigned long long)first);
         }
+        TL_REC(7, 1, tl0);
     }
 }
 
@@ -247,13 +260,30 @@ cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     const uint32_t n_tasks = n_word_tasks + n_node_tasks;
     {
         TimedLaunch tl("restore_report_init", stream);
-        report_init<<<1, 1, 0, stream>>>(a.report);
+        cudaError_t e = launch_pdl(report_init, 1, 1, 0, stream, a.report);
+        if (e != cudaSuccess) return e;
     }
     if (n_tasks) {
         TimedLaunch tl("restore", stream);
-        restore_kernel<<<n_tasks, kThreads, 0, stream>>>(a, n_word_tasks, n_tasks);
+        cudaError_t e = launch_pdl(restore_kernel, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks);
+        if (e != cudaSuccess) return e;
     }
     return cudaGetLastError();
 }
 
 }  // namespace medusa
+
+#ifdef MEDUSA_TIMELINE
+extern "C" int medusa_tl_attach_res(void* buf, unsigned cap) {
+    unsigned zero = 0;
+    medusa::TlRec* b = static_cast<medusa::TlRec*>(buf);
+    if (cudaMemcpyToSymbol(medusa::g_tl, &b, sizeof(b)) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(medusa::g_tl_cap, &cap, sizeof(cap)) != cudaSuccess) return -1;
+    return cudaMemcpyToSymbol(medusa::g_tl_n, &zero, sizeof(zero)) == cudaSuccess ? 0 : -1;
+}
+extern "C" unsigned medusa_tl_count_res() {
+    unsigned n = 0;
+    cudaMemcpyFromSymbol(&n, medusa::g_tl_n, sizeof(n));
+    return n;
+}
+#endif

@@ -163,6 +163,25 @@ def test_tiny_traces_status_and_slots(overlap_p):
             assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec), seed
 
 
+@pytest.mark.parametrize("seed", range(6))
+def test_long_chunks_many_nodes_and_window_batches(seed):
+    """Chunks holding ~1000 nodes (several live-mask node groups) whose windows
+    hold hundreds of registered mortals (several window batches), with heavy
+    address reuse: status and table identical to the oracle."""
+    words, off, node_t, allocs = tiny_trace(1000 + seed, n_steps=7000, max_words=2, max_allocs=2500,
+                                            overlap_p=0.0 if seed < 5 else 0.01)
+    st, s = _run_tiny(words, off, node_t, allocs)
+    m = oracle.materialize(words, off, node_t, allocs)
+    assert st == m["status"]
+    assert words.size > 2048 and node_t.size > 2000 and allocs.size > 1000
+    if st == 0:
+        mask, cb, rec = oracle.pack(m, words.size)
+        assert s.n_slots == m["n_slots"]
+        assert np.array_equal(_h(s.mask).view(np.uint32), mask)
+        assert np.array_equal(_h(s.chunk_base).view(np.uint32), cb)
+        assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec)
+
+
 def test_edge_cases():
     b = 0x7F00_0000_0000
     A = lambda rows: np.array(rows, dtype=ALLOC_DTYPE)

@@ -15,7 +15,7 @@ from workloads import ALLOC_DTYPE, T_NEVER
 BASE0 = 0x7F00_0000_0000
 
 
-def tiny_trace(seed, n_steps=120, overlap_p=0.0, max_words=6):
+def tiny_trace(seed, n_steps=120, overlap_p=0.0, max_words=6, max_allocs=60):
     rng = np.random.default_rng(seed)
     allocs = []  # [base, size, ta, tf]
     live = []
@@ -26,7 +26,7 @@ def tiny_trace(seed, n_steps=120, overlap_p=0.0, max_words=6):
     for _ in range(n_steps):
         r = rng.random()
         t += int(rng.choice([0, 1, 1, 2]))
-        if r < 0.35 and len(allocs) < 60:
+        if r < 0.35 and len(allocs) < max_allocs:
             tt = max(t, last_alloc_t + 1)
             size = int(rng.choice([0, 16, 64, 64, 128, 192, 256]))
             for _try in range(8):

@@ -8,6 +8,7 @@ from collections import defaultdict
 
 rep, kre = sys.argv[1], sys.argv[2]
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 30
+by = sys.argv[4] if len(sys.argv) > 4 else "inst"  # or "smp"
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--print-source", "cuda,sass", "--csv", "-k", f"regex:{kre}"],
                      capture_output=True, text=True).stdout
 agg = defaultdict(lambda: [0.0, 0.0])
@@ -41,5 +42,5 @@ for row in csv.reader(io.StringIO(out)):
 ti = sum(v[0] for v in agg.values()) or 1
 ts = sum(v[1] for v in agg.values()) or 1
 print(f"instructions {ti:.3g}  samples {ts:.0f}")
-for key, (i, s) in sorted(agg.items(), key=lambda kv: -kv[1][0])[:top]:
+for key, (i, s) in sorted(agg.items(), key=lambda kv: -kv[1][0 if by == 'inst' else 1])[:top]:
     print(f"{100*i/ti:5.1f}% inst {100*s/ts:5.1f}% smp  {key[0]}:{key[1]:<5d} {text.get(key, '').strip()[:90]}")

@@ -1,0 +1,106 @@
+"""Per-CTA timeline of one graph-captured step (diagnostic; not part of the product).
+
+Builds tools/libmedusa_tl.so with -DMEDUSA_TIMELINE (thread 0 of every CTA
+stamps %globaltimer at start and end), replays the bench step (materialize_async
+-> kernel_table_set -> restore) K times with an L2 scrub before each, and prints
+per kernel/role: CTA count, first start / last end relative to the step start,
+CTA duration percentiles, and the idle gap before each kernel.
+
+usage: python tools/timeline.py [--workload all10] [--steps 5]
+"""
+import argparse
+import ctypes
+import os
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import __graft_entry__ as g  # noqa: E402
+
+NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan",
+         (2, 0): "prepare/sort", (2, 1): "prepare/scatter", (3, 0): "rank",
+         (4, 0): "scan/classify", (4, 1): "scan/check", (4, 2): "scan/last-scan",
+         (5, 0): "emit", (6, 0): "report_init", (7, 0): "restore/words", (7, 1): "restore/gather",
+         (1, 20): " allocs:load+nj0", (1, 21): " allocs:stage", (1, 22): " allocs:search+reg",
+         (1, 23): " last:fence", (1, 24): " last:scan-c", (1, 25): " last:scan-b",
+         (2, 30): " sort:bitonic", (2, 31): " sort:merges",
+         (4, 10): " cls:A setup", (4, 11): " cls:B window", (4, 12): " cls:C tw+cand", (4, 13): " cls:D winsearch",
+         (4, 14): " cls:E I-search", (4, 15): " cls:F emit"}
+REC = np.dtype([("t0", "<u8"), ("t1", "<u8"), ("kernel", "<u4"), ("cta", "<u4"), ("sm", "<u4"), ("tag", "<u4")])
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="all10")
+    ap.add_argument("--steps", type=int, default=5)
+    args = ap.parse_args()
+    tl_path = g.build_medusa(out=os.path.join(ROOT, "tools", "libmedusa_tl.so"), defines=("MEDUSA_TIMELINE",))
+    import paper_conf_asplos_zengxgcl25_b200 as medusa
+    from workloads import CONFIGS, make_graph_set
+    medusa._lib = None
+    medusa.LIB_PATH = tl_path
+    L = medusa.lib()
+    for sfx in ("mat", "res"):
+        getattr(L, f"medusa_tl_attach_{sfx}").argtypes = [ctypes.c_void_p, ctypes.c_uint]
+        getattr(L, f"medusa_tl_count_{sfx}").restype = ctypes.c_uint
+    dev = torch.device("cuda:0")
+    gs = make_graph_set(args.workload, seed=1)
+    inp = medusa.upload(gs, dev)
+    slots = medusa.alloc_slots(gs.n_words, dev)
+    res = torch.zeros(2, dtype=torch.int64, device=dev)
+    dst = torch.empty_like(inp["words"])
+    fout = torch.empty(gs.n_nodes, dtype=torch.int64, device=dev)
+    rep = torch.empty(8, dtype=torch.int64, device=dev)
+    medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots)  # sizes scratch
+
+    def step():
+        medusa.materialize_async(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots, result=res)
+        medusa.kernel_table_set(inp["table"])
+        medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                       dst=dst, func_out=fout, report=rep, from_table=True)
+
+    cap = 1 << 16
+    buf = [torch.zeros(cap * REC.itemsize, dtype=torch.uint8, device=dev) for _ in range(2)]
+    step()  # eager once: the kernel table and scratch are allocated outside capture
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        step()
+    scrub = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    for _ in range(3):
+        graph.replay()
+    agg = {}
+    spans = []
+    ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+    for k in range(args.steps):
+        L.medusa_tl_attach_mat(ctypes.c_void_p(buf[0].data_ptr()), cap)
+        L.medusa_tl_attach_res(ctypes.c_void_p(buf[1].data_ptr()), cap)
+        scrub.fill_(k)
+        ev[0].record()
+        graph.replay()
+        ev[1].record()
+        torch.cuda.synchronize()
+        n0, n1 = L.medusa_tl_count_mat(), L.medusa_tl_count_res()
+        recs = np.concatenate([buf[0][: n0 * REC.itemsize].cpu().numpy().view(REC),
+                               buf[1][: n1 * REC.itemsize].cpu().numpy().view(REC)])
+        t_begin = recs["t0"].min()
+        spans.append(((recs["t1"].max() - t_begin) / 1e3, ev[0].elapsed_time(ev[1]) * 1e3))
+        for key in sorted(set(zip(recs["kernel"].tolist(), recs["tag"].tolist()))):
+            r = recs[(recs["kernel"] == key[0]) & (recs["tag"] == key[1])]
+            d = (r["t1"] - r["t0"]) / 1e3
+            agg.setdefault(key, []).append(((r["t0"].min() - t_begin) / 1e3, (r["t1"].max() - t_begin) / 1e3, len(r),
+                                            np.percentile(d, 50), np.percentile(d, 90), d.max()))
+    assert medusa.mat_result(res)[0] == 0
+    print(f"{args.workload}: step span (first CTA start -> last CTA end) {np.mean([s[0] for s in spans]):.1f} us; "
+          f"event time {np.mean([s[1] for s in spans]):.1f} us (incl. launch of the first kernel)")
+    print(f"{'kernel/role':18s} {'ctas':>6s} {'start':>8s} {'end':>8s} {'span':>7s} {'p50':>7s} {'p90':>7s} {'max':>7s}  (us)")
+    for key, rows in sorted(agg.items(), key=lambda kv: np.mean([r[0] for r in kv[1]])):
+        a = np.mean(np.array(rows), axis=0)
+        print(f"{NAMES.get(key, str(key)):18s} {a[2]:6.0f} {a[0]:8.1f} {a[1]:8.1f} {a[1]-a[0]:7.1f} {a[3]:7.2f} {a[4]:7.2f} {a[5]:7.2f}")
+
+
+if __name__ == "__main__":
+    main()
