@@ -55,7 +55,6 @@ constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
 constexpr int kSortTile = 2048;    // keys sorted per CTA before ranking
-constexpr int kRankKeys = 256;     // keys ranked per k_rank job (one per thread)
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
 constexpr int kWinCap = 128;       // mortal-window entries per batch (<= 4 per lane of one warp)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
@@ -105,7 +104,8 @@ struct Dev {  // scratch of one call (device pointers)
     uint64_t cap_c, cap_b;
     uint64_t* sk[2];                             // [n] sort keys: 0 unsorted, 1 sorted tiles
     uint32_t* sv[2];                             // [n] sort values (allocation index)
-    unsigned long long* rank;                    // [n] (contributions << 32) | rank
+    uint64_t* samp_k;                            // [n/32+1] every 32nd key of each sorted tile
+    uint32_t* samp_v;
     uint64_t* i_base;                            // [n]
     IRest* i_rest;                               // [n]
     uint32_t* i_tf;                              // [n]
@@ -119,7 +119,7 @@ struct P {  // kernel parameters
     Dev d;
     uint32_t C, nb;              // chunks, check blocks
     uint32_t node_ctas;          // k_trace: CTAs with the node role
-    uint32_t sort_ctas;          // k_prepare: CTAs with the sort role
+    uint32_t sort_ctas;          // k_isort: tiles of 2048 I keys (bound: allocation count / 2048)
     uint32_t check_ctas;         // k_scan_words: CTAs with the check role (after the C classify CTAs)
 };
 
@@ -468,19 +468,20 @@ __device__ __forceinline__ void warp_bitonic(uint64_t (&k)[E], uint32_t (&v)[E],
     }
 }
 
-// merge path inside shared memory: smallest i in [lo, hi) with less(B[d-1-i], A[i]), else hi
-__device__ __forceinline__ uint32_t merge_path_smem(const uint64_t* ka, const uint32_t* va, const uint64_t* kb,
-                                                    const uint32_t* vb, uint32_t d, uint32_t lo, uint32_t hi) {
-    while (lo < hi) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (kv_less(kb[d - 1 - mid], vb[d - 1 - mid], ka[mid], va[mid])) hi = mid; else lo = mid + 1;
-    }
-    return lo;
+// the I entry of sorted position r: arrays, fence, block summaries
+// one allocation record through the read-only path
+__device__ __forceinline__ medusa_alloc ld_alloc(const medusa_alloc* q) {
+    const unsigned long long* w = reinterpret_cast<const unsigned long long*>(q);
+    const unsigned long long b = __ldg(w), z = __ldg(w + 1), t = __ldg(w + 2);
+    medusa_alloc x;
+    x.base = b;
+    x.size = z;
+    x.t_alloc = (uint32_t)t;
+    x.t_free = (uint32_t)(t >> 32);
+    return x;
 }
 
-// the I entry of sorted position r: arrays, fence, block summaries
-__device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t nI, uint32_t id) {
-    const medusa_alloc x = p.a.alloc[id];
+__device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t nI, uint32_t id, const medusa_alloc& x) {
     p.d.i_base[r] = x.base;
     p.d.i_rest[r] = IRest{x.base + x.size, x.t_alloc, id};
     p.d.i_tf[r] = x.t_free;
@@ -490,67 +491,127 @@ __device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t n
     atomicMax(&p.d.blk_max_tf[r / kIBlk], x.t_free);
 }
 
+// Bitonic sort of 32*E (key, val) pairs held E per lane (element lane*E + r),
+// ascending by (key, val); shuffles and register compare-exchanges only.
+template <int E>
+__device__ __forceinline__ void warp_bitonic_kv(uint64_t (&k)[E], uint32_t (&v)[E]) {
+    const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+    for (uint32_t size = 2; size <= 32u * E; size <<= 1) {
+#pragma unroll
+        for (uint32_t j = size >> 1; j > 0; j >>= 1) {
+            if (j >= (uint32_t)E) {
+                const uint32_t lj = j / E;
+                const bool lower = (lane & lj) == 0;
+#pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const uint32_t e = lane * E + r;
+                    const uint64_t ok = __shfl_xor_sync(0xffffffffu, k[r], lj);
+                    const uint32_t ov = __shfl_xor_sync(0xffffffffu, v[r], lj);
+                    const bool up = (e & size) == 0;
+                    const bool other_less = kv_less(ok, ov, k[r], v[r]);
+                    if ((lower == up) ? other_less : !other_less) { k[r] = ok; v[r] = ov; }
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const int r2 = r ^ (int)j;
+                    if (r2 > r && kv_less(k[r2], v[r2], k[r], v[r]) == (((lane * E + r) & size) == 0)) {
+                        const uint64_t tk = k[r]; k[r] = k[r2]; k[r2] = tk;
+                        const uint32_t tv = v[r]; v[r] = v[r2]; v[r2] = tv;
+                    }
+                }
+            }
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------
+// 2a. k_isort (side stream, parallel to k_prepare): one 1024-thread CTA per tile
+//     of 2048 I keys (base, allocation index).  A register bitonic sort of 64
+//     keys per warp, then five merge-path rounds through shared memory
+//     (64 -> 128 -> ... -> 2048), two keys per thread held in registers between
+//     rounds.  A single tile is the whole list: its I entries are written here.
+constexpr int kSortThreads = 1024;
+constexpr int kSortPer = kSortTile / kSortThreads;  // 2
 struct SortShared {
-    uint64_t sk[2][kSortTile];
-    uint32_t sv[2][kSortTile];
+    uint64_t k[kSortTile];
+    uint32_t v[kSortTile];
 };
 
-__device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
+__global__ void __launch_bounds__(kSortThreads) k_isort(P p) {
+    extern __shared__ __align__(16) unsigned char sort_raw[];
+    SortShared& S = *reinterpret_cast<SortShared*>(sort_raw);
+    const unsigned long long tl0 = TL_NOW();
+    unsigned long long tl_p = tl0;
+    pdl_wait();
     const uint32_t n = p.d.ctl->nI;
-    const uint32_t t0 = tile * kSortTile;
-    if (t0 >= n) return;
-    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    unsigned long long tl_p = TL_NOW();
-    uint64_t k[8];
-    uint32_t v[8], pl[8];
+    const uint32_t t0 = blockIdx.x * kSortTile;
+    if (t0 < n) {
+        const uint32_t o = threadIdx.x * kSortPer;  // this thread's consecutive elements
+        uint64_t k[kSortPer];
+        uint32_t v[kSortPer];
 #pragma unroll
-    for (int r = 0; r < 8; ++r) {
-        const uint32_t g = t0 + warp * 256 + lane * 8 + r;
-        k[r] = g < n ? p.d.sk[0][g] : ~0ull;
-        v[r] = g < n ? p.d.sv[0][g] : 0xFFFFFFFFu;
-        pl[r] = 0;
-    }
-    warp_bitonic<8>(k, v, pl);
-#pragma unroll
-    for (int r = 0; r < 8; ++r) {
-        S.sk[0][warp * 256 + lane * 8 + r] = k[r];
-        S.sv[0][warp * 256 + lane * 8 + r] = v[r];
-    }
-    __syncthreads();
-    TL_PHASE(2, 30, tl_p);  // load + warp bitonic
-    int src = 0;
-#pragma unroll
-    for (uint32_t run = 256; run < kSortTile; run <<= 1) {
-        const uint32_t o = tid * 8;
-        const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
-        const uint32_t d = o - a0;
-        const uint64_t* ka = S.sk[src] + a0;
-        const uint32_t* va = S.sv[src] + a0;
-        const uint64_t* kb = S.sk[src] + b0;
-        const uint32_t* vb = S.sv[src] + b0;
-        uint32_t ia = merge_path_smem(ka, va, kb, vb, d, d > run ? d - run : 0, min(d, run));
-        uint32_t ib = d - ia;
-#pragma unroll
-        for (int q = 0; q < 8; ++q) {
-            const bool takeA = ib >= run || (ia < run && kv_less(ka[ia], va[ia], kb[ib], vb[ib]));
-            S.sk[src ^ 1][o + q] = takeA ? ka[ia] : kb[ib];
-            S.sv[src ^ 1][o + q] = takeA ? va[ia] : vb[ib];
-            if (takeA) ++ia; else ++ib;
+        for (int r = 0; r < kSortPer; ++r) {
+            const uint32_t g = t0 + o + r;
+            k[r] = g < n ? __ldcg(p.d.sk[0] + g) : ~0ull;
+            v[r] = g < n ? __ldcg(p.d.sv[0] + g) : 0xFFFFFFFFu;
         }
-        src ^= 1;
-        __syncthreads();
-    }
-    TL_PHASE(2, 31, tl_p);  // shared-memory merges
-    const bool single = n <= kSortTile;  // one tile: its order is final
-    for (uint32_t q = tid; q < kSortTile && t0 + q < n; q += blockDim.x) {
-        if (single) {
-            write_i_entry(p, q, n, S.sv[src][q]);
-        } else {
-            p.d.sk[1][t0 + q] = S.sk[src][q];
-            p.d.sv[1][t0 + q] = S.sv[src][q];
-            p.d.rank[t0 + q] = q;  // rank within the tile, no contribution yet
+        warp_bitonic_kv<kSortPer>(k, v);
+        TL_PHASE(2, 30, tl_p);  // load + warp bitonic
+#pragma unroll 1
+        for (uint32_t run = 32 * kSortPer; run < kSortTile; run <<= 1) {
+#pragma unroll
+            for (int r = 0; r < kSortPer; ++r) { S.k[o + r] = k[r]; S.v[o + r] = v[r]; }
+            __syncthreads();
+            const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
+            const uint32_t d = o - a0;
+            uint32_t lo = d > run ? d - run : 0, hi = min(d, run);
+            while (lo < hi) {  // merge path: A elements among the first d of the merged pair
+                const uint32_t mid = (lo + hi) >> 1;
+                const uint32_t pb = b0 + d - 1 - mid, pa = a0 + mid;
+                const uint64_t x = S.k[pa], y = S.k[pb];  // values only break key ties
+                if (x < y || (x == y && S.v[pa] < S.v[pb])) lo = mid + 1; else hi = mid;
+            }
+            uint32_t ia = lo, ib = d - lo;
+#pragma unroll
+            for (int r = 0; r < kSortPer; ++r) {
+                const uint32_t pa = a0 + min(ia, run - 1), pb = b0 + min(ib, run - 1);
+                const uint64_t ka = S.k[pa], kb = S.k[pb];
+                const uint32_t va = S.v[pa], vb = S.v[pb];
+                const bool takeA = ib >= run || (ia < run && kv_less(ka, va, kb, vb));
+                k[r] = takeA ? ka : kb;
+                v[r] = takeA ? va : vb;
+                if (takeA) ++ia; else ++ib;
+            }
+            __syncthreads();
         }
+        TL_PHASE(2, 31, tl_p);  // shared-memory merges
+        const bool single = n <= kSortTile;  // one tile: its order is final
+        medusa_alloc x[kSortPer];
+        if (single) {  // all record loads first (independent), then the writes
+#pragma unroll
+            for (int r = 0; r < kSortPer; ++r)
+                if (o + r < n) x[r] = ld_alloc(p.a.alloc + v[r]);
+        }
+#pragma unroll
+        for (int r = 0; r < kSortPer; ++r) {
+            const uint32_t q = o + r;
+            if (t0 + q >= n) break;
+            if (single) {
+                write_i_entry(p, q, n, v[r], x[r]);
+            } else {
+                p.d.sk[1][t0 + q] = k[r];
+                p.d.sv[1][t0 + q] = v[r];
+                if ((q & 31) == 0) {  // every 32nd key: the tile's sample for k_rank
+                    p.d.samp_k[t0 / 32 + q / 32] = k[r];
+                    p.d.samp_v[t0 / 32 + q / 32] = v[r];
+                }
+            }
+        }
+        TL_REC(2, 0, tl0);
     }
+    pdl_trigger();
 }
 
 // One registration list (chunks or check blocks): the CTA's 256 allocations
@@ -638,58 +699,118 @@ __device__ void scatter_role(const P& p, uint32_t cta, ScatterShared& S) {
                  S.pre, S.first, S.w, S.range);
 }
 
-union PrepShared {
-    SortShared sort;
-    ScatterShared scatter;
-};
-
 __global__ void __launch_bounds__(kThreads) k_prepare(P p) {
-    extern __shared__ __align__(16) unsigned char prep_raw[];
-    PrepShared& U = *reinterpret_cast<PrepShared*>(prep_raw);
+    __shared__ ScatterShared S;
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
-    if (blockIdx.x < p.sort_ctas) {
-        sort_role(p, blockIdx.x, U.sort);
-        TL_REC(2, 0, tl0);
-    } else {
-        scatter_role(p, blockIdx.x - p.sort_ctas, U.scatter);
-        TL_REC(2, 1, tl0);
-    }
+    scatter_role(p, blockIdx.x, S);
+    TL_REC(2, 1, tl0);
     pdl_trigger();
 }
 
 // ----------------------------------------------------------------------------
-// 3. k_rank: rank = index in own tile + count of keys below it in every other
-//    tile.  CTA (t, kb) stages sorted tile t in shared memory and counts, for the
-//    2048 keys of tile kb (kb != t), how many of tile t's keys are below; the
-//    thread adding a key's last contribution writes its I entry in place.
+// 2b. k_rank (after k_isort): global rank of every I key = its index in its sorted
+//     tile + the count of smaller keys in every other tile.  One CTA per range of
+//     32 consecutive keys of one tile (one key per lane); warp w counts against
+//     tiles b = w, w + 8, ...: the tile's 64-key sample (every 32nd key) comes in
+//     with one coalesced load and locates, by a shuffle search, the 32-key block
+//     of the tile holding each lane's lower bound; the block comes in with one
+//     more coalesced load and a shuffle search finishes the count.  The counts
+//     of the 8 warps meet in shared memory; warp 0 writes the 32 I entries.
+__device__ __forceinline__ bool kv_lt_lane(uint64_t k, uint32_t v, uint32_t src, uint64_t xk, uint32_t xv) {
+    const uint64_t sk = __shfl_sync(0xffffffffu, k, src);
+    const uint32_t sv = __shfl_sync(0xffffffffu, v, src);
+    return kv_less(sk, sv, xk, xv);
+}
+
 __global__ void __launch_bounds__(kThreads) k_rank(P p) {
-    __shared__ uint64_t sk[kSortTile];
-    __shared__ uint32_t sv[kSortTile];
+    __shared__ uint32_t s_cnt[kWarps][32];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t T = n_tiles(nI);
-    if (T <= 1) return;
-    const uint64_t* gk = p.d.sk[1];
-    const uint32_t* gv = p.d.sv[1];
-    const uint32_t KB = (nI + kRankKeys - 1) / kRankKeys;  // key blocks of kRankKeys
-    for (uint64_t job = blockIdx.x; job < (uint64_t)T * KB; job += gridDim.x) {
-        const uint32_t t = (uint32_t)(job / KB), kb = (uint32_t)(job % KB);
-        if (t == kb * kRankKeys / kSortTile) continue;  // a key block lies inside one tile
-        const uint32_t t0 = t * kSortTile, tn = min((uint32_t)kSortTile, nI - t0);
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t g0 = blockIdx.x * 32;  // this CTA's 32 keys
+    if (T > 1 && g0 < nI) {
+        const uint32_t ta = g0 / kSortTile;
+        const uint32_t g = g0 + lane;
+        const bool has = g < nI;
+        const uint64_t xk = has ? __ldcg(p.d.sk[1] + g) : ~0ull;
+        const uint32_t xv = has ? __ldcg(p.d.sv[1] + g) : 0xFFFFFFFFu;
+        uint32_t cnt = 0;
+        for (uint32_t tb = warp; tb < T; tb += kWarps) {
+            if (tb == ta) continue;
+            const uint32_t b0 = tb * kSortTile, nb = min((uint32_t)kSortTile, nI - b0);
+            const uint32_t ns = (nb + 31) / 32;  // samples of tile tb (<= 64)
+            // samples ns_l = lane, lane + 32
+            uint64_t sk0 = ~0ull, sk1 = ~0ull;
+            uint32_t sv0 = 0xFFFFFFFFu, sv1 = 0xFFFFFFFFu;
+            if (lane < ns) { sk0 = __ldcg(p.d.samp_k + b0 / 32 + lane); sv0 = __ldcg(p.d.samp_v + b0 / 32 + lane); }
+            if (lane + 32 < ns) { sk1 = __ldcg(p.d.samp_k + b0 / 32 + lane + 32); sv1 = __ldcg(p.d.samp_v + b0 / 32 + lane + 32); }
+            // j = #samples < x: the lower bound of x lies in block j - 1 (j >= 1)
+            uint32_t j = 0;
+            {
+                const bool hi_half = ns > 32 && kv_lt_lane(sk1, sv1, 0, xk, xv);  // sample 32 < x
+                // count of samples < x inside this lane's half (32 entries, ascending);
+                // the source lane's value of BOTH halves is fetched, the lane picks
+                uint32_t lo = 0, hi = 32;
+#pragma unroll
+                for (int st = 0; st < 6; ++st) {
+                    const uint32_t mid = (lo + hi) >> 1;
+                    const bool lt0 = kv_lt_lane(sk0, sv0, min(mid, 31u), xk, xv);
+                    const bool lt1 = ns > 32 && kv_lt_lane(sk1, sv1, min(mid, 31u), xk, xv);
+                    const bool lt = hi_half ? lt1 : lt0;
+                    if (lo < hi) { if (lt) lo = mid + 1; else hi = mid; }
+                }
+                j = (hi_half ? 32 : 0) + lo;
+                if (j > ns) j = ns;
+            }
+            // lane l's lower bound lies in block j_l - 1 (ascending over the lanes).
+            // Few distinct blocks (the usual case): load each with one coalesced
+            // load and count by a shuffle search; otherwise every lane searches its
+            // own block in memory (5 dependent loads).
+            const uint32_t blk = j ? j - 1 : 0xFFFFFFFFu;
+            const bool act = has && j;
+            const uint32_t prev = __shfl_up_sync(0xffffffffu, blk, 1);
+            const uint32_t n_runs = __popc(__ballot_sync(0xffffffffu, act && (lane == 0 || prev != blk)));
+            uint32_t c = 0;
+            if (n_runs <= 2) {
+                uint32_t pending = __ballot_sync(0xffffffffu, act);
+                while (pending) {
+                    const uint32_t bl = __shfl_sync(0xffffffffu, blk, __ffs(pending) - 1);
+                    const uint32_t q = bl * 32 + lane;
+                    const uint64_t bk = q < nb ? __ldcg(p.d.sk[1] + b0 + q) : ~0ull;
+                    const uint32_t bv = q < nb ? __ldcg(p.d.sv[1] + b0 + q) : 0xFFFFFFFFu;
+                    uint32_t lo = 0, hi = 32;  // entries of the block below x
+#pragma unroll
+                    for (int st = 0; st < 6; ++st) {
+                        const uint32_t mid = (lo + hi) >> 1;
+                        const bool lt = kv_lt_lane(bk, bv, min(mid, 31u), xk, xv);
+                        if (lo < hi) { if (lt) lo = mid + 1; else hi = mid; }
+                    }
+                    if (act && blk == bl) c = bl * 32 + lo;
+                    pending &= ~__ballot_sync(0xffffffffu, act && blk == bl);
+                }
+            } else if (act) {
+                const uint32_t q0 = blk * 32;
+                uint32_t lo = 0, hi = min(32u, nb - q0);
+                while (lo < hi) {
+                    const uint32_t mid = (lo + hi) >> 1;
+                    const uint64_t bk = __ldcg(p.d.sk[1] + b0 + q0 + mid);
+                    const bool lt = bk < xk || (bk == xk && __ldcg(p.d.sv[1] + b0 + q0 + mid) < xv);
+                    if (lt) lo = mid + 1; else hi = mid;
+                }
+                c = q0 + lo;
+            }
+            cnt += c;
+        }
+        s_cnt[warp][lane] = cnt;
         __syncthreads();
-        for (uint32_t q = threadIdx.x; q < tn; q += blockDim.x) { sk[q] = gk[t0 + q]; sv[q] = gv[t0 + q]; }
-        __syncthreads();
-        const uint32_t k0 = kb * kRankKeys, kn = min((uint32_t)kRankKeys, nI - k0);
-        for (uint32_t q = threadIdx.x; q < kn; q += blockDim.x) {
-            const uint32_t k = k0 + q;
-            const uint64_t kk = gk[k];
-            const uint32_t vk = gv[k];
-            uint32_t lo = 0, hi = tn;
-            while (lo < hi) { const uint32_t m = (lo + hi) >> 1; if (kv_less(sk[m], sv[m], kk, vk)) lo = m + 1; else hi = m; }
-            const unsigned long long old = atomicAdd(&p.d.rank[k], (1ull << 32) | lo);
-            if ((old >> 32) + 1 == T - 1) write_i_entry(p, (uint32_t)old + lo, nI, vk);
+        if (warp == 0 && has) {
+            uint32_t rank = g - ta * kSortTile;  // index inside its own tile
+#pragma unroll
+            for (int w = 0; w < kWarps; ++w) rank += s_cnt[w][lane];
+            write_i_entry(p, rank, nI, xv, ld_alloc(p.a.alloc + xv));
         }
     }
     pdl_trigger();
@@ -896,18 +1017,39 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         for (uint32_t g0 = 0; g0 < nn;) {
             const uint32_t ng = min((uint32_t)kNodeGrp, nn - g0);
             for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
+            for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
             if (tid == 0) S.gnext = 0xFFFFFFFFu;
             __syncthreads();
-            for (uint32_t pr = tid; pr < ng * mw; pr += kThreads) {
-                const uint32_t u = pr / mw, w = pr % mw;
-                const uint32_t t = S.nt[u];
-                uint32_t bits = 0;
-#pragma unroll 8
-                for (uint32_t b = 0; b < 32; ++b) {
-                    const uint32_t e = w * 32 + b;
-                    bits |= (e < m && S.wta[e] < t && t < S.wtf[e]) ? 1u << b : 0u;
+            // entry e is live at the nodes u0 <= u < u1 of the group (t_alloc < t_u < t_free):
+            // toggle bit e at u0 and u1, then a prefix XOR over u yields the masks
+            for (uint32_t e = tid; e < m; e += kThreads) {
+                const uint32_t ta = S.wta[e], tf = S.wtf[e];
+                uint32_t lo = 0, hi = ng;  // u0 = #{u : t_u <= t_alloc}
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt[mid] <= ta) lo = mid + 1; else hi = mid; }
+                const uint32_t u0 = lo;
+                hi = ng;  // u1 = #{u : t_u < t_free}
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt[mid] < tf) lo = mid + 1; else hi = mid; }
+                const uint32_t u1 = lo;
+                if (u0 < u1) {
+                    atomicXor(&S.live[u0][e >> 5], 1u << (e & 31));
+                    if (u1 < ng) atomicXor(&S.live[u1][e >> 5], 1u << (e & 31));
                 }
-                S.live[u][w] = bits;
+            }
+            __syncthreads();
+            static_assert(kNodeGrp == 128, "prefix XOR: 4 nodes per lane");
+            for (uint32_t w = warp; w < mw; w += kWarps) {  // one warp per mask word
+                uint32_t v[4], run = 0;
+#pragma unroll
+                for (int r = 0; r < 4; ++r) { v[r] = S.live[lane * 4 + r][w]; run ^= v[r]; v[r] = run; }
+                uint32_t incl = run;
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                    if (lane >= (uint32_t)d) incl ^= y;
+                }
+                const uint32_t before = incl ^ run;
+#pragma unroll
+                for (int r = 0; r < 4; ++r) S.live[lane * 4 + r][w] = v[r] ^ before;
             }
             __syncthreads();
             uint32_t gnext = 0xFFFFFFFFu;
@@ -943,9 +1085,6 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     }
     __syncthreads();
     TL_PHASE(4, 13, tl_p);  // D: window search
-    // (phases A-D read only what k_trace / k_prepare wrote; the I list, fences
-    //  and summaries come from k_rank, this launch's PDL predecessor)
-    pdl_wait();
     for (uint32_t f = tid; f < nf; f += kThreads) S.fence[f] = p.d.fence[f];
     __syncthreads();
     // E. I list, for the candidates still unresolved, compacted into a queue first
@@ -1019,7 +1158,6 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
     const MaterializeArgs& a = p.a;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
     {  // I-I: sorted neighbours must not overlap (all of I is live at the last launch)
         const uint32_t k = cta * blockDim.x + threadIdx.x;
@@ -1091,6 +1229,7 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
 __global__ void __launch_bounds__(kThreads, 4) k_scan_words(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
     if (blockIdx.x < p.C) {
         classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
         TL_REC(4, 0, tl0);
@@ -1173,6 +1312,8 @@ struct Scratch {
     std::vector<void*> bufs;
     Ctl* h_ctl = nullptr;
     int sm_count = 0;
+    cudaStream_t side = nullptr;  // the I-list sort branch (forked from / joined to the caller's stream)
+    cudaEvent_t fork = nullptr, join = nullptr;
 };
 std::mutex g_mu;
 std::vector<Scratch*> g_scratch;
@@ -1225,7 +1366,7 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
     if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.rng, N)) ||
         (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) || (e = grow(s, s.d.sk[0], N)) ||
         (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) || (e = grow(s, s.d.sv[1], N)) ||
-        (e = grow(s, s.d.rank, N)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
+        (e = grow(s, s.d.samp_k, N / 32 + 64)) || (e = grow(s, s.d.samp_v, N / 32 + 64)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
         (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
         (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)))
         return e;
@@ -1250,7 +1391,11 @@ Scratch* device_scratch(cudaError_t* e) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
         const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
         cudaFuncSetAttribute(k_scan_words, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem);
-        cudaFuncSetAttribute(k_prepare, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(PrepShared));
+        cudaFuncSetAttribute(k_isort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SortShared));
+        if ((*e = cudaStreamCreateWithFlags(&s.side, cudaStreamNonBlocking)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess)
+            return nullptr;
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
     return &s;
@@ -1276,14 +1421,25 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
     }
     if (n) {
+        // the registration lists are scattered on a forked branch while the caller's
+        // stream sorts and ranks the I list (its few fat CTAs are dispatched first,
+        // as PDL successors of k_trace); the branch joins before k_scan_words
+        if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(s.side, s.fork, 0))) return e;
         {
-            TimedLaunch tl("mat_prepare", stream);
-            if ((e = launch_pdl(k_prepare, sort_ctas + alloc_ctas, kThreads, sizeof(PrepShared), stream, p))) return e;
+            TimedLaunch tl("mat_isort", stream);
+            if ((e = launch_pdl(k_isort, sort_ctas, kSortThreads, sizeof(SortShared), stream, p))) return e;
         }
-        TimedLaunch tl("mat_rank", stream);
-        const uint64_t jobs = (uint64_t)sort_ctas * ((n + kRankKeys - 1) / kRankKeys);
-        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(jobs, (uint64_t)s.sm_count * 8));
-        if ((e = launch_pdl(k_rank, grid, kThreads, 0, stream, p))) return e;
+        {
+            TimedLaunch tl("mat_rank", stream);
+            // one CTA per 32 I keys (the list's size is known on the device only: bound
+            // by the allocation count; surplus CTAs exit at once)
+            if ((e = launch_pdl(k_rank, (unsigned)((n + 31) / 32), kThreads, 0, stream, p))) return e;
+        }
+        {
+            TimedLaunch tl("mat_prepare", s.side);
+            k_prepare<<<alloc_ctas, kThreads, 0, s.side>>>(p);
+        }
+        if ((e = cudaEventRecord(s.join, s.side)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     }
     if (C + check_ctas) {
         TimedLaunch tl("mat_classify", stream);
