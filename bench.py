@@ -408,7 +408,8 @@ def run_ours(args):
             "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
             "gpu_launches": len(launches),
             "graph_step": "one CUDA graph per step: medusa_materialize_async, medusa_kernel_table_set, "
-                          "medusa_restore(MEDUSA_N_SLOTS_FROM_TABLE); 9 libmedusa kernels per step",
+                          f"medusa_restore(MEDUSA_N_SLOTS_FROM_TABLE); {len(launches) // max(args.steps, 1)} "
+                          "libmedusa kernels per step",
             "sync_api_ms_per_step": max_over_ranks(sum(sync_ms), dist, dev) / args.steps,
             "instrumented_ms_per_step": sum(inst_ms) / args.steps,
             "clocks": clocks,

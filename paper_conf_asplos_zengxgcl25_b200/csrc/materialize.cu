@@ -54,7 +54,7 @@ constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
-constexpr int kSortTile = 2048;    // keys sorted per CTA before ranking
+constexpr int kSortTile = 1024;    // I keys sorted per CTA before ranking
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
 constexpr int kWinCap = 128;       // mortal-window entries per batch (<= 4 per lane of one warp)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
@@ -71,12 +71,19 @@ struct Ctl {
     unsigned long long gmax;    // greatest end
     unsigned long long need_c, need_b;  // set (exactly) only when a registration list overflowed
     unsigned long long n_slots;
+    unsigned long long n_queue;  // entries in the I-list queue
 };
 
 struct IRest {  // I-list entry (sorted order), base kept in a separate array
     uint64_t end;
     uint32_t t_alloc;
     uint32_t id;
+};
+
+struct IQ {  // a candidate word for the I-list search (k_iresolve)
+    uint64_t x;  // the word
+    uint32_t g;  // its index in the image
+    uint32_t t;  // launch position of its node
 };
 
 struct WinRec {  // a registered mortal allocation
@@ -111,7 +118,9 @@ struct Dev {  // scratch of one call (device pointers)
     uint32_t* i_tf;                              // [n]
     uint64_t* fence;                             // [kFenceCap]
     uint32_t* chunk_cnt;                         // [C] slots per chunk
-    uint64_t* staging;                           // [n_words] records, warp-dense per 32 words
+    uint64_t* staging;                           // [n_words] record of slot g at index g
+    IQ* queue;                                   // [cap_q] candidates for the I-list search
+    uint64_t cap_q;
 };
 
 struct P {  // kernel parameters
@@ -119,7 +128,7 @@ struct P {  // kernel parameters
     Dev d;
     uint32_t C, nb;              // chunks, check blocks
     uint32_t node_ctas;          // k_trace: CTAs with the node role
-    uint32_t sort_ctas;          // k_isort: tiles of 2048 I keys (bound: allocation count / 2048)
+    uint32_t sort_ctas;          // k_prepare: CTAs with the sort role (bound: allocation count / kSortTile)
     uint32_t check_ctas;         // k_scan_words: CTAs with the check role (after the C classify CTAs)
 };
 
@@ -527,26 +536,24 @@ __device__ __forceinline__ void warp_bitonic_kv(uint64_t (&k)[E], uint32_t (&v)[
 }
 
 // ----------------------------------------------------------------------------
-// 2a. k_isort (side stream, parallel to k_prepare): one 1024-thread CTA per tile
-//     of 2048 I keys (base, allocation index).  A register bitonic sort of 64
-//     keys per warp, then five merge-path rounds through shared memory
-//     (64 -> 128 -> ... -> 2048), two keys per thread held in registers between
-//     rounds.  A single tile is the whole list: its I entries are written here.
-constexpr int kSortThreads = 1024;
+// 2a. sort role of k_prepare (its first CTAs, dispatched ahead of the scatter
+//     CTAs): one tile of kSortTile I keys (base, allocation index) per CTA.  A
+//     register bitonic sort of 128 keys per warp, then three merge-path rounds
+//     through shared memory (128 -> 256 -> 512 -> 1024), four keys per thread held
+//     in registers between rounds.  A single tile is the whole list: its I entries
+//     are written here; otherwise every 32nd key is the tile's sample for k_rank.
+constexpr int kSortThreads = kThreads;
 constexpr int kSortPer = kSortTile / kSortThreads;  // 2
 struct SortShared {
     uint64_t k[kSortTile];
     uint32_t v[kSortTile];
 };
 
-__global__ void __launch_bounds__(kSortThreads) k_isort(P p) {
-    extern __shared__ __align__(16) unsigned char sort_raw[];
-    SortShared& S = *reinterpret_cast<SortShared*>(sort_raw);
+__device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
     const unsigned long long tl0 = TL_NOW();
     unsigned long long tl_p = tl0;
-    pdl_wait();
     const uint32_t n = p.d.ctl->nI;
-    const uint32_t t0 = blockIdx.x * kSortTile;
+    const uint32_t t0 = tile * kSortTile;
     if (t0 < n) {
         const uint32_t o = threadIdx.x * kSortPer;  // this thread's consecutive elements
         uint64_t k[kSortPer];
@@ -611,7 +618,6 @@ __global__ void __launch_bounds__(kSortThreads) k_isort(P p) {
         }
         TL_REC(2, 0, tl0);
     }
-    pdl_trigger();
 }
 
 // One registration list (chunks or check blocks): the CTA's 256 allocations
@@ -700,11 +706,18 @@ __device__ void scatter_role(const P& p, uint32_t cta, ScatterShared& S) {
 }
 
 __global__ void __launch_bounds__(kThreads) k_prepare(P p) {
-    __shared__ ScatterShared S;
+    __shared__ union {
+        SortShared sort;
+        ScatterShared scatter;
+    } U;
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
-    scatter_role(p, blockIdx.x, S);
-    TL_REC(2, 1, tl0);
+    if (blockIdx.x < p.sort_ctas) {
+        sort_role(p, blockIdx.x, U.sort);
+    } else {
+        scatter_role(p, blockIdx.x - p.sort_ctas, U.scatter);
+        TL_REC(2, 1, tl0);
+    }
     pdl_trigger();
 }
 
@@ -841,12 +854,14 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 // 4. k_scan_words: classify CTAs (one per chunk) and check CTAs
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
-    uint64_t fence[kFenceCap];
     uint32_t tw[MEDUSA_CHUNK_WORDS];     // node of every word, as an index from the chunk's first node
-    uint64_t wb[kWinCap], we[kWinCap];   // window sorted by (base, t_alloc)
+    uint64_t rb[kWinCap], re[kWinCap];   // one batch of registered mortals as loaded
+    uint32_t rta[kWinCap], rtf[kWinCap], rid[kWinCap];
+    uint64_t wb[kWinCap], we[kWinCap];   // the batch sorted by (base, t_alloc)
     uint32_t wta[kWinCap], wtf[kWinCap], wid[kWinCap];
     uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
-    uint32_t nt[kNodeGrp];                  // launch positions of nodes g0 .. g0 + kNodeGrp
+    uint32_t nt0[kNodeGrp];                 // launch positions of the chunk's first kNodeGrp nodes
+    uint32_t nt[kNodeGrp];                  // launch positions of nodes g0 .. g0 + kNodeGrp (later groups)
     uint32_t gnext;
     uint16_t cq[MEDUSA_CHUNK_WORDS];     // candidate words, then the I-list queue
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32];
@@ -855,34 +870,35 @@ struct ClsShared {
     unsigned long long mbar;
 };
 
-struct ChkShared {
-    uint64_t fence[kFenceCap];
-    uint64_t base[kWarps][kChkCap], end[kWarps][kChkCap];
-    uint32_t tf[kWarps][kChkCap], idx[kWarps][kChkCap];
-};
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-// warp 0: a batch of <= kWinCap registered mortals sorted by (base, t_alloc) in
-// registers, laid out in shared memory
+// threads 0..kWinCap-1: one batch of <= kWinCap registered mortals -> S.r*
+__device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
+    const uint32_t e = threadIdx.x;
+    if (e < m) {
+        const WinRec x = p.d.list_c[bs + e];
+        S.rb[e] = x.base;
+        S.re[e] = x.end;
+        S.rta[e] = x.t_alloc;
+        S.rtf[e] = x.t_free;
+        S.rid[e] = x.id;
+    }
+}
+
+// warp 0: the loaded batch sorted by (base, t_alloc) in registers, permuted into S.w*
 template <int E>
-__device__ __forceinline__ void window_prepare_e(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
+__device__ __forceinline__ void window_sort_e(ClsShared& S, uint32_t m) {
     const uint32_t lane = threadIdx.x & 31;
     uint64_t k[E];
     uint32_t v[E], pl[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
         const uint32_t e = lane * E + r;
-        if (e < m) {
-            const WinRec& x = p.d.list_c[bs + e];
-            k[r] = x.base;
-            v[r] = x.t_alloc;
-        } else {
-            k[r] = ~0ull;
-            v[r] = 0xFFFFFFFFu;
-        }
+        k[r] = e < m ? S.rb[e] : ~0ull;
+        v[r] = e < m ? S.rta[e] : 0xFFFFFFFFu;
         pl[r] = e;
     }
     warp_bitonic<E>(k, v, pl);
@@ -890,20 +906,20 @@ __device__ __forceinline__ void window_prepare_e(const P& p, ClsShared& S, uint6
     for (int r = 0; r < E; ++r) {
         const uint32_t e = lane * E + r;
         if (e < m) {
-            const WinRec x = p.d.list_c[bs + pl[r]];
-            S.wb[e] = x.base;
-            S.we[e] = x.end;
-            S.wta[e] = x.t_alloc;
-            S.wtf[e] = x.t_free;
-            S.wid[e] = x.id;
+            const uint32_t q = pl[r];
+            S.wb[e] = k[r];
+            S.we[e] = S.re[q];
+            S.wta[e] = v[r];
+            S.wtf[e] = S.rtf[q];
+            S.wid[e] = S.rid[q];
         }
     }
 }
 
-__device__ __forceinline__ void window_prepare(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
-    if (m <= 32) window_prepare_e<1>(p, S, bs, m);
-    else if (m <= 64) window_prepare_e<2>(p, S, bs, m);
-    else window_prepare_e<4>(p, S, bs, m);
+__device__ __forceinline__ void window_sort(ClsShared& S, uint32_t m) {
+    if (m <= 32) window_sort_e<1>(S, m);
+    else if (m <= 64) window_sort_e<2>(S, m);
+    else window_sort_e<4>(S, m);
 }
 
 __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
@@ -915,46 +931,54 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
     const uint64_t* gsrc = a.words + cs;
     const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
-    // A. the chunk's words -> shared memory with one bulk copy (TMA engine)
+    const uint32_t tx = tma ? n * 8 : 0;
+    const uint32_t mb = smem_u32(&S.mbar);
+    // A. one TMA transaction brings the chunk's words to shared memory; meanwhile
+    //    the list offsets (block_prefix) and the chunk's node range load
     if (tid == 0) {
         S.nc = 0;
         S.nq = 0;
         S.total = 0;
-        if (tma) {
-            const uint32_t mb = smem_u32(&S.mbar);
+        S.gnext = 0xFFFFFFFFu;
+        if (tx) {
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(tx) : "memory");
             asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                          ::"r"(smem_u32(S.words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
         }
     }
+    const uint32_t N = a.n_nodes;
+    const uint32_t jf = N ? min(__ldcg(p.d.jf + c), N - 1) : 0, jl = N ? min(__ldcg(p.d.jl + c), N - 1) : 0;
+    const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
-    const uint32_t nI = ctl->nI;
-    const uint32_t stride = fence_stride(nI);
-    const uint32_t nf = (nI + stride - 1) / stride;
-    const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
-    const uint32_t N = a.n_nodes;
     for (uint32_t q = tid; q < kChunkWords; q += kThreads) S.tw[q] = 0;
     if (tid < MEDUSA_CHUNK_WORDS / 32) S.hits[tid] = 0;
-    const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);
+    const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);  // (synchronizes the CTA)
     const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
-    __syncthreads();
-    TL_PHASE(4, 10, tl_p);  // A: setup, fences
-    // B. warp 0: first window batch; warps 1..7: node starts -> node index per word
-    const uint32_t jf = N ? min(p.d.jf[c], N - 1) : 0, jl = N ? min(p.d.jl[c], N - 1) : 0;
-    if (warp == 0) {
-        if (r0 < r1) window_prepare(p, S, r0, (uint32_t)min((uint64_t)kWinCap, r1 - r0));
-    } else if (N) {
-        for (uint32_t j = jf + 1 + (tid - 32); j <= jl; j += kThreads - 32) {
+    const uint32_t nn = N ? jl - jf + 1 : 0;
+    TL_PHASE(4, 10, tl_p);  // A: setup
+    // B. one round of loads: threads 0..127 the first window batch, threads
+    //    128..255 the chunk's node starts (-> node index per word) and the launch
+    //    positions of its first kNodeGrp nodes
+    const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
+    if (tid < kWinCap) {
+        window_load(p, S, r0, m0);
+    } else {
+        const uint32_t h = tid - kWinCap;
+        for (uint32_t j = jf + 1 + h; j <= jl; j += kThreads - kWinCap) {
             const uint64_t q = a.node_off[j] - cs;
             if (q < n) atomicMax(&S.tw[q], j - jf);
         }
+        if (h < kNodeGrp && h < nn) S.nt0[h] = a.node_t[jf + h];
     }
     __syncthreads();
-    TL_PHASE(4, 11, tl_p);  // B: first window, node starts
-    {  // running max over the chunk: tw[q] = index (from jf) of the node holding word q
+    TL_PHASE(4, 11, tl_p);  // B: window records, node starts
+    // warp 0 sorts the window batch; all warps: running max over the chunk,
+    // tw[q] = index (from jf) of the node holding word q
+    if (warp == 0 && m0) window_sort(S, m0);
+    {
         uint32_t loc[kWordsPerThread];
         uint32_t run = 0;
 #pragma unroll
@@ -973,8 +997,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 #pragma unroll
         for (int k = 0; k < kWordsPerThread; ++k) S.tw[tid * kWordsPerThread + k] = max(before, loc[k]);
     }
-    if (tma) {
-        const uint32_t mb = smem_u32(&S.mbar);
+    if (tx) {
         uint32_t done = 0;
         while (!done) {
             asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
@@ -997,7 +1020,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         if (cand) S.cq[base + __popc(bal & lanemask_lt())] = (uint16_t)q;
     }
     __syncthreads();
-    TL_PHASE(4, 12, tl_p);  // C: launch positions, TMA wait, candidates
+    TL_PHASE(4, 12, tl_p);  // C: window sort, launch positions, TMA wait, candidates
     const uint32_t nc = S.nc;
     // D. mortal window(s).  The entries live at one launch are pairwise disjoint,
     //    so the only possible container of word x of node u is the live entry
@@ -1005,30 +1028,31 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     //    shared memory, one AND with node u's live mask (bit e = entry e live at
     //    u's launch), one leading-zero count, one end check.  Masks are built per
     //    batch of <= kWinCap entries and group of kNodeGrp nodes.
-    const uint32_t nn = N ? jl - jf + 1 : 0;
     for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
         const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
-        if (bs != r0) {
+        if (bs != r0) {  // a further batch (windows of more than kWinCap entries)
+            window_load(p, S, bs, m);
             __syncthreads();
-            if (warp == 0) window_prepare(p, S, bs, m);
+            if (warp == 0) window_sort(S, m);
             __syncthreads();
         }
         const uint32_t mw = (m + 31) / 32;
         for (uint32_t g0 = 0; g0 < nn;) {
             const uint32_t ng = min((uint32_t)kNodeGrp, nn - g0);
-            for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
+            const uint32_t* nt = g0 ? S.nt : S.nt0;
+            if (g0)
+                for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
             for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
-            if (tid == 0) S.gnext = 0xFFFFFFFFu;
             __syncthreads();
             // entry e is live at the nodes u0 <= u < u1 of the group (t_alloc < t_u < t_free):
             // toggle bit e at u0 and u1, then a prefix XOR over u yields the masks
             for (uint32_t e = tid; e < m; e += kThreads) {
                 const uint32_t ta = S.wta[e], tf = S.wtf[e];
                 uint32_t lo = 0, hi = ng;  // u0 = #{u : t_u <= t_alloc}
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt[mid] <= ta) lo = mid + 1; else hi = mid; }
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] <= ta) lo = mid + 1; else hi = mid; }
                 const uint32_t u0 = lo;
                 hi = ng;  // u1 = #{u : t_u < t_free}
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt[mid] < tf) lo = mid + 1; else hi = mid; }
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] < tf) lo = mid + 1; else hi = mid; }
                 const uint32_t u1 = lo;
                 if (u0 < u1) {
                     atomicXor(&S.live[u0][e >> 5], 1u << (e & 31));
@@ -1079,19 +1103,19 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
             __syncthreads();
             const uint32_t gn = S.gnext;  // next group holding an unresolved candidate
             __syncthreads();
+            if (tid == 0) S.gnext = 0xFFFFFFFFu;
             if (gn == 0xFFFFFFFFu) break;
             g0 = gn;
         }
     }
     __syncthreads();
     TL_PHASE(4, 13, tl_p);  // D: window search
-    for (uint32_t f = tid; f < nf; f += kThreads) S.fence[f] = p.d.fence[f];
-    __syncthreads();
-    // E. I list, for the candidates still unresolved, compacted into a queue first
-    if (nI) {
-        const uint64_t f0 = S.fence[0];
+    // E. the candidates no mortal holds go to the I-list queue (k_iresolve);
+    //    one queue reservation per CTA
+    {
         uint32_t qv[kWordsPerThread];
         bool need[kWordsPerThread];
+        uint32_t mine = 0;
 #pragma unroll
         for (int k = 0; k < kWordsPerThread; ++k) {
             const uint32_t i = k * kThreads + tid;
@@ -1100,36 +1124,27 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
             if (i < nc) {
                 const uint32_t q = S.cq[i];
                 qv[k] = q;
-                need[k] = !((S.hits[q >> 5] >> (q & 31)) & 1u) && S.words[q] >= f0;
+                need[k] = !((S.hits[q >> 5] >> (q & 31)) & 1u);
             }
+            mine += need[k] ? 1u : 0u;
         }
-        __syncthreads();  // cq is rewritten below
+        uint32_t total;
+        const uint32_t pre = block_excl_scan(mine, &total);
+        if (tid == 0 && total) S.nq = (uint32_t)atomicAdd(&ctl->n_queue, (unsigned long long)total);
+        __syncthreads();
+        uint64_t pos = (uint64_t)S.nq + pre;
 #pragma unroll
         for (int k = 0; k < kWordsPerThread; ++k) {
-            const uint32_t bal = __ballot_sync(0xffffffffu, need[k]);
-            uint32_t base = 0;
-            if (lane == 0 && bal) base = atomicAdd(&S.nq, (uint32_t)__popc(bal));
-            base = __shfl_sync(0xffffffffu, base, 0);
-            if (need[k]) S.cq[base + __popc(bal & lanemask_lt())] = (uint16_t)qv[k];
-        }
-        __syncthreads();
-        const uint32_t nq = S.nq;
-        for (uint32_t i = tid; i < nq; i += kThreads) {
-            const uint32_t q = S.cq[i];
-            const uint64_t x = S.words[q];
-            const uint32_t t = __ldg(a.node_t + jf + S.tw[q]);  // launch position of the word's node
-            const uint32_t kk = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x) - 1;
-            const uint64_t base = p.d.i_base[kk];
-            const IRest e = p.d.i_rest[kk];
-            if (x < e.end && e.t_alloc < t) {
-                S.words[q] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (x - base);
-                atomicOr(&S.hits[q >> 5], 1u << (q & 31));
-            }
+            if (!need[k]) continue;
+            const uint32_t q = qv[k];
+            const uint32_t u = S.tw[q];
+            const uint32_t t = u < kNodeGrp ? S.nt0[u] : __ldg(a.node_t + jf + u);  // the word's launch position
+            if (pos < p.d.cap_q) p.d.queue[pos] = IQ{S.words[q], (uint32_t)(cs + q), t};
+            ++pos;
         }
     }
-    __syncthreads();
-    TL_PHASE(4, 14, tl_p);  // E: I-list search
-    // F. emission: mask words, warp-dense staging of records, chunk count
+    TL_PHASE(4, 14, tl_p);  // E: queue
+    // F. emission: mask words, records at their word index, the chunk's count
     const uint64_t n_mask = (a.n_words + 31) / 32;
     uint32_t cnt = 0;
 #pragma unroll
@@ -1138,14 +1153,14 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         const uint32_t bits = S.hits[q >> 5];
         const uint64_t mw = (cs + q) >> 5;
         if (lane == 0 && mw < n_mask) a.mask[mw] = bits;
-        if ((bits >> lane) & 1u) p.d.staging[(cs + q - lane) + __popc(bits & lanemask_lt())] = S.words[q];
+        if ((bits >> lane) & 1u) p.d.staging[cs + q] = S.words[q];
         cnt += __popc(bits);
     }
     if (lane == 0) atomicAdd(&S.total, cnt);
     __syncthreads();
     TL_PHASE(4, 15, tl_p);  // F: emission
-    // G. the chunk's slot count and its 256-chunk group sum (k_emit turns them
-    //    into chunk_base)
+    // G. the chunk's slot count so far and its 256-chunk group sum (k_iresolve
+    //    adds the I-list slots; k_emit turns them into chunk_base)
     if (tid == 0) {
         p.d.chunk_cnt[c] = S.total;
         if (S.total) atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)S.total);
@@ -1153,9 +1168,16 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     pdl_trigger();
 }
 
-// one warp per block of 32 allocation ordinals; the CTA also checks 256 adjacent
-// pairs of the sorted I list
-__device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
+// ----------------------------------------------------------------------------
+// 2d. k_check_mi (after k_rank): I-I (adjacent sorted I entries; the CTA checks
+//     256 pairs) and M-I (each mortal against the run of I entries its range
+//     meets, one warp per 32 allocation ordinals)
+__global__ void __launch_bounds__(kThreads) k_check_mi(P p) {
+    __shared__ uint64_t s_fence[kFenceCap];
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
+    pdl_trigger();
+    const uint32_t cta = blockIdx.x;
     const MaterializeArgs& a = p.a;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t nI = p.d.ctl->nI;
@@ -1165,15 +1187,11 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
     }
     const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) S.fence[f] = p.d.fence[f];
-    // list offsets of this CTA's kWarps check blocks
-    const uint32_t b0 = cta * kWarps;
-    const unsigned long long base = block_prefix(p.d.cnt_b, p.d.sup_b, min(b0, p.nb));
-    const uint32_t b = b0 + warp;
-    if (b >= p.nb) return;  // whole warp
-    const uint32_t cb = (lane <= warp && b0 + lane < p.nb) ? __ldcg(p.d.cnt_b + b0 + lane) : 0u;
-    const uint32_t before = __reduce_add_sync(0xffffffffu, lane < warp ? cb : 0u);
+    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = p.d.fence[f];
+    __syncthreads();
+    const uint32_t b = cta * kWarps + warp;
     const uint32_t j = b * kAblk + lane;
+    if (b >= p.nb || !nI) return;  // whole warp
     bool mine = false;
     medusa_alloc x{};
     const uint32_t N = a.n_nodes;
@@ -1184,33 +1202,10 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
     }
     const uint64_t xe = x.base + x.size;
     bool bad = false;
-    // M-M: mortals registered as live at some allocation of this block
-    const uint64_t r0 = base + before;
-    const uint64_t r1 = min(r0 + __shfl_sync(0xffffffffu, cb, warp), p.d.cap_b);
-    for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
-        const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
-        __syncwarp();
-        for (uint32_t q = lane; q < m; q += 32) {
-            const WinRec y = p.d.list_b[bs + q];
-            S.base[warp][q] = y.base;
-            S.end[warp][q] = y.end;
-            S.tf[warp][q] = y.t_free;
-            S.idx[warp][q] = y.id;
-        }
-        __syncwarp();
-        if (mine && !bad) {
-            for (uint32_t q = 0; q < m; ++q) {
-                if (S.idx[warp][q] < j && S.tf[warp][q] > x.t_alloc && S.base[warp][q] < xe && x.base < S.end[warp][q]) {
-                    bad = true;
-                    break;
-                }
-            }
-        }
-    }
     // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
-    if (mine && !bad && nI) {
-        const uint32_t e = i_count_le(S.fence, nf, stride, nI, p.d.i_base, xe - 1);  // bases < end
-        const uint32_t k0 = i_count_le(S.fence, nf, stride, nI, p.d.i_base, x.base);
+    if (mine) {
+        const uint32_t e = i_count_le(s_fence, nf, stride, nI, p.d.i_base, xe - 1);  // bases < end
+        const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);
         const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
         // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
         const bool freed_early = x.t_free <= t_last;
@@ -1223,27 +1218,124 @@ __device__ void check_role(const P& p, uint32_t cta, ChkShared& S) {
             bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
     }
     if (bad) flag(p.d.ctl, ST_TRACE);
+    TL_REC(9, 0, tl0);
+}
+
+// ----------------------------------------------------------------------------
+// 2c. k_check_mm (forked branch, after k_prepare): M-M -- every mortal j against
+//     the mortals registered as live at some allocation of its block of 32
+//     ordinals (one warp per block); runs while the I list is sorted and ranked.
+__global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
+    __shared__ uint64_t s_base[kWarps][kChkCap], s_end[kWarps][kChkCap];
+    __shared__ uint32_t s_tf[kWarps][kChkCap], s_idx[kWarps][kChkCap];
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
+    const MaterializeArgs& a = p.a;
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t b0 = blockIdx.x * kWarps;
+    const unsigned long long base = block_prefix(p.d.cnt_b, p.d.sup_b, min(b0, p.nb));
+    const uint32_t b = b0 + warp;
+    if (b < p.nb) {
+        const uint32_t cb = (lane <= warp && b0 + lane < p.nb) ? __ldcg(p.d.cnt_b + b0 + lane) : 0u;
+        const uint32_t before = __reduce_add_sync(0xffffffffu, lane < warp ? cb : 0u);
+        const uint32_t j = b * kAblk + lane;
+        bool mine = false;
+        medusa_alloc x{};
+        const uint32_t N = a.n_nodes;
+        const uint32_t t_last = N ? a.node_t[N - 1] : 0;
+        if (j < a.n_alloc) {
+            x = a.alloc[j];
+            mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
+        }
+        const uint64_t xe = x.base + x.size;
+        bool bad = false;
+        const uint64_t r0 = base + before;
+        const uint64_t r1 = min(r0 + __shfl_sync(0xffffffffu, cb, warp), p.d.cap_b);
+        for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
+            const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
+            __syncwarp();
+            for (uint32_t q = lane; q < m; q += 32) {
+                const WinRec y = p.d.list_b[bs + q];
+                s_base[warp][q] = y.base;
+                s_end[warp][q] = y.end;
+                s_tf[warp][q] = y.t_free;
+                s_idx[warp][q] = y.id;
+            }
+            __syncwarp();
+            if (mine && !bad) {
+                for (uint32_t q = 0; q < m; ++q) {
+                    if (s_idx[warp][q] < j && s_tf[warp][q] > x.t_alloc && s_base[warp][q] < xe && x.base < s_end[warp][q]) {
+                        bad = true;
+                        break;
+                    }
+                }
+            }
+        }
+        if (bad) flag(p.d.ctl, ST_TRACE);
+        TL_REC(8, 0, tl0);
+    }
     pdl_trigger();
 }
 
-__global__ void __launch_bounds__(kThreads, 4) k_scan_words(P p) {
+__global__ void __launch_bounds__(kThreads, 4) k_classify(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
-    if (blockIdx.x < p.C) {
-        classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
-        TL_REC(4, 0, tl0);
-    } else {
-        check_role(p, blockIdx.x - p.C, *reinterpret_cast<ChkShared*>(smem_raw));
-        TL_REC(4, 1, tl0);
+    classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
+    TL_REC(4, 0, tl0);
+}
+
+// ----------------------------------------------------------------------------
+// 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
+//     sorted I list -- fences in shared memory, then per candidate one group of
+//     bases and one entry (two dependent loads).  A hit writes its record at its
+//     word index, sets its mask bit and counts toward its chunk.
+__global__ void __launch_bounds__(kThreads) k_iresolve(P p) {
+    __shared__ uint64_t s_fence[kFenceCap];
+    const unsigned long long tl0 = TL_NOW();
+    pdl_wait();
+    const Ctl* ctl = p.d.ctl;
+    const uint32_t nI = ctl->nI;
+    const uint64_t nq = min((uint64_t)ctl->n_queue, p.d.cap_q);
+    if (nI && nq > (uint64_t)blockIdx.x * kThreads) {
+        const uint32_t stride = fence_stride(nI);
+        const uint32_t nf = (nI + stride - 1) / stride;
+        for (uint32_t f = threadIdx.x; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
+        __syncthreads();
+        const uint64_t n_mask = (p.a.n_words + 31) / 32;
+        for (uint64_t i0 = (uint64_t)blockIdx.x * kThreads; i0 < nq; i0 += (uint64_t)gridDim.x * kThreads) {
+            const uint64_t i = i0 + threadIdx.x;
+            bool hit = false;
+            uint32_t g = 0;
+            if (i < nq) {
+                const IQ q = p.d.queue[i];
+                g = q.g;
+                const uint32_t cnt = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
+                if (cnt) {
+                    const uint32_t kk = cnt - 1;
+                    const uint64_t base = p.d.i_base[kk];
+                    const IRest e = p.d.i_rest[kk];
+                    if (q.x < e.end && e.t_alloc < q.t) {
+                        hit = true;
+                        p.d.staging[g] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
+                        if ((g >> 5) < n_mask) atomicOr(p.a.mask + (g >> 5), 1u << (g & 31));
+                    }
+                }
+            }
+            const uint32_t c = g / kChunkWords;
+            warp_agg_add(p.d.chunk_cnt, c, hit);
+            warp_group_add_range(p.d.chunk_sup, c, c, hit);
+        }
     }
+    pdl_trigger();
+    TL_REC(10, 0, tl0);
 }
 
 // ----------------------------------------------------------------------------
 // 5. k_emit: compaction of the staged records into the slot table (one CTA per
 //    chunk, one thread per output record: coalesced stores)
 __global__ void __launch_bounds__(kThreads) k_emit(P p) {
-    __shared__ uint32_t s_pre[65];
+    __shared__ uint32_t s_pre[65], s_m[64];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const MaterializeArgs& a = p.a;
@@ -1263,7 +1355,9 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     }
     if (warp < 2) {
         const uint64_t mw = m0 + warp * 32 + lane;
-        const uint32_t pc = mw < n_mask ? __popc(a.mask[mw]) : 0u;
+        const uint32_t mv = mw < n_mask ? __ldcg(a.mask + mw) : 0u;
+        const uint32_t pc = __popc(mv);
+        s_m[warp * 32 + lane] = mv;
         uint32_t incl = pc;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
@@ -1281,7 +1375,8 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
         uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
         while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
         const uint64_t dst = prefix + r;
-        if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + (r - s_pre[lo])];
+        const uint32_t bit = __fns(s_m[lo], 0, (int)(r - s_pre[lo]) + 1);  // the (r - s_pre[lo])-th set bit
+        if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + bit];
     }
     pdl_trigger();
     TL_REC(5, 0, tl0);
@@ -1313,7 +1408,7 @@ struct Scratch {
     Ctl* h_ctl = nullptr;
     int sm_count = 0;
     cudaStream_t side = nullptr;  // the I-list sort branch (forked from / joined to the caller's stream)
-    cudaEvent_t fork = nullptr, join = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr, join2 = nullptr, lists = nullptr;
 };
 std::mutex g_mu;
 std::vector<Scratch*> g_scratch;
@@ -1368,8 +1463,9 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
         (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) || (e = grow(s, s.d.sv[1], N)) ||
         (e = grow(s, s.d.samp_k, N / 32 + 64)) || (e = grow(s, s.d.samp_v, N / 32 + 64)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
         (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
-        (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)))
+        (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)) || (e = grow(s, s.d.queue, WW)))
         return e;
+    s.d.cap_q = WW;
     s.d.cap_c = RC;
     s.d.cap_b = RB;
     s.cap_n = N; s.cap_C = CC; s.cap_nb = NB; s.cap_c = RC; s.cap_b = RB; s.cap_w = WW;
@@ -1389,19 +1485,26 @@ Scratch* device_scratch(cudaError_t* e) {
     Scratch& s = *g_scratch[dev];
     if (!s.h_ctl) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
-        const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
-        cudaFuncSetAttribute(k_scan_words, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem);
-        cudaFuncSetAttribute(k_isort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SortShared));
-        if ((*e = cudaStreamCreateWithFlags(&s.side, cudaStreamNonBlocking)) != cudaSuccess ||
+        cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ClsShared));
+        int prio_lo = 0, prio_hi = 0;
+        cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+        if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
-            (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess)
+            (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.join2, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.lists, cudaEventDisableTiming)) != cudaSuccess)
             return nullptr;
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
     return &s;
 }
 
-// the whole analysis on `stream` (no synchronization)
+// the whole analysis on `stream` (no synchronization).  After k_prepare (I-list
+// tile sort + registration lists) two branches:
+//   stream:           k_classify ------------------------------ [join] k_iresolve -> k_emit
+//   side (high prio): k_rank -> k_check_mi -> k_check_mm -> [join]
+// The side stream's higher priority gets the rank CTAs dispatched ahead of the
+// classify CTAs; k_iresolve needs both branches.
 cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P* out) {
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
@@ -1410,7 +1513,6 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     const uint32_t alloc_ctas = (uint32_t)((n + kThreads - 1) / kThreads);
     const uint32_t sort_ctas = (uint32_t)((n + kSortTile - 1) / kSortTile);
     const uint32_t check_ctas = n ? std::max<uint32_t>((nb + kWarps - 1) / kWarps, alloc_ctas) : 0;
-    const size_t scan_smem = std::max(sizeof(ClsShared), sizeof(ChkShared));
     P p{a, s.d, C, nb, node_ctas, sort_ctas, check_ctas};
     *out = p;
     cudaError_t e;
@@ -1421,29 +1523,38 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
     }
     if (n) {
-        // the registration lists are scattered on a forked branch while the caller's
-        // stream sorts and ranks the I list (its few fat CTAs are dispatched first,
-        // as PDL successors of k_trace); the branch joins before k_scan_words
+        {
+            TimedLaunch tl("mat_prepare", stream);
+            if ((e = launch_pdl(k_prepare, sort_ctas + alloc_ctas, kThreads, 0, stream, p))) return e;
+        }
         if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(s.side, s.fork, 0))) return e;
         {
-            TimedLaunch tl("mat_isort", stream);
-            if ((e = launch_pdl(k_isort, sort_ctas, kSortThreads, sizeof(SortShared), stream, p))) return e;
-        }
-        {
-            TimedLaunch tl("mat_rank", stream);
+            TimedLaunch tl("mat_rank", s.side);
             // one CTA per 32 I keys (the list's size is known on the device only: bound
             // by the allocation count; surplus CTAs exit at once)
-            if ((e = launch_pdl(k_rank, (unsigned)((n + 31) / 32), kThreads, 0, stream, p))) return e;
+            k_rank<<<(unsigned)((n + 31) / 32), kThreads, 0, s.side>>>(p);
         }
         {
-            TimedLaunch tl("mat_prepare", s.side);
-            k_prepare<<<alloc_ctas, kThreads, 0, s.side>>>(p);
+            TimedLaunch tl("mat_check_mi", s.side);
+            if ((e = launch_pdl(k_check_mi, check_ctas, kThreads, 0, s.side, p))) return e;
         }
-        if ((e = cudaEventRecord(s.join, s.side)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
-    }
-    if (C + check_ctas) {
+        {
+            TimedLaunch tl("mat_check_mm", s.side);
+            if ((e = launch_pdl(k_check_mm, (nb + kWarps - 1) / kWarps, kThreads, 0, s.side, p))) return e;
+        }
+        if ((e = cudaEventRecord(s.join, s.side))) return e;
+        if (C) {
+            TimedLaunch tl("mat_classify", stream);
+            if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
+        }
+        if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
+        if (C) {
+            TimedLaunch tl("mat_iresolve", stream);
+            if ((e = launch_pdl(k_iresolve, (unsigned)s.sm_count * 8, kThreads, 0, stream, p))) return e;
+        }
+    } else if (C) {
         TimedLaunch tl("mat_classify", stream);
-        if ((e = launch_pdl(k_scan_words, C + check_ctas, kThreads, scan_smem, stream, p))) return e;
+        if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
     }
     if (C) {
         TimedLaunch tl("mat_emit", stream);
