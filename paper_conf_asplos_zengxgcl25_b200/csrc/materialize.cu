@@ -71,7 +71,6 @@ struct Ctl {
     unsigned long long gmax;    // greatest end
     unsigned long long need_c, need_b;  // set (exactly) only when a registration list overflowed
     unsigned long long n_slots;
-    unsigned long long n_queue;  // entries in the I-list queue
 };
 
 struct IRest {  // I-list entry (sorted order), base kept in a separate array
@@ -119,8 +118,9 @@ struct Dev {  // scratch of one call (device pointers)
     uint64_t* fence;                             // [kFenceCap]
     uint32_t* chunk_cnt;                         // [C] slots per chunk
     uint64_t* staging;                           // [n_words] record of slot g at index g
-    IQ* queue;                                   // [cap_q] candidates for the I-list search
-    uint64_t cap_q;
+    IQ* queue;                                   // [C * 2048] candidates for the I-list search: region
+                                                 //  of classify warp w of chunk c at c*2048 + 256 w
+    uint32_t* qcnt;                              // [C * 8] entries in each region
 };
 
 struct P {  // kernel parameters
@@ -402,22 +402,36 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         warp_group_add_range(p.d.sup_c, r.x, r.y, reg_c);
         warp_group_add_range(p.d.sup_b, r.z, r.w, reg_b);
     }
-    // warp-aggregated: I positions, global prefilter bounds
+    // CTA-aggregated (one global atomic per CTA, not per warp: these are the same
+    // three addresses for every CTA): I positions, global prefilter bounds
+    __shared__ uint32_t s_ni, s_base;
+    __shared__ unsigned long long s_mn, s_mx;
+    if (threadIdx.x == 0) { s_ni = 0; s_mn = ~0ull; s_mx = 0; }
+    __syncthreads();
     const uint32_t bal = __ballot_sync(0xffffffffu, isI);
-    uint32_t base_pos = 0;
-    if (lane == 0 && bal) base_pos = atomicAdd(&p.d.ctl->nI, (unsigned)__popc(bal));
-    base_pos = __shfl_sync(0xffffffffu, base_pos, 0);
-    if (isI) {
-        const uint32_t pos = base_pos + __popc(bal & lanemask_lt());
-        p.d.sk[0][pos] = x.base;
-        p.d.sv[0][pos] = i;
-    }
+    uint32_t wpos = 0;
+    if (lane == 0 && bal) wpos = atomicAdd(&s_ni, (unsigned)__popc(bal));
     const bool live = valid && x.size != 0;
     const uint64_t mn = warp_min_u64(live ? x.base : ~0ull);
     const uint64_t mx = warp_max_u64(live ? x.base + x.size : 0ull);
     if (lane == 0 && mx) {
-        atomicMax(&p.d.ctl->gmin_c, ~(unsigned long long)mn);
-        atomicMax(&p.d.ctl->gmax, (unsigned long long)mx);
+        atomicMin(&s_mn, (unsigned long long)mn);
+        atomicMax(&s_mx, (unsigned long long)mx);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (s_ni) s_base = atomicAdd(&p.d.ctl->nI, s_ni);
+        if (s_mx) {
+            atomicMax(&p.d.ctl->gmin_c, ~s_mn);
+            atomicMax(&p.d.ctl->gmax, s_mx);
+        }
+    }
+    __syncthreads();
+    wpos = __shfl_sync(0xffffffffu, wpos, 0);
+    if (isI) {
+        const uint32_t pos = s_base + wpos + __popc(bal & lanemask_lt());
+        p.d.sk[0][pos] = x.base;
+        p.d.sv[0][pos] = i;
     }
     TL_PHASE(1, 22, tl_p);  // searches, registration counts, I compaction
 }
@@ -851,10 +865,13 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 }
 
 // ----------------------------------------------------------------------------
-// 4. k_scan_words: classify CTAs (one per chunk) and check CTAs
+// 4. k_classify: one CTA per 2048-word chunk.  The CTA sets up the chunk's
+//    mortal window (registered mortals sorted by base, per-node live masks);
+//    then each warp classifies its own 256 words with no further CTA barrier:
+//    word q of warp w is q = 256 w + 32 k + lane (k = 0..7).
+constexpr int kNsCap = 256;  // node starts of a chunk held in shared memory (more: search node_off)
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
-    uint32_t tw[MEDUSA_CHUNK_WORDS];     // node of every word, as an index from the chunk's first node
     uint64_t rb[kWinCap], re[kWinCap];   // one batch of registered mortals as loaded
     uint32_t rta[kWinCap], rtf[kWinCap], rid[kWinCap];
     uint64_t wb[kWinCap], we[kWinCap];   // the batch sorted by (base, t_alloc)
@@ -862,14 +879,14 @@ struct ClsShared {
     uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
     uint32_t nt0[kNodeGrp];                 // launch positions of the chunk's first kNodeGrp nodes
     uint32_t nt[kNodeGrp];                  // launch positions of nodes g0 .. g0 + kNodeGrp (later groups)
-    uint32_t gnext;
-    uint16_t cq[MEDUSA_CHUNK_WORDS];     // candidate words, then the I-list queue
-    uint32_t hits[MEDUSA_CHUNK_WORDS / 32];
-    uint32_t wmax[kWarps];
-    uint32_t nc, nq, total;
+    uint32_t ns[kNsCap];                    // start (word in chunk) of nodes jf + 1, jf + 2, ...
+    uint16_t cq[MEDUSA_CHUNK_WORDS];        // per warp (256 each): its candidates (word in chunk)
+    uint16_t cu[MEDUSA_CHUNK_WORDS];        // ... and their node (index from jf; 0xFFFF: larger)
+    uint32_t hits[MEDUSA_CHUNK_WORDS / 32]; // slot bits (warp w: words 8w .. 8w+7)
+    uint32_t wcnt[kWarps];                  // slots found per warp
+    uint32_t defer;                         // some candidate needs a later node group / window batch
     unsigned long long mbar;
 };
-
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
@@ -922,248 +939,257 @@ __device__ __forceinline__ void window_sort(ClsShared& S, uint32_t m) {
     else window_sort_e<4>(S, m);
 }
 
+// The live masks of nodes g0 .. g0+ng for the sorted batch of m entries (whole CTA;
+// nt = their launch positions).  Entry e is live at nodes u0 <= u < u1
+// (t_alloc < t_u < t_free): toggle bit e at u0 and u1, then a prefix XOR over u.
+__device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uint32_t ng, uint32_t m) {
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
+    __syncthreads();
+    for (uint32_t e = tid; e < m; e += kThreads) {
+        const uint32_t ta = S.wta[e], tf = S.wtf[e];
+        uint32_t lo = 0, hi = ng;  // u0 = #{u : t_u <= t_alloc}
+        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] <= ta) lo = mid + 1; else hi = mid; }
+        const uint32_t u0 = lo;
+        hi = ng;  // u1 = #{u : t_u < t_free}
+        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] < tf) lo = mid + 1; else hi = mid; }
+        const uint32_t u1 = lo;
+        if (u0 < u1) {
+            atomicXor(&S.live[u0][e >> 5], 1u << (e & 31));
+            if (u1 < ng) atomicXor(&S.live[u1][e >> 5], 1u << (e & 31));
+        }
+    }
+    __syncthreads();
+    static_assert(kNodeGrp == 128, "prefix XOR: 4 nodes per lane");
+    for (uint32_t w = warp; w < (m + 31) / 32; w += kWarps) {  // one warp per mask word
+        uint32_t v[4], run = 0;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) { v[r] = S.live[lane * 4 + r][w]; run ^= v[r]; v[r] = run; }
+        uint32_t incl = run;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= (uint32_t)d) incl ^= y;
+        }
+        const uint32_t before = incl ^ run;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) S.live[lane * 4 + r][w] = v[r] ^ before;
+    }
+    __syncthreads();
+}
+
+// The window entry holding word x at node u - g0 of the current group, or -1:
+// the live entries of one launch are pairwise disjoint, so the only possible
+// container is the live entry with the greatest base <= x.
+__device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint32_t ul, uint64_t x) {
+    uint32_t lo = 0, hi = m;  // entries with base <= x
+    while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
+    for (int w = ((int)lo - 1) >> 5; w >= 0; --w) {
+        uint32_t bits = S.live[ul][w];
+        const uint32_t top = lo - (uint32_t)w * 32;  // entries of word w below lo
+        if (top < 32) bits &= (1u << top) - 1u;
+        if (bits) {
+            const int e = w * 32 + 31 - __clz(bits);
+            return x < S.we[e] ? e : -1;
+        }
+    }
+    return -1;
+}
+
 __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    Ctl* ctl = p.d.ctl;
+    const Ctl* ctl = p.d.ctl;
     unsigned long long tl_p = TL_NOW();
     const uint64_t cs = (uint64_t)c * kChunkWords;
     const uint32_t n = (uint32_t)min((uint64_t)kChunkWords, a.n_words - cs);
     const uint64_t* gsrc = a.words + cs;
     const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
-    const uint32_t tx = tma ? n * 8 : 0;
     const uint32_t mb = smem_u32(&S.mbar);
-    // A. one TMA transaction brings the chunk's words to shared memory; meanwhile
-    //    the list offsets (block_prefix) and the chunk's node range load
+    // A. the chunk's words -> shared memory with one TMA bulk copy; meanwhile the
+    //    list offsets (block_prefix) and the chunk's node range load
     if (tid == 0) {
-        S.nc = 0;
-        S.nq = 0;
-        S.total = 0;
-        S.gnext = 0xFFFFFFFFu;
-        if (tx) {
+        S.defer = 0;
+        if (tma) {
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(tx) : "memory");
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
             asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                          ::"r"(smem_u32(S.words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
         }
     }
     const uint32_t N = a.n_nodes;
     const uint32_t jf = N ? min(__ldcg(p.d.jf + c), N - 1) : 0, jl = N ? min(__ldcg(p.d.jl + c), N - 1) : 0;
+    const uint32_t nn = N ? jl - jf + 1 : 0;
     const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
-    for (uint32_t q = tid; q < kChunkWords; q += kThreads) S.tw[q] = 0;
-    if (tid < MEDUSA_CHUNK_WORDS / 32) S.hits[tid] = 0;
     const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);  // (synchronizes the CTA)
     const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
-    const uint32_t nn = N ? jl - jf + 1 : 0;
     TL_PHASE(4, 10, tl_p);  // A: setup
     // B. one round of loads: threads 0..127 the first window batch, threads
-    //    128..255 the chunk's node starts (-> node index per word) and the launch
-    //    positions of its first kNodeGrp nodes
+    //    128..255 the starts of the chunk's nodes and the launch positions of
+    //    its first kNodeGrp nodes
     const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
     if (tid < kWinCap) {
         window_load(p, S, r0, m0);
     } else {
         const uint32_t h = tid - kWinCap;
-        for (uint32_t j = jf + 1 + h; j <= jl; j += kThreads - kWinCap) {
-            const uint64_t q = a.node_off[j] - cs;
-            if (q < n) atomicMax(&S.tw[q], j - jf);
-        }
+        for (uint32_t k = h; k + 1 < nn && k < kNsCap; k += kThreads - kWinCap)
+            S.ns[k] = (uint32_t)(a.node_off[jf + 1 + k] - cs);
         if (h < kNodeGrp && h < nn) S.nt0[h] = a.node_t[jf + h];
     }
     __syncthreads();
-    TL_PHASE(4, 11, tl_p);  // B: window records, node starts
-    // warp 0 sorts the window batch; all warps: running max over the chunk,
-    // tw[q] = index (from jf) of the node holding word q
     if (warp == 0 && m0) window_sort(S, m0);
-    {
-        uint32_t loc[kWordsPerThread];
-        uint32_t run = 0;
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) { run = max(run, S.tw[tid * kWordsPerThread + k]); loc[k] = run; }
-        uint32_t incl = run;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
-            if (lane >= d) incl = max(incl, y);
-        }
-        if (lane == 31) S.wmax[warp] = incl;
-        const uint32_t up = __shfl_up_sync(0xffffffffu, incl, 1);
-        __syncthreads();
-        uint32_t before = lane ? up : 0;
-        for (uint32_t ww = 0; ww < warp; ++ww) before = max(before, S.wmax[ww]);
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) S.tw[tid * kWordsPerThread + k] = max(before, loc[k]);
-    }
-    if (tx) {
+    __syncthreads();
+    TL_PHASE(4, 11, tl_p);  // B: window records, node starts, sort
+    const uint32_t ng0 = min((uint32_t)kNodeGrp, nn);
+    if (m0) build_live(S, S.nt0, ng0, m0);
+    if (tma) {
         uint32_t done = 0;
         while (!done) {
             asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
                          : "=r"(done) : "r"(mb) : "memory");
         }
     }
-    // C. candidates: words inside [least base, greatest end) of the trace
+    TL_PHASE(4, 12, tl_p);  // C: live masks, TMA wait
+    // D. this warp's words: candidates (inside [least base, greatest end) of the
+    //    trace) compacted into the warp's list; per candidate its node (upper bound
+    //    over the node starts) and the window lookup at node group 0 / batch 0
+    const bool narrow = nn - 1 <= (uint32_t)kNsCap;  // all node starts in shared memory
+    const bool more_batches = r1 - r0 > (uint64_t)kWinCap;
+    uint16_t* wl = S.cq + warp * 256;   // this warp's candidates (word in chunk)
+    uint16_t* wu = S.cu + warp * 256;   // ... and their node (index from jf)
+    uint32_t* wh = S.hits + warp * 8;   // hit bits of the warp's 256 words
+    uint32_t nc = 0;
 #pragma unroll
     for (int k = 0; k < kWordsPerThread; ++k) {
-        const uint32_t q = k * kThreads + tid;
-        bool cand = false;
-        if (q < n) {
-            const uint64_t x = S.words[q];
-            cand = x >= gmin && x < gmax;
-        }
-        const uint32_t bal = __ballot_sync(0xffffffffu, cand);
-        uint32_t base = 0;
-        if (lane == 0 && bal) base = atomicAdd(&S.nc, (uint32_t)__popc(bal));
-        base = __shfl_sync(0xffffffffu, base, 0);
-        if (cand) S.cq[base + __popc(bal & lanemask_lt())] = (uint16_t)q;
+        const uint32_t q = warp * 256 + k * 32 + lane;
+        const bool cand = q < n && S.words[q] >= gmin && S.words[q] < gmax;
+        const uint32_t b = __ballot_sync(0xffffffffu, cand);
+        if (cand) wl[nc + __popc(b & lanemask_lt())] = (uint16_t)q;
+        nc += __popc(b);
     }
-    __syncthreads();
-    TL_PHASE(4, 12, tl_p);  // C: window sort, launch positions, TMA wait, candidates
-    const uint32_t nc = S.nc;
-    // D. mortal window(s).  The entries live at one launch are pairwise disjoint,
-    //    so the only possible container of word x of node u is the live entry
-    //    with the greatest base <= x: one upper bound over the bases sorted in
-    //    shared memory, one AND with node u's live mask (bit e = entry e live at
-    //    u's launch), one leading-zero count, one end check.  Masks are built per
-    //    batch of <= kWinCap entries and group of kNodeGrp nodes.
-    for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
-        const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
-        if (bs != r0) {  // a further batch (windows of more than kWinCap entries)
-            window_load(p, S, bs, m);
-            __syncthreads();
-            if (warp == 0) window_sort(S, m);
-            __syncthreads();
+    if (lane < 8) wh[lane] = 0;
+    __syncwarp();
+    bool deferred = false;
+    for (uint32_t i = lane; i < nc; i += 32) {
+        const uint32_t q = wl[i];
+        const uint64_t x = S.words[q];
+        uint32_t u;
+        if (narrow) {
+            uint32_t lo = 0, hi = nn - 1;  // nodes jf+1.. starting at or before q
+            while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.ns[mid] <= q) lo = mid + 1; else hi = mid; }
+            u = lo;
+        } else {
+            uint32_t lo = jf + 1, hi = jl + 1;  // node_off[j] <= cs + q
+            while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (a.node_off[mid] <= cs + q) lo = mid + 1; else hi = mid; }
+            u = lo - (jf + 1);
         }
-        const uint32_t mw = (m + 31) / 32;
-        for (uint32_t g0 = 0; g0 < nn;) {
-            const uint32_t ng = min((uint32_t)kNodeGrp, nn - g0);
-            const uint32_t* nt = g0 ? S.nt : S.nt0;
-            if (g0)
-                for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
-            for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
-            __syncthreads();
-            // entry e is live at the nodes u0 <= u < u1 of the group (t_alloc < t_u < t_free):
-            // toggle bit e at u0 and u1, then a prefix XOR over u yields the masks
-            for (uint32_t e = tid; e < m; e += kThreads) {
-                const uint32_t ta = S.wta[e], tf = S.wtf[e];
-                uint32_t lo = 0, hi = ng;  // u0 = #{u : t_u <= t_alloc}
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] <= ta) lo = mid + 1; else hi = mid; }
-                const uint32_t u0 = lo;
-                hi = ng;  // u1 = #{u : t_u < t_free}
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] < tf) lo = mid + 1; else hi = mid; }
-                const uint32_t u1 = lo;
-                if (u0 < u1) {
-                    atomicXor(&S.live[u0][e >> 5], 1u << (e & 31));
-                    if (u1 < ng) atomicXor(&S.live[u1][e >> 5], 1u << (e & 31));
-                }
+        wu[i] = (uint16_t)min(u, 0xFFFFu);
+        bool hit = false;
+        if (m0 && u < ng0) {
+            const int e = window_find(S, m0, u, x);
+            if (e >= 0) {
+                hit = true;
+                S.words[q] = ((uint64_t)S.wid[e] << MEDUSA_OFF_BITS) | (x - S.wb[e]);
+                atomicOr(&S.hits[q >> 5], 1u << (q & 31));
             }
-            __syncthreads();
-            static_assert(kNodeGrp == 128, "prefix XOR: 4 nodes per lane");
-            for (uint32_t w = warp; w < mw; w += kWarps) {  // one warp per mask word
-                uint32_t v[4], run = 0;
-#pragma unroll
-                for (int r = 0; r < 4; ++r) { v[r] = S.live[lane * 4 + r][w]; run ^= v[r]; v[r] = run; }
-                uint32_t incl = run;
-#pragma unroll
-                for (int d = 1; d < 32; d <<= 1) {
-                    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                    if (lane >= (uint32_t)d) incl ^= y;
-                }
-                const uint32_t before = incl ^ run;
-#pragma unroll
-                for (int r = 0; r < 4; ++r) S.live[lane * 4 + r][w] = v[r] ^ before;
-            }
-            __syncthreads();
-            uint32_t gnext = 0xFFFFFFFFu;
-            for (uint32_t i = tid; i < nc; i += kThreads) {
-                const uint32_t q = S.cq[i];
-                if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
-                const uint32_t u = S.tw[q];
-                if (u < g0) continue;
-                if (u >= g0 + ng) { gnext = min(gnext, u); continue; }
-                const uint64_t x = S.words[q];
-                uint32_t lo = 0, hi = m;  // entries with base <= x
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
-                int e = -1;
-                for (int w = ((int)lo - 1) >> 5; w >= 0; --w) {
-                    uint32_t bits = S.live[u - g0][w];
-                    const uint32_t top = lo - (uint32_t)w * 32;  // entries of word w below lo
-                    if (top < 32) bits &= (1u << top) - 1u;
-                    if (bits) { e = w * 32 + 31 - __clz(bits); break; }
-                }
-                if (e >= 0 && x < S.we[e]) {
-                    S.words[q] = ((uint64_t)S.wid[e] << MEDUSA_OFF_BITS) | (x - S.wb[e]);
-                    atomicOr(&S.hits[q >> 5], 1u << (q & 31));
-                }
-            }
-            gnext = __reduce_min_sync(0xffffffffu, gnext);
-            if (lane == 0 && gnext != 0xFFFFFFFFu) atomicMin(&S.gnext, gnext);
-            __syncthreads();
-            const uint32_t gn = S.gnext;  // next group holding an unresolved candidate
-            __syncthreads();
-            if (tid == 0) S.gnext = 0xFFFFFFFFu;
-            if (gn == 0xFFFFFFFFu) break;
-            g0 = gn;
         }
+        if (!hit && m0 && (u >= ng0 || more_batches)) deferred = true;
     }
+    if (__any_sync(0xffffffffu, deferred) && lane == 0) S.defer = 1;
     __syncthreads();
     TL_PHASE(4, 13, tl_p);  // D: window search
-    // E. the candidates no mortal holds go to the I-list queue (k_iresolve);
-    //    one queue reservation per CTA
-    {
-        uint32_t qv[kWordsPerThread];
-        bool need[kWordsPerThread];
-        uint32_t mine = 0;
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            const uint32_t i = k * kThreads + tid;
-            need[k] = false;
-            qv[k] = 0;
-            if (i < nc) {
-                const uint32_t q = S.cq[i];
-                qv[k] = q;
-                need[k] = !((S.hits[q >> 5] >> (q & 31)) & 1u);
+    if (S.defer) {
+        // rare: chunks with more than kNodeGrp nodes or windows of more than kWinCap
+        // entries -- every batch against every node group, CTA-synchronous
+        for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
+            const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
+            if (bs != r0) {
+                __syncthreads();
+                window_load(p, S, bs, m);
+                __syncthreads();
+                if (warp == 0) window_sort(S, m);
+                __syncthreads();
             }
-            mine += need[k] ? 1u : 0u;
+            for (uint32_t g0 = (bs == r0 ? kNodeGrp : 0); g0 < nn; g0 += kNodeGrp) {
+                const uint32_t ng = min((uint32_t)kNodeGrp, nn - g0);
+                __syncthreads();
+                for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
+                __syncthreads();
+                build_live(S, S.nt, ng, m);
+                for (uint32_t i = lane; i < nc; i += 32) {
+                    const uint32_t q = wl[i];
+                    if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
+                    uint32_t u = wu[i];
+                    if (u == 0xFFFFu) {  // (node index beyond 16 bits: search again)
+                        uint32_t lo = jf + 1, hi = jl + 1;
+                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (a.node_off[mid] <= cs + q) lo = mid + 1; else hi = mid; }
+                        u = lo - (jf + 1);
+                    }
+                    if (u < g0 || u >= g0 + ng) continue;
+                    const uint64_t x = S.words[q];
+                    const int e = window_find(S, m, u - g0, x);
+                    if (e >= 0) {
+                        S.words[q] = ((uint64_t)S.wid[e] << MEDUSA_OFF_BITS) | (x - S.wb[e]);
+                        atomicOr(&S.hits[q >> 5], 1u << (q & 31));
+                    }
+                }
+            }
         }
-        uint32_t total;
-        const uint32_t pre = block_excl_scan(mine, &total);
-        if (tid == 0 && total) S.nq = (uint32_t)atomicAdd(&ctl->n_queue, (unsigned long long)total);
         __syncthreads();
-        uint64_t pos = (uint64_t)S.nq + pre;
-#pragma unroll
-        for (int k = 0; k < kWordsPerThread; ++k) {
-            if (!need[k]) continue;
-            const uint32_t q = qv[k];
-            const uint32_t u = S.tw[q];
-            const uint32_t t = u < kNodeGrp ? S.nt0[u] : __ldg(a.node_t + jf + u);  // the word's launch position
-            if (pos < p.d.cap_q) p.d.queue[pos] = IQ{S.words[q], (uint32_t)(cs + q), t};
-            ++pos;
-        }
     }
-    TL_PHASE(4, 14, tl_p);  // E: queue
-    // F. emission: mask words, records at their word index, the chunk's count
+    // E. the candidates no mortal holds go to this warp's queue region (k_iresolve)
+    IQ* wq = p.d.queue + cs + warp * 256;
+    uint32_t nq = 0;
+    for (uint32_t i0 = 0; i0 < nc; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        bool need = false;
+        uint32_t q = 0;
+        if (i < nc) {
+            q = wl[i];
+            need = !((S.hits[q >> 5] >> (q & 31)) & 1u);
+        }
+        const uint32_t b = __ballot_sync(0xffffffffu, need);
+        if (need) {
+            uint32_t u = wu[i];
+            if (u == 0xFFFFu) {
+                uint32_t lo = jf + 1, hi = jl + 1;
+                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (a.node_off[mid] <= cs + q) lo = mid + 1; else hi = mid; }
+                u = lo - (jf + 1);
+            }
+            const uint32_t t = u < kNodeGrp ? S.nt0[u] : __ldg(a.node_t + jf + u);  // the word's launch position
+            wq[nq + __popc(b & lanemask_lt())] = IQ{S.words[q], (uint32_t)(cs + q), t};
+        }
+        nq += __popc(b);
+    }
+    // F. per 32 words: the mask word (lane 0) and the records at their word index
     const uint64_t n_mask = (a.n_words + 31) / 32;
     uint32_t cnt = 0;
 #pragma unroll
     for (int k = 0; k < kWordsPerThread; ++k) {
-        const uint32_t q = k * kThreads + tid;
-        const uint32_t bits = S.hits[q >> 5];
+        const uint32_t q = warp * 256 + k * 32 + lane;
+        const uint32_t bits = wh[k];
         const uint64_t mw = (cs + q) >> 5;
-        if (lane == 0 && mw < n_mask) a.mask[mw] = bits;
+        if (lane == 0 && q < n && mw < n_mask) a.mask[mw] = bits;
         if ((bits >> lane) & 1u) p.d.staging[cs + q] = S.words[q];
         cnt += __popc(bits);
     }
-    if (lane == 0) atomicAdd(&S.total, cnt);
+    if (lane == 0) {
+        p.d.qcnt[c * kWarps + warp] = nq;
+        S.wcnt[warp] = cnt;
+    }
     __syncthreads();
-    TL_PHASE(4, 15, tl_p);  // F: emission
+    TL_PHASE(4, 14, tl_p);  // E/F: queue, emission
     // G. the chunk's slot count so far and its 256-chunk group sum (k_iresolve
     //    adds the I-list slots; k_emit turns them into chunk_base)
     if (tid == 0) {
-        p.d.chunk_cnt[c] = S.total;
-        if (S.total) atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)S.total);
+        uint32_t total = 0;
+#pragma unroll
+        for (int w = 0; w < kWarps; ++w) total += S.wcnt[w];
+        p.d.chunk_cnt[c] = total;
+        if (total) atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)total);
     }
     pdl_trigger();
 }
@@ -1287,44 +1313,57 @@ __global__ void __launch_bounds__(kThreads, 4) k_classify(P p) {
 
 // ----------------------------------------------------------------------------
 // 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
-//     sorted I list -- fences in shared memory, then per candidate one group of
-//     bases and one entry (two dependent loads).  A hit writes its record at its
-//     word index, sets its mask bit and counts toward its chunk.
+//     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
+//     CTA; warp w takes the queue region classify's warp w filled.  Per candidate
+//     one group of bases and one entry (two dependent loads); a hit writes its
+//     record at its word index and sets its mask bit; the chunk's count grows by
+//     one atomic per chunk.
 __global__ void __launch_bounds__(kThreads) k_iresolve(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
+    __shared__ uint32_t s_cnt[kWarps];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
-    const Ctl* ctl = p.d.ctl;
-    const uint32_t nI = ctl->nI;
-    const uint64_t nq = min((uint64_t)ctl->n_queue, p.d.cap_q);
-    if (nI && nq > (uint64_t)blockIdx.x * kThreads) {
+    const uint32_t nI = p.d.ctl->nI;
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (nI) {
         const uint32_t stride = fence_stride(nI);
         const uint32_t nf = (nI + stride - 1) / stride;
-        for (uint32_t f = threadIdx.x; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
+        for (uint32_t f = tid; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
         __syncthreads();
-        const uint64_t n_mask = (p.a.n_words + 31) / 32;
-        for (uint64_t i0 = (uint64_t)blockIdx.x * kThreads; i0 < nq; i0 += (uint64_t)gridDim.x * kThreads) {
-            const uint64_t i = i0 + threadIdx.x;
-            bool hit = false;
-            uint32_t g = 0;
-            if (i < nq) {
-                const IQ q = p.d.queue[i];
-                g = q.g;
-                const uint32_t cnt = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
-                if (cnt) {
-                    const uint32_t kk = cnt - 1;
-                    const uint64_t base = p.d.i_base[kk];
-                    const IRest e = p.d.i_rest[kk];
-                    if (q.x < e.end && e.t_alloc < q.t) {
-                        hit = true;
-                        p.d.staging[g] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
-                        if ((g >> 5) < n_mask) atomicOr(p.a.mask + (g >> 5), 1u << (g & 31));
+        for (uint32_t c = blockIdx.x; c < p.C; c += gridDim.x) {
+            const uint32_t nq = __ldcg(p.d.qcnt + c * kWarps + warp);
+            const IQ* wq = p.d.queue + (uint64_t)c * kChunkWords + warp * 256;
+            uint32_t cnt = 0;
+            for (uint32_t i0 = 0; i0 < nq; i0 += 32) {
+                const uint32_t i = i0 + lane;
+                bool hit = false;
+                if (i < nq) {
+                    const IQ q = wq[i];
+                    const uint32_t le = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
+                    if (le) {
+                        const uint64_t base = p.d.i_base[le - 1];
+                        const IRest e = p.d.i_rest[le - 1];
+                        if (q.x < e.end && e.t_alloc < q.t) {
+                            hit = true;
+                            p.d.staging[q.g] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
+                            atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
+                        }
                     }
                 }
+                cnt += __popc(__ballot_sync(0xffffffffu, hit));
             }
-            const uint32_t c = g / kChunkWords;
-            warp_agg_add(p.d.chunk_cnt, c, hit);
-            warp_group_add_range(p.d.chunk_sup, c, c, hit);
+            if (lane == 0) s_cnt[warp] = cnt;
+            __syncthreads();
+            if (tid == 0) {
+                uint32_t total = 0;
+#pragma unroll
+                for (int w = 0; w < kWarps; ++w) total += s_cnt[w];
+                if (total) {
+                    atomicAdd(p.d.chunk_cnt + c, total);
+                    atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)total);
+                }
+            }
+            __syncthreads();
         }
     }
     pdl_trigger();
@@ -1463,9 +1502,9 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
         (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) || (e = grow(s, s.d.sv[1], N)) ||
         (e = grow(s, s.d.samp_k, N / 32 + 64)) || (e = grow(s, s.d.samp_v, N / 32 + 64)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
         (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
-        (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)) || (e = grow(s, s.d.queue, WW)))
+        (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)) ||
+        (e = grow(s, s.d.queue, CC * kChunkWords)) || (e = grow(s, s.d.qcnt, CC * kWarps)))
         return e;
-    s.d.cap_q = WW;
     s.d.cap_c = RC;
     s.d.cap_b = RB;
     s.cap_n = N; s.cap_C = CC; s.cap_nb = NB; s.cap_c = RC; s.cap_b = RB; s.cap_w = WW;
@@ -1550,7 +1589,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
         if (C) {
             TimedLaunch tl("mat_iresolve", stream);
-            if ((e = launch_pdl(k_iresolve, (unsigned)s.sm_count * 8, kThreads, 0, stream, p))) return e;
+            if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * 4), kThreads, 0, stream, p))) return e;
         }
     } else if (C) {
         TimedLaunch tl("mat_classify", stream);
