@@ -757,8 +757,8 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t T = n_tiles(nI);
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t g0 = blockIdx.x * 32;  // this CTA's 32 keys
-    if (T > 1 && g0 < nI) {
+    // ranges of 32 keys, grid-stride (the grid is sized by the allocation count)
+    for (uint32_t g0 = blockIdx.x * 32; T > 1 && g0 < nI; g0 += gridDim.x * 32) {
         const uint32_t ta = g0 / kSortTile;
         const uint32_t g = g0 + lane;
         const bool has = g < nI;
@@ -839,6 +839,7 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
             for (int w = 0; w < kWarps; ++w) rank += s_cnt[w][lane];
             write_i_entry(p, rank, nI, xv, ld_alloc(p.a.alloc + xv));
         }
+        __syncthreads();  // s_cnt is rewritten by the next range
     }
     pdl_trigger();
     TL_REC(3, 0, tl0);
@@ -1274,27 +1275,37 @@ __global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
             mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
         }
         const uint64_t xe = x.base + x.size;
+        // the block's hull: only list entries meeting it (in address, time and
+        // ordinal) can collide with one of its mortals; they are compacted first
+        const uint64_t hb = warp_min_u64(mine ? x.base : ~0ull), he = warp_max_u64(mine ? xe : 0ull);
+        const uint32_t hta = __reduce_min_sync(0xffffffffu, mine ? x.t_alloc : 0xFFFFFFFFu);
+        const uint32_t hj = __reduce_max_sync(0xffffffffu, mine ? j : 0u);
         bool bad = false;
         const uint64_t r0 = base + before;
         const uint64_t r1 = min(r0 + __shfl_sync(0xffffffffu, cb, warp), p.d.cap_b);
-        for (uint64_t bs = r0; bs < r1; bs += kChkCap) {
-            const uint32_t m = (uint32_t)min((uint64_t)kChkCap, r1 - bs);
+        for (uint64_t bs = r0; bs < r1 && he; bs += 32) {
+            const uint32_t m = (uint32_t)min((uint64_t)32, r1 - bs);
+            WinRec y{};
+            bool keep = false;
+            if (lane < m) {
+                y = p.d.list_b[bs + lane];
+                keep = y.base < he && hb < y.end && y.t_free > hta && y.id < hj;
+            }
+            const uint32_t kb = __ballot_sync(0xffffffffu, keep);
             __syncwarp();
-            for (uint32_t q = lane; q < m; q += 32) {
-                const WinRec y = p.d.list_b[bs + q];
-                s_base[warp][q] = y.base;
-                s_end[warp][q] = y.end;
-                s_tf[warp][q] = y.t_free;
-                s_idx[warp][q] = y.id;
+            if (keep) {
+                const uint32_t o = __popc(kb & lanemask_lt());
+                s_base[warp][o] = y.base;
+                s_end[warp][o] = y.end;
+                s_tf[warp][o] = y.t_free;
+                s_idx[warp][o] = y.id;
             }
             __syncwarp();
-            if (mine && !bad) {
-                for (uint32_t q = 0; q < m; ++q) {
-                    if (s_idx[warp][q] < j && s_tf[warp][q] > x.t_alloc && s_base[warp][q] < xe && x.base < s_end[warp][q]) {
-                        bad = true;
-                        break;
-                    }
-                }
+            if (mine) {
+                const uint32_t nk = __popc(kb);
+                for (uint32_t q = 0; q < nk; ++q)
+                    bad |= (s_idx[warp][q] < j) & (s_tf[warp][q] > x.t_alloc) & (s_base[warp][q] < xe) &
+                           (x.base < s_end[warp][q]);
             }
         }
         if (bad) flag(p.d.ctl, ST_TRACE);
@@ -1571,7 +1582,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             TimedLaunch tl("mat_rank", s.side);
             // one CTA per 32 I keys (the list's size is known on the device only: bound
             // by the allocation count; surplus CTAs exit at once)
-            k_rank<<<(unsigned)((n + 31) / 32), kThreads, 0, s.side>>>(p);
+            k_rank<<<(unsigned)std::min<uint64_t>((n + 31) / 32, (uint64_t)s.sm_count * 8), kThreads, 0, s.side>>>(p);
         }
         {
             TimedLaunch tl("mat_check_mi", s.side);
