@@ -1600,7 +1600,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
         if (C) {
             TimedLaunch tl("mat_iresolve", stream);
-            if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * 4), kThreads, 0, stream, p))) return e;
+            if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * 8), kThreads, 0, stream, p))) return e;
         }
     } else if (C) {
         TimedLaunch tl("mat_classify", stream);

@@ -332,3 +332,68 @@ def test_async_reports_trace_error_and_capacity():
             assert medusa.mat_result(res) == (medusa.ERR_CAPACITY, n), seed
             seen_cap = True
     assert seen_bad and seen_cap
+
+
+def _long_lived_mortals_trace(seed, n_mortal=1200, n_nodes=60000):
+    """Many mortals live across the whole capture, one word per node: every chunk's
+    window holds all of them (several batches), every chunk holds 2048 nodes (more
+    than the node starts kept in shared memory), and the registration lists exceed
+    the library's first guess (the overflow / exact-resize path)."""
+    rng = np.random.default_rng(seed)
+    base0 = 0x7F00_0000_0000
+    t = 1
+    allocs = []
+    for i in range(n_mortal):  # disjoint, all live until the end of the capture
+        allocs.append((base0 + i * 4096, 2048 if i % 7 else 0, t, 0))
+        t += 1
+    i_perm = []
+    for k in range(16):  # a few I allocations (live at the last launch)
+        allocs.append((base0 + (1 << 30) + k * 8192, 4096, t, T_NEVER))
+        i_perm.append(len(allocs) - 1)
+        t += 1
+    node_t = []
+    words = []
+    for j in range(n_nodes):
+        t += 1
+        node_t.append(t)
+        r = rng.random()
+        if r < 0.5:
+            a = allocs[int(rng.integers(0, n_mortal))]
+            words.append(a[0] + int(rng.integers(0, 2049)))
+        elif r < 0.7:
+            a = allocs[i_perm[int(rng.integers(0, len(i_perm)))]]
+            words.append(a[0] + int(rng.integers(0, 4097)))
+        else:
+            words.append(int(rng.integers(0, 1 << 62)))
+    t += 1
+    arr = np.zeros(len(allocs), ALLOC_DTYPE)
+    for i, (b, sz, ta, tf) in enumerate(allocs):
+        arr[i] = (b, sz, ta, tf if tf else t)  # mortals freed after the capture...
+    t += 1
+    node_t.append(t)  # ... and before one last launch, so they are not in I
+    words.append(0)
+    off = np.arange(len(words) + 1, dtype=np.uint64)
+    return np.array(words, np.uint64), off, np.array(node_t, np.uint32), arr
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_overflow_retry_many_batches_wide_chunks(seed):
+    words, off, node_t, allocs = _long_lived_mortals_trace(seed)
+    m = oracle.materialize(words, off, node_t, allocs)
+    assert m["status"] == 0
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(DEV)
+    aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3)
+    inp = dict(words=t(words, np.int64), node_off=t(off, np.int64), node_t=t(node_t, np.int32),
+               allocs=torch.from_numpy(aa).to(DEV))
+    s = medusa.materialize(**inp)  # registrations overflow the first guess: resized, rerun
+    mask, cb, rec = oracle.pack(m, words.size)
+    assert s.n_slots == m["n_slots"]
+    assert np.array_equal(_h(s.mask).view(np.uint32), mask)
+    assert np.array_equal(_h(s.chunk_base).view(np.uint32), cb)
+    assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec)
+    # the async entry now runs with the grown scratch
+    res = torch.zeros(2, dtype=torch.int64, device=DEV)
+    out = medusa.alloc_slots(words.size, DEV)
+    medusa.materialize_async(**inp, out=out, result=res)
+    assert medusa.mat_result(res) == (0, m["n_slots"])
+    assert np.array_equal(_h(out.slot)[: m["n_slots"]].view(np.uint64), rec)
