@@ -25,7 +25,13 @@
  *   - The return value reports argument, trace and launch errors only.
  *     Data-dependent validation failures of a restore are not call errors:
  *     they are counted in the device-side medusa_report (the call is async).
- *   - Thread-safe: calls may come from several host threads and devices.
+ *   - Thread-safe: calls may come from several host threads and devices.  The
+ *     materialize entry points of one device share that device's scratch: the
+ *     synchronous one serializes itself; an asynchronous one must be ordered
+ *     (same stream, or events) against every other materialize on the device.
+ *   - Work is enqueued on the caller's `stream`.  Materialize forks part of its
+ *     work onto an internal stream and joins it back before returning, so the
+ *     call is one stream-ordered unit (and capturable, see below).
  *   - There is no CPU fallback: without a usable sm_100a device every call
  *     that would touch the GPU returns MEDUSA_ERR_CUDA.
  */
@@ -185,7 +191,9 @@ medusa_status medusa_materialize_async(const uint64_t *d_words, uint64_t n_words
  * for kernels hidden from the symbol tables, from enumerating the modules that
  * the triggering kernels (the model's first layer) loaded.
  * The copy is ordered on `stream`; a later medusa_restore must be ordered after
- * it (same stream, or an event).  Replaces any previous table of this device. */
+ * it (same stream, or an event).  Replaces any previous table of this device.
+ * The first call on a device (or one with a larger n_func) allocates the table:
+ * make it before capturing a CUDA graph that contains this call.             */
 medusa_status medusa_kernel_table_set(const uint64_t *d_func_addr, uint32_t n_func,
                                       cudaStream_t stream);
 
