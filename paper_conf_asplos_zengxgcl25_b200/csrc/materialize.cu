@@ -870,7 +870,6 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 //    mortal window (registered mortals sorted by base, per-node live masks);
 //    then each warp classifies its own 256 words with no further CTA barrier:
 //    word q of warp w is q = 256 w + 32 k + lane (k = 0..7).
-constexpr int kNsCap = 256;  // node starts of a chunk held in shared memory (more: search node_off)
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     uint64_t rb[kWinCap], re[kWinCap];   // one batch of registered mortals as loaded
@@ -878,11 +877,13 @@ struct ClsShared {
     uint64_t wb[kWinCap], we[kWinCap];   // the batch sorted by (base, t_alloc)
     uint32_t wta[kWinCap], wtf[kWinCap], wid[kWinCap];
     uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
-    uint32_t nt0[kNodeGrp];                 // launch positions of the chunk's first kNodeGrp nodes
-    uint32_t nt[kNodeGrp];                  // launch positions of nodes g0 .. g0 + kNodeGrp (later groups)
-    uint32_t ns[kNsCap];                    // start (word in chunk) of nodes jf + 1, jf + 2, ...
+    // Segments: segment s of the chunk = the words of the s-th distinct node start
+    // (segment 0 = node jf's words); s(q) = nsp[q/32] + popc(nsm[q/32] & bits 0..q%32)
+    uint32_t nsm[MEDUSA_CHUNK_WORDS / 32];  // bit q: a node starts at word q (q > 0)
+    uint32_t nsp[MEDUSA_CHUNK_WORDS / 32];  // exclusive popcount prefix of nsm
+    uint32_t nt0[kNodeGrp];                 // launch positions of segments 0 .. kNodeGrp-1
+    uint32_t nt[kNodeGrp];                  // launch positions of segments g0 .. g0+kNodeGrp-1 (later groups)
     uint16_t cq[MEDUSA_CHUNK_WORDS];        // per warp (256 each): its candidates (word in chunk)
-    uint16_t cu[MEDUSA_CHUNK_WORDS];        // ... and their node (index from jf; 0xFFFF: larger)
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32]; // slot bits (warp w: words 8w .. 8w+7)
     uint32_t wcnt[kWarps];                  // slots found per warp
     uint32_t defer;                         // some candidate needs a later node group / window batch
@@ -997,6 +998,33 @@ __device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint3
     return -1;
 }
 
+// segment (see ClsShared) of word q of the chunk
+__device__ __forceinline__ uint32_t seg_of(const ClsShared& S, uint32_t q) {
+    return S.nsp[q >> 5] + __popc(S.nsm[q >> 5] & (0xFFFFFFFFu >> (31 - (q & 31))));
+}
+
+// launch position of the node holding word q (segments beyond group 0: search node_off)
+__device__ __forceinline__ uint32_t seg_time(const P& p, const ClsShared& S, uint32_t s, uint64_t g, uint32_t jf,
+                                             uint32_t jl) {
+    if (s < kNodeGrp) return S.nt0[s];
+    uint32_t lo = jf + 1, hi = jl + 1;  // first node starting after word g
+    while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (p.a.node_off[mid] <= g) lo = mid + 1; else hi = mid; }
+    return __ldg(p.a.node_t + lo - 1);
+}
+
+// launch positions of segments g0 .. g0+ng-1 into nt (whole CTA; nt zeroed here)
+__device__ __forceinline__ void seg_times(const P& p, ClsShared& S, uint32_t* nt, uint32_t g0, uint32_t ng, uint64_t cs,
+                                          uint32_t jf, uint32_t jl) {
+    for (uint32_t u = threadIdx.x; u < ng; u += kThreads) nt[u] = 0;
+    __syncthreads();
+    if (threadIdx.x == 0 && g0 == 0) nt[0] = p.a.node_t[jf];
+    for (uint32_t j = jf + 1 + threadIdx.x; j <= jl; j += kThreads) {
+        const uint32_t s = seg_of(S, (uint32_t)(p.a.node_off[j] - cs));
+        if (s >= g0 && s < g0 + ng) atomicMax(nt + (s - g0), p.a.node_t[j]);  // the last node of a start is its non-empty one
+    }
+    __syncthreads();
+}
+
 __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -1025,26 +1053,39 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
+    if (tid < MEDUSA_CHUNK_WORDS / 32) S.nsm[tid] = 0;
     const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);  // (synchronizes the CTA)
     const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
     TL_PHASE(4, 10, tl_p);  // A: setup
     // B. one round of loads: threads 0..127 the first window batch, threads
-    //    128..255 the starts of the chunk's nodes and the launch positions of
-    //    its first kNodeGrp nodes
+    //    128..255 the starts of the chunk's nodes (-> start bitmask)
     const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
     if (tid < kWinCap) {
         window_load(p, S, r0, m0);
     } else {
-        const uint32_t h = tid - kWinCap;
-        for (uint32_t k = h; k + 1 < nn && k < kNsCap; k += kThreads - kWinCap)
-            S.ns[k] = (uint32_t)(a.node_off[jf + 1 + k] - cs);
-        if (h < kNodeGrp && h < nn) S.nt0[h] = a.node_t[jf + h];
+        for (uint32_t j = jf + 1 + (tid - kWinCap); j <= jl; j += kThreads - kWinCap) {
+            const uint32_t q = (uint32_t)(a.node_off[j] - cs);
+            atomicOr(&S.nsm[q >> 5], 1u << (q & 31));
+        }
     }
     __syncthreads();
     if (warp == 0 && m0) window_sort(S, m0);
+    if (warp == 1) {  // exclusive popcount prefix of the 64 start-mask words
+        const uint32_t c0 = __popc(S.nsm[2 * lane]), c1 = __popc(S.nsm[2 * lane + 1]);
+        uint32_t incl = c0 + c1;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= (uint32_t)d) incl += y;
+        }
+        S.nsp[2 * lane] = incl - c0 - c1;
+        S.nsp[2 * lane + 1] = incl - c1;
+    }
     __syncthreads();
+    const uint32_t n_seg = N ? S.nsp[63] + __popc(S.nsm[63]) + 1 : 0;
+    const uint32_t ng0 = min((uint32_t)kNodeGrp, n_seg);
+    seg_times(p, S, S.nt0, 0, ng0, cs, jf, jl);
     TL_PHASE(4, 11, tl_p);  // B: window records, node starts, sort
-    const uint32_t ng0 = min((uint32_t)kNodeGrp, nn);
     if (m0) build_live(S, S.nt0, ng0, m0);
     if (tma) {
         uint32_t done = 0;
@@ -1055,12 +1096,10 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     }
     TL_PHASE(4, 12, tl_p);  // C: live masks, TMA wait
     // D. this warp's words: candidates (inside [least base, greatest end) of the
-    //    trace) compacted into the warp's list; per candidate its node (upper bound
-    //    over the node starts) and the window lookup at node group 0 / batch 0
-    const bool narrow = nn - 1 <= (uint32_t)kNsCap;  // all node starts in shared memory
+    //    trace) compacted into the warp's list; per candidate its segment (O(1) from
+    //    the start bitmask) and the window lookup at node group 0 / batch 0
     const bool more_batches = r1 - r0 > (uint64_t)kWinCap;
     uint16_t* wl = S.cq + warp * 256;   // this warp's candidates (word in chunk)
-    uint16_t* wu = S.cu + warp * 256;   // ... and their node (index from jf)
     uint32_t* wh = S.hits + warp * 8;   // hit bits of the warp's 256 words
     uint32_t nc = 0;
 #pragma unroll
@@ -1077,17 +1116,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     for (uint32_t i = lane; i < nc; i += 32) {
         const uint32_t q = wl[i];
         const uint64_t x = S.words[q];
-        uint32_t u;
-        if (narrow) {
-            uint32_t lo = 0, hi = nn - 1;  // nodes jf+1.. starting at or before q
-            while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.ns[mid] <= q) lo = mid + 1; else hi = mid; }
-            u = lo;
-        } else {
-            uint32_t lo = jf + 1, hi = jl + 1;  // node_off[j] <= cs + q
-            while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (a.node_off[mid] <= cs + q) lo = mid + 1; else hi = mid; }
-            u = lo - (jf + 1);
-        }
-        wu[i] = (uint16_t)min(u, 0xFFFFu);
+        const uint32_t u = seg_of(S, q);
         bool hit = false;
         if (m0 && u < ng0) {
             const int e = window_find(S, m0, u, x);
@@ -1103,8 +1132,8 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     __syncthreads();
     TL_PHASE(4, 13, tl_p);  // D: window search
     if (S.defer) {
-        // rare: chunks with more than kNodeGrp nodes or windows of more than kWinCap
-        // entries -- every batch against every node group, CTA-synchronous
+        // rare: chunks with more than kNodeGrp segments or windows of more than
+        // kWinCap entries -- every batch against every segment group, CTA-synchronous
         for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
             const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
             if (bs != r0) {
@@ -1114,21 +1143,15 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                 if (warp == 0) window_sort(S, m);
                 __syncthreads();
             }
-            for (uint32_t g0 = (bs == r0 ? kNodeGrp : 0); g0 < nn; g0 += kNodeGrp) {
-                const uint32_t ng = min((uint32_t)kNodeGrp, nn - g0);
+            for (uint32_t g0 = (bs == r0 ? kNodeGrp : 0); g0 < n_seg; g0 += kNodeGrp) {
+                const uint32_t ng = min((uint32_t)kNodeGrp, n_seg - g0);
                 __syncthreads();
-                for (uint32_t u = tid; u < ng; u += kThreads) S.nt[u] = a.node_t[jf + g0 + u];
-                __syncthreads();
+                seg_times(p, S, S.nt, g0, ng, cs, jf, jl);
                 build_live(S, S.nt, ng, m);
                 for (uint32_t i = lane; i < nc; i += 32) {
                     const uint32_t q = wl[i];
                     if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
-                    uint32_t u = wu[i];
-                    if (u == 0xFFFFu) {  // (node index beyond 16 bits: search again)
-                        uint32_t lo = jf + 1, hi = jl + 1;
-                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (a.node_off[mid] <= cs + q) lo = mid + 1; else hi = mid; }
-                        u = lo - (jf + 1);
-                    }
+                    const uint32_t u = seg_of(S, q);
                     if (u < g0 || u >= g0 + ng) continue;
                     const uint64_t x = S.words[q];
                     const int e = window_find(S, m, u - g0, x);
@@ -1154,13 +1177,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         }
         const uint32_t b = __ballot_sync(0xffffffffu, need);
         if (need) {
-            uint32_t u = wu[i];
-            if (u == 0xFFFFu) {
-                uint32_t lo = jf + 1, hi = jl + 1;
-                while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (a.node_off[mid] <= cs + q) lo = mid + 1; else hi = mid; }
-                u = lo - (jf + 1);
-            }
-            const uint32_t t = u < kNodeGrp ? S.nt0[u] : __ldg(a.node_t + jf + u);  // the word's launch position
+            const uint32_t t = seg_time(p, S, seg_of(S, q), cs + q, jf, jl);  // the word's launch position
             wq[nq + __popc(b & lanemask_lt())] = IQ{S.words[q], (uint32_t)(cs + q), t};
         }
         nq += __popc(b);
