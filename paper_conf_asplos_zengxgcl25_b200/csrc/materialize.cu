@@ -1474,8 +1474,9 @@ struct Scratch {
     std::vector<void*> bufs;
     Ctl* h_ctl = nullptr;
     int sm_count = 0;
-    cudaStream_t side = nullptr;  // the I-list sort branch (forked from / joined to the caller's stream)
-    cudaEvent_t fork = nullptr, join = nullptr, join2 = nullptr, lists = nullptr;
+    cudaStream_t side = nullptr;  // the I-list rank branch (highest priority; forked from the caller's stream)
+    cudaStream_t low = nullptr;   // the trace-check branch (default priority; joined before the call ends)
+    cudaEvent_t fork = nullptr, join = nullptr, ranked = nullptr, classified = nullptr, emitted = nullptr;
 };
 std::mutex g_mu;
 std::vector<Scratch*> g_scratch;
@@ -1556,10 +1557,12 @@ Scratch* device_scratch(cudaError_t* e) {
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
+            (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_lo)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess ||
-            (*e = cudaEventCreateWithFlags(&s.join2, cudaEventDisableTiming)) != cudaSuccess ||
-            (*e = cudaEventCreateWithFlags(&s.lists, cudaEventDisableTiming)) != cudaSuccess)
+            (*e = cudaEventCreateWithFlags(&s.ranked, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.classified, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.emitted, cudaEventDisableTiming)) != cudaSuccess)
             return nullptr;
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
@@ -1567,11 +1570,13 @@ Scratch* device_scratch(cudaError_t* e) {
 }
 
 // the whole analysis on `stream` (no synchronization).  After k_prepare (I-list
-// tile sort + registration lists) two branches:
-//   stream:           k_classify ------------------------------ [join] k_iresolve -> k_emit
-//   side (high prio): k_rank -> k_check_mi -> k_check_mm -> [join]
-// The side stream's higher priority gets the rank CTAs dispatched ahead of the
-// classify CTAs; k_iresolve needs both branches.
+// tile sort + registration lists):
+//   stream:            k_classify [classified] ............................ [emitted][join]
+//   side (high prio):  k_rank [ranked] ... [classified] k_iresolve -> k_emit [emitted]
+//   low (default):     [classified][ranked] k_check_mi -> k_check_mm [join]
+// The high-priority stream gets the rank CTAs dispatched ahead of the classify
+// CTAs and the queue resolution / emission ahead of the trace checks, which
+// fill in around them and complete the call.
 cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P* out) {
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
@@ -1601,29 +1606,41 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             // by the allocation count; surplus CTAs exit at once)
             k_rank<<<(unsigned)std::min<uint64_t>((n + 31) / 32, (uint64_t)s.sm_count * 8), kThreads, 0, s.side>>>(p);
         }
-        {
-            TimedLaunch tl("mat_check_mi", s.side);
-            if ((e = launch_pdl(k_check_mi, check_ctas, kThreads, 0, s.side, p))) return e;
-        }
-        {
-            TimedLaunch tl("mat_check_mm", s.side);
-            if ((e = launch_pdl(k_check_mm, (nb + kWarps - 1) / kWarps, kThreads, 0, s.side, p))) return e;
-        }
-        if ((e = cudaEventRecord(s.join, s.side))) return e;
+        if ((e = cudaEventRecord(s.ranked, s.side))) return e;
         if (C) {
             TimedLaunch tl("mat_classify", stream);
             if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
         }
-        if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
+        if ((e = cudaEventRecord(s.classified, stream))) return e;
+        // high priority after the classify: queue resolution and emission (the
+        // rank is already on this stream)
+        if ((e = cudaStreamWaitEvent(s.side, s.classified, 0))) return e;
         if (C) {
-            TimedLaunch tl("mat_iresolve", stream);
-            if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * 8), kThreads, 0, stream, p))) return e;
+            {
+                TimedLaunch tl("mat_iresolve", s.side);
+                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 8), kThreads, 0, s.side>>>(p);
+            }
+            TimedLaunch tl("mat_emit", s.side);
+            if ((e = launch_pdl(k_emit, C, kThreads, 0, s.side, p))) return e;
         }
+        if ((e = cudaEventRecord(s.emitted, s.side))) return e;
+        // default priority: the trace checks fill in around them
+        if ((e = cudaStreamWaitEvent(s.low, s.classified, 0)) || (e = cudaStreamWaitEvent(s.low, s.ranked, 0))) return e;
+        {
+            TimedLaunch tl("mat_check_mi", s.low);
+            k_check_mi<<<check_ctas, kThreads, 0, s.low>>>(p);
+        }
+        {
+            TimedLaunch tl("mat_check_mm", s.low);
+            if ((e = launch_pdl(k_check_mm, (nb + kWarps - 1) / kWarps, kThreads, 0, s.low, p))) return e;
+        }
+        if ((e = cudaEventRecord(s.join, s.low))) return e;
+        if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
-        TimedLaunch tl("mat_classify", stream);
-        if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
-    }
-    if (C) {
+        {
+            TimedLaunch tl("mat_classify", stream);
+            if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
+        }
         TimedLaunch tl("mat_emit", stream);
         if ((e = launch_pdl(k_emit, C, kThreads, 0, stream, p))) return e;
     }
