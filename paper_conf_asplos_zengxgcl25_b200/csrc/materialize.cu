@@ -1213,11 +1213,17 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 }
 
 // ----------------------------------------------------------------------------
-// 2d. k_check_mi (after k_rank): I-I (adjacent sorted I entries; the CTA checks
-//     256 pairs) and M-I (each mortal against the run of I entries its range
-//     meets, one warp per 32 allocation ordinals)
-__global__ void __launch_bounds__(kThreads) k_check_mi(P p) {
+// 2c. k_check (after k_rank and k_classify, default priority): the R-Q7 checks.
+//     I-I: adjacent sorted I entries (the CTA checks 256 pairs).  Per warp, a
+//     block of 32 allocation ordinals: M-M -- each mortal j against the mortals
+//     registered as live at some allocation of the block (hull-filtered,
+//     branch-free scan); M-I -- each mortal against the run of I entries its
+//     range meets (one fence search; the common "no I entry in range" case costs
+//     two more loads).
+__global__ void __launch_bounds__(kThreads) k_check(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
+    __shared__ uint64_t s_base[kWarps][32], s_end[kWarps][32];
+    __shared__ uint32_t s_tf[kWarps][32], s_idx[kWarps][32];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     pdl_trigger();
@@ -1231,74 +1237,30 @@ __global__ void __launch_bounds__(kThreads) k_check_mi(P p) {
     }
     const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = p.d.fence[f];
-    __syncthreads();
-    const uint32_t b = cta * kWarps + warp;
+    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = __ldcg(p.d.fence + f);
+    const uint32_t b0 = cta * kWarps;
+    const unsigned long long lbase = block_prefix(p.d.cnt_b, p.d.sup_b, min(b0, p.nb));  // (synchronizes)
+    const uint32_t b = b0 + warp;
+    if (b >= p.nb) return;  // whole warp
     const uint32_t j = b * kAblk + lane;
-    if (b >= p.nb || !nI) return;  // whole warp
     bool mine = false;
     medusa_alloc x{};
     const uint32_t N = a.n_nodes;
     const uint32_t t_last = N ? a.node_t[N - 1] : 0;
     if (j < a.n_alloc) {
-        x = a.alloc[j];
+        x = ld_alloc(a.alloc + j);
         mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
     }
     const uint64_t xe = x.base + x.size;
     bool bad = false;
-    // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
-    if (mine) {
-        const uint32_t e = i_count_le(s_fence, nf, stride, nI, p.d.i_base, xe - 1);  // bases < end
-        const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);
-        const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
-        // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
-        const bool freed_early = x.t_free <= t_last;
-        uint32_t k = s;
-        for (; k < e && (k % kIBlk) != 0; ++k)
-            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
-        for (; k + kIBlk <= e; k += kIBlk)
-            bad |= freed_early ? ~p.d.blk_min_ta_c[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
-        for (; k < e; ++k)
-            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
-    }
-    if (bad) flag(p.d.ctl, ST_TRACE);
-    TL_REC(9, 0, tl0);
-}
-
-// ----------------------------------------------------------------------------
-// 2c. k_check_mm (forked branch, after k_prepare): M-M -- every mortal j against
-//     the mortals registered as live at some allocation of its block of 32
-//     ordinals (one warp per block); runs while the I list is sorted and ranked.
-__global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
-    __shared__ uint64_t s_base[kWarps][kChkCap], s_end[kWarps][kChkCap];
-    __shared__ uint32_t s_tf[kWarps][kChkCap], s_idx[kWarps][kChkCap];
-    const unsigned long long tl0 = TL_NOW();
-    pdl_wait();
-    const MaterializeArgs& a = p.a;
-    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t b0 = blockIdx.x * kWarps;
-    const unsigned long long base = block_prefix(p.d.cnt_b, p.d.sup_b, min(b0, p.nb));
-    const uint32_t b = b0 + warp;
-    if (b < p.nb) {
+    // M-M
+    {
         const uint32_t cb = (lane <= warp && b0 + lane < p.nb) ? __ldcg(p.d.cnt_b + b0 + lane) : 0u;
         const uint32_t before = __reduce_add_sync(0xffffffffu, lane < warp ? cb : 0u);
-        const uint32_t j = b * kAblk + lane;
-        bool mine = false;
-        medusa_alloc x{};
-        const uint32_t N = a.n_nodes;
-        const uint32_t t_last = N ? a.node_t[N - 1] : 0;
-        if (j < a.n_alloc) {
-            x = a.alloc[j];
-            mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
-        }
-        const uint64_t xe = x.base + x.size;
-        // the block's hull: only list entries meeting it (in address, time and
-        // ordinal) can collide with one of its mortals; they are compacted first
         const uint64_t hb = warp_min_u64(mine ? x.base : ~0ull), he = warp_max_u64(mine ? xe : 0ull);
         const uint32_t hta = __reduce_min_sync(0xffffffffu, mine ? x.t_alloc : 0xFFFFFFFFu);
         const uint32_t hj = __reduce_max_sync(0xffffffffu, mine ? j : 0u);
-        bool bad = false;
-        const uint64_t r0 = base + before;
+        const uint64_t r0 = lbase + before;
         const uint64_t r1 = min(r0 + __shfl_sync(0xffffffffu, cb, warp), p.d.cap_b);
         for (uint64_t bs = r0; bs < r1 && he; bs += 32) {
             const uint32_t m = (uint32_t)min((uint64_t)32, r1 - bs);
@@ -1325,13 +1287,28 @@ __global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
                            (x.base < s_end[warp][q]);
             }
         }
-        if (bad) flag(p.d.ctl, ST_TRACE);
-        TL_REC(8, 0, tl0);
     }
-    pdl_trigger();
+    // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
+    if (mine && nI) {
+        const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);  // bases <= base
+        const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
+        uint32_t e = k0;  // bases < end
+        if (k0 < nI && p.d.i_base[k0] < xe) e = i_count_le(s_fence, nf, stride, nI, p.d.i_base, xe - 1);
+        // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
+        const bool freed_early = x.t_free <= t_last;
+        uint32_t k = s;
+        for (; k < e && (k % kIBlk) != 0; ++k)
+            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
+        for (; k + kIBlk <= e; k += kIBlk)
+            bad |= freed_early ? ~p.d.blk_min_ta_c[k / kIBlk] < x.t_free : p.d.blk_max_tf[k / kIBlk] > x.t_alloc;
+        for (; k < e; ++k)
+            bad |= freed_early ? p.d.i_rest[k].t_alloc < x.t_free : p.d.i_tf[k] > x.t_alloc;
+    }
+    if (bad) flag(p.d.ctl, ST_TRACE);
+    TL_REC(9, 0, tl0);
 }
 
-__global__ void __launch_bounds__(kThreads, 4) k_classify(P p) {
+__global__ void __launch_bounds__(kThreads, 6) k_classify(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
@@ -1573,7 +1550,7 @@ Scratch* device_scratch(cudaError_t* e) {
 // tile sort + registration lists):
 //   stream:            k_classify [classified] ............................ [emitted][join]
 //   side (high prio):  k_rank [ranked] ... [classified] k_iresolve -> k_emit [emitted]
-//   low (default):     [classified][ranked] k_check_mi -> k_check_mm [join]
+//   low (default):     [classified][ranked] k_check [join]
 // The high-priority stream gets the rank CTAs dispatched ahead of the classify
 // CTAs and the queue resolution / emission ahead of the trace checks, which
 // fill in around them and complete the call.
@@ -1627,12 +1604,8 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         // default priority: the trace checks fill in around them
         if ((e = cudaStreamWaitEvent(s.low, s.classified, 0)) || (e = cudaStreamWaitEvent(s.low, s.ranked, 0))) return e;
         {
-            TimedLaunch tl("mat_check_mi", s.low);
-            k_check_mi<<<check_ctas, kThreads, 0, s.low>>>(p);
-        }
-        {
-            TimedLaunch tl("mat_check_mm", s.low);
-            if ((e = launch_pdl(k_check_mm, (nb + kWarps - 1) / kWarps, kThreads, 0, s.low, p))) return e;
+            TimedLaunch tl("mat_check", s.low);
+            k_check<<<check_ctas, kThreads, 0, s.low>>>(p);
         }
         if ((e = cudaEventRecord(s.join, s.low))) return e;
         if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;

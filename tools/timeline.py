@@ -23,7 +23,7 @@ import __graft_entry__ as g  # noqa: E402
 NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan",
          (2, 0): "prepare/sort", (2, 1): "prepare/scatter", (3, 0): "rank",
          (4, 0): "classify",
-         (5, 0): "emit", (8, 0): "check_mm", (9, 0): "check_mi", (10, 0): "iresolve", (6, 0): "report_init", (7, 0): "restore/words", (7, 1): "restore/gather",
+         (5, 0): "emit", (8, 0): "check_mm", (9, 0): "check", (10, 0): "iresolve", (6, 0): "report_init", (7, 0): "restore/words", (7, 1): "restore/gather",
          (1, 20): " allocs:load+nj0", (1, 21): " allocs:stage", (1, 22): " allocs:search+reg",
          (1, 23): " last:fence", (1, 24): " last:scan-c", (1, 25): " last:scan-b",
          (3, 40): " rank:pdl-wait", (3, 41): " rank:staging", (3, 42): " rank:search+red", (3, 43): " rank:ticket",
