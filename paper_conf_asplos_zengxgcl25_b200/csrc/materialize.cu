@@ -1534,7 +1534,7 @@ Scratch* device_scratch(cudaError_t* e) {
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
-            (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_lo)) != cudaSuccess ||
+            (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.ranked, cudaEventDisableTiming)) != cudaSuccess ||
@@ -1602,7 +1602,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         }
         if ((e = cudaEventRecord(s.emitted, s.side))) return e;
         // default priority: the trace checks fill in around them
-        if ((e = cudaStreamWaitEvent(s.low, s.classified, 0)) || (e = cudaStreamWaitEvent(s.low, s.ranked, 0))) return e;
+        if ((e = cudaStreamWaitEvent(s.low, s.ranked, 0))) return e;
         {
             TimedLaunch tl("mat_check", s.low);
             k_check<<<check_ctas, kThreads, 0, s.low>>>(p);
