@@ -436,7 +436,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     TL_PHASE(1, 22, tl_p);  // searches, registration counts, I compaction
 }
 
-__global__ void __launch_bounds__(kThreads, 4) k_trace(P p) {
+__global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     if (blockIdx.x < p.node_ctas) {
@@ -719,7 +719,7 @@ __device__ void scatter_role(const P& p, uint32_t cta, ScatterShared& S) {
                  S.pre, S.first, S.w, S.range);
 }
 
-__global__ void __launch_bounds__(kThreads) k_prepare(P p) {
+__global__ void __launch_bounds__(kThreads, 6) k_prepare(P p) {
     __shared__ union {
         SortShared sort;
         ScatterShared scatter;
@@ -1220,7 +1220,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 //     branch-free scan); M-I -- each mortal against the run of I entries its
 //     range meets (one fence search; the common "no I entry in range" case costs
 //     two more loads).
-__global__ void __launch_bounds__(kThreads) k_check(P p) {
+__global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
     __shared__ uint64_t s_base[kWarps][32], s_end[kWarps][32];
     __shared__ uint32_t s_tf[kWarps][32], s_idx[kWarps][32];
@@ -1323,7 +1323,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_classify(P p) {
 //     one group of bases and one entry (two dependent loads); a hit writes its
 //     record at its word index and sets its mask bit; the chunk's count grows by
 //     one atomic per chunk.
-__global__ void __launch_bounds__(kThreads) k_iresolve(P p) {
+__global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
     __shared__ uint32_t s_cnt[kWarps];
     const unsigned long long tl0 = TL_NOW();
