@@ -61,7 +61,7 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-__global__ void __launch_bounds__(kThreads, 6)
+__global__ void __launch_bounds__(kThreads, 8)
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     __shared__ __align__(128) uint64_t s_words[kTaskWords];
     __shared__ uint32_t s_mask[kMaskPerTask];
