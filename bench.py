@@ -1,8 +1,9 @@
 """Benchmark of the Medusa restoration hot path on B200 (one JSON line on rank 0).
 
 A step = one pass of the whole hot path over one graph set already resident in
-HBM: medusa_materialize (classify every word + emit the indirect-index-pointer
-table) -> medusa_kernel_table_set -> medusa_restore (relocate + validate every
+HBM: medusa_kernel_table_set (install the triggering-kernel address table;
+independent of the analysis) -> medusa_materialize (classify every word + emit
+the indirect-index-pointer table) -> medusa_restore (relocate + validate every
 slot, fill every node's kernel address).  Metric (BASELINE.json): graph nodes
 restored per second, whole job; plus the relocate pass's HBM GB/s.
 
@@ -198,8 +199,8 @@ def run_ours(args):
     scrub = torch.empty(max(2 * l2, 256 << 20) // 4, dtype=torch.int32, device=dev)
 
     def step():
+        medusa.kernel_table_set(inp["table"])  # (independent of the analysis)
         medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots)
-        medusa.kernel_table_set(inp["table"])
         medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
                        dst=dst, func_out=fout, report=rep)
 
@@ -216,7 +217,7 @@ def run_ours(args):
     assert int(medusa.report_numpy(rep)[0]) == 0, "restore reported validation failures"
     n_slots = slots.n_slots
 
-    # ---- the step as one CUDA graph: materialize_async -> kernel_table_set ->
+    # ---- the step as one CUDA graph: kernel_table_set -> materialize_async ->
     #      restore(slot count from the table): the same kernels, no host round trip
     res = torch.zeros(2, dtype=torch.int64, device=dev)
     gdst = torch.empty_like(inp["words"])
@@ -224,8 +225,8 @@ def run_ours(args):
     grep = torch.empty(8, dtype=torch.int64, device=dev)
 
     def step_async():
+        medusa.kernel_table_set(inp["table"])  # (independent of the analysis)
         medusa.materialize_async(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots, result=res)
-        medusa.kernel_table_set(inp["table"])
         medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
                        dst=gdst, func_out=gfout, report=grep, from_table=True)
 
@@ -351,8 +352,8 @@ def run_ours(args):
     def e2e_step():
         for k, v in pinned.items():
             d_in[k].copy_(v, non_blocking=True)
-        medusa.materialize(d_in["words"], d_in["node_off"], d_in["node_t"], d_in["allocs"], out=slots)
         medusa.kernel_table_set(d_in["table"])
+        medusa.materialize(d_in["words"], d_in["node_off"], d_in["node_t"], d_in["allocs"], out=slots)
         medusa.restore(d_in["words"], slots, d_in["old_base"], d_in["new_base"], d_in["new_size"],
                        d_in["func_id"], dst=dst, func_out=fout, report=rep)
         out_h.copy_(dst, non_blocking=True)
@@ -407,7 +408,7 @@ def run_ours(args):
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
             "gpu_launches": len(launches),
-            "graph_step": "one CUDA graph per step: medusa_materialize_async, medusa_kernel_table_set, "
+            "graph_step": "one CUDA graph per step: medusa_kernel_table_set, medusa_materialize_async, "
                           f"medusa_restore(MEDUSA_N_SLOTS_FROM_TABLE); {len(launches) // max(args.steps, 1)} "
                           "libmedusa kernels per step",
             "sync_api_ms_per_step": max_over_ranks(sum(sync_ms), dist, dev) / args.steps,

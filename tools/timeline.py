@@ -58,8 +58,8 @@ def main():
     medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots)  # sizes scratch
 
     def step():
+        medusa.kernel_table_set(inp["table"])  # (independent of the analysis)
         medusa.materialize_async(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots, result=res)
-        medusa.kernel_table_set(inp["table"])
         medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
                        dst=dst, func_out=fout, report=rep, from_table=True)
 
