@@ -177,6 +177,33 @@ __device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* total)
     return before + x - v;
 }
 
+// block_excl_scan of two independent values at once (one pair of barriers)
+__device__ __forceinline__ void block_excl_scan2(uint32_t v0, uint32_t v1, uint32_t& e0, uint32_t& e1, uint32_t& t0,
+                                                 uint32_t& t1) {
+    __shared__ uint32_t s_w2[2][kWarps];
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t x0 = v0, x1 = v1;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y0 = __shfl_up_sync(0xffffffffu, x0, d), y1 = __shfl_up_sync(0xffffffffu, x1, d);
+        if (lane >= (uint32_t)d) { x0 += y0; x1 += y1; }
+    }
+    if (lane == 31) { s_w2[0][warp] = x0; s_w2[1][warp] = x1; }
+    __syncthreads();
+    uint32_t b0 = 0, b1 = 0;
+    t0 = t1 = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) {
+        const uint32_t a0 = s_w2[0][w], a1 = s_w2[1][w];
+        if ((uint32_t)w < warp) { b0 += a0; b1 += a1; }
+        t0 += a0;
+        t1 += a1;
+    }
+    __syncthreads();
+    e0 = b0 + x0 - v0;
+    e1 = b1 + x1 - v1;
+}
+
 // Sum of cnt[0, k) of a two-level counter (sup[g] = sum of cnt[256g, 256g + 256)):
 // at most k/256 + 255 loads, spread over the CTA, and one reduction; every thread
 // receives the value.  Call with the whole CTA (blockDim.x == kThreads == 256).
@@ -199,6 +226,31 @@ __device__ __forceinline__ unsigned long long block_prefix(const uint32_t* cnt, 
     for (int w = 0; w < kWarps; ++w) t += s_r[w];
     __syncthreads();
     return t;
+}
+
+// block_prefix of two counters at once (one reduction)
+__device__ __forceinline__ void block_prefix2(const uint32_t* cnt0, const unsigned long long* sup0, uint32_t k0,
+                                              const uint32_t* cnt1, const unsigned long long* sup1, uint32_t k1,
+                                              unsigned long long& r0, unsigned long long& r1) {
+    __shared__ unsigned long long s_r2[2][kWarps];
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    unsigned long long a0 = 0, a1 = 0;
+    const uint32_t g0 = k0 >> 8, g1 = k1 >> 8;
+    for (uint32_t q = threadIdx.x; q < g0; q += kThreads) a0 += __ldcg(sup0 + q);
+    for (uint32_t q = threadIdx.x; q < g1; q += kThreads) a1 += __ldcg(sup1 + q);
+    if ((g0 << 8) + threadIdx.x < k0) a0 += __ldcg(cnt0 + (g0 << 8) + threadIdx.x);
+    if ((g1 << 8) + threadIdx.x < k1) a1 += __ldcg(cnt1 + (g1 << 8) + threadIdx.x);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+        a0 += __shfl_xor_sync(0xffffffffu, a0, d);
+        a1 += __shfl_xor_sync(0xffffffffu, a1, d);
+    }
+    if (lane == 0) { s_r2[0][warp] = a0; s_r2[1][warp] = a1; }
+    __syncthreads();
+    r0 = r1 = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) { r0 += s_r2[0][w]; r1 += s_r2[1][w]; }
+    __syncthreads();
 }
 
 // first index k in [lo, n) with t[k] >= x (galloping from lo; t ascending)
@@ -634,89 +686,104 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
     }
 }
 
-// One registration list (chunks or check blocks): the CTA's 256 allocations
-// register in keys [lo_i, hi_i] (empty when lo_i > hi_i).  Keys are handled in
-// tiles of 256: a tile's list offsets = block_prefix + a CTA scan of the counts;
-// the tile's (allocation, key) pairs are dealt out evenly over the CTA, so one
-// long-lived allocation does not serialize its warp.
-__device__ void scatter_list(const P& p, const uint32_t* cnt, const unsigned long long* sup, uint32_t* fill,
-                             WinRec* list, uint64_t cap, unsigned long long* need, uint32_t lo_i, uint32_t hi_i,
-                             const WinRec& w, uint32_t* s_off, uint32_t* s_pre, uint32_t* s_first, WinRec* s_w,
-                             uint32_t* s_range) {
-    const uint32_t tid = threadIdx.x;
-    const bool has = lo_i <= hi_i;
-    if (tid == 0) { s_range[0] = 0xFFFFFFFFu; s_range[1] = 0; }
-    __syncthreads();
-    {
-        const uint32_t mn = __reduce_min_sync(0xffffffffu, has ? lo_i : 0xFFFFFFFFu);
-        const uint32_t mx = __reduce_max_sync(0xffffffffu, has ? hi_i : 0u);
-        if ((tid & 31) == 0 && mn <= mx) { atomicMin(&s_range[0], mn); atomicMax(&s_range[1], mx); }
-    }
-    s_w[tid] = w;
-    __syncthreads();
-    const uint32_t lo = s_range[0], hi = s_range[1];
-    if (lo > hi) return;  // whole CTA
-    unsigned long long base = block_prefix(cnt, sup, lo);
-    for (uint32_t t0 = lo; t0 <= hi; t0 += kThreads) {
-        // list offset of every key of the tile
-        const uint32_t key = t0 + tid;
-        uint32_t tile_total;
-        const uint32_t ex = block_excl_scan(key <= hi ? __ldcg(cnt + key) : 0u, &tile_total);
-        s_off[tid] = (uint32_t)min(base + ex, 0xFFFFFFFFull);
-        base += tile_total;
-        // this thread's pairs inside the tile, dealt out over the CTA
-        const uint32_t a = max(lo_i, t0), b = min(hi_i, t0 + kThreads - 1);
-        const uint32_t len = (has && a <= b && a <= hi_i) ? b - a + 1 : 0u;
-        uint32_t n_pairs;
-        const uint32_t pre = block_excl_scan(len, &n_pairs);
-        s_pre[tid] = pre;
-        s_first[tid] = a;
-        __syncthreads();
-        for (uint32_t q0 = 0; q0 < n_pairs; q0 += kThreads) {
-            const uint32_t q = q0 + tid;
-            const bool act = q < n_pairs;
-            uint32_t own = 0, k = 0;
-            if (act) {  // owner: last thread whose pair range starts at or before q
-                uint32_t l = 0, h = kThreads;
-                while (h - l > 1) { const uint32_t m = (l + h) >> 1; if (s_pre[m] <= q) l = m; else h = m; }
-                own = l;
-                k = s_first[own] + (q - s_pre[own]);
-            }
-            const uint32_t rank = warp_agg_inc(fill, act ? k : 0, act);
-            if (act) {
-                const uint64_t pos = (uint64_t)s_off[k - t0] + rank;
-                if (pos < cap) {
-                    list[pos] = s_w[own];
-                } else {
-                    atomicMax(need, (unsigned long long)pos + 1);
-                    flag(p.d.ctl, ST_OVERFLOW);
-                }
-            }
-        }
-        __syncthreads();  // s_off / s_pre / s_first are rewritten by the next tile
-    }
-}
-
+// Registration lists (l = 0: chunks, l = 1: check blocks): allocation i of the
+// CTA registers in keys [lo_l, hi_l] (empty when lo > hi).  Both lists are built
+// in the same pass (shared barriers and load rounds).  Keys are handled in tiles
+// of 256: a tile's list offsets = group prefix (block_prefix2) + a CTA scan of
+// the counts; the tile's (allocation, key) pairs of both lists are dealt out
+// evenly over the CTA, so one long-lived allocation does not serialize its warp.
 struct ScatterShared {
-    uint32_t off[kThreads], pre[kThreads], first[kThreads], range[2];
+    uint32_t off[2][kThreads], pre[2][kThreads], first[2][kThreads], range[2][2];
     WinRec w[kThreads];
 };
 
 __device__ void scatter_role(const P& p, uint32_t cta, ScatterShared& S) {
-    const uint32_t i = cta * kThreads + threadIdx.x;
+    const uint32_t tid = threadIdx.x;
+    const uint32_t i = cta * kThreads + tid;
     const bool valid = i < p.a.n_alloc;
     uint4 r = make_uint4(1, 0, 1, 0);
     if (valid) r = p.d.rng[i];
     WinRec w{};
     if (r.x <= r.y || r.z <= r.w) {
-        const medusa_alloc x = p.a.alloc[i];
+        const medusa_alloc x = ld_alloc(p.a.alloc + i);
         w = WinRec{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
     }
-    scatter_list(p, p.d.cnt_c, p.d.sup_c, p.d.fill_c, p.d.list_c, p.d.cap_c, &p.d.ctl->need_c, r.x, r.y, w, S.off,
-                 S.pre, S.first, S.w, S.range);
+    const uint32_t lo_i[2] = {r.x, r.z}, hi_i[2] = {r.y, r.w};
+    const uint32_t* cnt[2] = {p.d.cnt_c, p.d.cnt_b};
+    if (tid < 2) { S.range[tid][0] = 0xFFFFFFFFu; S.range[tid][1] = 0; }
+    S.w[tid] = w;
     __syncthreads();
-    scatter_list(p, p.d.cnt_b, p.d.sup_b, p.d.fill_b, p.d.list_b, p.d.cap_b, &p.d.ctl->need_b, r.z, r.w, w, S.off,
-                 S.pre, S.first, S.w, S.range);
+#pragma unroll
+    for (int l = 0; l < 2; ++l) {
+        const bool has = lo_i[l] <= hi_i[l];
+        const uint32_t mn = __reduce_min_sync(0xffffffffu, has ? lo_i[l] : 0xFFFFFFFFu);
+        const uint32_t mx = __reduce_max_sync(0xffffffffu, has ? hi_i[l] : 0u);
+        if ((tid & 31) == 0 && mn <= mx) { atomicMin(&S.range[l][0], mn); atomicMax(&S.range[l][1], mx); }
+    }
+    __syncthreads();
+    const uint32_t lo[2] = {S.range[0][0], S.range[1][0]}, hi[2] = {S.range[0][1], S.range[1][1]};
+    const bool any[2] = {lo[0] <= hi[0], lo[1] <= hi[1]};
+    if (!any[0] && !any[1]) return;  // whole CTA
+    unsigned long long base[2];
+    block_prefix2(cnt[0], p.d.sup_c, any[0] ? lo[0] : 0, cnt[1], p.d.sup_b, any[1] ? lo[1] : 0, base[0], base[1]);
+    const uint32_t ntile = max(any[0] ? (hi[0] - lo[0]) / kThreads + 1 : 0u, any[1] ? (hi[1] - lo[1]) / kThreads + 1 : 0u);
+    for (uint32_t t = 0; t < ntile; ++t) {
+        uint32_t t0[2], v[2], len[2], a_[2];
+#pragma unroll
+        for (int l = 0; l < 2; ++l) {
+            t0[l] = lo[l] + t * kThreads;
+            const uint32_t key = t0[l] + tid;
+            v[l] = (any[l] && key <= hi[l]) ? __ldcg(cnt[l] + key) : 0u;
+            const uint32_t a = max(lo_i[l], t0[l]), b = min(hi_i[l], t0[l] + kThreads - 1);
+            len[l] = (any[l] && lo_i[l] <= hi_i[l] && a <= b) ? b - a + 1 : 0u;
+            a_[l] = a;
+        }
+        uint32_t ex0, ex1, tot0, tot1;
+        block_excl_scan2(v[0], v[1], ex0, ex1, tot0, tot1);
+        S.off[0][tid] = (uint32_t)min(base[0] + ex0, 0xFFFFFFFFull);
+        S.off[1][tid] = (uint32_t)min(base[1] + ex1, 0xFFFFFFFFull);
+        base[0] += tot0;
+        base[1] += tot1;
+        uint32_t p0, p1, np0, np1;
+        block_excl_scan2(len[0], len[1], p0, p1, np0, np1);
+        S.pre[0][tid] = p0;
+        S.pre[1][tid] = p1;
+        S.first[0][tid] = a_[0];
+        S.first[1][tid] = a_[1];
+        __syncthreads();
+        const uint32_t total = np0 + np1;
+        for (uint32_t q0 = 0; q0 < total; q0 += kThreads) {
+            const uint32_t q = q0 + tid;
+            const bool act = q < total;
+            const uint32_t l = q < np0 ? 0u : 1u;
+            const uint32_t qq = l ? q - np0 : q;
+            uint32_t own = 0, k = 0;
+            if (act) {  // owner: last thread whose pair range starts at or before qq
+                const uint32_t* pre = S.pre[l];
+                uint32_t lo2 = 0, hi2 = kThreads;
+                while (hi2 - lo2 > 1) { const uint32_t m = (lo2 + hi2) >> 1; if (pre[m] <= qq) lo2 = m; else hi2 = m; }
+                own = lo2;
+                k = S.first[l][own] + (qq - pre[own]);
+            }
+            // one atomic per distinct (list, key) of the warp
+            const uint32_t tag = act ? (k | (l << 31)) : 0xFFFFFFFFu;
+            const uint32_t peers = __match_any_sync(0xffffffffu, tag);
+            const uint32_t leader = __ffs(peers) - 1;
+            uint32_t rb = 0;
+            if (act && (tid & 31) == leader) rb = atomicAdd((l ? p.d.fill_b : p.d.fill_c) + k, (uint32_t)__popc(peers));
+            rb = __shfl_sync(0xffffffffu, rb, leader);
+            if (act) {
+                const uint64_t pos = (uint64_t)S.off[l][k - (l ? t0[1] : t0[0])] + rb + __popc(peers & lanemask_lt());
+                if (pos < (l ? p.d.cap_b : p.d.cap_c)) {
+                    (l ? p.d.list_b : p.d.list_c)[pos] = S.w[own];
+                } else {
+                    atomicMax(l ? &p.d.ctl->need_b : &p.d.ctl->need_c, (unsigned long long)pos + 1);
+                    flag(p.d.ctl, ST_OVERFLOW);
+                }
+            }
+        }
+        __syncthreads();  // off / pre / first are rewritten by the next tile
+    }
 }
 
 __global__ void __launch_bounds__(kThreads, 6) k_prepare(P p) {
