@@ -357,6 +357,7 @@ __device__ void nodes_role(const P& p, uint64_t i) {
 }
 
 constexpr int kTWin = 2048;  // node times / allocation times staged per alloc CTA
+constexpr int kNodesPerThread = 4;  // node role of k_trace (keeps its grid inside one wave)
 
 __device__ void allocs_role(const P& p, uint32_t cta) {
     __shared__ uint32_t s_nt[kTWin];  // node_t[nj0, nj0 + nw)
@@ -491,8 +492,10 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
 __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
-    if (blockIdx.x < p.node_ctas) {
-        nodes_role(p, (uint64_t)blockIdx.x * blockDim.x + threadIdx.x);
+    if (blockIdx.x < p.node_ctas) {  // kNodesPerThread nodes per thread, CTA-strided
+#pragma unroll
+        for (int k = 0; k < kNodesPerThread; ++k)
+            nodes_role(p, ((uint64_t)blockIdx.x * kNodesPerThread + k) * blockDim.x + threadIdx.x);
         TL_REC(1, 0, tl0);
     } else {
         allocs_role(p, blockIdx.x - p.node_ctas);
@@ -1625,7 +1628,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
     const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
-    const uint32_t node_ctas = (a.n_nodes + 1 + kThreads - 1) / kThreads;
+    const uint32_t node_ctas = (a.n_nodes + 1 + kThreads * kNodesPerThread - 1) / (kThreads * kNodesPerThread);
     const uint32_t alloc_ctas = (uint32_t)((n + kThreads - 1) / kThreads);
     const uint32_t sort_ctas = (uint32_t)((n + kSortTile - 1) / kSortTile);
     const uint32_t check_ctas = n ? std::max<uint32_t>((nb + kWarps - 1) / kWarps, alloc_ctas) : 0;
