@@ -37,6 +37,8 @@ thread_local std::vector<TimingRec> g_timing_recs;
 
 }  // namespace
 
+bool timing_enabled() { return g_timing; }
+
 TimedLaunch::TimedLaunch(const char* n, cudaStream_t s) : name(n), stream(s), slot(nullptr) {
     if (!g_timing) return;
     TimingRec r{n, nullptr, nullptr};

@@ -65,7 +65,10 @@ inline cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned 
 }
 
 // ---- instrumentation (api.cu) -------------------------------------------------
-// Brackets one launch with events when the calling thread enabled timing.
+// Brackets one launch with events when the calling thread enabled timing.  While
+// timing is on, materialize runs its branches serially on the caller's stream, so
+// every kernel's duration is its own (no concurrent branch inside the events).
+bool timing_enabled();
 struct TimedLaunch {
     TimedLaunch(const char* name, cudaStream_t s);
     ~TimedLaunch();

@@ -1635,6 +1635,9 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     P p{a, s.d, C, nb, node_ctas, sort_ctas, check_ctas};
     *out = p;
     cudaError_t e;
+    // branches (serialized on the caller's stream while per-launch timing is on)
+    const bool serial = timing_enabled();
+    cudaStream_t side = serial ? stream : s.side, low = serial ? stream : s.low;
     if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) return e;
     if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) return e;
     {
@@ -1646,14 +1649,14 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             TimedLaunch tl("mat_prepare", stream);
             if ((e = launch_pdl(k_prepare, sort_ctas + alloc_ctas, kThreads, 0, stream, p))) return e;
         }
-        if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(s.side, s.fork, 0))) return e;
+        if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(side, s.fork, 0))) return e;
         {
-            TimedLaunch tl("mat_rank", s.side);
+            TimedLaunch tl("mat_rank", side);
             // one CTA per 32 I keys (the list's size is known on the device only: bound
             // by the allocation count; surplus CTAs exit at once)
-            k_rank<<<(unsigned)std::min<uint64_t>((n + 31) / 32, (uint64_t)s.sm_count * 8), kThreads, 0, s.side>>>(p);
+            k_rank<<<(unsigned)std::min<uint64_t>((n + 31) / 32, (uint64_t)s.sm_count * 8), kThreads, 0, side>>>(p);
         }
-        if ((e = cudaEventRecord(s.ranked, s.side))) return e;
+        if ((e = cudaEventRecord(s.ranked, side))) return e;
         if (C) {
             TimedLaunch tl("mat_classify", stream);
             if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
@@ -1661,23 +1664,23 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaEventRecord(s.classified, stream))) return e;
         // high priority after the classify: queue resolution and emission (the
         // rank is already on this stream)
-        if ((e = cudaStreamWaitEvent(s.side, s.classified, 0))) return e;
+        if ((e = cudaStreamWaitEvent(side, s.classified, 0))) return e;
         if (C) {
             {
-                TimedLaunch tl("mat_iresolve", s.side);
-                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 8), kThreads, 0, s.side>>>(p);
+                TimedLaunch tl("mat_iresolve", side);
+                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 8), kThreads, 0, side>>>(p);
             }
-            TimedLaunch tl("mat_emit", s.side);
-            if ((e = launch_pdl(k_emit, C, kThreads, 0, s.side, p))) return e;
+            TimedLaunch tl("mat_emit", side);
+            if ((e = launch_pdl(k_emit, C, kThreads, 0, side, p))) return e;
         }
-        if ((e = cudaEventRecord(s.emitted, s.side))) return e;
+        if ((e = cudaEventRecord(s.emitted, side))) return e;
         // default priority: the trace checks fill in around them
-        if ((e = cudaStreamWaitEvent(s.low, s.ranked, 0))) return e;
+        if ((e = cudaStreamWaitEvent(low, s.ranked, 0))) return e;
         {
-            TimedLaunch tl("mat_check", s.low);
-            k_check<<<check_ctas, kThreads, 0, s.low>>>(p);
+            TimedLaunch tl("mat_check", low);
+            k_check<<<check_ctas, kThreads, 0, low>>>(p);
         }
-        if ((e = cudaEventRecord(s.join, s.low))) return e;
+        if ((e = cudaEventRecord(s.join, low))) return e;
         if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
         {
