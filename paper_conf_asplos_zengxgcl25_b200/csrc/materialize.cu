@@ -1124,17 +1124,21 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
     if (tid < MEDUSA_CHUNK_WORDS / 32) S.nsm[tid] = 0;
+    if (tid < kNodeGrp) S.nt0[tid] = 0;
+    const uint32_t t_jf = N ? __ldg(a.node_t + jf) : 0;
     const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);  // (synchronizes the CTA)
     const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
     TL_PHASE(4, 10, tl_p);  // A: setup
     // B. one round of loads: threads 0..127 the first window batch, threads
     //    128..255 the starts of the chunk's nodes (-> start bitmask)
     const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
+    uint32_t my_q = 0xFFFFFFFFu, my_t = 0;  // this thread's first node (start, launch position)
     if (tid < kWinCap) {
         window_load(p, S, r0, m0);
     } else {
         for (uint32_t j = jf + 1 + (tid - kWinCap); j <= jl; j += kThreads - kWinCap) {
             const uint32_t q = (uint32_t)(a.node_off[j] - cs);
+            if (my_q == 0xFFFFFFFFu) { my_q = q; my_t = a.node_t[j]; }
             atomicOr(&S.nsm[q >> 5], 1u << (q & 31));
         }
     }
@@ -1154,7 +1158,19 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     __syncthreads();
     const uint32_t n_seg = N ? S.nsp[63] + __popc(S.nsm[63]) + 1 : 0;
     const uint32_t ng0 = min((uint32_t)kNodeGrp, n_seg);
-    seg_times(p, S, S.nt0, 0, ng0, cs, jf, jl);
+    // launch positions of segments 0..ng0-1 (the last node of a start is its non-empty one)
+    if (tid == 0 && N) atomicMax(&S.nt0[0], t_jf);
+    if (my_q != 0xFFFFFFFFu) {
+        const uint32_t sg = seg_of(S, my_q);
+        if (sg < kNodeGrp) atomicMax(&S.nt0[sg], my_t);
+    }
+    if (nn > (uint32_t)(kThreads - kWinCap) + 1) {  // more nodes than threads 128..255: the rest
+        for (uint32_t j = jf + 1 + (kThreads - kWinCap) + tid; j <= jl; j += kThreads) {
+            const uint32_t sg = seg_of(S, (uint32_t)(a.node_off[j] - cs));
+            if (sg < kNodeGrp) atomicMax(&S.nt0[sg], a.node_t[j]);
+        }
+    }
+    __syncthreads();
     TL_PHASE(4, 11, tl_p);  // B: window records, node starts, sort
     if (m0) build_live(S, S.nt0, ng0, m0);
     if (tma) {
