@@ -293,6 +293,13 @@ def run_ours(args):
     rl = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
           "frac": achieved / peak, "traffic": traffic.get(dom), "peak_source": peak_src,
           "alg_bytes_per_launch": alg[dom]}
+    inst = traffic.get("_inst", {}).get(dom)
+    if inst:  # the instruction-issue view: warp instructions per launch from the
+        # committed ncu launch list / this run's launch duration, against 4 schedulers x SMs x clock
+        sm_count = torch.cuda.get_device_properties(dev).multi_processor_count
+        issue_peak = 4 * sm_count * 1.965e9 / 1e12  # T warp-instructions/s at the 1965 MHz max SM clock
+        rl["issue"] = {"warp_inst_per_launch": inst, "achieved": inst / dom_avg_s / 1e12, "peak": issue_peak,
+                       "unit": "T warp-inst/s", "frac": inst / dom_avg_s / 1e12 / issue_peak}
     rst = per["restore"]
     restore_avg_s = rst[1] / rst[0] / 1e3
     relocate = {"kernel": "restore", "GB/s": alg["restore"] / restore_avg_s / 1e9,

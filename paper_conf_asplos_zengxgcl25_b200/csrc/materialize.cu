@@ -956,6 +956,7 @@ struct ClsShared {
     uint16_t cq[MEDUSA_CHUNK_WORDS];        // per warp (256 each): its candidates (word in chunk)
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32]; // slot bits (warp w: words 8w .. 8w+7)
     uint32_t wcnt[kWarps];                  // slots found per warp
+    uint64_t hull_lo, hull_hi;              // [least base, greatest end) of the current window batch
     uint32_t defer;                         // some candidate needs a later node group / window batch
     unsigned long long mbar;
 };
@@ -991,6 +992,7 @@ __device__ __forceinline__ void window_sort_e(ClsShared& S, uint32_t m) {
         pl[r] = e;
     }
     warp_bitonic<E>(k, v, pl);
+    uint64_t hi = 0;
 #pragma unroll
     for (int r = 0; r < E; ++r) {
         const uint32_t e = lane * E + r;
@@ -1001,7 +1003,13 @@ __device__ __forceinline__ void window_sort_e(ClsShared& S, uint32_t m) {
             S.wta[e] = v[r];
             S.wtf[e] = S.rtf[q];
             S.wid[e] = S.rid[q];
+            hi = max(hi, S.re[q]);
         }
+    }
+    hi = warp_max_u64(hi);
+    if (lane == 0) {  // the batch's address hull: words outside it skip the lookup
+        S.hull_lo = k[0];  // lane 0 holds the smallest base
+        S.hull_hi = hi;
     }
 }
 
@@ -1054,6 +1062,7 @@ __device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uin
 // the live entries of one launch are pairwise disjoint, so the only possible
 // container is the live entry with the greatest base <= x.
 __device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint32_t ul, uint64_t x) {
+    if (x < S.hull_lo || x >= S.hull_hi) return -1;
     uint32_t lo = 0, hi = m;  // entries with base <= x
     while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
     for (int w = ((int)lo - 1) >> 5; w >= 0; --w) {

@@ -6,11 +6,12 @@ import sys
 
 NAMES = {"k_classify": "mat_classify", "restore_kernel": "restore", "k_trace": "mat_trace",
          "k_prepare": "mat_prepare", "k_rank": "mat_rank", "k_check_mi": "mat_check_mi",
-         "k_check_mm": "mat_check_mm", "k_iresolve": "mat_iresolve", "k_emit": "mat_emit"}
+         "k_check_mm": "mat_check_mm", "k_check": "mat_check", "k_iresolve": "mat_iresolve", "k_emit": "mat_emit"}
 rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 10]
 h = rows[0]
 ix = {k: i for i, k in enumerate(h)}
 per = {}
+inst = {}
 for r in rows[1:]:
     if r[ix["ID"]] == "ID":
         continue
@@ -18,10 +19,13 @@ for r in rows[1:]:
     if name not in NAMES:
         continue
     m = r[ix["Metric Name"]]
-    if m not in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+    if m not in ("dram__bytes_read.sum", "dram__bytes_write.sum", "smsp__inst_executed.sum"):
         continue
     v = float(r[ix["Metric Value"]].replace(",", ""))
     u = r[ix["Metric Unit"]]
+    if m == "smsp__inst_executed.sum":
+        inst[NAMES[name]] = v * {"inst": 1, "Kinst": 1e3, "Minst": 1e6, "Ginst": 1e9}.get(u, 1)
+        continue
     v *= {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}.get(u, 1)
     key = (NAMES[name], int(r[ix["ID"]]))
     per.setdefault(key, 0.0)
@@ -29,6 +33,7 @@ for r in rows[1:]:
 out = {}
 for (bench_name, kid), v in sorted(per.items(), key=lambda kv: kv[0][1]):
     out[bench_name] = v  # the last launch wins
+out["_inst"] = inst  # warp instructions per launch (smsp__inst_executed.sum), same launches
 out["_note"] = ("per-launch dram__bytes_read.sum + dram__bytes_write.sum of the last bench step in the ncu launch "
                 f"list {sys.argv[1].split('/')[-1]} (--clock-control none; ncu flushes caches between launches, so "
                 "this is cold-cache traffic)")
