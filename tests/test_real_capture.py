@@ -1,0 +1,44 @@
+"""NEXT-1 / NEXT-2 on the device: a real PyTorch decoder captured
+into a CUDA graph, its allocation trace and kernel-node parameter image
+materialized by libmedusa (checked against the oracle), restored for a second
+address space (replayed allocations), written back into a clone of the
+graph, and run: the output must equal the original graph's bit for bit, with
+every original buffer poisoned."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover - CPU-only hosts
+    pytest.skip("needs a GPU", allow_module_level=True)
+pytest.importorskip("cuda.bindings.driver")
+
+import oracle  # noqa: E402
+import paper_conf_asplos_zengxgcl25_b200 as medusa  # noqa: E402
+from workloads.capture import real_graph  # noqa: E402
+
+
+def test_real_graph_materialize_restore_replay():
+    r = real_graph.end_to_end(torch, medusa)
+    assert r["n_kernel"] > 20
+    # allocations made during the capture exist (the graph's pool), and were
+    # poisoned in the second arena before the rebuilt graph ran
+    assert len(r["allocs"]) > r["n_pre"] > 0
+    # the GPU table equals the oracle's on the real trace
+    m = oracle.materialize(r["words"], r["off"], r["node_t"], r["allocs"])
+    assert m["status"] == 0
+    mask, cb, rec = oracle.pack(m, r["words"].size)
+    s = r["slots"]
+    assert s.n_slots == m["n_slots"] > 0
+    assert np.array_equal(medusa.to_numpy_u64(s.slot)[: s.n_slots], rec)
+    assert np.array_equal(s.mask.cpu().numpy().view(np.uint32), mask)
+    # restore: every slot valid; the oracle restores the same bytes
+    assert int(r["report"][0]) == 0
+    dst_o, _, rep_o = oracle.restore(r["words"], m["slot_g"], m["slot_id"], m["slot_off"], r["allocs"]["base"],
+                                     r["new_base"], r["allocs"]["size"])
+    assert np.array_equal(r["restored"], dst_o) and int(rep_o[0]) == 0
+    # every rebuilt graph computes the same output, bit for bit
+    assert r["n_graphs"] == 4
+    for ob, ref in zip(r["outs_b"], r["refs"]):
+        assert torch.equal(ob, ref)

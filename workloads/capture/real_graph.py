@@ -1,0 +1,395 @@
+"""Real-capture workload and end-to-end check.
+
+A small decoder (random weights, no network) is captured into a CUDA graph by
+PyTorch.  The graph's memory comes from a torch.cuda.MemPool whose segments are
+served by the tracing allocator in trace_alloc.cpp, which logs every segment
+allocation / free together with the number of nodes the capturing graph held
+at that moment: one total order of allocations and kernel launches.
+The parameter image is read from the captured graph itself:
+cuGraphKernelNodeGetParams gives each kernel node's function and argument
+pointers, cuFuncGetParamInfo / cuKernelGetParamInfo the device-side layout
+(offset, size) of every argument (Fig. 4d); memset nodes contribute
+their destination pointer as a one-word blob.
+
+The "online process" is emulated in the same process (same kernel handles, so
+the kernel table of §5 is not exercised here): the allocation sequence is
+replayed in a second arena (different addresses), the contents of every
+traced segment are copied over (= loading the same weights and inputs), the
+first arena is poisoned, and a clone of the graph gets every kernel / memset
+node's parameters replaced by the restored image (cuGraphKernelNodeSetParams,
+NEXT-2).  Its output must equal, bit for bit, the output the original graph
+produced; a pointer the analysis missed would read poisoned memory.
+
+Device-only module (needs a GPU, the CUDA driver bindings and torch).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB = os.path.join(HERE, "libtrace_alloc.so")
+SRC = os.path.join(HERE, "trace_alloc.cpp")
+T_END = 0xFFFFFFFF
+
+
+def build(force=False):
+    """Compile the tracing allocator (plain C++ against the CUDA runtime)."""
+    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
+        subprocess.run(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-I/usr/local/cuda/include", "-o", LIB, SRC,
+                        "-L/usr/local/cuda/lib64", "-lcudart"], check=True, capture_output=True)
+    return LIB
+
+
+def _lib():
+    L = ctypes.CDLL(build())
+    L.ta_init.argtypes = [ctypes.c_uint64]
+    L.ta_init.restype = ctypes.c_int
+    L.ta_select.argtypes = [ctypes.c_int]
+    L.ta_log.argtypes = [ctypes.c_int]
+    L.ta_capture_begin.argtypes = [ctypes.c_int64]
+    L.ta_raw_malloc.argtypes = [ctypes.c_uint64]
+    L.ta_raw_malloc.restype = ctypes.c_uint64
+    L.ta_events.argtypes = [ctypes.POINTER(ctypes.c_int64), ctypes.c_int64]
+    L.ta_events.restype = ctypes.c_int64
+    L.ta_arena_base.argtypes = [ctypes.c_int]
+    L.ta_arena_base.restype = ctypes.c_uint64
+    return L
+
+
+def tiny_decoder(torch, d=256, layers=2, vocab=512, heads=4):
+    """A decoder-only transformer with random weights: embedding, per layer RMSNorm
+    + causal attention + SwiGLU MLP (cuBLAS GEMMs, softmax, elementwise), lm head."""
+    nn = torch.nn
+
+    class Layer(nn.Module):
+        def __init__(self):
+            super().__init__()
+            self.n1 = nn.Parameter(torch.rand(d) + 0.5)
+            self.qkv = nn.Linear(d, 3 * d, bias=False)
+            self.o = nn.Linear(d, d, bias=False)
+            self.n2 = nn.Parameter(torch.rand(d) + 0.5)
+            self.up = nn.Linear(d, 4 * d, bias=False)
+            self.gate = nn.Linear(d, 4 * d, bias=False)
+            self.down = nn.Linear(4 * d, d, bias=False)
+
+        def forward(self, x, mask):
+            b, s, _ = x.shape
+            h = x * torch.rsqrt(x.pow(2).mean(-1, keepdim=True) + 1e-6) * self.n1
+            q, k, v = self.qkv(h).view(b, s, 3, heads, d // heads).permute(2, 0, 3, 1, 4)
+            a = torch.softmax((q @ k.transpose(-1, -2)) * (d // heads) ** -0.5 + mask, dim=-1) @ v
+            x = x + self.o(a.transpose(1, 2).reshape(b, s, d))
+            h = x * torch.rsqrt(x.pow(2).mean(-1, keepdim=True) + 1e-6) * self.n2
+            return x + self.down(torch.nn.functional.silu(self.gate(h)) * self.up(h))
+
+    class Model(nn.Module):
+        def __init__(self):
+            super().__init__()
+            self.emb = nn.Embedding(vocab, d)
+            self.layers = nn.ModuleList([Layer() for _ in range(layers)])
+            self.head = nn.Linear(d, vocab, bias=False)
+
+        def forward(self, ids, mask):
+            x = self.emb(ids)
+            for layer in self.layers:
+                x = layer(x, mask)
+            return self.head(x)
+
+    return Model()
+
+
+def _check(res):
+    """The value(s) of a cuda-python call after checking its error code."""
+    if not isinstance(res, tuple):
+        res = (res,)
+    if int(res[0]) != 0:
+        raise RuntimeError(f"CUDA call failed: {res[0]}")
+    if len(res) == 1:
+        return None
+    return res[1] if len(res) == 2 else res[1:]
+
+
+def _param_layout(cu, params):
+    """[(offset, size)] of every argument of a kernel node (device-side layout)."""
+    out = []
+    kern = int(params.kern) if params.kern is not None else 0
+    for i in range(4096):
+        r = cu.cuKernelGetParamInfo(params.kern, i) if kern else cu.cuFuncGetParamInfo(params.func, i)
+        if int(r[0]) != 0:
+            break
+        out.append((int(r[1]), int(r[2])))
+    return out
+
+
+def capture(torch, batches=(8, 4, 2, 1), seq=16, seed=0, arena_bytes=1 << 30):
+    """Process A: build the model in the traced pool and capture one forward per
+    batch size into its own CUDA graph, largest first, all graphs sharing one
+    memory pool (vLLM's order); replay each once.  Returns the graphs, each
+    graph's nodes in launch order, the trace and the reference outputs."""
+    from cuda.bindings import driver as cu
+
+    L = _lib()
+    if L.ta_init(arena_bytes) != 0:
+        raise RuntimeError("tracing allocator: cudaMalloc of the arenas failed")
+    alloc = torch.cuda.memory.CUDAPluggableAllocator(build(), "ta_malloc", "ta_free")
+    L.ta_select(0)
+    L.ta_clear()
+    L.ta_log(1)
+    pool = torch.cuda.MemPool(alloc.allocator())
+    torch.manual_seed(seed)
+    with torch.cuda.use_mem_pool(pool):
+        model = tiny_decoder(torch).cuda().eval()
+        ids = torch.randint(0, 512, (max(batches), seq), device="cuda")  # static input, sliced per graph
+        mask = torch.full((seq, seq), float("-inf"), device="cuda").triu(1)
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s), torch.no_grad():
+            for b in batches:
+                model(ids[:b], mask)
+        torch.cuda.current_stream().wait_stream(s)
+        torch.cuda.synchronize()
+    graphs, outs = [], []
+    for k, b in enumerate(batches):
+        g = torch.cuda.CUDAGraph(keep_graph=True)  # (raw_cuda_graph needs the graph kept)
+        L.ta_capture_begin(k)
+        with torch.no_grad(), torch.cuda.graph(g, pool=pool.id):
+            outs.append(model(ids[:b], mask))
+        L.ta_capture_end()
+        graphs.append(g)
+    L.ta_log(0)
+    for g in graphs:
+        g.instantiate()
+        g.replay()
+    torch.cuda.synchronize()
+    refs = [o.detach().cpu().clone() for o in outs]
+
+    # the trace
+    n_ev = L.ta_events(None, 0)
+    buf = (ctypes.c_int64 * (5 * n_ev))()
+    L.ta_events(buf, n_ev)
+    ev = np.frombuffer(buf, dtype=np.int64).reshape(n_ev, 5).copy()
+
+    # every graph's nodes in launch order (a stream capture is one chain)
+    raw, orders = [], []
+    for g in graphs:
+        graph = cu.CUgraph(g.raw_cuda_graph())
+        n_all = int(cu.cuGraphGetNodes(graph, 0)[2])
+        orders.append(_topo(cu, list(cu.cuGraphGetNodes(graph, n_all)[1])))
+        raw.append(graph)
+    return dict(L=L, pool=pool, alloc=alloc, model=model, ids=ids, mask=mask, graph_objs=graphs, graphs=raw,
+                nodes=orders, events=ev, outs=outs, refs=refs)
+
+
+def _topo(cu, nodes):
+    """Nodes in dependency order (ties by creation order)."""
+    idx = {int(n): k for k, n in enumerate(nodes)}
+    indeg = {}
+    succ = {int(n): [] for n in nodes}
+    for n in nodes:
+        r = cu.cuGraphNodeGetDependencies(n, 0)
+        cnt = int(r[2])
+        deps = list(cu.cuGraphNodeGetDependencies(n, cnt)[1]) if cnt else []
+        indeg[int(n)] = len(deps)
+        for d_ in deps:
+            succ[int(d_)].append(n)
+    ready = sorted([n for n in nodes if indeg[int(n)] == 0], key=lambda n: idx[int(n)])
+    out = []
+    while ready:
+        n = ready.pop(0)
+        out.append(n)
+        for m in succ[int(n)]:
+            indeg[int(m)] -= 1
+            if indeg[int(m)] == 0:
+                ready.append(m)
+        ready.sort(key=lambda n: idx[int(n)])
+    return out
+
+
+def parameter_image(cu, graph_nodes):
+    """Per kernel / memset node of every graph (graph order, then launch order):
+    its blob (8-byte words) and how to rebuild it."""
+    recs = []
+    for gi, nodes in enumerate(graph_nodes):
+        recs += _graph_image(cu, gi, nodes)
+    return recs
+
+
+def _graph_image(cu, gi, nodes):
+    recs = []
+    for pos, n in enumerate(nodes):
+        t = cu.cuGraphNodeGetType(n)[1]
+        if t == cu.CUgraphNodeType.CU_GRAPH_NODE_TYPE_KERNEL:
+            p = cu.cuGraphKernelNodeGetParams(n)[1]
+            layout = _param_layout(cu, p)
+            size = max((o + s for o, s in layout), default=0)
+            blob = bytearray((size + 7) // 8 * 8)
+            kp = ctypes.cast(int(p.kernelParams), ctypes.POINTER(ctypes.c_void_p)) if int(p.kernelParams) else None
+            for i, (o, s_) in enumerate(layout):
+                if kp is None or not kp[i]:
+                    raise RuntimeError("kernel node without kernelParams")
+                blob[o:o + s_] = ctypes.string_at(kp[i], s_)
+            recs.append(dict(kind="kernel", graph=gi, node=n, pos=pos, params=p, layout=layout, blob=bytes(blob)))
+        elif t == cu.CUgraphNodeType.CU_GRAPH_NODE_TYPE_MEMSET:
+            p = cu.cuGraphMemsetNodeGetParams(n)[1]
+            recs.append(dict(kind="memset", graph=gi, node=n, pos=pos, params=p, blob=int(p.dst).to_bytes(8, "little")))
+        else:
+            recs.append(dict(kind="other", graph=gi, node=n, pos=pos, type=t))
+    return recs
+
+
+def trace_arrays(ev, recs):
+    """medusa inputs from the trace and the node list: allocation records with
+    event positions, and each kernel / memset node's launch position."""
+    from workloads import ALLOC_DTYPE
+
+    n_in = {}
+    for r in recs:
+        n_in[r["graph"]] = n_in.get(r["graph"], 0) + 1
+    node_pos = {}
+    t = 1
+    cap, emitted = -1, 0
+
+    def emit_until(c, upto):
+        nonlocal t, emitted
+        while emitted < min(upto, n_in.get(c, 0)):
+            node_pos[(c, emitted)] = t
+            t += 1
+            emitted += 1
+
+    ev_t = []
+    for k in range(ev.shape[0]):
+        kind = int(ev[k, 0])
+        if kind == 3:  # capture `ev[k, 4]` begins
+            cap, emitted = int(ev[k, 4]), 0
+        elif kind == 4:  # ... ends: all its nodes were launched before what follows
+            emit_until(cap, 1 << 62)
+            cap = -1
+        elif cap >= 0 and int(ev[k, 3]) >= 0:
+            emit_until(cap, int(ev[k, 3]))  # nodes captured before this call
+        ev_t.append(t)
+        t += 1
+    allocs = []
+    live = {}
+    for k in range(ev.shape[0]):
+        kind, ptr, size = int(ev[k, 0]), int(ev[k, 1]) & ((1 << 64) - 1), int(ev[k, 2])
+        if kind >= 3:
+            continue
+        if kind == 1:
+            live[ptr] = len(allocs)
+            allocs.append([ptr, size, ev_t[k], T_END])
+        elif ptr in live:
+            allocs[live.pop(ptr)][3] = ev_t[k]
+    arr = np.zeros(len(allocs), ALLOC_DTYPE)
+    for i, (b, s, ta, tf) in enumerate(allocs):
+        arr[i] = (b, s, ta, tf)
+    used = [r for r in recs if r["kind"] in ("kernel", "memset")]
+    words = np.frombuffer(b"".join(r["blob"] for r in used), dtype=np.uint64).copy()
+    off = np.zeros(len(used) + 1, np.uint64)
+    off[1:] = np.cumsum([len(r["blob"]) // 8 for r in used])
+    node_t = np.array([node_pos[(r["graph"], r["pos"])] for r in used], np.uint32)
+    return words, off, node_t, arr, used
+
+
+def online_bases(L, allocs, events):
+    """Replay the (de)allocation sequence in the second arena: new base of every
+    allocation ordinal."""
+    L.ta_free.argtypes = [ctypes.c_void_p, ctypes.c_ssize_t, ctypes.c_int, ctypes.c_void_p]
+    L.ta_select(1)
+    new_base = np.zeros(len(allocs), np.uint64)
+    moved = {}
+    i = 0
+    for k in range(events.shape[0]):
+        ptr = int(events[k, 1]) & ((1 << 64) - 1)
+        if int(events[k, 0]) == 1:
+            new_base[i] = L.ta_raw_malloc(int(events[k, 2]))
+            moved[ptr] = int(new_base[i])
+            i += 1
+        elif ptr in moved:
+            L.ta_free(ctypes.c_void_p(moved.pop(ptr)), 0, 0, None)
+    L.ta_select(0)
+    return new_base
+
+
+def end_to_end(torch, medusa, seed=0):
+    """Capture (process A), materialize the real image on the GPU, replay the
+    allocations in the second arena, copy the live segments over and poison the
+    first arena, restore the image on the GPU, write the restored parameters
+    into a clone of the graph and run it.  Returns the facts the test checks."""
+    from cuda.bindings import driver as cu
+    from cuda.bindings import runtime as rt
+
+    A = capture(torch, seed=seed)
+    recs = parameter_image(cu, A["nodes"])
+    words, off, node_t, allocs, used = trace_arrays(A["events"], recs)
+    dev = torch.device("cuda")
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(dev)
+    aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3)
+    inp = dict(words=t(words, np.int64), node_off=t(off, np.int64), node_t=t(node_t, np.int32),
+               allocs=torch.from_numpy(aa).to(dev))
+    slots = medusa.materialize(**inp)
+    new_base = online_bases(A["L"], allocs, A["events"])
+    live = allocs["t_free"] == T_END
+    first_launch = int(node_t.min()) if node_t.size else 0
+    for i in np.nonzero(live)[0]:
+        if int(allocs["t_alloc"][i]) < first_launch:
+            # allocated before the capture (weights, inputs, workspaces): "the online
+            # process loads the same weights / inputs"
+            _check(rt.cudaMemcpy(int(new_base[i]), int(allocs["base"][i]), int(allocs["size"][i]),
+                                 rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice))
+        else:  # the graph's own pool (activations, the output): recomputed by the graph
+            _check(rt.cudaMemset(int(new_base[i]), 0xEE, int(allocs["size"][i])))
+    for i in np.nonzero(live)[0]:  # nothing may still point into the first arena
+        _check(rt.cudaMemset(int(allocs["base"][i]), 0xFF, int(allocs["size"][i])))
+    torch.cuda.synchronize()
+    dst, _, rep = medusa.restore(inp["words"], slots, t(allocs["base"], np.int64), t(new_base, np.int64),
+                                 t(allocs["size"], np.int64))
+    restored = medusa.to_numpy_u64(dst)
+    report = medusa.report_numpy(rep)
+    # the restored parameters into a clone of every graph (NEXT-2), run them all
+    clones = [_check(cu.cuGraphClone(g)) for g in A["graphs"]]
+    keep = []
+    for k, r in enumerate(used):
+        blob = restored[int(off[k]):int(off[k + 1])].tobytes()
+        node_b = _check(cu.cuGraphNodeFindInClone(r["node"], clones[r["graph"]]))
+        if r["kind"] == "kernel":
+            hb = ctypes.create_string_buffer(blob, max(len(blob), 8))
+            argv = (ctypes.c_void_p * max(len(r["layout"]), 1))()
+            for i, (o, _s) in enumerate(r["layout"]):
+                argv[i] = ctypes.addressof(hb) + o
+            p = r["params"]
+            p.kernelParams = ctypes.addressof(argv)
+            p.extra = 0
+            _check(cu.cuGraphKernelNodeSetParams(node_b, p))
+            keep += [hb, argv]
+        else:
+            p = r["params"]
+            p.dst = int.from_bytes(blob, "little")
+            _check(cu.cuGraphMemsetNodeSetParams(node_b, p))
+    stream = torch.cuda.current_stream().cuda_stream
+    for gb in clones:
+        _check(cu.cuGraphLaunch(_check(cu.cuGraphInstantiate(gb, 0)), stream))
+    torch.cuda.synchronize()
+    # the outputs: each of A's output tensors sits in some traced allocation; same offset in B
+    outs_b = []
+    for out, ref in zip(A["outs"], A["refs"]):
+        op = out.data_ptr()
+        i = int(np.nonzero((allocs["base"] <= op) & (op < allocs["base"] + allocs["size"]))[0][-1])
+        ob = torch.empty_like(ref)
+        _check(rt.cudaMemcpy(ob.data_ptr(), int(new_base[i]) + (op - int(allocs["base"][i])),
+                             ob.numel() * ob.element_size(), rt.cudaMemcpyKind.cudaMemcpyDeviceToHost))
+        outs_b.append(ob)
+    n_kernel = sum(1 for r in recs if r["kind"] == "kernel")
+    names = set()
+    for r in used:
+        if r["kind"] == "kernel":
+            res = cu.cuKernelGetName(r["params"].kern) if int(r["params"].kern) else cu.cuFuncGetName(r["params"].func)
+            if int(res[0]) == 0:
+                names.add(res[1].decode() if isinstance(res[1], bytes) else str(res[1]))
+    n_pre = int(np.sum(allocs["t_alloc"] < first_launch))
+    return dict(words=words, off=off, node_t=node_t, allocs=allocs, slots=slots, new_base=new_base, n_pre=n_pre,
+                restored=restored, report=report, refs=A["refs"], outs_b=outs_b, n_graphs=len(A["graphs"]),
+                n_nodes=len(recs),
+                n_kernel=n_kernel, n_other=sum(1 for r in recs if r["kind"] == "other"), kernel_names=names)
