@@ -42,3 +42,31 @@ def test_real_graph_materialize_restore_replay():
     assert r["n_graphs"] == 4
     for ob, ref in zip(r["outs_b"], r["refs"]):
         assert torch.equal(ob, ref)
+
+
+def test_fresh_process_online_phase(tmp_path):
+    """Offline and online phases in two fresh processes: same loading sequence,
+    replayed allocations, kernel addresses by dlsym + first-layer triggering
+    capture + module enumeration (§5), restore with the kernel-address fill,
+    every graph built from scratch (cuGraphAddKernelNode): outputs bit-identical."""
+    import json
+    import os
+    import subprocess
+    import sys
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    tool = os.path.join(root, "tools", "real_capture_online.py")
+
+    def phase(name):  # each phase in a process of its own (fresh CUDA state)
+        r = subprocess.run([sys.executable, tool, name, str(tmp_path)], capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-2000:]
+        return json.loads(r.stdout.strip().splitlines()[-1])
+
+    off = phase("offline")
+    assert off["names"] > 10 and off["slots"] > 0
+    res = phase("online")
+    assert res["same_loading"]
+    assert res["kernels"]["unresolved"] == 0
+    assert res["report"][0] == 0 and res["report"][5] == 0  # no bad slot, no unresolved kernel
+    assert res["moved_bases"] == res["allocations"]  # a genuinely different address space
+    assert res["outputs_equal"] and all(res["outputs_equal"])

@@ -393,3 +393,289 @@ def end_to_end(torch, medusa, seed=0):
                 restored=restored, report=report, refs=A["refs"], outs_b=outs_b, n_graphs=len(A["graphs"]),
                 n_nodes=len(recs),
                 n_kernel=n_kernel, n_other=sum(1 for r in recs if r["kind"] == "other"), kernel_names=names)
+
+
+# ---------------------------------------------------------------------------
+# Offline / online in separate processes (NEXT-4: kernel addresses in a fresh
+# process come from a triggering capture + module / library enumeration)
+
+_ATTRS = ("CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION", "CU_LAUNCH_ATTRIBUTE_CLUSTER_SCHEDULING_POLICY_PREFERENCE",
+          "CU_LAUNCH_ATTRIBUTE_PRIORITY")
+
+
+def _kernel_name(cu, p):
+    res = cu.cuKernelGetName(p.kern) if int(p.kern) else cu.cuFuncGetName(p.func)
+    if int(res[0]) != 0:
+        return None
+    return res[1].decode() if isinstance(res[1], bytes) else str(res[1])
+
+
+def _node_attrs(cu, node):
+    out = {}
+    for a in _ATTRS:
+        aid = getattr(cu.CUkernelNodeAttrID, a)
+        r = cu.cuGraphKernelNodeGetAttribute(node, aid)
+        if int(r[0]) != 0:
+            continue
+        v = r[1]
+        if a.endswith("CLUSTER_DIMENSION"):
+            out[a] = [int(v.clusterDim.x), int(v.clusterDim.y), int(v.clusterDim.z)]
+        elif a.endswith("POLICY_PREFERENCE"):
+            out[a] = int(v.clusterSchedulingPolicyPreference)
+        else:
+            out[a] = int(v.priority)
+    return out
+
+
+def offline(torch, medusa, out_dir, seed=0):
+    """The offline (materialization-time) process: capture, extract, materialize on
+    the GPU; save everything the online process needs (the indirect index
+    pointer table, kernel-name ids, launch configurations, the trace)."""
+    import json
+    from cuda.bindings import driver as cu
+
+    A = capture(torch, seed=seed)
+    recs = parameter_image(cu, A["nodes"])
+    words, off, node_t, allocs, used = trace_arrays(A["events"], recs)
+    if any(r["kind"] != "kernel" for r in used):
+        raise RuntimeError("offline/online demo handles kernel nodes only")
+    dev = torch.device("cuda")
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(dev)
+    aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3)
+    slots = medusa.materialize(t(words, np.int64), t(off, np.int64), t(node_t, np.int32), torch.from_numpy(aa).to(dev))
+    names, func_id, meta = [], [], []
+    for r in used:
+        nm = _kernel_name(cu, r["params"])
+        if nm not in names:
+            names.append(nm)
+        func_id.append(names.index(nm))
+        p = r["params"]
+        meta.append(dict(graph=r["graph"], grid=[int(p.gridDimX), int(p.gridDimY), int(p.gridDimZ)],
+                         block=[int(p.blockDimX), int(p.blockDimY), int(p.blockDimZ)], smem=int(p.sharedMemBytes),
+                         layout=r["layout"], attrs=_node_attrs(cu, r["node"])))
+    outs = []
+    for o, ref in zip(A["outs"], A["refs"]):
+        op = o.data_ptr()
+        i = int(np.nonzero((allocs["base"] <= op) & (op < allocs["base"] + allocs["size"]))[0][-1])
+        outs.append(dict(alloc=i, offset=op - int(allocs["base"][i]), shape=list(ref.shape)))
+        np.save(os.path.join(out_dir, f"ref{len(outs) - 1}.npy"), ref.numpy())
+    first_capture = int(np.nonzero(A["events"][:, 0] == 3)[0][0])
+    np.savez(os.path.join(out_dir, "image.npz"), words=words, off=off, node_t=node_t, allocs=aa,
+             mask=slots.mask.cpu().numpy(), chunk_base=slots.chunk_base.cpu().numpy(),
+             slot=slots.slot[: slots.n_slots].cpu().numpy(), func_id=np.array(func_id, np.uint32),
+             events=A["events"])
+    json.dump(dict(names=names, meta=meta, outs=outs, n_slots=slots.n_slots, graphs=len(A["graphs"]),
+                   load_events=first_capture, seed=seed), open(os.path.join(out_dir, "meta.json"), "w"))
+    return dict(nodes=len(used), names=len(names), slots=slots.n_slots)
+
+
+def _dlsym_kernels(torch, names):
+    """dlopen the library, dlsym the kernel's (host stub) symbol, then
+    cudaGetFuncBySymbol.  Returns {name: CUfunction}."""
+    # the CUDA runtime instance PyTorch registered its kernels with
+    cudart = None
+    for soname in ("libcudart.so.12", "libcudart.so"):
+        try:
+            cudart = ctypes.CDLL(soname, mode=os.RTLD_NOLOAD | os.RTLD_GLOBAL)
+            break
+        except OSError:
+            continue
+    if cudart is None:
+        return {}
+    cudart.cudaGetFuncBySymbol.argtypes = [ctypes.POINTER(ctypes.c_void_p), ctypes.c_void_p]
+    cudart.cudaGetFuncBySymbol.restype = ctypes.c_int
+
+    libdir = os.path.join(os.path.dirname(torch.__file__), "lib")
+    libs = []
+    for f in ("libtorch_cuda.so", "libc10_cuda.so"):
+        try:
+            libs.append(ctypes.CDLL(os.path.join(libdir, f), mode=os.RTLD_NOLOAD | os.RTLD_GLOBAL))
+        except OSError:
+            pass
+    out = {}
+    for nm in names:
+        for lib in libs:
+            try:
+                stub = ctypes.cast(getattr(lib, nm), ctypes.c_void_p).value
+            except AttributeError:
+                continue
+            fn = ctypes.c_void_p(0)
+            if cudart.cudaGetFuncBySymbol(ctypes.byref(fn), ctypes.c_void_p(stub)) == 0 and fn.value:
+                out[nm] = int(fn.value)
+                break
+    return out
+
+
+def _resolve_kernels(torch, cu, model, ids, mask, names):
+    """Kernel addresses in this process (§5): dlsym + cudaGetFuncBySymbol first;
+    for the rest, capture the model's first layer (the triggering kernels,
+    P:254-259), take the addresses of its nodes, and enumerate the modules /
+    libraries those kernels came from, matching names.
+    Returns ({name: CUfunction}, stats)."""
+    found = _dlsym_kernels(torch, names)
+    n_dlsym = len(found)
+    g = torch.cuda.CUDAGraph(keep_graph=True)
+    with torch.no_grad(), torch.cuda.graph(g):  # default pool: not part of the replayed trace
+        model.layers[0](model.emb(ids[:1]), mask)  # the first layer
+    graph = cu.CUgraph(g.raw_cuda_graph())
+    n = int(cu.cuGraphGetNodes(graph, 0)[2])
+    modules, libraries = {}, {}
+    n_trig = 0
+    for node in cu.cuGraphGetNodes(graph, n)[1]:
+        if cu.cuGraphNodeGetType(node)[1] != cu.CUgraphNodeType.CU_GRAPH_NODE_TYPE_KERNEL:
+            continue
+        p = cu.cuGraphKernelNodeGetParams(node)[1]
+        nm = _kernel_name(cu, p)
+        if int(p.kern):
+            fn = _check(cu.cuKernelGetFunction(p.kern))
+            lib = _check(cu.cuKernelGetLibrary(p.kern))
+            libraries[int(lib)] = lib
+        else:
+            fn = p.func
+            mod = _check(cu.cuFuncGetModule(fn))
+            modules[int(mod)] = mod
+        if nm in names and nm not in found:
+            found[nm] = int(fn)
+            n_trig += 1
+    n_enum = 0
+    for mod in modules.values():
+        cnt = _check(cu.cuModuleGetFunctionCount(mod))
+        for fn in _check(cu.cuModuleEnumerateFunctions(cnt, mod)):
+            r = cu.cuFuncGetName(fn)
+            nm = (r[1].decode() if isinstance(r[1], bytes) else str(r[1])) if int(r[0]) == 0 else None
+            if nm in names and nm not in found:
+                found[nm] = int(fn)
+                n_enum += 1
+    for lib in libraries.values():
+        cnt = _check(cu.cuLibraryGetKernelCount(lib))
+        for k in _check(cu.cuLibraryEnumerateKernels(cnt, lib)):
+            r = cu.cuKernelGetName(k)
+            nm = (r[1].decode() if isinstance(r[1], bytes) else str(r[1])) if int(r[0]) == 0 else None
+            if nm in names and nm not in found:
+                found[nm] = int(_check(cu.cuKernelGetFunction(k)))
+                n_enum += 1
+    stats = dict(dlsym=n_dlsym, triggering=n_trig, enumerated=n_enum,
+                 unresolved=sum(1 for nm in names if nm not in found))
+    return found, stats
+
+
+def online(torch, medusa, in_dir, arena_bytes=1 << 30):
+    """The online process (a fresh one): load the same model into the traced
+    pool, replay the rest of the offline allocation sequence, resolve kernel
+    addresses, restore (relocate + validate + kernel-address fill), build every
+    graph from scratch and run it.  Returns the facts to check."""
+    import json
+    from cuda.bindings import driver as cu
+    from cuda.bindings import runtime as rt
+
+    meta = json.load(open(os.path.join(in_dir, "meta.json")))
+    z = np.load(os.path.join(in_dir, "image.npz"))
+    ev_a = z["events"]
+    L = _lib()
+    if L.ta_init(arena_bytes) != 0:
+        raise RuntimeError("tracing allocator: cudaMalloc of the arenas failed")
+    alloc = torch.cuda.memory.CUDAPluggableAllocator(build(), "ta_malloc", "ta_free")
+    L.ta_select(0)
+    L.ta_clear()
+    L.ta_log(1)
+    pool = torch.cuda.MemPool(alloc.allocator())
+    torch.manual_seed(meta["seed"])
+    batches = (8, 4, 2, 1)
+    with torch.cuda.use_mem_pool(pool):  # the same loading sequence as offline
+        model = tiny_decoder(torch).cuda().eval()
+        seq = meta["outs"][0]["shape"][1]
+        ids = torch.randint(0, 512, (max(batches), seq), device="cuda")
+        mask = torch.full((seq, seq), float("-inf"), device="cuda").triu(1)
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s), torch.no_grad():
+            for b in batches:
+                model(ids[:b], mask)
+        torch.cuda.current_stream().wait_stream(s)
+        torch.cuda.synchronize()
+    L.ta_log(0)
+    n_ev = L.ta_events(None, 0)
+    buf = (ctypes.c_int64 * (5 * n_ev))()
+    L.ta_events(buf, n_ev)
+    ev_b = np.frombuffer(buf, dtype=np.int64).reshape(n_ev, 5)
+    nl = meta["load_events"]
+    same_loading = n_ev == nl and bool(np.array_equal(ev_b[:, [0, 2]], ev_a[:nl, [0, 2]]))
+    # new base of every allocation ordinal: loading phase as it happened here, the
+    # rest replayed (P:216)
+    L.ta_free.argtypes = [ctypes.c_void_p, ctypes.c_ssize_t, ctypes.c_int, ctypes.c_void_p]
+    new_base = []
+    moved = {}
+    for k in range(ev_a.shape[0]):
+        kind, ptr = int(ev_a[k, 0]), int(ev_a[k, 1]) & ((1 << 64) - 1)
+        if kind == 1:
+            nb = int(ev_b[k, 1]) & ((1 << 64) - 1) if k < nl else L.ta_raw_malloc(int(ev_a[k, 2]))
+            new_base.append(nb)
+            moved[ptr] = nb
+        elif kind == 2 and k >= nl and ptr in moved:
+            L.ta_free(ctypes.c_void_p(moved.pop(ptr)), 0, 0, None)
+    new_base = np.array(new_base, np.uint64)
+    allocs = z["allocs"].view(np.uint64).reshape(-1, 3)
+    # kernel addresses
+    found, kstats = _resolve_kernels(torch, cu, model, ids, mask, meta["names"])
+    table = np.array([found.get(nm, 0) for nm in meta["names"]], np.uint64)
+    dev = torch.device("cuda")
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(dev)
+    slots = medusa.Slots(t(z["mask"], np.int32), t(z["chunk_base"], np.int32), t(z["slot"], np.int64),
+                         int(meta["n_slots"]))
+    medusa.kernel_table_set(t(table, np.int64))
+    dst, fout, rep = medusa.restore(t(z["words"], np.int64), slots, t(allocs[:, 0], np.int64),
+                                    t(new_base, np.int64), t(allocs[:, 1], np.int64), t(z["func_id"], np.int32))
+    torch.cuda.synchronize()
+    restored = medusa.to_numpy_u64(dst)
+    func_out = medusa.to_numpy_u64(fout)
+    report = medusa.report_numpy(rep)
+    if kstats["unresolved"] or int(report[5]):
+        missing = [nm for nm in meta["names"] if nm not in found]
+        return dict(same_loading=same_loading, kernels=kstats, report=[int(x) for x in report],
+                    unresolved_names=missing[:5], outputs_equal=[])
+    # every graph built from scratch: nodes in launch order, one chain
+    off = z["off"]
+    keep, graphs = [], [_check(cu.cuGraphCreate(0)) for _ in range(meta["graphs"])]
+    prev = [None] * meta["graphs"]
+    for j, m in enumerate(meta["meta"]):
+        blob = restored[int(off[j]):int(off[j + 1])].tobytes()
+        hb = ctypes.create_string_buffer(blob, max(len(blob), 8))
+        argv = (ctypes.c_void_p * max(len(m["layout"]), 1))()
+        for i, (o, _s) in enumerate(m["layout"]):
+            argv[i] = ctypes.addressof(hb) + o
+        keep += [hb, argv]
+        p = cu.CUDA_KERNEL_NODE_PARAMS()
+        p.func = cu.CUfunction(int(func_out[j]))
+        p.gridDimX, p.gridDimY, p.gridDimZ = m["grid"]
+        p.blockDimX, p.blockDimY, p.blockDimZ = m["block"]
+        p.sharedMemBytes = m["smem"]
+        p.kernelParams = ctypes.addressof(argv)
+        p.extra = 0
+        gi = m["graph"]
+        deps = [prev[gi]] if prev[gi] is not None else []
+        node = _check(cu.cuGraphAddKernelNode(graphs[gi], deps, len(deps), p))
+        for a, v in m["attrs"].items():
+            val = cu.CUkernelNodeAttrValue()
+            if a.endswith("CLUSTER_DIMENSION"):
+                val.clusterDim.x, val.clusterDim.y, val.clusterDim.z = v
+            elif a.endswith("POLICY_PREFERENCE"):
+                val.clusterSchedulingPolicyPreference = v
+            else:
+                val.priority = v
+            _check(cu.cuGraphKernelNodeSetAttribute(node, getattr(cu.CUkernelNodeAttrID, a), val))
+        prev[gi] = node
+    stream = torch.cuda.current_stream().cuda_stream
+    for g in graphs:
+        _check(cu.cuGraphLaunch(_check(cu.cuGraphInstantiate(g, 0)), stream))
+    torch.cuda.synchronize()
+    equal = []
+    for k, o in enumerate(meta["outs"]):
+        ref = np.load(os.path.join(in_dir, f"ref{k}.npy"))
+        ob = np.empty_like(ref)
+        _check(rt.cudaMemcpy(ob.ctypes.data, int(new_base[o["alloc"]]) + o["offset"], ob.nbytes,
+                             rt.cudaMemcpyKind.cudaMemcpyDeviceToHost))
+        equal.append(bool(np.array_equal(ob, ref)))
+    moved_bases = int(np.sum(new_base != allocs[:, 0]))
+    return dict(same_loading=same_loading, kernels=kstats, report=[int(x) for x in report], outputs_equal=equal,
+                nodes=len(meta["meta"]), allocations=int(len(new_base)), moved_bases=moved_bases,
+                slots=int(meta["n_slots"]))
