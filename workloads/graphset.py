@@ -149,6 +149,7 @@ class GraphSet:
     node_perm: np.ndarray  # bool[N] kernel owns permanent buffers
     alloc_kind: np.ndarray  # u8[n_alloc]: 0 weight 1 kv 2 static 3 profiling 4 warmup 5 capture-temp 6 permanent
     models: list
+    capture_t: np.ndarray = None  # u32[n_graphs, 2]: event positions (begin, end) of each graph's capture
 
     @property
     def n_words(self):
@@ -178,6 +179,7 @@ class _Builder:
         self.func_names = {}
         self.func_kind = []
         self.models = []
+        self.captures = []
         self._const_cache = {}
         self.rate_scale = 1.0  # the toy set uses 4x rates so every category shows up
 
@@ -220,6 +222,15 @@ class _Builder:
         self.recent_freed.append(aid)
         if len(self.recent_freed) > 512:
             del self.recent_freed[:256]
+
+    def begin_capture(self):
+        """cudaStreamBeginCapture: an event of its own in the one total order."""
+        self.t += 1
+        self._capture_begin = self.t
+
+    def end_capture(self):
+        self.t += 1
+        self.captures.append((self._capture_begin, self.t))
 
     # -- nodes ---------------------------------------------------------------
     def func(self, key, kind):
@@ -391,6 +402,7 @@ class _Builder:
             node_perm=np.asarray(self.n_perm, dtype=bool),
             alloc_kind=np.asarray(self.a_kind, dtype=np.uint8),
             models=list(self.models),
+            capture_t=np.asarray(self.captures, dtype=np.uint32).reshape(-1, 2),
         )
 
 
@@ -451,7 +463,9 @@ def _run_model(B: _Builder, m_index: int, cfg: ModelCfg):
     # 5. capture, largest batch size first, one graph at a time.
     for b in sorted(BATCH_SIZES, reverse=True):
         _forward(B, ctx, b=b, k=kmap[b], pool="default", kind=AK_WARMUP, record=False)
+        B.begin_capture()
         _forward(B, ctx, b=b, k=kmap[b], pool="graph", kind=AK_CAPTURE, record=True)
+        B.end_capture()
     B.end_model()
 
 
@@ -546,6 +560,7 @@ def _run_toy(B: _Builder):
     KV = [B.malloc(8 * MiB, AK_KV) for _ in range(2)]
     S = [B.malloc(s, AK_STATIC) for s in (2048, 2048, 2048, 1 << 19, 1024, 4 * MiB + 1024)]
     # 23 allocations so far; the graph adds E, F, 35 temps and 4 permanent buffers = 64.
+    B.begin_capture()
     E = B.malloc(H * 2, AK_CAPTURE, "graph")
     B.node("embed", [(E, 0), (S[0], 0), (W[0], 0)], ("toy", "embed"), DLSYM, 1)
     temps = [E]
@@ -574,6 +589,12 @@ def _run_toy(B: _Builder):
                 B.free(alive[0])
     F = B.malloc(H * 2, AK_CAPTURE, "graph")
     B.node("rmsnorm", [(F, 0), (temps[-1], 0), (W[1], 0)], ("toy", "rmsnorm"), DLSYM, 1)
+    B.end_capture()
+    # the graph's temporaries are released after the capture; its
+    # permanent buffers stay
+    for a in temps + [F]:
+        if B.a_tf[a] == T_NEVER:
+            B.free(a)
     B.end_model()
     assert len(B.a_base) == 64, len(B.a_base)
 
@@ -619,11 +640,12 @@ def replicate(gs: GraphSet, R: int, va_stride: int = 1 << 44) -> GraphSet:
     in time, with allocation ordinals and kernel-name ids offset by r copies."""
     assert R >= 1
     span = int(max(int(gs.node_t.max(initial=0)), int(gs.allocs["t_alloc"].max(initial=0)),
+                   int(gs.capture_t.max(initial=0)),
                    int(np.where(gs.allocs["t_free"] == T_NEVER, 0, gs.allocs["t_free"]).max(initial=0)))) + 1
     assert span * R < T_NEVER
     is_addr = gs.tags != TAG_CONST
     words, tags, tid, toff, offs, nts, fids = [], [], [], [], [np.zeros(1, np.uint64)], [], []
-    allocs, new_base = [], []
+    allocs, new_base, caps = [], [], []
     K = gs.table.size
     for r in range(R):
         d = np.uint64(va_stride * r)
@@ -643,10 +665,12 @@ def replicate(gs: GraphSet, R: int, va_stride: int = 1 << 44) -> GraphSet:
         a["t_free"] = np.where(never, T_NEVER, a["t_free"] + np.uint32(r * span))
         allocs.append(a)
         new_base.append(gs.new_base + d)
+        caps.append(gs.capture_t + np.uint32(r * span))
     return GraphSet(
         name=f"{gs.name}x{R}", words=np.concatenate(words), node_word_off=np.concatenate(offs),
         node_t=np.concatenate(nts), func_id=np.concatenate(fids), allocs=np.concatenate(allocs),
         new_base=np.concatenate(new_base), new_size=np.tile(gs.new_size, R), table=np.tile(gs.table, R),
         func_kind=np.tile(gs.func_kind, R), tags=np.concatenate(tags), truth_id=np.concatenate(tid),
         truth_off=np.concatenate(toff), node_model=np.tile(gs.node_model, R), node_bs=np.tile(gs.node_bs, R),
-        node_perm=np.tile(gs.node_perm, R), alloc_kind=np.tile(gs.alloc_kind, R), models=gs.models * R)
+        node_perm=np.tile(gs.node_perm, R), alloc_kind=np.tile(gs.alloc_kind, R), models=gs.models * R,
+        capture_t=np.concatenate(caps))
