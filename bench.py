@@ -170,6 +170,77 @@ def run_reference(args):
     }), flush=True)
 
 
+def bench_buffers(medusa, gs, inp, slots, dev, stream, scrub, steps, peak):
+    """medusa_buffers_plan (offline, synchronous) and medusa_buffers_save /
+    medusa_buffers_restore (offline dump / online copy-back) on the workload.  The
+    synthetic trace's addresses are not device memory, so the permanent buffers get
+    real ones: an arena in ordinal order (old) and one in shuffled order (new)."""
+    import torch
+    ev = lambda: torch.cuda.Event(enable_timing=True)
+    plan = medusa.buffers_plan(inp["allocs"], inp["capture_t"], slots.slot, slots.n_slots)
+    torch.cuda.synchronize(dev)
+    perm = plan.perm.cpu().numpy().view(np.uint32)
+    sizes = gs.allocs["size"][perm].astype(np.int64)
+    old_arena = torch.randint(0, 256, (max(int(sizes.sum()), 16),), dtype=torch.uint8, device=dev)
+    new_arena = torch.zeros_like(old_arena)
+    pos = np.concatenate([[0], np.cumsum(sizes)[:-1]]).astype(np.int64)
+    base = np.zeros(gs.n_alloc, np.uint64)
+    nb = np.zeros(gs.n_alloc, np.uint64)
+    base[perm] = old_arena.data_ptr() + pos
+    nb[perm[np.random.default_rng(0).permutation(perm.size)]] = new_arena.data_ptr() + pos
+    d_base = torch.from_numpy(base.view(np.int64)).to(dev)
+    d_nb = torch.from_numpy(nb.view(np.int64)).to(dev)
+    blob = torch.empty(max(plan.blob_bytes, 16), dtype=torch.uint8, device=dev)
+    rep = torch.empty(2, dtype=torch.int64, device=dev)
+    for _ in range(3):
+        medusa.buffers_plan(inp["allocs"], inp["capture_t"], slots.slot, slots.n_slots)
+        medusa.buffers_save(plan, d_base, blob=blob, report=rep)
+        medusa.buffers_restore(plan, blob, d_nb, inp["new_size"], report=rep)
+    torch.cuda.synchronize(dev)
+    assert torch.equal(blob[:plan.blob_bytes], old_arena[:plan.blob_bytes])
+    assert int(rep[0].item()) == 0
+
+    def t(fn):
+        out = []
+        for k in range(steps):
+            scrub.fill_(k)
+            a, b = ev(), ev()
+            a.record(stream)
+            fn()
+            b.record(stream)
+            out.append((a, b))
+        torch.cuda.synchronize(dev)
+        return statistics.median(a.elapsed_time(b) for a, b in out)
+
+    plan_ms = t(lambda: medusa.buffers_plan(inp["allocs"], inp["capture_t"], slots.slot, slots.n_slots))
+    save_ms = t(lambda: medusa.buffers_save(plan, d_base, blob=blob, report=rep))
+    rest_ms = t(lambda: medusa.buffers_restore(plan, blob, d_nb, inp["new_size"], report=rep))
+    torch.cuda.synchronize(dev)
+    ok = int(rep[0].item()) == 0
+    # kernel-only durations (libmedusa's per-launch events), L2 scrubbed before each call
+    medusa.timing_enable(True)
+    for k in range(steps):
+        scrub.fill_(k)
+        medusa.buffers_save(plan, d_base, blob=blob, report=rep)
+        scrub.fill_(k)
+        medusa.buffers_restore(plan, blob, d_nb, inp["new_size"], report=rep)
+    kt = {}
+    for name, ms in medusa.timing_read(1 << 16):
+        kt.setdefault(name, []).append(ms)
+    medusa.timing_enable(False)
+    kernel_us = {n: 1e3 * statistics.median(v) for n, v in kt.items()}
+    moved = 2 * plan.blob_bytes + 12 * plan.n_perm + 8 * plan.n_perm  # bytes + perm/off + base(+size)
+    return {"n_perm": plan.n_perm, "perm_kernel_frac": float(gs.node_perm.mean()), "blob_bytes": plan.blob_bytes,
+            "classes": {k: int((plan.cls == v).sum().item()) for k, v in
+                        (("unused", 0), ("param", 1), ("temp", 2), ("perm", 3))},
+            "plan_ms": plan_ms, "save_us": save_ms * 1e3, "restore_us": rest_ms * 1e3,
+            "restore_GB/s": moved / (rest_ms / 1e3) / 1e9, "restore_frac_of_peak": moved / (rest_ms / 1e3) / 1e9 / peak,
+            "restore_ok": ok, "kernel_us": kernel_us,
+            "restore_kernel_GB/s": moved / (kernel_us["buf_restore"] / 1e6) / 1e9,
+            "note": "median of K calls, L2 scrubbed before each; medusa_buffers_restore = the online copy-back "
+                    "(P:220-224), bytes = 2 x blob + 20 B per buffer"}
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -346,6 +417,10 @@ def run_ours(args):
         del binp, bslots, bdst, bfout, big
         torch.cuda.empty_cache()
 
+    # ---- copy-free buffer contents restoration (§4.3): plan
+    #      from this step's table, the permanent buffers given real addresses ----
+    buf = bench_buffers(medusa, gs, inp, slots, dev, stream, scrub, args.steps, peak) if args.buffers else None
+
     # ---- end to end: pinned host buffers -> H2D -> whole path -> D2H of results ----
     h = medusa.host_arrays(gs)
     pinned = {k: torch.from_numpy(v).pin_memory() for k, v in h.items()}
@@ -412,6 +487,7 @@ def run_ours(args):
             "materialize_ms": mat_s * 1e3,
             "kernels": kernels,
             "sustained_relocate": sus,
+            "buffers": buf,
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
             "gpu_launches": len(launches),
@@ -438,6 +514,7 @@ def main():
     ap.add_argument("--sustained", type=int, default=32, help="replicas in the sustained-relocate call (0: skip)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-buffers", dest="buffers", action="store_false")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)

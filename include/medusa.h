@@ -225,6 +225,80 @@ medusa_status medusa_restore(const uint64_t *d_src_words, uint64_t *d_dst_words,
                              const uint32_t *d_func_id, uint64_t *d_func_out, uint32_t n_nodes,
                              medusa_report *d_report, cudaStream_t stream);
 
+/* ---- copy-free buffer contents restoration (§4.3) ------------
+ *
+ * Besides the pointers, the contents of the buffers the graph nodes point to
+ * must be right.  Most need no saving: model-parameter buffers are
+ * "allocated before the CUDA graphs capturing" and temporary buffers
+ * are allocated during a capture and "deallocated after capturing".
+ * Only the permanent ones -- allocated during a capture, never freed, "used
+ * across different launches of CUDA graphs" (two 4-byte buffers for
+ * 9.0% of the kernels) -- are dumped offline and copied back online.
+ *
+ * Class of allocation i (d_class[i]):                                         */
+#define MEDUSA_BUF_UNUSED 0u /* no slot of the table refers to it (not a graph parameter) */
+#define MEDUSA_BUF_PARAM 1u  /* t_alloc inside no capture interval: "allocated before the CUDA
+                                graphs capturing" -- contents not saved */
+#define MEDUSA_BUF_TEMP 2u   /* allocated during a capture, freed (t_free != MEDUSA_T_END):
+                                temporary -- contents discarded */
+#define MEDUSA_BUF_PERM 3u   /* allocated during a capture, never freed: permanent
+                                -- contents saved and restored */
+
+/* Save / restore report (device memory, 16 bytes): segments not copied and the
+ * least such segment index k ("none" = UINT64_MAX). */
+typedef struct {
+    uint64_t n_bad, first_bad;
+} medusa_buf_report;
+
+/* medusa_buffers_plan -- offline: classify every allocation and lay out the blob.
+ *
+ * Inputs (device): d_alloc[n_alloc] the trace given to medusa_materialize;
+ *   d_capture_t[2*n_capture] the event positions (begin, end) of every graph
+ *   capture, in the same total order as the trace (cudaStreamBeginCapture /
+ *   EndCapture); intervals must satisfy begin < end and end_k <= begin_{k+1}
+ *   (graphs are captured one at a time), else MEDUSA_ERR_INVALID_ARG.
+ *   Allocation i is made during capture k iff begin_k < t_alloc_i < end_k.
+ *   d_slot[n_slots]: the materialized slot records; records whose allocation
+ *   index is >= n_alloc are ignored.
+ * Outputs (device, caller-owned): d_class u8[n_alloc] (MEDUSA_BUF_*);
+ *   d_perm u32[perm_capacity]: the PERM allocation indices, increasing;
+ *   d_perm_off u64[perm_capacity + 1]: segment k of the blob is
+ *   [d_perm_off[k], d_perm_off[k+1]) and holds the d_alloc[].size bytes of
+ *   allocation d_perm[k]; d_perm_off[n_perm] = blob size.
+ *   *h_n_perm, *h_blob_bytes (host).  perm_capacity = n_alloc always suffices.
+ * Errors: INVALID_ARG (null / misaligned pointers, bad capture intervals),
+ *   CAPACITY (n_perm > perm_capacity: d_class complete, *h_n_perm and
+ *   *h_blob_bytes hold the sizes needed, the lists are truncated).
+ * Synchronizes `stream` (reads the counts back).                             */
+medusa_status medusa_buffers_plan(const medusa_alloc *d_alloc, uint32_t n_alloc,
+                                  const uint32_t *d_capture_t, uint32_t n_capture,
+                                  const uint64_t *d_slot, uint64_t n_slots,
+                                  uint8_t *d_class, uint32_t *d_perm, uint64_t *d_perm_off,
+                                  uint32_t perm_capacity, uint32_t *h_n_perm, uint64_t *h_blob_bytes,
+                                  cudaStream_t stream);
+
+/* medusa_buffers_save -- offline: d_blob[d_perm_off[k] ...] = the bytes of
+ * allocation d_perm[k] at address d_base[d_perm[k]] (device memory of this
+ * process, normally the trace's bases).  d_perm / d_perm_off / n_perm as
+ * produced by medusa_buffers_plan; d_blob: u8[d_perm_off[n_perm]], 16-byte
+ * aligned, not overlapping any saved buffer.  Segments with d_perm[k] >=
+ * n_alloc are not copied and counted in *d_report.  Fully asynchronous on
+ * `stream`; capturable.                                                      */
+medusa_status medusa_buffers_save(const uint32_t *d_perm, const uint64_t *d_perm_off, uint32_t n_perm,
+                                  const uint64_t *d_base, uint32_t n_alloc, uint8_t *d_blob,
+                                  medusa_buf_report *d_report, cudaStream_t stream);
+
+/* medusa_buffers_restore -- online: copy segment k of d_blob to
+ * d_new_base[d_perm[k]], the address the replayed allocation returned (P:176,
+ * P:186), unless d_perm[k] >= n_alloc (the replay made fewer allocations) or
+ * the segment is longer than d_new_size[d_perm[k]]; those segments are not
+ * copied and are counted in *d_report (DESIGN.md R-B4).  No other byte is
+ * written.  Targets must not overlap the blob or each other.  Fully
+ * asynchronous on `stream`; capturable.                                      */
+medusa_status medusa_buffers_restore(const uint8_t *d_blob, const uint32_t *d_perm, const uint64_t *d_perm_off,
+                                     uint32_t n_perm, const uint64_t *d_new_base, const uint64_t *d_new_size,
+                                     uint32_t n_alloc, medusa_buf_report *d_report, cudaStream_t stream);
+
 /* cudaError_t value behind the last MEDUSA_ERR_CUDA returned on this thread. */
 int medusa_last_cuda_error(void);
 

@@ -61,6 +61,13 @@ def lib():
         L.medusa_kernel_table_set.restype = I
         L.medusa_restore.argtypes = [P, P, U64, ctypes.POINTER(_Slots), U64, P, P, P, U32, P, P, U32, P, P]
         L.medusa_restore.restype = I
+        L.medusa_buffers_plan.argtypes = [P, U32, P, U32, P, U64, P, P, P, U32, ctypes.POINTER(U32),
+                                          ctypes.POINTER(U64), P]
+        L.medusa_buffers_plan.restype = I
+        L.medusa_buffers_save.argtypes = [P, P, U32, P, U32, P, P, P]
+        L.medusa_buffers_save.restype = I
+        L.medusa_buffers_restore.argtypes = [P, P, P, U32, P, P, U32, P, P]
+        L.medusa_buffers_restore.restype = I
         L.medusa_last_cuda_error.argtypes = []
         L.medusa_last_cuda_error.restype = I
         L.medusa_status_string.argtypes = [I]
@@ -178,6 +185,72 @@ def restore(src, slots, old_base, new_base, new_size, func_id=None, dst=None, fu
     return dst, func_out, report
 
 
+BUF_UNUSED, BUF_PARAM, BUF_TEMP, BUF_PERM = 0, 1, 2, 3
+
+
+class BufferPlan:
+    """Output of medusa_buffers_plan (device tensors): class per allocation, the
+    permanent allocations and the blob layout."""
+
+    def __init__(self, cls, perm, perm_off, n_perm, blob_bytes):
+        self.cls = cls  # uint8[n_alloc]
+        self.perm = perm  # int32[n_perm] allocation indices
+        self.perm_off = perm_off  # int64[n_perm + 1] blob offsets
+        self.n_perm = int(n_perm)
+        self.blob_bytes = int(blob_bytes)
+
+
+def buffers_plan(allocs, capture_t, slot, n_slots, stream=None, capacity=None):
+    """medusa_buffers_plan.  allocs int64[n_alloc, 3] (medusa_alloc records), capture_t
+    int32[n_capture, 2] (begin, end) event positions, slot int64[>= n_slots] (the
+    materialized records, e.g. Slots.slot) -> BufferPlan.  capacity defaults to
+    n_alloc (always enough)."""
+    dev = allocs.device
+    n_alloc = allocs.shape[0] if allocs.dim() else 0
+    cap = n_alloc if capacity is None else int(capacity)
+    cls = torch.empty(max(n_alloc, 1), dtype=torch.uint8, device=dev)
+    perm = torch.empty(max(cap, 1), dtype=torch.int32, device=dev)
+    perm_off = torch.empty(cap + 1, dtype=torch.int64, device=dev)
+    n_perm, nbytes = ctypes.c_uint32(0), ctypes.c_uint64(0)
+    st = lib().medusa_buffers_plan(_ptr(allocs), n_alloc, _ptr(capture_t), capture_t.numel() // 2,
+                                   _ptr(slot), int(n_slots), _ptr(cls), _ptr(perm), _ptr(perm_off), cap,
+                                   ctypes.byref(n_perm), ctypes.byref(nbytes), _stream(stream))
+    if st != OK:
+        e = MedusaError(st, "medusa_buffers_plan")
+        e.n_perm, e.blob_bytes = int(n_perm.value), int(nbytes.value)
+        raise e
+    n = int(n_perm.value)
+    return BufferPlan(cls[:n_alloc], perm[:n], perm_off[:n + 1], n, nbytes.value)
+
+
+def buffers_save(plan, base, blob=None, report=None, stream=None):
+    """medusa_buffers_save: blob uint8[plan.blob_bytes] <- the PERM buffers' bytes at
+    base[i] (int64[n_alloc] device addresses) -> (blob, report int64[2])."""
+    dev = base.device
+    if blob is None:
+        blob = torch.empty(max(plan.blob_bytes, 16), dtype=torch.uint8, device=dev)
+    if report is None:
+        report = torch.empty(2, dtype=torch.int64, device=dev)
+    st = lib().medusa_buffers_save(_ptr(plan.perm), _ptr(plan.perm_off), plan.n_perm, _ptr(base), base.numel(),
+                                   _ptr(blob), _ptr(report), _stream(stream))
+    if st != OK:
+        raise MedusaError(st, "medusa_buffers_save")
+    return blob, report
+
+
+def buffers_restore(plan, blob, new_base, new_size, report=None, stream=None):
+    """medusa_buffers_restore: copy each saved segment to its replayed allocation
+    -> report int64[2] (n_bad, first_bad)."""
+    if report is None:
+        report = torch.empty(2, dtype=torch.int64, device=blob.device)
+    st = lib().medusa_buffers_restore(_ptr(blob), _ptr(plan.perm), _ptr(plan.perm_off), plan.n_perm,
+                                      _ptr(new_base), _ptr(new_size), new_base.numel(), _ptr(report),
+                                      _stream(stream))
+    if st != OK:
+        raise MedusaError(st, "medusa_buffers_restore")
+    return report
+
+
 def timing_enable(on=True):
     lib().medusa_timing_enable(1 if on else 0)
 
@@ -208,6 +281,7 @@ def host_arrays(gs):
         new_size=np.ascontiguousarray(gs.new_size).view(np.int64),
         func_id=np.ascontiguousarray(gs.func_id).view(np.int32),
         table=np.ascontiguousarray(gs.table).view(np.int64),
+        capture_t=np.ascontiguousarray(gs.capture_t, dtype=np.uint32).view(np.int32).reshape(-1, 2),
     )
 
 

@@ -207,4 +207,53 @@ medusa_status medusa_restore(const uint64_t* d_src_words, uint64_t* d_dst_words,
     return MEDUSA_OK;
 }
 
+medusa_status medusa_buffers_plan(const medusa_alloc* d_alloc, uint32_t n_alloc, const uint32_t* d_capture_t,
+                                  uint32_t n_capture, const uint64_t* d_slot, uint64_t n_slots, uint8_t* d_class,
+                                  uint32_t* d_perm, uint64_t* d_perm_off, uint32_t perm_capacity,
+                                  uint32_t* h_n_perm, uint64_t* h_blob_bytes, cudaStream_t stream) {
+    if (h_n_perm) *h_n_perm = 0;
+    if (h_blob_bytes) *h_blob_bytes = 0;
+    if (!h_n_perm || !h_blob_bytes || !d_perm_off || !aligned8(d_perm_off)) return MEDUSA_ERR_INVALID_ARG;
+    if (n_alloc > 0 && (!d_alloc || !d_class || !aligned8(d_alloc))) return MEDUSA_ERR_INVALID_ARG;
+    if (n_capture > 0 && (!d_capture_t || (reinterpret_cast<uintptr_t>(d_capture_t) & 3))) return MEDUSA_ERR_INVALID_ARG;
+    if (n_slots > 0 && (!d_slot || !aligned8(d_slot))) return MEDUSA_ERR_INVALID_ARG;
+    if (perm_capacity > 0 && (!d_perm || (reinterpret_cast<uintptr_t>(d_perm) & 3))) return MEDUSA_ERR_INVALID_ARG;
+    cudaError_t ce = cudaSuccess;
+    medusa_status st = run_buffers_plan(d_alloc, n_alloc, d_capture_t, n_capture, d_slot, n_slots, d_class, d_perm,
+                                        d_perm_off, perm_capacity, h_n_perm, h_blob_bytes, stream, &ce);
+    if (st == MEDUSA_ERR_CUDA) g_last_cuda_error = (int)ce;
+    return st;
+}
+
+static medusa_status buffers_copy_args(const uint32_t* d_perm, const uint64_t* d_perm_off, uint32_t n_perm,
+                                       const void* d_blob, medusa_buf_report* d_report) {
+    if (!d_report || !aligned8(d_report) || !d_perm_off || !aligned8(d_perm_off)) return MEDUSA_ERR_INVALID_ARG;
+    if (n_perm > 0 && (!d_perm || (reinterpret_cast<uintptr_t>(d_perm) & 3))) return MEDUSA_ERR_INVALID_ARG;
+    if (n_perm > 0 && (!d_blob || (reinterpret_cast<uintptr_t>(d_blob) & 15))) return MEDUSA_ERR_INVALID_ARG;
+    return MEDUSA_OK;
+}
+
+medusa_status medusa_buffers_save(const uint32_t* d_perm, const uint64_t* d_perm_off, uint32_t n_perm,
+                                  const uint64_t* d_base, uint32_t n_alloc, uint8_t* d_blob,
+                                  medusa_buf_report* d_report, cudaStream_t stream) {
+    medusa_status st = buffers_copy_args(d_perm, d_perm_off, n_perm, d_blob, d_report);
+    if (st != MEDUSA_OK) return st;
+    if (n_alloc > 0 && (!d_base || !aligned8(d_base))) return MEDUSA_ERR_INVALID_ARG;
+    cudaError_t e = launch_buffers_copy(true, d_blob, nullptr, d_perm, d_perm_off, n_perm, d_base, nullptr, n_alloc,
+                                        d_report, stream);
+    return e == cudaSuccess ? MEDUSA_OK : cuda_fail(e);
+}
+
+medusa_status medusa_buffers_restore(const uint8_t* d_blob, const uint32_t* d_perm, const uint64_t* d_perm_off,
+                                     uint32_t n_perm, const uint64_t* d_new_base, const uint64_t* d_new_size,
+                                     uint32_t n_alloc, medusa_buf_report* d_report, cudaStream_t stream) {
+    medusa_status st = buffers_copy_args(d_perm, d_perm_off, n_perm, d_blob, d_report);
+    if (st != MEDUSA_OK) return st;
+    if (n_alloc > 0 && (!d_new_base || !d_new_size || !aligned8(d_new_base) || !aligned8(d_new_size)))
+        return MEDUSA_ERR_INVALID_ARG;
+    cudaError_t e = launch_buffers_copy(false, nullptr, d_blob, d_perm, d_perm_off, n_perm, d_new_base, d_new_size,
+                                        n_alloc, d_report, stream);
+    return e == cudaSuccess ? MEDUSA_OK : cuda_fail(e);
+}
+
 }  // extern "C"

@@ -159,4 +159,13 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
 medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
                                     cudaError_t* cuda_err);
 
+// ---- buffer contents (buffers.cu) ---------------------------------------------
+medusa_status run_buffers_plan(const medusa_alloc* alloc, uint32_t n_alloc, const uint32_t* cap, uint32_t n_cap,
+                               const uint64_t* slot, uint64_t n_slots, uint8_t* cls, uint32_t* perm,
+                               uint64_t* perm_off, uint32_t capacity, uint32_t* h_n_perm, uint64_t* h_bytes,
+                               cudaStream_t stream, cudaError_t* err);
+cudaError_t launch_buffers_copy(bool to_blob, uint8_t* blob_w, const uint8_t* blob_r, const uint32_t* perm,
+                                const uint64_t* perm_off, uint32_t n_perm, const uint64_t* base, const uint64_t* size,
+                                uint32_t n_alloc, medusa_buf_report* rep, cudaStream_t stream);
+
 }  // namespace medusa

@@ -73,6 +73,19 @@ def test_argument_errors_need_no_device(lib):
                               P(0), U32(0), r, P(0)) == -1
     # kernel table: null with a size
     assert lib.medusa_kernel_table_set(P(0), U32(4), P(0)) == -1
+    # buffers plan: null outputs, misaligned trace, captures without array
+    np_, nb = U32(5), U64(5)
+    assert lib.medusa_buffers_plan(P(8), U32(1), P(0), U32(0), P(0), U64(0), P(8), P(8), P(8), U32(1), None,
+                                   ctypes.byref(nb), P(0)) == -1
+    assert nb.value == 0
+    assert lib.medusa_buffers_plan(P(12), U32(1), P(0), U32(0), P(0), U64(0), P(8), P(8), P(8), U32(1),
+                                   ctypes.byref(np_), ctypes.byref(nb), P(0)) == -1
+    assert lib.medusa_buffers_plan(P(8), U32(1), P(0), U32(2), P(0), U64(0), P(8), P(8), P(8), U32(1),
+                                   ctypes.byref(np_), ctypes.byref(nb), P(0)) == -1
+    # save / restore: null report, misaligned blob (16-byte rule), missing replay arrays
+    assert lib.medusa_buffers_save(P(8), P(8), U32(1), P(8), U32(1), P(16), P(0), P(0)) == -1
+    assert lib.medusa_buffers_save(P(8), P(8), U32(1), P(8), U32(1), P(24), P(64), P(0)) == -1
+    assert lib.medusa_buffers_restore(P(16), P(8), P(8), U32(1), P(0), P(0), U32(3), P(64), P(0)) == -1
 
 
 def test_no_cpu_fallback_without_gpu(lib):
@@ -81,3 +94,5 @@ def test_no_cpu_fallback_without_gpu(lib):
     if torch.cuda.is_available():
         pytest.skip("GPU present")
     assert lib.medusa_kernel_table_set(ctypes.c_void_p(0), ctypes.c_uint32(0), ctypes.c_void_p(0)) == -5
+    P, U32 = ctypes.c_void_p, ctypes.c_uint32
+    assert lib.medusa_buffers_restore(P(16), P(8), P(8), U32(0), P(0), P(0), U32(0), P(64), P(0)) == -5
