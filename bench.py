@@ -451,24 +451,98 @@ def run_ours(args):
         e2e_step()
         e2e_ev[k][1].record(stream)
     barrier()
-    e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_ev)
-    e2e_value = nodes_total / (max_over_ranks(e2e_ms, dist, dev) / 1e3)
+    e2e_serial_ms = sum(a.elapsed_time(b) for a, b in e2e_ev)
     assert np.array_equal(out_h.numpy().view(np.uint64), medusa.to_numpy_u64(dst))
+
+    # pipelined end to end (the same public API calls, asynchronous variant): step k's
+    # inputs go up on a copy stream, its analysis + restore run on the compute stream,
+    # its results come down on a second copy stream, with two buffer sets so that
+    # step k+1's upload and step k-1's download overlap step k's kernels.  Every step
+    # still copies its full inputs in and its full results out.
+    s_in, s_cp, s_out = torch.cuda.Stream(dev), torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+    sets = []
+    for _ in range(2):
+        sets.append(dict(
+            d_in={k: torch.empty_like(v, device=dev) for k, v in pinned.items()},
+            slots=medusa.alloc_slots(gs.n_words, dev), res=torch.zeros(2, dtype=torch.int64, device=dev),
+            dst=torch.empty(gs.n_words, dtype=torch.int64, device=dev),
+            fout=torch.empty(gs.n_nodes, dtype=torch.int64, device=dev),
+            rep=torch.empty(8, dtype=torch.int64, device=dev),
+            out_h=torch.empty(gs.n_words, dtype=torch.int64).pin_memory(),
+            fout_h=torch.empty(gs.n_nodes, dtype=torch.int64).pin_memory(),
+            rep_h=torch.empty(8, dtype=torch.int64).pin_memory(),
+            res_h=torch.empty(2, dtype=torch.int64).pin_memory(),
+            ev_in=torch.cuda.Event(), ev_cp=torch.cuda.Event(), ev_out=torch.cuda.Event()))
+
+    def e2e_pipelined(n):
+        for k in range(n):
+            S = sets[k % 2]
+            with torch.cuda.stream(s_in):
+                if k >= 2:
+                    s_in.wait_event(S["ev_cp"])  # the set's inputs are no longer read
+                for name, v in pinned.items():
+                    S["d_in"][name].copy_(v, non_blocking=True)
+                S["ev_in"].record(s_in)
+            with torch.cuda.stream(s_cp):
+                s_cp.wait_event(S["ev_in"])
+                if k >= 2:
+                    s_cp.wait_event(S["ev_out"])  # the set's outputs have been read back
+                d = S["d_in"]
+                medusa.kernel_table_set(d["table"], stream=s_cp)
+                medusa.materialize_async(d["words"], d["node_off"], d["node_t"], d["allocs"], out=S["slots"],
+                                         result=S["res"], stream=s_cp)
+                medusa.restore(d["words"], S["slots"], d["old_base"], d["new_base"], d["new_size"], d["func_id"],
+                               dst=S["dst"], func_out=S["fout"], report=S["rep"], stream=s_cp, from_table=True)
+                S["ev_cp"].record(s_cp)
+            with torch.cuda.stream(s_out):
+                s_out.wait_event(S["ev_cp"])
+                S["out_h"].copy_(S["dst"], non_blocking=True)
+                S["fout_h"].copy_(S["fout"], non_blocking=True)
+                S["rep_h"].copy_(S["rep"], non_blocking=True)
+                S["res_h"].copy_(S["res"], non_blocking=True)
+                S["ev_out"].record(s_out)
+
+    e2e_pipelined(2)
+    barrier()
+    pa, pb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    pa.record(s_in)
+    e2e_pipelined(args.steps)
+    for S in sets:
+        s_out.wait_event(S["ev_out"])
+    pb.record(s_out)
+    barrier()
+    e2e_ms = pa.elapsed_time(pb)
+    for S in sets:  # every set's last step: status, slot count, restored words, handles, report
+        assert int(S["res_h"][0].item()) & 0xFFFFFFFF == 0 and int(S["res_h"][1].item()) == n_slots
+        assert torch.equal(S["out_h"], out_h) and torch.equal(S["fout_h"], fout_h)
+        assert int(S["rep_h"][0].item()) == 0
+    e2e_value = nodes_total / (max_over_ranks(e2e_ms, dist, dev) / 1e3)
+    e2e_serial = nodes_total / (max_over_ranks(e2e_serial_ms, dist, dev) / 1e3)
 
     # ---- CPU baseline: the oracle as it stands, rank 0 at N=1 only ----
     cpu = None
     if ws == 1 and not args.no_cpu_baseline:
         ge.build_oracle()
         import oracle
-        reps, t_cpu, t0 = 0, 0.0, time.perf_counter()
+        reps, t_mat, t_res, t0 = 0, 0.0, 0.0, time.perf_counter()
         while time.perf_counter() - t0 < args.cpu_seconds:
             t1 = time.perf_counter()
             m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+            t2 = time.perf_counter()
             oracle.restore(gs.words, m["slot_g"], m["slot_id"], m["slot_off"], gs.allocs["base"], gs.new_base,
                            gs.new_size, gs.func_id, gs.table)
-            t_cpu += time.perf_counter() - t1
+            t_mat += t2 - t1
+            t_res += time.perf_counter() - t2
             reps += 1
+        t_cpu = t_mat + t_res
+        gpu_mat_s = mat_s
+        gpu_res_s = restore_avg_s
         cpu = {"value": gs.n_nodes * reps / t_cpu, "unit": "nodes/s", "cores": 1, "kind": "oracle",
+               "materialize_nodes_per_s": gs.n_nodes * reps / t_mat,
+               "restore_nodes_per_s": gs.n_nodes * reps / t_res,
+               "gpu_speedup": {"whole_path": value / (gs.n_nodes * reps / t_cpu),
+                               "materialize": (gs.n_nodes / gpu_mat_s) / (gs.n_nodes * reps / t_mat),
+                               "restore": (gs.n_nodes / gpu_res_s) / (gs.n_nodes * reps / t_res)},
                "sample": f"the full per-rank {cfg} set, {reps} passes (materialize + restore), "
                          f"single-threaded oracle/oracle.cpp; host has {os.cpu_count()} cores"}
 
@@ -476,7 +550,8 @@ def run_ours(args):
         line = {
             "metric": "graph nodes restored/sec (materialize + restore, whole hot path)",
             "value": value, "unit": "nodes/s", "n_gpus": ws, "steps": args.steps, "warmup": max(args.warmup, 3),
-            "ms_per_step": max_ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "ms_per_step": max_ms / args.steps, "higher_is_better": True,
+            "step_ms_p10_p50_p90": [float(np.percentile(step_ms, q)) for q in (10, 50, 90)], "scaling": "weak", "vs_baseline": None,
             "dtype": "u64", "data": "synthetic",
             "config": {"workload": f"{cfg} per rank: {desc}", "nodes_per_rank": gs.n_nodes, "words": gs.n_words,
                        "allocs": gs.n_alloc, "slots": n_slots, "kernel_names": int(gs.table.size),
@@ -489,7 +564,13 @@ def run_ours(args):
             "sustained_relocate": sus,
             "buffers": buf,
             "cpu_baseline": cpu,
-            "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+            "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                    "mode": "pipelined: inputs up (copy stream) / materialize_async + restore (compute stream) / "
+                            "results down (copy stream), two buffer sets; every step copies all its inputs and "
+                            "results; timed from the first upload to the last download",
+                    "serial_value": e2e_serial,
+                    "serial_mode": "one step at a time: H2D, medusa_materialize (host round trip), "
+                                   "medusa_restore, D2H, on one stream"},
             "gpu_launches": len(launches),
             "graph_step": "one CUDA graph per step: medusa_kernel_table_set, medusa_materialize_async, "
                           f"medusa_restore(MEDUSA_N_SLOTS_FROM_TABLE); {len(launches) // max(args.steps, 1)} "
