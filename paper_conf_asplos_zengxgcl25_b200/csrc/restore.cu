@@ -61,13 +61,16 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-__global__ void __launch_bounds__(kThreads, 8)
+template <int CPB>
+__global__ void __launch_bounds__(kThreads, (CPB == 1 ? 8 : 6))
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
-    __shared__ __align__(128) uint64_t s_words[kTaskWords];
-    __shared__ uint32_t s_mask[kMaskPerTask];
-    __shared__ uint32_t s_pre[kMaskPerTask];
+    constexpr uint32_t kWords = CPB * kTaskWords;   // words of this CTA (CPB consecutive chunks)
+    constexpr uint32_t kMask = CPB * kMaskPerTask;  // their mask words
+    __shared__ __align__(128) uint64_t s_words[kWords];
+    __shared__ uint32_t s_mask[kMask];
+    __shared__ uint32_t s_pre[kMask];
     __shared__ uint32_t s_rec0, s_nrec;
-    __shared__ __align__(8) unsigned long long s_mbar;
+    __shared__ __align__(8) unsigned long long s_mbar[CPB];
 
     const uint32_t tid = threadIdx.x;
     const uint32_t task = blockIdx.x;
@@ -75,13 +78,12 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     const unsigned long long tl0 = TL_NOW();
 
     if (task < n_word_tasks) {
-        const uint64_t ws = (uint64_t)task * kTaskWords;
-        const uint32_t n = (uint32_t)min((uint64_t)kTaskWords, a.n_words - ws);
+        const uint64_t ws = (uint64_t)task * kWords;
+        const uint32_t n = (uint32_t)min((uint64_t)kWords, a.n_words - ws);
         const uint64_t* gsrc = a.src + ws;
         uint64_t* gdst = a.dst + ws;
         const bool tma = (((reinterpret_cast<uintptr_t>(gsrc) | reinterpret_cast<uintptr_t>(gdst)) & 15) == 0) &&
                          (n % 2 == 0);
-        const uint32_t mb = smem_u32(&s_mbar);
         if (tid == 0) {  // warm L2 with this CTA's slice of the replayed base table
             const uint64_t bytes = (uint64_t)a.n_alloc * 8;
             const uint64_t per = ((bytes + n_word_tasks - 1) / n_word_tasks + 255) & ~255ull;
@@ -97,47 +99,63 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 }
             }
         }
-        // 1. the chunk's words: one bulk copy into shared memory; meanwhile the
-        //    mask words and the record range
+        // 1. the CTA's words: one bulk copy per chunk into shared memory (all issued
+        //    at once); meanwhile the mask words and the record range
         if (tid == 0 && tma) {
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+#pragma unroll
+            for (int c = 0; c < CPB; ++c) {
+                const uint32_t mb = smem_u32(&s_mbar[c]);
+                asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+            }
             asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
-            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                         ::"r"(smem_u32(s_words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
+#pragma unroll
+            for (int c = 0; c < CPB; ++c) {
+                const uint32_t q0 = c * kTaskWords;
+                if (q0 >= n) break;
+                const uint32_t nc = min(n - q0, kTaskWords);
+                const uint32_t mb = smem_u32(&s_mbar[c]);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(nc * 8) : "memory");
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(smem_u32(s_words + q0)), "l"(gsrc + q0), "r"(nc * 8), "r"(mb) : "memory");
+            }
         }
         if (!tma)
             for (uint32_t q = tid; q < n; q += kThreads) s_words[q] = ld_stream(gsrc + q);
         const uint64_t n_mask = (a.n_words + 31) / 32;
         const uint64_t mw0 = ws / 32;
-        if (tid < kMaskPerTask) {
-            s_mask[tid] = (mw0 + tid < n_mask) ? a.mask[mw0 + tid] : 0u;
-        } else if (tid == kMaskPerTask) {
-            const uint32_t r0 = a.chunk_base[task], r1 = a.chunk_base[task + 1];
+        const uint64_t n_chunks = (a.n_words + kTaskWords - 1) / kTaskWords;
+        for (uint32_t m = tid; m < kMask; m += kThreads) s_mask[m] = (mw0 + m < n_mask) ? a.mask[mw0 + m] : 0u;
+        if (tid == kThreads - 1) {
+            const uint64_t c0 = (uint64_t)task * CPB;
+            const uint32_t r0 = a.chunk_base[c0], r1 = a.chunk_base[min(c0 + CPB, n_chunks)];
             s_rec0 = r0;
             s_nrec = r1 > r0 ? r1 - r0 : 0;
         }
         __syncthreads();
-        // 2. exclusive prefix of the 64 mask popcounts (warp 0)
+        // 2. exclusive prefix of the mask popcounts (warp 0; kMask / 32 words per lane)
         if (tid < 32) {
-            const uint32_t p0 = __popc(s_mask[2 * tid]), p1 = __popc(s_mask[2 * tid + 1]);
-            uint32_t incl = p0 + p1;
+            constexpr int kPer = kMask / 32;
+            uint32_t pc[kPer], incl = 0;
+#pragma unroll
+            for (int j = 0; j < kPer; ++j) { pc[j] = __popc(s_mask[kPer * tid + j]); incl += pc[j]; }
+            const uint32_t own = incl;
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
                 const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
                 if (tid >= d) incl += y;
             }
-            s_pre[2 * tid] = incl - p0 - p1;
-            s_pre[2 * tid + 1] = incl - p1;
+            uint32_t run = incl - own;
+#pragma unroll
+            for (int j = 0; j < kPer; ++j) { s_pre[kPer * tid + j] = run; run += pc[j]; }
         }
         const uint64_t rec0 = s_rec0;
         const uint32_t n_rec = s_nrec;
-        const uint32_t n_rec_c = min(n_rec, (uint32_t)kTaskWords);
+        const uint32_t n_rec_c = min(n_rec, kWords);
         // 3. records, two per thread per round: load, gather, (after the prefix is
         //    ready) locate the word, validate and rewrite it in shared memory
         uint32_t n_id = 0, n_rg = 0, n_st = 0;
         uint64_t first = ~0ull;
-        bool words_ready = !tma;
+        uint32_t ready_mask = tma ? 0u : ~0u;  // chunks whose words have landed
         for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += 2 * kThreads) {
             uint64_t exp[2], nv[2];
             uint32_t kind[2];  // 0 ok, 1 bad id, 2 bad range, 3 none
@@ -169,45 +187,68 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 }
             }
             if (rb == 0) __syncthreads();  // s_pre ready
-            if (!words_ready) {
-                uint32_t ready = 0;
-                while (!ready) {
-                    asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
-                                 : "=r"(ready) : "r"(mb) : "memory");
-                }
-                words_ready = true;
-            }
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 if (kind[u] == 3) continue;
                 const uint32_t r = rb + tid + u * kThreads;
-                uint32_t lo = 0, hi = kMaskPerTask;  // mask word m with s_pre[m] <= r < s_pre[m] + popc
+                uint32_t lo = 0, hi = kMask;  // mask word m with s_pre[m] <= r < s_pre[m] + popc
                 while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
                 const uint32_t bit = __fns(s_mask[lo], 0, r - s_pre[lo] + 1);
                 const uint32_t q = lo * 32 + bit;
                 bool bad = true;
                 if (bit >= 32 || q >= n) {
                     ++n_id;  // more records than mask bits: nothing to apply
-                } else if (kind[u] == 0) {
-                    if (s_words[q] == exp[u]) { s_words[q] = nv[u]; bad = false; }
-                    else ++n_st;
-                } else if (kind[u] == 1) {
-                    ++n_id;
                 } else {
-                    ++n_rg;
+                    const uint32_t c = q / kTaskWords;
+                    if (!((ready_mask >> c) & 1u)) {  // this chunk's words: wait for its bulk copy
+                        const uint32_t mb = smem_u32(&s_mbar[c]);
+                        uint32_t ready = 0;
+                        while (!ready) {
+                            asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
+                                         : "=r"(ready) : "r"(mb) : "memory");
+                        }
+                        ready_mask |= 1u << c;
+                    }
+                    if (kind[u] == 0) {
+                        if (s_words[q] == exp[u]) { s_words[q] = nv[u]; bad = false; }
+                        else ++n_st;
+                    } else if (kind[u] == 1) {
+                        ++n_id;
+                    } else {
+                        ++n_rg;
+                    }
                 }
                 if (bad) first = min(first, ws + (q < n ? q : 0));
             }
         }
         // slots the mask shows beyond the table's records have nothing to apply
-        if (tid == 0 && n_rec > (uint32_t)kTaskWords) n_id += n_rec - kTaskWords;
+        if (tid == 0 && n_rec > kWords) n_id += n_rec - kWords;
+        // every chunk's bulk copy must have landed before its words go back out
+        if (tid == 0 && tma) {
+#pragma unroll
+            for (int c = 0; c < CPB; ++c) {
+                if ((ready_mask >> c) & 1u || c * kTaskWords >= n) continue;
+                const uint32_t mb = smem_u32(&s_mbar[c]);
+                uint32_t ready = 0;
+                while (!ready) {
+                    asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
+                                 : "=r"(ready) : "r"(mb) : "memory");
+                }
+            }
+        }
         __syncthreads();
-        // 4. the chunk's words back to HBM
+        // 4. the CTA's words back to HBM
         if (tma) {
             if (tid == 0) {
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
-                             ::"l"(gdst), "r"(smem_u32(s_words)), "r"(n * 8) : "memory");
+#pragma unroll
+                for (int c = 0; c < CPB; ++c) {
+                    const uint32_t q0 = c * kTaskWords;
+                    if (q0 >= n) break;
+                    const uint32_t nc = min(n - q0, kTaskWords);
+                    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                                 ::"l"(gdst + q0), "r"(smem_u32(s_words + q0)), "r"(nc * 8) : "memory");
+                }
                 asm volatile("cp.async.bulk.commit_group;" ::: "memory");
                 asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
             }
@@ -254,8 +295,13 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
 
 }  // namespace
 
+#ifndef MEDUSA_RESTORE_CPB
+#define MEDUSA_RESTORE_CPB 2
+#endif
+constexpr int kCPB = MEDUSA_RESTORE_CPB;  // chunks per restore CTA
+
 cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
-    const uint32_t n_word_tasks = (uint32_t)((a.n_words + kTaskWords - 1) / kTaskWords);
+    const uint32_t n_word_tasks = (uint32_t)((a.n_words + kCPB * kTaskWords - 1) / (kCPB * kTaskWords));
     const uint32_t n_node_tasks = a.func_id ? (a.n_nodes + kNodesPerTask - 1) / kNodesPerTask : 0;
     const uint32_t n_tasks = n_word_tasks + n_node_tasks;
     {
@@ -265,7 +311,7 @@ cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     }
     if (n_tasks) {
         TimedLaunch tl("restore", stream);
-        cudaError_t e = launch_pdl(restore_kernel, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks);
+        cudaError_t e = launch_pdl(restore_kernel<kCPB>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks);
         if (e != cudaSuccess) return e;
     }
     return cudaGetLastError();
