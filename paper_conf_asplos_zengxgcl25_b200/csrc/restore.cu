@@ -61,6 +61,35 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
+// Kernel-address fill of 2048 nodes (gather task gt): func_out[j] =
+// table[func_id[j]], unresolved ids counted.
+__device__ __forceinline__ void gather_role(const RestoreArgs& a, uint32_t gt, unsigned long long* rep) {
+    const uint32_t tid = threadIdx.x;
+    const uint64_t j0 = (uint64_t)gt * kNodesPerTask;
+    uint32_t n_bad = 0;
+    uint64_t first = ~0ull;
+#pragma unroll
+    for (int k = 0; k < kNodesPerTask / kThreads; ++k) {
+        const uint64_t j = j0 + tid + k * kThreads;
+        if (j < a.n_nodes) {
+            const uint32_t f = a.func_id[j];
+            uint64_t addr = 0;
+            if (f < a.n_func) addr = __ldg(a.table + f);
+            if (addr == 0) {
+                ++n_bad;
+                first = min(first, j);
+            }
+            a.func_out[j] = addr;
+        }
+    }
+    pdl_wait();
+    pdl_trigger();
+    if (n_bad) {
+        atomicAdd(rep + 5, (unsigned long long)n_bad);
+        atomicMin(rep + 6, (unsigned long long)first);
+    }
+}
+
 template <int CPB>
 __global__ void __launch_bounds__(kThreads, (CPB == 1 ? 8 : 6))
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
@@ -266,29 +295,141 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         }
         TL_REC(7, 0, tl0);
     } else if (task < n_tasks) {
-        const uint64_t j0 = (uint64_t)(task - n_word_tasks) * kNodesPerTask;
-        uint32_t n_bad = 0;
-        uint64_t first = ~0ull;
+        gather_role(a, task - n_word_tasks, rep);
+        TL_REC(7, 1, tl0);
+    }
+}
+
+// In place (dst == src): only the slot words are read and written -- the words
+// in between are constants that stay where they are.  One CTA per
+// CPB chunks: mask words + record range, popcount prefix, then per record:
+// load, gather, locate its word, read it, validate, write it back.  No word
+// staging, so the pass moves ~8 B/slot of image instead of 16 B/word.
+template <int CPB>
+__global__ void __launch_bounds__(kThreads)
+restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
+    constexpr uint32_t kWords = CPB * kTaskWords;
+    constexpr uint32_t kMask = CPB * kMaskPerTask;
+    constexpr uint32_t kPer = 2;  // records per thread per round
+    __shared__ uint32_t s_mask[kMask];
+    __shared__ uint32_t s_pre[kMask];
+    __shared__ uint32_t s_rec0, s_nrec;
+    const uint32_t tid = threadIdx.x;
+    const uint32_t task = blockIdx.x;
+    unsigned long long* rep = reinterpret_cast<unsigned long long*>(a.report);
+    const unsigned long long tl0 = TL_NOW();
+    if (task < n_word_tasks) {
+        const uint64_t ws = (uint64_t)task * kWords;
+        const uint32_t n = (uint32_t)min((uint64_t)kWords, a.n_words - ws);
+        const uint64_t n_mask = (a.n_words + 31) / 32;
+        const uint64_t mw0 = ws / 32;
+        const uint64_t n_chunks = (a.n_words + kTaskWords - 1) / kTaskWords;
+        for (uint32_t m = tid; m < kMask; m += kThreads) s_mask[m] = (mw0 + m < n_mask) ? a.mask[mw0 + m] : 0u;
+        if (tid == kThreads - 1) {
+            const uint64_t c0 = (uint64_t)task * CPB;
+            const uint32_t r0 = a.chunk_base[c0], r1 = a.chunk_base[min(c0 + CPB, n_chunks)];
+            s_rec0 = r0;
+            s_nrec = r1 > r0 ? r1 - r0 : 0;
+        }
+        __syncthreads();
+        if (tid < 32) {
+            constexpr int kMw = kMask / 32;
+            uint32_t pc[kMw], incl = 0;
 #pragma unroll
-        for (int k = 0; k < kNodesPerTask / kThreads; ++k) {
-            const uint64_t j = j0 + tid + k * kThreads;
-            if (j < a.n_nodes) {
-                const uint32_t f = a.func_id[j];
-                uint64_t addr = 0;
-                if (f < a.n_func) addr = __ldg(a.table + f);
-                if (addr == 0) {
-                    ++n_bad;
-                    first = min(first, j);
+            for (int j = 0; j < kMw; ++j) { pc[j] = __popc(s_mask[kMw * tid + j]); incl += pc[j]; }
+            const uint32_t own = incl;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                if (tid >= d) incl += y;
+            }
+            uint32_t run = incl - own;
+#pragma unroll
+            for (int j = 0; j < kMw; ++j) { s_pre[kMw * tid + j] = run; run += pc[j]; }
+        }
+        const uint64_t rec0 = s_rec0;
+        const uint32_t n_rec = s_nrec;
+        const uint32_t n_rec_c = min(n_rec, kWords);
+        uint32_t n_id = 0, n_rg = 0, n_st = 0;
+        uint64_t first = ~0ull;
+        for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += kPer * kThreads) {
+            uint64_t exp[kPer], nv[kPer];
+            uint32_t kind[kPer];  // 0 ok, 1 bad id, 2 bad range, 3 none
+#pragma unroll
+            for (int u = 0; u < kPer; ++u) {
+                const uint32_t r = rb + tid + u * kThreads;
+                kind[u] = 3;
+                exp[u] = nv[u] = 0;
+                if (r < n_rec_c) {
+                    kind[u] = 1;
+                    const uint64_t k = rec0 + r;
+                    if (k < a.n_slots) {
+                        const uint64_t rec = a.slot[k];
+                        const uint64_t id = rec >> MEDUSA_OFF_BITS;
+                        const uint64_t off = rec & kOffMask;
+                        if (id < a.n_alloc) {
+                            const uint64_t sz = __ldg(a.new_size + id);
+                            const uint64_t ob = __ldg(a.old_base + id);
+                            const uint64_t nb = __ldg(a.new_base + id);
+                            if (off < sz) {
+                                kind[u] = 0;
+                                exp[u] = ob + off;
+                                nv[u] = nb + off;
+                            } else {
+                                kind[u] = 2;
+                            }
+                        }
+                    }
                 }
-                a.func_out[j] = addr;
+            }
+            if (rb == 0) __syncthreads();  // s_pre ready
+            uint32_t qs[kPer];
+            uint64_t cur[kPer];
+#pragma unroll
+            for (int u = 0; u < kPer; ++u) {  // locate every word first, then load them together
+                qs[u] = 0xFFFFFFFFu;
+                if (kind[u] == 3) continue;
+                const uint32_t r = rb + tid + u * kThreads;
+                uint32_t lo = 0, hi = kMask;
+                while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
+                const uint32_t bit = __fns(s_mask[lo], 0, r - s_pre[lo] + 1);
+                const uint32_t q = lo * 32 + bit;
+                if (bit < 32 && q < n) {
+                    qs[u] = q;
+                    if (kind[u] == 0) cur[u] = ld_stream(a.src + ws + q);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kPer; ++u) {
+                if (kind[u] == 3) continue;
+                const uint32_t q = qs[u];
+                bool bad = true;
+                if (q == 0xFFFFFFFFu) {
+                    ++n_id;  // more records than mask bits: nothing to apply
+                } else if (kind[u] == 0) {
+                    if (cur[u] == exp[u]) { st_stream(a.dst + ws + q, nv[u]); bad = false; }
+                    else ++n_st;
+                } else if (kind[u] == 1) {
+                    ++n_id;
+                } else {
+                    ++n_rg;
+                }
+                if (bad) first = min(first, ws + (q != 0xFFFFFFFFu ? q : 0));
             }
         }
+        if (tid == 0 && n_rec > kWords) n_id += n_rec - kWords;
         pdl_wait();
         pdl_trigger();
-        if (n_bad) {
-            atomicAdd(rep + 5, (unsigned long long)n_bad);
-            atomicMin(rep + 6, (unsigned long long)first);
+        if (n_id | n_rg | n_st) {
+            atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));
+            atomicMin(rep + 1, (unsigned long long)first);
+            if (n_id) atomicAdd(rep + 2, (unsigned long long)n_id);
+            if (n_rg) atomicAdd(rep + 3, (unsigned long long)n_rg);
+            if (n_st) atomicAdd(rep + 4, (unsigned long long)n_st);
         }
+        TL_REC(7, 2, tl0);
+    } else if (task < n_tasks) {
+        gather_role(a, task - n_word_tasks, rep);
         TL_REC(7, 1, tl0);
     }
 }
@@ -298,10 +439,16 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
 #ifndef MEDUSA_RESTORE_CPB
 #define MEDUSA_RESTORE_CPB 2
 #endif
-constexpr int kCPB = MEDUSA_RESTORE_CPB;  // chunks per restore CTA
+constexpr int kCPB = MEDUSA_RESTORE_CPB;  // chunks per restore CTA (out of place)
+#ifndef MEDUSA_RESTORE_CPB_IP
+#define MEDUSA_RESTORE_CPB_IP 2
+#endif
+constexpr int kCPBInPlace = MEDUSA_RESTORE_CPB_IP;  // chunks per restore CTA (in place)
 
 cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
-    const uint32_t n_word_tasks = (uint32_t)((a.n_words + kCPB * kTaskWords - 1) / (kCPB * kTaskWords));
+    const bool in_place = a.src == a.dst;
+    const uint64_t cpb = in_place ? kCPBInPlace : kCPB;
+    const uint32_t n_word_tasks = (uint32_t)((a.n_words + cpb * kTaskWords - 1) / (cpb * kTaskWords));
     const uint32_t n_node_tasks = a.func_id ? (a.n_nodes + kNodesPerTask - 1) / kNodesPerTask : 0;
     const uint32_t n_tasks = n_word_tasks + n_node_tasks;
     {
@@ -311,7 +458,9 @@ cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     }
     if (n_tasks) {
         TimedLaunch tl("restore", stream);
-        cudaError_t e = launch_pdl(restore_kernel<kCPB>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks);
+        cudaError_t e = in_place
+            ? launch_pdl(restore_inplace_kernel<kCPBInPlace>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks)
+            : launch_pdl(restore_kernel<kCPB>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks);
         if (e != cudaSuccess) return e;
     }
     return cudaGetLastError();

@@ -101,6 +101,24 @@ def test_in_place_and_misaligned(graph_sets):
     assert np.array_equal(medusa.to_numpy_u64(dst_v), packed[3])
 
 
+@pytest.mark.parametrize("name", ["toy", "all10"])
+def test_in_place_full_path(graph_sets, name):
+    """In-place restore (the online phase patches the loaded image) at full size:
+    bit-exact restored image, kernel-address fill and report."""
+    gs = graph_sets(name)
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    medusa.kernel_table_set(inp["table"])
+    buf = inp["words"].clone()
+    _, fout, rep = medusa.restore(buf, slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                                  dst=buf)
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size,
+                             gs.func_id, gs.table)
+    assert np.array_equal(medusa.to_numpy_u64(buf), packed[3])
+    assert np.array_equal(medusa.to_numpy_u64(fout), packed[4])
+    assert np.array_equal(medusa.report_numpy(rep), packed[5])
+
+
 def test_fault_injection_matches_oracle(graph_sets):
     gs = graph_sets("toy")
     inp = medusa.upload(gs, DEV)
@@ -127,6 +145,13 @@ def test_fault_injection_matches_oracle(graph_sets):
     assert np.array_equal(medusa.to_numpy_u64(dst), dst_o)
     assert np.array_equal(medusa.to_numpy_u64(fout), fout_o)
     assert np.array_equal(medusa.report_numpy(rep), rep_o)
+    # the same faults in place (dst == src: only slot words are read and written)
+    buf = t(src)
+    dst_i, fout_i, rep_i = medusa.restore(buf, slots, t(ob), t(nb), t(ns), t(fid, torch.int32), dst=buf)
+    assert dst_i.data_ptr() == buf.data_ptr()
+    assert np.array_equal(medusa.to_numpy_u64(buf), dst_o)
+    assert np.array_equal(medusa.to_numpy_u64(fout_i), fout_o)
+    assert np.array_equal(medusa.report_numpy(rep_i), rep_o)
     # the report is rewritten completely by the next call
     medusa.kernel_table_set(inp["table"])
     _, _, rep2 = medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"],

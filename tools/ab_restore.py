@@ -23,9 +23,11 @@ def main():
     ap.add_argument("--cpb", type=int, nargs="+", default=[1, 2, 4])
     ap.add_argument("--reps", type=int, default=30)
     ap.add_argument("--replicas", type=int, default=32)
+    ap.add_argument("--inplace", action="store_true", help="variants of the in-place kernel (MEDUSA_RESTORE_CPB_IP)")
     args = ap.parse_args()
     libs = {c: g.build_medusa(out=os.path.join(ROOT, "tools", f"libmedusa_cpb{c}.so"),
-                              defines=(f"MEDUSA_RESTORE_CPB={c}",)) for c in args.cpb}
+                              defines=(f"MEDUSA_RESTORE_CPB{'_IP' if args.inplace else ''}={c}",))
+            for c in args.cpb}
     import paper_conf_asplos_zengxgcl25_b200 as medusa
     from bench import algorithmic_bytes
     from workloads import make_graph_set
@@ -45,13 +47,16 @@ def main():
         medusa._lib = None
         medusa.LIB_PATH = path
         medusa.lib()
-        line = [f"CPB={c}"]
+        line = [f"CPB{'_IP' if args.inplace else ''}={c}"]
         for si, (x, inp, sl, alg) in enumerate(sets):
             medusa.kernel_table_set(inp["table"])
-            dst = torch.empty_like(inp["words"])
+            dst = inp["words"].clone() if args.inplace else torch.empty_like(inp["words"])
             fout = torch.empty(x.n_nodes, dtype=torch.int64, device=dev)
             rep = torch.empty(8, dtype=torch.int64, device=dev)
-            run = lambda: medusa.restore(inp["words"], sl, inp["old_base"], inp["new_base"], inp["new_size"],
+            src = dst if args.inplace else inp["words"]
+            # in place: identity relocation (old == new) so that every replay is a valid restore
+            nb = inp["old_base"] if args.inplace else inp["new_base"]
+            run = lambda: medusa.restore(src, sl, inp["old_base"], nb, inp["new_size"],
                                          inp["func_id"], dst=dst, func_out=fout, report=rep)
             for _ in range(3):
                 run()
@@ -69,7 +74,7 @@ def main():
                 ts.append(a.elapsed_time(b))
             t = statistics.median(ts) / 1e3
             assert int(medusa.report_numpy(rep)[0]) == 0
-            if si == 0:
+            if si == 0 and not args.inplace:
                 h = (dst.cpu().numpy().copy(), fout.cpu().numpy().copy())
                 if ref is None:
                     ref = h
