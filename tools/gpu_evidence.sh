@@ -9,13 +9,13 @@ timeout 600 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byte
 python tools/launch_table.py gpurun_out/launches_$TAG.csv > gpurun_out/launch_table_$TAG.txt 2>&1
 python tools/make_traffic.py gpurun_out/launches_$TAG.csv gpurun_out/ncu_traffic_$TAG.json > /dev/null
 # full capture of the dominant materialize kernel and of restore (a warm step)
-timeout 900 ncu --set full --clock-control none --import-source on -k "regex:k_classify|restore_kernel" -s 4 -c 2 -o gpurun_out/prof_$TAG python bench.py --steps 1 --warmup 4 --sustained 0 --no-cpu-baseline > gpurun_out/ncu_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k "regex:k_classify|restore_kernel|restore_inplace_kernel|k_buf_copy" -s 4 -c 5 -o gpurun_out/prof_$TAG python bench.py --steps 1 --warmup 4 --sustained 0 --no-cpu-baseline > gpurun_out/ncu_$TAG.log 2>&1
 tail -2 gpurun_out/ncu_$TAG.log
 # per-CTA timeline of one graph-captured step
 timeout 300 python tools/timeline.py --steps 5 > gpurun_out/timeline_$TAG.txt 2>&1
 # sanitizers on the GPU parity tests that use small sets
 for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "toy or tiny or edge or capacity or fault or async" > gpurun_out/sanitizer_${tool}_$TAG.log 2>&1
+  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_buffers.py -m gpu -x -q -k "toy or tiny or edge or capacity or fault or async or real_memory or errors" > gpurun_out/sanitizer_${tool}_$TAG.log 2>&1
   echo "$tool exit=$?" | tee -a gpurun_out/sanitizer_summary_$TAG.txt
   tail -3 gpurun_out/sanitizer_${tool}_$TAG.log | tee -a gpurun_out/sanitizer_summary_$TAG.txt
 done

@@ -6,7 +6,7 @@ rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 10]
 h = rows[0]
 idx = {k: i for i, k in enumerate(h)}
 data = [r for r in rows[1:] if r[idx["Metric Name"]] == "gpu__time_duration.sum"]
-names = [r[idx["Kernel Name"]].split("(")[0].split("::")[-1] for r in data]
+names = [r[idx["Kernel Name"]].split("(")[0].split("::")[-1].split("<")[0] for r in data]
 vals = [float(r[idx["Metric Value"]]) for r in data]
 unit = data[0][idx["Metric Unit"]] if data else "ns"
 scale = {"ns": 1e-3, "nsecond": 1e-3, "us": 1, "usecond": 1, "ms": 1e3, "msecond": 1e3}[unit]

@@ -6,7 +6,8 @@ import sys
 
 NAMES = {"k_classify": "mat_classify", "restore_kernel": "restore", "k_trace": "mat_trace",
          "k_prepare": "mat_prepare", "k_rank": "mat_rank", "k_check_mi": "mat_check_mi",
-         "k_check_mm": "mat_check_mm", "k_check": "mat_check", "k_iresolve": "mat_iresolve", "k_emit": "mat_emit"}
+         "k_check_mm": "mat_check_mm", "k_check": "mat_check", "k_iresolve": "mat_iresolve", "k_emit": "mat_emit",
+         "restore_inplace_kernel": "restore_inplace", "k_buf_copy<true>": "buf_save", "k_buf_copy<false>": "buf_restore"}
 rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 10]
 h = rows[0]
 ix = {k: i for i, k in enumerate(h)}
@@ -16,6 +17,8 @@ for r in rows[1:]:
     if r[ix["ID"]] == "ID":
         continue
     name = r[ix["Kernel Name"]].split("(")[0].split("::")[-1]
+    if name not in NAMES:
+        name = name.split("<")[0]  # restore_kernel<2> etc.
     if name not in NAMES:
         continue
     m = r[ix["Metric Name"]]
