@@ -23,5 +23,8 @@ print(json.dumps({
     "allocated_before_capture": r["n_pre"], "slots": r["slots"].n_slots,
     "slot_words_share": r["slots"].n_slots / max(int(r["words"].size), 1),
     "restore_report_bad": int(r["report"][0]), "outputs_bit_identical": all(bool(torch.equal(a, b)) for a, b in zip(r["outs_b"], r["refs"])),
+    "buffer_classes": {k: int((r["buf_class"] == v).sum()) for k, v in (("unused", 0), ("param", 1), ("temp", 2), ("perm", 3))},
+    "permanent_buffers": r["n_perm"], "saved_blob_bytes": r["blob_bytes"],
+    "outputs_equal_without_permanent_contents": [bool(torch.equal(a, b)) for a, b in zip(r["outs_unrestored"], r["refs"])],
     "kernels_sample": sorted(r["kernel_names"])[:8],
 }, indent=1))

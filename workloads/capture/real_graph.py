@@ -138,7 +138,8 @@ def capture(torch, batches=(8, 4, 2, 1), seq=16, seed=0, arena_bytes=1 << 30):
     L.ta_select(0)
     L.ta_clear()
     L.ta_log(1)
-    pool = torch.cuda.MemPool(alloc.allocator())
+    pool = torch.cuda.MemPool(alloc.allocator())       # model loading + warm-up
+    gpool = torch.cuda.MemPool(alloc.allocator())      # the graphs' private pool (vLLM's graph pool)
     torch.manual_seed(seed)
     with torch.cuda.use_mem_pool(pool):
         model = tiny_decoder(torch).cuda().eval()
@@ -151,15 +152,24 @@ def capture(torch, batches=(8, 4, 2, 1), seq=16, seed=0, arena_bytes=1 << 30):
                 model(ids[:b], mask)
         torch.cuda.current_stream().wait_stream(s)
         torch.cuda.synchronize()
-    graphs, outs = [], []
+    graphs, outs, magic = [], [], []
     for k, b in enumerate(batches):
         g = torch.cuda.CUDAGraph(keep_graph=True)  # (raw_cuda_graph needs the graph kept)
         L.ta_capture_begin(k)
-        with torch.no_grad(), torch.cuda.graph(g, pool=pool.id):
-            outs.append(model(ids[:b], mask))
+        with torch.no_grad(), torch.cuda.graph(g, pool=gpool.id):
+            if k == 0:
+                # one permanent buffer per graph: allocated during the
+                # (first) capture before any temporary, never freed, its 4-byte
+                # content (a "magic number") written outside the graphs and read by
+                # every replay.  (Allocated later, a graph's buffer could reuse a
+                # block an earlier graph's temporaries occupy in the shared pool.)
+                magic = [torch.empty((), device="cuda") for _ in batches]
+            outs.append(model(ids[:b], mask) * magic[k])
         L.ta_capture_end()
         graphs.append(g)
     L.ta_log(0)
+    for m in magic:
+        m.fill_(1.0)
     for g in graphs:
         g.instantiate()
         g.replay()
@@ -179,8 +189,8 @@ def capture(torch, batches=(8, 4, 2, 1), seq=16, seed=0, arena_bytes=1 << 30):
         n_all = int(cu.cuGraphGetNodes(graph, 0)[2])
         orders.append(_topo(cu, list(cu.cuGraphGetNodes(graph, n_all)[1])))
         raw.append(graph)
-    return dict(L=L, pool=pool, alloc=alloc, model=model, ids=ids, mask=mask, graph_objs=graphs, graphs=raw,
-                nodes=orders, events=ev, outs=outs, refs=refs)
+    return dict(L=L, pool=pool, gpool=gpool, alloc=alloc, model=model, ids=ids, mask=mask, graph_objs=graphs,
+                graphs=raw, nodes=orders, events=ev, outs=outs, refs=refs, magic=magic)
 
 
 def _topo(cu, nodes):
@@ -242,7 +252,8 @@ def _graph_image(cu, gi, nodes):
 
 def trace_arrays(ev, recs):
     """medusa inputs from the trace and the node list: allocation records with
-    event positions, and each kernel / memset node's launch position."""
+    event positions, each kernel / memset node's launch position, and the
+    (begin, end) positions of every capture (for medusa_buffers_plan)."""
     from workloads import ALLOC_DTYPE
 
     n_in = {}
@@ -260,13 +271,16 @@ def trace_arrays(ev, recs):
             emitted += 1
 
     ev_t = []
+    caps = []
     for k in range(ev.shape[0]):
         kind = int(ev[k, 0])
         if kind == 3:  # capture `ev[k, 4]` begins
             cap, emitted = int(ev[k, 4]), 0
+            caps.append([t, 0])
         elif kind == 4:  # ... ends: all its nodes were launched before what follows
             emit_until(cap, 1 << 62)
             cap = -1
+            caps[-1][1] = t
         elif cap >= 0 and int(ev[k, 3]) >= 0:
             emit_until(cap, int(ev[k, 3]))  # nodes captured before this call
         ev_t.append(t)
@@ -290,7 +304,18 @@ def trace_arrays(ev, recs):
     off = np.zeros(len(used) + 1, np.uint64)
     off[1:] = np.cumsum([len(r["blob"]) // 8 for r in used])
     node_t = np.array([node_pos[(r["graph"], r["pos"])] for r in used], np.uint32)
-    return words, off, node_t, arr, used
+    capture_t = np.array(caps, np.uint32).reshape(-1, 2)
+    return words, off, node_t, arr, used, capture_t
+
+
+def _alloc_of(allocs, ptr):
+    """Ordinal of the latest allocation whose range holds ptr."""
+    return int(np.nonzero((allocs["base"] <= ptr) & (ptr < allocs["base"] + allocs["size"]))[0][-1])
+
+
+def _in_capture(allocs, capture_t, i):
+    ta = int(allocs["t_alloc"][i])
+    return any(int(b) < ta < int(e) for b, e in capture_t)
 
 
 def online_bases(L, allocs, events):
@@ -323,23 +348,28 @@ def end_to_end(torch, medusa, seed=0):
 
     A = capture(torch, seed=seed)
     recs = parameter_image(cu, A["nodes"])
-    words, off, node_t, allocs, used = trace_arrays(A["events"], recs)
+    words, off, node_t, allocs, used, capture_t = trace_arrays(A["events"], recs)
     dev = torch.device("cuda")
     t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(dev)
     aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3)
     inp = dict(words=t(words, np.int64), node_off=t(off, np.int64), node_t=t(node_t, np.int32),
                allocs=torch.from_numpy(aa).to(dev))
     slots = medusa.materialize(**inp)
+    # copy-free buffer contents (§4.3): classify, and dump the permanent buffers
+    # offline
+    plan = medusa.buffers_plan(inp["allocs"], t(capture_t, np.int32), slots.slot, slots.n_slots)
+    buf_blob, rep_save = medusa.buffers_save(plan, t(allocs["base"], np.int64))
+    torch.cuda.synchronize()
+    cls = plan.cls.cpu().numpy()
     new_base = online_bases(A["L"], allocs, A["events"])
     live = allocs["t_free"] == T_END
-    first_launch = int(node_t.min()) if node_t.size else 0
     for i in np.nonzero(live)[0]:
-        if int(allocs["t_alloc"][i]) < first_launch:
-            # allocated before the capture (weights, inputs, workspaces): "the online
+        if cls[i] == medusa.BUF_PARAM or (cls[i] == medusa.BUF_UNUSED and not _in_capture(allocs, capture_t, i)):
+            # allocated before the captures (weights, inputs, workspaces): "the online
             # process loads the same weights / inputs"
             _check(rt.cudaMemcpy(int(new_base[i]), int(allocs["base"][i]), int(allocs["size"][i]),
                                  rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice))
-        else:  # the graph's own pool (activations, the output): recomputed by the graph
+        else:  # the graphs' own pool: poisoned; only the permanent buffers come back (from the blob)
             _check(rt.cudaMemset(int(new_base[i]), 0xEE, int(allocs["size"][i])))
     for i in np.nonzero(live)[0]:  # nothing may still point into the first arena
         _check(rt.cudaMemset(int(allocs["base"][i]), 0xFF, int(allocs["size"][i])))
@@ -369,18 +399,28 @@ def end_to_end(torch, medusa, seed=0):
             p.dst = int.from_bytes(blob, "little")
             _check(cu.cuGraphMemsetNodeSetParams(node_b, p))
     stream = torch.cuda.current_stream().cuda_stream
-    for gb in clones:
-        _check(cu.cuGraphLaunch(_check(cu.cuGraphInstantiate(gb, 0)), stream))
+    execs = [_check(cu.cuGraphInstantiate(gb, 0)) for gb in clones]
+
+    def run_and_read():
+        for ge in execs:
+            _check(cu.cuGraphLaunch(ge, stream))
+        torch.cuda.synchronize()
+        # the outputs: each of A's output tensors sits in some traced allocation; same offset in B
+        res = []
+        for out, ref in zip(A["outs"], A["refs"]):
+            op = out.data_ptr()
+            i = int(np.nonzero((allocs["base"] <= op) & (op < allocs["base"] + allocs["size"]))[0][-1])
+            ob = torch.empty_like(ref)
+            _check(rt.cudaMemcpy(ob.data_ptr(), int(new_base[i]) + (op - int(allocs["base"][i])),
+                                 ob.numel() * ob.element_size(), rt.cudaMemcpyKind.cudaMemcpyDeviceToHost))
+            res.append(ob)
+        return res
+
+    # negative control: the permanent buffers not restored yet (poisoned)
+    outs_unrestored = run_and_read()
+    rep_buf = medusa.buffers_restore(plan, buf_blob, t(new_base, np.int64), t(allocs["size"], np.int64))
     torch.cuda.synchronize()
-    # the outputs: each of A's output tensors sits in some traced allocation; same offset in B
-    outs_b = []
-    for out, ref in zip(A["outs"], A["refs"]):
-        op = out.data_ptr()
-        i = int(np.nonzero((allocs["base"] <= op) & (op < allocs["base"] + allocs["size"]))[0][-1])
-        ob = torch.empty_like(ref)
-        _check(rt.cudaMemcpy(ob.data_ptr(), int(new_base[i]) + (op - int(allocs["base"][i])),
-                             ob.numel() * ob.element_size(), rt.cudaMemcpyKind.cudaMemcpyDeviceToHost))
-        outs_b.append(ob)
+    outs_b = run_and_read()
     n_kernel = sum(1 for r in recs if r["kind"] == "kernel")
     names = set()
     for r in used:
@@ -388,9 +428,13 @@ def end_to_end(torch, medusa, seed=0):
             res = cu.cuKernelGetName(r["params"].kern) if int(r["params"].kern) else cu.cuFuncGetName(r["params"].func)
             if int(res[0]) == 0:
                 names.add(res[1].decode() if isinstance(res[1], bytes) else str(res[1]))
-    n_pre = int(np.sum(allocs["t_alloc"] < first_launch))
+    n_pre = int(np.sum(allocs["t_alloc"] < int(capture_t[0, 0]))) if capture_t.size else len(allocs)
     return dict(words=words, off=off, node_t=node_t, allocs=allocs, slots=slots, new_base=new_base, n_pre=n_pre,
                 restored=restored, report=report, refs=A["refs"], outs_b=outs_b, n_graphs=len(A["graphs"]),
+                capture_t=capture_t, buf_class=cls, n_perm=plan.n_perm, blob_bytes=plan.blob_bytes,
+                perm=plan.perm.cpu().numpy().view(np.uint32).copy(), perm_off=plan.perm_off.cpu().numpy().copy(),
+                buf_report=[int(x) for x in medusa.report_numpy(rep_save)] + [int(x) for x in medusa.report_numpy(rep_buf)],
+                outs_unrestored=outs_unrestored, magic_allocs=[_alloc_of(allocs, m.data_ptr()) for m in A["magic"]],
                 n_nodes=len(recs),
                 n_kernel=n_kernel, n_other=sum(1 for r in recs if r["kind"] == "other"), kernel_names=names)
 
@@ -436,13 +480,20 @@ def offline(torch, medusa, out_dir, seed=0):
 
     A = capture(torch, seed=seed)
     recs = parameter_image(cu, A["nodes"])
-    words, off, node_t, allocs, used = trace_arrays(A["events"], recs)
+    words, off, node_t, allocs, used, capture_t = trace_arrays(A["events"], recs)
     if any(r["kind"] != "kernel" for r in used):
         raise RuntimeError("offline/online demo handles kernel nodes only")
     dev = torch.device("cuda")
     t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(dev)
     aa = np.ascontiguousarray(allocs).view(np.int64).reshape(-1, 3)
-    slots = medusa.materialize(t(words, np.int64), t(off, np.int64), t(node_t, np.int32), torch.from_numpy(aa).to(dev))
+    d_allocs = torch.from_numpy(aa).to(dev)
+    slots = medusa.materialize(t(words, np.int64), t(off, np.int64), t(node_t, np.int32), d_allocs)
+    # the permanent buffers' contents (§4.3): classified and dumped offline
+    plan = medusa.buffers_plan(d_allocs, t(capture_t, np.int32), slots.slot, slots.n_slots)
+    blob, rep_save = medusa.buffers_save(plan, t(allocs["base"], np.int64))
+    torch.cuda.synchronize()
+    if int(medusa.report_numpy(rep_save)[0]):
+        raise RuntimeError("medusa_buffers_save reported segments it could not copy")
     names, func_id, meta = [], [], []
     for r in used:
         nm = _kernel_name(cu, r["params"])
@@ -463,10 +514,13 @@ def offline(torch, medusa, out_dir, seed=0):
     np.savez(os.path.join(out_dir, "image.npz"), words=words, off=off, node_t=node_t, allocs=aa,
              mask=slots.mask.cpu().numpy(), chunk_base=slots.chunk_base.cpu().numpy(),
              slot=slots.slot[: slots.n_slots].cpu().numpy(), func_id=np.array(func_id, np.uint32),
-             events=A["events"])
+             events=A["events"], buf_perm=plan.perm.cpu().numpy(), buf_perm_off=plan.perm_off.cpu().numpy(),
+             buf_blob=blob[: plan.blob_bytes].cpu().numpy())
     json.dump(dict(names=names, meta=meta, outs=outs, n_slots=slots.n_slots, graphs=len(A["graphs"]),
-                   load_events=first_capture, seed=seed), open(os.path.join(out_dir, "meta.json"), "w"))
-    return dict(nodes=len(used), names=len(names), slots=slots.n_slots)
+                   load_events=first_capture, seed=seed, n_perm=plan.n_perm, blob_bytes=plan.blob_bytes),
+              open(os.path.join(out_dir, "meta.json"), "w"))
+    return dict(nodes=len(used), names=len(names), slots=slots.n_slots, n_perm=plan.n_perm,
+                blob_bytes=plan.blob_bytes)
 
 
 def _dlsym_kernels(torch, names):
@@ -625,10 +679,18 @@ def online(torch, medusa, in_dir, arena_bytes=1 << 30):
     medusa.kernel_table_set(t(table, np.int64))
     dst, fout, rep = medusa.restore(t(z["words"], np.int64), slots, t(allocs[:, 0], np.int64),
                                     t(new_base, np.int64), t(allocs[:, 1], np.int64), t(z["func_id"], np.int32))
+    # the permanent buffers' saved contents into the replayed allocations (§4.3)
+    blob = torch.from_numpy(z["buf_blob"]).to(dev)
+    if blob.numel() < 16:
+        blob = torch.zeros(16, dtype=torch.uint8, device=dev)
+    bplan = medusa.BufferPlan(None, t(z["buf_perm"], np.int32), t(z["buf_perm_off"], np.int64), int(meta["n_perm"]),
+                              int(meta["blob_bytes"]))
+    rep_buf = medusa.buffers_restore(bplan, blob, t(new_base, np.int64), t(allocs[:, 1], np.int64))
     torch.cuda.synchronize()
     restored = medusa.to_numpy_u64(dst)
     func_out = medusa.to_numpy_u64(fout)
     report = medusa.report_numpy(rep)
+    buf_report = [int(x) for x in medusa.report_numpy(rep_buf)]
     if kstats["unresolved"] or int(report[5]):
         missing = [nm for nm in meta["names"] if nm not in found]
         return dict(same_loading=same_loading, kernels=kstats, report=[int(x) for x in report],
@@ -678,4 +740,5 @@ def online(torch, medusa, in_dir, arena_bytes=1 << 30):
     moved_bases = int(np.sum(new_base != allocs[:, 0]))
     return dict(same_loading=same_loading, kernels=kstats, report=[int(x) for x in report], outputs_equal=equal,
                 nodes=len(meta["meta"]), allocations=int(len(new_base)), moved_bases=moved_bases,
-                slots=int(meta["n_slots"]))
+                slots=int(meta["n_slots"]), n_perm=int(meta["n_perm"]), blob_bytes=int(meta["blob_bytes"]),
+                buf_report=buf_report)
