@@ -105,6 +105,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     const uint32_t task = blockIdx.x;
     unsigned long long* rep = reinterpret_cast<unsigned long long*>(a.report);
     const unsigned long long tl0 = TL_NOW();
+    unsigned long long tl_p = tl0;
 
     if (task < n_word_tasks) {
         const uint64_t ws = (uint64_t)task * kWords;
@@ -129,25 +130,30 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             }
         }
         // 1. the CTA's words: one bulk copy per chunk into shared memory (all issued
-        //    at once); meanwhile the mask words and the record range
-        if (tid == 0 && tma) {
+        //    at once); meanwhile the mask words and the record range.  (Issuing the
+        //    copies after those small loads measured the same: their ~3 us is not
+        //    queueing behind the bulk reads.)
+        auto issue_tma = [&]() {
+            if (tid == 0 && tma) {
 #pragma unroll
-            for (int c = 0; c < CPB; ++c) {
-                const uint32_t mb = smem_u32(&s_mbar[c]);
-                asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
-            }
-            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+                for (int c = 0; c < CPB; ++c) {
+                    const uint32_t mb = smem_u32(&s_mbar[c]);
+                    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+                }
+                asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 #pragma unroll
-            for (int c = 0; c < CPB; ++c) {
-                const uint32_t q0 = c * kTaskWords;
-                if (q0 >= n) break;
-                const uint32_t nc = min(n - q0, kTaskWords);
-                const uint32_t mb = smem_u32(&s_mbar[c]);
-                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(nc * 8) : "memory");
-                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                             ::"r"(smem_u32(s_words + q0)), "l"(gsrc + q0), "r"(nc * 8), "r"(mb) : "memory");
+                for (int c = 0; c < CPB; ++c) {
+                    const uint32_t q0 = c * kTaskWords;
+                    if (q0 >= n) break;
+                    const uint32_t nc = min(n - q0, kTaskWords);
+                    const uint32_t mb = smem_u32(&s_mbar[c]);
+                    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(nc * 8) : "memory");
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                                 ::"r"(smem_u32(s_words + q0)), "l"(gsrc + q0), "r"(nc * 8), "r"(mb) : "memory");
+                }
             }
-        }
+        };
+        issue_tma();
         if (!tma)
             for (uint32_t q = tid; q < n; q += kThreads) s_words[q] = ld_stream(gsrc + q);
         const uint64_t n_mask = (a.n_words + 31) / 32;
@@ -161,6 +167,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             s_nrec = r1 > r0 ? r1 - r0 : 0;
         }
         __syncthreads();
+        TL_PHASE(7, 10, tl_p);  // mask + record range loaded
         // 2. exclusive prefix of the mask popcounts (warp 0; kMask / 32 words per lane)
         if (tid < 32) {
             constexpr int kPer = kMask / 32;
@@ -216,6 +223,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 }
             }
             if (rb == 0) __syncthreads();  // s_pre ready
+            if (rb == 0) TL_PHASE(7, 11, tl_p);  // first records + gathers in
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 if (kind[u] == 3) continue;
@@ -266,6 +274,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             }
         }
         __syncthreads();
+        TL_PHASE(7, 12, tl_p);  // all records applied (incl. waiting for the words)
         // 4. the CTA's words back to HBM
         if (tma) {
             if (tid == 0) {
@@ -284,6 +293,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         } else {
             for (uint32_t q = tid; q < n; q += kThreads) st_stream(gdst + q, s_words[q]);
         }
+        TL_PHASE(7, 13, tl_p);  // bulk store issued and read out of shared memory
         pdl_wait();  // report_init (this launch's PDL predecessor) has run
         pdl_trigger();
         if (n_id | n_rg | n_st) {

@@ -29,7 +29,9 @@ NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan
          (3, 40): " rank:pdl-wait", (3, 41): " rank:staging", (3, 42): " rank:search+red", (3, 43): " rank:ticket",
          (3, 44): " rank:i-entries", (2, 30): " isort:bitonic", (2, 31): " isort:merges",
          (4, 10): " cls:A setup", (4, 11): " cls:B window", (4, 12): " cls:C tw+cand", (4, 13): " cls:D winsearch",
-         (4, 14): " cls:E queue", (4, 15): " cls:F emit"}
+         (4, 14): " cls:E queue", (4, 15): " cls:F emit",
+         (7, 2): "restore/in-place", (7, 10): " res:mask+range", (7, 11): " res:records+gathers",
+         (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store"}
 REC = np.dtype([("t0", "<u8"), ("t1", "<u8"), ("kernel", "<u4"), ("cta", "<u4"), ("sm", "<u4"), ("tag", "<u4")])
 
 
@@ -38,7 +40,9 @@ def main():
     ap.add_argument("--workload", default="all10")
     ap.add_argument("--steps", type=int, default=5)
     args = ap.parse_args()
-    tl_path = g.build_medusa(out=os.path.join(ROOT, "tools", "libmedusa_tl.so"), defines=("MEDUSA_TIMELINE",))
+    extra = tuple(d for d in os.environ.get("MEDUSA_DEFINES", "").split() if d)  # A/B variants
+    tl_path = g.build_medusa(out=os.path.join(ROOT, "tools", "libmedusa_tl" + "".join("_" + d for d in extra) + ".so"),
+                             defines=("MEDUSA_TIMELINE",) + extra)
     import paper_conf_asplos_zengxgcl25_b200 as medusa
     from workloads import CONFIGS, make_graph_set
     medusa._lib = None
