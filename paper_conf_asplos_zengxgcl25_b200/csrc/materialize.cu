@@ -56,7 +56,7 @@ constexpr int kAblk = 32;          // allocation ordinals per overlap-check bloc
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
 constexpr int kSortTile = 1024;    // I keys sorted per CTA before ranking
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
-constexpr int kWinCap = 128;       // mortal-window entries per batch (<= 4 per lane of one warp)
+constexpr int kWinCap = 96;        // mortal-window entries per batch (<= 4 per lane of one warp; 96 keeps 7 classify CTAs per SM)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
 constexpr int kWarps = kThreads / 32;
 constexpr int kIBlk = 32;          // I-list summary block
@@ -1403,7 +1403,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     TL_REC(9, 0, tl0);
 }
 
-__global__ void __launch_bounds__(kThreads, 6) k_classify(P p) {
+__global__ void __launch_bounds__(kThreads, 7) k_classify(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
