@@ -36,7 +36,7 @@ constexpr int kPlanThreads = 256;
 constexpr int kPlanPer = 4;
 constexpr int kTile = kPlanThreads * kPlanPer;  // allocations per plan CTA
 constexpr int kCopyThreads = 256;
-constexpr uint32_t kTaskBytes = 2048;  // blob bytes per warp task (32 lanes x 4 units x 16 B)
+constexpr uint32_t kTaskBytes = 1024;  // blob bytes per warp task (32 lanes x 2 units x 16 B)
 
 struct PlanResult {
     uint32_t bad_capture;
@@ -218,7 +218,7 @@ __global__ void k_buf_init(medusa_buf_report* rep) {
 // is 16-byte aligned moves as one 16-byte load + store (all four loads of a
 // lane are issued before its stores); anything else goes byte by byte.
 template <bool kToBlob>
-__global__ void __launch_bounds__(kCopyThreads, 3)
+__global__ void __launch_bounds__(kCopyThreads, 4)
 k_buf_copy(uint8_t* blob_w, const uint8_t* __restrict__ blob_r, const uint32_t* __restrict__ perm,
            const uint64_t* __restrict__ off, uint32_t n_perm, const uint64_t* __restrict__ base,
            const uint64_t* __restrict__ size, uint32_t n_alloc, medusa_buf_report* rep) {
@@ -231,19 +231,8 @@ k_buf_copy(uint8_t* blob_w, const uint8_t* __restrict__ blob_r, const uint32_t* 
     uint64_t* ws = s_s + wslot;
     uint64_t* we = s_e + wslot;
     uint64_t* wa = s_a + wslot;
-    // 1. validation (R-B4): a segment whose allocation the replay did not make,
-    //    or that is longer than the replayed allocation, is not copied
-    uint32_t n_bad = 0;
-    uint64_t first = ~0ull;
-    for (uint64_t k = gtid; k < n_perm; k += nthreads) {
-        const uint32_t id = perm[k];
-        if (id >= n_alloc || (size && off[k + 1] - off[k] > size[id])) {
-            ++n_bad;
-            first = min(first, k);
-        }
-    }
     if (n_perm > 0) {
-        // 2. the copy: warp w moves the contiguous blob range [w*per, (w+1)*per)
+        // 1. the copy: warp w moves the contiguous blob range [w*per, (w+1)*per)
         //    in batches of 2 KB; its descriptor window slides along the range
         const uint64_t total = __ldg(off + n_perm);
         const uint64_t nwarps = nthreads >> 5;
@@ -272,7 +261,21 @@ k_buf_copy(uint8_t* blob_w, const uint8_t* __restrict__ blob_r, const uint32_t* 
             __syncwarp();
         };
         if (r0 < r1) {
-            uint32_t k = warp_last_le(off, 0, n_perm, r0);
+            // the segment holding r0: one probe of 32 offsets around the index a
+            // uniform segment size predicts (one round when the guess is close, as
+            // for equally sized buffers); else the 32-ary search
+            uint32_t k;
+            {
+                const uint64_t guess = (uint64_t)((double)r0 / (double)total * (double)n_perm);
+                const uint32_t g0 = (uint32_t)min(guess > 8 ? guess - 8 : (uint64_t)0, (uint64_t)(n_perm > 32 ? n_perm - 32 : 0));
+                const uint32_t kk = g0 + lane;
+                const bool le = kk < n_perm && __ldg(off + kk) <= r0;
+                const uint32_t b = __ballot_sync(0xffffffffu, le);
+                // bracketed: off[g0] <= r0 and (the probe ends past r0, or it reaches n_perm)
+                const bool hit_lo = b & 1u;
+                const bool hit_hi = (b != 0xffffffffu) || g0 + 32 >= n_perm;
+                k = (hit_lo && hit_hi) ? g0 + 31 - __clz(b) : warp_last_le(off, 0, n_perm, r0);
+            }
             load_window(k);
             for (uint64_t t0 = r0; t0 < r1; t0 += kTaskBytes) {
                 const uint64_t t1 = min(t0 + kTaskBytes, r1);
@@ -289,25 +292,37 @@ k_buf_copy(uint8_t* blob_w, const uint8_t* __restrict__ blob_r, const uint32_t* 
                             if (ws[j + b] <= q) j += b;  // j + b <= 31
                         return j;
                     };
-                    // fast path: whole unit inside one valid segment, aligned target
+                    // fast path: whole unit inside one valid segment, aligned target.
+                    // The four units' segment searches run interleaved (independent
+                    // shared-memory chains), then all loads are issued, then the stores.
                     uint4 v[kUnits];
                     uint64_t dst_a[kUnits];
                     bool fast[kUnits];
+                    uint32_t jr[kUnits];
+#pragma unroll
+                    for (int r = 0; r < kUnits; ++r) jr[r] = 0;
+#pragma unroll
+                    for (int b = 16; b >= 1; b >>= 1) {
+#pragma unroll
+                        for (int r = 0; r < kUnits; ++r) {
+                            const uint64_t p = t0 + 16ull * (lane + 32 * r);
+                            if (ws[jr[r] + b] <= p) jr[r] += b;  // jr + b <= 31
+                        }
+                    }
 #pragma unroll
                     for (int r = 0; r < kUnits; ++r) {
                         const uint64_t p = t0 + 16ull * (lane + 32 * r);
                         fast[r] = false;
                         if (q_next[r] != p || p >= t1 || p >= w_end) continue;
-                        const uint32_t j = find(p);
+                        const uint32_t j = jr[r];
                         if (p + 16 > we[j]) continue;
                         const uint64_t a = wa[j] + (p - ws[j]);
                         if ((a & 15) != 0) continue;
-                        fast[r] = true;
                         if (!((okm >> j) & 1)) {  // invalid segment: nothing to move
                             q_next[r] = ~0ull;
-                            fast[r] = false;
                             continue;
                         }
+                        fast[r] = true;
                         if (kToBlob) {
                             v[r] = __ldg(reinterpret_cast<const uint4*>(a));
                             dst_a[r] = reinterpret_cast<uint64_t>(blob_w + p);
@@ -344,6 +359,18 @@ k_buf_copy(uint8_t* blob_w, const uint8_t* __restrict__ blob_r, const uint32_t* 
                     load_window(k);
                 }
             }
+        }
+    }
+    // 2. validation (R-B4), counted once per segment: a segment whose allocation
+    //    the replay did not make, or that is longer than the replayed allocation,
+    //    was not copied.  (After the copy: its loads overlap the stores draining.)
+    uint32_t n_bad = 0;
+    uint64_t first = ~0ull;
+    for (uint64_t k = gtid; k < n_perm; k += nthreads) {
+        const uint32_t id = perm[k];
+        if (id >= n_alloc || (size && off[k + 1] - off[k] > size[id])) {
+            ++n_bad;
+            first = min(first, k);
         }
     }
     pdl_wait();  // k_buf_init has initialised the report

@@ -15,7 +15,7 @@ if ip:
     for k, v in ip.items():
         if isinstance(v, dict): print(f"in place {k}: {v['avg_us']:.1f} us {v['GB/s']:.0f} GB/s ({100*v['frac_of_peak']:.1f}%) {v['nodes_per_s']/1e9:.2f} G nodes/s")
 bu = d.get('buffers')
-if bu: print(f"buffers: {bu['n_perm']} perm ({bu['blob_bytes']/1e6:.2f} MB) plan {bu['plan_ms']:.3f} ms save {bu['save_us']:.1f} us restore {bu['restore_us']:.1f} us = {bu['restore_GB/s']:.0f} GB/s ok={bu['restore_ok']} {bu['classes']}\n   kernels {bu.get('kernel_us')} restore kernel {bu.get('restore_kernel_GB/s', 0):.0f} GB/s")
+if bu: print(f"buffers: {bu['n_perm']} perm ({bu['blob_bytes']/1e6:.2f} MB) plan {bu['plan_ms']:.3f} ms save {bu['save_us']:.1f} us restore {bu['restore_us']:.1f} us = {bu['restore_GB/s']:.0f} GB/s ok={bu['restore_ok']} {bu['classes']}\n   kernels {bu.get('kernel_us')} events {bu.get('restore_events_GB/s', 0):.0f} GB/s")
 for k, v in d["kernels"].items():
     print(f"  {k:22s} n={v['launches']:4d} avg {v['avg_us']:8.2f} us  share {100*v['share_of_step']:5.1f}%  " +
           (f"{v['GB/s']:.0f} GB/s" if 'GB/s' in v else ""))
