@@ -172,6 +172,85 @@ def run_reference(args):
     }), flush=True)
 
 
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_all_cores(oracle, gs, seconds):
+    """SURVEY.md §8(d) oracle timing (b): the unchanged oracle on every host core.
+    The node range is split into one contiguous part per thread for MATERIALIZE
+    (each part is a complete sub-problem: a word's class depends only on its node's
+    launch position and the whole trace, which every part receives) and the word
+    range for RESTORE (each part gets its slots, rebased; the kernel-address
+    gather runs with the first part).  Python threads around ctypes calls (the GIL
+    is released inside the oracle).  Returns (nodes/s, materialize nodes/s,
+    restore nodes/s, threads, passes); the parts' outputs are checked against the
+    single-threaded run on the first pass."""
+    import threading
+    P = os.cpu_count() or 1
+    N, W = gs.n_nodes, gs.n_words
+    off = gs.node_word_off.astype(np.int64)
+    jcut = [N * k // P for k in range(P + 1)]
+    wcut = [int(off[j]) for j in jcut]
+
+    def run_parallel(fn):
+        out = [None] * P
+        th = [threading.Thread(target=lambda k=k: out.__setitem__(k, fn(k))) for k in range(P)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        return out
+
+    def mat_part(k):
+        j0, j1 = jcut[k], jcut[k + 1]
+        w0, w1 = wcut[k], wcut[k + 1]
+        m = oracle.materialize(gs.words[w0:w1], (off[j0:j1 + 1] - w0).astype(np.uint64), gs.node_t[j0:j1], gs.allocs)
+        return m["slot_g"] + np.uint64(w0), m["slot_id"], m["slot_off"]
+
+    ref = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+    ref_dst = oracle.restore(gs.words, ref["slot_g"], ref["slot_id"], ref["slot_off"], gs.allocs["base"],
+                             gs.new_base, gs.new_size, gs.func_id, gs.table)[0]
+    t_mat = t_res = 0.0
+    reps = 0
+    t_start = time.perf_counter()
+    while time.perf_counter() - t_start < seconds or reps == 0:
+        t1 = time.perf_counter()
+        parts = run_parallel(mat_part)
+        t2 = time.perf_counter()
+        g = np.concatenate([q[0] for q in parts])
+        sid = np.concatenate([q[1] for q in parts])
+        soff = np.concatenate([q[2] for q in parts])
+        bounds = np.searchsorted(g, np.array(wcut, dtype=np.uint64))
+        dst = np.empty_like(gs.words)
+
+        def res_part(k):
+            w0, w1 = wcut[k], wcut[k + 1]
+            s0, s1 = bounds[k], bounds[k + 1]
+            first = k == 0
+            d, _, _ = oracle.restore(gs.words[w0:w1], g[s0:s1] - np.uint64(w0), sid[s0:s1], soff[s0:s1],
+                                     gs.allocs["base"], gs.new_base, gs.new_size,
+                                     gs.func_id if first else None, gs.table if first else None)
+            dst[w0:w1] = d
+
+        t3 = time.perf_counter()
+        run_parallel(res_part)
+        t4 = time.perf_counter()
+        if reps == 0:
+            assert np.array_equal(g, ref["slot_g"]) and np.array_equal(soff, ref["slot_off"])
+            assert np.array_equal(dst, ref_dst)
+        t_mat += t2 - t1
+        t_res += t4 - t3
+        reps += 1
+    return N * reps / (t_mat + t_res), N * reps / t_mat, N * reps / t_res, P, reps
+
+
 def bench_inplace(medusa, gs, inp, slots, dev, stream, scrub, steps, peak, alg, replicas):
     import torch
     from workloads.graphset import replicate
@@ -620,7 +699,13 @@ def run_ours(args):
                                "materialize": (gs.n_nodes / gpu_mat_s) / (gs.n_nodes * reps / t_mat),
                                "restore": (gs.n_nodes / gpu_res_s) / (gs.n_nodes * reps / t_res)},
                "sample": f"the full per-rank {cfg} set, {reps} passes (materialize + restore), "
-                         f"single-threaded oracle/oracle.cpp; host has {os.cpu_count()} cores"}
+                         f"single-threaded oracle/oracle.cpp; host has {os.cpu_count()} cores ({cpu_model()})"}
+        v, vm, vr, thr, preps = oracle_all_cores(oracle, gs, args.cpu_seconds / 2)
+        cpu["all_cores"] = {"value": v, "unit": "nodes/s", "cores": thr, "materialize_nodes_per_s": vm,
+                            "restore_nodes_per_s": vr, "gpu_speedup_whole_path": value / v,
+                            "sample": f"the same set, {preps} passes; the unchanged oracle on {thr} threads "
+                                      "(node ranges for materialize, word ranges for restore; outputs equal "
+                                      "the single-threaded run); time of the split / merge in numpy excluded"}
 
     if rank == 0:
         line = {

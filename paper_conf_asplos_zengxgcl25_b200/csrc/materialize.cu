@@ -796,13 +796,16 @@ __global__ void __launch_bounds__(kThreads, 6) k_prepare(P p) {
     } U;
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
+    // early trigger: k_classify's CTAs take the free slots and do their setup
+    // (inputs and k_trace's outputs only) while this grid runs; they wait for its
+    // completion before reading the registration lists
+    pdl_trigger();
     if (blockIdx.x < p.sort_ctas) {
         sort_role(p, blockIdx.x, U.sort);
     } else {
         scatter_role(p, blockIdx.x - p.sort_ctas, U.scatter);
         TL_REC(2, 1, tl0);
     }
-    pdl_trigger();
 }
 
 // ----------------------------------------------------------------------------
@@ -1138,21 +1141,15 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);  // (synchronizes the CTA)
     const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
     TL_PHASE(4, 10, tl_p);  // A: setup
-    // B. one round of loads: threads 0..127 the first window batch, threads
-    //    128..255 the starts of the chunk's nodes (-> start bitmask)
-    const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
+    // B. the starts of the chunk's nodes (-> start bitmask, its popcount prefix,
+    //    the launch positions of the first kNodeGrp segments)
     uint32_t my_q = 0xFFFFFFFFu, my_t = 0;  // this thread's first node (start, launch position)
-    if (tid < kWinCap) {
-        window_load(p, S, r0, m0);
-    } else {
-        for (uint32_t j = jf + 1 + (tid - kWinCap); j <= jl; j += kThreads - kWinCap) {
-            const uint32_t q = (uint32_t)(a.node_off[j] - cs);
-            if (my_q == 0xFFFFFFFFu) { my_q = q; my_t = a.node_t[j]; }
-            atomicOr(&S.nsm[q >> 5], 1u << (q & 31));
-        }
+    for (uint32_t j = jf + 1 + tid; j <= jl; j += kThreads) {
+        const uint32_t q = (uint32_t)(a.node_off[j] - cs);
+        if (my_q == 0xFFFFFFFFu) { my_q = q; my_t = a.node_t[j]; }
+        atomicOr(&S.nsm[q >> 5], 1u << (q & 31));
     }
     __syncthreads();
-    if (warp == 0 && m0) window_sort(S, m0);
     if (warp == 1) {  // exclusive popcount prefix of the 64 start-mask words
         const uint32_t c0 = __popc(S.nsm[2 * lane]), c1 = __popc(S.nsm[2 * lane + 1]);
         uint32_t incl = c0 + c1;
@@ -1173,15 +1170,14 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         const uint32_t sg = seg_of(S, my_q);
         if (sg < kNodeGrp) atomicMax(&S.nt0[sg], my_t);
     }
-    if (nn > (uint32_t)(kThreads - kWinCap) + 1) {  // more nodes than threads 128..255: the rest
-        for (uint32_t j = jf + 1 + (kThreads - kWinCap) + tid; j <= jl; j += kThreads) {
+    if (nn > (uint32_t)kThreads + 1) {  // more nodes than threads: the rest
+        for (uint32_t j = jf + 1 + kThreads + tid; j <= jl; j += kThreads) {
             const uint32_t sg = seg_of(S, (uint32_t)(a.node_off[j] - cs));
             if (sg < kNodeGrp) atomicMax(&S.nt0[sg], a.node_t[j]);
         }
     }
-    __syncthreads();
-    TL_PHASE(4, 11, tl_p);  // B: window records, node starts, sort
-    if (m0) build_live(S, S.nt0, ng0, m0);
+    // C. this warp's words: candidates (inside [least base, greatest end) of the
+    //    trace) compacted into the warp's list
     if (tma) {
         uint32_t done = 0;
         while (!done) {
@@ -1189,11 +1185,6 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                          : "=r"(done) : "r"(mb) : "memory");
         }
     }
-    TL_PHASE(4, 12, tl_p);  // C: live masks, TMA wait
-    // D. this warp's words: candidates (inside [least base, greatest end) of the
-    //    trace) compacted into the warp's list; per candidate its segment (O(1) from
-    //    the start bitmask) and the window lookup at node group 0 / batch 0
-    const bool more_batches = r1 - r0 > (uint64_t)kWinCap;
     uint16_t* wl = S.cq + warp * 256;   // this warp's candidates (word in chunk)
     uint32_t* wh = S.hits + warp * 8;   // hit bits of the warp's 256 words
     uint32_t nc = 0;
@@ -1206,7 +1197,22 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         nc += __popc(b);
     }
     if (lane < 8) wh[lane] = 0;
-    __syncwarp();
+    TL_PHASE(4, 11, tl_p);  // B/C: node starts, TMA wait, candidates
+    // Everything above reads only the inputs and k_trace's outputs (two launches
+    // back): it overlaps k_prepare's tail.  The registration lists are k_prepare's.
+    pdl_wait();
+    // D. the first window batch: loaded, sorted by (base, t_alloc) in warp 0's
+    //    registers, live masks of the first node group
+    const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
+    if (tid < kWinCap) window_load(p, S, r0, m0);
+    __syncthreads();
+    if (warp == 0 && m0) window_sort(S, m0);
+    __syncthreads();
+    if (m0) build_live(S, S.nt0, ng0, m0);
+    TL_PHASE(4, 12, tl_p);  // D: window, sort, live masks
+    // E. per candidate its segment (O(1) from the start bitmask) and the window
+    //    lookup at node group 0 / batch 0
+    const bool more_batches = r1 - r0 > (uint64_t)kWinCap;
     bool deferred = false;
     for (uint32_t i = lane; i < nc; i += 32) {
         const uint32_t q = wl[i];
@@ -1406,8 +1412,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
 __global__ void __launch_bounds__(kThreads, 7) k_classify(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const unsigned long long tl0 = TL_NOW();
-    pdl_wait();
-    classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));
+    classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));  // (waits for k_prepare inside)
     TL_REC(4, 0, tl0);
 }
 
