@@ -1477,50 +1477,64 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
 
 // ----------------------------------------------------------------------------
 // 5. k_emit: compaction of the staged records into the slot table (one CTA per
-//    chunk, one thread per output record: coalesced stores)
+//    kEmitChunks chunks, one thread per output record: coalesced stores)
+constexpr int kEmitChunks = 2;  // chunks per k_emit CTA (the grid fits one wave)
+
 __global__ void __launch_bounds__(kThreads) k_emit(P p) {
-    __shared__ uint32_t s_pre[65], s_m[64];
+    __shared__ uint32_t s_pre[kEmitChunks][65], s_m[kEmitChunks][64];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t c = blockIdx.x;
+    const uint32_t c0 = blockIdx.x * kEmitChunks;
+    const uint32_t nch = min((uint32_t)kEmitChunks, p.C - c0);
     const uint64_t n_mask = (a.n_words + 31) / 32;
-    const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
-    // this chunk's first slot: the sum of the slot counts of all earlier chunks
-    const uint64_t prefix = block_prefix(p.d.chunk_cnt, p.d.chunk_sup, c);
-    const uint32_t total = __ldcg(p.d.chunk_cnt + c);
-    if (tid == 0) {
-        a.chunk_base[c] = (uint32_t)prefix;
-        if (c + 1 == p.C) {
-            a.chunk_base[c + 1] = (uint32_t)(prefix + total);
-            p.d.ctl->n_slots = prefix + total;
-        }
-    }
-    if (warp < 2) {
-        const uint64_t mw = m0 + warp * 32 + lane;
-        const uint32_t mv = mw < n_mask ? __ldcg(a.mask + mw) : 0u;
+    // the first chunk's first slot: the sum of the slot counts of all earlier chunks
+    uint64_t prefix = block_prefix(p.d.chunk_cnt, p.d.chunk_sup, c0);
+    uint32_t total[kEmitChunks];
+#pragma unroll
+    for (int h = 0; h < kEmitChunks; ++h) total[h] = (uint32_t)h < nch ? __ldcg(p.d.chunk_cnt + c0 + h) : 0u;
+    if (warp < 2 * kEmitChunks) {  // popcount prefix of each half of each chunk's 64 mask words
+        const uint32_t h = warp >> 1, half = warp & 1;
+        const uint64_t mw = (uint64_t)(c0 + h) * (kChunkWords / 32) + half * 32 + lane;
+        const uint32_t mv = (h < nch && mw < n_mask) ? __ldcg(a.mask + mw) : 0u;
         const uint32_t pc = __popc(mv);
-        s_m[warp * 32 + lane] = mv;
+        s_m[h][half * 32 + lane] = mv;
         uint32_t incl = pc;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
             const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
             if (lane >= d) incl += y;
         }
-        s_pre[warp * 32 + lane] = incl - pc;
-        if (warp == 0 && lane == 31) s_pre[64] = incl;  // first-half total
+        s_pre[h][half * 32 + lane] = incl - pc;
+        if (half == 0 && lane == 31) s_pre[h][64] = incl;  // first-half total
     }
     __syncthreads();
-    const uint32_t half0 = s_pre[64];
-    if (tid >= 32 && tid < 64) s_pre[tid] += half0;  // second half after the first
+    if (tid >= 32 && tid < 64) {
+#pragma unroll
+        for (int h = 0; h < kEmitChunks; ++h) s_pre[h][tid] += s_pre[h][64];  // second half after the first
+    }
     __syncthreads();
-    for (uint32_t r = tid; r < total; r += kThreads) {
-        uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
-        while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
-        const uint64_t dst = prefix + r;
-        const uint32_t bit = __fns(s_m[lo], 0, (int)(r - s_pre[lo]) + 1);  // the (r - s_pre[lo])-th set bit
-        if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + bit];
+#pragma unroll
+    for (int h = 0; h < kEmitChunks; ++h) {
+        if ((uint32_t)h >= nch) break;
+        const uint32_t c = c0 + h;
+        const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
+        if (tid == 0) {
+            a.chunk_base[c] = (uint32_t)prefix;
+            if (c + 1 == p.C) {
+                a.chunk_base[c + 1] = (uint32_t)(prefix + total[h]);
+                p.d.ctl->n_slots = prefix + total[h];
+            }
+        }
+        for (uint32_t r = tid; r < total[h]; r += kThreads) {
+            uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
+            while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
+            const uint64_t dst = prefix + r;
+            const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);  // the (r - s_pre[lo])-th set bit
+            if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + bit];
+        }
+        prefix += total[h];
     }
     pdl_trigger();
     TL_REC(5, 0, tl0);
@@ -1634,7 +1648,7 @@ Scratch* device_scratch(cudaError_t* e) {
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
-            (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
+            (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_lo)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.ranked, cudaEventDisableTiming)) != cudaSuccess ||
@@ -1698,10 +1712,10 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if (C) {
             {
                 TimedLaunch tl("mat_iresolve", side);
-                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 8), kThreads, 0, side>>>(p);
+                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
             }
             TimedLaunch tl("mat_emit", side);
-            if ((e = launch_pdl(k_emit, C, kThreads, 0, side, p))) return e;
+            if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
         }
         if ((e = cudaEventRecord(s.emitted, side))) return e;
         // default priority: the trace checks fill in around them
@@ -1718,7 +1732,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
         }
         TimedLaunch tl("mat_emit", stream);
-        if ((e = launch_pdl(k_emit, C, kThreads, 0, stream, p))) return e;
+        if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
     }
     return cudaGetLastError();
 }
