@@ -24,10 +24,17 @@ def main():
     ap.add_argument("--reps", type=int, default=30)
     ap.add_argument("--replicas", type=int, default=32)
     ap.add_argument("--inplace", action="store_true", help="variants of the in-place kernel (MEDUSA_RESTORE_CPB_IP)")
+    ap.add_argument("--defines", nargs="+", help="variants given as preprocessor defines (e.g. MEDUSA_RESTORE_EARLY=0)")
     args = ap.parse_args()
-    libs = {c: g.build_medusa(out=os.path.join(ROOT, "tools", f"libmedusa_cpb{c}.so"),
-                              defines=(f"MEDUSA_RESTORE_CPB{'_IP' if args.inplace else ''}={c}",))
-            for c in args.cpb}
+    if args.defines:
+        names = args.defines
+        libs = {d: g.build_medusa(out=os.path.join(ROOT, "tools", f"libmedusa_{d.replace('=', '_')}.so"), defines=(d,))
+                for d in names}
+    else:
+        names = args.cpb
+        libs = {c: g.build_medusa(out=os.path.join(ROOT, "tools", f"libmedusa_cpb{c}.so"),
+                                  defines=(f"MEDUSA_RESTORE_CPB{'_IP' if args.inplace else ''}={c}",))
+                for c in args.cpb}
     import paper_conf_asplos_zengxgcl25_b200 as medusa
     from bench import algorithmic_bytes
     from workloads import make_graph_set
@@ -42,12 +49,12 @@ def main():
         sets.append((x, inp, sl, algorithmic_bytes(x, sl.n_slots, x.table.size)["restore"]))
     scrub = torch.empty(256 << 20 >> 2, dtype=torch.int32, device=dev)
     ref = None
-    for c in args.cpb:
+    for c in names:
         path = libs[c]
         medusa._lib = None
         medusa.LIB_PATH = path
         medusa.lib()
-        line = [f"CPB{'_IP' if args.inplace else ''}={c}"]
+        line = [c if args.defines else f"CPB{'_IP' if args.inplace else ''}={c}"]
         for si, (x, inp, sl, alg) in enumerate(sets):
             medusa.kernel_table_set(inp["table"])
             dst = inp["words"].clone() if args.inplace else torch.empty_like(inp["words"])
@@ -78,7 +85,7 @@ def main():
                 h = (dst.cpu().numpy().copy(), fout.cpu().numpy().copy())
                 if ref is None:
                     ref = h
-                assert np.array_equal(h[0], ref[0]) and np.array_equal(h[1], ref[1]), f"CPB={c} output differs"
+                assert np.array_equal(h[0], ref[0]) and np.array_equal(h[1], ref[1]), f"{c}: output differs"
             line.append(f"{'all10' if si == 0 else 'x%d' % args.replicas}: {t * 1e6:8.1f} us "
                         f"{alg / t / 1e9:6.0f} GB/s")
         print("  ".join(line), flush=True)
