@@ -20,7 +20,6 @@ import argparse
 import json
 import os
 import statistics
-import subprocess
 import sys
 import time
 
@@ -70,49 +69,64 @@ def load_traffic():
 
 
 class ClockSampler:
-    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clock and throttle reasons sampled DURING the timed region: an NVML
+    polling thread (~0.5 ms period; nvidia-smi's 50 ms loop cannot land inside a
+    ~6 ms region), samples kept between mark_start() and mark_end() (host times
+    taken right after the barriers + synchronizes that bracket the region)."""
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4), ("hw_power_brake_slowdown", 0x80))
 
     def __init__(self, gpu_index):
-        self.proc = None
+        import threading
+        self.rows, self.t0, self.t1, self.max_mhz = [], None, None, 0.0
+        self.stop_ev = threading.Event()
+        self.thread = None
         try:
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "50",
-                 "-i", str(gpu_index)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            import pynvml
+            pynvml.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            idx = int(vis.split(",")[gpu_index]) if vis and vis.split(",")[gpu_index].isdigit() else gpu_index
+            h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.max_mhz = float(pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM))
+
+            def poll():
+                while not self.stop_ev.is_set():
+                    try:
+                        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+                        rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                        self.rows.append((time.perf_counter(), float(sm), int(rs)))
+                    except Exception:
+                        pass
+                    time.sleep(0.0005)
+
+            self.thread = threading.Thread(target=poll, daemon=True)
+            self.switch = sys.getswitchinterval()
+            sys.setswitchinterval(0.0002)  # let the poller in while the main thread enqueues
+            self.thread.start()
         except Exception:
-            self.proc = None
+            self.thread = None
+
+    def mark_start(self):
+        self.t0 = time.perf_counter()
+
+    def mark_end(self):
+        self.t1 = time.perf_counter()
 
     def stop(self):
-        if self.proc is None:
+        if self.thread is None:
             return None
-        self.proc.terminate()
-        try:
-            out, _ = self.proc.communicate(timeout=5)
-        except Exception:
-            self.proc.kill()
-            out, _ = self.proc.communicate()
-        rows = []
-        for line in out.strip().splitlines():
-            f = [x.strip() for x in line.split(",")]
-            if len(f) < 9:
-                continue
-            try:
-                rows.append(dict(sm=float(f[1]), max=float(f[2]), power=float(f[3]) if f[3] not in ("[N/A]", "") else 0.0,
-                                 hw=f[5], hwt=f[6], swt=f[7], pcap=f[8]))
-            except ValueError:
-                continue
+        self.stop_ev.set()
+        self.thread.join(timeout=5)
+        sys.setswitchinterval(self.switch)
+        rows = [r for r in self.rows if self.t0 is not None and self.t1 is not None and self.t0 <= r[0] <= self.t1]
         if not rows:
+            print(f"clock sampler: {len(self.rows)} samples, none inside the timed region", file=sys.stderr)
             return None
-        loaded = [r for r in rows if r["sm"] > 0.5 * r["max"]] or rows
-        reasons = set()
-        for r in rows:
-            for k, nm in (("hw", "hw_slowdown"), ("hwt", "hw_thermal_slowdown"), ("swt", "sw_thermal_slowdown"),
-                          ("pcap", "sw_power_cap")):
-                if r[k].lower().startswith("active"):
-                    reasons.add(nm)
-        return {"sm_mhz": statistics.median(r["sm"] for r in loaded), "sm_max_mhz": max(r["max"] for r in rows),
-                "reasons": sorted(reasons), "samples": len(rows), "samples_under_load": len(loaded)}
+        loaded = [r for r in rows if r[1] > 0.5 * self.max_mhz] or rows
+        reasons = sorted({nm for r in rows for nm, bit in self.REASONS if r[2] & bit})
+        return {"sm_mhz": statistics.median(r[1] for r in loaded), "sm_max_mhz": self.max_mhz, "reasons": reasons,
+                "samples": len(rows), "samples_under_load": len(loaded),
+                "source": "NVML polled every ~0.5 ms inside the headline timed region"}
 
 
 def rank_seed(cfg, rank):
@@ -463,7 +477,9 @@ def run_ours(args):
         barrier()
         return [a.elapsed_time(b) for a, b in ev]
 
+    sampler.mark_start()
     step_ms = timed(graph.replay)  # the headline
+    sampler.mark_end()
     st_, ns_ = medusa.mat_result(res)
     assert st_ == 0 and ns_ == n_slots, (st_, ns_)
     assert int(medusa.report_numpy(grep)[0]) == 0 and torch.equal(gdst, dst) and torch.equal(gfout, fout)

@@ -1409,7 +1409,10 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     TL_REC(9, 0, tl0);
 }
 
-__global__ void __launch_bounds__(kThreads, 7) k_classify(P p) {
+#ifndef MEDUSA_CLS_MINB
+#define MEDUSA_CLS_MINB 7  // classify CTAs per SM (shared memory allows 7)
+#endif
+__global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const unsigned long long tl0 = TL_NOW();
     classify_role(p, blockIdx.x, *reinterpret_cast<ClsShared*>(smem_raw));  // (waits for k_prepare inside)
