@@ -69,64 +69,50 @@ def load_traffic():
 
 
 class ClockSampler:
-    """SM clock and throttle reasons sampled DURING the timed region: an NVML
-    polling thread (~0.5 ms period; nvidia-smi's 50 ms loop cannot land inside a
-    ~6 ms region), samples kept between mark_start() and mark_end() (host times
-    taken right after the barriers + synchronizes that bracket the region)."""
+    """SM clock and throttle reasons sampled DURING the timed region: after the
+    K steps are enqueued, the host polls NVML until the last step's end event
+    has fired (nvidia-smi's 50 ms loop cannot land inside a ~6 ms region)."""
     REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
                ("sw_power_cap", 0x4), ("hw_power_brake_slowdown", 0x80))
 
     def __init__(self, gpu_index):
-        import threading
-        self.rows, self.t0, self.t1, self.max_mhz = [], None, None, 0.0
-        self.stop_ev = threading.Event()
-        self.thread = None
+        self.rows, self.h, self.max_mhz = [], None, 0.0
         try:
             import pynvml
             pynvml.nvmlInit()
             vis = os.environ.get("CUDA_VISIBLE_DEVICES")
-            idx = int(vis.split(",")[gpu_index]) if vis and vis.split(",")[gpu_index].isdigit() else gpu_index
-            h = pynvml.nvmlDeviceGetHandleByIndex(idx)
-            self.max_mhz = float(pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM))
-
-            def poll():
-                while not self.stop_ev.is_set():
-                    try:
-                        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-                        rs = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-                        self.rows.append((time.perf_counter(), float(sm), int(rs)))
-                    except Exception:
-                        pass
-                    time.sleep(0.0005)
-
-            self.thread = threading.Thread(target=poll, daemon=True)
-            self.switch = sys.getswitchinterval()
-            sys.setswitchinterval(0.0002)  # let the poller in while the main thread enqueues
-            self.thread.start()
+            parts = vis.split(",") if vis else []
+            idx = int(parts[gpu_index]) if gpu_index < len(parts) and parts[gpu_index].isdigit() else gpu_index
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.nvml = pynvml
+            self.max_mhz = float(pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM))
         except Exception:
-            self.thread = None
+            self.h = None
 
-    def mark_start(self):
-        self.t0 = time.perf_counter()
+    def sample(self):
+        if self.h is None:
+            return
+        try:
+            sm = self.nvml.nvmlDeviceGetClockInfo(self.h, self.nvml.NVML_CLOCK_SM)
+            rs = self.nvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            self.rows.append((float(sm), int(rs)))
+        except Exception:
+            pass
 
-    def mark_end(self):
-        self.t1 = time.perf_counter()
+    def poll_until(self, event):
+        """Samples while the GPU is still inside the timed region (event not yet reached)."""
+        while not event.query():
+            self.sample()
 
     def stop(self):
-        if self.thread is None:
-            return None
-        self.stop_ev.set()
-        self.thread.join(timeout=5)
-        sys.setswitchinterval(self.switch)
-        rows = [r for r in self.rows if self.t0 is not None and self.t1 is not None and self.t0 <= r[0] <= self.t1]
+        rows = self.rows
         if not rows:
-            print(f"clock sampler: {len(self.rows)} samples, none inside the timed region", file=sys.stderr)
             return None
-        loaded = [r for r in rows if r[1] > 0.5 * self.max_mhz] or rows
-        reasons = sorted({nm for r in rows for nm, bit in self.REASONS if r[2] & bit})
-        return {"sm_mhz": statistics.median(r[1] for r in loaded), "sm_max_mhz": self.max_mhz, "reasons": reasons,
+        loaded = [r for r in rows if r[0] > 0.5 * self.max_mhz] or rows
+        reasons = sorted({nm for r in rows for nm, bit in self.REASONS if r[1] & bit})
+        return {"sm_mhz": statistics.median(r[0] for r in loaded), "sm_max_mhz": self.max_mhz, "reasons": reasons,
                 "samples": len(rows), "samples_under_load": len(loaded),
-                "source": "NVML polled every ~0.5 ms inside the headline timed region"}
+                "source": "NVML, polled by the host between enqueueing the K timed steps and the last step's end event"}
 
 
 def rank_seed(cfg, rank):
@@ -466,7 +452,7 @@ def run_ours(args):
     for i in range(20):  # bring clocks up before the timed steps
         scrub.fill_(i)
 
-    def timed(fn):
+    def timed(fn, sampler=None):
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
         barrier()
         for k in range(args.steps):
@@ -474,12 +460,13 @@ def run_ours(args):
             ev[k][0].record(stream)
             fn()
             ev[k][1].record(stream)
+        if sampler is not None:
+            sampler.poll_until(ev[-1][1])
         barrier()
         return [a.elapsed_time(b) for a, b in ev]
 
-    sampler.mark_start()
-    step_ms = timed(graph.replay)  # the headline
-    sampler.mark_end()
+    step_ms = timed(graph.replay, sampler)  # the headline
+    clocks = sampler.stop()
     st_, ns_ = medusa.mat_result(res)
     assert st_ == 0 and ns_ == n_slots, (st_, ns_)
     assert int(medusa.report_numpy(grep)[0]) == 0 and torch.equal(gdst, dst) and torch.equal(gfout, fout)
@@ -501,7 +488,6 @@ def run_ours(args):
     inst_ms = timed(step_queued)
     launches = medusa.timing_read(1 << 20)
     medusa.timing_enable(False)
-    clocks = sampler.stop()
     total_ms = sum(step_ms)
     max_ms = max_over_ranks(total_ms, dist, dev)
     nodes_total = gs.n_nodes * args.steps * ws
