@@ -618,7 +618,7 @@ def run_ours(args):
     # still copies its full inputs in and its full results out.
     s_in, s_cp, s_out = torch.cuda.Stream(dev), torch.cuda.Stream(dev), torch.cuda.Stream(dev)
     sets = []
-    for _ in range(2):
+    for _ in range(args.e2e_sets):
         sets.append(dict(
             d_in={k: torch.empty_like(v, device=dev) for k, v in pinned.items()},
             slots=medusa.alloc_slots(gs.n_words, dev), res=torch.zeros(2, dtype=torch.int64, device=dev),
@@ -633,16 +633,16 @@ def run_ours(args):
 
     def e2e_pipelined(n):
         for k in range(n):
-            S = sets[k % 2]
+            S = sets[k % len(sets)]
             with torch.cuda.stream(s_in):
-                if k >= 2:
+                if k >= len(sets):
                     s_in.wait_event(S["ev_cp"])  # the set's inputs are no longer read
                 for name, v in pinned.items():
                     S["d_in"][name].copy_(v, non_blocking=True)
                 S["ev_in"].record(s_in)
             with torch.cuda.stream(s_cp):
                 s_cp.wait_event(S["ev_in"])
-                if k >= 2:
+                if k >= len(sets):
                     s_cp.wait_event(S["ev_out"])  # the set's outputs have been read back
                 d = S["d_in"]
                 medusa.kernel_table_set(d["table"], stream=s_cp)
@@ -663,12 +663,16 @@ def run_ours(args):
     barrier()
     pa, pb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     pa.record(s_in)
+    t_host = time.perf_counter()
     e2e_pipelined(args.steps)
+    t_host = time.perf_counter() - t_host
     for S in sets:
         s_out.wait_event(S["ev_out"])
     pb.record(s_out)
     barrier()
     e2e_ms = pa.elapsed_time(pb)
+    print(f"e2e pipelined: {args.e2e_sets} buffer sets, host enqueue {1e3 * t_host / args.steps:.3f} ms/step, "
+          f"device {e2e_ms / args.steps:.3f} ms/step", file=sys.stderr)
     for S in sets:  # every set's last step: status, slot count, restored words, handles, report
         assert int(S["res_h"][0].item()) & 0xFFFFFFFF == 0 and int(S["res_h"][1].item()) == n_slots
         assert torch.equal(S["out_h"], out_h) and torch.equal(S["fout_h"], fout_h)
@@ -761,6 +765,7 @@ def main():
     ap.add_argument("--sustained", type=int, default=32, help="replicas in the sustained-relocate call (0: skip)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-sets", type=int, default=2, help="buffer sets in the pipelined end-to-end leg")
     ap.add_argument("--no-buffers", dest="buffers", action="store_false")
     args = ap.parse_args()
     if args.impl == "reference":

@@ -28,8 +28,8 @@ NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan
          (1, 23): " last:fence", (1, 24): " last:scan-c", (1, 25): " last:scan-b",
          (3, 40): " rank:pdl-wait", (3, 41): " rank:staging", (3, 42): " rank:search+red", (3, 43): " rank:ticket",
          (3, 44): " rank:i-entries", (2, 30): " isort:bitonic", (2, 31): " isort:merges",
-         (4, 10): " cls:A setup", (4, 11): " cls:B window", (4, 12): " cls:C tw+cand", (4, 13): " cls:D winsearch",
-         (4, 14): " cls:E queue", (4, 15): " cls:F emit",
+         (4, 10): " cls:A setup", (4, 11): " cls:B starts+cand", (4, 12): " cls:C live", (4, 13): " cls:D winsearch",
+         (4, 14): " cls:E queue", (4, 15): " cls:pdl-wait", (4, 16): " cls:win-load", (4, 17): " cls:sort",
          (7, 2): "restore/in-place", (7, 10): " res:mask+range", (7, 11): " res:records+gathers",
          (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store"}
 REC = np.dtype([("t0", "<u8"), ("t1", "<u8"), ("kernel", "<u4"), ("cta", "<u4"), ("sm", "<u4"), ("tag", "<u4")])
