@@ -1731,8 +1731,10 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
         {
+            // no k_prepare in between: a plain launch (k_classify reads k_trace's
+            // outputs before its griddepcontrol.wait, which is only safe two launches back)
             TimedLaunch tl("mat_classify", stream);
-            if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
+            k_classify<<<C, kThreads, sizeof(ClsShared), stream>>>(p);
         }
         TimedLaunch tl("mat_emit", stream);
         if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
