@@ -241,6 +241,21 @@ def test_edge_cases():
     assert st == medusa.ERR_TRACE
 
 
+def test_no_allocations_after_a_large_call(graph_sets):
+    """The allocation-free path (no k_prepare between k_trace and k_classify) right
+    after a ten-model call left its chunk / node scratch behind: nothing but
+    constants, no stale node range used."""
+    gs = graph_sets("all10")
+    inp = medusa.upload(gs, DEV)
+    medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    n = gs.n_words // 3  # many chunks and nodes, all constants
+    off = gs.node_word_off[: int(np.searchsorted(gs.node_word_off, n)) + 1].copy()
+    off[-1] = n
+    st, s = _run_tiny(gs.words[:n], off, gs.node_t[: off.size - 1], np.zeros(0, ALLOC_DTYPE))
+    assert st == 0 and s.n_slots == 0
+    assert not _h(s.mask).any() and not _h(s.chunk_base).any()
+
+
 def test_capacity_too_small(graph_sets):
     gs = graph_sets("toy")
     m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
