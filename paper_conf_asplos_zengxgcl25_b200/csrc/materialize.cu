@@ -356,12 +356,13 @@ __device__ void nodes_role(const P& p, uint64_t i) {
     }
 }
 
-constexpr int kTWin = 2048;  // node times / allocation times staged per alloc CTA
+constexpr int kTWinN = 2048;  // node times staged per alloc CTA
+constexpr int kTWinA = 1024;  // allocation times staged per alloc CTA (2048: +1.3 us of k_trace, ALL10)
 constexpr int kNodesPerThread = 4;  // node role of k_trace (keeps its grid inside one wave)
 
 __device__ void allocs_role(const P& p, uint32_t cta) {
-    __shared__ uint32_t s_nt[kTWin];  // node_t[nj0, nj0 + nw)
-    __shared__ uint32_t s_at[kTWin];  // t_alloc of allocations [i0, i0 + na)
+    __shared__ uint32_t s_nt[kTWinN];  // node_t[nj0, nj0 + nw)
+    __shared__ uint32_t s_at[kTWinA];  // t_alloc of allocations [i0, i0 + na)
     __shared__ uint32_t s_nj0;
     const uint32_t i0 = cta * blockDim.x;
     const uint32_t i = i0 + threadIdx.x;
@@ -382,8 +383,8 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     __syncthreads();
     TL_PHASE(1, 20, tl_p);  // record load, node-window start
     const uint32_t nj0 = s_nj0;
-    const uint32_t nw = min((uint32_t)kTWin, N - nj0);
-    const uint32_t na = (uint32_t)min((uint64_t)kTWin, (uint64_t)a.n_alloc - i0);
+    const uint32_t nw = min((uint32_t)kTWinN, N - nj0);
+    const uint32_t na = (uint32_t)min((uint64_t)kTWinA, (uint64_t)a.n_alloc - i0);
     for (uint32_t k = threadIdx.x; k < nw; k += blockDim.x) s_nt[k] = a.node_t[nj0 + k];
     for (uint32_t k = threadIdx.x; k < na; k += blockDim.x) s_at[k] = a.alloc[i0 + k].t_alloc;
     __syncthreads();
