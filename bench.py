@@ -609,25 +609,51 @@ def run_ours(args):
     buf = bench_buffers(medusa, gs, inp, slots, dev, stream, scrub, args.steps, peak) if args.buffers else None
 
     # ---- end to end: pinned host buffers -> H2D -> whole path -> D2H of results ----
+    # A step's inputs are staged in one pinned host buffer (each array at a 256-B
+    # aligned offset) and go up with one copy; its results (restored words, kernel
+    # addresses, report, outcome) sit in one device buffer and come down with one
+    # copy (nine separate input copies cost ~0.13 ms per step: tools/e2e_probe.py).
     h = medusa.host_arrays(gs)
-    pinned = {k: torch.from_numpy(v).pin_memory() for k, v in h.items()}
-    out_h = torch.empty(gs.n_words, dtype=torch.int64).pin_memory()
-    fout_h = torch.empty(gs.n_nodes, dtype=torch.int64).pin_memory()
-    rep_h = torch.empty(8, dtype=torch.int64).pin_memory()
-    d_in = {k: torch.empty_like(v, device=dev) for k, v in pinned.items()}
-    h2d = sum(v.numel() * v.element_size() for v in pinned.values())
-    d2h = out_h.numel() * 8 + fout_h.numel() * 8 + 64
+
+    def layout(specs):
+        lay, off = {}, 0
+        for name, dt, shape in specs:
+            nb = int(np.prod(shape)) * torch.empty(0, dtype=dt).element_size()
+            lay[name] = (off, nb, dt, shape)
+            off = (off + nb + 255) & ~255
+        return lay, off
+
+    def views(buf, lay):
+        return {k: buf[o:o + nb].view(dt).view(shape) for k, (o, nb, dt, shape) in lay.items()}
+
+    in_lay, in_bytes = layout([(k, torch.from_numpy(v).dtype, tuple(v.shape)) for k, v in h.items()])
+    out_lay, out_bytes = layout([("dst", torch.int64, (gs.n_words,)), ("fout", torch.int64, (gs.n_nodes,)),
+                                 ("rep", torch.int64, (8,)), ("res", torch.int64, (2,))])
+    h_in = torch.empty(in_bytes, dtype=torch.uint8).pin_memory()
+    for k, v in views(h_in, in_lay).items():
+        v.copy_(torch.from_numpy(h[k]))
+    h2d, d2h = in_bytes, out_bytes
+
+    def make_set():
+        S = dict(d_in_buf=torch.empty(in_bytes, dtype=torch.uint8, device=dev),
+                 d_out_buf=torch.zeros(out_bytes, dtype=torch.uint8, device=dev),
+                 h_out_buf=torch.empty(out_bytes, dtype=torch.uint8).pin_memory(),
+                 slots=medusa.alloc_slots(gs.n_words, dev),
+                 ev_in=torch.cuda.Event(), ev_cp=torch.cuda.Event(), ev_out=torch.cuda.Event())
+        S["d_in"], S["d_out"], S["h_out"] = views(S["d_in_buf"], in_lay), views(S["d_out_buf"], out_lay), \
+            views(S["h_out_buf"], out_lay)
+        return S
+
+    ser = make_set()
 
     def e2e_step():
-        for k, v in pinned.items():
-            d_in[k].copy_(v, non_blocking=True)
-        medusa.kernel_table_set(d_in["table"])
-        medusa.materialize(d_in["words"], d_in["node_off"], d_in["node_t"], d_in["allocs"], out=slots)
-        medusa.restore(d_in["words"], slots, d_in["old_base"], d_in["new_base"], d_in["new_size"],
-                       d_in["func_id"], dst=dst, func_out=fout, report=rep)
-        out_h.copy_(dst, non_blocking=True)
-        fout_h.copy_(fout, non_blocking=True)
-        rep_h.copy_(rep, non_blocking=True)
+        d, o = ser["d_in"], ser["d_out"]
+        ser["d_in_buf"].copy_(h_in, non_blocking=True)
+        medusa.kernel_table_set(d["table"])
+        medusa.materialize(d["words"], d["node_off"], d["node_t"], d["allocs"], out=ser["slots"])
+        medusa.restore(d["words"], ser["slots"], d["old_base"], d["new_base"], d["new_size"],
+                       d["func_id"], dst=o["dst"], func_out=o["fout"], report=o["rep"])
+        ser["h_out_buf"].copy_(ser["d_out_buf"], non_blocking=True)
 
     for _ in range(2):
         e2e_step()
@@ -639,7 +665,9 @@ def run_ours(args):
         e2e_ev[k][1].record(stream)
     barrier()
     e2e_serial_ms = sum(a.elapsed_time(b) for a, b in e2e_ev)
+    out_h, fout_h = ser["h_out"]["dst"], ser["h_out"]["fout"]
     assert np.array_equal(out_h.numpy().view(np.uint64), medusa.to_numpy_u64(dst))
+    assert int(ser["h_out"]["rep"][0].item()) == 0
 
     # pipelined end to end (the same public API calls, asynchronous variant): step k's
     # inputs go up on a copy stream, its analysis + restore run on the compute stream,
@@ -647,19 +675,7 @@ def run_ours(args):
     # step k+1's upload and step k-1's download overlap step k's kernels.  Every step
     # still copies its full inputs in and its full results out.
     s_in, s_cp, s_out = torch.cuda.Stream(dev), torch.cuda.Stream(dev), torch.cuda.Stream(dev)
-    sets = []
-    for _ in range(args.e2e_sets):
-        sets.append(dict(
-            d_in={k: torch.empty_like(v, device=dev) for k, v in pinned.items()},
-            slots=medusa.alloc_slots(gs.n_words, dev), res=torch.zeros(2, dtype=torch.int64, device=dev),
-            dst=torch.empty(gs.n_words, dtype=torch.int64, device=dev),
-            fout=torch.empty(gs.n_nodes, dtype=torch.int64, device=dev),
-            rep=torch.empty(8, dtype=torch.int64, device=dev),
-            out_h=torch.empty(gs.n_words, dtype=torch.int64).pin_memory(),
-            fout_h=torch.empty(gs.n_nodes, dtype=torch.int64).pin_memory(),
-            rep_h=torch.empty(8, dtype=torch.int64).pin_memory(),
-            res_h=torch.empty(2, dtype=torch.int64).pin_memory(),
-            ev_in=torch.cuda.Event(), ev_cp=torch.cuda.Event(), ev_out=torch.cuda.Event()))
+    sets = [make_set() for _ in range(args.e2e_sets)]
 
     def e2e_pipelined(n):
         for k in range(n):
@@ -667,26 +683,22 @@ def run_ours(args):
             with torch.cuda.stream(s_in):
                 if k >= len(sets):
                     s_in.wait_event(S["ev_cp"])  # the set's inputs are no longer read
-                for name, v in pinned.items():
-                    S["d_in"][name].copy_(v, non_blocking=True)
+                S["d_in_buf"].copy_(h_in, non_blocking=True)
                 S["ev_in"].record(s_in)
             with torch.cuda.stream(s_cp):
                 s_cp.wait_event(S["ev_in"])
                 if k >= len(sets):
                     s_cp.wait_event(S["ev_out"])  # the set's outputs have been read back
-                d = S["d_in"]
+                d, o = S["d_in"], S["d_out"]
                 medusa.kernel_table_set(d["table"], stream=s_cp)
                 medusa.materialize_async(d["words"], d["node_off"], d["node_t"], d["allocs"], out=S["slots"],
-                                         result=S["res"], stream=s_cp)
+                                         result=o["res"], stream=s_cp)
                 medusa.restore(d["words"], S["slots"], d["old_base"], d["new_base"], d["new_size"], d["func_id"],
-                               dst=S["dst"], func_out=S["fout"], report=S["rep"], stream=s_cp, from_table=True)
+                               dst=o["dst"], func_out=o["fout"], report=o["rep"], stream=s_cp, from_table=True)
                 S["ev_cp"].record(s_cp)
             with torch.cuda.stream(s_out):
                 s_out.wait_event(S["ev_cp"])
-                S["out_h"].copy_(S["dst"], non_blocking=True)
-                S["fout_h"].copy_(S["fout"], non_blocking=True)
-                S["rep_h"].copy_(S["rep"], non_blocking=True)
-                S["res_h"].copy_(S["res"], non_blocking=True)
+                S["h_out_buf"].copy_(S["d_out_buf"], non_blocking=True)
                 S["ev_out"].record(s_out)
 
     e2e_pipelined(2)
@@ -704,9 +716,10 @@ def run_ours(args):
     print(f"e2e pipelined: {args.e2e_sets} buffer sets, host enqueue {1e3 * t_host / args.steps:.3f} ms/step, "
           f"device {e2e_ms / args.steps:.3f} ms/step", file=sys.stderr)
     for S in sets:  # every set's last step: status, slot count, restored words, handles, report
-        assert int(S["res_h"][0].item()) & 0xFFFFFFFF == 0 and int(S["res_h"][1].item()) == n_slots
-        assert torch.equal(S["out_h"], out_h) and torch.equal(S["fout_h"], fout_h)
-        assert int(S["rep_h"][0].item()) == 0
+        ho = S["h_out"]
+        assert int(ho["res"][0].item()) & 0xFFFFFFFF == 0 and int(ho["res"][1].item()) == n_slots
+        assert torch.equal(ho["dst"], out_h) and torch.equal(ho["fout"], fout_h)
+        assert int(ho["rep"][0].item()) == 0
     e2e_value = nodes_total / (max_over_ranks(e2e_ms, dist, dev) / 1e3)
     e2e_serial = nodes_total / (max_over_ranks(e2e_serial_ms, dist, dev) / 1e3)
 
@@ -765,8 +778,9 @@ def run_ours(args):
             "paper_context": PAPER_CONTEXT,
             "e2e": {"value": e2e_value, "unit": "nodes/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                     "mode": "pipelined: inputs up (copy stream) / materialize_async + restore (compute stream) / "
-                            "results down (copy stream), two buffer sets; every step copies all its inputs and "
-                            "results; timed from the first upload to the last download",
+                            "results down (copy stream), two buffer sets; every step copies all its inputs (one "
+                            "pinned staging buffer, one H2D copy) and all its results (one device buffer, one D2H "
+                            "copy); timed from the first upload to the last download",
                     "serial_value": e2e_serial,
                     "serial_mode": "one step at a time: H2D, medusa_materialize (host round trip), "
                                    "medusa_restore, D2H, on one stream"},
