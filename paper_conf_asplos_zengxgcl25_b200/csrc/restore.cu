@@ -457,7 +457,16 @@ constexpr int kCPBInPlace = MEDUSA_RESTORE_CPB_IP;  // chunks per restore CTA (i
 
 cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     const bool in_place = a.src == a.dst;
-    const uint64_t cpb = in_place ? kCPBInPlace : kCPB;
+    static int sm_count = 0;
+    if (!sm_count) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sm_count, cudaDevAttrMultiProcessorCount, dev);
+    }
+    // small images (a single model's graph set): one chunk per CTA, so the CTAs
+    // spread over more SMs and each chain of dependent loads is half as long
+    const bool small = (a.n_words + 2ull * kTaskWords - 1) / (2ull * kTaskWords) < (uint64_t)sm_count;
+    const uint64_t cpb = small ? 1 : (in_place ? kCPBInPlace : kCPB);
     const uint32_t n_word_tasks = (uint32_t)((a.n_words + cpb * kTaskWords - 1) / (cpb * kTaskWords));
     const uint32_t n_node_tasks = a.func_id ? (a.n_nodes + kNodesPerTask - 1) / kNodesPerTask : 0;
     const uint32_t n_tasks = n_word_tasks + n_node_tasks;
@@ -469,8 +478,10 @@ cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     if (n_tasks) {
         TimedLaunch tl("restore", stream);
         cudaError_t e = in_place
-            ? launch_pdl(restore_inplace_kernel<kCPBInPlace>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks)
-            : launch_pdl(restore_kernel<kCPB>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks);
+            ? (small ? launch_pdl(restore_inplace_kernel<1>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks)
+                     : launch_pdl(restore_inplace_kernel<kCPBInPlace>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks))
+            : (small ? launch_pdl(restore_kernel<1>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks)
+                     : launch_pdl(restore_kernel<kCPB>, n_tasks, kThreads, 0, stream, a, n_word_tasks, n_tasks));
         if (e != cudaSuccess) return e;
     }
     return cudaGetLastError();
