@@ -8,7 +8,9 @@
 //
 // The pass is HBM-bound: per word it reads 8 B and writes 8 B; the mask adds
 // 1/8 B, each slot record 8 B (about 18% of words are slots).  Design (B200):
-//   * one CTA of 256 threads per 2048-word chunk.  The chunk's 16 KB of words
+//   * one CTA of 256 threads per two consecutive 2048-word chunks (one chunk per
+//     CTA for images under two chunks per SM, e.g. a single model's set, so the
+//     grid still spreads over the SMs).  The chunk's 16 KB of words
 //     move HBM -> shared memory -> HBM with the TMA engine (cp.async.bulk load
 //     completing on an mbarrier, cp.async.bulk store from shared memory), so no
 //     thread holds image words in registers; ~17 KB of shared memory and ~35
