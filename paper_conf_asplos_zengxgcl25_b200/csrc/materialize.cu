@@ -13,10 +13,9 @@
 //  * M = every other allocation ("mortal": capture temporaries, warm-up and
 //    profiling scratch).  A mortal is registered in exactly the word chunks that
 //    hold words of nodes launched during its lifetime; a chunk's window (~60
-//    entries for the ten-model set) is sorted by (base, t_alloc) in registers of
-//    one warp, laid out in shared memory and searched with an upper bound on
-//    (word, launch position), a backward walk while the prefix max of end still
-//    reaches the word, and the time check.
+//    entries for the ten-model set) sits in shared memory in list order with a
+//    per-node live bit mask; a word is looked up among the entries live at its
+//    node (about four in the BASELINE sets) by a range test.
 //  * Well-formedness (no two simultaneously-live allocations overlap) is checked
 //    exactly: I-I by adjacency of the sorted list, M-I with per-32-entry
 //    min(t_alloc) / max(t_free) summaries over the address run a mortal meets,
@@ -941,15 +940,14 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 
 // ----------------------------------------------------------------------------
 // 4. k_classify: one CTA per 2048-word chunk.  The CTA sets up the chunk's
-//    mortal window (registered mortals sorted by base, per-node live masks);
+//    mortal window (registered mortals in list order, per-node live masks);
 //    then each warp classifies its own 256 words with no further CTA barrier:
 //    word q of warp w is q = 256 w + 32 k + lane (k = 0..7).
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     uint64_t rb[kWinCap], re[kWinCap];   // one batch of registered mortals as loaded
     uint32_t rta[kWinCap], rtf[kWinCap], rid[kWinCap];
-    uint64_t wb[kWinCap], we[kWinCap];   // the batch sorted by (base, t_alloc)
-    uint32_t wta[kWinCap], wtf[kWinCap], wid[kWinCap];
+    uint64_t hmin[kWinCap / 32], hmax[kWinCap / 32];  // per loading warp: least base, greatest end
     uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
     // Segments: segment s of the chunk = the words of the s-th distinct node start
     // (segment 0 = node jf's words); s(q) = nsp[q/32] + popc(nsm[q/32] & bits 0..q%32)
@@ -969,9 +967,11 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-// threads 0..kWinCap-1: one batch of <= kWinCap registered mortals -> S.r*
+// threads 0..kWinCap-1 (whole warps): one batch of <= kWinCap registered mortals
+// -> S.r*, and each loading warp's least base / greatest end (the batch's hull)
 __device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
     const uint32_t e = threadIdx.x;
+    uint64_t b = ~0ull, en = 0;
     if (e < m) {
         const WinRec x = p.d.list_c[bs + e];
         S.rb[e] = x.base;
@@ -979,59 +979,32 @@ __device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint64_t b
         S.rta[e] = x.t_alloc;
         S.rtf[e] = x.t_free;
         S.rid[e] = x.id;
+        b = x.base;
+        en = x.end;
+    }
+    b = warp_min_u64(b);
+    en = warp_max_u64(en);
+    if ((e & 31) == 0) {
+        S.hmin[e >> 5] = b;
+        S.hmax[e >> 5] = en;
     }
 }
 
-// warp 0: the loaded batch sorted by (base, t_alloc) in registers, permuted into S.w*
-template <int E>
-__device__ __forceinline__ void window_sort_e(ClsShared& S, uint32_t m) {
-    const uint32_t lane = threadIdx.x & 31;
-    uint64_t k[E];
-    uint32_t v[E], pl[E];
-#pragma unroll
-    for (int r = 0; r < E; ++r) {
-        const uint32_t e = lane * E + r;
-        k[r] = e < m ? S.rb[e] : ~0ull;
-        v[r] = e < m ? S.rta[e] : 0xFFFFFFFFu;
-        pl[r] = e;
-    }
-    warp_bitonic<E>(k, v, pl);
-    uint64_t hi = 0;
-#pragma unroll
-    for (int r = 0; r < E; ++r) {
-        const uint32_t e = lane * E + r;
-        if (e < m) {
-            const uint32_t q = pl[r];
-            S.wb[e] = k[r];
-            S.we[e] = S.re[q];
-            S.wta[e] = v[r];
-            S.wtf[e] = S.rtf[q];
-            S.wid[e] = S.rid[q];
-            hi = max(hi, S.re[q]);
-        }
-    }
-    hi = warp_max_u64(hi);
-    if (lane == 0) {  // the batch's address hull: words outside it skip the lookup
-        S.hull_lo = k[0];  // lane 0 holds the smallest base
-        S.hull_hi = hi;
-    }
-}
-
-__device__ __forceinline__ void window_sort(ClsShared& S, uint32_t m) {
-    if (m <= 32) window_sort_e<1>(S, m);
-    else if (m <= 64) window_sort_e<2>(S, m);
-    else window_sort_e<4>(S, m);
-}
-
-// The live masks of nodes g0 .. g0+ng for the sorted batch of m entries (whole CTA;
+// The live masks of nodes g0 .. g0+ng for the loaded batch of m entries (whole CTA;
 // nt = their launch positions).  Entry e is live at nodes u0 <= u < u1
 // (t_alloc < t_u < t_free): toggle bit e at u0 and u1, then a prefix XOR over u.
 __device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uint32_t ng, uint32_t m) {
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) {  // the batch's address hull
+        uint64_t lo = ~0ull, hi = 0;
+        for (uint32_t w = 0; w < (m + 31) / 32; ++w) { lo = min(lo, S.hmin[w]); hi = max(hi, S.hmax[w]); }
+        S.hull_lo = lo;
+        S.hull_hi = hi;
+    }
     for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
     __syncthreads();
     for (uint32_t e = tid; e < m; e += kThreads) {
-        const uint32_t ta = S.wta[e], tf = S.wtf[e];
+        const uint32_t ta = S.rta[e], tf = S.rtf[e];
         uint32_t lo = 0, hi = ng;  // u0 = #{u : t_u <= t_alloc}
         while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] <= ta) lo = mid + 1; else hi = mid; }
         const uint32_t u0 = lo;
@@ -1063,19 +1036,18 @@ __device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uin
 }
 
 // The window entry holding word x at node u - g0 of the current group, or -1:
-// the live entries of one launch are pairwise disjoint, so the only possible
-// container is the live entry with the greatest base <= x.
+// the live entries of one launch are pairwise disjoint (a well-formed trace), so
+// the first live entry whose range holds x is the only one.
 __device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint32_t ul, uint64_t x) {
     if (x < S.hull_lo || x >= S.hull_hi) return -1;
-    uint32_t lo = 0, hi = m;  // entries with base <= x
-    while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.wb[mid] <= x) lo = mid + 1; else hi = mid; }
-    for (int w = ((int)lo - 1) >> 5; w >= 0; --w) {
+    // the entries live at the node (a handful: ~4 mortals are live at a launch in
+    // the BASELINE sets) -- at most one holds x
+    for (uint32_t w = 0; w < (m + 31) / 32; ++w) {
         uint32_t bits = S.live[ul][w];
-        const uint32_t top = lo - (uint32_t)w * 32;  // entries of word w below lo
-        if (top < 32) bits &= (1u << top) - 1u;
-        if (bits) {
-            const int e = w * 32 + 31 - __clz(bits);
-            return x < S.we[e] ? e : -1;
+        while (bits) {
+            const uint32_t e = w * 32 + __ffs(bits) - 1;
+            bits &= bits - 1;
+            if (S.rb[e] <= x && x < S.re[e]) return (int)e;
         }
     }
     return -1;
@@ -1202,15 +1174,13 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     // Everything above reads only the inputs and k_trace's outputs (two launches
     // back): it overlaps k_prepare's tail.  The registration lists are k_prepare's.
     pdl_wait();
-    // D. the first window batch: loaded, sorted by (base, t_alloc) in warp 0's
-    //    registers, live masks of the first node group
+    // D. the first window batch (in list order: no sort) and the live masks of
+    //    the first node group
     const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
     if (tid < kWinCap) window_load(p, S, r0, m0);
     __syncthreads();
-    if (warp == 0 && m0) window_sort(S, m0);
-    __syncthreads();
     if (m0) build_live(S, S.nt0, ng0, m0);
-    TL_PHASE(4, 12, tl_p);  // D: window, sort, live masks
+    TL_PHASE(4, 12, tl_p);  // D: window, live masks
     // E. per candidate its segment (O(1) from the start bitmask) and the window
     //    lookup at node group 0 / batch 0
     const bool more_batches = r1 - r0 > (uint64_t)kWinCap;
@@ -1224,7 +1194,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
             const int e = window_find(S, m0, u, x);
             if (e >= 0) {
                 hit = true;
-                S.words[q] = ((uint64_t)S.wid[e] << MEDUSA_OFF_BITS) | (x - S.wb[e]);
+                S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rb[e]);
                 atomicOr(&S.hits[q >> 5], 1u << (q & 31));
             }
         }
@@ -1242,8 +1212,6 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                 __syncthreads();
                 window_load(p, S, bs, m);
                 __syncthreads();
-                if (warp == 0) window_sort(S, m);
-                __syncthreads();
             }
             for (uint32_t g0 = (bs == r0 ? kNodeGrp : 0); g0 < n_seg; g0 += kNodeGrp) {
                 const uint32_t ng = min((uint32_t)kNodeGrp, n_seg - g0);
@@ -1258,7 +1226,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                     const uint64_t x = S.words[q];
                     const int e = window_find(S, m, u - g0, x);
                     if (e >= 0) {
-                        S.words[q] = ((uint64_t)S.wid[e] << MEDUSA_OFF_BITS) | (x - S.wb[e]);
+                        S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rb[e]);
                         atomicOr(&S.hits[q >> 5], 1u << (q & 31));
                     }
                 }
