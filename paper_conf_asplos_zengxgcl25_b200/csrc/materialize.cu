@@ -1394,10 +1394,10 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 //     CTA; warp w takes the queue region classify's warp w filled.  Per candidate
 //     one group of bases and one entry (two dependent loads); a hit writes its
 //     record at its word index and sets its mask bit; the chunk's count grows by
-//     one atomic per chunk.
+//     one atomic per warp (no CTA barrier: the warps run through the chunks
+//     independently).
 __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
-    __shared__ uint32_t s_cnt[kWarps];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
@@ -1429,18 +1429,11 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                 }
                 cnt += __popc(__ballot_sync(0xffffffffu, hit));
             }
-            if (lane == 0) s_cnt[warp] = cnt;
-            __syncthreads();
-            if (tid == 0) {
-                uint32_t total = 0;
-#pragma unroll
-                for (int w = 0; w < kWarps; ++w) total += s_cnt[w];
-                if (total) {
-                    atomicAdd(p.d.chunk_cnt + c, total);
-                    atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)total);
-                }
+            // per-warp counts (no CTA barrier: the warps run ahead independently)
+            if (lane == 0 && cnt) {
+                atomicAdd(p.d.chunk_cnt + c, cnt);
+                atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)cnt);
             }
-            __syncthreads();
         }
     }
     pdl_trigger();
