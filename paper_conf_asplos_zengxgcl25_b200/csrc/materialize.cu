@@ -1041,13 +1041,19 @@ __device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uin
 __device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint32_t ul, uint64_t x) {
     if (x < S.hull_lo || x >= S.hull_hi) return -1;
     // the entries live at the node (a handful: ~4 mortals are live at a launch in
-    // the BASELINE sets) -- at most one holds x
+    // the BASELINE sets) -- at most one holds x.  32-bit shared-window addresses
+    // (ld.shared): no generic-to-shared base rebuilt inside the loop
+    const uint32_t a_live = smem_u32(&S.live[ul][0]), a_rb = smem_u32(S.rb), a_re = smem_u32(S.re);
     for (uint32_t w = 0; w < (m + 31) / 32; ++w) {
-        uint32_t bits = S.live[ul][w];
+        uint32_t bits;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(bits) : "r"(a_live + 4 * w));
         while (bits) {
             const uint32_t e = w * 32 + __ffs(bits) - 1;
             bits &= bits - 1;
-            if (S.rb[e] <= x && x < S.re[e]) return (int)e;
+            uint64_t b, en;
+            asm volatile("ld.shared.u64 %0, [%1];" : "=l"(b) : "r"(a_rb + 8 * e));
+            asm volatile("ld.shared.u64 %0, [%1];" : "=l"(en) : "r"(a_re + 8 * e));
+            if (b <= x && x < en) return (int)e;
         }
     }
     return -1;
