@@ -459,12 +459,8 @@ constexpr int kCPBInPlace = MEDUSA_RESTORE_CPB_IP;  // chunks per restore CTA (i
 
 cudaError_t launch_restore(const RestoreArgs& a, cudaStream_t stream) {
     const bool in_place = a.src == a.dst;
-    static int sm_count = 0;
-    if (!sm_count) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sm_count, cudaDevAttrMultiProcessorCount, dev);
-    }
+    int dev = 0, sm_count = 148;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sm_count, cudaDevAttrMultiProcessorCount, dev);
     // small images (a single model's graph set): one chunk per CTA, so the CTAs
     // spread over more SMs and each chain of dependent loads is half as long
     const bool small = (a.n_words + 2ull * kTaskWords - 1) / (2ull * kTaskWords) < (uint64_t)sm_count;

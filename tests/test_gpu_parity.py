@@ -81,8 +81,9 @@ def test_restore_driven_by_oracle_table(graph_sets):
     assert np.array_equal(medusa.report_numpy(rep), rep_o)
 
 
-def test_in_place_and_misaligned(graph_sets):
-    gs = graph_sets("qwen1.5-4b")
+@pytest.mark.parametrize("name", ["qwen1.5-4b", "all10"])  # one chunk per restore CTA / two
+def test_in_place_and_misaligned(graph_sets, name):
+    gs = graph_sets(name)
     m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size)
     inp = medusa.upload(gs, DEV)
     slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
