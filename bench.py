@@ -553,6 +553,10 @@ def run_ours(args):
         issue_peak = 4 * sm_count * 1.965e9 / 1e12  # T warp-instructions/s at the 1965 MHz max SM clock
         rl["issue"] = {"warp_inst_per_launch": inst, "achieved": inst / dom_avg_s / 1e12, "peak": issue_peak,
                        "unit": "T warp-inst/s", "frac": inst / dom_avg_s / 1e12 / issue_peak}
+    if dom == "mat_classify":
+        rl["note"] = ("k_classify reads each word once (TMA) but its time goes to dependent shared-memory work "
+                      "behind CTA barriers (window setup, per-candidate node and window lookups): latency- and "
+                      "issue-bound, not HBM-bound; stall breakdown in profiles/r1_classify_stalls.txt, DESIGN.md §6")
     rst = per["restore"]
     restore_avg_s = rst[1] / rst[0] / 1e3
     relocate = {"kernel": "restore", "GB/s": alg["restore"] / restore_avg_s / 1e9,
