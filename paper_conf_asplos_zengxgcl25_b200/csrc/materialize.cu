@@ -1167,13 +1167,18 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     uint16_t* wl = S.cq + warp * 256;   // this warp's candidates (word in chunk)
     uint32_t* wh = S.hits + warp * 8;   // hit bits of the warp's 256 words
     uint32_t nc = 0;
+    const uint32_t lt = lanemask_lt();
 #pragma unroll
-    for (int k = 0; k < kWordsPerThread; ++k) {
-        const uint32_t q = warp * 256 + k * 32 + lane;
-        const bool cand = q < n && S.words[q] >= gmin && S.words[q] < gmax;
-        const uint32_t b = __ballot_sync(0xffffffffu, cand);
-        if (cand) wl[nc + __popc(b & lanemask_lt())] = (uint16_t)q;
-        nc += __popc(b);
+    for (int k = 0; k < kWordsPerThread / 2; ++k) {  // two words per lane: one 16-B shared load
+        const uint32_t q = warp * 256 + k * 64 + 2 * lane;
+        const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(&S.words[q]);
+        const bool c0 = q < n && v.x >= gmin && v.x < gmax;
+        const bool c1 = q + 1 < n && v.y >= gmin && v.y < gmax;
+        const uint32_t b0 = __ballot_sync(0xffffffffu, c0), b1 = __ballot_sync(0xffffffffu, c1);
+        uint32_t o = nc + __popc(b0 & lt) + __popc(b1 & lt);  // ascending word order
+        if (c0) wl[o++] = (uint16_t)q;
+        if (c1) wl[o] = (uint16_t)(q + 1);
+        nc += __popc(b0) + __popc(b1);
     }
     if (lane < 8) wh[lane] = 0;
     TL_PHASE(4, 11, tl_p);  // B/C: node starts, TMA wait, candidates
@@ -1261,14 +1266,18 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     // F. per 32 words: the mask word (lane 0) and the records at their word index
     const uint64_t n_mask = (a.n_words + 31) / 32;
     uint32_t cnt = 0;
+    if (lane < 8) {  // the warp's 8 mask words, one lane each
+        const uint32_t q0 = warp * 256 + lane * 32;
+        const uint64_t mw = (cs + q0) >> 5;
+        const uint32_t bits = wh[lane];
+        if (q0 < n && mw < n_mask) a.mask[mw] = bits;
+        cnt = __popc(bits);
+    }
+    cnt = __reduce_add_sync(0xffffffffu, cnt);
 #pragma unroll
     for (int k = 0; k < kWordsPerThread; ++k) {
         const uint32_t q = warp * 256 + k * 32 + lane;
-        const uint32_t bits = wh[k];
-        const uint64_t mw = (cs + q) >> 5;
-        if (lane == 0 && q < n && mw < n_mask) a.mask[mw] = bits;
-        if ((bits >> lane) & 1u) p.d.staging[cs + q] = S.words[q];
-        cnt += __popc(bits);
+        if ((wh[k] >> lane) & 1u) p.d.staging[cs + q] = S.words[q];
     }
     if (lane == 0) {
         p.d.qcnt[c * kWarps + warp] = nq;
