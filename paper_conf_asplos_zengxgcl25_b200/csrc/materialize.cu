@@ -963,6 +963,15 @@ struct ClsShared {
     unsigned long long mbar;
 };
 
+#ifndef MEDUSA_CLS_SMEM
+#define MEDUSA_CLS_SMEM 33792
+#endif
+// k_classify's dynamic shared memory: the window state (26 KB) padded to 33 KB, so
+// that 6 classify CTAs fit on an SM (228 KB) instead of 8: the CTAs k_classify
+// launches early (PDL) then leave room for the rank branch, which otherwise waits
+// for classify CTAs to finish (k_rank started 6 us later, step span +2 us)
+constexpr size_t kClsSmem = MEDUSA_CLS_SMEM > sizeof(ClsShared) ? MEDUSA_CLS_SMEM : sizeof(ClsShared);
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
@@ -1624,7 +1633,7 @@ Scratch* device_scratch(cudaError_t* e) {
     Scratch& s = *g_scratch[dev];
     if (!s.h_ctl) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
-        cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ClsShared));
+        cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kClsSmem);
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
@@ -1683,7 +1692,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaEventRecord(s.ranked, side))) return e;
         if (C) {
             TimedLaunch tl("mat_classify", stream);
-            if ((e = launch_pdl(k_classify, C, kThreads, sizeof(ClsShared), stream, p))) return e;
+            if ((e = launch_pdl(k_classify, C, kThreads, kClsSmem, stream, p))) return e;
         }
         if ((e = cudaEventRecord(s.classified, stream))) return e;
         // high priority after the classify: queue resolution and emission (the
@@ -1711,7 +1720,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             // no k_prepare in between: a plain launch (k_classify reads k_trace's
             // outputs before its griddepcontrol.wait, which is only safe two launches back)
             TimedLaunch tl("mat_classify", stream);
-            k_classify<<<C, kThreads, sizeof(ClsShared), stream>>>(p);
+            k_classify<<<C, kThreads, kClsSmem, stream>>>(p);
         }
         TimedLaunch tl("mat_emit", stream);
         if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
