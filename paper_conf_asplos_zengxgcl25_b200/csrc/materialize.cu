@@ -21,23 +21,27 @@
 //    min(t_alloc) / max(t_free) summaries over the address run a mortal meets,
 //    M-M inside blocks of 32 allocation ordinals against the mortals registered
 //    as live there.
-// Pipeline: five launches on `stream`, one host synchronization at the end.  Role
-// split by blockIdx where two independent phases share a launch:
-//   k_trace         [nodes] CSR / launch-order checks, first/last node per chunk
-//                   [allocs] trace checks, I/M split, registration ranges and
-//                   counts; the last alloc CTA scans the counts into offsets
-//   k_prepare       [sort] I keys sorted in tiles of 2048 (register bitonic per
-//                   warp + shared-memory merges); [scatter] registration lists
-//   k_rank          global rank of every I key = its index in its tile + the count
-//                   below it in every other tile; the last contribution writes
-//                   the I arrays, the fences and the block summaries
-//   k_scan_words    [classify] one CTA per 2048-word chunk: TMA bulk copy of the
-//                   chunk's words to shared memory, candidate compaction, window
-//                   search, I-list search through a compacted queue, mask words,
-//                   warp-dense staging of the records, the chunk's slot count; the
-//                   last classify CTA scans counts -> chunk_base
-//                   [check] M-M, M-I and I-I overlap checks
-//   k_emit          compaction of the staged records into the slot table
+// Pipeline (the synchronous entry adds one host read at the end):
+//   memset (counters) -> k_trace -> k_prepare -> k_classify ............ (join) [-> k_result]
+//   side (high priority):  k_rank -> (after k_classify) k_iresolve -> k_emit ---^
+//   low (default priority): (after k_rank) k_check ----------------------------^
+//   k_trace      [nodes] CSR / launch-order checks, first/last node per chunk;
+//                [allocs] trace checks, I/M split, registration ranges, two-level
+//                registration counts, I compaction
+//   k_prepare    [sort] I keys sorted in tiles of 1024 (register bitonic per warp
+//                + shared-memory merges); [scatter] registration lists.  Triggers
+//                its dependents at once: k_classify's setup overlaps it
+//   k_rank       global rank of every I key -> the sorted I arrays, the fences and
+//                the per-32 summaries
+//   k_classify   one CTA per 2048-word chunk: before griddepcontrol.wait the TMA
+//                copy of the chunk's words, node starts, candidate compaction;
+//                after it the mortal window, per-node live masks, the lookups;
+//                mask words, records at their word index, I-list candidates into
+//                a per-warp queue, the chunk's slot count
+//   k_check      M-M, M-I and I-I overlap checks
+//   k_iresolve   queued candidates against the sorted I list
+//   k_emit       chunk_base (two-level prefix) and the records compacted into the
+//                slot table
 #include <algorithm>
 #include <mutex>
 #include <vector>
