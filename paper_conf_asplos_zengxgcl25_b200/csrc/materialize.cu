@@ -1508,26 +1508,57 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
         for (int h = 0; h < kEmitChunks; ++h) s_pre[h][tid] += s_pre[h][64];  // second half after the first
     }
     __syncthreads();
+    if (tid == 0) {
 #pragma unroll
-    for (int h = 0; h < kEmitChunks; ++h) {
-        if ((uint32_t)h >= nch) break;
-        const uint32_t c = c0 + h;
-        const uint64_t m0 = (uint64_t)c * (kChunkWords / 32);
-        if (tid == 0) {
-            a.chunk_base[c] = (uint32_t)prefix;
-            if (c + 1 == p.C) {
-                a.chunk_base[c + 1] = (uint32_t)(prefix + total[h]);
-                p.d.ctl->n_slots = prefix + total[h];
+        for (int h = 0; h < kEmitChunks; ++h) {
+            if ((uint32_t)h >= nch) break;
+            const uint64_t pf = prefix + (h ? total[0] : 0u);
+            a.chunk_base[c0 + h] = (uint32_t)pf;
+            if (c0 + h + 1 == p.C) {
+                a.chunk_base[c0 + h + 1] = (uint32_t)(pf + total[h]);
+                p.d.ctl->n_slots = pf + total[h];
             }
         }
-        for (uint32_t r = tid; r < total[h]; r += kThreads) {
-            uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
-            while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
-            const uint64_t dst = prefix + r;
-            const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);  // the (r - s_pre[lo])-th set bit
-            if (dst < a.capacity) a.slot[dst] = p.d.staging[(m0 + lo) * 32 + bit];
+    }
+    // records: every load of the CTA's (up to kRecPerThread per chunk per thread)
+    // issued before the first store -- the loads do not wait for each other
+    constexpr int kRecPerThread = 2;
+    uint64_t val[kEmitChunks][kRecPerThread], dst[kEmitChunks][kRecPerThread];
+#pragma unroll
+    for (int h = 0; h < kEmitChunks; ++h) {
+        const uint64_t m0 = (uint64_t)(c0 + h) * (kChunkWords / 32);
+        const uint64_t pf = prefix + (h ? total[0] : 0u);
+#pragma unroll
+        for (int k = 0; k < kRecPerThread; ++k) {
+            const uint32_t r = tid + k * kThreads;
+            dst[h][k] = ~0ull;
+            if (r < total[h]) {
+                uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
+                while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
+                const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);  // the (r - s_pre[lo])-th set bit
+                if (pf + r < a.capacity) {
+                    dst[h][k] = pf + r;
+                    val[h][k] = __ldcg(p.d.staging + (m0 + lo) * 32 + bit);
+                }
+            }
         }
-        prefix += total[h];
+    }
+#pragma unroll
+    for (int h = 0; h < kEmitChunks; ++h)
+#pragma unroll
+        for (int k = 0; k < kRecPerThread; ++k)
+            if (dst[h][k] != ~0ull) a.slot[dst[h][k]] = val[h][k];
+    // the rest (chunks with more than kRecPerThread * kThreads records)
+#pragma unroll
+    for (int h = 0; h < kEmitChunks; ++h) {
+        const uint64_t m0 = (uint64_t)(c0 + h) * (kChunkWords / 32);
+        const uint64_t pf = prefix + (h ? total[0] : 0u);
+        for (uint32_t r = tid + kRecPerThread * kThreads; r < total[h]; r += kThreads) {
+            uint32_t lo = 0, hi = 64;
+            while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
+            const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);
+            if (pf + r < a.capacity) a.slot[pf + r] = p.d.staging[(m0 + lo) * 32 + bit];
+        }
     }
     pdl_trigger();
     TL_REC(5, 0, tl0);
