@@ -22,9 +22,9 @@
 //    M-M inside blocks of 32 allocation ordinals against the mortals registered
 //    as live there.
 // Pipeline (the synchronous entry adds one host read at the end):
-//   memset (counters) -> k_trace -> k_prepare -> k_classify -> k_iresolve -> k_emit [-> k_result]
-//   side (high priority):   k_rank ----------------------------------^ (after the rank)
-//   low (default priority): (after k_rank) k_check ------------------------------^ (joined)
+//   memset (counters) -> k_trace -> k_prepare -> k_classify ............ (join) [-> k_result]
+//   side (high priority):  k_rank -> (after k_classify) k_iresolve -> k_emit ---^
+//   low (default priority): (after k_rank) k_check ----------------------------^
 //   k_trace      [nodes] CSR / launch-order checks, first/last node per chunk;
 //                [allocs] trace checks, I/M split, registration ranges, two-level
 //                registration counts, I compaction
@@ -1591,7 +1591,7 @@ struct Scratch {
     int sm_count = 0;
     cudaStream_t side = nullptr;  // the I-list rank branch (highest priority; forked from the caller's stream)
     cudaStream_t low = nullptr;   // the trace-check branch (default priority; joined before the call ends)
-    cudaEvent_t fork = nullptr, join = nullptr, ranked = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr, ranked = nullptr, classified = nullptr, emitted = nullptr;
 };
 std::mutex g_mu;
 std::vector<Scratch*> g_scratch;
@@ -1675,19 +1675,23 @@ Scratch* device_scratch(cudaError_t* e) {
             (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_lo)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess ||
-            (*e = cudaEventCreateWithFlags(&s.ranked, cudaEventDisableTiming)) != cudaSuccess)
+            (*e = cudaEventCreateWithFlags(&s.ranked, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.classified, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.emitted, cudaEventDisableTiming)) != cudaSuccess)
             return nullptr;
         cudaDeviceGetAttribute(&s.sm_count, cudaDevAttrMultiProcessorCount, dev);
     }
     return &s;
 }
 
-// the whole analysis on `stream` (no synchronization):
-//   stream:            k_trace -> k_prepare -> k_classify -> [ranked] k_iresolve -> [join] k_emit
-//   side (high prio):  [fork] k_rank [ranked]
-//   low (default):     [ranked] k_check [join]
-// k_emit is on the caller's stream so that what follows it there (k_result,
-// a restore) follows it programmatically; the checks join just before it.
+// the whole analysis on `stream` (no synchronization).  After k_prepare (I-list
+// tile sort + registration lists):
+//   stream:            k_classify [classified] ............................ [emitted][join]
+//   side (high prio):  k_rank [ranked] ... [classified] k_iresolve -> k_emit [emitted]
+//   low (default):     [classified][ranked] k_check [join]
+// The high-priority stream gets the rank CTAs dispatched ahead of the classify
+// CTAs and the queue resolution / emission ahead of the trace checks, which
+// fill in around them and complete the call.
 cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P* out) {
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
@@ -1725,27 +1729,27 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             TimedLaunch tl("mat_classify", stream);
             if ((e = launch_pdl(k_classify, C, kThreads, kClsSmem, stream, p))) return e;
         }
-        // the trace checks (default priority) after the rank
+        if ((e = cudaEventRecord(s.classified, stream))) return e;
+        // high priority after the classify: queue resolution and emission (the
+        // rank is already on this stream)
+        if ((e = cudaStreamWaitEvent(side, s.classified, 0))) return e;
+        if (C) {
+            {
+                TimedLaunch tl("mat_iresolve", side);
+                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
+            }
+            TimedLaunch tl("mat_emit", side);
+            if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
+        }
+        if ((e = cudaEventRecord(s.emitted, side))) return e;
+        // default priority: the trace checks fill in around them
         if ((e = cudaStreamWaitEvent(low, s.ranked, 0))) return e;
         {
             TimedLaunch tl("mat_check", low);
             k_check<<<check_ctas, kThreads, 0, low>>>(p);
         }
         if ((e = cudaEventRecord(s.join, low))) return e;
-        // queue resolution and emission on the caller's stream after the classify and
-        // the rank: k_emit's successors follow it programmatically
-        if ((e = cudaStreamWaitEvent(stream, s.ranked, 0))) return e;
-        if (C) {
-            {
-                TimedLaunch tl("mat_iresolve", stream);
-                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, stream>>>(p);
-            }
-            if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
-            TimedLaunch tl("mat_emit", stream);
-            if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
-        } else if ((e = cudaStreamWaitEvent(stream, s.join, 0))) {
-            return e;
-        }
+        if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
         {
             // no k_prepare in between: a plain launch (k_classify reads k_trace's
