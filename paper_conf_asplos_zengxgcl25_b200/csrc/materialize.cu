@@ -1320,8 +1320,8 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 //     two more loads).
 __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
-    __shared__ uint64_t s_base[kWarps][32], s_end[kWarps][32];
-    __shared__ uint32_t s_tf[kWarps][32], s_idx[kWarps][32];
+    __shared__ ulonglong2 s_be[kWarps][32];  // (base, end): one 16-byte broadcast load
+    __shared__ uint2 s_ti[kWarps][32];       // (t_free, id): one 8-byte broadcast load
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     pdl_trigger();
@@ -1372,17 +1372,17 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
             __syncwarp();
             if (keep) {
                 const uint32_t o = __popc(kb & lanemask_lt());
-                s_base[warp][o] = y.base;
-                s_end[warp][o] = y.end;
-                s_tf[warp][o] = y.t_free;
-                s_idx[warp][o] = y.id;
+                s_be[warp][o] = make_ulonglong2(y.base, y.end);
+                s_ti[warp][o] = make_uint2(y.t_free, y.id);
             }
             __syncwarp();
             if (mine) {
                 const uint32_t nk = __popc(kb);
-                for (uint32_t q = 0; q < nk; ++q)
-                    bad |= (s_idx[warp][q] < j) & (s_tf[warp][q] > x.t_alloc) & (s_base[warp][q] < xe) &
-                           (x.base < s_end[warp][q]);
+                for (uint32_t q = 0; q < nk; ++q) {
+                    const ulonglong2 be = s_be[warp][q];
+                    const uint2 ti = s_ti[warp][q];
+                    bad |= (ti.y < j) & (ti.x > x.t_alloc) & (be.x < xe) & (x.base < be.y);
+                }
             }
         }
     }
