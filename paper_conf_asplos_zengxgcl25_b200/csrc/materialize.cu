@@ -949,7 +949,7 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 //    word q of warp w is q = 256 w + 32 k + lane (k = 0..7).
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
-    uint64_t rb[kWinCap], re[kWinCap];   // one batch of registered mortals as loaded
+    ulonglong2 rbe[kWinCap];             // (base, end) of one batch of registered mortals as loaded
     uint32_t rta[kWinCap], rtf[kWinCap], rid[kWinCap];
     uint64_t hmin[kWinCap / 32], hmax[kWinCap / 32];  // per loading warp: least base, greatest end
     uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
@@ -987,8 +987,7 @@ __device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint64_t b
     uint64_t b = ~0ull, en = 0;
     if (e < m) {
         const WinRec x = p.d.list_c[bs + e];
-        S.rb[e] = x.base;
-        S.re[e] = x.end;
+        S.rbe[e] = make_ulonglong2(x.base, x.end);
         S.rta[e] = x.t_alloc;
         S.rtf[e] = x.t_free;
         S.rid[e] = x.id;
@@ -1056,16 +1055,15 @@ __device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint3
     // the entries live at the node (a handful: ~4 mortals are live at a launch in
     // the BASELINE sets) -- at most one holds x.  32-bit shared-window addresses
     // (ld.shared): no generic-to-shared base rebuilt inside the loop
-    const uint32_t a_live = smem_u32(&S.live[ul][0]), a_rb = smem_u32(S.rb), a_re = smem_u32(S.re);
+    const uint32_t a_live = smem_u32(&S.live[ul][0]), a_rbe = smem_u32(S.rbe);
     for (uint32_t w = 0; w < (m + 31) / 32; ++w) {
         uint32_t bits;
         asm volatile("ld.shared.u32 %0, [%1];" : "=r"(bits) : "r"(a_live + 4 * w));
         while (bits) {
             const uint32_t e = w * 32 + __ffs(bits) - 1;
             bits &= bits - 1;
-            uint64_t b, en;
-            asm volatile("ld.shared.u64 %0, [%1];" : "=l"(b) : "r"(a_rb + 8 * e));
-            asm volatile("ld.shared.u64 %0, [%1];" : "=l"(en) : "r"(a_re + 8 * e));
+            uint64_t b, en;  // one 16-byte load of (base, end)
+            asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(b), "=l"(en) : "r"(a_rbe + 16 * e));
             if (b <= x && x < en) return (int)e;
         }
     }
@@ -1218,7 +1216,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
             const int e = window_find(S, m0, u, x);
             if (e >= 0) {
                 hit = true;
-                S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rb[e]);
+                S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rbe[e].x);
                 atomicOr(&S.hits[q >> 5], 1u << (q & 31));
             }
         }
@@ -1250,7 +1248,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                     const uint64_t x = S.words[q];
                     const int e = window_find(S, m, u - g0, x);
                     if (e >= 0) {
-                        S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rb[e]);
+                        S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rbe[e].x);
                         atomicOr(&S.hits[q >> 5], 1u << (q & 31));
                     }
                 }
