@@ -25,10 +25,13 @@
  *   - The return value reports argument, trace and launch errors only.
  *     Data-dependent validation failures of a restore are not call errors:
  *     they are counted in the device-side medusa_report (the call is async).
- *   - Thread-safe: calls may come from several host threads and devices.  The
- *     materialize entry points of one device share that device's scratch: the
- *     synchronous one serializes itself; an asynchronous one must be ordered
- *     (same stream, or events) against every other materialize on the device.
+ *   - Thread-safe: calls may come from several host threads and devices; calls
+ *     on different devices never wait for each other.  The materialize entry
+ *     points of one device share that device's scratch: the synchronous one
+ *     holds the device's lock until its work is done (other threads' materialize
+ *     calls on that device wait); an asynchronous one holds it while enqueueing
+ *     only and must be ordered (same stream, or events) against every other
+ *     materialize on the device.
  *   - Work is enqueued on the caller's `stream`.  Materialize forks part of its
  *     work onto an internal stream and joins it back before returning, so the
  *     call is one stream-ordered unit (and capturable, see below).
@@ -104,10 +107,12 @@ typedef struct {
  *   n_bad_func     nodes whose kernel-name id is >= the table size or maps to 0
  *                  (unresolved); their func_out is 0
  *   first_bad_node least such node index
- *   reserved       0 (used internally while the call is in flight)            */
+ *   n_bad_chunk    chunks whose d_chunk_base range disagrees with their mask
+ *                  (see medusa_restore, "table consistency"); their words are
+ *                  copied unchanged and their slots counted nowhere else     */
 typedef struct {
     uint64_t n_bad_slot, first_bad_word, n_bad_id, n_bad_range, n_stale;
-    uint64_t n_bad_func, first_bad_node, reserved;
+    uint64_t n_bad_func, first_bad_node, n_bad_chunk;
 } medusa_report;
 
 #define MEDUSA_CHUNK_WORDS 2048u   /* chunk size of d_chunk_base (fixed; part of the ABI) */
@@ -208,6 +213,13 @@ medusa_status medusa_kernel_table_set(const uint64_t *d_func_addr, uint32_t n_fu
  *   d_new_base[i] is the address the i-th allocation returned when the
  *   (de)allocation sequence was replayed.  Non-slot words
  *   are copied unchanged (constants keep their plain values).
+ *   Table consistency (DESIGN.md R-TABLE; a table medusa_materialize wrote is
+ *   always consistent): chunk c (words [2048c, 2048c + 2048)) is consistent iff
+ *   d_chunk_base[c+1] - d_chunk_base[c] (>= 0) equals the number of mask bits of
+ *   its words (bits of words >= n_words are ignored).  Then its i-th slot word
+ *   (ascending) pairs with record d_chunk_base[c] + i; a record index >= n_slots
+ *   means the record is missing: that slot counts as n_bad_id.  An inconsistent
+ *   chunk is copied unchanged and counted once in n_bad_chunk.
  *   Kernel-address fill: d_func_out[j] = table[d_func_id[j]] if the id is below
  *   the installed table's size and the entry is non-zero, else 0 (n_bad_func).
  *   d_func_id, d_func_out, n_nodes: all NULL/0 to skip the fill.
@@ -298,6 +310,24 @@ medusa_status medusa_buffers_save(const uint32_t *d_perm, const uint64_t *d_perm
 medusa_status medusa_buffers_restore(const uint8_t *d_blob, const uint32_t *d_perm, const uint64_t *d_perm_off,
                                      uint32_t n_perm, const uint64_t *d_new_base, const uint64_t *d_new_size,
                                      uint32_t n_alloc, medusa_buf_report *d_report, cudaStream_t stream);
+
+/* ---- library-owned memory ------------------------------------------------
+ * medusa_materialize / _async use per-device scratch the library allocates and
+ * grows on demand (x1.5 past the previous size); medusa_kernel_table_set owns a
+ * per-device table.  A growth never frees the buffers it replaces: a CUDA graph
+ * that captured an earlier call holds their addresses by value, so replaying it
+ * stays memory-safe (it keeps reading and writing the old, still-allocated
+ * buffers).  They are freed only by medusa_scratch_release or at process exit.
+ *
+ * medusa_scratch_bytes: live scratch bytes of the current device (retired
+ *   buffers excluded).
+ * medusa_scratch_release: synchronizes the current device, then frees its
+ *   scratch, every retired scratch buffer and every retired kernel table (the
+ *   installed table stays).  Every CUDA graph that captured a materialize or a
+ *   retired table on this device is invalid afterwards and must not be replayed.
+ *   The next materialize reallocates (outside any capture).                   */
+uint64_t medusa_scratch_bytes(void);
+medusa_status medusa_scratch_release(void);
 
 /* cudaError_t value behind the last MEDUSA_ERR_CUDA returned on this thread. */
 int medusa_last_cuda_error(void);

@@ -34,6 +34,8 @@ def _load():
         lib.oracle_pack_slots.restype = None
         lib.oracle_restore.argtypes = [P, P, U64, P, P, P, U64, P, P, P, U32, P, P, U32, P, U32, P]
         lib.oracle_restore.restype = None
+        lib.oracle_restore_packed.argtypes = [P, P, U64, P, P, P, U64, P, P, P, U32, P, P, U32, P, U32, P]
+        lib.oracle_restore_packed.restype = None
         _lib = lib
     return _lib
 
@@ -88,7 +90,7 @@ def pack(m, n_words):
 
 
 REPORT_FIELDS = ("n_bad_slot", "first_bad_word", "n_bad_id", "n_bad_range", "n_stale",
-                 "n_bad_func", "first_bad_node", "reserved")
+                 "n_bad_func", "first_bad_node", "n_bad_chunk")
 
 
 def restore(src, slot_g, slot_id, slot_off, old_base, new_base, new_size, func_id=None, table=None):
@@ -111,4 +113,30 @@ def restore(src, slot_g, slot_id, slot_off, old_base, new_base, new_size, func_i
                        func_id.size if func_id is not None else 0,
                        _p(table) if table is not None else ctypes.c_void_p(0),
                        table.size if table is not None else 0, _p(rep))
+    return dst, fout, rep
+
+
+def restore_packed(src, mask, chunk_base, records, n_slots, old_base, new_base, new_size, func_id=None,
+                   table=None):
+    """oracle_restore_packed (DESIGN.md R-TABLE) -> (dst u64[n_words], func_out or None, report u64[8])."""
+    lib = _load()
+    src = _c(src, np.uint64)
+    dst = np.zeros_like(src)
+    mask, chunk_base, records = _c(mask, np.uint32), _c(chunk_base, np.uint32), _c(records, np.uint64)
+    assert chunk_base.size == (src.size + CHUNK_WORDS - 1) // CHUNK_WORDS + 1 and mask.size >= (src.size + 31) // 32
+    assert records.size >= min(int(n_slots), int(chunk_base.max(initial=0)))
+    old_base, new_base, new_size = _c(old_base, np.uint64), _c(new_base, np.uint64), _c(new_size, np.uint64)
+    rep = np.zeros(8, np.uint64)
+    fout = None
+    if func_id is not None:
+        func_id = _c(func_id, np.uint32)
+        table = _c(table, np.uint64)
+        fout = np.zeros(func_id.size, np.uint64)
+    lib.oracle_restore_packed(_p(src), _p(dst), src.size, _p(mask), _p(chunk_base), _p(records), int(n_slots),
+                              _p(old_base), _p(new_base), _p(new_size), new_base.size,
+                              _p(func_id) if func_id is not None else ctypes.c_void_p(0),
+                              _p(fout) if fout is not None else ctypes.c_void_p(0),
+                              func_id.size if func_id is not None else 0,
+                              _p(table) if table is not None else ctypes.c_void_p(0),
+                              table.size if table is not None else 0, _p(rep))
     return dst, fout, rep

@@ -28,6 +28,12 @@
 //                           and the kernel-address fill.
 //                           Pinned by identity, constant shift, untouched
 //                           constants, fault injection (closed forms).
+//   oracle_restore_packed -- the same restoration driven by the table in its ABI
+//                           layout (mask, chunk_base, records, n_slots), with
+//                           the table-consistency reading DESIGN.md R-TABLE.
+//                           Pinned by equality with oracle_restore on every
+//                           packed table oracle_pack_slots writes, and by a
+//                           hand-computed inconsistent-table fixture.
 #include <cstdint>
 #include <cstring>
 #include <map>
@@ -237,6 +243,50 @@ void oracle_restore(const uint64_t* src, uint64_t* dst, uint64_t n_words,
         }
     }
     for (int q = 0; q < 8; ++q) report[q] = r[q];
+}
+
+// RESTORE driven by the packed table (DESIGN.md R-TABLE).  Chunk c = words
+// [2048c, min(2048c + 2048, n_words)).  Its slot words are the words of the
+// chunk whose mask bit is set, ascending.  The chunk is consistent iff
+// chunk_base[c+1] >= chunk_base[c] and chunk_base[c+1] - chunk_base[c] equals
+// its number of slot words; then its i-th slot word g pairs with record
+// k = chunk_base[c] + i, which is missing if k >= n_slots (counted as a bad
+// id at g); otherwise record k = id << 40 | off is validated and applied
+// exactly as in oracle_restore.  An inconsistent chunk keeps every word and
+// adds 1 to report[7] (n_bad_chunk).  The kernel-address fill is oracle_restore's.
+void oracle_restore_packed(const uint64_t* src, uint64_t* dst, uint64_t n_words,
+                           const uint32_t* mask, const uint32_t* chunk_base, const uint64_t* records,
+                           uint64_t n_slots, const uint64_t* old_base, const uint64_t* new_base,
+                           const uint64_t* new_size, uint32_t n_alloc, const uint32_t* func_id,
+                           uint64_t* func_out, uint32_t n_nodes, const uint64_t* table, uint32_t n_func,
+                           uint64_t* report) {
+    const uint64_t CHUNK = 2048;
+    const uint64_t n_chunks = (n_words + CHUNK - 1) / CHUNK;
+    std::vector<uint64_t> g_list, id_list, off_list;  // the slots the consistent chunks pair up
+    std::vector<uint64_t> missing;                    // slot words whose record is missing
+    uint64_t bad_chunks = 0;
+    for (uint64_t c = 0; c < n_chunks; ++c) {
+        std::vector<uint64_t> words_with_bit;
+        for (uint64_t g = c * CHUNK; g < n_words && g < (c + 1) * CHUNK; ++g)
+            if ((mask[g / 32] >> (g % 32)) & 1u) words_with_bit.push_back(g);
+        uint64_t lo = chunk_base[c], hi = chunk_base[c + 1];
+        if (hi < lo || hi - lo != words_with_bit.size()) { ++bad_chunks; continue; }
+        for (uint64_t i = 0; i < words_with_bit.size(); ++i) {
+            uint64_t k = lo + i;
+            if (k >= n_slots) { missing.push_back(words_with_bit[i]); continue; }
+            g_list.push_back(words_with_bit[i]);
+            id_list.push_back(records[k] >> 40);
+            off_list.push_back(records[k] & ((1ull << 40) - 1));
+        }
+    }
+    // ids of 2^24 and more cannot come from a record (24 bits); a missing record is
+    // given an id no replay has, so oracle_restore counts it as a bad id
+    std::vector<uint32_t> id32(id_list.size());
+    for (size_t q = 0; q < id_list.size(); ++q) id32[q] = (uint32_t)id_list[q];
+    for (uint64_t g : missing) { g_list.push_back(g); id32.push_back(0xFFFFFFFFu); off_list.push_back(0); }
+    oracle_restore(src, dst, n_words, g_list.data(), id32.data(), off_list.data(), g_list.size(), old_base,
+                   new_base, new_size, n_alloc, func_id, func_out, n_nodes, table, n_func, report);
+    report[7] = bad_chunks;
 }
 
 }  // extern "C"

@@ -23,7 +23,7 @@ CHUNK_WORDS = 2048
 OFF_BITS = 40
 T_END = 0xFFFFFFFF
 REPORT_FIELDS = ("n_bad_slot", "first_bad_word", "n_bad_id", "n_bad_range", "n_stale",
-                 "n_bad_func", "first_bad_node", "reserved")
+                 "n_bad_func", "first_bad_node", "n_bad_chunk")
 
 
 class MedusaError(RuntimeError):
@@ -76,6 +76,10 @@ def lib():
         L.medusa_timing_enable.restype = None
         L.medusa_timing_read.argtypes = [ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(ctypes.c_float), I]
         L.medusa_timing_read.restype = I
+        L.medusa_scratch_bytes.argtypes = []
+        L.medusa_scratch_bytes.restype = U64
+        L.medusa_scratch_release.argtypes = []
+        L.medusa_scratch_release.restype = I
         _lib = L
     return _lib
 
@@ -249,6 +253,19 @@ def buffers_restore(plan, blob, new_base, new_size, report=None, stream=None):
     if st != OK:
         raise MedusaError(st, "medusa_buffers_restore")
     return report
+
+
+def scratch_bytes():
+    """medusa_scratch_bytes: live materialize scratch of the current device."""
+    return int(lib().medusa_scratch_bytes())
+
+
+def scratch_release():
+    """medusa_scratch_release: free the current device's scratch and retired buffers
+    (synchronizes; invalidates CUDA graphs that captured a materialize)."""
+    st = lib().medusa_scratch_release()
+    if st != OK:
+        raise MedusaError(st, "medusa_scratch_release")
 
 
 def timing_enable(on=True):

@@ -21,6 +21,7 @@ struct DeviceTable {
     uint32_t capacity = 0;
     uint32_t n_func = 0;
     bool set = false;
+    std::vector<uint64_t*> retired;  // earlier tables: a captured graph may still read them
 };
 std::mutex g_mu;
 std::vector<DeviceTable> g_tables;
@@ -75,6 +76,21 @@ const char* medusa_status_string(medusa_status s) {
 }
 
 void medusa_timing_enable(int on) { g_timing = on != 0; }
+
+uint64_t medusa_scratch_bytes(void) { return scratch_bytes(); }
+
+medusa_status medusa_scratch_release(void) {
+    cudaError_t e = release_scratch();  // synchronizes the device
+    if (e != cudaSuccess) return cuda_fail(e);
+    int dev = 0;
+    if ((e = cudaGetDevice(&dev)) != cudaSuccess) return cuda_fail(e);
+    std::lock_guard<std::mutex> lk(g_mu);
+    if ((int)g_tables.size() > dev) {
+        for (uint64_t* p : g_tables[dev].retired) cudaFree(p);
+        g_tables[dev].retired.clear();
+    }
+    return MEDUSA_OK;
+}
 
 int medusa_timing_read(const char** names, float* ms, int max) {
     int n = 0;
@@ -152,7 +168,9 @@ medusa_status medusa_kernel_table_set(const uint64_t* d_func_addr, uint32_t n_fu
         uint64_t* p = nullptr;
         e = cudaMalloc(&p, (size_t)cap * sizeof(uint64_t));
         if (e != cudaSuccess) return cuda_fail(e);
-        if (t.d_table) cudaFree(t.d_table);  // implicit device synchronization: no restore still reads it
+        // the old table stays allocated: restores in flight, and CUDA graphs that
+        // captured a medusa_restore, hold its address (freed by medusa_scratch_release)
+        if (t.d_table) t.retired.push_back(t.d_table);
         t.d_table = p;
         t.capacity = cap;
     }

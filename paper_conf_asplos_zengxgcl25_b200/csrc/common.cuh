@@ -159,6 +159,11 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
 medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
                                     cudaError_t* cuda_err);
 
+// Live materialize scratch of the current device, in bytes; and its release
+// (synchronizes the device, frees the scratch and every retired buffer).
+uint64_t scratch_bytes();
+cudaError_t release_scratch();
+
 // ---- buffer contents (buffers.cu) ---------------------------------------------
 medusa_status run_buffers_plan(const medusa_alloc* alloc, uint32_t n_alloc, const uint32_t* cap, uint32_t n_cap,
                                const uint64_t* slot, uint64_t n_slots, uint8_t* cls, uint32_t* perm,

@@ -1091,7 +1091,9 @@ __device__ __forceinline__ void seg_times(const P& p, ClsShared& S, uint32_t* nt
     __syncthreads();
     if (threadIdx.x == 0 && g0 == 0) nt[0] = p.a.node_t[jf];
     for (uint32_t j = jf + 1 + threadIdx.x; j <= jl; j += kThreads) {
-        const uint32_t s = seg_of(S, (uint32_t)(p.a.node_off[j] - cs));
+        const uint32_t q = (uint32_t)(p.a.node_off[j] - cs);
+        if (q >= kChunkWords) continue;
+        const uint32_t s = seg_of(S, q);
         if (s >= g0 && s < g0 + ng) atomicMax(nt + (s - g0), p.a.node_t[j]);  // the last node of a start is its non-empty one
     }
     __syncthreads();
@@ -1107,6 +1109,17 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const uint64_t* gsrc = a.words + cs;
     const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
     const uint32_t mb = smem_u32(&S.mbar);
+    // A malformed CSR or launch order (flagged by k_trace, two launches back and
+    // therefore complete) leaves jf / jl and the node offsets meaningless: write
+    // the empty counts the later kernels read and do nothing else (the call
+    // returns INVALID_ARG; no shared-memory index is ever derived from node_off)
+    if (__ldcg(&ctl->status) & ST_INVALID) {
+        if (tid < kWarps) p.d.qcnt[c * kWarps + tid] = 0;
+        if (tid == 0) p.d.chunk_cnt[c] = 0;
+        pdl_wait();
+        pdl_trigger();
+        return;
+    }
     // A. the chunk's words -> shared memory with one TMA bulk copy; meanwhile the
     //    list offsets (block_prefix) and the chunk's node range load
     if (tid == 0) {
@@ -1136,6 +1149,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     uint32_t my_q = 0xFFFFFFFFu, my_t = 0;  // this thread's first node (start, launch position)
     for (uint32_t j = jf + 1 + tid; j <= jl; j += kThreads) {
         const uint32_t q = (uint32_t)(a.node_off[j] - cs);
+        if (q >= n) continue;  // (a valid CSR puts every start of (jf, jl] inside the chunk)
         if (my_q == 0xFFFFFFFFu) { my_q = q; my_t = a.node_t[j]; }
         atomicOr(&S.nsm[q >> 5], 1u << (q & 31));
     }
@@ -1162,7 +1176,9 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     }
     if (nn > (uint32_t)kThreads + 1) {  // more nodes than threads: the rest
         for (uint32_t j = jf + 1 + kThreads + tid; j <= jl; j += kThreads) {
-            const uint32_t sg = seg_of(S, (uint32_t)(a.node_off[j] - cs));
+            const uint32_t q = (uint32_t)(a.node_off[j] - cs);
+            if (q >= n) continue;
+            const uint32_t sg = seg_of(S, q);
             if (sg < kNodeGrp) atomicMax(&S.nt0[sg], a.node_t[j]);
         }
     }
@@ -1590,8 +1606,15 @@ struct Scratch {
     cudaStream_t side = nullptr;  // the I-list rank branch (highest priority; forked from the caller's stream)
     cudaStream_t low = nullptr;   // the trace-check branch (default priority; joined before the call ends)
     cudaEvent_t fork = nullptr, join = nullptr, ranked = nullptr, classified = nullptr, emitted = nullptr;
+    // Buffers retired by a growth.  A CUDA graph that captured an earlier
+    // medusa_materialize_async holds their addresses by value, so they stay
+    // allocated (replaying such a graph stays memory-safe) until
+    // medusa_scratch_release() or process exit.
+    std::vector<void*> graveyard;
+    size_t bytes = 0;  // live scratch bytes (zero region + buffers)
+    std::mutex mu;  // one materialize at a time per device (the scratch is shared); devices run concurrently
 };
-std::mutex g_mu;
+std::mutex g_mu;  // guards g_scratch only
 std::vector<Scratch*> g_scratch;
 
 template <class T>
@@ -1601,25 +1624,33 @@ cudaError_t grow(Scratch& s, T*& p, size_t elems) {
     if (e != cudaSuccess) return e;
     p = q;
     s.bufs.push_back(q);
+    s.bytes += std::max<size_t>(elems, 1) * sizeof(T);
     return cudaSuccess;
 }
 
-void release(Scratch& s) {
-    for (void* p : s.bufs) cudaFree(p);
+// the current buffers -> the graveyard (not freed: see Scratch::graveyard)
+void retire(Scratch& s) {
+    for (void* p : s.bufs) s.graveyard.push_back(p);
     s.bufs.clear();
-    if (s.zero_region) cudaFree(s.zero_region);
+    if (s.zero_region) s.graveyard.push_back(s.zero_region);
     s.zero_region = nullptr;
+    s.bytes = 0;
     s.cap_n = s.cap_C = s.cap_nb = s.cap_c = s.cap_b = s.cap_w = 0;
 }
+
+// grow geometrically (x1.5) past the previous capacity, so a sequence of growing
+// calls retires a bounded amount of memory
+size_t grown(size_t need, size_t old) { return need <= old ? old : std::max(need, old + old / 2); }
 
 cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t need_c, size_t need_b) {
     if (n <= s.cap_n && C <= s.cap_C && nb <= s.cap_nb && W <= s.cap_w && need_c <= s.cap_c && need_b <= s.cap_b)
         return cudaSuccess;
-    cudaDeviceSynchronize();
-    release(s);
-    const size_t N = std::max<size_t>(n, 1024), CC = std::max<size_t>(C, 64), NB = std::max<size_t>(nb, 64);
-    const size_t WW = std::max<size_t>(W, 2048);
-    const size_t RC = std::max<size_t>(need_c, N + 4 * CC), RB = std::max<size_t>(need_b, 3 * N);
+    const size_t N = grown(std::max<size_t>(n, 1024), s.cap_n), CC = grown(std::max<size_t>(C, 64), s.cap_C);
+    const size_t NB = grown(std::max<size_t>(nb, 64), s.cap_nb);
+    const size_t WW = grown(std::max<size_t>(W, 2048), s.cap_w);
+    const size_t RC = grown(std::max<size_t>(need_c, N + 4 * CC), s.cap_c);
+    const size_t RB = grown(std::max<size_t>(need_b, 3 * N), s.cap_b);
+    retire(s);
     const size_t NS = N / kIBlk + 1;
     cudaError_t e;
     // zero region: Ctl | sup_c chunk_sup [CC/256+1] sup_b [NB/256+1] (u64) | cnt_c fill_c [CC+1] |
@@ -1627,6 +1658,7 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
     const size_t GC = CC / 256 + 1, GB = NB / 256 + 1;
     s.zero_bytes = 256 + (2 * GC + GB) * 8 + 2 * (CC + 1) * 4 + 2 * (NB + 1) * 4 + 2 * NS * 4 + 64;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
+    s.bytes += s.zero_bytes;
     char* z = (char*)s.zero_region;
     s.d.ctl = (Ctl*)z;
     size_t o = 256;
@@ -1657,13 +1689,20 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t n
 
 namespace {
 
-Scratch* device_scratch(cudaError_t* e) {
+// this device's scratch, returned with its lock held (*lk)
+Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
     int dev = 0;
     *e = cudaGetDevice(&dev);
     if (*e != cudaSuccess) return nullptr;
-    if ((int)g_scratch.size() <= dev) g_scratch.resize(dev + 1, nullptr);
-    if (!g_scratch[dev]) g_scratch[dev] = new Scratch();
-    Scratch& s = *g_scratch[dev];
+    Scratch* sp;
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        if ((int)g_scratch.size() <= dev) g_scratch.resize(dev + 1, nullptr);
+        if (!g_scratch[dev]) g_scratch[dev] = new Scratch();
+        sp = g_scratch[dev];
+    }
+    *lk = std::unique_lock<std::mutex>(sp->mu);
+    Scratch& s = *sp;
     if (!s.h_ctl) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kClsSmem);
@@ -1767,8 +1806,8 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
                               cudaError_t* cuda_err) {
     *n_slots = 0;
     cudaError_t e;
-    std::lock_guard<std::mutex> lk(g_mu);
-    Scratch* sp = device_scratch(&e);
+    std::unique_lock<std::mutex> lk;  // this device's scratch, for the whole call (other devices run concurrently)
+    Scratch* sp = device_scratch(&e, &lk);
     if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     Scratch& s = *sp;
     const uint64_t n = a.n_alloc;
@@ -1800,8 +1839,8 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
 medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
                                     cudaError_t* cuda_err) {
     cudaError_t e;
-    std::lock_guard<std::mutex> lk(g_mu);
-    Scratch* sp = device_scratch(&e);
+    std::unique_lock<std::mutex> lk;  // held while enqueueing only
+    Scratch* sp = device_scratch(&e, &lk);
     if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     Scratch& s = *sp;
     const uint64_t n = a.n_alloc;
@@ -1814,6 +1853,32 @@ medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result*
     if ((e = launch_pdl(k_result, 1, 1, 0, stream, p, d_result))) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     if ((e = cudaGetLastError()) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     return MEDUSA_OK;
+}
+
+uint64_t scratch_bytes() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+    std::lock_guard<std::mutex> g(g_mu);
+    if ((int)g_scratch.size() <= dev || !g_scratch[dev]) return 0;
+    return g_scratch[dev]->bytes;
+}
+
+cudaError_t release_scratch() {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    Scratch* sp = nullptr;
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        if ((int)g_scratch.size() > dev) sp = g_scratch[dev];
+    }
+    if (!sp) return cudaSuccess;
+    std::lock_guard<std::mutex> lk(sp->mu);
+    if ((e = cudaDeviceSynchronize()) != cudaSuccess) return e;
+    retire(*sp);
+    for (void* p : sp->graveyard) cudaFree(p);
+    sp->graveyard.clear();
+    return cudaGetLastError();
 }
 
 }  // namespace medusa

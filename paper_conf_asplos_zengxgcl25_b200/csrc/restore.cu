@@ -55,7 +55,7 @@ __global__ void report_init(medusa_report* r) {
     r->n_stale = 0;
     r->n_bad_func = 0;
     r->first_bad_node = ~0ull;
-    r->reserved = 0;
+    r->n_bad_chunk = 0;
     TL_REC(6, 0, tl0);
 }
 
@@ -92,15 +92,129 @@ __device__ __forceinline__ void gather_role(const RestoreArgs& a, uint32_t gt, u
     }
 }
 
+// Table view of the CTA's CPB chunks (DESIGN.md R-TABLE): the mask words (bits of
+// words past n_words cleared), their popcount prefix (pre[kMask] = the CTA's
+// slot count), the chunk_base entries, and which chunks are consistent -- chunk
+// h is iff its record range [cb[h], cb[h+1]) holds exactly as many records as
+// its mask has bits.  The i-th set bit of a consistent chunk pairs with record
+// cb[h] + i; an inconsistent chunk is copied unchanged and counted (n_bad_chunk).
+template <int CPB>
+struct TableView {
+    static constexpr uint32_t kMask = CPB * kMaskPerTask;
+    uint32_t mask[kMask];
+    uint32_t pre[kMask + 1];
+    uint32_t cb[CPB + 1];
+    uint32_t ok;  // bit h: chunk h consistent
+};
+
+// (whole CTA) the mask words and the chunk_base entries; ends with a barrier
+template <int CPB>
+__device__ __forceinline__ void table_load(const RestoreArgs& a, uint32_t task, TableView<CPB>& T) {
+    constexpr uint32_t kMask = TableView<CPB>::kMask;
+    const uint64_t n_mask = (a.n_words + 31) / 32;
+    const uint64_t mw0 = (uint64_t)task * kMask;
+    const uint64_t n_chunks = (a.n_words + kTaskWords - 1) / kTaskWords;
+    for (uint32_t m = threadIdx.x; m < kMask; m += kThreads) {
+        const uint64_t mw = mw0 + m;
+        uint32_t v = 0;
+        if (mw < n_mask) {
+            v = a.mask[mw];
+            const uint64_t left = a.n_words - mw * 32;  // words of this mask word inside the image
+            if (left < 32) v &= (1u << left) - 1u;
+        }
+        T.mask[m] = v;
+    }
+    if (threadIdx.x >= kThreads - (CPB + 1)) {  // chunks past the image read the total: 0 records, 0 bits
+        const uint32_t h = threadIdx.x - (kThreads - (CPB + 1));
+        T.cb[h] = a.chunk_base[min((uint64_t)task * CPB + h, n_chunks)];
+    }
+    __syncthreads();
+}
+
+// (warp 0) exclusive popcount prefix of the mask words and the consistency bits
+template <int CPB>
+__device__ __forceinline__ void table_prefix(TableView<CPB>& T) {
+    constexpr int kPer = TableView<CPB>::kMask / 32;
+    const uint32_t lane = threadIdx.x & 31;
+    uint32_t pc[kPer], incl = 0;
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) { pc[j] = __popc(T.mask[kPer * lane + j]); incl += pc[j]; }
+    const uint32_t own = incl;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= (uint32_t)d) incl += y;
+    }
+    uint32_t run = incl - own;
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) { T.pre[kPer * lane + j] = run; run += pc[j]; }
+    if (lane == 31) T.pre[TableView<CPB>::kMask] = incl;
+    __syncwarp();
+    if (lane == 0) {
+        uint32_t ok = 0;
+#pragma unroll
+        for (int h = 0; h < CPB; ++h) {
+            const uint32_t bits = T.pre[(h + 1) * kMaskPerTask] - T.pre[h * kMaskPerTask];
+            if (T.cb[h + 1] >= T.cb[h] && T.cb[h + 1] - T.cb[h] == bits) ok |= 1u << h;
+        }
+        T.ok = ok;
+    }
+}
+
+// record index of the CTA's r-th slot bit; false if its chunk is inconsistent
+template <int CPB>
+__device__ __forceinline__ bool table_rec(const TableView<CPB>& T, uint32_t r, uint64_t& k) {
+    const uint32_t h = (CPB == 2 && r >= T.pre[kMaskPerTask]) ? 1u : 0u;
+    k = (uint64_t)T.cb[h] + (r - T.pre[h * kMaskPerTask]);
+    return (T.ok >> h) & 1u;
+}
+
+// word (in the CTA) of the r-th slot bit, r < pre[kMask]
+template <int CPB>
+__device__ __forceinline__ uint32_t table_word(const TableView<CPB>& T, uint32_t r) {
+    uint32_t lo = 0, hi = TableView<CPB>::kMask;
+    while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (T.pre[mid] <= r) lo = mid; else hi = mid; }
+    return lo * 32 + __fns(T.mask[lo], 0, (int)(r - T.pre[lo]) + 1);
+}
+
+// record k -> kind (0 ok, 1 bad id / missing record, 2 bad range), expected source
+// word and relocated value (DESIGN.md R-Q8, R-TABLE)
+__device__ __forceinline__ uint32_t load_rec(const RestoreArgs& a, uint64_t k, uint64_t& exp, uint64_t& nv) {
+    exp = nv = 0;
+    if (k >= a.n_slots) return 1;  // no record: the caller's slot count ends before it
+    const uint64_t rec = a.slot[k];
+    const uint64_t id = rec >> MEDUSA_OFF_BITS;
+    const uint64_t off = rec & kOffMask;
+    if (id >= a.n_alloc) return 1;
+    const uint64_t sz = __ldg(a.new_size + id);
+    const uint64_t ob = __ldg(a.old_base + id);
+    const uint64_t nb = __ldg(a.new_base + id);
+    if (off >= sz) return 2;
+    exp = ob + off;
+    nv = nb + off;
+    return 0;
+}
+
+__device__ __forceinline__ void report_add(unsigned long long* rep, uint32_t n_id, uint32_t n_rg, uint32_t n_st,
+                                           uint64_t first, uint32_t n_chunk) {
+    if (n_id | n_rg | n_st) {
+        atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));
+        atomicMin(rep + 1, (unsigned long long)first);
+        if (n_id) atomicAdd(rep + 2, (unsigned long long)n_id);
+        if (n_rg) atomicAdd(rep + 3, (unsigned long long)n_rg);
+        if (n_st) atomicAdd(rep + 4, (unsigned long long)n_st);
+    }
+    if (n_chunk) atomicAdd(rep + 7, (unsigned long long)n_chunk);
+}
+
 template <int CPB>
 __global__ void __launch_bounds__(kThreads, (CPB == 1 ? 8 : 6))
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     constexpr uint32_t kWords = CPB * kTaskWords;   // words of this CTA (CPB consecutive chunks)
     constexpr uint32_t kMask = CPB * kMaskPerTask;  // their mask words
+    constexpr uint32_t kAllOk = (1u << CPB) - 1u;
     __shared__ __align__(128) uint64_t s_words[kWords];
-    __shared__ uint32_t s_mask[kMask];
-    __shared__ uint32_t s_pre[kMask];
-    __shared__ uint32_t s_rec0, s_nrec;
+    __shared__ TableView<CPB> T;
     __shared__ __align__(8) unsigned long long s_mbar[CPB];
 
     const uint32_t tid = threadIdx.x;
@@ -132,69 +246,44 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             }
         }
         // 1. the CTA's words: one bulk copy per chunk into shared memory (all issued
-        //    at once); meanwhile the mask words and the record range.  (Issuing the
+        //    at once); meanwhile the mask words and the record ranges.  (Issuing the
         //    copies after those small loads measured the same: their ~3 us is not
         //    queueing behind the bulk reads.)
-        auto issue_tma = [&]() {
-            if (tid == 0 && tma) {
+        if (tid == 0 && tma) {
 #pragma unroll
-                for (int c = 0; c < CPB; ++c) {
-                    const uint32_t mb = smem_u32(&s_mbar[c]);
-                    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
-                }
-                asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-#pragma unroll
-                for (int c = 0; c < CPB; ++c) {
-                    const uint32_t q0 = c * kTaskWords;
-                    if (q0 >= n) break;
-                    const uint32_t nc = min(n - q0, kTaskWords);
-                    const uint32_t mb = smem_u32(&s_mbar[c]);
-                    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(nc * 8) : "memory");
-                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                                 ::"r"(smem_u32(s_words + q0)), "l"(gsrc + q0), "r"(nc * 8), "r"(mb) : "memory");
-                }
+            for (int c = 0; c < CPB; ++c) {
+                const uint32_t mb = smem_u32(&s_mbar[c]);
+                asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
             }
-        };
-        issue_tma();
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+#pragma unroll
+            for (int c = 0; c < CPB; ++c) {
+                const uint32_t q0 = c * kTaskWords;
+                if (q0 >= n) break;
+                const uint32_t nc = min(n - q0, kTaskWords);
+                const uint32_t mb = smem_u32(&s_mbar[c]);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(nc * 8) : "memory");
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(smem_u32(s_words + q0)), "l"(gsrc + q0), "r"(nc * 8), "r"(mb) : "memory");
+            }
+        }
         if (!tma)
             for (uint32_t q = tid; q < n; q += kThreads) s_words[q] = ld_stream(gsrc + q);
-        const uint64_t n_mask = (a.n_words + 31) / 32;
-        const uint64_t mw0 = ws / 32;
-        const uint64_t n_chunks = (a.n_words + kTaskWords - 1) / kTaskWords;
-        for (uint32_t m = tid; m < kMask; m += kThreads) s_mask[m] = (mw0 + m < n_mask) ? a.mask[mw0 + m] : 0u;
-        if (tid == kThreads - 1) {
-            const uint64_t c0 = (uint64_t)task * CPB;
-            const uint32_t r0 = a.chunk_base[c0], r1 = a.chunk_base[min(c0 + CPB, n_chunks)];
-            s_rec0 = r0;
-            s_nrec = r1 > r0 ? r1 - r0 : 0;
-        }
-        __syncthreads();
+        table_load<CPB>(a, task, T);
         TL_PHASE(7, 10, tl_p);  // mask + record range loaded
-        // 2. exclusive prefix of the mask popcounts (warp 0; kMask / 32 words per lane)
-        if (tid < 32) {
-            constexpr int kPer = kMask / 32;
-            uint32_t pc[kPer], incl = 0;
-#pragma unroll
-            for (int j = 0; j < kPer; ++j) { pc[j] = __popc(s_mask[kPer * tid + j]); incl += pc[j]; }
-            const uint32_t own = incl;
-#pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                if (tid >= d) incl += y;
-            }
-            uint32_t run = incl - own;
-#pragma unroll
-            for (int j = 0; j < kPer; ++j) { s_pre[kPer * tid + j] = run; run += pc[j]; }
-        }
-        const uint64_t rec0 = s_rec0;
-        const uint32_t n_rec = s_nrec;
-        const uint32_t n_rec_c = min(n_rec, kWords);
+        // 2. popcount prefix and consistency (warp 0) while the other warps load the
+        //    first records, assuming every chunk consistent (the normal case:
+        //    record cb[0] + r for bit r); checked after the barrier
+        if (tid < 32) table_prefix<CPB>(T);
+        const uint32_t cb0 = T.cb[0];
+        uint32_t n_bits = T.cb[CPB] >= cb0 ? min(T.cb[CPB] - cb0, kWords) : 0u;  // exact once verified
         // 3. records, two per thread per round: load, gather, (after the prefix is
         //    ready) locate the word, validate and rewrite it in shared memory
         uint32_t n_id = 0, n_rg = 0, n_st = 0;
         uint64_t first = ~0ull;
         uint32_t ready_mask = tma ? 0u : ~0u;  // chunks whose words have landed
-        for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += 2 * kThreads) {
+        bool fast = true;
+        for (uint32_t rb = 0; rb < max(n_bits, 1u); rb += 2 * kThreads) {
             uint64_t exp[2], nv[2];
             uint32_t kind[2];  // 0 ok, 1 bad id, 2 bad range, 3 none
 #pragma unroll
@@ -202,66 +291,50 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 const uint32_t r = rb + tid + u * kThreads;
                 kind[u] = 3;
                 exp[u] = nv[u] = 0;
-                if (r < n_rec_c) {
-                    kind[u] = 1;
-                    const uint64_t k = rec0 + r;
-                    if (k < a.n_slots) {
-                        const uint64_t rec = a.slot[k];
-                        const uint64_t id = rec >> MEDUSA_OFF_BITS;
-                        const uint64_t off = rec & kOffMask;
-                        if (id < a.n_alloc) {
-                            const uint64_t sz = __ldg(a.new_size + id);
-                            const uint64_t ob = __ldg(a.old_base + id);
-                            const uint64_t nb = __ldg(a.new_base + id);
-                            if (off < sz) {
-                                kind[u] = 0;
-                                exp[u] = ob + off;
-                                nv[u] = nb + off;
-                            } else {
-                                kind[u] = 2;
-                            }
-                        }
+                uint64_t k = (uint64_t)cb0 + r;
+                if (r < n_bits && (fast || table_rec<CPB>(T, r, k))) kind[u] = load_rec(a, k, exp[u], nv[u]);
+            }
+            if (rb == 0) {
+                __syncthreads();  // prefix and consistency ready
+                TL_PHASE(7, 11, tl_p);  // first records + gathers in
+                n_bits = T.pre[kMask];
+                if (T.ok != kAllOk) {  // (rare) an inconsistent chunk: round 0 again, chunk by chunk
+                    fast = false;
+#pragma unroll
+                    for (int u = 0; u < 2; ++u) {
+                        const uint32_t r = tid + u * kThreads;
+                        uint64_t k;
+                        kind[u] = (r < n_bits && table_rec<CPB>(T, r, k)) ? load_rec(a, k, exp[u], nv[u]) : 3u;
                     }
                 }
             }
-            if (rb == 0) __syncthreads();  // s_pre ready
-            if (rb == 0) TL_PHASE(7, 11, tl_p);  // first records + gathers in
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 if (kind[u] == 3) continue;
                 const uint32_t r = rb + tid + u * kThreads;
-                uint32_t lo = 0, hi = kMask;  // mask word m with s_pre[m] <= r < s_pre[m] + popc
-                while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
-                const uint32_t bit = __fns(s_mask[lo], 0, r - s_pre[lo] + 1);
-                const uint32_t q = lo * 32 + bit;
-                bool bad = true;
-                if (bit >= 32 || q >= n) {
-                    ++n_id;  // more records than mask bits: nothing to apply
-                } else {
-                    const uint32_t c = q / kTaskWords;
-                    if (!((ready_mask >> c) & 1u)) {  // this chunk's words: wait for its bulk copy
-                        const uint32_t mb = smem_u32(&s_mbar[c]);
-                        uint32_t ready = 0;
-                        while (!ready) {
-                            asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
-                                         : "=r"(ready) : "r"(mb) : "memory");
-                        }
-                        ready_mask |= 1u << c;
+                const uint32_t q = table_word<CPB>(T, r);
+                const uint32_t c = q / kTaskWords;
+                if (!((ready_mask >> c) & 1u)) {  // this chunk's words: wait for its bulk copy
+                    const uint32_t mb = smem_u32(&s_mbar[c]);
+                    uint32_t ready = 0;
+                    while (!ready) {
+                        asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
+                                     : "=r"(ready) : "r"(mb) : "memory");
                     }
-                    if (kind[u] == 0) {
-                        if (s_words[q] == exp[u]) { s_words[q] = nv[u]; bad = false; }
-                        else ++n_st;
-                    } else if (kind[u] == 1) {
-                        ++n_id;
-                    } else {
-                        ++n_rg;
-                    }
+                    ready_mask |= 1u << c;
                 }
-                if (bad) first = min(first, ws + (q < n ? q : 0));
+                bool bad = true;
+                if (kind[u] == 0) {
+                    if (s_words[q] == exp[u]) { s_words[q] = nv[u]; bad = false; }
+                    else ++n_st;
+                } else if (kind[u] == 1) {
+                    ++n_id;
+                } else {
+                    ++n_rg;
+                }
+                if (bad) first = min(first, ws + q);
             }
         }
-        // slots the mask shows beyond the table's records have nothing to apply
-        if (tid == 0 && n_rec > kWords) n_id += n_rec - kWords;
         // every chunk's bulk copy must have landed before its words go back out
         if (tid == 0 && tma) {
 #pragma unroll
@@ -298,13 +371,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         TL_PHASE(7, 13, tl_p);  // bulk store issued and read out of shared memory
         pdl_wait();  // report_init (this launch's PDL predecessor) has run
         pdl_trigger();
-        if (n_id | n_rg | n_st) {
-            atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));
-            atomicMin(rep + 1, (unsigned long long)first);
-            if (n_id) atomicAdd(rep + 2, (unsigned long long)n_id);
-            if (n_rg) atomicAdd(rep + 3, (unsigned long long)n_rg);
-            if (n_st) atomicAdd(rep + 4, (unsigned long long)n_st);
-        }
+        report_add(rep, n_id, n_rg, n_st, first, tid == 0 ? __popc(kAllOk & ~T.ok) : 0u);
         TL_REC(7, 0, tl0);
     } else if (task < n_tasks) {
         gather_role(a, task - n_word_tasks, rep);
@@ -314,7 +381,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
 
 // In place (dst == src): only the slot words are read and written -- the words
 // in between are constants that stay where they are.  One CTA per
-// CPB chunks: mask words + record range, popcount prefix, then per record:
+// CPB chunks: mask words + record ranges, popcount prefix, then per record:
 // load, gather, locate its word, read it, validate, write it back.  No word
 // staging, so the pass moves ~8 B/slot of image instead of 16 B/word.
 template <int CPB>
@@ -322,49 +389,23 @@ __global__ void __launch_bounds__(kThreads)
 restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     constexpr uint32_t kWords = CPB * kTaskWords;
     constexpr uint32_t kMask = CPB * kMaskPerTask;
+    constexpr uint32_t kAllOk = (1u << CPB) - 1u;
     constexpr uint32_t kPer = 2;  // records per thread per round
-    __shared__ uint32_t s_mask[kMask];
-    __shared__ uint32_t s_pre[kMask];
-    __shared__ uint32_t s_rec0, s_nrec;
+    __shared__ TableView<CPB> T;
     const uint32_t tid = threadIdx.x;
     const uint32_t task = blockIdx.x;
     unsigned long long* rep = reinterpret_cast<unsigned long long*>(a.report);
     const unsigned long long tl0 = TL_NOW();
     if (task < n_word_tasks) {
         const uint64_t ws = (uint64_t)task * kWords;
-        const uint32_t n = (uint32_t)min((uint64_t)kWords, a.n_words - ws);
-        const uint64_t n_mask = (a.n_words + 31) / 32;
-        const uint64_t mw0 = ws / 32;
-        const uint64_t n_chunks = (a.n_words + kTaskWords - 1) / kTaskWords;
-        for (uint32_t m = tid; m < kMask; m += kThreads) s_mask[m] = (mw0 + m < n_mask) ? a.mask[mw0 + m] : 0u;
-        if (tid == kThreads - 1) {
-            const uint64_t c0 = (uint64_t)task * CPB;
-            const uint32_t r0 = a.chunk_base[c0], r1 = a.chunk_base[min(c0 + CPB, n_chunks)];
-            s_rec0 = r0;
-            s_nrec = r1 > r0 ? r1 - r0 : 0;
-        }
-        __syncthreads();
-        if (tid < 32) {
-            constexpr int kMw = kMask / 32;
-            uint32_t pc[kMw], incl = 0;
-#pragma unroll
-            for (int j = 0; j < kMw; ++j) { pc[j] = __popc(s_mask[kMw * tid + j]); incl += pc[j]; }
-            const uint32_t own = incl;
-#pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
-                if (tid >= d) incl += y;
-            }
-            uint32_t run = incl - own;
-#pragma unroll
-            for (int j = 0; j < kMw; ++j) { s_pre[kMw * tid + j] = run; run += pc[j]; }
-        }
-        const uint64_t rec0 = s_rec0;
-        const uint32_t n_rec = s_nrec;
-        const uint32_t n_rec_c = min(n_rec, kWords);
+        table_load<CPB>(a, task, T);
+        if (tid < 32) table_prefix<CPB>(T);
+        const uint32_t cb0 = T.cb[0];
+        uint32_t n_bits = T.cb[CPB] >= cb0 ? min(T.cb[CPB] - cb0, kWords) : 0u;
         uint32_t n_id = 0, n_rg = 0, n_st = 0;
         uint64_t first = ~0ull;
-        for (uint32_t rb = 0; rb < max(n_rec_c, 1u); rb += kPer * kThreads) {
+        bool fast = true;
+        for (uint32_t rb = 0; rb < max(n_bits, 1u); rb += kPer * kThreads) {
             uint64_t exp[kPer], nv[kPer];
             uint32_t kind[kPer];  // 0 ok, 1 bad id, 2 bad range, 3 none
 #pragma unroll
@@ -372,53 +413,36 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 const uint32_t r = rb + tid + u * kThreads;
                 kind[u] = 3;
                 exp[u] = nv[u] = 0;
-                if (r < n_rec_c) {
-                    kind[u] = 1;
-                    const uint64_t k = rec0 + r;
-                    if (k < a.n_slots) {
-                        const uint64_t rec = a.slot[k];
-                        const uint64_t id = rec >> MEDUSA_OFF_BITS;
-                        const uint64_t off = rec & kOffMask;
-                        if (id < a.n_alloc) {
-                            const uint64_t sz = __ldg(a.new_size + id);
-                            const uint64_t ob = __ldg(a.old_base + id);
-                            const uint64_t nb = __ldg(a.new_base + id);
-                            if (off < sz) {
-                                kind[u] = 0;
-                                exp[u] = ob + off;
-                                nv[u] = nb + off;
-                            } else {
-                                kind[u] = 2;
-                            }
-                        }
+                uint64_t k = (uint64_t)cb0 + r;
+                if (r < n_bits && (fast || table_rec<CPB>(T, r, k))) kind[u] = load_rec(a, k, exp[u], nv[u]);
+            }
+            if (rb == 0) {
+                __syncthreads();  // prefix and consistency ready
+                n_bits = T.pre[kMask];
+                if (T.ok != kAllOk) {
+                    fast = false;
+#pragma unroll
+                    for (int u = 0; u < kPer; ++u) {
+                        const uint32_t r = tid + u * kThreads;
+                        uint64_t k;
+                        kind[u] = (r < n_bits && table_rec<CPB>(T, r, k)) ? load_rec(a, k, exp[u], nv[u]) : 3u;
                     }
                 }
             }
-            if (rb == 0) __syncthreads();  // s_pre ready
             uint32_t qs[kPer];
             uint64_t cur[kPer];
 #pragma unroll
             for (int u = 0; u < kPer; ++u) {  // locate every word first, then load them together
-                qs[u] = 0xFFFFFFFFu;
                 if (kind[u] == 3) continue;
-                const uint32_t r = rb + tid + u * kThreads;
-                uint32_t lo = 0, hi = kMask;
-                while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= r) lo = mid; else hi = mid; }
-                const uint32_t bit = __fns(s_mask[lo], 0, r - s_pre[lo] + 1);
-                const uint32_t q = lo * 32 + bit;
-                if (bit < 32 && q < n) {
-                    qs[u] = q;
-                    if (kind[u] == 0) cur[u] = ld_stream(a.src + ws + q);
-                }
+                qs[u] = table_word<CPB>(T, rb + tid + u * kThreads);
+                if (kind[u] == 0) cur[u] = ld_stream(a.src + ws + qs[u]);
             }
 #pragma unroll
             for (int u = 0; u < kPer; ++u) {
                 if (kind[u] == 3) continue;
                 const uint32_t q = qs[u];
                 bool bad = true;
-                if (q == 0xFFFFFFFFu) {
-                    ++n_id;  // more records than mask bits: nothing to apply
-                } else if (kind[u] == 0) {
+                if (kind[u] == 0) {
                     if (cur[u] == exp[u]) { st_stream(a.dst + ws + q, nv[u]); bad = false; }
                     else ++n_st;
                 } else if (kind[u] == 1) {
@@ -426,19 +450,12 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 } else {
                     ++n_rg;
                 }
-                if (bad) first = min(first, ws + (q != 0xFFFFFFFFu ? q : 0));
+                if (bad) first = min(first, ws + q);
             }
         }
-        if (tid == 0 && n_rec > kWords) n_id += n_rec - kWords;
         pdl_wait();
         pdl_trigger();
-        if (n_id | n_rg | n_st) {
-            atomicAdd(rep + 0, (unsigned long long)(n_id + n_rg + n_st));
-            atomicMin(rep + 1, (unsigned long long)first);
-            if (n_id) atomicAdd(rep + 2, (unsigned long long)n_id);
-            if (n_rg) atomicAdd(rep + 3, (unsigned long long)n_rg);
-            if (n_st) atomicAdd(rep + 4, (unsigned long long)n_st);
-        }
+        report_add(rep, n_id, n_rg, n_st, first, tid == 0 ? __popc(kAllOk & ~T.ok) : 0u);
         TL_REC(7, 2, tl0);
     } else if (task < n_tasks) {
         gather_role(a, task - n_word_tasks, rep);

@@ -438,3 +438,28 @@ def test_overflow_retry_many_batches_wide_chunks(seed):
     medusa.materialize_async(**inp, out=out, result=res)
     assert medusa.mat_result(res) == (0, m["n_slots"])
     assert np.array_equal(_h(out.slot)[: m["n_slots"]].view(np.uint64), rec)
+
+
+def test_malformed_csr_across_chunks_is_rejected_safely(graph_sets):
+    """A non-monotone CSR spanning several chunks, and one whose last offset is not
+    n_words, come back INVALID_ARG without touching memory out of range (the CUDA
+    context stays usable: a valid ten-model call right after is bit-exact)."""
+    b = 0x7F00_0000_0000
+    w = np.uint64(b) + np.arange(4096, dtype=np.uint64) * np.uint64(8)
+    A = np.array([(b, 8 * 4096, 1, T_NEVER)], dtype=ALLOC_DTYPE)
+    nt = np.array([2, 3, 4], np.uint32)
+    for off in ([0, 3000, 100, 4096], [0, 3000, 5000, 4096], [0, 100, 3000, 5000], [0, 2047, 6000, 9000],
+                [7, 100, 2000, 4096]):
+        st, _ = _run_tiny(w, np.array(off, np.uint64), nt, A)
+        assert st == medusa.ERR_INVALID_ARG, off
+    res = torch.zeros(2, dtype=torch.int64, device=DEV)
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(DEV)
+    aa = torch.from_numpy(np.ascontiguousarray(A).view(np.int64).reshape(-1, 3)).to(DEV)
+    medusa.materialize_async(t(w, np.int64), t(np.array([0, 3000, 100, 4096], np.uint64), np.int64),
+                             t(nt, np.int32), aa, out=medusa.alloc_slots(w.size, DEV), result=res)
+    assert medusa.mat_result(res)[0] == medusa.ERR_INVALID_ARG
+    gs = graph_sets("all10")
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    m, packed = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size)
+    _check_materialize(slots, m, packed, gs.n_words)
