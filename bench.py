@@ -9,9 +9,20 @@ restored per second, whole job; plus the relocate pass's HBM GB/s.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload all10] [--impl ours|reference]
 
-N > 1 runs under torchrun: every rank restores its own independent instance
-(seed offset per rank), no data-path collective (weak scaling); NCCL is used
-only for the start/stop barriers and the max-over-ranks of the device time.
+Multi-GPU: the path shards per instance, so every rank (one
+process per GPU) restores its own independently generated instance and no data
+crosses GPUs.  `--gpus N` without WORLD_SIZE in the environment starts the N
+rank processes itself; under torchrun WORLD_SIZE must equal N.  The ranks meet
+only on the host: a gloo process group supplies the start/stop barriers, the
+max over ranks of the device-timed regions and the gathering of per-rank
+results -- no NCCL, no collective on the data path.  Every rank runs
+  * the headline workload (`--workload`, default the ten-model set; rank r's
+    instance is generated with seed + 1000 r): value = N x nodes x K / max_r t_r;
+  * C5 (BASELINE.json configs[4]): its own Llama-2-13B-shaped instance with seed
+    100 + r, timed concurrently on every GPU: aggregate nodes/s
+    = sum of nodes / max time, per-GPU relocate GB/s, sustained relocate per GPU;
+  * parity: after timing, each rank's table, restored words, kernel addresses
+    and report of both workloads are compared with the CPU oracle.
 --impl reference times the CPU oracle (oracle/, plain C++) on the same config.
 """
 from __future__ import annotations
@@ -70,11 +81,14 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def load_traffic():
-    """Per-launch DRAM bytes of each kernel from the committed ncu --set full capture."""
+def load_traffic(workload):
+    """Per-launch DRAM bytes (and warp instructions, `_inst`) of each kernel of this
+    workload, from the committed ncu launch list of the same command
+    (profiles/ncu_traffic.json, one entry per workload); {} if none was captured
+    for it (then `traffic` is null: another workload's counters are never used)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
-        return json.load(open(p))
+        return json.load(open(p)).get(workload, {})
     except Exception:
         return {}
 
@@ -143,24 +157,93 @@ def graph_kernel_nodes(graph):
     return k
 
 
+C5 = "llama2-13b"  # BASELINE.json configs[4]: one Llama-2-13B-shaped instance per GPU, seed 100 + gpu
+
+
 def rank_seed(cfg, rank):
-    """Seed of the independent instance rank `rank` restores (weak scaling)."""
+    """Seed of the independent instance rank `rank` restores (weak scaling):
+    C5 uses 100 + rank, the other configs seed + 1000 rank."""
     from workloads.graphset import CONFIGS
+    if cfg == C5:
+        return CONFIGS[cfg]["seed"] + rank
     return CONFIGS[cfg]["seed"] + SEED_STRIDE * rank
 
 
-def max_over_ranks(x, dist, device):
-    """Max of a per-rank scalar over all ranks (the job's time is the slowest rank's)."""
+def max_over_ranks(x, dist, device=None):
+    """Max of a per-rank scalar over all ranks (the job's time is the slowest rank's),
+    over the host-side gloo group (no device collective)."""
     import torch
-    t = torch.tensor([float(x)], dtype=torch.float64, device=device)
+    t = torch.tensor([float(x)], dtype=torch.float64)
     if dist is not None and dist.is_initialized() and dist.get_world_size() > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
 
+def gather_to_all(obj, dist):
+    """Every rank's `obj`, in rank order (gloo all_gather_object; [obj] on one rank)."""
+    if dist is not None and dist.is_initialized() and dist.get_world_size() > 1:
+        out = [None] * dist.get_world_size()
+        dist.all_gather_object(out, obj)
+        return out
+    return [obj]
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     return int(os.environ.get("RANK", "0")), ws, int(os.environ.get("LOCAL_RANK", "0"))
+
+
+def config_dict(cfg, desc, gs, n_slots, seed, ws):
+    """The `config` object of the JSON line -- identical for both arms."""
+    return {"workload": f"{cfg} per rank: {desc}", "nodes_per_rank": gs.n_nodes, "words": gs.n_words,
+            "allocs": gs.n_alloc, "slots": int(n_slots), "kernel_names": int(gs.table.size), "seed": seed,
+            "l2": "GPU arm: 256 MiB (2x L2) scrub written before every timed step; CPU arm: not applicable",
+            "parallelism": f"{ws} independent instances (one per GPU), no collective"}
+
+
+def plumbing_selftest(args):
+    """`--selftest-plumbing` (CPU, tests/test_multi.py): the multi-rank plumbing of
+    run_ours without a GPU -- the gloo group the launcher's env describes, a
+    barrier, the max of a rank-dependent time, the gather -- printed by rank 0.
+    Produces no bench value."""
+    import torch.distributed as dist
+    rank, ws, local = dist_env()
+    if ws > 1:
+        dist.init_process_group("gloo", rank=rank, world_size=ws)
+        dist.barrier()
+    t = max_over_ranks(10.0 + rank, dist)
+    got = gather_to_all({"rank": rank, "local": local, "seed_c5": rank_seed(C5, rank),
+                         "seed_all10": rank_seed("all10", rank), "pid": os.getpid()}, dist)
+    if rank == 0:
+        print(json.dumps({"world_size": ws, "max_ms": t, "ranks": got}), flush=True)
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def spawn_ranks(args, n_visible=None):
+    """`--gpus N` outside torchrun: start N rank processes of this script (RANK /
+    LOCAL_RANK / WORLD_SIZE / MASTER_* set as torchrun would) and wait for them."""
+    import socket
+    import subprocess
+    if n_visible is None:
+        import torch
+        n_visible = torch.cuda.device_count()
+    n_dev = n_visible
+    if n_dev < args.gpus:
+        raise SystemExit(f"bench.py --gpus {args.gpus}: only {n_dev} GPU(s) visible")
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    procs = []
+    for r in range(args.gpus):
+        env = dict(os.environ, RANK=str(r), LOCAL_RANK=str(r), WORLD_SIZE=str(args.gpus),
+                   LOCAL_WORLD_SIZE=str(args.gpus), MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        procs.append(subprocess.Popen([sys.executable, os.path.abspath(__file__), *sys.argv[1:]], env=env))
+    rcs = [p.wait() for p in procs]
+    if any(rcs):
+        raise SystemExit(f"bench.py rank exit codes {rcs}")
 
 
 def run_reference(args):
@@ -174,7 +257,9 @@ def run_reference(args):
     from workloads import make_graph_set
 
     cfg, desc = WORKLOADS[args.workload]
-    gs = make_graph_set(cfg)
+    seed = rank_seed(cfg, 0)
+    gs = make_graph_set(cfg, seed=seed)
+    n_slots = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)["n_slots"]
 
     def step():
         m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
@@ -190,12 +275,13 @@ def run_reference(args):
     value = gs.n_nodes * args.steps / dt
     print(json.dumps({
         "impl": "reference", "metric": "graph nodes restored/sec (materialize + restore, whole hot path)",
-        "value": value, "unit": "nodes/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "value": value, "unit": "nodes/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "u64", "data": "synthetic",
-        "config": {"workload": f"{cfg}: {desc}", "nodes": gs.n_nodes, "words": gs.n_words, "allocs": gs.n_alloc},
+        "config": config_dict(cfg, desc, gs, n_slots, seed, args.gpus),
         "cpu_baseline": {"value": value, "unit": "nodes/s", "cores": 1, "kind": "oracle",
-                         "sample": f"full {cfg} graph set per step, single-threaded oracle/oracle.cpp (-O2)"},
+                         "sample": f"full {cfg} graph set per step (materialize + restore), single-threaded "
+                                   f"oracle/oracle.cpp (-O2), on rank 0 only"},
         "e2e": {"value": value, "unit": "nodes/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -408,6 +494,127 @@ def bench_buffers(medusa, gs, inp, slots, dev, stream, scrub, steps, peak):
                     "bytes = 2 x blob + 20 B per buffer"}
 
 
+def oracle_parity(gs, slots, n_slots, dst, fout, rep):
+    """This rank's GPU outputs against the CPU oracle on the same instance: the
+    table (mask, chunk prefix, records), restored words, kernel addresses, report."""
+    import oracle
+    import paper_conf_asplos_zengxgcl25_b200 as medusa
+    m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)
+    if m["status"] != 0:
+        return {"ok": False, "why": f"oracle status {m['status']}"}
+    mask, cb, rec = oracle.pack(m, gs.n_words)
+    odst, ofout, orep = oracle.restore(gs.words, m["slot_g"], m["slot_id"], m["slot_off"], gs.allocs["base"],
+                                       gs.new_base, gs.new_size, gs.func_id, gs.table)
+    h = lambda t: t.detach().cpu().numpy()
+    checks = {
+        "n_slots": n_slots == m["n_slots"],
+        "mask": np.array_equal(h(slots.mask).view(np.uint32), mask),
+        "chunk_base": np.array_equal(h(slots.chunk_base).view(np.uint32), cb),
+        "records": np.array_equal(h(slots.slot)[:m["n_slots"]].view(np.uint64), rec),
+        "words": np.array_equal(medusa.to_numpy_u64(dst), odst),
+        "func_out": np.array_equal(medusa.to_numpy_u64(fout), ofout),
+        "report": np.array_equal(medusa.report_numpy(rep), orep),
+    }
+    return {"ok": all(checks.values()), "failed": [k for k, v in checks.items() if not v],
+            "slots": int(m["n_slots"]), "words": gs.n_words}
+
+
+def bench_c5(medusa, args, rank, dev, stream, scrub, barrier, peak):
+    """C5 (BASELINE.json configs[4]): this rank's own
+    Llama-2-13B-shaped instance (seed 100 + rank), the whole-path step captured
+    as one CUDA graph and timed on every GPU at once (barrier-bracketed device
+    events); the restore alone (latency mode, graph replays); one sustained
+    restore over R replicas; parity with the oracle after timing."""
+    import torch
+    from workloads import make_graph_set
+    from workloads.graphset import replicate
+    seed = rank_seed(C5, rank)
+    gs = make_graph_set(C5, seed=seed)
+    inp = medusa.upload(gs, dev)
+    sl = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])  # sizes the scratch
+    n_slots = sl.n_slots
+    res = torch.zeros(2, dtype=torch.int64, device=dev)
+    dst = torch.empty_like(inp["words"])
+    fout = torch.empty(gs.n_nodes, dtype=torch.int64, device=dev)
+    rep = torch.empty(8, dtype=torch.int64, device=dev)
+    medusa.kernel_table_set(inp["table"])
+
+    def step():
+        medusa.kernel_table_set(inp["table"])
+        medusa.materialize_async(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=sl, result=res)
+        medusa.restore(inp["words"], sl, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                       dst=dst, func_out=fout, report=rep, from_table=True)
+
+    def rest():
+        medusa.restore(inp["words"], sl, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
+                       dst=dst, func_out=fout, report=rep, from_table=True)
+
+    graphs = {}
+    for name, fn in (("step", step), ("restore", rest)):
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            fn()
+        graphs[name] = g
+    for _ in range(3):
+        graphs["step"].replay()
+    torch.cuda.synchronize(dev)
+
+    def timed(g):
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        barrier()
+        for k in range(args.steps):
+            scrub.fill_(k)
+            ev[k][0].record(stream)
+            g.replay()
+            ev[k][1].record(stream)
+        barrier()
+        return [a.elapsed_time(b) for a, b in ev]
+
+    step_ms = timed(graphs["step"])
+    rest_ms = timed(graphs["restore"])
+    st, ns = medusa.mat_result(res)
+    assert st == 0 and ns == n_slots, (st, ns)
+    par = oracle_parity(gs, sl, n_slots, dst, fout, rep)
+    alg = algorithmic_bytes(gs, n_slots, gs.table.size)["restore"]
+    t_rest = statistics.median(rest_ms) / 1e3
+    out = {"rank": rank, "seed": seed, "nodes": gs.n_nodes, "words": gs.n_words, "slots": n_slots,
+           "sum_ms": sum(step_ms), "ms_per_step": statistics.median(step_ms),
+           "relocate_us": t_rest * 1e6, "relocate_GB/s": alg / t_rest / 1e9, "relocate_frac": alg / t_rest / 1e9 / peak,
+           "parity": par}
+    del graphs
+    if args.c5_sustained > 0:
+        R = args.c5_sustained
+        big = replicate(gs, R)
+        binp = medusa.upload(big, dev)
+        bsl = medusa.materialize(binp["words"], binp["node_off"], binp["node_t"], binp["allocs"])
+        medusa.kernel_table_set(binp["table"])
+        bdst = torch.empty_like(binp["words"])
+        bfout = torch.empty(big.n_nodes, dtype=torch.int64, device=dev)
+        brep = torch.empty(8, dtype=torch.int64, device=dev)
+        call = lambda: medusa.restore(binp["words"], bsl, binp["old_base"], binp["new_base"], binp["new_size"],
+                                      binp["func_id"], dst=bdst, func_out=bfout, report=brep)
+        for _ in range(2):
+            call()
+        torch.cuda.synchronize(dev)
+        assert int(medusa.report_numpy(brep)[0]) == 0
+        balg = algorithmic_bytes(big, bsl.n_slots, big.table.size)["restore"]
+        reps = 10
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        e0.record(stream)
+        for _ in range(reps):
+            call()
+        e1.record(stream)
+        barrier()
+        t = e0.elapsed_time(e1) / 1e3 / reps
+        out["sustained"] = {"replicas": R, "alg_bytes": balg, "avg_ms": t * 1e3, "GB/s": balg / t / 1e9,
+                            "frac_of_peak": balg / t / 1e9 / peak, "nodes_per_s": big.n_nodes / t}
+        medusa.kernel_table_set(inp["table"])
+        del binp, bsl, bdst, bfout, big
+        torch.cuda.empty_cache()
+    return out
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -421,8 +628,8 @@ def run_ours(args):
         raise SystemExit("bench.py needs a GPU (there is no CPU fallback)")
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
+    if ws > 1:  # host-side group only: barriers, max of device times, per-rank results (no NCCL)
+        dist.init_process_group("gloo", rank=rank, world_size=ws)
 
     cfg, desc = WORKLOADS[args.workload]
     seed = rank_seed(cfg, rank)
@@ -500,6 +707,9 @@ def run_ours(args):
     st_, ns_ = medusa.mat_result(res)
     assert st_ == 0 and ns_ == n_slots, (st_, ns_)
     assert int(medusa.report_numpy(grep)[0]) == 0 and torch.equal(gdst, dst) and torch.equal(gfout, fout)
+    head_parity = oracle_parity(gs, slots, n_slots, gdst, gfout, grep)  # this rank's instance vs the CPU oracle
+    assert head_parity["ok"], head_parity
+    scratch = medusa.scratch_bytes()
     sync_ms = timed(step)  # the same path through the synchronous API (host round trip after materialize)
     # the same K steps again with every libmedusa launch bracketed by events on its
     # stream: per-kernel durations for the roofline and the breakdown
@@ -531,7 +741,7 @@ def run_ours(args):
         d[1] += ms
     alg = algorithmic_bytes(gs, n_slots, gs.table.size)
     peak, peak_src = measured_peak()
-    traffic = load_traffic()
+    traffic = load_traffic(cfg)
     kernels = {}
     for name, (cnt, ms) in sorted(per.items(), key=lambda kv: -kv[1][1]):
         avg = ms / cnt
@@ -727,6 +937,26 @@ def run_ours(args):
     e2e_value = nodes_total / (max_over_ranks(e2e_ms, dist, dev) / 1e3)
     e2e_serial = nodes_total / (max_over_ranks(e2e_serial_ms, dist, dev) / 1e3)
 
+    # ---- C5: one Llama-2-13B-shaped instance per GPU, all GPUs at once ----
+    c5 = bench_c5(medusa, args, rank, dev, stream, scrub, barrier, peak) if args.c5 else None
+    if c5 is not None:
+        assert c5["parity"]["ok"], c5["parity"]
+    per_rank = gather_to_all({"rank": rank, "device": torch.cuda.get_device_name(dev), "seed": seed,
+                              "sum_ms": total_ms, "headline_parity": head_parity, "c5": c5}, dist)
+    multi = {"collective": "none: ranks meet only in a host-side gloo group (barriers, max of device times, "
+                           "this gather); no NCCL, nothing crosses GPUs",
+             "headline_per_rank": [{"rank": r["rank"], "seed": r["seed"], "ms_per_step": r["sum_ms"] / args.steps,
+                                    "parity": r["headline_parity"]} for r in per_rank]}
+    if c5 is not None:
+        c5s = [r["c5"] for r in per_rank]
+        c5_max_ms = max(c["sum_ms"] for c in c5s)
+        multi["c5"] = {
+            "workload": "C5: one Llama-2-13B-shaped instance per GPU (16,150 nodes, seed 100 + rank), whole path as "
+                        "one CUDA graph per step, L2 scrubbed before each step, all GPUs timed at once",
+            "aggregate_nodes_per_s": sum(c["nodes"] for c in c5s) * args.steps / (c5_max_ms / 1e3),
+            "ms_per_step": c5_max_ms / args.steps,
+            "per_gpu": c5s}
+
     # ---- CPU baseline: the oracle as it stands, rank 0 at N=1 only ----
     cpu = None
     if ws == 1 and not args.no_cpu_baseline:
@@ -767,10 +997,11 @@ def run_ours(args):
             "ms_per_step": max_ms / args.steps, "higher_is_better": True,
             "step_ms_p10_p50_p90": [float(np.percentile(step_ms, q)) for q in (10, 50, 90)], "scaling": "weak", "vs_baseline": None,
             "dtype": "u64", "data": "synthetic",
-            "config": {"workload": f"{cfg} per rank: {desc}", "nodes_per_rank": gs.n_nodes, "words": gs.n_words,
-                       "allocs": gs.n_alloc, "slots": n_slots, "kernel_names": int(gs.table.size),
-                       "l2": f"scrubbed before every timed step ({scrub.numel() * 4 >> 20} MiB write; L2 {l2 >> 20} MiB)",
-                       "seed": seed, "parallelism": f"{ws} independent instances, no collective"},
+            "config": config_dict(cfg, desc, gs, n_slots, rank_seed(cfg, 0), ws),
+            "multi_gpu": multi,
+            "scratch": {"bytes": scratch, "bytes_per_word": scratch / gs.n_words,
+                        "note": "library-owned materialize scratch of this device after the headline workload "
+                                "(medusa_scratch_bytes)"},
             "roofline": rl,
             "relocate": relocate,
             "materialize_ms": mat_s * 1e3,
@@ -807,7 +1038,7 @@ def run_ours(args):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--gpus", type=int, default=None, help="GPUs (default: WORLD_SIZE under torchrun, else 1)")
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
@@ -817,9 +1048,22 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-sets", type=int, default=2, help="buffer sets in the pipelined end-to-end leg")
     ap.add_argument("--no-buffers", dest="buffers", action="store_false")
+    ap.add_argument("--c5-sustained", type=int, default=256,
+                    help="replicas of the per-GPU C5 instance in its sustained-relocate call (0: skip)")
+    ap.add_argument("--no-c5", dest="c5", action="store_false", help="skip the per-GPU C5 block")
+    ap.add_argument("--selftest-plumbing", action="store_true", help=argparse.SUPPRESS)
     args = ap.parse_args()
+    ws_env = os.environ.get("WORLD_SIZE")
+    if args.gpus is None:
+        args.gpus = int(ws_env) if ws_env else 1
+    if ws_env is not None and int(ws_env) != args.gpus:
+        raise SystemExit(f"bench.py --gpus {args.gpus} under a launcher with WORLD_SIZE={ws_env}")
     if args.impl == "reference":
-        run_reference(args)
+        run_reference(args)  # rank 0 only: the CPU oracle (other ranks exit at once)
+    elif ws_env is None and args.gpus > 1:
+        spawn_ranks(args, n_visible=args.gpus if args.selftest_plumbing else None)
+    elif args.selftest_plumbing:
+        plumbing_selftest(args)
     else:
         run_ours(args)
 

@@ -1,6 +1,7 @@
 """Multi-process host logic (gloo, world size 2, CPU): every rank restores its own
 instance (distinct seeds, no data exchange) and the job time is the max over
-ranks -- the same helpers bench.py uses under torchrun with NCCL."""
+ranks -- the same helpers and the same gloo group bench.py uses (no NCCL);
+bench.py --gpus 2 starts its own rank processes when no launcher did."""
 import json
 import os
 import socket
@@ -54,3 +55,45 @@ def test_reference_arm_runs_on_cpu():
     d = json.loads(r.stdout.strip().splitlines()[-1])
     assert d["impl"] == "reference" and d["unit"] == "nodes/s" and d["value"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_bench_launches_its_own_ranks_over_gloo():
+    """`bench.py --gpus 2` outside torchrun: two rank processes with the launcher's
+    environment, a gloo group, the max over ranks and the gather (plumbing only)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--selftest-plumbing"],
+                       capture_output=True, text=True, cwd=ROOT, timeout=300, env=env)
+    assert r.returncode == 0, r.stderr
+    d = json.loads(r.stdout.strip().splitlines()[-1])
+    assert d["world_size"] == 2 and d["max_ms"] == 11.0
+    assert [x["rank"] for x in d["ranks"]] == [0, 1] and [x["local"] for x in d["ranks"]] == [0, 1]
+    assert d["ranks"][0]["pid"] != d["ranks"][1]["pid"]
+    assert [x["seed_c5"] for x in d["ranks"]] == [100, 101]  # C5: seed 100 + gpu (SURVEY.md §8(d))
+    assert d["ranks"][0]["seed_all10"] != d["ranks"][1]["seed_all10"]
+
+
+def test_launcher_world_size_must_match_gpus():
+    env = dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--selftest-plumbing"],
+                       capture_output=True, text=True, cwd=ROOT, timeout=300, env=env)
+    assert r.returncode != 0 and "WORLD_SIZE=2" in r.stderr
+
+
+def test_reference_arm_config_equals_ours():
+    """The reference arm prints the config object bench.py's own arm builds for the
+    same workload (same keys and values; the slot count is the oracle's, which the
+    GPU arm's parity check equals)."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--workload", "toy",
+                        "--steps", "1", "--warmup", "1", "--gpus", "2"], capture_output=True, text=True, cwd=ROOT,
+                       timeout=300, env={k: v for k, v in os.environ.items() if k != "WORLD_SIZE"})
+    assert r.returncode == 0, r.stderr
+    d = json.loads(r.stdout.strip().splitlines()[-1])
+    sys.path.insert(0, ROOT)
+    import bench
+    import oracle
+    from workloads import make_graph_set
+    seed = bench.rank_seed("toy", 0)
+    gs = make_graph_set("toy", seed=seed)
+    n_slots = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)["n_slots"]
+    ours = bench.config_dict("toy", bench.WORKLOADS["toy"][1], gs, n_slots, seed, 2)
+    assert d["config"] == ours and d["n_gpus"] == 2

@@ -1,5 +1,9 @@
 """profiles/ncu_traffic.json from an ncu launch list with dram__bytes_{read,write}.sum:
-per-launch DRAM bytes of the last launch of each kernel, keyed by bench.py's names."""
+per-launch DRAM bytes of the last launch of each kernel, keyed by bench.py's names,
+stored under the workload the launch list ran (bench.py reads only its own).
+
+  python tools/make_traffic.py LAUNCHES.csv OUT.json WORKLOAD   (OUT.json is merged into)"""
+import os
 import csv
 import json
 import sys
@@ -40,5 +44,8 @@ out["_inst"] = inst  # warp instructions per launch (smsp__inst_executed.sum), s
 out["_note"] = ("per-launch dram__bytes_read.sum + dram__bytes_write.sum of the last bench step in the ncu launch "
                 f"list {sys.argv[1].split('/')[-1]} (--clock-control none; ncu flushes caches between launches, so "
                 "this is cold-cache traffic)")
-json.dump(out, open(sys.argv[2], "w"), indent=1)
+wl = sys.argv[3] if len(sys.argv) > 3 else "all10"
+allw = json.load(open(sys.argv[2])) if os.path.exists(sys.argv[2]) else {}
+allw[wl] = out
+json.dump(allw, open(sys.argv[2], "w"), indent=1)
 print(json.dumps(out, indent=1))
