@@ -53,7 +53,7 @@ namespace {
 
 MEDUSA_TL_DEFINE
 
-constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
+constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
@@ -72,7 +72,6 @@ struct Ctl {
     unsigned int pad1;
     unsigned long long gmin_c;  // ~(least base) via atomicMax
     unsigned long long gmax;    // greatest end
-    unsigned long long need_c, need_b;  // set (exactly) only when a registration list overflowed
     unsigned long long n_slots;
 };
 
@@ -88,29 +87,27 @@ struct IQ {  // a candidate word for the I-list search (k_iresolve)
     uint32_t t;  // launch position of its node
 };
 
-struct WinRec {  // a registered mortal allocation
-    uint64_t base;
-    uint64_t end;
-    uint32_t t_alloc;
-    uint32_t t_free;
-    uint32_t id;
-    uint32_t pad;
+// The mortal tree: a 32-ary max tree over allocation ordinals.
+// Leaf i = {v_i, t_alloc_i} with v_i = t_free_i for a mortal (non-empty, not in
+// I) and 0 otherwise; node k of level l >= 1 covers ordinals [k 32^l, (k+1) 32^l)
+// and holds {max v, t_alloc of its first ordinal}.  "The mortals allocated before
+// T1 and freed after T0" is a descent that keeps the nodes with max v > T0 and
+// first t_alloc < T1 (t_alloc increases with the ordinal on a well-formed trace).
+constexpr int kMaxLevels = 6;  // 32^5 > 2^24 allocations
+struct Tree {
+    uint2* leaf;                  // [n]
+    uint2* node;                  // levels 1..top, level l at node + off[l]
+    uint32_t off[kMaxLevels + 1]; // off[1] = 0
+    uint32_t cnt[kMaxLevels + 1]; // nodes of level l (cnt[0] = n)
+    uint32_t top;                 // the level with <= 32 nodes (0 if n <= 32)
 };
 
 struct Dev {  // scratch of one call (device pointers)
     Ctl* ctl;
     uint32_t *jf, *jl;                           // [C] first / last node of each chunk
-    uint4* rng;                                  // [n]: c_lo, c_hi, b_lo, b_hi
-    // two-level registration counters (zeroed): cnt[k] per chunk / check block,
-    // sup[g] = sum of cnt over the 256 keys of group g, so any prefix sum is one
-    // CTA-wide reduction (block_prefix) and no serial scan is needed
-    uint32_t *cnt_c, *fill_c;                    // [C+1]
-    uint32_t *cnt_b, *fill_b;                    // [nb+1]
-    unsigned long long *sup_c, *sup_b;           // [C/256+1], [nb/256+1]
+    Tree tree;
     unsigned long long* chunk_sup;               // [C/256+1] slots per 256 chunks
     uint32_t *blk_min_ta_c, *blk_max_tf;         // [n/32+1] (zeroed; min kept as ~max(~t))
-    WinRec *list_c, *list_b;
-    uint64_t cap_c, cap_b;
     uint64_t* sk[2];                             // [n] sort keys: 0 unsorted, 1 sorted tiles
     uint32_t* sv[2];                             // [n] sort values (allocation index)
     uint64_t* samp_k;                            // [n/32+1] every 32nd key of each sorted tile
@@ -129,10 +126,8 @@ struct Dev {  // scratch of one call (device pointers)
 struct P {  // kernel parameters
     MaterializeArgs a;
     Dev d;
-    uint32_t C, nb;              // chunks, check blocks
+    uint32_t C, nb;              // chunks, check blocks (32 ordinals each)
     uint32_t node_ctas;          // k_trace: CTAs with the node role
-    uint32_t sort_ctas;          // k_prepare: CTAs with the sort role (bound: allocation count / kSortTile)
-    uint32_t check_ctas;         // k_scan_words: CTAs with the check role (after the C classify CTAs)
 };
 
 __device__ __forceinline__ void flag(Ctl* c, unsigned int bit) { atomicOr(&c->status, bit); }
@@ -154,58 +149,6 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
 
 __device__ __forceinline__ uint32_t n_tiles(uint32_t nI) { return (nI + kSortTile - 1) / kSortTile; }
 __device__ __forceinline__ uint32_t fence_stride(uint32_t nI) { return nI ? (nI + kFenceCap - 1) / kFenceCap : 1; }
-
-// Exclusive scan of one value per thread over the CTA (blockDim.x == kThreads);
-// *total = the sum.  Call with the whole CTA.
-__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* total) {
-    __shared__ uint32_t s_w[kWarps];
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t x = v;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
-        if (lane >= (uint32_t)d) x += y;
-    }
-    if (lane == 31) s_w[warp] = x;
-    __syncthreads();
-    uint32_t before = 0, tot = 0;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) {
-        const uint32_t t = s_w[w];
-        if ((uint32_t)w < warp) before += t;
-        tot += t;
-    }
-    __syncthreads();  // s_w may be rewritten by the next call
-    *total = tot;
-    return before + x - v;
-}
-
-// block_excl_scan of two independent values at once (one pair of barriers)
-__device__ __forceinline__ void block_excl_scan2(uint32_t v0, uint32_t v1, uint32_t& e0, uint32_t& e1, uint32_t& t0,
-                                                 uint32_t& t1) {
-    __shared__ uint32_t s_w2[2][kWarps];
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t x0 = v0, x1 = v1;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y0 = __shfl_up_sync(0xffffffffu, x0, d), y1 = __shfl_up_sync(0xffffffffu, x1, d);
-        if (lane >= (uint32_t)d) { x0 += y0; x1 += y1; }
-    }
-    if (lane == 31) { s_w2[0][warp] = x0; s_w2[1][warp] = x1; }
-    __syncthreads();
-    uint32_t b0 = 0, b1 = 0;
-    t0 = t1 = 0;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) {
-        const uint32_t a0 = s_w2[0][w], a1 = s_w2[1][w];
-        if ((uint32_t)w < warp) { b0 += a0; b1 += a1; }
-        t0 += a0;
-        t1 += a1;
-    }
-    __syncthreads();
-    e0 = b0 + x0 - v0;
-    e1 = b1 + x1 - v1;
-}
 
 // Sum of cnt[0, k) of a two-level counter (sup[g] = sum of cnt[256g, 256g + 256)):
 // at most k/256 + 255 loads, spread over the CTA, and one reduction; every thread
@@ -231,108 +174,18 @@ __device__ __forceinline__ unsigned long long block_prefix(const uint32_t* cnt, 
     return t;
 }
 
-// block_prefix of two counters at once (one reduction)
-__device__ __forceinline__ void block_prefix2(const uint32_t* cnt0, const unsigned long long* sup0, uint32_t k0,
-                                              const uint32_t* cnt1, const unsigned long long* sup1, uint32_t k1,
-                                              unsigned long long& r0, unsigned long long& r1) {
-    __shared__ unsigned long long s_r2[2][kWarps];
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    unsigned long long a0 = 0, a1 = 0;
-    const uint32_t g0 = k0 >> 8, g1 = k1 >> 8;
-    for (uint32_t q = threadIdx.x; q < g0; q += kThreads) a0 += __ldcg(sup0 + q);
-    for (uint32_t q = threadIdx.x; q < g1; q += kThreads) a1 += __ldcg(sup1 + q);
-    if ((g0 << 8) + threadIdx.x < k0) a0 += __ldcg(cnt0 + (g0 << 8) + threadIdx.x);
-    if ((g1 << 8) + threadIdx.x < k1) a1 += __ldcg(cnt1 + (g1 << 8) + threadIdx.x);
-#pragma unroll
-    for (int d = 16; d > 0; d >>= 1) {
-        a0 += __shfl_xor_sync(0xffffffffu, a0, d);
-        a1 += __shfl_xor_sync(0xffffffffu, a1, d);
-    }
-    if (lane == 0) { s_r2[0][warp] = a0; s_r2[1][warp] = a1; }
-    __syncthreads();
-    r0 = r1 = 0;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) { r0 += s_r2[0][w]; r1 += s_r2[1][w]; }
-    __syncthreads();
+// one allocation record through the read-only path
+__device__ __forceinline__ medusa_alloc ld_alloc(const medusa_alloc* q) {
+    const unsigned long long* w = reinterpret_cast<const unsigned long long*>(q);
+    const unsigned long long b = __ldg(w), z = __ldg(w + 1), t = __ldg(w + 2);
+    medusa_alloc x;
+    x.base = b;
+    x.size = z;
+    x.t_alloc = (uint32_t)t;
+    x.t_free = (uint32_t)(t >> 32);
+    return x;
 }
 
-// first index k in [lo, n) with t[k] >= x (galloping from lo; t ascending)
-__device__ __forceinline__ uint32_t gallop_ge(const uint32_t* t, uint32_t lo, uint32_t n, uint32_t x) {
-    uint32_t step = 1, prev = lo, hi = lo;
-    while (hi < n && t[hi] < x) { prev = hi + 1; hi = hi + step; step <<= 1; }
-    if (hi > n) hi = n;
-    uint32_t l = prev;
-    while (l < hi) { const uint32_t m = (l + hi) >> 1; if (t[m] < x) l = m + 1; else hi = m; }
-    return l;
-}
-__device__ __forceinline__ uint32_t gallop_alloc_ge(const medusa_alloc* al, uint32_t lo, uint32_t n, uint32_t x) {
-    uint32_t step = 1, prev = lo, hi = lo;
-    while (hi < n && al[hi].t_alloc < x) { prev = hi + 1; hi = hi + step; step <<= 1; }
-    if (hi > n) hi = n;
-    uint32_t l = prev;
-    while (l < hi) { const uint32_t m = (l + hi) >> 1; if (al[m].t_alloc < x) l = m + 1; else hi = m; }
-    return l;
-}
-
-// count of entries <= x in the ascending u32 array t[0, n) (warp-cooperative
-// 32-ary search: ~4 dependent global rounds for 10^5 entries; all lanes agree)
-__device__ __forceinline__ uint32_t warp_count_le(const uint32_t* t, uint32_t n, uint32_t x) {
-    const uint32_t lane = threadIdx.x & 31;
-    uint32_t lo = 0, hi = n;  // the count lies in [lo, hi]
-    while (hi - lo > 32) {
-        const uint32_t step = (hi - lo + 31) / 32;
-        const uint32_t pr = lo + lane * step;
-        const bool le = pr < hi && t[pr] <= x;
-        const uint32_t b = __ballot_sync(0xffffffffu, le);
-        const uint32_t k = __popc(b);  // probes <= x form a prefix
-        if (k == 0) return lo;
-        const uint32_t last_le = lo + (k - 1) * step;
-        const uint32_t next = lo + k * step;
-        lo = last_le + 1;
-        if (next < hi) hi = next;
-    }
-    const uint32_t pr = lo + lane;
-    return lo + __popc(__ballot_sync(0xffffffffu, pr < hi && t[pr] <= x));
-}
-
-// atomicAdd(&ctr[key], 1) for every active lane, one atomic per distinct key in the
-// warp; returns the previous value + this lane's rank among the lanes with its key
-__device__ __forceinline__ uint32_t warp_agg_inc(uint32_t* ctr, uint32_t key, bool active) {
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t peers = __match_any_sync(0xffffffffu, active ? key : 0xFFFFFFFFu);
-    const uint32_t leader = __ffs(peers) - 1;
-    uint32_t base = 0;
-    if (active && lane == leader) base = atomicAdd(ctr + key, (uint32_t)__popc(peers));
-    base = __shfl_sync(0xffffffffu, base, leader);
-    return base + __popc(peers & lanemask_lt());
-}
-
-// ctr[key] += 1 for every active lane, one fire-and-forget atomic per distinct key
-__device__ __forceinline__ void warp_agg_add(uint32_t* ctr, uint32_t key, bool active) {
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t peers = __match_any_sync(0xffffffffu, active ? key : 0xFFFFFFFFu);
-    if (active && lane == __ffs(peers) - 1) atomicAdd(ctr + key, (uint32_t)__popc(peers));
-}
-
-// sup[g] += |[lo, hi] ∩ group g| for every 256-key group g the active lanes'
-// ranges meet; one atomic per distinct group of the warp (full-warp call)
-__device__ __forceinline__ void warp_group_add_range(unsigned long long* sup, uint32_t lo, uint32_t hi, bool active) {
-    const uint32_t g0 = active ? lo >> 8 : 0, g1 = active ? hi >> 8 : 0;
-    const uint32_t ng = __reduce_max_sync(0xffffffffu, active ? g1 - g0 + 1 : 0u);
-    for (uint32_t k = 0; k < ng; ++k) {
-        const uint32_t g = g0 + k;
-        const bool act = active && g <= g1;
-        const uint32_t n = act ? min(hi, g * 256 + 255) - max(lo, g * 256) + 1 : 0u;
-        uint32_t key = act ? g : 0xFFFFFFFFu;
-        while (true) {
-            const uint32_t gm = __reduce_min_sync(0xffffffffu, key);
-            if (gm == 0xFFFFFFFFu) break;
-            const uint32_t sum = __reduce_add_sync(0xffffffffu, key == gm ? n : 0u);
-            if ((threadIdx.x & 31) == 0) atomicAdd(sup + gm, (unsigned long long)sum);
-            if (key == gm) key = 0xFFFFFFFFu;
-        }
-    }
-}
 
 // ----------------------------------------------------------------------------
 // 1. k_trace
@@ -359,111 +212,51 @@ __device__ void nodes_role(const P& p, uint64_t i) {
     }
 }
 
-constexpr int kTWinN = 2048;  // node times staged per alloc CTA
-constexpr int kTWinA = 1024;  // allocation times staged per alloc CTA (2048: +1.3 us of k_trace, ALL10)
 constexpr int kNodesPerThread = 4;  // node role of k_trace (keeps its grid inside one wave)
 
+// One allocation per thread: the trace checks (R-Q7, R-Q9), the I / M split, the
+// mortal tree (leaf, level 1 by the warp, higher levels by one atomic per CTA),
+// the I compaction and the prefilter bounds.  One coalesced record load, no search.
 __device__ void allocs_role(const P& p, uint32_t cta) {
-    __shared__ uint32_t s_nt[kTWinN];  // node_t[nj0, nj0 + nw)
-    __shared__ uint32_t s_at[kTWinA];  // t_alloc of allocations [i0, i0 + na)
-    __shared__ uint32_t s_nj0;
+    const MaterializeArgs& a = p.a;
+    const Tree& T = p.d.tree;
     const uint32_t i0 = cta * blockDim.x;
     const uint32_t i = i0 + threadIdx.x;
-    const MaterializeArgs& a = p.a;
-    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t N = a.n_nodes;
     const bool valid = i < a.n_alloc;
     unsigned long long tl_p = TL_NOW();
     medusa_alloc x{};
-    if (valid) x = a.alloc[i];
-    const uint32_t t_last = N ? a.node_t[N - 1] : 0;
-    // the node times around this CTA's allocations, and the allocation times after them
-    if (threadIdx.x < 32) {
-        const uint32_t ta0 = a.alloc[i0].t_alloc;
-        const uint32_t nj0 = N ? warp_count_le(a.node_t, N, ta0) : 0;
-        if (lane == 0) s_nj0 = nj0;
-    }
-    __syncthreads();
-    TL_PHASE(1, 20, tl_p);  // record load, node-window start
-    const uint32_t nj0 = s_nj0;
-    const uint32_t nw = min((uint32_t)kTWinN, N - nj0);
-    const uint32_t na = (uint32_t)min((uint64_t)kTWinA, (uint64_t)a.n_alloc - i0);
-    for (uint32_t k = threadIdx.x; k < nw; k += blockDim.x) s_nt[k] = a.node_t[nj0 + k];
-    for (uint32_t k = threadIdx.x; k < na; k += blockDim.x) s_at[k] = a.alloc[i0 + k].t_alloc;
-    __syncthreads();
-    TL_PHASE(1, 21, tl_p);  // time windows staged
+    if (valid) x = ld_alloc(a.alloc + i);
+    const uint32_t t_last = N ? __ldg(a.node_t + N - 1) : 0;
+    uint32_t ta_next = __shfl_down_sync(0xffffffffu, x.t_alloc, 1);  // the next ordinal's t_alloc
+    if (lane == 31 && i + 1 < a.n_alloc) ta_next = (uint32_t)__ldg(reinterpret_cast<const unsigned long long*>(a.alloc + i + 1) + 2);
     bool isI = false;
-    uint4 r = make_uint4(1, 0, 1, 0);  // empty ranges
-    bool reg_c = false, reg_b = false;
+    uint32_t v = 0;  // leaf value: t_free of a mortal, else 0
     if (valid) {
         if (x.size > (1ull << MEDUSA_OFF_BITS) || x.base + x.size < x.base) flag(p.d.ctl, ST_INVALID);
         if (!(x.t_alloc < x.t_free)) flag(p.d.ctl, ST_TRACE);
-        if (i + 1 < a.n_alloc && !(x.t_alloc < a.alloc[i + 1].t_alloc)) flag(p.d.ctl, ST_TRACE);
+        if (i + 1 < a.n_alloc && !(x.t_alloc < ta_next)) flag(p.d.ctl, ST_TRACE);
         if (x.size != 0) {
             isI = N && x.t_alloc < t_last && t_last < x.t_free;
-            if (!isI) {
-                if (p.C && N && x.t_alloc < x.t_free) {
-                    // nodes launched while i is live: [j0, j1) = t in (t_alloc, t_free)
-                    uint32_t lo = 0, hi = nw;  // window entries <= t_alloc
-                    while (lo < hi) { uint32_t m = (lo + hi) >> 1; if (s_nt[m] <= x.t_alloc) lo = m + 1; else hi = m; }
-                    uint32_t j0;
-                    if (lo < nw) {
-                        j0 = nj0 + lo;
-                    } else {  // beyond the staged window (or the trace is not ordered)
-                        uint32_t l2 = nj0 + nw, h2 = N;
-                        while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (a.node_t[m] <= x.t_alloc) l2 = m + 1; else h2 = m; }
-                        j0 = l2;
-                    }
-                    uint32_t j1;
-                    if (j0 < nj0 + nw && nw && x.t_free <= s_nt[nw - 1]) {
-                        uint32_t l2 = j0 - nj0, h2 = nw;  // first entry >= t_free
-                        while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (s_nt[m] < x.t_free) l2 = m + 1; else h2 = m; }
-                        j1 = nj0 + l2;
-                    } else {
-                        j1 = gallop_ge(a.node_t, max(j0, nj0 + nw), N, x.t_free);
-                    }
-                    // chunks holding their words (exact: no entry for memory no launch can see)
-                    if (j0 < j1) {
-                        const uint64_t w0 = a.node_off[j0], w1 = a.node_off[j1];
-                        if (w0 < w1 && w1 <= a.n_words) {
-                            r.x = (uint32_t)(w0 / kChunkWords);
-                            r.y = (uint32_t)((w1 - 1) / kChunkWords);
-                            reg_c = true;
-                        }
-                    }
-                }
-                // ordinals allocated while i is live: (i, u), u = #{k : t_alloc_k < t_free_i}
-                uint32_t u;
-                if (na && x.t_free <= s_at[na - 1]) {
-                    uint32_t l2 = i - i0 + 1, h2 = na;
-                    while (l2 < h2) { uint32_t m = (l2 + h2) >> 1; if (s_at[m] < x.t_free) l2 = m + 1; else h2 = m; }
-                    u = i0 + l2;
-                } else {
-                    u = gallop_alloc_ge(a.alloc, max(i + 1, i0 + na), a.n_alloc, x.t_free);
-                }
-                if (i + 1 < u) {
-                    r.z = (i + 1) / kAblk; r.w = (u - 1) / kAblk;
-                    reg_b = true;
-                }
-            }
+            if (!isI) v = x.t_free;
         }
-        p.d.rng[i] = r;
+        T.leaf[i] = make_uint2(v, x.t_alloc);
     }
-    // registration counts (one atomic per distinct key of the warp) and their
-    // 256-key group sums
-    {
-        const uint32_t lc = reg_c ? r.y - r.x + 1 : 0, lb = reg_b ? r.w - r.z + 1 : 0;
-        const uint32_t mc = __reduce_max_sync(0xffffffffu, lc), mbk = __reduce_max_sync(0xffffffffu, lb);
-        for (uint32_t k = 0; k < mc; ++k) warp_agg_add(p.d.cnt_c, r.x + k, k < lc);
-        for (uint32_t k = 0; k < mbk; ++k) warp_agg_add(p.d.cnt_b, r.z + k, k < lb);
-        warp_group_add_range(p.d.sup_c, r.x, r.y, reg_c);
-        warp_group_add_range(p.d.sup_b, r.z, r.w, reg_b);
-    }
+    TL_PHASE(1, 20, tl_p);  // record load, checks
+    // the mortal tree above the leaves: level 1 = this warp's 32 ordinals
+    const uint32_t wmax = __reduce_max_sync(0xffffffffu, v);
+    if (T.top >= 1 && lane == 0 && valid) T.node[T.off[1] + (i >> 5)] = make_uint2(wmax, x.t_alloc);
+    // levels >= 2: the first ordinal's t_alloc directly, the max by one atomic per CTA
+    // (a CTA's 256 ordinals lie inside one node of every level >= 2)
+    for (uint32_t l = 2; l <= T.top; ++l)
+        if (valid && (i & ((1u << (5 * l)) - 1)) == 0) T.node[T.off[l] + (i >> (5 * l))].y = x.t_alloc;
     // CTA-aggregated (one global atomic per CTA, not per warp: these are the same
     // three addresses for every CTA): I positions, global prefilter bounds
-    __shared__ uint32_t s_ni, s_base;
+    __shared__ uint32_t s_ni, s_base, s_wmax[kWarps];
     __shared__ unsigned long long s_mn, s_mx;
     if (threadIdx.x == 0) { s_ni = 0; s_mn = ~0ull; s_mx = 0; }
+    if (lane == 0) s_wmax[warp] = wmax;
     __syncthreads();
     const uint32_t bal = __ballot_sync(0xffffffffu, isI);
     uint32_t wpos = 0;
@@ -482,6 +275,11 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
             atomicMax(&p.d.ctl->gmin_c, ~s_mn);
             atomicMax(&p.d.ctl->gmax, s_mx);
         }
+        uint32_t cmax = 0;
+#pragma unroll
+        for (int w = 0; w < kWarps; ++w) cmax = max(cmax, s_wmax[w]);
+        if (cmax)
+            for (uint32_t l = 2; l <= T.top; ++l) atomicMax(&T.node[T.off[l] + (i0 >> (5 * l))].x, cmax);
     }
     __syncthreads();
     wpos = __shfl_sync(0xffffffffu, wpos, 0);
@@ -490,7 +288,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         p.d.sk[0][pos] = x.base;
         p.d.sv[0][pos] = i;
     }
-    TL_PHASE(1, 22, tl_p);  // searches, registration counts, I compaction
+    TL_PHASE(1, 22, tl_p);  // tree, I compaction
 }
 
 __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
@@ -509,60 +307,9 @@ __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 2. k_prepare: sort tiles of I keys by (base, index) | registration lists
-
-// Bitonic sort of 32*E (key, val) pairs held E per lane (element e = lane*E + r),
-// ascending by (key, val), carrying a payload; shuffles and register
-// compare-exchanges only (no shared memory).
-template <int E>
-__device__ __forceinline__ void warp_bitonic(uint64_t (&k)[E], uint32_t (&v)[E], uint32_t (&pl)[E]) {
-    const uint32_t lane = threadIdx.x & 31;
-#pragma unroll
-    for (uint32_t size = 2; size <= 32u * E; size <<= 1) {
-#pragma unroll
-        for (uint32_t j = size >> 1; j > 0; j >>= 1) {
-            if (j >= (uint32_t)E) {
-                const uint32_t lj = j / E;
-#pragma unroll
-                for (int r = 0; r < E; ++r) {
-                    const uint32_t e = lane * E + r;
-                    const uint64_t ok = __shfl_xor_sync(0xffffffffu, k[r], lj);
-                    const uint32_t ov = __shfl_xor_sync(0xffffffffu, v[r], lj);
-                    const uint32_t op = __shfl_xor_sync(0xffffffffu, pl[r], lj);
-                    const bool up = (e & size) == 0;
-                    const bool lower = (e & j) == 0;
-                    const bool other_less = kv_less(ok, ov, k[r], v[r]);
-                    // lower element keeps the min when ascending, the max when descending
-                    if ((lower == up) ? other_less : !other_less) { k[r] = ok; v[r] = ov; pl[r] = op; }
-                }
-            } else {
-#pragma unroll
-                for (int r = 0; r < E; ++r) {
-                    const int r2 = r ^ (int)j;
-                    if (r2 > r && kv_less(k[r2], v[r2], k[r], v[r]) == (((lane * E + r) & size) == 0)) {
-                        const uint64_t tk = k[r]; k[r] = k[r2]; k[r2] = tk;
-                        const uint32_t tv = v[r]; v[r] = v[r2]; v[r2] = tv;
-                        const uint32_t tp = pl[r]; pl[r] = pl[r2]; pl[r2] = tp;
-                    }
-                }
-            }
-        }
-    }
-}
+// 2. k_isort: sort tiles of I keys by (base, index)
 
 // the I entry of sorted position r: arrays, fence, block summaries
-// one allocation record through the read-only path
-__device__ __forceinline__ medusa_alloc ld_alloc(const medusa_alloc* q) {
-    const unsigned long long* w = reinterpret_cast<const unsigned long long*>(q);
-    const unsigned long long b = __ldg(w), z = __ldg(w + 1), t = __ldg(w + 2);
-    medusa_alloc x;
-    x.base = b;
-    x.size = z;
-    x.t_alloc = (uint32_t)t;
-    x.t_free = (uint32_t)(t >> 32);
-    return x;
-}
-
 __device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t nI, uint32_t id, const medusa_alloc& x) {
     p.d.i_base[r] = x.base;
     p.d.i_rest[r] = IRest{x.base + x.size, x.t_alloc, id};
@@ -609,8 +356,7 @@ __device__ __forceinline__ void warp_bitonic_kv(uint64_t (&k)[E], uint32_t (&v)[
 }
 
 // ----------------------------------------------------------------------------
-// 2a. sort role of k_prepare (its first CTAs, dispatched ahead of the scatter
-//     CTAs): one tile of kSortTile I keys (base, allocation index) per CTA.  A
+// 2a. sort role: one tile of kSortTile I keys (base, allocation index) per CTA.  A
 //     register bitonic sort of 128 keys per warp, then three merge-path rounds
 //     through shared memory (128 -> 256 -> 512 -> 1024), four keys per thread held
 //     in registers between rounds.  A single tile is the whole list: its I entries
@@ -693,123 +439,14 @@ __device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
     }
 }
 
-// Registration lists (l = 0: chunks, l = 1: check blocks): allocation i of the
-// CTA registers in keys [lo_l, hi_l] (empty when lo > hi).  Both lists are built
-// in the same pass (shared barriers and load rounds).  Keys are handled in tiles
-// of 256: a tile's list offsets = group prefix (block_prefix2) + a CTA scan of
-// the counts; the tile's (allocation, key) pairs of both lists are dealt out
-// evenly over the CTA, so one long-lived allocation does not serialize its warp.
-struct ScatterShared {
-    uint32_t off[2][kThreads], pre[2][kThreads], first[2][kThreads], range[2][2];
-    WinRec w[kThreads];
-};
-
-__device__ void scatter_role(const P& p, uint32_t cta, ScatterShared& S) {
-    const uint32_t tid = threadIdx.x;
-    const uint32_t i = cta * kThreads + tid;
-    const bool valid = i < p.a.n_alloc;
-    uint4 r = make_uint4(1, 0, 1, 0);
-    if (valid) r = p.d.rng[i];
-    WinRec w{};
-    if (r.x <= r.y || r.z <= r.w) {
-        const medusa_alloc x = ld_alloc(p.a.alloc + i);
-        w = WinRec{x.base, x.base + x.size, x.t_alloc, x.t_free, i, 0};
-    }
-    const uint32_t lo_i[2] = {r.x, r.z}, hi_i[2] = {r.y, r.w};
-    const uint32_t* cnt[2] = {p.d.cnt_c, p.d.cnt_b};
-    if (tid < 2) { S.range[tid][0] = 0xFFFFFFFFu; S.range[tid][1] = 0; }
-    S.w[tid] = w;
-    __syncthreads();
-#pragma unroll
-    for (int l = 0; l < 2; ++l) {
-        const bool has = lo_i[l] <= hi_i[l];
-        const uint32_t mn = __reduce_min_sync(0xffffffffu, has ? lo_i[l] : 0xFFFFFFFFu);
-        const uint32_t mx = __reduce_max_sync(0xffffffffu, has ? hi_i[l] : 0u);
-        if ((tid & 31) == 0 && mn <= mx) { atomicMin(&S.range[l][0], mn); atomicMax(&S.range[l][1], mx); }
-    }
-    __syncthreads();
-    const uint32_t lo[2] = {S.range[0][0], S.range[1][0]}, hi[2] = {S.range[0][1], S.range[1][1]};
-    const bool any[2] = {lo[0] <= hi[0], lo[1] <= hi[1]};
-    if (!any[0] && !any[1]) return;  // whole CTA
-    unsigned long long base[2];
-    block_prefix2(cnt[0], p.d.sup_c, any[0] ? lo[0] : 0, cnt[1], p.d.sup_b, any[1] ? lo[1] : 0, base[0], base[1]);
-    const uint32_t ntile = max(any[0] ? (hi[0] - lo[0]) / kThreads + 1 : 0u, any[1] ? (hi[1] - lo[1]) / kThreads + 1 : 0u);
-    for (uint32_t t = 0; t < ntile; ++t) {
-        uint32_t t0[2], v[2], len[2], a_[2];
-#pragma unroll
-        for (int l = 0; l < 2; ++l) {
-            t0[l] = lo[l] + t * kThreads;
-            const uint32_t key = t0[l] + tid;
-            v[l] = (any[l] && key <= hi[l]) ? __ldcg(cnt[l] + key) : 0u;
-            const uint32_t a = max(lo_i[l], t0[l]), b = min(hi_i[l], t0[l] + kThreads - 1);
-            len[l] = (any[l] && lo_i[l] <= hi_i[l] && a <= b) ? b - a + 1 : 0u;
-            a_[l] = a;
-        }
-        uint32_t ex0, ex1, tot0, tot1;
-        block_excl_scan2(v[0], v[1], ex0, ex1, tot0, tot1);
-        S.off[0][tid] = (uint32_t)min(base[0] + ex0, 0xFFFFFFFFull);
-        S.off[1][tid] = (uint32_t)min(base[1] + ex1, 0xFFFFFFFFull);
-        base[0] += tot0;
-        base[1] += tot1;
-        uint32_t p0, p1, np0, np1;
-        block_excl_scan2(len[0], len[1], p0, p1, np0, np1);
-        S.pre[0][tid] = p0;
-        S.pre[1][tid] = p1;
-        S.first[0][tid] = a_[0];
-        S.first[1][tid] = a_[1];
-        __syncthreads();
-        const uint32_t total = np0 + np1;
-        for (uint32_t q0 = 0; q0 < total; q0 += kThreads) {
-            const uint32_t q = q0 + tid;
-            const bool act = q < total;
-            const uint32_t l = q < np0 ? 0u : 1u;
-            const uint32_t qq = l ? q - np0 : q;
-            uint32_t own = 0, k = 0;
-            if (act) {  // owner: last thread whose pair range starts at or before qq
-                const uint32_t* pre = S.pre[l];
-                uint32_t lo2 = 0, hi2 = kThreads;
-                while (hi2 - lo2 > 1) { const uint32_t m = (lo2 + hi2) >> 1; if (pre[m] <= qq) lo2 = m; else hi2 = m; }
-                own = lo2;
-                k = S.first[l][own] + (qq - pre[own]);
-            }
-            // one atomic per distinct (list, key) of the warp
-            const uint32_t tag = act ? (k | (l << 31)) : 0xFFFFFFFFu;
-            const uint32_t peers = __match_any_sync(0xffffffffu, tag);
-            const uint32_t leader = __ffs(peers) - 1;
-            uint32_t rb = 0;
-            if (act && (tid & 31) == leader) rb = atomicAdd((l ? p.d.fill_b : p.d.fill_c) + k, (uint32_t)__popc(peers));
-            rb = __shfl_sync(0xffffffffu, rb, leader);
-            if (act) {
-                const uint64_t pos = (uint64_t)S.off[l][k - (l ? t0[1] : t0[0])] + rb + __popc(peers & lanemask_lt());
-                if (pos < (l ? p.d.cap_b : p.d.cap_c)) {
-                    (l ? p.d.list_b : p.d.list_c)[pos] = S.w[own];
-                } else {
-                    atomicMax(l ? &p.d.ctl->need_b : &p.d.ctl->need_c, (unsigned long long)pos + 1);
-                    flag(p.d.ctl, ST_OVERFLOW);
-                }
-            }
-        }
-        __syncthreads();  // off / pre / first are rewritten by the next tile
-    }
-}
-
-__global__ void __launch_bounds__(kThreads, 6) k_prepare(P p) {
-    __shared__ union {
-        SortShared sort;
-        ScatterShared scatter;
-    } U;
+// one CTA per tile of kSortTile I keys (side stream, after k_trace)
+__global__ void __launch_bounds__(kThreads) k_isort(P p) {
+    __shared__ SortShared S;
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
-    // early trigger: k_classify's CTAs take the free slots and do their setup
-    // (inputs and k_trace's outputs only) while this grid runs; they wait for its
-    // completion before reading the registration lists
+    sort_role(p, blockIdx.x, S);
+    (void)tl0;
     pdl_trigger();
-    if (blockIdx.x < p.sort_ctas) {
-        sort_role(p, blockIdx.x, U.sort);
-    } else {
-        scatter_role(p, blockIdx.x - p.sort_ctas, U.scatter);
-        TL_REC(2, 1, tl0);
-    }
 }
 
 // ----------------------------------------------------------------------------
@@ -947,9 +584,10 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 //    mortal window (registered mortals in list order, per-node live masks);
 //    then each warp classifies its own 256 words with no further CTA barrier:
 //    word q of warp w is q = 256 w + 32 k + lane (k = 0..7).
+constexpr int kFront = 256;  // tree-query frontier nodes held per level
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
-    ulonglong2 rbe[kWinCap];             // (base, end) of one batch of registered mortals as loaded
+    ulonglong2 rbe[kWinCap];             // (base, end) of one batch of window entries
     uint32_t rta[kWinCap], rtf[kWinCap], rid[kWinCap];
     uint64_t hmin[kWinCap / 32], hmax[kWinCap / 32];  // per loading warp: least base, greatest end
     uint32_t live[kNodeGrp][kWinCap / 32];  // live[u] bit e: window entry e live at node g0 + u
@@ -963,7 +601,10 @@ struct ClsShared {
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32]; // slot bits (warp w: words 8w .. 8w+7)
     uint32_t wcnt[kWarps];                  // slots found per warp
     uint64_t hull_lo, hull_hi;              // [least base, greatest end) of the current window batch
-    uint32_t defer;                         // some candidate needs a later node group / window batch
+    uint32_t front[2][kFront];              // tree-query frontier (by level parity)
+    uint32_t fn[kMaxLevels + 1];            // frontier size per level
+    uint32_t wid[kWinCap];                  // tree-query results: the window entries' allocation ordinals
+    uint32_t nres;
     unsigned long long mbar;
 };
 
@@ -980,19 +621,21 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-// threads 0..kWinCap-1 (whole warps): one batch of <= kWinCap registered mortals
-// -> S.r*, and each loading warp's least base / greatest end (the batch's hull)
-__device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint64_t bs, uint32_t m) {
+// threads 0..kWinCap-1 (whole warps): the records of the m <= kWinCap window
+// entries the tree query found -> S.r*, and each loading warp's least base /
+// greatest end (the batch's hull)
+__device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint32_t m) {
     const uint32_t e = threadIdx.x;
     uint64_t b = ~0ull, en = 0;
     if (e < m) {
-        const WinRec x = p.d.list_c[bs + e];
-        S.rbe[e] = make_ulonglong2(x.base, x.end);
+        const uint32_t id = S.wid[e];
+        const medusa_alloc x = ld_alloc(p.a.alloc + id);
+        S.rbe[e] = make_ulonglong2(x.base, x.base + x.size);
         S.rta[e] = x.t_alloc;
         S.rtf[e] = x.t_free;
-        S.rid[e] = x.id;
+        S.rid[e] = id;
         b = x.base;
-        en = x.end;
+        en = x.base + x.size;
     }
     b = warp_min_u64(b);
     en = warp_max_u64(en);
@@ -1000,6 +643,61 @@ __device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint64_t b
         S.hmin[e >> 5] = b;
         S.hmax[e >> 5] = en;
     }
+}
+
+// CTA-wide descent of the mortal tree: the window entries of the
+// chunk = the ordinals i in [o_lo, o_hi) with v_i > T0 (a mortal freed after the
+// chunk's first launch) and t_alloc_i < T1 (allocated before its last launch)
+// and, when every segment's launch position is in nt0 (exact), live at one of
+// them: t_alloc_i < nt0[u] < t_free_i for some u.  One level per round: each warp
+// expands one kept node into its 32 children with one coalesced load.  The
+// entries go to S.wid[0 .. S.nres).  Returns false if a level keeps more than
+// kFront nodes or the entries exceed kWinCap (the caller halves the range).
+__device__ bool tree_query(const Tree& T, ClsShared& S, uint32_t T0, uint32_t T1, uint32_t o_lo, uint32_t o_hi,
+                           uint32_t ng0, bool exact) {
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid <= (uint32_t)kMaxLevels) S.fn[tid] = 0;
+    if (tid == 0) S.nres = 0;
+    __syncthreads();
+    for (int l = (int)T.top; l >= 0; --l) {
+        const bool root = l == (int)T.top;  // the virtual root: its children are the top level
+        const uint32_t np = root ? 1u : S.fn[l + 1];
+        const uint32_t* par = S.front[(l + 1) & 1];
+        uint32_t* out = l > 0 ? S.front[l & 1] : S.wid;
+        uint32_t* cnt = l > 0 ? &S.fn[l] : &S.nres;
+        const uint32_t cap = l > 0 ? (uint32_t)kFront : (uint32_t)kWinCap;
+        const uint32_t sh = 5u * (uint32_t)l;  // a node of level l covers 2^sh ordinals
+        bool ovf = false;
+        for (uint32_t f = warp; f < np; f += kWarps) {
+            const uint32_t c = (root ? 0u : par[f]) * 32 + lane;
+            bool keep = false;
+            if (c < T.cnt[l]) {
+                const uint64_t first = (uint64_t)c << sh, last = first + (1ull << sh);
+                if (first < o_hi && last > o_lo) {
+                    const uint2 nd = l > 0 ? __ldcg(T.node + T.off[l] + c) : __ldcg(T.leaf + c);
+                    keep = nd.x > T0 && nd.y < T1;
+                    if (keep && l == 0 && exact) {  // live at one of the chunk's launches
+                        uint32_t lo = 0, hi = ng0;   // the first segment launched after t_alloc
+                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt0[mid] <= nd.y) lo = mid + 1; else hi = mid; }
+                        keep = lo < ng0 && S.nt0[lo] < nd.x;
+                    }
+                }
+            }
+            const uint32_t b = __ballot_sync(0xffffffffu, keep);
+            if (b) {
+                uint32_t base = 0;
+                if (lane == 0) base = atomicAdd(cnt, (uint32_t)__popc(b));
+                base = __shfl_sync(0xffffffffu, base, 0);
+                const uint32_t pos = base + __popc(b & lanemask_lt());
+                if (keep) {
+                    if (pos < cap) out[pos] = c;
+                    else ovf = true;
+                }
+            }
+        }
+        if (__syncthreads_or(ovf)) return false;
+    }
+    return true;
 }
 
 // The live masks of nodes g0 .. g0+ng for the loaded batch of m entries (whole CTA;
@@ -1109,40 +807,43 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const uint64_t* gsrc = a.words + cs;
     const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
     const uint32_t mb = smem_u32(&S.mbar);
-    // A malformed CSR or launch order (flagged by k_trace, two launches back and
-    // therefore complete) leaves jf / jl and the node offsets meaningless: write
-    // the empty counts the later kernels read and do nothing else (the call
-    // returns INVALID_ARG; no shared-memory index is ever derived from node_off)
+    // A. the chunk's words -> shared memory with one TMA bulk copy, issued before
+    //    waiting for k_trace (the words are an input)
+    if (tid == 0 && tma) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                     ::"r"(smem_u32(S.words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
+    }
+    if (tid < MEDUSA_CHUNK_WORDS / 32) S.nsm[tid] = 0;
+    if (tid < kNodeGrp) S.nt0[tid] = 0;
+    pdl_wait();  // k_trace: node ranges, status, prefilter bounds, the mortal tree
+    // A malformed CSR or launch order (flagged by k_trace) leaves jf / jl and the
+    // node offsets meaningless: write the empty counts the later kernels read and
+    // do nothing else (the call returns INVALID_ARG; no shared-memory index is
+    // ever derived from node_off); the bulk copy is waited for before leaving
     if (__ldcg(&ctl->status) & ST_INVALID) {
         if (tid < kWarps) p.d.qcnt[c * kWarps + tid] = 0;
         if (tid == 0) p.d.chunk_cnt[c] = 0;
-        pdl_wait();
+        if (tid == 0 && tma) {
+            uint32_t done = 0;
+            while (!done) {
+                asm volatile("{ .reg .pred P; mbarrier.try_wait.parity.shared::cta.b64 P, [%1], 0; selp.u32 %0, 1, 0, P; }"
+                             : "=r"(done) : "r"(mb) : "memory");
+            }
+        }
         pdl_trigger();
         return;
-    }
-    // A. the chunk's words -> shared memory with one TMA bulk copy; meanwhile the
-    //    list offsets (block_prefix) and the chunk's node range load
-    if (tid == 0) {
-        S.defer = 0;
-        if (tma) {
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
-            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(n * 8) : "memory");
-            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                         ::"r"(smem_u32(S.words)), "l"(gsrc), "r"(n * 8), "r"(mb) : "memory");
-        }
     }
     const uint32_t N = a.n_nodes;
     const uint32_t jf = N ? min(__ldcg(p.d.jf + c), N - 1) : 0, jl = N ? min(__ldcg(p.d.jl + c), N - 1) : 0;
     const uint32_t nn = N ? jl - jf + 1 : 0;
-    const uint64_t gmin = ~ctl->gmin_c, gmax = ctl->gmax;
+    const uint64_t gmin = ~__ldcg(&ctl->gmin_c), gmax = __ldcg(&ctl->gmax);
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
-    if (tid < MEDUSA_CHUNK_WORDS / 32) S.nsm[tid] = 0;
-    if (tid < kNodeGrp) S.nt0[tid] = 0;
-    const uint32_t t_jf = N ? __ldg(a.node_t + jf) : 0;
-    const uint64_t r0 = block_prefix(p.d.cnt_c, p.d.sup_c, c);  // (synchronizes the CTA)
-    const uint64_t r1 = min(r0 + __ldcg(p.d.cnt_c + c), p.d.cap_c);
+    const uint32_t t_jf = N ? __ldg(a.node_t + jf) : 0, t_jl = N ? __ldg(a.node_t + jl) : 0;
+    __syncthreads();  // nsm / nt0 zeroed before any thread sets a bit
     TL_PHASE(4, 10, tl_p);  // A: setup
     // B. the starts of the chunk's nodes (-> start bitmask, its popcount prefix,
     //    the launch positions of the first kNodeGrp segments)
@@ -1209,68 +910,53 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     }
     if (lane < 8) wh[lane] = 0;
     TL_PHASE(4, 11, tl_p);  // B/C: node starts, TMA wait, candidates
-    // Everything above reads only the inputs and k_trace's outputs (two launches
-    // back): it overlaps k_prepare's tail.  The registration lists are k_prepare's.
-    pdl_wait();
-    // D. the first window batch (in list order: no sort) and the live masks of
-    //    the first node group
-    const uint32_t m0 = (uint32_t)min((uint64_t)kWinCap, r1 - r0);
-    if (tid < kWinCap) window_load(p, S, r0, m0);
-    __syncthreads();
-    if (m0) build_live(S, S.nt0, ng0, m0);
-    TL_PHASE(4, 12, tl_p);  // D: window, live masks
-    // E. per candidate its segment (O(1) from the start bitmask) and the window
-    //    lookup at node group 0 / batch 0
-    const bool more_batches = r1 - r0 > (uint64_t)kWinCap;
-    bool deferred = false;
-    for (uint32_t i = lane; i < nc; i += 32) {
-        const uint32_t q = wl[i];
-        const uint64_t x = S.words[q];
-        const uint32_t u = seg_of(S, q);
-        bool hit = false;
-        if (m0 && u < ng0) {
-            const int e = window_find(S, m0, u, x);
-            if (e >= 0) {
-                hit = true;
-                S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rbe[e].x);
-                atomicOr(&S.hits[q >> 5], 1u << (q & 31));
-            }
+    // D. the window: the mortals live at one of the chunk's launches, found by a
+    //    descent of the mortal tree (normally one batch of <= kWinCap entries; a
+    //    query that overflows is retried on half the ordinal range, and the
+    //    ranges are then processed one batch after another).  Per batch and node
+    //    group (normally one: <= kNodeGrp segments): the live masks, then each
+    //    warp looks its own candidates up among the entries live at their node.
+    const bool exact = n_seg <= (uint32_t)kNodeGrp;
+    const uint32_t n_alloc = a.n_alloc;
+    uint32_t o_lo = 0, wlen = n_alloc;
+    while (N && o_lo < n_alloc) {
+        const uint32_t o_hi = (uint32_t)min((uint64_t)o_lo + wlen, (uint64_t)n_alloc);
+        if (!tree_query(p.d.tree, S, t_jf, t_jl, o_lo, o_hi, ng0, exact)) {
+            wlen = (wlen + 1) / 2;
+            continue;
         }
-        if (!hit && m0 && (u >= ng0 || more_batches)) deferred = true;
-    }
-    if (__any_sync(0xffffffffu, deferred) && lane == 0) S.defer = 1;
-    __syncthreads();
-    TL_PHASE(4, 13, tl_p);  // D: window search
-    if (S.defer) {
-        // rare: chunks with more than kNodeGrp segments or windows of more than
-        // kWinCap entries -- every batch against every segment group, CTA-synchronous
-        for (uint64_t bs = r0; bs < r1; bs += kWinCap) {
-            const uint32_t m = (uint32_t)min((uint64_t)kWinCap, r1 - bs);
-            if (bs != r0) {
-                __syncthreads();
-                window_load(p, S, bs, m);
-                __syncthreads();
-            }
-            for (uint32_t g0 = (bs == r0 ? kNodeGrp : 0); g0 < n_seg; g0 += kNodeGrp) {
+        const uint32_t m = S.nres;
+        __syncthreads();  // every thread has read nres before a later query resets it
+        TL_PHASE(4, 12, tl_p);  // D: tree query
+        if (m) {
+            if (tid < kWinCap) window_load(p, S, m);
+            __syncthreads();
+            for (uint32_t g0 = 0; g0 < n_seg; g0 += kNodeGrp) {
                 const uint32_t ng = min((uint32_t)kNodeGrp, n_seg - g0);
-                __syncthreads();
-                seg_times(p, S, S.nt, g0, ng, cs, jf, jl);
-                build_live(S, S.nt, ng, m);
+                const uint32_t* nt = S.nt0;
+                if (g0) {
+                    seg_times(p, S, S.nt, g0, ng, cs, jf, jl);
+                    nt = S.nt;
+                }
+                build_live(S, nt, ng, m);
                 for (uint32_t i = lane; i < nc; i += 32) {
                     const uint32_t q = wl[i];
-                    if ((S.hits[q >> 5] >> (q & 31)) & 1u) continue;
+                    if ((wh[(q & 255) >> 5] >> (q & 31)) & 1u) continue;  // found in an earlier batch
                     const uint32_t u = seg_of(S, q);
                     if (u < g0 || u >= g0 + ng) continue;
                     const uint64_t x = S.words[q];
                     const int e = window_find(S, m, u - g0, x);
                     if (e >= 0) {
                         S.words[q] = ((uint64_t)S.rid[e] << MEDUSA_OFF_BITS) | (x - S.rbe[e].x);
-                        atomicOr(&S.hits[q >> 5], 1u << (q & 31));
+                        atomicOr(&wh[(q & 255) >> 5], 1u << (q & 31));
                     }
                 }
+                __syncthreads();  // the live masks / window are rewritten by the next group / batch
             }
         }
-        __syncthreads();
+        TL_PHASE(4, 13, tl_p);  // D: live masks, window search
+        o_lo = o_hi;
+        wlen = (uint32_t)min((uint64_t)wlen * 2, (uint64_t)n_alloc);
     }
     // E. the candidates no mortal holds go to this warp's queue region (k_iresolve)
     IQ* wq = p.d.queue + cs + warp * 256;
@@ -1325,22 +1011,27 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 }
 
 // ----------------------------------------------------------------------------
-// 2c. k_check (after k_rank and k_classify, default priority): the R-Q7 checks.
+// 2c. k_check (after k_rank, default priority): the R-Q7 checks.
 //     I-I: adjacent sorted I entries (the CTA checks 256 pairs).  Per warp, a
 //     block of 32 allocation ordinals: M-M -- each mortal j against the mortals
-//     registered as live at some allocation of the block (hull-filtered,
-//     branch-free scan); M-I -- each mortal against the run of I entries its
-//     range meets (one fence search; the common "no I entry in range" case costs
-//     two more loads).
+//     i < j still live when j is allocated (t_free_i > t_alloc_j), found by a
+//     depth-first descent of the mortal tree (nodes with max t_free > the block's
+//     least t_alloc and first ordinal < its greatest ordinal), then
+//     hull-filtered and tested pairwise; M-I -- each mortal against the run of
+//     I entries its range meets (one fence search; the common "no I entry in
+//     range" case costs two more loads).
+constexpr int kStk = 32 * kMaxLevels + 32;  // DFS stack per warp: < 32 entries per level on the path
 __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
     __shared__ ulonglong2 s_be[kWarps][32];  // (base, end): one 16-byte broadcast load
     __shared__ uint2 s_ti[kWarps][32];       // (t_free, id): one 8-byte broadcast load
+    __shared__ uint32_t s_stk[kWarps][kStk];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     pdl_trigger();
     const uint32_t cta = blockIdx.x;
     const MaterializeArgs& a = p.a;
+    const Tree& T = p.d.tree;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t nI = p.d.ctl->nI;
     {  // I-I: sorted neighbours must not overlap (all of I is live at the last launch)
@@ -1350,11 +1041,10 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
     for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = __ldcg(p.d.fence + f);
-    const uint32_t b0 = cta * kWarps;
-    const unsigned long long lbase = block_prefix(p.d.cnt_b, p.d.sup_b, min(b0, p.nb));  // (synchronizes)
-    const uint32_t b = b0 + warp;
+    __syncthreads();
+    const uint32_t b = cta * kWarps + warp;
     if (b >= p.nb) return;  // whole warp
-    const uint32_t j = b * kAblk + lane;
+    const uint32_t j = b * 32 + lane;
     bool mine = false;
     medusa_alloc x{};
     const uint32_t N = a.n_nodes;
@@ -1366,38 +1056,59 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
     const uint64_t xe = x.base + x.size;
     bool bad = false;
     // M-M
-    {
-        const uint32_t cb = (lane <= warp && b0 + lane < p.nb) ? __ldcg(p.d.cnt_b + b0 + lane) : 0u;
-        const uint32_t before = __reduce_add_sync(0xffffffffu, lane < warp ? cb : 0u);
-        const uint64_t hb = warp_min_u64(mine ? x.base : ~0ull), he = warp_max_u64(mine ? xe : 0ull);
-        const uint32_t hta = __reduce_min_sync(0xffffffffu, mine ? x.t_alloc : 0xFFFFFFFFu);
-        const uint32_t hj = __reduce_max_sync(0xffffffffu, mine ? j : 0u);
-        const uint64_t r0 = lbase + before;
-        const uint64_t r1 = min(r0 + __shfl_sync(0xffffffffu, cb, warp), p.d.cap_b);
-        for (uint64_t bs = r0; bs < r1 && he; bs += 32) {
-            const uint32_t m = (uint32_t)min((uint64_t)32, r1 - bs);
-            WinRec y{};
+    const uint64_t hb = warp_min_u64(mine ? x.base : ~0ull), he = warp_max_u64(mine ? xe : 0ull);
+    const uint32_t hta = __reduce_min_sync(0xffffffffu, mine ? x.t_alloc : 0xFFFFFFFFu);
+    const uint32_t hj = __reduce_max_sync(0xffffffffu, mine ? j : 0u);
+    if (he) {
+        uint32_t* stk = s_stk[warp];
+        uint32_t sp = 0;
+        int lvl = (int)T.top + 1;  // the virtual root: its children are the top level
+        uint32_t node = 0;
+        while (true) {
+            const int cl = lvl - 1;  // level of the children
+            const uint32_t c = node * 32 + lane;
+            const uint32_t sh = 5u * (uint32_t)cl;
             bool keep = false;
-            if (lane < m) {
-                y = p.d.list_b[bs + lane];
-                keep = y.base < he && hb < y.end && y.t_free > hta && y.id < hj;
+            uint2 nd = make_uint2(0, 0);
+            if (c < T.cnt[cl] && ((uint64_t)c << sh) < hj) {
+                nd = cl > 0 ? __ldcg(T.node + T.off[cl] + c) : __ldcg(T.leaf + c);
+                keep = nd.x > hta;
             }
             const uint32_t kb = __ballot_sync(0xffffffffu, keep);
-            __syncwarp();
-            if (keep) {
-                const uint32_t o = __popc(kb & lanemask_lt());
-                s_be[warp][o] = make_ulonglong2(y.base, y.end);
-                s_ti[warp][o] = make_uint2(y.t_free, y.id);
-            }
-            __syncwarp();
-            if (mine) {
-                const uint32_t nk = __popc(kb);
-                for (uint32_t q = 0; q < nk; ++q) {
-                    const ulonglong2 be = s_be[warp][q];
-                    const uint2 ti = s_ti[warp][q];
-                    bad |= (ti.y < j) & (ti.x > x.t_alloc) & (be.x < xe) & (x.base < be.y);
+            if (cl > 0) {  // push the kept children (the stack holds (level << 24) | node)
+                if (keep) stk[sp + __popc(kb & lanemask_lt())] = ((uint32_t)cl << 24) | c;
+                sp += __popc(kb);
+            } else if (kb) {  // leaves: mortals i < hj with t_free_i > hta
+                uint64_t yb = 0, ye = 0;
+                bool k2 = false;
+                if (keep) {
+                    const medusa_alloc r = ld_alloc(a.alloc + c);
+                    yb = r.base;
+                    ye = r.base + r.size;
+                    k2 = yb < he && hb < ye;
+                }
+                const uint32_t k2b = __ballot_sync(0xffffffffu, k2);
+                __syncwarp();
+                if (k2) {
+                    const uint32_t o = __popc(k2b & lanemask_lt());
+                    s_be[warp][o] = make_ulonglong2(yb, ye);
+                    s_ti[warp][o] = make_uint2(nd.x, c);  // (t_free, id)
+                }
+                __syncwarp();
+                if (mine) {
+                    const uint32_t nk = __popc(k2b);
+                    for (uint32_t q = 0; q < nk; ++q) {
+                        const ulonglong2 be = s_be[warp][q];
+                        const uint2 ti = s_ti[warp][q];
+                        bad |= (ti.y < j) & (ti.x > x.t_alloc) & (be.x < xe) & (x.base < be.y);
+                    }
                 }
             }
+            __syncwarp();
+            if (sp == 0) break;
+            const uint32_t e = stk[--sp];
+            lvl = (int)(e >> 24);
+            node = e & 0xFFFFFFu;
         }
     }
     // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
@@ -1586,7 +1297,6 @@ __global__ void k_result(P p, medusa_mat_result* r) {
     int32_t st = MEDUSA_OK;
     if (c.status & ST_INVALID) st = MEDUSA_ERR_INVALID_ARG;
     else if (c.status & ST_TRACE) st = MEDUSA_ERR_TRACE;
-    else if (c.status & ST_OVERFLOW) st = MEDUSA_ERR_RETRY;
     else if (c.n_slots > p.a.capacity) st = MEDUSA_ERR_CAPACITY;
     r->status = st;
     r->reserved = 0;
@@ -1595,15 +1305,33 @@ __global__ void k_result(P p, medusa_mat_result* r) {
 
 // ----------------------------------------------------------------------------
 // host side: per-device scratch, launches
+
+// level sizes of the mortal tree over n ordinals (cnt[0] = n; the top level has
+// <= 32 nodes); node levels 1..top stored back to back
+Tree tree_shape(uint64_t n) {
+    Tree t{};
+    t.cnt[0] = (uint32_t)n;
+    uint32_t l = 0, o = 0;
+    while (t.cnt[l] > 32 && l < (uint32_t)kMaxLevels) {
+        t.cnt[l + 1] = (t.cnt[l] + 31) / 32;
+        ++l;
+        t.off[l] = o;
+        o += t.cnt[l];
+    }
+    t.top = l;
+    t.off[kMaxLevels] = o;  // (scratch sizing: total node count)
+    return t;
+}
+
 struct Scratch {
-    size_t cap_n = 0, cap_C = 0, cap_nb = 0, cap_c = 0, cap_b = 0, cap_w = 0;
+    size_t cap_n = 0, cap_C = 0, cap_w = 0;
     void* zero_region = nullptr;
     size_t zero_bytes = 0;
     Dev d{};
     std::vector<void*> bufs;
     Ctl* h_ctl = nullptr;
     int sm_count = 0;
-    cudaStream_t side = nullptr;  // the I-list rank branch (highest priority; forked from the caller's stream)
+    cudaStream_t side = nullptr;  // the I-list sort + rank branch (highest priority; forked from the caller's stream)
     cudaStream_t low = nullptr;   // the trace-check branch (default priority; joined before the call ends)
     cudaEvent_t fork = nullptr, join = nullptr, ranked = nullptr, classified = nullptr, emitted = nullptr;
     // Buffers retired by a growth.  A CUDA graph that captured an earlier
@@ -1635,53 +1363,43 @@ void retire(Scratch& s) {
     if (s.zero_region) s.graveyard.push_back(s.zero_region);
     s.zero_region = nullptr;
     s.bytes = 0;
-    s.cap_n = s.cap_C = s.cap_nb = s.cap_c = s.cap_b = s.cap_w = 0;
+    s.cap_n = s.cap_C = s.cap_w = 0;
 }
 
 // grow geometrically (x1.5) past the previous capacity, so a sequence of growing
 // calls retires a bounded amount of memory
 size_t grown(size_t need, size_t old) { return need <= old ? old : std::max(need, old + old / 2); }
 
-cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t nb, size_t W, size_t need_c, size_t need_b) {
-    if (n <= s.cap_n && C <= s.cap_C && nb <= s.cap_nb && W <= s.cap_w && need_c <= s.cap_c && need_b <= s.cap_b)
-        return cudaSuccess;
+cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W) {
+    if (n <= s.cap_n && C <= s.cap_C && W <= s.cap_w) return cudaSuccess;
     const size_t N = grown(std::max<size_t>(n, 1024), s.cap_n), CC = grown(std::max<size_t>(C, 64), s.cap_C);
-    const size_t NB = grown(std::max<size_t>(nb, 64), s.cap_nb);
     const size_t WW = grown(std::max<size_t>(W, 2048), s.cap_w);
-    const size_t RC = grown(std::max<size_t>(need_c, N + 4 * CC), s.cap_c);
-    const size_t RB = grown(std::max<size_t>(need_b, 3 * N), s.cap_b);
     retire(s);
     const size_t NS = N / kIBlk + 1;
+    const size_t NT = tree_shape(N).off[kMaxLevels] + 64;  // tree nodes (levels >= 1) for up to N ordinals
     cudaError_t e;
-    // zero region: Ctl | sup_c chunk_sup [CC/256+1] sup_b [NB/256+1] (u64) | cnt_c fill_c [CC+1] |
-    //              cnt_b fill_b [NB+1] | blk_min_ta_c blk_max_tf [NS]
-    const size_t GC = CC / 256 + 1, GB = NB / 256 + 1;
-    s.zero_bytes = 256 + (2 * GC + GB) * 8 + 2 * (CC + 1) * 4 + 2 * (NB + 1) * 4 + 2 * NS * 4 + 64;
+    // zero region: Ctl | chunk_sup [CC/256+1] (u64) | blk_min_ta_c blk_max_tf [NS] | tree nodes [NT] (uint2)
+    const size_t GC = CC / 256 + 1;
+    s.zero_bytes = 256 + GC * 8 + 2 * NS * 4 + 64 + NT * 8;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
     s.bytes += s.zero_bytes;
     char* z = (char*)s.zero_region;
     s.d.ctl = (Ctl*)z;
     size_t o = 256;
-    s.d.sup_c = (unsigned long long*)(z + o); o += GC * 8;
     s.d.chunk_sup = (unsigned long long*)(z + o); o += GC * 8;
-    s.d.sup_b = (unsigned long long*)(z + o); o += GB * 8;
-    s.d.cnt_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
-    s.d.fill_c = (uint32_t*)(z + o); o += (CC + 1) * 4;
-    s.d.cnt_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
-    s.d.fill_b = (uint32_t*)(z + o); o += (NB + 1) * 4;
     s.d.blk_min_ta_c = (uint32_t*)(z + o); o += NS * 4;
     s.d.blk_max_tf = (uint32_t*)(z + o); o += NS * 4;
-    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.rng, N)) ||
-        (e = grow(s, s.d.list_c, RC)) || (e = grow(s, s.d.list_b, RB)) || (e = grow(s, s.d.sk[0], N)) ||
-        (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) || (e = grow(s, s.d.sv[1], N)) ||
-        (e = grow(s, s.d.samp_k, N / 32 + 64)) || (e = grow(s, s.d.samp_v, N / 32 + 64)) || (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) ||
-        (e = grow(s, s.d.i_tf, N)) || (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
-        (e = grow(s, s.d.chunk_cnt, CC)) || (e = grow(s, s.d.staging, WW)) ||
-        (e = grow(s, s.d.queue, CC * kChunkWords)) || (e = grow(s, s.d.qcnt, CC * kWarps)))
+    o = (o + 63) & ~(size_t)63;
+    s.d.tree.node = (uint2*)(z + o);
+    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) ||
+        (e = grow(s, s.d.sk[0], N)) || (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) ||
+        (e = grow(s, s.d.sv[1], N)) || (e = grow(s, s.d.samp_k, N / 32 + 64)) || (e = grow(s, s.d.samp_v, N / 32 + 64)) ||
+        (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
+        (e = grow(s, s.d.fence, (size_t)kFenceCap)) || (e = grow(s, s.d.chunk_cnt, CC)) ||
+        (e = grow(s, s.d.staging, WW)) || (e = grow(s, s.d.queue, CC * kChunkWords)) ||
+        (e = grow(s, s.d.qcnt, CC * kWarps)))
         return e;
-    s.d.cap_c = RC;
-    s.d.cap_b = RB;
-    s.cap_n = N; s.cap_C = CC; s.cap_nb = NB; s.cap_c = RC; s.cap_b = RB; s.cap_w = WW;
+    s.cap_n = N; s.cap_C = CC; s.cap_w = WW;
     return cudaSuccess;
 }
 
@@ -1721,23 +1439,26 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
     return &s;
 }
 
-// the whole analysis on `stream` (no synchronization).  After k_prepare (I-list
-// tile sort + registration lists):
-//   stream:            k_classify [classified] ............................ [emitted][join]
-//   side (high prio):  k_rank [ranked] ... [classified] k_iresolve -> k_emit [emitted]
-//   low (default):     [classified][ranked] k_check [join]
-// The high-priority stream gets the rank CTAs dispatched ahead of the classify
-// CTAs and the queue resolution / emission ahead of the trace checks, which
-// fill in around them and complete the call.
+// the whole analysis on `stream` (no synchronization):
+//   stream:            memset -> k_trace [fork] -> k_classify [classified] ......... [emitted][join]
+//   side (high prio):                 [fork] k_isort -> k_rank [ranked] [classified] k_iresolve -> k_emit [emitted]
+//   low (default):                                       [ranked] k_check [join]
+// The high-priority stream gets the sort / rank CTAs dispatched ahead of the
+// classify CTAs and the queue resolution / emission ahead of the trace checks,
+// which fill in around them and complete the call.
 cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P* out) {
     const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
-    const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
+    const uint32_t nb = (uint32_t)((n + 31) / 32);
     const uint32_t node_ctas = (a.n_nodes + 1 + kThreads * kNodesPerThread - 1) / (kThreads * kNodesPerThread);
     const uint32_t alloc_ctas = (uint32_t)((n + kThreads - 1) / kThreads);
     const uint32_t sort_ctas = (uint32_t)((n + kSortTile - 1) / kSortTile);
-    const uint32_t check_ctas = n ? std::max<uint32_t>((nb + kWarps - 1) / kWarps, alloc_ctas) : 0;
-    P p{a, s.d, C, nb, node_ctas, sort_ctas, check_ctas};
+    const uint32_t check_ctas = (nb + kWarps - 1) / kWarps;
+    Dev d = s.d;
+    const Tree shape = tree_shape(n);
+    d.tree.top = shape.top;
+    for (int l = 0; l <= kMaxLevels; ++l) { d.tree.cnt[l] = shape.cnt[l]; d.tree.off[l] = shape.off[l]; }
+    P p{a, d, C, nb, node_ctas};
     *out = p;
     cudaError_t e;
     // branches (serialized on the caller's stream while per-launch timing is on)
@@ -1750,22 +1471,26 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
     }
     if (n) {
-        {
-            TimedLaunch tl("mat_prepare", stream);
-            if ((e = launch_pdl(k_prepare, sort_ctas + alloc_ctas, kThreads, 0, stream, p))) return e;
-        }
         if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(side, s.fork, 0))) return e;
+        {
+            TimedLaunch tl("mat_isort", side);
+            k_isort<<<sort_ctas, kThreads, 0, side>>>(p);
+        }
         {
             TimedLaunch tl("mat_rank", side);
             // one CTA per 32 I keys (the list's size is known on the device only: bound
             // by the allocation count; surplus CTAs exit at once)
-            k_rank<<<(unsigned)std::min<uint64_t>((n + 31) / 32, (uint64_t)s.sm_count * 8), kThreads, 0, side>>>(p);
+            if ((e = launch_pdl(k_rank, (unsigned)std::min<uint64_t>((n + 31) / 32, (uint64_t)s.sm_count * 8), kThreads,
+                                0, side, p)))
+                return e;
         }
         if ((e = cudaEventRecord(s.ranked, side))) return e;
-        if (C) {
-            TimedLaunch tl("mat_classify", stream);
-            if ((e = launch_pdl(k_classify, C, kThreads, kClsSmem, stream, p))) return e;
-        }
+    }
+    if (C) {
+        TimedLaunch tl("mat_classify", stream);
+        if ((e = launch_pdl(k_classify, C, kThreads, kClsSmem, stream, p))) return e;
+    }
+    if (n) {
         if ((e = cudaEventRecord(s.classified, stream))) return e;
         // high priority after the classify: queue resolution and emission (the
         // rank is already on this stream)
@@ -1788,12 +1513,6 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaEventRecord(s.join, low))) return e;
         if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
-        {
-            // no k_prepare in between: a plain launch (k_classify reads k_trace's
-            // outputs before its griddepcontrol.wait, which is only safe two launches back)
-            TimedLaunch tl("mat_classify", stream);
-            k_classify<<<C, kThreads, kClsSmem, stream>>>(p);
-        }
         TimedLaunch tl("mat_emit", stream);
         if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
     }
@@ -1810,30 +1529,20 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     Scratch* sp = device_scratch(&e, &lk);
     if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     Scratch& s = *sp;
-    const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
-    const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
-    size_t need_c = 0, need_b = 0;
-    for (int attempt = 0; attempt < 3; ++attempt) {
-        if ((e = ensure(s, n, C, nb, a.n_words, need_c, need_b)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-        P p;
-        if ((e = enqueue(s, a, stream, &p)) != cudaSuccess) break;
-        if ((e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess) break;
-        if ((e = cudaStreamSynchronize(stream)) != cudaSuccess) break;
-        const Ctl h = *s.h_ctl;
-        if (h.status & ST_INVALID) return MEDUSA_ERR_INVALID_ARG;
-        if (h.status & ST_TRACE) return MEDUSA_ERR_TRACE;
-        if (h.status & ST_OVERFLOW) {  // registration lists larger than guessed: size exactly, rerun
-            need_c = std::max<size_t>(need_c, h.need_c);
-            need_b = std::max<size_t>(need_b, h.need_b);
-            continue;
-        }
-        *n_slots = h.n_slots;
-        return h.n_slots > a.capacity ? MEDUSA_ERR_CAPACITY : MEDUSA_OK;
+    P p;
+    if ((e = ensure(s, a.n_alloc, C, a.n_words)) != cudaSuccess ||
+        (e = enqueue(s, a, stream, &p)) != cudaSuccess ||
+        (e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(stream)) != cudaSuccess) {
+        *cuda_err = e;
+        return MEDUSA_ERR_CUDA;
     }
-    if (e != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
-    *cuda_err = cudaErrorUnknown;
-    return MEDUSA_ERR_CUDA;
+    const Ctl h = *s.h_ctl;
+    if (h.status & ST_INVALID) return MEDUSA_ERR_INVALID_ARG;
+    if (h.status & ST_TRACE) return MEDUSA_ERR_TRACE;
+    *n_slots = h.n_slots;
+    return h.n_slots > a.capacity ? MEDUSA_ERR_CAPACITY : MEDUSA_OK;
 }
 
 medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
@@ -1843,11 +1552,9 @@ medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result*
     Scratch* sp = device_scratch(&e, &lk);
     if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     Scratch& s = *sp;
-    const uint64_t n = a.n_alloc;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
-    const uint32_t nb = (uint32_t)((n + kAblk - 1) / kAblk);
     // never (re)allocates while the caller may be capturing a graph, unless it must grow
-    if ((e = ensure(s, n, C, nb, a.n_words, 0, 0)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    if ((e = ensure(s, a.n_alloc, C, a.n_words)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     P p;
     if ((e = enqueue(s, a, stream, &p)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     if ((e = launch_pdl(k_result, 1, 1, 0, stream, p, d_result))) { *cuda_err = e; return MEDUSA_ERR_CUDA; }

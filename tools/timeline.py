@@ -21,14 +21,14 @@ sys.path.insert(0, ROOT)
 import __graft_entry__ as g  # noqa: E402
 
 NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan",
-         (2, 0): "prepare/sort", (2, 1): "prepare/scatter", (3, 0): "rank",
+         (2, 0): "isort", (2, 1): "prepare/scatter", (3, 0): "rank",
          (4, 0): "classify",
          (5, 0): "emit", (8, 0): "check_mm", (9, 0): "check", (10, 0): "iresolve", (6, 0): "report_init", (7, 0): "restore/words", (7, 1): "restore/gather",
-         (1, 20): " allocs:load+nj0", (1, 21): " allocs:stage", (1, 22): " allocs:search+reg",
+         (1, 20): " allocs:load+checks", (1, 21): " allocs:stage", (1, 22): " allocs:tree+I",
          (1, 23): " last:fence", (1, 24): " last:scan-c", (1, 25): " last:scan-b",
          (3, 40): " rank:pdl-wait", (3, 41): " rank:staging", (3, 42): " rank:search+red", (3, 43): " rank:ticket",
          (3, 44): " rank:i-entries", (2, 30): " isort:bitonic", (2, 31): " isort:merges",
-         (4, 10): " cls:A setup", (4, 11): " cls:B starts+cand", (4, 12): " cls:C live", (4, 13): " cls:D winsearch",
+         (4, 10): " cls:A setup", (4, 11): " cls:B starts+cand", (4, 12): " cls:D query", (4, 13): " cls:D live+search",
          (4, 14): " cls:E queue", (4, 15): " cls:pdl-wait", (4, 16): " cls:win-load", (4, 17): " cls:sort",
          (7, 2): "restore/in-place", (7, 10): " res:mask+range", (7, 11): " res:records+gathers",
          (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store"}
