@@ -57,7 +57,6 @@ constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
-constexpr int kSortTile = 1024;    // I keys sorted per CTA before ranking
 constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
 constexpr int kWinCap = 96;        // mortal-window entries per batch (<= 4 per lane of one warp; 96 keeps 7 classify CTAs per SM)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
@@ -104,13 +103,13 @@ struct Tree {
 
 struct Dev {  // scratch of one call (device pointers)
     Ctl* ctl;
-    uint32_t *jf, *jl;                           // [C] first / last node of each chunk
+    uint2 *jf, *jl;                              // [C] first / last node of each chunk and its launch position
     Tree tree;
     unsigned long long* chunk_sup;               // [C/256+1] slots per 256 chunks
     uint32_t *blk_min_ta_c, *blk_max_tf;         // [n/32+1] (zeroed; min kept as ~max(~t))
-    uint64_t* sk[2];                             // [n] sort keys: 0 unsorted, 1 sorted tiles
-    uint32_t* sv[2];                             // [n] sort values (allocation index)
-    uint64_t* samp_k;                            // [n/32+1] every 32nd key of each sorted tile
+    uint64_t *sk0, *sk;                          // [n] I keys (base): compacted by k_trace / sorted tiles
+    uint32_t *sv0, *sv;                          // [n] their allocation ordinals
+    uint64_t* samp_k;                            // [n/64+1] every 64th key of each sorted tile
     uint32_t* samp_v;
     uint64_t* i_base;                            // [n]
     IRest* i_rest;                               // [n]
@@ -147,7 +146,6 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
     return v;
 }
 
-__device__ __forceinline__ uint32_t n_tiles(uint32_t nI) { return (nI + kSortTile - 1) / kSortTile; }
 __device__ __forceinline__ uint32_t fence_stride(uint32_t nI) { return nI ? (nI + kFenceCap - 1) / kFenceCap : 1; }
 
 // Sum of cnt[0, k) of a two-level counter (sup[g] = sum of cnt[256g, 256g + 256)):
@@ -207,8 +205,8 @@ __device__ void nodes_role(const P& p, uint64_t i) {
     for (uint64_t c = o0 / kChunkWords; c <= (o1 - 1) / kChunkWords; ++c) {
         const uint64_t cs = c * kChunkWords;
         const uint64_t ce = min(cs + kChunkWords, a.n_words) - 1;
-        if (o0 <= cs) p.d.jf[c] = (uint32_t)i;
-        if (ce < o1) p.d.jl[c] = (uint32_t)i;
+        if (o0 <= cs) p.d.jf[c] = make_uint2((uint32_t)i, a.node_t[i]);
+        if (ce < o1) p.d.jl[c] = make_uint2((uint32_t)i, a.node_t[i]);
     }
 }
 
@@ -216,7 +214,7 @@ constexpr int kNodesPerThread = 4;  // node role of k_trace (keeps its grid insi
 
 // One allocation per thread: the trace checks (R-Q7, R-Q9), the I / M split, the
 // mortal tree (leaf, level 1 by the warp, higher levels by one atomic per CTA),
-// the I compaction and the prefilter bounds.  One coalesced record load, no search.
+// the prefilter bounds and the I compaction.  One coalesced record load, no search.
 __device__ void allocs_role(const P& p, uint32_t cta) {
     const MaterializeArgs& a = p.a;
     const Tree& T = p.d.tree;
@@ -252,7 +250,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     for (uint32_t l = 2; l <= T.top; ++l)
         if (valid && (i & ((1u << (5 * l)) - 1)) == 0) T.node[T.off[l] + (i >> (5 * l))].y = x.t_alloc;
     // CTA-aggregated (one global atomic per CTA, not per warp: these are the same
-    // three addresses for every CTA): I positions, global prefilter bounds
+    // addresses for every CTA): I positions, global prefilter bounds, upper tree levels
     __shared__ uint32_t s_ni, s_base, s_wmax[kWarps];
     __shared__ unsigned long long s_mn, s_mx;
     if (threadIdx.x == 0) { s_ni = 0; s_mn = ~0ull; s_mx = 0; }
@@ -285,15 +283,18 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     wpos = __shfl_sync(0xffffffffu, wpos, 0);
     if (isI) {
         const uint32_t pos = s_base + wpos + __popc(bal & lanemask_lt());
-        p.d.sk[0][pos] = x.base;
-        p.d.sv[0][pos] = i;
+        p.d.sk0[pos] = x.base;
+        p.d.sv0[pos] = i;
     }
-    TL_PHASE(1, 22, tl_p);  // tree, I compaction
+    TL_PHASE(1, 22, tl_p);  // tree, prefilter bounds, I compaction
 }
 
 __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
+    // k_classify's CTAs may start in the slots this grid leaves free and issue
+    // their word copies; they read nothing of this grid before griddepcontrol.wait
+    pdl_trigger();
     if (blockIdx.x < p.node_ctas) {  // kNodesPerThread nodes per thread, CTA-strided
 #pragma unroll
         for (int k = 0; k < kNodesPerThread; ++k)
@@ -303,7 +304,6 @@ __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
         allocs_role(p, blockIdx.x - p.node_ctas);
         TL_REC(1, 1, tl0);
     }
-    pdl_trigger();
 }
 
 // ----------------------------------------------------------------------------
@@ -356,112 +356,132 @@ __device__ __forceinline__ void warp_bitonic_kv(uint64_t (&k)[E], uint32_t (&v)[
 }
 
 // ----------------------------------------------------------------------------
-// 2a. sort role: one tile of kSortTile I keys (base, allocation index) per CTA.  A
-//     register bitonic sort of 128 keys per warp, then three merge-path rounds
-//     through shared memory (128 -> 256 -> 512 -> 1024), four keys per thread held
-//     in registers between rounds.  A single tile is the whole list: its I entries
-//     are written here; otherwise every 32nd key is the tile's sample for k_rank.
-constexpr int kSortThreads = kThreads;
-constexpr int kSortPer = kSortTile / kSortThreads;  // 2
-struct SortShared {
-    uint64_t k[kSortTile];
-    uint32_t v[kSortTile];
+// 2a. k_isort (side stream, after k_trace): tile t = the I keys at compacted
+//     positions [t S, t S + S), S = kIsortTile = 1024 (k_trace compacts the I
+//     allocations: non-empty, t_alloc < T_last < t_free).  Sorted by (base,
+//     ordinal): a register bitonic sort of 128 keys per warp, then three
+//     merge-path rounds through shared memory (128 -> 256 -> 512 -> 1024), four
+//     keys per thread held in registers between rounds.  A single tile is the
+//     whole list: its I entries are written here and k_rank has nothing to do.  Otherwise the sorted tile goes
+//     to sk / sv and every kSampleStride-th key is its sample for k_rank.
+constexpr int kIsortThreads = 256;  // (1024-thread CTAs measured slower: they find no slot beside
+                                     //  the classify CTAs, and one CTA sorting 3-4k keys is a long chain)
+constexpr int kSortPer = 4;                                  // keys per thread in registers
+constexpr int kIsortTile = kIsortThreads * kSortPer;         // 1024
+constexpr int kSampleStride = 32;                            // <= 32 samples per tile
+struct ISortShared {
+    uint64_t k[kIsortTile];
+    uint32_t v[kIsortTile];
 };
+constexpr size_t kIsortSmem = sizeof(ISortShared);
 
-__device__ void sort_role(const P& p, uint32_t tile, SortShared& S) {
+__global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    ISortShared& S = *reinterpret_cast<ISortShared*>(smem_raw);
     const unsigned long long tl0 = TL_NOW();
     unsigned long long tl_p = tl0;
     const uint32_t n = p.d.ctl->nI;
-    const uint32_t t0 = tile * kSortTile;
-    if (t0 < n) {
-        const uint32_t o = threadIdx.x * kSortPer;  // this thread's consecutive elements
-        uint64_t k[kSortPer];
-        uint32_t v[kSortPer];
+    const uint32_t t0 = blockIdx.x * kIsortTile;
+    if (t0 >= n) return;
+    const uint32_t o = threadIdx.x * kSortPer;  // this thread's consecutive elements
+    uint64_t k[kSortPer];
+    uint32_t v[kSortPer];
 #pragma unroll
-        for (int r = 0; r < kSortPer; ++r) {
-            const uint32_t g = t0 + o + r;
-            k[r] = g < n ? __ldcg(p.d.sk[0] + g) : ~0ull;
-            v[r] = g < n ? __ldcg(p.d.sv[0] + g) : 0xFFFFFFFFu;
-        }
-        warp_bitonic_kv<kSortPer>(k, v);
-        TL_PHASE(2, 30, tl_p);  // load + warp bitonic
-#pragma unroll 1
-        for (uint32_t run = 32 * kSortPer; run < kSortTile; run <<= 1) {
-#pragma unroll
-            for (int r = 0; r < kSortPer; ++r) { S.k[o + r] = k[r]; S.v[o + r] = v[r]; }
-            __syncthreads();
-            const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
-            const uint32_t d = o - a0;
-            uint32_t lo = d > run ? d - run : 0, hi = min(d, run);
-            while (lo < hi) {  // merge path: A elements among the first d of the merged pair
-                const uint32_t mid = (lo + hi) >> 1;
-                const uint32_t pb = b0 + d - 1 - mid, pa = a0 + mid;
-                const uint64_t x = S.k[pa], y = S.k[pb];  // values only break key ties
-                if (x < y || (x == y && S.v[pa] < S.v[pb])) lo = mid + 1; else hi = mid;
-            }
-            uint32_t ia = lo, ib = d - lo;
-#pragma unroll
-            for (int r = 0; r < kSortPer; ++r) {
-                const uint32_t pa = a0 + min(ia, run - 1), pb = b0 + min(ib, run - 1);
-                const uint64_t ka = S.k[pa], kb = S.k[pb];
-                const uint32_t va = S.v[pa], vb = S.v[pb];
-                const bool takeA = ib >= run || (ia < run && kv_less(ka, va, kb, vb));
-                k[r] = takeA ? ka : kb;
-                v[r] = takeA ? va : vb;
-                if (takeA) ++ia; else ++ib;
-            }
-            __syncthreads();
-        }
-        TL_PHASE(2, 31, tl_p);  // shared-memory merges
-        const bool single = n <= kSortTile;  // one tile: its order is final
-        medusa_alloc x[kSortPer];
-        if (single) {  // all record loads first (independent), then the writes
-#pragma unroll
-            for (int r = 0; r < kSortPer; ++r)
-                if (o + r < n) x[r] = ld_alloc(p.a.alloc + v[r]);
-        }
-#pragma unroll
-        for (int r = 0; r < kSortPer; ++r) {
-            const uint32_t q = o + r;
-            if (t0 + q >= n) break;
-            if (single) {
-                write_i_entry(p, q, n, v[r], x[r]);
-            } else {
-                p.d.sk[1][t0 + q] = k[r];
-                p.d.sv[1][t0 + q] = v[r];
-                if ((q & 31) == 0) {  // every 32nd key: the tile's sample for k_rank
-                    p.d.samp_k[t0 / 32 + q / 32] = k[r];
-                    p.d.samp_v[t0 / 32 + q / 32] = v[r];
-                }
-            }
-        }
-        TL_REC(2, 0, tl0);
+    for (int r = 0; r < kSortPer; ++r) {
+        const uint32_t g = t0 + o + r;
+        k[r] = g < n ? __ldcg(p.d.sk0 + g) : ~0ull;
+        v[r] = g < n ? __ldcg(p.d.sv0 + g) : 0xFFFFFFFFu;
     }
-}
-
-// one CTA per tile of kSortTile I keys (side stream, after k_trace)
-__global__ void __launch_bounds__(kThreads) k_isort(P p) {
-    __shared__ SortShared S;
-    const unsigned long long tl0 = TL_NOW();
-    pdl_wait();
-    sort_role(p, blockIdx.x, S);
-    (void)tl0;
+    warp_bitonic_kv<kSortPer>(k, v);
+    TL_PHASE(2, 30, tl_p);  // load + warp bitonic
+#pragma unroll 1
+    for (uint32_t run = 32 * kSortPer; run < kIsortTile; run <<= 1) {
+#pragma unroll
+        for (int r = 0; r < kSortPer; ++r) { S.k[o + r] = k[r]; S.v[o + r] = v[r]; }
+        __syncthreads();
+        const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
+        const uint32_t d = o - a0;
+        uint32_t lo = d > run ? d - run : 0, hi = min(d, run);
+        while (lo < hi) {  // merge path: A elements among the first d of the merged pair
+            const uint32_t mid = (lo + hi) >> 1;
+            const uint32_t pb = b0 + d - 1 - mid, pa = a0 + mid;
+            const uint64_t x = S.k[pa], y = S.k[pb];  // values only break key ties
+            if (x < y || (x == y && S.v[pa] < S.v[pb])) lo = mid + 1; else hi = mid;
+        }
+        uint32_t ia = lo, ib = d - lo;
+#pragma unroll
+        for (int r = 0; r < kSortPer; ++r) {
+            const uint32_t pa = a0 + min(ia, run - 1), pb = b0 + min(ib, run - 1);
+            const uint64_t ka = S.k[pa], kb = S.k[pb];
+            const uint32_t va = S.v[pa], vb = S.v[pb];
+            const bool takeA = ib >= run || (ia < run && kv_less(ka, va, kb, vb));
+            k[r] = takeA ? ka : kb;
+            v[r] = takeA ? va : vb;
+            if (takeA) ++ia; else ++ib;
+        }
+        __syncthreads();
+    }
+    TL_PHASE(2, 31, tl_p);  // shared-memory merges
+    const bool single = n <= (uint32_t)kIsortTile;  // one tile: its order is final
+    medusa_alloc x[kSortPer];
+    if (single) {  // all record loads first (independent), then the writes
+#pragma unroll
+        for (int r = 0; r < kSortPer; ++r)
+            if (o + r < n) x[r] = ld_alloc(p.a.alloc + v[r]);
+    }
+#pragma unroll
+    for (int r = 0; r < kSortPer; ++r) {
+        const uint32_t q = o + r;
+        if (t0 + q >= n) break;
+        if (single) {
+            write_i_entry(p, q, n, v[r], x[r]);
+        } else {
+            p.d.sk[t0 + q] = k[r];
+            p.d.sv[t0 + q] = v[r];
+            if ((q % kSampleStride) == 0) {  // the tile's sample for k_rank
+                p.d.samp_k[t0 / kSampleStride + q / kSampleStride] = k[r];
+                p.d.samp_v[t0 / kSampleStride + q / kSampleStride] = v[r];
+            }
+        }
+    }
+    TL_REC(2, 0, tl0);
     pdl_trigger();
 }
 
 // ----------------------------------------------------------------------------
-// 2b. k_rank (after k_isort): global rank of every I key = its index in its sorted
-//     tile + the count of smaller keys in every other tile.  One CTA per range of
-//     32 consecutive keys of one tile (one key per lane); warp w counts against
-//     tiles b = w, w + 8, ...: the tile's 64-key sample (every 32nd key) comes in
-//     with one coalesced load and locates, by a shuffle search, the 32-key block
-//     of the tile holding each lane's lower bound; the block comes in with one
-//     more coalesced load and a shuffle search finishes the count.  The counts
-//     of the 8 warps meet in shared memory; warp 0 writes the 32 I entries.
+// 2b. k_rank (after k_isort, only with more than one tile): global rank of every
+//     I key = its index in its sorted tile + the count of smaller keys in every
+//     other tile.  One CTA per range of 32 consecutive keys of one tile (one key
+//     per lane); warp w counts against tiles b = w, w + 8, ...: the tile's <= 32
+//     samples (every 32nd key) come in with one coalesced load and locate, by a
+//     shuffle search, the 32-key block of the tile holding each lane's lower
+//     bound; the block comes in with one more coalesced load and a shuffle
+//     search finishes the count.  The counts of the 8 warps meet in shared
+//     memory; warp 0 writes the 32 I entries.
 __device__ __forceinline__ bool kv_lt_lane(uint64_t k, uint32_t v, uint32_t src, uint64_t xk, uint32_t xv) {
     const uint64_t sk = __shfl_sync(0xffffffffu, k, src);
     const uint32_t sv = __shfl_sync(0xffffffffu, v, src);
     return kv_less(sk, sv, xk, xv);
+}
+
+// number of the <= 64 ascending entries (entry e: lane e % 32 of half e / 32) that
+// are below (xk, xv) -- this lane's key; ne = entries present
+__device__ __forceinline__ uint32_t count_lt64(uint64_t k0, uint32_t v0, uint64_t k1, uint32_t v1, uint32_t ne,
+                                               uint64_t xk, uint32_t xv) {
+    const bool hi_half = ne > 32 && kv_lt_lane(k1, v1, 0, xk, xv);  // entry 32 < x
+    // count below x inside the lane's half (32 ascending entries); the source
+    // lane's value of BOTH halves is fetched, the lane picks
+    uint32_t lo = 0, hi = 32;
+#pragma unroll
+    for (int st = 0; st < 6; ++st) {
+        const uint32_t mid = (lo + hi) >> 1;
+        const bool lt0 = kv_lt_lane(k0, v0, min(mid, 31u), xk, xv);
+        const bool lt1 = kv_lt_lane(k1, v1, min(mid, 31u), xk, xv);
+        const bool lt = hi_half ? lt1 : lt0;
+        if (lo < hi) { if (lt) lo = mid + 1; else hi = mid; }
+    }
+    const uint32_t c = (hi_half ? 32 : 0) + lo;
+    return c > ne ? ne : c;
 }
 
 __global__ void __launch_bounds__(kThreads) k_rank(P p) {
@@ -469,47 +489,31 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
-    const uint32_t T = n_tiles(nI);
+    const uint32_t T = (nI + kIsortTile - 1) / kIsortTile;
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     // ranges of 32 keys, grid-stride (the grid is sized by the allocation count)
     for (uint32_t g0 = blockIdx.x * 32; T > 1 && g0 < nI; g0 += gridDim.x * 32) {
-        const uint32_t ta = g0 / kSortTile;
+        const uint32_t ta = g0 / kIsortTile;
         const uint32_t g = g0 + lane;
         const bool has = g < nI;
-        const uint64_t xk = has ? __ldcg(p.d.sk[1] + g) : ~0ull;
-        const uint32_t xv = has ? __ldcg(p.d.sv[1] + g) : 0xFFFFFFFFu;
+        const uint64_t xk = has ? __ldcg(p.d.sk + g) : ~0ull;
+        const uint32_t xv = has ? __ldcg(p.d.sv + g) : 0xFFFFFFFFu;
         uint32_t cnt = 0;
         for (uint32_t tb = warp; tb < T; tb += kWarps) {
             if (tb == ta) continue;
-            const uint32_t b0 = tb * kSortTile, nb = min((uint32_t)kSortTile, nI - b0);
-            const uint32_t ns = (nb + 31) / 32;  // samples of tile tb (<= 64)
-            // samples ns_l = lane, lane + 32
+            const uint32_t b0 = tb * kIsortTile, nb = min((uint32_t)kIsortTile, nI - b0);
+            const uint32_t ns = (nb + kSampleStride - 1) / kSampleStride;  // samples of tile tb (<= 64)
+            const uint32_t s0 = b0 / kSampleStride;
             uint64_t sk0 = ~0ull, sk1 = ~0ull;
             uint32_t sv0 = 0xFFFFFFFFu, sv1 = 0xFFFFFFFFu;
-            if (lane < ns) { sk0 = __ldcg(p.d.samp_k + b0 / 32 + lane); sv0 = __ldcg(p.d.samp_v + b0 / 32 + lane); }
-            if (lane + 32 < ns) { sk1 = __ldcg(p.d.samp_k + b0 / 32 + lane + 32); sv1 = __ldcg(p.d.samp_v + b0 / 32 + lane + 32); }
+            if (lane < ns) { sk0 = __ldcg(p.d.samp_k + s0 + lane); sv0 = __ldcg(p.d.samp_v + s0 + lane); }
+            if (lane + 32 < ns) { sk1 = __ldcg(p.d.samp_k + s0 + lane + 32); sv1 = __ldcg(p.d.samp_v + s0 + lane + 32); }
             // j = #samples < x: the lower bound of x lies in block j - 1 (j >= 1)
-            uint32_t j = 0;
-            {
-                const bool hi_half = ns > 32 && kv_lt_lane(sk1, sv1, 0, xk, xv);  // sample 32 < x
-                // count of samples < x inside this lane's half (32 entries, ascending);
-                // the source lane's value of BOTH halves is fetched, the lane picks
-                uint32_t lo = 0, hi = 32;
-#pragma unroll
-                for (int st = 0; st < 6; ++st) {
-                    const uint32_t mid = (lo + hi) >> 1;
-                    const bool lt0 = kv_lt_lane(sk0, sv0, min(mid, 31u), xk, xv);
-                    const bool lt1 = ns > 32 && kv_lt_lane(sk1, sv1, min(mid, 31u), xk, xv);
-                    const bool lt = hi_half ? lt1 : lt0;
-                    if (lo < hi) { if (lt) lo = mid + 1; else hi = mid; }
-                }
-                j = (hi_half ? 32 : 0) + lo;
-                if (j > ns) j = ns;
-            }
+            const uint32_t j = count_lt64(sk0, sv0, sk1, sv1, ns, xk, xv);
             // lane l's lower bound lies in block j_l - 1 (ascending over the lanes).
             // Few distinct blocks (the usual case): load each with one coalesced
             // load and count by a shuffle search; otherwise every lane searches its
-            // own block in memory (5 dependent loads).
+            // own block in memory (6 dependent loads).
             const uint32_t blk = j ? j - 1 : 0xFFFFFFFFu;
             const bool act = has && j;
             const uint32_t prev = __shfl_up_sync(0xffffffffu, blk, 1);
@@ -519,26 +523,24 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
                 uint32_t pending = __ballot_sync(0xffffffffu, act);
                 while (pending) {
                     const uint32_t bl = __shfl_sync(0xffffffffu, blk, __ffs(pending) - 1);
-                    const uint32_t q = bl * 32 + lane;
-                    const uint64_t bk = q < nb ? __ldcg(p.d.sk[1] + b0 + q) : ~0ull;
-                    const uint32_t bv = q < nb ? __ldcg(p.d.sv[1] + b0 + q) : 0xFFFFFFFFu;
-                    uint32_t lo = 0, hi = 32;  // entries of the block below x
-#pragma unroll
-                    for (int st = 0; st < 6; ++st) {
-                        const uint32_t mid = (lo + hi) >> 1;
-                        const bool lt = kv_lt_lane(bk, bv, min(mid, 31u), xk, xv);
-                        if (lo < hi) { if (lt) lo = mid + 1; else hi = mid; }
-                    }
-                    if (act && blk == bl) c = bl * 32 + lo;
+                    const uint32_t q0 = bl * kSampleStride, ne = min((uint32_t)kSampleStride, nb - q0);
+                    const uint32_t qa = q0 + lane, qb = q0 + 32 + lane;
+                    const uint64_t ka = qa < nb ? __ldcg(p.d.sk + b0 + qa) : ~0ull;
+                    const uint32_t va = qa < nb ? __ldcg(p.d.sv + b0 + qa) : 0xFFFFFFFFu;
+                    const bool two = kSampleStride > 32 && qb < nb;
+                    const uint64_t kb = two ? __ldcg(p.d.sk + b0 + qb) : ~0ull;
+                    const uint32_t vb = two ? __ldcg(p.d.sv + b0 + qb) : 0xFFFFFFFFu;
+                    const uint32_t below = count_lt64(ka, va, kb, vb, ne, xk, xv);
+                    if (act && blk == bl) c = q0 + below;
                     pending &= ~__ballot_sync(0xffffffffu, act && blk == bl);
                 }
             } else if (act) {
-                const uint32_t q0 = blk * 32;
-                uint32_t lo = 0, hi = min(32u, nb - q0);
+                const uint32_t q0 = blk * kSampleStride;
+                uint32_t lo = 0, hi = min((uint32_t)kSampleStride, nb - q0);
                 while (lo < hi) {
                     const uint32_t mid = (lo + hi) >> 1;
-                    const uint64_t bk = __ldcg(p.d.sk[1] + b0 + q0 + mid);
-                    const bool lt = bk < xk || (bk == xk && __ldcg(p.d.sv[1] + b0 + q0 + mid) < xv);
+                    const uint64_t bk = __ldcg(p.d.sk + b0 + q0 + mid);
+                    const bool lt = bk < xk || (bk == xk && __ldcg(p.d.sv + b0 + q0 + mid) < xv);
                     if (lt) lo = mid + 1; else hi = mid;
                 }
                 c = q0 + lo;
@@ -548,7 +550,7 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
         s_cnt[warp][lane] = cnt;
         __syncthreads();
         if (warp == 0 && has) {
-            uint32_t rank = g - ta * kSortTile;  // index inside its own tile
+            uint32_t rank = g - ta * kIsortTile;  // index inside its own tile
 #pragma unroll
             for (int w = 0; w < kWarps; ++w) rank += s_cnt[w][lane];
             write_i_entry(p, rank, nI, xv, ld_alloc(p.a.alloc + xv));
@@ -649,54 +651,86 @@ __device__ __forceinline__ void window_load(const P& p, ClsShared& S, uint32_t m
 // chunk = the ordinals i in [o_lo, o_hi) with v_i > T0 (a mortal freed after the
 // chunk's first launch) and t_alloc_i < T1 (allocated before its last launch)
 // and, when every segment's launch position is in nt0 (exact), live at one of
-// them: t_alloc_i < nt0[u] < t_free_i for some u.  One level per round: each warp
-// expands one kept node into its 32 children with one coalesced load.  The
-// entries go to S.wid[0 .. S.nres).  Returns false if a level keeps more than
-// kFront nodes or the entries exceed kWinCap (the caller halves the range).
-__device__ bool tree_query(const Tree& T, ClsShared& S, uint32_t T0, uint32_t T1, uint32_t o_lo, uint32_t o_hi,
-                           uint32_t ng0, bool exact) {
-    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid <= (uint32_t)kMaxLevels) S.fn[tid] = 0;
-    if (tid == 0) S.nres = 0;
-    __syncthreads();
-    for (int l = (int)T.top; l >= 0; --l) {
-        const bool root = l == (int)T.top;  // the virtual root: its children are the top level
-        const uint32_t np = root ? 1u : S.fn[l + 1];
-        const uint32_t* par = S.front[(l + 1) & 1];
-        uint32_t* out = l > 0 ? S.front[l & 1] : S.wid;
-        uint32_t* cnt = l > 0 ? &S.fn[l] : &S.nres;
-        const uint32_t cap = l > 0 ? (uint32_t)kFront : (uint32_t)kWinCap;
-        const uint32_t sh = 5u * (uint32_t)l;  // a node of level l covers 2^sh ordinals
-        bool ovf = false;
-        for (uint32_t f = warp; f < np; f += kWarps) {
-            const uint32_t c = (root ? 0u : par[f]) * 32 + lane;
-            bool keep = false;
-            if (c < T.cnt[l]) {
-                const uint64_t first = (uint64_t)c << sh, last = first + (1ull << sh);
-                if (first < o_hi && last > o_lo) {
-                    const uint2 nd = l > 0 ? __ldcg(T.node + T.off[l] + c) : __ldcg(T.leaf + c);
-                    keep = nd.x > T0 && nd.y < T1;
-                    if (keep && l == 0 && exact) {  // live at one of the chunk's launches
-                        uint32_t lo = 0, hi = ng0;   // the first segment launched after t_alloc
-                        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt0[mid] <= nd.y) lo = mid + 1; else hi = mid; }
-                        keep = lo < ng0 && S.nt0[lo] < nd.x;
-                    }
-                }
-            }
-            const uint32_t b = __ballot_sync(0xffffffffu, keep);
-            if (b) {
-                uint32_t base = 0;
-                if (lane == 0) base = atomicAdd(cnt, (uint32_t)__popc(b));
-                base = __shfl_sync(0xffffffffu, base, 0);
-                const uint32_t pos = base + __popc(b & lanemask_lt());
-                if (keep) {
-                    if (pos < cap) out[pos] = c;
-                    else ovf = true;
-                }
-            }
-        }
-        if (__syncthreads_or(ovf)) return false;
+// them: t_alloc_i < nt0[u] < t_free_i for some u.  The descent starts at the
+// highest level with <= kThreads nodes (one thread each: q_seed) and goes one
+// level per round (q_expand: each warp expands one kept node into its 32
+// children with one coalesced load).  Kept nodes of level l go to
+// S.front[l & 1], the entries (level 0) to S.wid[0 .. S.nres).
+struct QRange {
+    uint32_t T0, T1, o_lo, o_hi, ng0;
+    bool exact;
+};
+
+__device__ __forceinline__ int q_start(const Tree& T) {
+    int l = (int)T.top;
+    while (l > 0 && T.cnt[l - 1] <= (uint32_t)kThreads) --l;
+    return l;
+}
+
+__device__ __forceinline__ bool q_test(const Tree& T, const ClsShared& S, int l, uint32_t c, const QRange& q) {
+    if (c >= T.cnt[l]) return false;
+    const uint32_t sh = 5u * (uint32_t)l;  // a node of level l covers 2^sh ordinals
+    const uint64_t first = (uint64_t)c << sh, last = first + (1ull << sh);
+    if (!(first < q.o_hi && last > q.o_lo)) return false;
+    const uint2 nd = l > 0 ? __ldcg(T.node + T.off[l] + c) : __ldcg(T.leaf + c);
+    bool keep = nd.x > q.T0 && nd.y < q.T1;
+    if (keep && l == 0 && q.exact) {  // live at one of the chunk's launches
+        uint32_t lo = 0, hi = q.ng0;   // the first segment launched after t_alloc
+        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt0[mid] <= nd.y) lo = mid + 1; else hi = mid; }
+        keep = lo < q.ng0 && S.nt0[lo] < nd.x;
     }
+    return keep;
+}
+
+// (whole warp) appends the lanes' kept nodes of level l; false if the list overflows
+__device__ __forceinline__ bool q_push(ClsShared& S, int l, bool keep, uint32_t c) {
+    const uint32_t b = __ballot_sync(0xffffffffu, keep);
+    if (!b) return true;
+    const uint32_t lane = threadIdx.x & 31;
+    uint32_t* out = l > 0 ? S.front[l & 1] : S.wid;
+    uint32_t* cnt = l > 0 ? &S.fn[l] : &S.nres;
+    const uint32_t cap = l > 0 ? (uint32_t)kFront : (uint32_t)kWinCap;
+    uint32_t base = 0;
+    if (lane == 0) base = atomicAdd(cnt, (uint32_t)__popc(b));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    const uint32_t pos = base + __popc(b & lanemask_lt());
+    if (keep && pos < cap) out[pos] = c;
+    return !(keep && pos >= cap);
+}
+
+// (whole CTA, no barrier) the start level's nodes, one per thread
+__device__ __forceinline__ bool q_seed(const Tree& T, ClsShared& S, int l, const QRange& q) {
+    const uint32_t c = threadIdx.x;
+    return q_push(S, l, q_test(T, S, l, c, q), c);
+}
+
+// (whole CTA, no barrier) the children at level l of the kept nodes of level l+1
+__device__ __forceinline__ bool q_expand(const Tree& T, ClsShared& S, int l, const QRange& q) {
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t np = min(S.fn[l + 1], (uint32_t)kFront);
+    const uint32_t* par = S.front[(l + 1) & 1];
+    bool ok = true;
+    for (uint32_t f = warp; f < np; f += kWarps) {
+        const uint32_t c = par[f] * 32 + lane;
+        ok &= q_push(S, l, q_test(T, S, l, c, q), c);
+    }
+    return ok;
+}
+
+// (whole CTA) counters of a query; the caller's next barrier publishes them
+__device__ __forceinline__ void q_reset(ClsShared& S) {
+    if (threadIdx.x <= (uint32_t)kMaxLevels) S.fn[threadIdx.x] = 0;
+    if (threadIdx.x == 0) S.nres = 0;
+}
+
+// a whole query over [q.o_lo, q.o_hi); false on overflow (the caller halves the range)
+__device__ bool tree_query(const Tree& T, ClsShared& S, const QRange& q) {
+    q_reset(S);
+    __syncthreads();
+    const int l0 = q_start(T);
+    if (__syncthreads_or(!q_seed(T, S, l0, q))) return false;
+    for (int l = l0 - 1; l >= 0; --l)
+        if (__syncthreads_or(!q_expand(T, S, l, q))) return false;
     return true;
 }
 
@@ -808,7 +842,8 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     const bool tma = ((reinterpret_cast<uintptr_t>(gsrc) & 15) == 0) && (n % 2 == 0);
     const uint32_t mb = smem_u32(&S.mbar);
     // A. the chunk's words -> shared memory with one TMA bulk copy, issued before
-    //    waiting for k_trace (the words are an input)
+    //    waiting for k_trace (the words are an input; k_trace lets this grid start
+    //    at once in the slots it leaves free)
     if (tid == 0 && tma) {
         asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -818,12 +853,14 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     }
     if (tid < MEDUSA_CHUNK_WORDS / 32) S.nsm[tid] = 0;
     if (tid < kNodeGrp) S.nt0[tid] = 0;
+    q_reset(S);
     pdl_wait();  // k_trace: node ranges, status, prefilter bounds, the mortal tree
+    const uint32_t st = __ldcg(&ctl->status);
     // A malformed CSR or launch order (flagged by k_trace) leaves jf / jl and the
     // node offsets meaningless: write the empty counts the later kernels read and
     // do nothing else (the call returns INVALID_ARG; no shared-memory index is
     // ever derived from node_off); the bulk copy is waited for before leaving
-    if (__ldcg(&ctl->status) & ST_INVALID) {
+    if (st & ST_INVALID) {
         if (tid < kWarps) p.d.qcnt[c * kWarps + tid] = 0;
         if (tid == 0) p.d.chunk_cnt[c] = 0;
         if (tid == 0 && tma) {
@@ -837,16 +874,26 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         return;
     }
     const uint32_t N = a.n_nodes;
-    const uint32_t jf = N ? min(__ldcg(p.d.jf + c), N - 1) : 0, jl = N ? min(__ldcg(p.d.jl + c), N - 1) : 0;
+    const uint2 jf2 = N ? __ldcg(p.d.jf + c) : make_uint2(0, 0), jl2 = N ? __ldcg(p.d.jl + c) : make_uint2(0, 0);
+    const uint32_t jf = N ? min(jf2.x, N - 1) : 0, jl = N ? min(jl2.x, N - 1) : 0;
+    const uint32_t t_jf = jf2.y, t_jl = jl2.y;  // the chunk's first and last launch positions
     const uint32_t nn = N ? jl - jf + 1 : 0;
     const uint64_t gmin = ~__ldcg(&ctl->gmin_c), gmax = __ldcg(&ctl->gmax);
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
-    const uint32_t t_jf = N ? __ldg(a.node_t + jf) : 0, t_jl = N ? __ldg(a.node_t + jl) : 0;
-    __syncthreads();  // nsm / nt0 zeroed before any thread sets a bit
+    const uint32_t n_alloc = a.n_alloc;
+    const bool use_tree = N && n_alloc;
+    const Tree& T = p.d.tree;
+    const int l0 = q_start(T);
+    QRange qr{t_jf, t_jl, 0u, n_alloc, 0u, true};
+    __syncthreads();  // nsm / nt0 / query counters zeroed before any thread sets them
     TL_PHASE(4, 10, tl_p);  // A: setup
     // B. the starts of the chunk's nodes (-> start bitmask, its popcount prefix,
-    //    the launch positions of the first kNodeGrp segments)
+    //    the launch positions of the first kNodeGrp segments), interleaved with
+    //    the first two rounds of the window's tree query (the internal levels
+    //    need only the chunk's first and last launch positions)
+    bool qok = true;
+    if (use_tree && l0 >= 1) qok &= q_seed(T, S, l0, qr);
     uint32_t my_q = 0xFFFFFFFFu, my_t = 0;  // this thread's first node (start, launch position)
     for (uint32_t j = jf + 1 + tid; j <= jl; j += kThreads) {
         const uint32_t q = (uint32_t)(a.node_off[j] - cs);
@@ -866,9 +913,12 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         S.nsp[2 * lane] = incl - c0 - c1;
         S.nsp[2 * lane + 1] = incl - c1;
     }
+    if (use_tree && l0 >= 2) qok &= q_expand(T, S, l0 - 1, qr);
     __syncthreads();
     const uint32_t n_seg = N ? S.nsp[63] + __popc(S.nsm[63]) + 1 : 0;
     const uint32_t ng0 = min((uint32_t)kNodeGrp, n_seg);
+    qr.ng0 = ng0;
+    qr.exact = n_seg <= (uint32_t)kNodeGrp;
     // launch positions of segments 0..ng0-1 (the last node of a start is its non-empty one)
     if (tid == 0 && N) atomicMax(&S.nt0[0], t_jf);
     if (my_q != 0xFFFFFFFFu) {
@@ -909,22 +959,36 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         nc += __popc(b0) + __popc(b1);
     }
     if (lane < 8) wh[lane] = 0;
-    TL_PHASE(4, 11, tl_p);  // B/C: node starts, TMA wait, candidates
-    // D. the window: the mortals live at one of the chunk's launches, found by a
-    //    descent of the mortal tree (normally one batch of <= kWinCap entries; a
-    //    query that overflows is retried on half the ordinal range, and the
-    //    ranges are then processed one batch after another).  Per batch and node
-    //    group (normally one: <= kNodeGrp segments): the live masks, then each
-    //    warp looks its own candidates up among the entries live at their node.
-    const bool exact = n_seg <= (uint32_t)kNodeGrp;
-    const uint32_t n_alloc = a.n_alloc;
-    uint32_t o_lo = 0, wlen = n_alloc;
-    while (N && o_lo < n_alloc) {
-        const uint32_t o_hi = (uint32_t)min((uint64_t)o_lo + wlen, (uint64_t)n_alloc);
-        if (!tree_query(p.d.tree, S, t_jf, t_jl, o_lo, o_hi, ng0, exact)) {
-            wlen = (wlen + 1) / 2;
-            continue;
+    // the rest of the query (the leaves need nt0: complete after this barrier)
+    qok = !__syncthreads_or(!qok);
+    TL_PHASE(4, 11, tl_p);  // B/C: node starts, TMA wait, candidates, upper query levels
+    if (use_tree && qok) {
+        for (int l = l0 >= 2 ? l0 - 2 : 0; l >= 0; --l) {
+            if (l == l0) qok = !__syncthreads_or(!q_seed(T, S, l, qr));  // (l0 == 0: the leaves are the start level)
+            else qok = !__syncthreads_or(!q_expand(T, S, l, qr));
+            if (!qok) break;
         }
+    }
+    // D. the window: the mortals live at one of the chunk's launches (normally one
+    //    batch of <= kWinCap entries; a query that overflows is retried on half the
+    //    ordinal range, and the ranges are then processed one batch after
+    //    another).  Per batch and node group (normally one: <= kNodeGrp
+    //    segments): the live masks, then each warp looks its own candidates up
+    //    among the entries live at their node.
+    bool have = qok;  // results of the first query (the whole ordinal range) in S.wid
+    uint32_t o_lo = 0, wlen = qok ? n_alloc : (n_alloc + 1) / 2;
+    while (use_tree && o_lo < n_alloc) {
+        uint32_t o_hi = n_alloc;
+        if (!have) {
+            o_hi = (uint32_t)min((uint64_t)o_lo + wlen, (uint64_t)n_alloc);
+            qr.o_lo = o_lo;
+            qr.o_hi = o_hi;
+            if (!tree_query(T, S, qr)) {
+                wlen = (wlen + 1) / 2;
+                continue;
+            }
+        }
+        have = false;
         const uint32_t m = S.nres;
         __syncthreads();  // every thread has read nres before a later query resets it
         TL_PHASE(4, 12, tl_p);  // D: tree query
@@ -1011,51 +1075,43 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
 }
 
 // ----------------------------------------------------------------------------
-// 2c. k_check (after k_rank, default priority): the R-Q7 checks.
-//     I-I: adjacent sorted I entries (the CTA checks 256 pairs).  Per warp, a
-//     block of 32 allocation ordinals: M-M -- each mortal j against the mortals
-//     i < j still live when j is allocated (t_free_i > t_alloc_j), found by a
-//     depth-first descent of the mortal tree (nodes with max t_free > the block's
-//     least t_alloc and first ordinal < its greatest ordinal), then
-//     hull-filtered and tested pairwise; M-I -- each mortal against the run of
-//     I entries its range meets (one fence search; the common "no I entry in
-//     range" case costs two more loads).
+// 2c. The R-Q7 checks (default priority; they only set ST_TRACE), per warp a
+//     block of 32 allocation ordinals, one per lane ("mine" = a mortal):
+//     k_check_mm (after k_trace): M-M -- each mortal j against the mortals
+//       i < j still live when j is allocated (t_free_i > t_alloc_j), found by a
+//       depth-first descent of the mortal tree (nodes with max t_free > the
+//       block's least t_alloc and first ordinal < its greatest ordinal), then
+//       hull-filtered and tested pairwise;
+//     k_check_mi (after k_rank): I-I -- adjacent sorted I entries; M-I -- each
+//       mortal against the run of I entries its range meets (one fence search;
+//       the common "no I entry in range" case costs two more loads).
 constexpr int kStk = 32 * kMaxLevels + 32;  // DFS stack per warp: < 32 entries per level on the path
-__global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
-    __shared__ uint64_t s_fence[kFenceCap];
+
+// this lane's allocation of block b and whether it is a mortal
+__device__ __forceinline__ bool check_mine(const P& p, uint32_t j, medusa_alloc& x, uint32_t& t_last) {
+    const uint32_t N = p.a.n_nodes;
+    t_last = N ? p.a.node_t[N - 1] : 0;
+    x = medusa_alloc{};
+    if (j >= p.a.n_alloc) return false;
+    x = ld_alloc(p.a.alloc + j);
+    return x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
+}
+
+__global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
     __shared__ ulonglong2 s_be[kWarps][32];  // (base, end): one 16-byte broadcast load
     __shared__ uint2 s_ti[kWarps][32];       // (t_free, id): one 8-byte broadcast load
     __shared__ uint32_t s_stk[kWarps][kStk];
     const unsigned long long tl0 = TL_NOW();
-    pdl_wait();
-    pdl_trigger();
-    const uint32_t cta = blockIdx.x;
-    const MaterializeArgs& a = p.a;
     const Tree& T = p.d.tree;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t nI = p.d.ctl->nI;
-    {  // I-I: sorted neighbours must not overlap (all of I is live at the last launch)
-        const uint32_t k = cta * blockDim.x + threadIdx.x;
-        if (k + 1 < nI && p.d.i_rest[k].end > p.d.i_base[k + 1]) flag(p.d.ctl, ST_TRACE);
-    }
-    const uint32_t stride = fence_stride(nI);
-    const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = __ldcg(p.d.fence + f);
-    __syncthreads();
-    const uint32_t b = cta * kWarps + warp;
+    const uint32_t b = blockIdx.x * kWarps + warp;
     if (b >= p.nb) return;  // whole warp
     const uint32_t j = b * 32 + lane;
-    bool mine = false;
-    medusa_alloc x{};
-    const uint32_t N = a.n_nodes;
-    const uint32_t t_last = N ? a.node_t[N - 1] : 0;
-    if (j < a.n_alloc) {
-        x = ld_alloc(a.alloc + j);
-        mine = x.size != 0 && !(N && x.t_alloc < t_last && t_last < x.t_free);
-    }
+    medusa_alloc x;
+    uint32_t t_last;
+    const bool mine = check_mine(p, j, x, t_last);
     const uint64_t xe = x.base + x.size;
     bool bad = false;
-    // M-M
     const uint64_t hb = warp_min_u64(mine ? x.base : ~0ull), he = warp_max_u64(mine ? xe : 0ull);
     const uint32_t hta = __reduce_min_sync(0xffffffffu, mine ? x.t_alloc : 0xFFFFFFFFu);
     const uint32_t hj = __reduce_max_sync(0xffffffffu, mine ? j : 0u);
@@ -1082,7 +1138,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
                 uint64_t yb = 0, ye = 0;
                 bool k2 = false;
                 if (keep) {
-                    const medusa_alloc r = ld_alloc(a.alloc + c);
+                    const medusa_alloc r = ld_alloc(p.a.alloc + c);
                     yb = r.base;
                     ye = r.base + r.size;
                     k2 = yb < he && hb < ye;
@@ -1111,6 +1167,32 @@ __global__ void __launch_bounds__(kThreads, 6) k_check(P p) {
             node = e & 0xFFFFFFu;
         }
     }
+    if (bad) flag(p.d.ctl, ST_TRACE);
+    TL_REC(8, 0, tl0);
+}
+
+__global__ void __launch_bounds__(kThreads, 6) k_check_mi(P p) {
+    __shared__ uint64_t s_fence[kFenceCap];
+    const unsigned long long tl0 = TL_NOW();
+    const uint32_t cta = blockIdx.x;
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t nI = p.d.ctl->nI;
+    {  // I-I: sorted neighbours must not overlap (all of I is live at the last launch)
+        const uint32_t k = cta * blockDim.x + threadIdx.x;
+        if (k + 1 < nI && p.d.i_rest[k].end > p.d.i_base[k + 1]) flag(p.d.ctl, ST_TRACE);
+    }
+    const uint32_t stride = fence_stride(nI);
+    const uint32_t nf = (nI + stride - 1) / stride;
+    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = __ldcg(p.d.fence + f);
+    __syncthreads();
+    const uint32_t b = cta * kWarps + warp;
+    if (b >= p.nb) return;  // whole warp
+    const uint32_t j = b * 32 + lane;
+    medusa_alloc x;
+    uint32_t t_last;
+    const bool mine = check_mine(p, j, x, t_last);
+    const uint64_t xe = x.base + x.size;
+    bool bad = false;
     // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
     if (mine && nI) {
         const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);  // bases <= base
@@ -1333,7 +1415,8 @@ struct Scratch {
     int sm_count = 0;
     cudaStream_t side = nullptr;  // the I-list sort + rank branch (highest priority; forked from the caller's stream)
     cudaStream_t low = nullptr;   // the trace-check branch (default priority; joined before the call ends)
-    cudaEvent_t fork = nullptr, join = nullptr, ranked = nullptr, classified = nullptr, emitted = nullptr;
+    cudaEvent_t fork = nullptr, traced = nullptr, join = nullptr, ranked = nullptr, classified = nullptr,
+                emitted = nullptr;
     // Buffers retired by a growth.  A CUDA graph that captured an earlier
     // medusa_materialize_async holds their addresses by value, so they stay
     // allocated (replaying such a graph stays memory-safe) until
@@ -1392,8 +1475,8 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W) {
     o = (o + 63) & ~(size_t)63;
     s.d.tree.node = (uint2*)(z + o);
     if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) ||
-        (e = grow(s, s.d.sk[0], N)) || (e = grow(s, s.d.sk[1], N)) || (e = grow(s, s.d.sv[0], N)) ||
-        (e = grow(s, s.d.sv[1], N)) || (e = grow(s, s.d.samp_k, N / 32 + 64)) || (e = grow(s, s.d.samp_v, N / 32 + 64)) ||
+        (e = grow(s, s.d.sk0, N)) || (e = grow(s, s.d.sv0, N)) || (e = grow(s, s.d.sk, N)) || (e = grow(s, s.d.sv, N)) ||
+        (e = grow(s, s.d.samp_k, N / kSampleStride + 64)) || (e = grow(s, s.d.samp_v, N / kSampleStride + 64)) ||
         (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
         (e = grow(s, s.d.fence, (size_t)kFenceCap)) || (e = grow(s, s.d.chunk_cnt, CC)) ||
         (e = grow(s, s.d.staging, WW)) || (e = grow(s, s.d.queue, CC * kChunkWords)) ||
@@ -1424,12 +1507,14 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
     if (!s.h_ctl) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kClsSmem);
+        cudaFuncSetAttribute(k_isort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kIsortSmem);
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
             (*e = cudaStreamCreateWithPriority(&s.low, cudaStreamNonBlocking, prio_lo)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming)) != cudaSuccess ||
+            (*e = cudaEventCreateWithFlags(&s.traced, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.ranked, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.classified, cudaEventDisableTiming)) != cudaSuccess ||
             (*e = cudaEventCreateWithFlags(&s.emitted, cudaEventDisableTiming)) != cudaSuccess)
@@ -1440,9 +1525,9 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
 }
 
 // the whole analysis on `stream` (no synchronization):
-//   stream:            memset -> k_trace [fork] -> k_classify [classified] ......... [emitted][join]
-//   side (high prio):                 [fork] k_isort -> k_rank [ranked] [classified] k_iresolve -> k_emit [emitted]
-//   low (default):                                       [ranked] k_check [join]
+//   stream:            memset -> k_trace [traced] -> k_classify [classified] .............. [emitted][join]
+//   side (high prio):             [traced] k_isort -> k_rank [ranked] [classified] k_iresolve -> k_emit [emitted]
+//   low (default):                    [traced] k_check_mm ... [ranked] k_check_mi [join]
 // The high-priority stream gets the sort / rank CTAs dispatched ahead of the
 // classify CTAs and the queue resolution / emission ahead of the trace checks,
 // which fill in around them and complete the call.
@@ -1452,7 +1537,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     const uint32_t nb = (uint32_t)((n + 31) / 32);
     const uint32_t node_ctas = (a.n_nodes + 1 + kThreads * kNodesPerThread - 1) / (kThreads * kNodesPerThread);
     const uint32_t alloc_ctas = (uint32_t)((n + kThreads - 1) / kThreads);
-    const uint32_t sort_ctas = (uint32_t)((n + kSortTile - 1) / kSortTile);
+    const uint32_t sort_ctas = (uint32_t)((n + kIsortTile - 1) / kIsortTile);
     const uint32_t check_ctas = (nb + kWarps - 1) / kWarps;
     Dev d = s.d;
     const Tree shape = tree_shape(n);
@@ -1471,12 +1556,12 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
     }
     if (n) {
-        if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(side, s.fork, 0))) return e;
+        if ((e = cudaEventRecord(s.traced, stream)) || (e = cudaStreamWaitEvent(side, s.traced, 0))) return e;
         {
             TimedLaunch tl("mat_isort", side);
-            k_isort<<<sort_ctas, kThreads, 0, side>>>(p);
+            k_isort<<<sort_ctas, kIsortThreads, kIsortSmem, side>>>(p);
         }
-        {
+        if (n > (uint64_t)kIsortTile) {  // (with one tile k_isort writes the I list itself)
             TimedLaunch tl("mat_rank", side);
             // one CTA per 32 I keys (the list's size is known on the device only: bound
             // by the allocation count; surplus CTAs exit at once)
@@ -1504,11 +1589,17 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
         }
         if ((e = cudaEventRecord(s.emitted, side))) return e;
-        // default priority: the trace checks fill in around them
+        // default priority: the trace checks fill in around them (M-M needs the
+        // mortal tree only, M-I and I-I the sorted I list)
+        if ((e = cudaStreamWaitEvent(low, s.traced, 0))) return e;
+        {
+            TimedLaunch tl("mat_check_mm", low);
+            k_check_mm<<<check_ctas, kThreads, 0, low>>>(p);
+        }
         if ((e = cudaStreamWaitEvent(low, s.ranked, 0))) return e;
         {
-            TimedLaunch tl("mat_check", low);
-            k_check<<<check_ctas, kThreads, 0, low>>>(p);
+            TimedLaunch tl("mat_check_mi", low);
+            k_check_mi<<<check_ctas, kThreads, 0, low>>>(p);
         }
         if ((e = cudaEventRecord(s.join, low))) return e;
         if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
