@@ -53,7 +53,7 @@ namespace {
 
 MEDUSA_TL_DEFINE
 
-constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2;
+constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
@@ -72,6 +72,7 @@ struct Ctl {
     unsigned long long gmin_c;  // ~(least base) via atomicMax
     unsigned long long gmax;    // greatest end
     unsigned long long n_slots;
+    unsigned int need_pw, pad2;           // entries per warp region a call needed (set only on overflow)
 };
 
 struct IRest {  // I-list entry (sorted order), base kept in a separate array
@@ -116,10 +117,15 @@ struct Dev {  // scratch of one call (device pointers)
     uint32_t* i_tf;                              // [n]
     uint64_t* fence;                             // [kFenceCap]
     uint32_t* chunk_cnt;                         // [C] slots per chunk
-    uint64_t* staging;                           // [n_words] record of slot g at index g
-    IQ* queue;                                   // [C * 2048] candidates for the I-list search: region
-                                                 //  of classify warp w of chunk c at c*2048 + 256 w
-    uint32_t* qcnt;                              // [C * 8] entries in each region
+    // Warp-local record regions: classify warp w of chunk c (its
+    // 256 words) owns entries [(8c + w) cap_pw, (8c + w + 1) cap_pw) of each,
+    // filled in word order
+    uint64_t* rec;                               // records of the window hits
+    IQ* queue;                                   // candidates left for the I-list search
+    uint64_t* irec;                              // the I-list record of queue entry k (hits only)
+    uint32_t cap_pw;                             // entries per warp region (128; 256 after an overflow)
+    uint32_t* qcnt;                              // [C * 8] queue entries of classify warp w of chunk c
+    uint32_t *imask, *qmask;                     // [ceil(n_words/32)] words resolved by the I list / queued
 };
 
 struct P {  // kernel parameters
@@ -586,7 +592,7 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
 //    mortal window (registered mortals in list order, per-node live masks);
 //    then each warp classifies its own 256 words with no further CTA barrier:
 //    word q of warp w is q = 256 w + 32 k + lane (k = 0..7).
-constexpr int kFront = 256;  // tree-query frontier nodes held per level
+constexpr int kFront = 128;  // tree-query frontier nodes held per level (ALL10: <= 29)
 struct ClsShared {
     uint64_t words[MEDUSA_CHUNK_WORDS];  // TMA destination; hit words then hold their record
     ulonglong2 rbe[kWinCap];             // (base, end) of one batch of window entries
@@ -598,12 +604,16 @@ struct ClsShared {
     uint32_t nsm[MEDUSA_CHUNK_WORDS / 32];  // bit q: a node starts at word q (q > 0)
     uint32_t nsp[MEDUSA_CHUNK_WORDS / 32];  // exclusive popcount prefix of nsm
     uint32_t nt0[kNodeGrp];                 // launch positions of segments 0 .. kNodeGrp-1
-    uint32_t nt[kNodeGrp];                  // launch positions of segments g0 .. g0+kNodeGrp-1 (later groups)
     uint16_t cq[MEDUSA_CHUNK_WORDS];        // per warp (256 each): its candidates (word in chunk)
     uint32_t hits[MEDUSA_CHUNK_WORDS / 32]; // slot bits (warp w: words 8w .. 8w+7)
-    uint32_t wcnt[kWarps];                  // slots found per warp
+    uint32_t qbits[MEDUSA_CHUNK_WORDS / 32];// queued-candidate bits (same layout)
+
     uint64_t hull_lo, hull_hi;              // [least base, greatest end) of the current window batch
-    uint32_t front[2][kFront];              // tree-query frontier (by level parity)
+    union {
+        uint32_t front[2][kFront];          // tree-query frontier (by level parity)
+        uint32_t nt[kNodeGrp];              // launch positions of segments g0 .. g0+kNodeGrp-1 (later groups;
+                                            //  used between queries only)
+    };
     uint32_t fn[kMaxLevels + 1];            // frontier size per level
     uint32_t wid[kWinCap];                  // tree-query results: the window entries' allocation ordinals
     uint32_t nres;
@@ -855,14 +865,18 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
     if (tid < kNodeGrp) S.nt0[tid] = 0;
     q_reset(S);
     pdl_wait();  // k_trace: node ranges, status, prefilter bounds, the mortal tree
+    // every value this CTA needs from k_trace, loaded in one round (the node
+    // range is read before the status is known; it is used only if valid)
+    const uint32_t N = a.n_nodes;
     const uint32_t st = __ldcg(&ctl->status);
+    const uint2 jf2 = N ? __ldcg(p.d.jf + c) : make_uint2(0, 0), jl2 = N ? __ldcg(p.d.jl + c) : make_uint2(0, 0);
+    const uint64_t gmin = ~__ldcg(&ctl->gmin_c), gmax = __ldcg(&ctl->gmax);
     // A malformed CSR or launch order (flagged by k_trace) leaves jf / jl and the
     // node offsets meaningless: write the empty counts the later kernels read and
     // do nothing else (the call returns INVALID_ARG; no shared-memory index is
     // ever derived from node_off); the bulk copy is waited for before leaving
     if (st & ST_INVALID) {
         if (tid < kWarps) p.d.qcnt[c * kWarps + tid] = 0;
-        if (tid == 0) p.d.chunk_cnt[c] = 0;
         if (tid == 0 && tma) {
             uint32_t done = 0;
             while (!done) {
@@ -873,12 +887,9 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         pdl_trigger();
         return;
     }
-    const uint32_t N = a.n_nodes;
-    const uint2 jf2 = N ? __ldcg(p.d.jf + c) : make_uint2(0, 0), jl2 = N ? __ldcg(p.d.jl + c) : make_uint2(0, 0);
     const uint32_t jf = N ? min(jf2.x, N - 1) : 0, jl = N ? min(jl2.x, N - 1) : 0;
     const uint32_t t_jf = jf2.y, t_jl = jl2.y;  // the chunk's first and last launch positions
     const uint32_t nn = N ? jl - jf + 1 : 0;
-    const uint64_t gmin = ~__ldcg(&ctl->gmin_c), gmax = __ldcg(&ctl->gmax);
     if (!tma)
         for (uint32_t q = tid; q < n; q += kThreads) S.words[q] = ld_stream(gsrc + q);
     const uint32_t n_alloc = a.n_alloc;
@@ -958,7 +969,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         if (c1) wl[o] = (uint16_t)(q + 1);
         nc += __popc(b0) + __popc(b1);
     }
-    if (lane < 8) wh[lane] = 0;
+    if (lane < 8) { wh[lane] = 0; S.qbits[warp * 8 + lane] = 0; }
     // the rest of the query (the leaves need nt0: complete after this barrier)
     qok = !__syncthreads_or(!qok);
     TL_PHASE(4, 11, tl_p);  // B/C: node starts, TMA wait, candidates, upper query levels
@@ -1022,55 +1033,65 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         o_lo = o_hi;
         wlen = (uint32_t)min((uint64_t)wlen * 2, (uint64_t)n_alloc);
     }
-    // E. the candidates no mortal holds go to this warp's queue region (k_iresolve)
-    IQ* wq = p.d.queue + cs + warp * 256;
-    uint32_t nq = 0;
-    for (uint32_t i0 = 0; i0 < nc; i0 += 32) {
-        const uint32_t i = i0 + lane;
-        bool need = false;
-        uint32_t q = 0;
-        if (i < nc) {
-            q = wl[i];
-            need = !((S.hits[q >> 5] >> (q & 31)) & 1u);
+    // E. the warp's candidates: window hits (records in S.words) and the rest,
+    //    queued for the I-list search, written to the warp's record and queue
+    //    regions in word order; no CTA barrier: every warp finishes on its own
+    {
+        uint32_t* wqb = S.qbits + warp * 8;
+        const uint32_t region = (c * kWarps + warp) * p.d.cap_pw, cap = p.d.cap_pw;
+        const uint32_t lt = lanemask_lt();
+        uint32_t kr = 0, kq = 0;
+        for (uint32_t i0 = 0; i0 < nc; i0 += 32) {
+            const uint32_t i = i0 + lane;
+            bool hit = false, need = false;
+            uint32_t q = 0;
+            if (i < nc) {
+                q = wl[i];
+                hit = (wh[(q & 255) >> 5] >> (q & 31)) & 1u;
+                need = !hit;
+            }
+            const uint32_t bh = __ballot_sync(0xffffffffu, hit), bn = __ballot_sync(0xffffffffu, need);
+            if (hit) {
+                const uint32_t k = kr + __popc(bh & lt);
+                if (k < cap) p.d.rec[region + k] = S.words[q];
+            } else if (need) {
+                const uint32_t k = kq + __popc(bn & lt);
+                const uint32_t t = seg_time(p, S, seg_of(S, q), cs + q, jf, jl);  // the word's launch position
+                if (k < cap) p.d.queue[region + k] = IQ{S.words[q], (uint32_t)(cs + q), t};
+                atomicOr(&wqb[(q & 255) >> 5], 1u << (q & 31));
+            }
+            kr += __popc(bh);
+            kq += __popc(bn);
         }
-        const uint32_t b = __ballot_sync(0xffffffffu, need);
-        if (need) {
-            const uint32_t t = seg_time(p, S, seg_of(S, q), cs + q, jf, jl);  // the word's launch position
-            wq[nq + __popc(b & lanemask_lt())] = IQ{S.words[q], (uint32_t)(cs + q), t};
+        if (max(kr, kq) > cap) {  // the warp's regions are too small: rerun with whole-warp ones
+            if (lane == 0) {
+                atomicMax(&p.d.ctl->need_pw, max(kr, kq));
+                flag(p.d.ctl, ST_OVERFLOW);
+            }
+            kq = min(kq, cap);
         }
-        nq += __popc(b);
+        __syncwarp();
+        const uint64_t n_mask = (a.n_words + 31) / 32;
+        if (lane < 8) {  // the warp's 8 mask words, one lane each
+            const uint32_t qw = warp * 256 + lane * 32;
+            const uint64_t mw = (cs + qw) >> 5;
+            if (qw < n && mw < n_mask) {
+                a.mask[mw] = wh[lane];
+                p.d.imask[mw] = 0;
+                p.d.qmask[mw] = wqb[lane];
+            }
+        }
+        if (lane == 0) {
+            p.d.qcnt[c * kWarps + warp] = kq;
+            // the chunk's slot count (k_iresolve adds the I-list slots; k_emit turns
+            // the counts into chunk_base) and its 256-chunk group sum
+            if (kr) {
+                atomicAdd(p.d.chunk_cnt + c, kr);
+                atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)kr);
+            }
+        }
     }
-    // F. per 32 words: the mask word (lane 0) and the records at their word index
-    const uint64_t n_mask = (a.n_words + 31) / 32;
-    uint32_t cnt = 0;
-    if (lane < 8) {  // the warp's 8 mask words, one lane each
-        const uint32_t q0 = warp * 256 + lane * 32;
-        const uint64_t mw = (cs + q0) >> 5;
-        const uint32_t bits = wh[lane];
-        if (q0 < n && mw < n_mask) a.mask[mw] = bits;
-        cnt = __popc(bits);
-    }
-    cnt = __reduce_add_sync(0xffffffffu, cnt);
-#pragma unroll
-    for (int k = 0; k < kWordsPerThread; ++k) {
-        const uint32_t q = warp * 256 + k * 32 + lane;
-        if ((wh[k] >> lane) & 1u) p.d.staging[cs + q] = S.words[q];
-    }
-    if (lane == 0) {
-        p.d.qcnt[c * kWarps + warp] = nq;
-        S.wcnt[warp] = cnt;
-    }
-    __syncthreads();
-    TL_PHASE(4, 14, tl_p);  // E/F: queue, emission
-    // G. the chunk's slot count so far and its 256-chunk group sum (k_iresolve
-    //    adds the I-list slots; k_emit turns them into chunk_base)
-    if (tid == 0) {
-        uint32_t total = 0;
-#pragma unroll
-        for (int w = 0; w < kWarps; ++w) total += S.wcnt[w];
-        p.d.chunk_cnt[c] = total;
-        if (total) atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)total);
-    }
+    TL_PHASE(4, 15, tl_p);  // E: records, queue, mask words
     pdl_trigger();
 }
 
@@ -1226,9 +1247,10 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 // ----------------------------------------------------------------------------
 // 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
 //     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
-//     CTA; warp w takes the queue region classify's warp w filled.  Per candidate
+//     CTA; warp w takes the queue range classify's warp w filled.  Per candidate
 //     one group of bases and one entry (two dependent loads); a hit writes its
-//     record at its word index and sets its mask bit; the chunk's count grows by
+//     record beside its queue entry and sets its bit in the mask and in the
+//     I-resolved mask; the chunk's count grows by
 //     one atomic per warp (no CTA barrier: the warps run through the chunks
 //     independently).
 __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
@@ -1244,21 +1266,22 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
         __syncthreads();
         for (uint32_t c = blockIdx.x; c < p.C; c += gridDim.x) {
             const uint32_t nq = __ldcg(p.d.qcnt + c * kWarps + warp);
-            const IQ* wq = p.d.queue + (uint64_t)c * kChunkWords + warp * 256;
+            const uint32_t q0 = (c * kWarps + warp) * p.d.cap_pw;
             uint32_t cnt = 0;
             for (uint32_t i0 = 0; i0 < nq; i0 += 32) {
-                const uint32_t i = i0 + lane;
+                const uint32_t k = q0 + i0 + lane;
                 bool hit = false;
-                if (i < nq) {
-                    const IQ q = wq[i];
+                if (i0 + lane < nq) {
+                    const IQ q = p.d.queue[k];
                     const uint32_t le = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
                     if (le) {
                         const uint64_t base = p.d.i_base[le - 1];
                         const IRest e = p.d.i_rest[le - 1];
                         if (q.x < e.end && e.t_alloc < q.t) {
                             hit = true;
-                            p.d.staging[q.g] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
+                            p.d.irec[k] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
                             atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
+                            atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
                         }
                     }
                 }
@@ -1276,12 +1299,18 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
 }
 
 // ----------------------------------------------------------------------------
-// 5. k_emit: compaction of the staged records into the slot table (one CTA per
-//    kEmitChunks chunks, one thread per output record: coalesced stores)
+// 5. k_emit: the slot table (one CTA per kEmitChunks chunks, one thread per
+//    output record: coalesced stores).  Record r of chunk c is the r-th set bit q
+//    of its mask words; it comes from the window-hit region of the classify warp
+//    that owned q if q is not in the I-resolved mask (rank among that warp's
+//    window hits below q), else from beside its queue entry (rank among the
+//    warp's queued words below q).  Regions are read in order: no word-indexed
+//    staging.
 constexpr int kEmitChunks = 2;  // chunks per k_emit CTA (the grid fits one wave)
 
 __global__ void __launch_bounds__(kThreads) k_emit(P p) {
-    __shared__ uint32_t s_pre[kEmitChunks][65], s_m[kEmitChunks][64];
+    __shared__ uint32_t s_m[kEmitChunks][64], s_i[kEmitChunks][64], s_q[kEmitChunks][64];
+    __shared__ uint32_t s_pre[kEmitChunks][65], s_prm[kEmitChunks][65], s_prq[kEmitChunks][65];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const MaterializeArgs& a = p.a;
@@ -1294,25 +1323,38 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     uint32_t total[kEmitChunks];
 #pragma unroll
     for (int h = 0; h < kEmitChunks; ++h) total[h] = (uint32_t)h < nch ? __ldcg(p.d.chunk_cnt + c0 + h) : 0u;
-    if (warp < 2 * kEmitChunks) {  // popcount prefix of each half of each chunk's 64 mask words
+    if (warp < 2 * kEmitChunks) {  // popcount prefixes of each half of each chunk's 64 mask words
         const uint32_t h = warp >> 1, half = warp & 1;
         const uint64_t mw = (uint64_t)(c0 + h) * (kChunkWords / 32) + half * 32 + lane;
-        const uint32_t mv = (h < nch && mw < n_mask) ? __ldcg(a.mask + mw) : 0u;
-        const uint32_t pc = __popc(mv);
-        s_m[h][half * 32 + lane] = mv;
-        uint32_t incl = pc;
+        const bool in = h < nch && mw < n_mask;
+        const uint32_t mv = in ? __ldcg(a.mask + mw) : 0u, iv = in ? __ldcg(p.d.imask + mw) : 0u;
+        const uint32_t qv = in ? __ldcg(p.d.qmask + mw) : 0u;
+        const uint32_t x = half * 32 + lane;
+        s_m[h][x] = mv;
+        s_i[h][x] = iv;
+        s_q[h][x] = qv;
+        uint32_t c3[3] = {(uint32_t)__popc(mv), (uint32_t)__popc(mv & ~iv), (uint32_t)__popc(qv)};
+        uint32_t* pre[3] = {s_pre[h], s_prm[h], s_prq[h]};
 #pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
-            if (lane >= d) incl += y;
+        for (int t = 0; t < 3; ++t) {
+            uint32_t incl = c3[t];
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                if (lane >= d) incl += y;
+            }
+            pre[t][x] = incl - c3[t];
+            if (half == 0 && lane == 31) pre[t][64] = incl;  // first-half total
         }
-        s_pre[h][half * 32 + lane] = incl - pc;
-        if (half == 0 && lane == 31) s_pre[h][64] = incl;  // first-half total
     }
     __syncthreads();
-    if (tid >= 32 && tid < 64) {
+    if (tid >= 32 && tid < 64) {  // second halves after the first
 #pragma unroll
-        for (int h = 0; h < kEmitChunks; ++h) s_pre[h][tid] += s_pre[h][64];  // second half after the first
+        for (int h = 0; h < kEmitChunks; ++h) {
+            s_pre[h][tid] += s_pre[h][64];
+            s_prm[h][tid] += s_prm[h][64];
+            s_prq[h][tid] += s_prq[h][64];
+        }
     }
     __syncthreads();
     if (tid == 0) {
@@ -1330,23 +1372,31 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     // records: every load of the CTA's (up to kRecPerThread per chunk per thread)
     // issued before the first store -- the loads do not wait for each other
     constexpr int kRecPerThread = 2;
+    auto source = [&](int h, uint32_t r) -> uint64_t {  // the record of the chunk's r-th slot
+        uint32_t lo = 0, hi = 64;  // last mask word m with s_pre[m] <= r
+        while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
+        const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);  // the (r - s_pre[lo])-th set bit
+        const uint32_t below = (1u << bit) - 1u;
+        const uint32_t w = lo / 8;  // the classify warp that owned the word
+        const uint64_t region = (uint64_t)((c0 + h) * kWarps + w) * p.d.cap_pw;
+        if ((s_i[h][lo] >> bit) & 1u) {  // resolved by the I list: beside its queue entry
+            const uint32_t k = s_prq[h][lo] - s_prq[h][w * 8] + __popc(s_q[h][lo] & below);
+            return k < p.d.cap_pw ? __ldcg(p.d.irec + region + k) : 0ull;
+        }
+        const uint32_t k = s_prm[h][lo] - s_prm[h][w * 8] + __popc(s_m[h][lo] & ~s_i[h][lo] & below);
+        return k < p.d.cap_pw ? __ldcg(p.d.rec + region + k) : 0ull;
+    };
     uint64_t val[kEmitChunks][kRecPerThread], dst[kEmitChunks][kRecPerThread];
 #pragma unroll
     for (int h = 0; h < kEmitChunks; ++h) {
-        const uint64_t m0 = (uint64_t)(c0 + h) * (kChunkWords / 32);
         const uint64_t pf = prefix + (h ? total[0] : 0u);
 #pragma unroll
         for (int k = 0; k < kRecPerThread; ++k) {
             const uint32_t r = tid + k * kThreads;
             dst[h][k] = ~0ull;
-            if (r < total[h]) {
-                uint32_t lo = 0, hi = 64;  // last group m with s_pre[m] <= r
-                while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
-                const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);  // the (r - s_pre[lo])-th set bit
-                if (pf + r < a.capacity) {
-                    dst[h][k] = pf + r;
-                    val[h][k] = __ldcg(p.d.staging + (m0 + lo) * 32 + bit);
-                }
+            if (r < total[h] && pf + r < a.capacity) {
+                dst[h][k] = pf + r;
+                val[h][k] = source(h, r);
             }
         }
     }
@@ -1358,19 +1408,15 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     // the rest (chunks with more than kRecPerThread * kThreads records)
 #pragma unroll
     for (int h = 0; h < kEmitChunks; ++h) {
-        const uint64_t m0 = (uint64_t)(c0 + h) * (kChunkWords / 32);
         const uint64_t pf = prefix + (h ? total[0] : 0u);
-        for (uint32_t r = tid + kRecPerThread * kThreads; r < total[h]; r += kThreads) {
-            uint32_t lo = 0, hi = 64;
-            while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
-            const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);
-            if (pf + r < a.capacity) a.slot[pf + r] = p.d.staging[(m0 + lo) * 32 + bit];
-        }
+        for (uint32_t r = tid + kRecPerThread * kThreads; r < total[h]; r += kThreads)
+            if (pf + r < a.capacity) a.slot[pf + r] = source(h, r);
     }
     pdl_trigger();
     TL_REC(5, 0, tl0);
 }
 
+// ----------------------------------------------------------------------------
 // 6. k_result (async entry): the outcome as a medusa_mat_result
 __global__ void k_result(P p, medusa_mat_result* r) {
     pdl_wait();
@@ -1379,6 +1425,7 @@ __global__ void k_result(P p, medusa_mat_result* r) {
     int32_t st = MEDUSA_OK;
     if (c.status & ST_INVALID) st = MEDUSA_ERR_INVALID_ARG;
     else if (c.status & ST_TRACE) st = MEDUSA_ERR_TRACE;
+    else if (c.status & ST_OVERFLOW) st = MEDUSA_ERR_RETRY;
     else if (c.n_slots > p.a.capacity) st = MEDUSA_ERR_CAPACITY;
     r->status = st;
     r->reserved = 0;
@@ -1406,7 +1453,7 @@ Tree tree_shape(uint64_t n) {
 }
 
 struct Scratch {
-    size_t cap_n = 0, cap_C = 0, cap_w = 0;
+    size_t cap_n = 0, cap_C = 0, cap_w = 0, cap_r = 0, cap_q = 0;
     void* zero_region = nullptr;
     size_t zero_bytes = 0;
     Dev d{};
@@ -1446,24 +1493,32 @@ void retire(Scratch& s) {
     if (s.zero_region) s.graveyard.push_back(s.zero_region);
     s.zero_region = nullptr;
     s.bytes = 0;
-    s.cap_n = s.cap_C = s.cap_w = 0;
+    s.cap_n = s.cap_C = s.cap_w = s.cap_r = s.cap_q = 0;
 }
 
 // grow geometrically (x1.5) past the previous capacity, so a sequence of growing
 // calls retires a bounded amount of memory
 size_t grown(size_t need, size_t old) { return need <= old ? old : std::max(need, old + old / 2); }
 
-cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W) {
-    if (n <= s.cap_n && C <= s.cap_C && W <= s.cap_w) return cudaSuccess;
+// Warp regions of 128 entries (half the warp's 256 words; the BASELINE sets:
+// ~10% window hits and ~9% queued candidates, at most ~30% in any 256 words); a
+// call whose warp needs more sets ST_OVERFLOW, and the synchronous entry reruns
+// with regions of the whole warp (256, always enough).
+constexpr size_t kRegion = 128;
+cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
+    const size_t PC = need_pw > kRegion ? (size_t)(kChunkWords / kWarps) : kRegion;
+    if (n <= s.cap_n && C <= s.cap_C && W <= s.cap_w && PC <= s.cap_r) return cudaSuccess;
     const size_t N = grown(std::max<size_t>(n, 1024), s.cap_n), CC = grown(std::max<size_t>(C, 64), s.cap_C);
     const size_t WW = grown(std::max<size_t>(W, 2048), s.cap_w);
+    const size_t RR = std::max(PC, s.cap_r), QQ = CC * kWarps * RR;
     retire(s);
     const size_t NS = N / kIBlk + 1;
     const size_t NT = tree_shape(N).off[kMaxLevels] + 64;  // tree nodes (levels >= 1) for up to N ordinals
     cudaError_t e;
-    // zero region: Ctl | chunk_sup [CC/256+1] (u64) | blk_min_ta_c blk_max_tf [NS] | tree nodes [NT] (uint2)
+    // zero region: Ctl | chunk_sup [CC/256+1] (u64) | blk_min_ta_c blk_max_tf [NS] | chunk_cnt [CC] |
+    //              tree nodes [NT] (uint2)
     const size_t GC = CC / 256 + 1;
-    s.zero_bytes = 256 + GC * 8 + 2 * NS * 4 + 64 + NT * 8;
+    s.zero_bytes = 256 + GC * 8 + 2 * NS * 4 + CC * 4 + 64 + NT * 8;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
     s.bytes += s.zero_bytes;
     char* z = (char*)s.zero_region;
@@ -1472,17 +1527,20 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W) {
     s.d.chunk_sup = (unsigned long long*)(z + o); o += GC * 8;
     s.d.blk_min_ta_c = (uint32_t*)(z + o); o += NS * 4;
     s.d.blk_max_tf = (uint32_t*)(z + o); o += NS * 4;
+    s.d.chunk_cnt = (uint32_t*)(z + o); o += CC * 4;
     o = (o + 63) & ~(size_t)63;
     s.d.tree.node = (uint2*)(z + o);
     if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) ||
         (e = grow(s, s.d.sk0, N)) || (e = grow(s, s.d.sv0, N)) || (e = grow(s, s.d.sk, N)) || (e = grow(s, s.d.sv, N)) ||
         (e = grow(s, s.d.samp_k, N / kSampleStride + 64)) || (e = grow(s, s.d.samp_v, N / kSampleStride + 64)) ||
         (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
-        (e = grow(s, s.d.fence, (size_t)kFenceCap)) || (e = grow(s, s.d.chunk_cnt, CC)) ||
-        (e = grow(s, s.d.staging, WW)) || (e = grow(s, s.d.queue, CC * kChunkWords)) ||
-        (e = grow(s, s.d.qcnt, CC * kWarps)))
+        (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
+        (e = grow(s, s.d.rec, QQ)) || (e = grow(s, s.d.queue, QQ)) || (e = grow(s, s.d.irec, QQ)) ||
+        (e = grow(s, s.d.qcnt, CC * kWarps)) ||
+        (e = grow(s, s.d.imask, WW / 32 + 1)) || (e = grow(s, s.d.qmask, WW / 32 + 1)))
         return e;
-    s.cap_n = N; s.cap_C = CC; s.cap_w = WW;
+    s.d.cap_pw = (uint32_t)RR;
+    s.cap_n = N; s.cap_C = CC; s.cap_w = WW; s.cap_r = RR; s.cap_q = QQ;
     return cudaSuccess;
 }
 
@@ -1621,19 +1679,28 @@ medusa_status run_materialize(const MaterializeArgs& a, uint64_t* n_slots, cudaS
     if (!sp) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     Scratch& s = *sp;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
-    P p;
-    if ((e = ensure(s, a.n_alloc, C, a.n_words)) != cudaSuccess ||
-        (e = enqueue(s, a, stream, &p)) != cudaSuccess ||
-        (e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess ||
-        (e = cudaStreamSynchronize(stream)) != cudaSuccess) {
-        *cuda_err = e;
-        return MEDUSA_ERR_CUDA;
+    size_t need_pw = 0;
+    for (int attempt = 0; attempt < 2; ++attempt) {
+        P p;
+        if ((e = ensure(s, a.n_alloc, C, a.n_words, need_pw)) != cudaSuccess ||
+            (e = enqueue(s, a, stream, &p)) != cudaSuccess ||
+            (e = cudaMemcpyAsync(s.h_ctl, s.d.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, stream)) != cudaSuccess ||
+            (e = cudaStreamSynchronize(stream)) != cudaSuccess) {
+            *cuda_err = e;
+            return MEDUSA_ERR_CUDA;
+        }
+        const Ctl h = *s.h_ctl;
+        if (h.status & ST_INVALID) return MEDUSA_ERR_INVALID_ARG;
+        if (h.status & ST_TRACE) return MEDUSA_ERR_TRACE;
+        if (h.status & ST_OVERFLOW) {  // a warp's record / queue region too small: whole-warp regions, rerun
+            need_pw = std::max<size_t>(need_pw, h.need_pw);
+            continue;
+        }
+        *n_slots = h.n_slots;
+        return h.n_slots > a.capacity ? MEDUSA_ERR_CAPACITY : MEDUSA_OK;
     }
-    const Ctl h = *s.h_ctl;
-    if (h.status & ST_INVALID) return MEDUSA_ERR_INVALID_ARG;
-    if (h.status & ST_TRACE) return MEDUSA_ERR_TRACE;
-    *n_slots = h.n_slots;
-    return h.n_slots > a.capacity ? MEDUSA_ERR_CAPACITY : MEDUSA_OK;
+    *cuda_err = cudaErrorUnknown;  // (the exact sizes cannot overflow)
+    return MEDUSA_ERR_CUDA;
 }
 
 medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result* d_result, cudaStream_t stream,
@@ -1645,7 +1712,7 @@ medusa_status run_materialize_async(const MaterializeArgs& a, medusa_mat_result*
     Scratch& s = *sp;
     const uint32_t C = (uint32_t)((a.n_words + kChunkWords - 1) / kChunkWords);
     // never (re)allocates while the caller may be capturing a graph, unless it must grow
-    if ((e = ensure(s, a.n_alloc, C, a.n_words)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
+    if ((e = ensure(s, a.n_alloc, C, a.n_words, 0)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     P p;
     if ((e = enqueue(s, a, stream, &p)) != cudaSuccess) { *cuda_err = e; return MEDUSA_ERR_CUDA; }
     if ((e = launch_pdl(k_result, 1, 1, 0, stream, p, d_result))) { *cuda_err = e; return MEDUSA_ERR_CUDA; }

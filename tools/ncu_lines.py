@@ -1,46 +1,46 @@
-"""Aggregate ncu SASS metrics per CUDA source line (mixed cuda,sass page).
-usage: python tools/ncu_lines.py report.ncu-rep kernel_regex [top]"""
+"""Per-source-line totals of an ncu source page exported with
+--print-source cuda,sass --csv: warp-instructions executed and stall samples,
+summed over the SASS of each CUDA line (diagnostic)."""
 import csv
-import io
-import subprocess
 import sys
-from collections import defaultdict
 
-rep, kre = sys.argv[1], sys.argv[2]
-top = int(sys.argv[3]) if len(sys.argv) > 3 else 30
-by = sys.argv[4] if len(sys.argv) > 4 else "inst"  # or "smp"
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--print-source", "cuda,sass", "--csv", "-k", f"regex:{kre}"],
-                     capture_output=True, text=True).stdout
-agg = defaultdict(lambda: [0.0, 0.0])
-text = {}
-cur_file = "?"
+path, top = sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 30
+rows = list(csv.reader(open(path)))
+out = {}
+src = {}
+cur_file = None
 hdr = None
-for row in csv.reader(io.StringIO(out)):
-    if not row:
+last_line = ""
+for r in rows:
+    if len(r) == 2 and r[0] == "File Path":
+        cur_file = r[1].split("/")[-1]
         continue
-    if row[0] == "File Path":
-        cur_file = row[1].split("/")[-1]
+    if r and r[0] == "Line No":
+        hdr = {k: i for i, k in enumerate(r)}
         continue
-    if row[0] == "Line No":
-        hdr = {k: i for i, k in enumerate(row)}
+    if hdr is None or len(r) < len(hdr):
         continue
-    if hdr is None or len(row) < len(hdr):
+    line = r[0] or last_line
+    last_line = line
+    if not line:
         continue
     try:
-        ln = int(row[0])
+        ie = float(r[hdr["Instructions Executed"]] or 0)
+        ss = float(r[hdr["Warp Stall Sampling (All Samples)"]] or 0)
     except ValueError:
         continue
-    key = (cur_file, ln)
-    text[key] = row[1]
-    ie = row[hdr["Instructions Executed"]] if "Instructions Executed" in hdr else ""
-    ss = row[hdr["Warp Stall Sampling (All Samples)"]] if "Warp Stall Sampling (All Samples)" in hdr else ""
-    try:
-        agg[key][0] += float(ie or 0)
-        agg[key][1] += float(ss or 0)
-    except ValueError:
-        pass
-ti = sum(v[0] for v in agg.values()) or 1
-ts = sum(v[1] for v in agg.values()) or 1
-print(f"instructions {ti:.3g}  samples {ts:.0f}")
-for key, (i, s) in sorted(agg.items(), key=lambda kv: -kv[1][0 if by == 'inst' else 1])[:top]:
-    print(f"{100*i/ti:5.1f}% inst {100*s/ts:5.1f}% smp  {key[0]}:{key[1]:<5d} {text.get(key, '').strip()[:90]}")
+    key = (cur_file, int(line), (r[1] or src.get((cur_file, line), ""))[:90])
+    if r[1]:
+        src[(cur_file, line)] = r[1]
+    a = out.setdefault(key, [0.0, 0.0])
+    a[0] += ie
+    a[1] += ss
+ti = sum(v[0] for v in out.values()) or 1
+ts = sum(v[1] for v in out.values()) or 1
+print(f"total warp instructions {ti:.0f}, stall samples {ts:.0f}")
+print("by instructions:")
+for k, v in sorted(out.items(), key=lambda kv: -kv[1][0])[:top]:
+    print(f"{100*v[0]/ti:5.1f}% inst {100*v[1]/ts:5.1f}% stall  {k[0]}:{k[1]}  {k[2]}")
+print("by stall samples:")
+for k, v in sorted(out.items(), key=lambda kv: -kv[1][1])[:top]:
+    print(f"{100*v[0]/ti:5.1f}% inst {100*v[1]/ts:5.1f}% stall  {k[0]}:{k[1]}  {k[2]}")

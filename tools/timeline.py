@@ -29,7 +29,7 @@ NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan
          (3, 40): " rank:pdl-wait", (3, 41): " rank:staging", (3, 42): " rank:search+red", (3, 43): " rank:ticket",
          (3, 44): " rank:i-entries", (2, 30): " isort:bitonic", (2, 31): " isort:merges",
          (4, 10): " cls:A setup", (4, 11): " cls:B starts+cand", (4, 12): " cls:D query", (4, 13): " cls:D live+search",
-         (4, 14): " cls:E queue", (4, 15): " cls:pdl-wait", (4, 16): " cls:win-load", (4, 17): " cls:sort",
+         (4, 14): " cls:E queue", (4, 15): " cls:E records+queue", (4, 16): " cls:win-load", (4, 17): " cls:sort",
          (7, 2): "restore/in-place", (7, 10): " res:mask+range", (7, 11): " res:records+gathers",
          (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store"}
 REC = np.dtype([("t0", "<u8"), ("t1", "<u8"), ("kernel", "<u4"), ("cta", "<u4"), ("sm", "<u4"), ("tag", "<u4")])
@@ -39,6 +39,8 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--workload", default="all10")
     ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--serial", action="store_true",
+                    help="every kernel alone (libmedusa's per-launch timing mode: branches serialized)")
     args = ap.parse_args()
     extra = tuple(d for d in os.environ.get("MEDUSA_DEFINES", "").split() if d)  # A/B variants
     tl_path = g.build_medusa(out=os.path.join(ROOT, "tools", "libmedusa_tl" + "".join("_" + d for d in extra) + ".so"),
@@ -71,12 +73,17 @@ def main():
     buf = [torch.zeros(cap * REC.itemsize, dtype=torch.uint8, device=dev) for _ in range(2)]
     step()  # eager once: the kernel table and scratch are allocated outside capture
     torch.cuda.synchronize()
-    graph = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(graph):
-        step()
+    if args.serial:  # eager steps (per-launch events cannot be captured)
+        medusa.timing_enable(True)
+        run = step
+    else:
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            step()
+        run = graph.replay
     scrub = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     for _ in range(3):
-        graph.replay()
+        run()
     agg = {}
     spans = []
     ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -85,7 +92,7 @@ def main():
         L.medusa_tl_attach_res(ctypes.c_void_p(buf[1].data_ptr()), cap)
         scrub.fill_(k)
         ev[0].record()
-        graph.replay()
+        run()
         ev[1].record()
         torch.cuda.synchronize()
         n0, n1 = L.medusa_tl_count_mat(), L.medusa_tl_count_res()
@@ -98,6 +105,9 @@ def main():
             d = (r["t1"] - r["t0"]) / 1e3
             agg.setdefault(key, []).append(((r["t0"].min() - t_begin) / 1e3, (r["t1"].max() - t_begin) / 1e3, len(r),
                                             np.percentile(d, 50), np.percentile(d, 90), d.max()))
+    if args.serial:
+        medusa.timing_read(1 << 16)
+        medusa.timing_enable(False)
     assert medusa.mat_result(res)[0] == 0
     print(f"{args.workload}: step span (first CTA start -> last CTA end) {np.mean([s[0] for s in spans]):.1f} us; "
           f"event time {np.mean([s[1] for s in spans]):.1f} us (incl. launch of the first kernel)")
