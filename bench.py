@@ -60,8 +60,31 @@ PAPER_CONTEXT = {
 SEED_STRIDE = 1000  # rank r restores the instance generated with seed + r * SEED_STRIDE
 
 
-def algorithmic_bytes(gs, n_slots, n_func):
-    """Bytes the method itself must move."""
+def path_counts(gs, slot_id=None):
+    """Host-side counts the per-kernel algorithmic bytes need (from the inputs and,
+    for the window / I-list split, the oracle's slot ids when given)."""
+    a = gs.allocs
+    nt = gs.node_t
+    t_last = int(nt[-1]) if nt.size else 0
+    live = a["size"] > 0
+    isI = live & (a["t_alloc"] < t_last) & (t_last < a["t_free"]) if nt.size else np.zeros(a.size, bool)
+    gmin = int(a["base"][live].min()) if live.any() else 0
+    gmax = int((a["base"][live] + a["size"][live]).max()) if live.any() else 0
+    w = gs.words
+    cand = int(((w >= np.uint64(gmin)) & (w < np.uint64(gmax))).sum()) if gmax else 0
+    n_i = int(isI.sum())
+    out = {"n_I": n_i, "candidates": cand}
+    if slot_id is not None:
+        i_hits = int(isI[slot_id.astype(np.int64)].sum())
+        out.update(i_hits=i_hits, window_hits=int(slot_id.size) - i_hits, queued=cand - (int(slot_id.size) - i_hits))
+    return out
+
+
+def algorithmic_bytes(gs, n_slots, n_func, counts=None):
+    """Bytes the method itself must move per launch of each kernel (SURVEY.md
+    §8(d) for mat_classify = K1+K2 and restore = K3+K4; DESIGN.md §5 for the
+    others: what the kernel must read and write, intermediate structures included,
+    at their per-unit sizes)."""
     W, N, A = gs.n_words, gs.n_nodes, gs.n_alloc
     n_mask = (W + 31) // 32
     C = (W + 2047) // 2048
@@ -69,7 +92,23 @@ def algorithmic_bytes(gs, n_slots, n_func):
     classify = (8 * W + 4 * n_mask + 4 * (C + 1) + 8 * n_slots + 12 * N)
     # in place (dst == src): only the slot words are read and written
     inplace = (4 * n_mask + 4 * (C + 1) + 8 * n_slots + 16 * n_slots + 24 * A + 12 * N + 8 * n_func + 64)
-    return dict(restore=restore, mat_classify=classify, restore_inplace=inplace)
+    out = dict(restore=restore, mat_classify=classify, restore_inplace=inplace)
+    if counts is not None and "queued" in counts:
+        nI, q = counts["n_I"], counts["queued"]
+        T = max(1, (nI + 1023) // 1024)
+        out.update(
+            # records + node CSR in; tree leaves (8 B/alloc), tree nodes, I keys (12 B), chunk node ranges (16 B)
+            mat_trace=24 * A + 12 * N + 8 * A + 8 * ((A + 31) // 32) + 12 * nI + 16 * C,
+            mat_isort=24 * nI,                                     # I keys in, sorted tiles out
+            # each key + per other tile one 32-key sample block and one 32-key block (12 B/key), I entry out
+            mat_rank=(12 * nI + 24 * (T - 1) * nI + 52 * nI) if T > 1 else 0,
+            mat_iresolve=16 * q + 8 * counts["i_hits"] + 8 * n_mask,   # queue in, records + masks out
+            mat_emit=3 * 4 * n_mask + 16 * n_slots + 4 * (C + 1),    # 3 masks, records in + table out
+            mat_check_mm=24 * A + 8 * A,                          # own records, tree leaves
+            mat_check_mi=24 * A + 28 * nI,                        # own records, the sorted I list
+            restore_report_init=64,
+        )
+    return out
 
 
 def measured_peak():
@@ -516,7 +555,7 @@ def oracle_parity(gs, slots, n_slots, dst, fout, rep):
         "report": np.array_equal(medusa.report_numpy(rep), orep),
     }
     return {"ok": all(checks.values()), "failed": [k for k, v in checks.items() if not v],
-            "slots": int(m["n_slots"]), "words": gs.n_words}
+            "slots": int(m["n_slots"]), "words": gs.n_words}, m["slot_id"]
 
 
 def bench_c5(medusa, args, rank, dev, stream, scrub, barrier, peak):
@@ -574,7 +613,7 @@ def bench_c5(medusa, args, rank, dev, stream, scrub, barrier, peak):
     rest_ms = timed(graphs["restore"])
     st, ns = medusa.mat_result(res)
     assert st == 0 and ns == n_slots, (st, ns)
-    par = oracle_parity(gs, sl, n_slots, dst, fout, rep)
+    par = oracle_parity(gs, sl, n_slots, dst, fout, rep)[0]
     alg = algorithmic_bytes(gs, n_slots, gs.table.size)["restore"]
     t_rest = statistics.median(rest_ms) / 1e3
     out = {"rank": rank, "seed": seed, "nodes": gs.n_nodes, "words": gs.n_words, "slots": n_slots,
@@ -707,18 +746,20 @@ def run_ours(args):
     st_, ns_ = medusa.mat_result(res)
     assert st_ == 0 and ns_ == n_slots, (st_, ns_)
     assert int(medusa.report_numpy(grep)[0]) == 0 and torch.equal(gdst, dst) and torch.equal(gfout, fout)
-    head_parity = oracle_parity(gs, slots, n_slots, gdst, gfout, grep)  # this rank's instance vs the CPU oracle
+    head_parity, head_slot_id = oracle_parity(gs, slots, n_slots, gdst, gfout, grep)  # this rank's instance vs the CPU oracle
     assert head_parity["ok"], head_parity
     scratch = medusa.scratch_bytes()
     sync_ms = timed(step)  # the same path through the synchronous API (host round trip after materialize)
     # the same K steps again with every libmedusa launch bracketed by events on its
     # stream: per-kernel durations for the roofline and the breakdown
     def step_queued():
-        # as step(), with a ~30 us device spin between the analysis (whose slot-count
-        # read-back leaves the GPU idle) and the restore: the host has enqueued the
-        # restore's launches before the GPU reaches them, so its launch events see
-        # device time, not the host's launch latency
+        # as step(), with a device spin (~0.2 ms) queued before the analysis and one
+        # (~30 us) between the analysis (whose slot-count read-back leaves the GPU
+        # idle) and the restore: the host has enqueued each call's launches and
+        # events before the GPU reaches them, so the launch events see device time,
+        # not the host's launch latency
         medusa.kernel_table_set(inp["table"])
+        torch.cuda._sleep(400000)
         medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots)
         torch.cuda._sleep(60000)
         medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
@@ -739,7 +780,8 @@ def run_ours(args):
         d = per.setdefault(name, [0, 0.0])
         d[0] += 1
         d[1] += ms
-    alg = algorithmic_bytes(gs, n_slots, gs.table.size)
+    counts = path_counts(gs, head_slot_id)
+    alg = algorithmic_bytes(gs, n_slots, gs.table.size, counts)
     peak, peak_src = measured_peak()
     traffic = load_traffic(cfg)
     kernels = {}
@@ -749,6 +791,8 @@ def run_ours(args):
         if name in alg:
             entry["alg_bytes"] = alg[name]
             entry["GB/s"] = alg[name] / (avg / 1e3) / 1e9
+        if traffic.get(name):
+            entry["dram_bytes_ncu"] = traffic[name]
         kernels[name] = entry
     dom = max((n for n in per if n in alg), key=lambda n: per[n][1])
     dom_avg_s = per[dom][1] / per[dom][0] / 1e3
@@ -764,9 +808,16 @@ def run_ours(args):
         rl["issue"] = {"warp_inst_per_launch": inst, "achieved": inst / dom_avg_s / 1e12, "peak": issue_peak,
                        "unit": "T warp-inst/s", "frac": inst / dom_avg_s / 1e12 / issue_peak}
     if dom == "mat_classify":
-        rl["note"] = ("k_classify reads each word once (TMA) but its time goes to dependent shared-memory work "
-                      "behind CTA barriers (window setup, per-candidate node and window lookups): latency- and "
-                      "issue-bound, not HBM-bound; stall breakdown in profiles/r1_classify_stalls.txt, DESIGN.md §6")
+        rl["note"] = ("k_classify reads each word once (TMA) but its time goes to dependent work behind CTA "
+                      "barriers (node starts, mortal-tree query, window loads, live masks) and the per-candidate "
+                      "lookups: latency- and issue-bound, not HBM-bound; stall breakdown in "
+                      "profiles/r2_classify_stalls.txt, DESIGN.md §6")
+    # the whole step against the roofline: SURVEY.md §8(d)'s algorithmic bytes of the
+    # path (K1+K2 + K3+K4) over the device-timed step
+    step_alg = alg["mat_classify"] + alg["restore"]
+    step_s = max_ms / args.steps / 1e3
+    rl["whole_step"] = {"alg_bytes": step_alg, "ms_per_step": step_s * 1e3, "achieved": step_alg / step_s / 1e9,
+                        "frac": step_alg / step_s / 1e9 / peak, "unit": "GB/s"}
     rst = per["restore"]
     restore_avg_s = rst[1] / rst[0] / 1e3
     relocate = {"kernel": "restore", "GB/s": alg["restore"] / restore_avg_s / 1e9,
@@ -999,6 +1050,7 @@ def run_ours(args):
             "dtype": "u64", "data": "synthetic",
             "config": config_dict(cfg, desc, gs, n_slots, rank_seed(cfg, 0), ws),
             "multi_gpu": multi,
+            "path_counts": counts,
             "scratch": {"bytes": scratch, "bytes_per_word": scratch / gs.n_words,
                         "note": "library-owned materialize scratch of this device after the headline workload "
                                 "(medusa_scratch_bytes)"},
@@ -1026,8 +1078,10 @@ def run_ours(args):
                           f"{len(launches) // max(args.steps, 1)} per step: no k_result)",
             "sync_api_ms_per_step": max_over_ranks(sum(sync_ms), dist, dev) / args.steps,
             "instrumented_ms_per_step": sum(inst_ms) / args.steps,
-            "instrumented_note": "per-kernel events, branches serialized, a ~30 us device spin queued before the "
-                                 "restore (share_of_step = share of the summed kernel times, as in the ncu launch list)",
+            "instrumented_note": "per-kernel events, branches serialized, device spins queued before the analysis "
+                                 "(~0.2 ms) and before the restore (~30 us) so no event waits for the host; "
+                                 "instrumented_ms_per_step includes the spins (share_of_step = share of the summed "
+                                 "kernel times, as in the ncu launch list)",
             "clocks": clocks,
         }
         print(json.dumps(line), flush=True)

@@ -121,8 +121,8 @@ struct Dev {  // scratch of one call (device pointers)
     // 256 words) owns entries [(8c + w) cap_pw, (8c + w + 1) cap_pw) of each,
     // filled in word order
     uint64_t* rec;                               // records of the window hits
-    IQ* queue;                                   // candidates left for the I-list search
-    uint64_t* irec;                              // the I-list record of queue entry k (hits only)
+    IQ* queue;                                   // candidates left for the I-list search; k_iresolve
+                                                 //  overwrites a hit's word (x) with its record
     uint32_t cap_pw;                             // entries per warp region (128; 256 after an overflow)
     uint32_t* qcnt;                              // [C * 8] queue entries of classify warp w of chunk c
     uint32_t *imask, *qmask;                     // [ceil(n_words/32)] words resolved by the I list / queued
@@ -1249,7 +1249,7 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 //     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
 //     CTA; warp w takes the queue range classify's warp w filled.  Per candidate
 //     one group of bases and one entry (two dependent loads); a hit writes its
-//     record beside its queue entry and sets its bit in the mask and in the
+//     record over its queue entry's word and sets its bit in the mask and in the
 //     I-resolved mask; the chunk's count grows by
 //     one atomic per warp (no CTA barrier: the warps run through the chunks
 //     independently).
@@ -1279,7 +1279,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                         const IRest e = p.d.i_rest[le - 1];
                         if (q.x < e.end && e.t_alloc < q.t) {
                             hit = true;
-                            p.d.irec[k] = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
+                            p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
                             atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
                             atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
                         }
@@ -1303,7 +1303,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
 //    output record: coalesced stores).  Record r of chunk c is the r-th set bit q
 //    of its mask words; it comes from the window-hit region of the classify warp
 //    that owned q if q is not in the I-resolved mask (rank among that warp's
-//    window hits below q), else from beside its queue entry (rank among the
+//    window hits below q), else from its queue entry, where k_iresolve left it (rank among the
 //    warp's queued words below q).  Regions are read in order: no word-indexed
 //    staging.
 constexpr int kEmitChunks = 2;  // chunks per k_emit CTA (the grid fits one wave)
@@ -1381,7 +1381,7 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
         const uint64_t region = (uint64_t)((c0 + h) * kWarps + w) * p.d.cap_pw;
         if ((s_i[h][lo] >> bit) & 1u) {  // resolved by the I list: beside its queue entry
             const uint32_t k = s_prq[h][lo] - s_prq[h][w * 8] + __popc(s_q[h][lo] & below);
-            return k < p.d.cap_pw ? __ldcg(p.d.irec + region + k) : 0ull;
+            return k < p.d.cap_pw ? __ldcg(&p.d.queue[region + k].x) : 0ull;
         }
         const uint32_t k = s_prm[h][lo] - s_prm[h][w * 8] + __popc(s_m[h][lo] & ~s_i[h][lo] & below);
         return k < p.d.cap_pw ? __ldcg(p.d.rec + region + k) : 0ull;
@@ -1535,7 +1535,7 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
         (e = grow(s, s.d.samp_k, N / kSampleStride + 64)) || (e = grow(s, s.d.samp_v, N / kSampleStride + 64)) ||
         (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
         (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
-        (e = grow(s, s.d.rec, QQ)) || (e = grow(s, s.d.queue, QQ)) || (e = grow(s, s.d.irec, QQ)) ||
+        (e = grow(s, s.d.rec, QQ)) || (e = grow(s, s.d.queue, QQ)) ||
         (e = grow(s, s.d.qcnt, CC * kWarps)) ||
         (e = grow(s, s.d.imask, WW / 32 + 1)) || (e = grow(s, s.d.qmask, WW / 32 + 1)))
         return e;
