@@ -372,9 +372,12 @@ __device__ __forceinline__ void warp_bitonic_kv(uint64_t (&k)[E], uint32_t (&v)[
 //     to sk / sv and every kSampleStride-th key is its sample for k_rank.
 constexpr int kIsortThreads = 256;  // (1024-thread CTAs measured slower: they find no slot beside
                                      //  the classify CTAs, and one CTA sorting 3-4k keys is a long chain)
-constexpr int kSortPer = 4;                                  // keys per thread in registers
+#ifndef MEDUSA_ISORT_PER
+#define MEDUSA_ISORT_PER 4
+#endif
+constexpr int kSortPer = MEDUSA_ISORT_PER;                   // keys per thread in registers
 constexpr int kIsortTile = kIsortThreads * kSortPer;         // 1024
-constexpr int kSampleStride = 32;                            // <= 32 samples per tile
+constexpr int kSampleStride = kIsortTile / 64 > 32 ? kIsortTile / 64 : 32;  // <= 64 samples per tile
 struct ISortShared {
     uint64_t k[kIsortTile];
     uint32_t v[kIsortTile];
