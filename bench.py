@@ -45,6 +45,8 @@ WORKLOADS = {
     "llama2-7b": ("llama2-7b", "Llama-2-7B-shaped graph set with kernel table (12,518 nodes)"),
     "llama2-13b": ("llama2-13b", "Llama-2-13B-shaped instance (16,150 nodes)"),
     "toy": ("toy", "toy 2-layer decoder, 200 nodes"),
+    "all10-inband": ("all10-inband", "stress: the ten-model set with ~8% of words in-band non-pointer constants "
+                                     "(VA holes, freed memory)"),
 }
 # the paper's own end-to-end numbers, quoted beside ours: another
 # machine's, not the target (the paper never times these passes on their own)

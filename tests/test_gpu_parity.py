@@ -45,7 +45,7 @@ def _check_materialize(slots, m, packed, n_words):
     assert np.array_equal(_h(slots.slot)[: slots.n_slots].view(np.uint64), rec)
 
 
-@pytest.mark.parametrize("name", ["toy", "qwen1.5-4b", "llama2-7b", "llama2-13b", "all10"])
+@pytest.mark.parametrize("name", ["toy", "qwen1.5-4b", "llama2-7b", "llama2-13b", "all10", "all10-inband"])
 def test_full_path_parity(graph_sets, name):
     gs = graph_sets(name)
     inp = medusa.upload(gs, DEV)

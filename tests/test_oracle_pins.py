@@ -157,7 +157,7 @@ def test_p4_p5_p6_p7_closed_forms(graph_sets, name):
 
 
 # ---------------------------------------------------------------- P8
-@pytest.mark.parametrize("name", ["toy", "qwen1.5-4b"])
+@pytest.mark.parametrize("name", ["toy", "qwen1.5-4b", "all10-inband"])
 def test_p8_generator_ground_truth(graph_sets, name):
     gs = graph_sets(name)
     m = oracle.materialize(gs.words, gs.node_word_off, gs.node_t, gs.allocs)

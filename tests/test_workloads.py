@@ -45,3 +45,18 @@ def test_replicate_is_r_shifted_copies(graph_sets):
         assert np.array_equal(m3["off"][sl], m1["off"])
     consts = gs.tags == TAG_CONST
     assert np.array_equal(big.words[gs.n_words:2 * gs.n_words][consts], gs.words[consts])
+
+
+def test_inband_stress_config(graph_sets):
+    """all10-inband: the ten-model set (Table 1 totals kept) with 5-10% of all words
+    in-band non-pointer constants -- inside [least base, greatest end) of the
+    trace, so the classify prefilter passes them -- and still well-formed."""
+    gs = graph_sets("all10-inband")
+    assert gs.n_nodes == 139364
+    assert oracle.check(gs.n_words, gs.node_word_off, gs.node_t, gs.allocs) == oracle.OK
+    a = gs.allocs
+    live = a["size"] > 0
+    lo, hi = a["base"][live].min(), (a["base"][live] + a["size"][live]).max()
+    inband = (gs.words >= lo) & (gs.words < hi)
+    frac = float((inband & (gs.tags != 1)).mean())
+    assert 0.05 <= frac <= 0.10, frac

@@ -168,8 +168,9 @@ AK_WEIGHT, AK_KV, AK_STATIC, AK_PROFILE, AK_WARMUP, AK_CAPTURE, AK_PERM = range(
 
 
 class _Builder:
-    def __init__(self, seed: int):
+    def __init__(self, seed: int, rates=_RATES):
         self.rng = np.random.default_rng(seed)
+        self.rates = rates
         self.t = 0
         self.a_base, self.a_size, self.a_ta, self.a_tf = [], [], [], []
         self.a_seg, self.a_kind = [], []
@@ -319,7 +320,7 @@ class _Builder:
         if bad.any():
             vals[cidx[bad]] ^= np.uint64(1 << 47)
         u = rng.random(cidx.size) / self.rate_scale
-        RATE_GAP, RATE_OPE, RATE_DANGLING, RATE_FP = _RATES
+        RATE_GAP, RATE_OPE, RATE_DANGLING, RATE_FP = self.rates
         for p, uu in zip(cidx, u):
             if uu >= RATE_GAP + RATE_OPE + RATE_DANGLING + RATE_FP:
                 continue
@@ -606,25 +607,32 @@ CONFIGS = {
     "llama2-7b": dict(models=["llama2-7b"], seed=3),
     "all10": dict(models=ALL10, seed=4),
     "llama2-13b": dict(models=["llama2-13b"], seed=100),  # C5: seed 100 + gpu index
+    # stress: ALL10 with ~8% of all words in-band non-pointer constants (addresses in
+    # VA holes and in freed memory, inside [least base, greatest end) of the trace),
+    # so the classify prefilter cannot reject them for free
+    "all10-inband": dict(models=ALL10, seed=5, rates=(0.08, 0.005, 0.015, 0.0005)),
 }
 
 
 def make_graph_set(config: str, seed: int | None = None, models: list | None = None) -> GraphSet:
     """Build one of the BASELINE.json configurations.
 
-    config: 'toy' | 'qwen1.5-4b' | 'llama2-7b' | 'all10' | 'llama2-13b' | any single model name.
+    config: 'toy' | 'qwen1.5-4b' | 'llama2-7b' | 'all10' | 'llama2-13b' | 'all10-inband' (stress) |
+    any single model name.
     seed defaults to the config's fixed seed.
     """
+    rates = _RATES
     if config in CONFIGS:
         spec = CONFIGS[config]
         mlist = spec["models"] if models is None else models
         seed = spec["seed"] if seed is None else seed
+        rates = spec.get("rates", _RATES)
     elif config in MODELS:
         mlist = [config] if models is None else models
         seed = 0 if seed is None else seed
     else:
         raise KeyError(config)
-    B = _Builder(seed)
+    B = _Builder(seed, rates)
     if mlist is None:
         _run_toy(B)
     else:
