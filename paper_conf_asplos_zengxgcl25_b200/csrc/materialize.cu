@@ -57,7 +57,7 @@ constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
-constexpr int kFenceCap = 2048;    // I-list fences held in shared memory
+constexpr int kFenceCap = 8192;    // I-list fences (every stride-th sorted base; searched through L1)
 constexpr int kWinCap = 96;        // mortal-window entries per batch (<= 4 per lane of one warp; 96 keeps 7 classify CTAs per SM)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
 constexpr int kWarps = kThreads / 32;
@@ -110,6 +110,9 @@ struct Dev {  // scratch of one call (device pointers)
     uint32_t *blk_min_ta_c, *blk_max_tf;         // [n/32+1] (zeroed; min kept as ~max(~t))
     uint64_t *sk0, *sk;                          // [n] I keys (base): compacted by k_trace / sorted tiles
     uint32_t *sv0, *sv;                          // [n] their allocation ordinals
+    uint32_t* icnt;                              // [n/256+1] I keys of each k_trace alloc CTA (ordered mode)
+    uint64_t* tmax_k;                            // [n/1024+1] greatest key of each sorted tile
+    uint32_t* tmax_v;
     uint64_t* samp_k;                            // [n/64+1] every 64th key of each sorted tile
     uint32_t* samp_v;
     uint64_t* i_base;                            // [n]
@@ -133,6 +136,9 @@ struct P {  // kernel parameters
     Dev d;
     uint32_t C, nb;              // chunks, check blocks (32 ordinals each)
     uint32_t node_ctas;          // k_trace: CTAs with the node role
+    uint32_t alloc_ctas;         // k_trace: CTAs with the allocation role
+    uint32_t ordered;            // I keys compacted in ordinal order (k_isort gathers them by the
+                                 //  CTA prefix of icnt); else in atomic order (very large traces)
 };
 
 __device__ __forceinline__ void flag(Ctl* c, unsigned int bit) { atomicOr(&c->status, bit); }
@@ -257,14 +263,15 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         if (valid && (i & ((1u << (5 * l)) - 1)) == 0) T.node[T.off[l] + (i >> (5 * l))].y = x.t_alloc;
     // CTA-aggregated (one global atomic per CTA, not per warp: these are the same
     // addresses for every CTA): I positions, global prefilter bounds, upper tree levels
-    __shared__ uint32_t s_ni, s_base, s_wmax[kWarps];
+    __shared__ uint32_t s_ni, s_base, s_wmax[kWarps], s_wi[kWarps];
     __shared__ unsigned long long s_mn, s_mx;
-    if (threadIdx.x == 0) { s_ni = 0; s_mn = ~0ull; s_mx = 0; }
-    if (lane == 0) s_wmax[warp] = wmax;
-    __syncthreads();
     const uint32_t bal = __ballot_sync(0xffffffffu, isI);
-    uint32_t wpos = 0;
-    if (lane == 0 && bal) wpos = atomicAdd(&s_ni, (unsigned)__popc(bal));
+    if (threadIdx.x == 0) { s_mn = ~0ull; s_mx = 0; }
+    if (lane == 0) { s_wmax[warp] = wmax; s_wi[warp] = __popc(bal); }
+    __syncthreads();
+    uint32_t wpos = 0;  // the warp's first I key in the CTA: ordinal order
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) wpos += (uint32_t)w < warp ? s_wi[w] : 0u;
     const bool live = valid && x.size != 0;
     const uint64_t mn = warp_min_u64(live ? x.base : ~0ull);
     const uint64_t mx = warp_max_u64(live ? x.base + x.size : 0ull);
@@ -274,7 +281,17 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-        if (s_ni) s_base = atomicAdd(&p.d.ctl->nI, s_ni);
+        uint32_t ni = 0;
+#pragma unroll
+        for (int w = 0; w < kWarps; ++w) ni += s_wi[w];
+        s_ni = ni;
+        // ordered: the CTA's keys at its own region, k_isort finds them by the CTA
+        // prefix of icnt; else one atomic hands out positions
+        if (p.ordered) { s_base = cta * kThreads; p.d.icnt[cta] = ni; }
+        if (ni) {
+            const uint32_t b = atomicAdd(&p.d.ctl->nI, ni);
+            if (!p.ordered) s_base = b;
+        }
         if (s_mx) {
             atomicMax(&p.d.ctl->gmin_c, ~s_mn);
             atomicMax(&p.d.ctl->gmax, s_mx);
@@ -286,7 +303,6 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
             for (uint32_t l = 2; l <= T.top; ++l) atomicMax(&T.node[T.off[l] + (i0 >> (5 * l))].x, cmax);
     }
     __syncthreads();
-    wpos = __shfl_sync(0xffffffffu, wpos, 0);
     if (isI) {
         const uint32_t pos = s_base + wpos + __popc(bal & lanemask_lt());
         p.d.sk0[pos] = x.base;
@@ -384,22 +400,53 @@ struct ISortShared {
 };
 constexpr size_t kIsortSmem = sizeof(ISortShared);
 
+constexpr uint32_t kOrderedCtas = 16384;  // ordered compaction up to 16384 k_trace alloc CTAs (4 M allocations)
+
 __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     ISortShared& S = *reinterpret_cast<ISortShared*>(smem_raw);
+    uint32_t* s_pre = reinterpret_cast<uint32_t*>(smem_raw + sizeof(ISortShared));  // [alloc_ctas + 1]
+    __shared__ uint32_t s_wsum[kIsortThreads / 32];
     const unsigned long long tl0 = TL_NOW();
     unsigned long long tl_p = tl0;
     const uint32_t n = p.d.ctl->nI;
     const uint32_t t0 = blockIdx.x * kIsortTile;
     if (t0 >= n) return;
-    const uint32_t o = threadIdx.x * kSortPer;  // this thread's consecutive elements
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (p.ordered) {  // where each k_trace CTA's I keys start in ordinal order (exclusive prefix of icnt)
+        const uint32_t nbk = p.alloc_ctas;
+        const uint32_t per = (nbk + kIsortThreads - 1) / kIsortThreads;
+        const uint32_t b0 = min(tid * per, nbk), b1 = min(b0 + per, nbk);
+        uint32_t sum = 0;
+        for (uint32_t b = b0; b < b1; ++b) { const uint32_t c = __ldcg(p.d.icnt + b); s_pre[b] = sum; sum += c; }
+        uint32_t incl = sum;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= (uint32_t)d) incl += y;
+        }
+        if (lane == 31) s_wsum[warp] = incl;
+        __syncthreads();
+        uint32_t before = incl - sum;
+        for (uint32_t w = 0; w < warp; ++w) before += s_wsum[w];
+        for (uint32_t b = b0; b < b1; ++b) s_pre[b] += before;
+        if (tid == kIsortThreads - 1) s_pre[nbk] = before + sum;
+        __syncthreads();
+    }
+    const uint32_t o = tid * kSortPer;  // this thread's consecutive elements
     uint64_t k[kSortPer];
     uint32_t v[kSortPer];
 #pragma unroll
     for (int r = 0; r < kSortPer; ++r) {
         const uint32_t g = t0 + o + r;
-        k[r] = g < n ? __ldcg(p.d.sk0 + g) : ~0ull;
-        v[r] = g < n ? __ldcg(p.d.sv0 + g) : 0xFFFFFFFFu;
+        uint32_t q = g;
+        if (p.ordered && g < n) {  // the CTA holding compacted position g: last b with s_pre[b] <= g
+            uint32_t lo = 0, hi = p.alloc_ctas;
+            while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= g) lo = mid; else hi = mid; }
+            q = lo * kThreads + (g - s_pre[lo]);
+        }
+        k[r] = g < n ? __ldcg(p.d.sk0 + q) : ~0ull;
+        v[r] = g < n ? __ldcg(p.d.sv0 + q) : 0xFFFFFFFFu;
     }
     warp_bitonic_kv<kSortPer>(k, v);
     TL_PHASE(2, 30, tl_p);  // load + warp bitonic
@@ -451,6 +498,10 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
                 p.d.samp_k[t0 / kSampleStride + q / kSampleStride] = k[r];
                 p.d.samp_v[t0 / kSampleStride + q / kSampleStride] = v[r];
             }
+            if (t0 + q + 1 == min(t0 + kIsortTile, n)) {  // the tile's greatest key
+                p.d.tmax_k[blockIdx.x] = k[r];
+                p.d.tmax_v[blockIdx.x] = v[r];
+            }
         }
     }
     TL_REC(2, 0, tl0);
@@ -465,8 +516,11 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
 //     samples (every 32nd key) come in with one coalesced load and locate, by a
 //     shuffle search, the 32-key block of the tile holding each lane's lower
 //     bound; the block comes in with one more coalesced load and a shuffle
-//     search finishes the count.  The counts of the 8 warps meet in shared
-//     memory; warp 0 writes the 32 I entries.
+//     search finishes the count.  A tile whose key range lies wholly above or
+//     below the 32 keys is counted from its least and greatest key alone (the I
+//     keys are compacted in ordinal order, so with several models in one set most
+//     tiles hold another model's disjoint address region).  The counts of the 8
+//     warps meet in shared memory; warp 0 writes the 32 I entries.
 __device__ __forceinline__ bool kv_lt_lane(uint64_t k, uint32_t v, uint32_t src, uint64_t xk, uint32_t xv) {
     const uint64_t sk = __shfl_sync(0xffffffffu, k, src);
     const uint32_t sv = __shfl_sync(0xffffffffu, v, src);
@@ -513,6 +567,16 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
             const uint32_t b0 = tb * kIsortTile, nb = min((uint32_t)kIsortTile, nI - b0);
             const uint32_t ns = (nb + kSampleStride - 1) / kSampleStride;  // samples of tile tb (<= 64)
             const uint32_t s0 = b0 / kSampleStride;
+            {  // the tile's key range: lanes below its least key count 0, above its greatest nb
+                const uint64_t mnk = __ldcg(p.d.samp_k + s0), mxk = __ldcg(p.d.tmax_k + tb);
+                const uint32_t mnv = __ldcg(p.d.samp_v + s0), mxv = __ldcg(p.d.tmax_v + tb);
+                const bool above = has && kv_less(mxk, mxv, xk, xv);
+                const bool below = !has || kv_less(xk, xv, mnk, mnv);
+                if (__all_sync(0xffffffffu, above || below)) {  // (ordered I keys: most tiles of the ten-model set)
+                    cnt += above ? nb : 0u;
+                    continue;
+                }
+            }
             uint64_t sk0 = ~0ull, sk1 = ~0ull;
             uint32_t sv0 = 0xFFFFFFFFu, sv1 = 0xFFFFFFFFu;
             if (lane < ns) { sk0 = __ldcg(p.d.samp_k + s0 + lane); sv0 = __ldcg(p.d.samp_v + s0 + lane); }
@@ -574,8 +638,8 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
 // bases read with independent loads)
 __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t nf, uint32_t stride, uint32_t nI,
                                                const uint64_t* i_base, uint64_t x) {
-    uint32_t lo = 0, hi = nf;
-    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (fence[mid] <= x) lo = mid + 1; else hi = mid; }
+    uint32_t lo = 0, hi = nf;  // (fence: global, read-only here: the binary search runs out of L1)
+    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (__ldg(fence + mid) <= x) lo = mid + 1; else hi = mid; }
     if (lo == 0) return 0;
     const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
     uint32_t c = g0 + 1;
@@ -1187,6 +1251,7 @@ __global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
             __syncwarp();
             if (sp == 0) break;
             const uint32_t e = stk[--sp];
+            __syncwarp();  // every lane has read the popped entry before the next push reuses its slot
             lvl = (int)(e >> 24);
             node = e & 0xFFFFFFu;
         }
@@ -1195,8 +1260,7 @@ __global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
     TL_REC(8, 0, tl0);
 }
 
-__global__ void __launch_bounds__(kThreads, 6) k_check_mi(P p) {
-    __shared__ uint64_t s_fence[kFenceCap];
+__global__ void __launch_bounds__(kThreads) k_check_mi(P p) {
     const unsigned long long tl0 = TL_NOW();
     const uint32_t cta = blockIdx.x;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -1207,8 +1271,6 @@ __global__ void __launch_bounds__(kThreads, 6) k_check_mi(P p) {
     }
     const uint32_t stride = fence_stride(nI);
     const uint32_t nf = (nI + stride - 1) / stride;
-    for (uint32_t f = threadIdx.x; f < nf; f += blockDim.x) s_fence[f] = __ldcg(p.d.fence + f);
-    __syncthreads();
     const uint32_t b = cta * kWarps + warp;
     if (b >= p.nb) return;  // whole warp
     const uint32_t j = b * 32 + lane;
@@ -1219,10 +1281,10 @@ __global__ void __launch_bounds__(kThreads, 6) k_check_mi(P p) {
     bool bad = false;
     // M-I: the I entries meeting [base, end) are one run [s, e) of the sorted list
     if (mine && nI) {
-        const uint32_t k0 = i_count_le(s_fence, nf, stride, nI, p.d.i_base, x.base);  // bases <= base
+        const uint32_t k0 = i_count_le(p.d.fence, nf, stride, nI, p.d.i_base, x.base);  // bases <= base
         const uint32_t s = (k0 > 0 && p.d.i_rest[k0 - 1].end > x.base) ? k0 - 1 : k0;
         uint32_t e = k0;  // bases < end
-        if (k0 < nI && p.d.i_base[k0] < xe) e = i_count_le(s_fence, nf, stride, nI, p.d.i_base, xe - 1);
+        if (k0 < nI && p.d.i_base[k0] < xe) e = i_count_le(p.d.fence, nf, stride, nI, p.d.i_base, xe - 1);
         // overlap with I entry e: m freed before T_last -> t_alloc_e < t_free_m; else t_free_e > t_alloc_m
         const bool freed_early = x.t_free <= t_last;
         uint32_t k = s;
@@ -1249,51 +1311,60 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 
 // ----------------------------------------------------------------------------
 // 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
-//     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
-//     CTA; warp w takes the queue range classify's warp w filled.  Per candidate
-//     one group of bases and one entry (two dependent loads); a hit writes its
-//     record over its queue entry's word and sets its bit in the mask and in the
-//     I-resolved mask; the chunk's count grows by
-//     one atomic per warp (no CTA barrier: the warps run through the chunks
-//     independently).
-__global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
-    __shared__ uint64_t s_fence[kFenceCap];
+//     sorted I list.  One CTA per kIresChunks chunks; warp w takes the queue
+//     regions classify's warp w of those chunks filled, as one list (their loads
+//     overlap).  Per candidate: the fence search (global fences, through L1),
+//     one load of the <= stride bases of its group, one load of the entry; a hit
+//     writes its record over its queue entry's word and sets its bit in the mask
+//     and in the I-resolved mask; each chunk's count grows by one atomic per warp.
+constexpr int kIresChunks = 2;
+__global__ void __launch_bounds__(kThreads) k_iresolve(P p) {
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
-    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (nI) {
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t c0 = blockIdx.x * kIresChunks;
+    if (nI && c0 < p.C) {
         const uint32_t stride = fence_stride(nI);
         const uint32_t nf = (nI + stride - 1) / stride;
-        for (uint32_t f = tid; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
-        __syncthreads();
-        for (uint32_t c = blockIdx.x; c < p.C; c += gridDim.x) {
-            const uint32_t nq = __ldcg(p.d.qcnt + c * kWarps + warp);
-            const uint32_t q0 = (c * kWarps + warp) * p.d.cap_pw;
-            uint32_t cnt = 0;
-            for (uint32_t i0 = 0; i0 < nq; i0 += 32) {
-                const uint32_t k = q0 + i0 + lane;
-                bool hit = false;
-                if (i0 + lane < nq) {
-                    const IQ q = p.d.queue[k];
-                    const uint32_t le = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
-                    if (le) {
-                        const uint64_t base = p.d.i_base[le - 1];
-                        const IRest e = p.d.i_rest[le - 1];
-                        if (q.x < e.end && e.t_alloc < q.t) {
-                            hit = true;
-                            p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
-                            atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
-                            atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
-                        }
+        uint32_t nq[kIresChunks], tot = 0;
+#pragma unroll
+        for (int h = 0; h < kIresChunks; ++h) {
+            nq[h] = c0 + h < p.C ? __ldcg(p.d.qcnt + (c0 + h) * kWarps + warp) : 0u;
+            tot += nq[h];
+        }
+        uint32_t cnt[kIresChunks] = {};
+        for (uint32_t i0 = 0; i0 < tot; i0 += 32) {
+            const uint32_t i = i0 + lane;
+            bool hit = false;
+            uint32_t h = 0;
+            if (i < tot) {
+                uint32_t j = i;
+                while (h + 1 < kIresChunks && j >= nq[h]) { j -= nq[h]; ++h; }
+                const uint32_t k = ((c0 + h) * kWarps + warp) * p.d.cap_pw + j;
+                const IQ q = p.d.queue[k];
+                const uint32_t le = i_count_le(p.d.fence, nf, stride, nI, p.d.i_base, q.x);
+                if (le) {
+                    const uint64_t base = p.d.i_base[le - 1];
+                    const IRest e = p.d.i_rest[le - 1];
+                    if (q.x < e.end && e.t_alloc < q.t) {
+                        hit = true;
+                        p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
+                        atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
+                        atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
                     }
                 }
-                cnt += __popc(__ballot_sync(0xffffffffu, hit));
             }
-            // per-warp counts (no CTA barrier: the warps run ahead independently)
-            if (lane == 0 && cnt) {
-                atomicAdd(p.d.chunk_cnt + c, cnt);
-                atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)cnt);
+#pragma unroll
+            for (int hh = 0; hh < kIresChunks; ++hh) cnt[hh] += __popc(__ballot_sync(0xffffffffu, hit && h == (uint32_t)hh));
+        }
+        // per-warp counts (no CTA barrier: the warps run independently)
+        if (lane == 0) {
+#pragma unroll
+            for (int h = 0; h < kIresChunks; ++h) {
+                if (!cnt[h]) continue;
+                atomicAdd(p.d.chunk_cnt + c0 + h, cnt[h]);
+                atomicAdd(p.d.chunk_sup + ((c0 + h) >> 8), (unsigned long long)cnt[h]);
             }
         }
     }
@@ -1534,7 +1605,9 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
     o = (o + 63) & ~(size_t)63;
     s.d.tree.node = (uint2*)(z + o);
     if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) ||
-        (e = grow(s, s.d.sk0, N)) || (e = grow(s, s.d.sv0, N)) || (e = grow(s, s.d.sk, N)) || (e = grow(s, s.d.sv, N)) ||
+        (e = grow(s, s.d.sk0, N + kThreads)) || (e = grow(s, s.d.sv0, N + kThreads)) || (e = grow(s, s.d.sk, N)) ||
+        (e = grow(s, s.d.sv, N)) || (e = grow(s, s.d.icnt, N / kThreads + 2)) ||
+        (e = grow(s, s.d.tmax_k, N / kIsortTile + 2)) || (e = grow(s, s.d.tmax_v, N / kIsortTile + 2)) ||
         (e = grow(s, s.d.samp_k, N / kSampleStride + 64)) || (e = grow(s, s.d.samp_v, N / kSampleStride + 64)) ||
         (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
         (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
@@ -1568,7 +1641,8 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
     if (!s.h_ctl) {
         if ((*e = cudaMallocHost(&s.h_ctl, sizeof(Ctl))) != cudaSuccess) return nullptr;
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kClsSmem);
-        cudaFuncSetAttribute(k_isort, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kIsortSmem);
+        cudaFuncSetAttribute(k_isort, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(kIsortSmem + (kOrderedCtas + 1) * 4));
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
@@ -1604,7 +1678,8 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     const Tree shape = tree_shape(n);
     d.tree.top = shape.top;
     for (int l = 0; l <= kMaxLevels; ++l) { d.tree.cnt[l] = shape.cnt[l]; d.tree.off[l] = shape.off[l]; }
-    P p{a, d, C, nb, node_ctas};
+    const uint32_t ordered = alloc_ctas <= kOrderedCtas ? 1u : 0u;
+    P p{a, d, C, nb, node_ctas, alloc_ctas, ordered};
     *out = p;
     cudaError_t e;
     // branches (serialized on the caller's stream while per-launch timing is on)
@@ -1620,7 +1695,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaEventRecord(s.traced, stream)) || (e = cudaStreamWaitEvent(side, s.traced, 0))) return e;
         {
             TimedLaunch tl("mat_isort", side);
-            k_isort<<<sort_ctas, kIsortThreads, kIsortSmem, side>>>(p);
+            k_isort<<<sort_ctas, kIsortThreads, kIsortSmem + (ordered ? (alloc_ctas + 1) * 4 : 0), side>>>(p);
         }
         if (n > (uint64_t)kIsortTile) {  // (with one tile k_isort writes the I list itself)
             TimedLaunch tl("mat_rank", side);
@@ -1644,7 +1719,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if (C) {
             {
                 TimedLaunch tl("mat_iresolve", side);
-                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
+                k_iresolve<<<(C + kIresChunks - 1) / kIresChunks, kThreads, 0, side>>>(p);
             }
             TimedLaunch tl("mat_emit", side);
             if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;

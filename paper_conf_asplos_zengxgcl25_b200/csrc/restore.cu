@@ -195,6 +195,27 @@ __device__ __forceinline__ uint32_t load_rec(const RestoreArgs& a, uint64_t k, u
     return 0;
 }
 
+// the two halves of load_rec, for the in-place pass: the record load, then (once
+// it has landed) the replay-table gathers
+__device__ __forceinline__ uint64_t rec_load(const RestoreArgs& a, uint64_t k) {
+    return k < a.n_slots ? a.slot[k] : 0ull;
+}
+__device__ __forceinline__ uint32_t rec_kind(const RestoreArgs& a, uint64_t k, uint64_t rec, uint64_t& exp,
+                                             uint64_t& nv) {
+    exp = nv = 0;
+    if (k >= a.n_slots) return 1;
+    const uint64_t id = rec >> MEDUSA_OFF_BITS;
+    const uint64_t off = rec & kOffMask;
+    if (id >= a.n_alloc) return 1;
+    const uint64_t sz = __ldg(a.new_size + id);
+    const uint64_t ob = __ldg(a.old_base + id);
+    const uint64_t nb = __ldg(a.new_base + id);
+    if (off >= sz) return 2;
+    exp = ob + off;
+    nv = nb + off;
+    return 0;
+}
+
 __device__ __forceinline__ void report_add(unsigned long long* rep, uint32_t n_id, uint32_t n_rg, uint32_t n_st,
                                            uint64_t first, uint32_t n_chunk) {
     if (n_id | n_rg | n_st) {
@@ -390,7 +411,10 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     constexpr uint32_t kWords = CPB * kTaskWords;
     constexpr uint32_t kMask = CPB * kMaskPerTask;
     constexpr uint32_t kAllOk = (1u << CPB) - 1u;
-    constexpr uint32_t kPer = 2;  // records per thread per round
+#ifndef MEDUSA_INPLACE_PER
+#define MEDUSA_INPLACE_PER 2
+#endif
+    constexpr uint32_t kPer = MEDUSA_INPLACE_PER;  // records per thread per round
     __shared__ TableView<CPB> T;
     const uint32_t tid = threadIdx.x;
     const uint32_t task = blockIdx.x;
@@ -405,27 +429,29 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         uint32_t n_id = 0, n_rg = 0, n_st = 0;
         uint64_t first = ~0ull;
         bool fast = true;
+        // per round: the records (issued first), then -- independent of them -- each
+        // slot word located from the mask and loaded, then the replay-table gathers
+        // of the records: two dependent rounds, not three
         for (uint32_t rb = 0; rb < max(n_bits, 1u); rb += kPer * kThreads) {
-            uint64_t exp[kPer], nv[kPer];
-            uint32_t kind[kPer];  // 0 ok, 1 bad id, 2 bad range, 3 none
+            uint64_t rec[kPer], kk[kPer];
+            bool has[kPer];
 #pragma unroll
             for (int u = 0; u < kPer; ++u) {
                 const uint32_t r = rb + tid + u * kThreads;
-                kind[u] = 3;
-                exp[u] = nv[u] = 0;
-                uint64_t k = (uint64_t)cb0 + r;
-                if (r < n_bits && (fast || table_rec<CPB>(T, r, k))) kind[u] = load_rec(a, k, exp[u], nv[u]);
+                kk[u] = (uint64_t)cb0 + r;
+                has[u] = r < n_bits && (fast || table_rec<CPB>(T, r, kk[u]));
+                rec[u] = has[u] ? rec_load(a, kk[u]) : 0ull;
             }
             if (rb == 0) {
                 __syncthreads();  // prefix and consistency ready
                 n_bits = T.pre[kMask];
-                if (T.ok != kAllOk) {
+                if (T.ok != kAllOk) {  // (rare) an inconsistent chunk: round 0 again, chunk by chunk
                     fast = false;
 #pragma unroll
                     for (int u = 0; u < kPer; ++u) {
                         const uint32_t r = tid + u * kThreads;
-                        uint64_t k;
-                        kind[u] = (r < n_bits && table_rec<CPB>(T, r, k)) ? load_rec(a, k, exp[u], nv[u]) : 3u;
+                        has[u] = r < n_bits && table_rec<CPB>(T, r, kk[u]);
+                        rec[u] = has[u] ? rec_load(a, kk[u]) : 0ull;
                     }
                 }
             }
@@ -433,10 +459,14 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             uint64_t cur[kPer];
 #pragma unroll
             for (int u = 0; u < kPer; ++u) {  // locate every word first, then load them together
-                if (kind[u] == 3) continue;
+                if (!has[u]) continue;
                 qs[u] = table_word<CPB>(T, rb + tid + u * kThreads);
-                if (kind[u] == 0) cur[u] = ld_stream(a.src + ws + qs[u]);
+                cur[u] = ld_stream(a.src + ws + qs[u]);
             }
+            uint64_t exp[kPer], nv[kPer];
+            uint32_t kind[kPer];  // 0 ok, 1 bad id, 2 bad range, 3 none
+#pragma unroll
+            for (int u = 0; u < kPer; ++u) kind[u] = has[u] ? rec_kind(a, kk[u], rec[u], exp[u], nv[u]) : 3u;
 #pragma unroll
             for (int u = 0; u < kPer; ++u) {
                 if (kind[u] == 3) continue;
