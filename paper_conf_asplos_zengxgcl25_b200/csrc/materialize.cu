@@ -57,7 +57,9 @@ constexpr uint32_t ST_INVALID = 1, ST_TRACE = 2, ST_OVERFLOW = 4;
 constexpr int kThreads = 256;
 constexpr int kAblk = 32;          // allocation ordinals per overlap-check block (one warp)
 constexpr int kChkCap = 64;        // registered mortals staged per warp batch
-constexpr int kFenceCap = 8192;    // I-list fences (every stride-th sorted base; searched through L1)
+constexpr int kFenceCap = 2048;    // I-list fences (every stride-th sorted base): k_iresolve holds them in
+                                   //  shared memory (8192 searched through L1, and 4096 in shared memory
+                                   //  with a CTA's two chunks overlapped, measured slower: DESIGN.md §6)
 constexpr int kWinCap = 96;        // mortal-window entries per batch (<= 4 per lane of one warp; 96 keeps 7 classify CTAs per SM)
 constexpr int kWordsPerThread = MEDUSA_CHUNK_WORDS / kThreads;  // 8
 constexpr int kWarps = kThreads / 32;
@@ -638,8 +640,8 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
 // bases read with independent loads)
 __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t nf, uint32_t stride, uint32_t nI,
                                                const uint64_t* i_base, uint64_t x) {
-    uint32_t lo = 0, hi = nf;  // (fence: global, read-only here: the binary search runs out of L1)
-    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (__ldg(fence + mid) <= x) lo = mid + 1; else hi = mid; }
+    uint32_t lo = 0, hi = nf;  // (fence: shared memory in k_iresolve, global in k_check_mi)
+    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (fence[mid] <= x) lo = mid + 1; else hi = mid; }
     if (lo == 0) return 0;
     const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
     uint32_t c = g0 + 1;
@@ -1311,60 +1313,51 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 
 // ----------------------------------------------------------------------------
 // 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
-//     sorted I list.  One CTA per kIresChunks chunks; warp w takes the queue
-//     regions classify's warp w of those chunks filled, as one list (their loads
-//     overlap).  Per candidate: the fence search (global fences, through L1),
-//     one load of the <= stride bases of its group, one load of the entry; a hit
-//     writes its record over its queue entry's word and sets its bit in the mask
-//     and in the I-resolved mask; each chunk's count grows by one atomic per warp.
-constexpr int kIresChunks = 2;
-__global__ void __launch_bounds__(kThreads) k_iresolve(P p) {
+//     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
+//     CTA; warp w takes the queue range classify's warp w filled.  Per candidate
+//     one group of bases and one entry (two dependent loads); a hit writes its
+//     record over its queue entry's word and sets its bit in the mask and in the
+//     I-resolved mask; the chunk's count grows by
+//     one atomic per warp (no CTA barrier: the warps run through the chunks
+//     independently).
+__global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
+    __shared__ uint64_t s_fence[kFenceCap];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
-    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t c0 = blockIdx.x * kIresChunks;
-    if (nI && c0 < p.C) {
+    const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (nI) {
         const uint32_t stride = fence_stride(nI);
         const uint32_t nf = (nI + stride - 1) / stride;
-        uint32_t nq[kIresChunks], tot = 0;
-#pragma unroll
-        for (int h = 0; h < kIresChunks; ++h) {
-            nq[h] = c0 + h < p.C ? __ldcg(p.d.qcnt + (c0 + h) * kWarps + warp) : 0u;
-            tot += nq[h];
-        }
-        uint32_t cnt[kIresChunks] = {};
-        for (uint32_t i0 = 0; i0 < tot; i0 += 32) {
-            const uint32_t i = i0 + lane;
-            bool hit = false;
-            uint32_t h = 0;
-            if (i < tot) {
-                uint32_t j = i;
-                while (h + 1 < kIresChunks && j >= nq[h]) { j -= nq[h]; ++h; }
-                const uint32_t k = ((c0 + h) * kWarps + warp) * p.d.cap_pw + j;
-                const IQ q = p.d.queue[k];
-                const uint32_t le = i_count_le(p.d.fence, nf, stride, nI, p.d.i_base, q.x);
-                if (le) {
-                    const uint64_t base = p.d.i_base[le - 1];
-                    const IRest e = p.d.i_rest[le - 1];
-                    if (q.x < e.end && e.t_alloc < q.t) {
-                        hit = true;
-                        p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
-                        atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
-                        atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
+        for (uint32_t f = tid; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
+        __syncthreads();
+        for (uint32_t c = blockIdx.x; c < p.C; c += gridDim.x) {
+            const uint32_t nq = __ldcg(p.d.qcnt + c * kWarps + warp);
+            const uint32_t q0 = (c * kWarps + warp) * p.d.cap_pw;
+            uint32_t cnt = 0;
+            for (uint32_t i0 = 0; i0 < nq; i0 += 32) {
+                const uint32_t k = q0 + i0 + lane;
+                bool hit = false;
+                if (i0 + lane < nq) {
+                    const IQ q = p.d.queue[k];
+                    const uint32_t le = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
+                    if (le) {
+                        const uint64_t base = p.d.i_base[le - 1];
+                        const IRest e = p.d.i_rest[le - 1];
+                        if (q.x < e.end && e.t_alloc < q.t) {
+                            hit = true;
+                            p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
+                            atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
+                            atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
+                        }
                     }
                 }
+                cnt += __popc(__ballot_sync(0xffffffffu, hit));
             }
-#pragma unroll
-            for (int hh = 0; hh < kIresChunks; ++hh) cnt[hh] += __popc(__ballot_sync(0xffffffffu, hit && h == (uint32_t)hh));
-        }
-        // per-warp counts (no CTA barrier: the warps run independently)
-        if (lane == 0) {
-#pragma unroll
-            for (int h = 0; h < kIresChunks; ++h) {
-                if (!cnt[h]) continue;
-                atomicAdd(p.d.chunk_cnt + c0 + h, cnt[h]);
-                atomicAdd(p.d.chunk_sup + ((c0 + h) >> 8), (unsigned long long)cnt[h]);
+            // per-warp counts (no CTA barrier: the warps run ahead independently)
+            if (lane == 0 && cnt) {
+                atomicAdd(p.d.chunk_cnt + c, cnt);
+                atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)cnt);
             }
         }
     }
@@ -1678,7 +1671,10 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     const Tree shape = tree_shape(n);
     d.tree.top = shape.top;
     for (int l = 0; l <= kMaxLevels; ++l) { d.tree.cnt[l] = shape.cnt[l]; d.tree.off[l] = shape.off[l]; }
-    const uint32_t ordered = alloc_ctas <= kOrderedCtas ? 1u : 0u;
+    // ordinal-ordered I compaction pays when the set spans several address regions
+    // (several models: most rank tiles then hold another model's keys); a single
+    // model's set (<= 128 k_trace CTAs, ~4 tiles) skips the gather it costs k_isort
+    const uint32_t ordered = (alloc_ctas > 128 && alloc_ctas <= kOrderedCtas) ? 1u : 0u;
     P p{a, d, C, nb, node_ctas, alloc_ctas, ordered};
     *out = p;
     cudaError_t e;
@@ -1719,7 +1715,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if (C) {
             {
                 TimedLaunch tl("mat_iresolve", side);
-                k_iresolve<<<(C + kIresChunks - 1) / kIresChunks, kThreads, 0, side>>>(p);
+                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
             }
             TimedLaunch tl("mat_emit", side);
             if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
