@@ -97,7 +97,8 @@ struct IQ {  // a candidate word for the I-list search (k_iresolve)
 // first t_alloc < T1 (t_alloc increases with the ordinal on a well-formed trace).
 constexpr int kMaxLevels = 6;  // 32^5 > 2^24 allocations
 struct Tree {
-    uint2* leaf;                  // [n]
+    uint2* leaf;                  // [n] {v, t_alloc}
+    ulonglong2* leaf_be;          // [n] {base, base + size}: a kept leaf is a window entry as loaded
     uint2* node;                  // levels 1..top, level l at node + off[l]
     uint32_t off[kMaxLevels + 1]; // off[1] = 0
     uint32_t cnt[kMaxLevels + 1]; // nodes of level l (cnt[0] = n)
@@ -254,6 +255,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
             if (!isI) v = x.t_free;
         }
         T.leaf[i] = make_uint2(v, x.t_alloc);
+        T.leaf_be[i] = make_ulonglong2(x.base, x.base + x.size);
     }
     TL_PHASE(1, 20, tl_p);  // record load, checks
     // the mortal tree above the leaves: level 1 = this warp's 32 ordinals
@@ -1216,8 +1218,10 @@ __global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
             const uint32_t sh = 5u * (uint32_t)cl;
             bool keep = false;
             uint2 nd = make_uint2(0, 0);
+            ulonglong2 be = make_ulonglong2(0, 0);
             if (c < T.cnt[cl] && ((uint64_t)c << sh) < hj) {
                 nd = cl > 0 ? __ldcg(T.node + T.off[cl] + c) : __ldcg(T.leaf + c);
+                if (cl == 0) be = __ldcg(T.leaf_be + c);  // (same round)
                 keep = nd.x > hta;
             }
             const uint32_t kb = __ballot_sync(0xffffffffu, keep);
@@ -1225,14 +1229,8 @@ __global__ void __launch_bounds__(kThreads) k_check_mm(P p) {
                 if (keep) stk[sp + __popc(kb & lanemask_lt())] = ((uint32_t)cl << 24) | c;
                 sp += __popc(kb);
             } else if (kb) {  // leaves: mortals i < hj with t_free_i > hta
-                uint64_t yb = 0, ye = 0;
-                bool k2 = false;
-                if (keep) {
-                    const medusa_alloc r = ld_alloc(p.a.alloc + c);
-                    yb = r.base;
-                    ye = r.base + r.size;
-                    k2 = yb < he && hb < ye;
-                }
+                const uint64_t yb = be.x, ye = be.y;
+                const bool k2 = keep && yb < he && hb < ye;
                 const uint32_t k2b = __ballot_sync(0xffffffffu, k2);
                 __syncwarp();
                 if (k2) {
@@ -1597,7 +1595,7 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
     s.d.chunk_cnt = (uint32_t*)(z + o); o += CC * 4;
     o = (o + 63) & ~(size_t)63;
     s.d.tree.node = (uint2*)(z + o);
-    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) ||
+    if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) || (e = grow(s, s.d.tree.leaf_be, N)) ||
         (e = grow(s, s.d.sk0, N + kThreads)) || (e = grow(s, s.d.sv0, N + kThreads)) || (e = grow(s, s.d.sk, N)) ||
         (e = grow(s, s.d.sv, N)) || (e = grow(s, s.d.icnt, N / kThreads + 2)) ||
         (e = grow(s, s.d.tmax_k, N / kIsortTile + 2)) || (e = grow(s, s.d.tmax_v, N / kIsortTile + 2)) ||
