@@ -756,14 +756,14 @@ def run_ours(args):
     # stream: per-kernel durations for the roofline and the breakdown
     def step_queued():
         # as step(), with a device spin (~0.2 ms) queued before the analysis and one
-        # (~30 us) between the analysis (whose slot-count read-back leaves the GPU
+        # (~0.1 ms) between the analysis (whose slot-count read-back leaves the GPU
         # idle) and the restore: the host has enqueued each call's launches and
         # events before the GPU reaches them, so the launch events see device time,
         # not the host's launch latency
         medusa.kernel_table_set(inp["table"])
         torch.cuda._sleep(400000)
         medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"], out=slots)
-        torch.cuda._sleep(60000)
+        torch.cuda._sleep(200000)
         medusa.restore(inp["words"], slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"],
                        dst=dst, func_out=fout, report=rep)
 
@@ -1081,7 +1081,7 @@ def run_ours(args):
             "sync_api_ms_per_step": max_over_ranks(sum(sync_ms), dist, dev) / args.steps,
             "instrumented_ms_per_step": sum(inst_ms) / args.steps,
             "instrumented_note": "per-kernel events, branches serialized, device spins queued before the analysis "
-                                 "(~0.2 ms) and before the restore (~30 us) so no event waits for the host; "
+                                 "(~0.2 ms) and before the restore (~0.1 ms) so no event waits for the host; "
                                  "instrumented_ms_per_step includes the spins (share_of_step = share of the summed "
                                  "kernel times, as in the ncu launch list)",
             "clocks": clocks,

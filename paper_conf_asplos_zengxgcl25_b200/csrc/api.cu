@@ -35,6 +35,19 @@ struct TimingRec {
 };
 thread_local bool g_timing = false;
 thread_local std::vector<TimingRec> g_timing_recs;
+thread_local std::vector<cudaEvent_t> g_event_pool;  // events reused across reads (creating one per
+                                                       // launch made the host slower than the GPU)
+
+cudaEvent_t pooled_event() {
+    if (!g_event_pool.empty()) {
+        cudaEvent_t e = g_event_pool.back();
+        g_event_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
 
 }  // namespace
 
@@ -42,9 +55,7 @@ bool timing_enabled() { return g_timing; }
 
 TimedLaunch::TimedLaunch(const char* n, cudaStream_t s) : name(n), stream(s), slot(nullptr) {
     if (!g_timing) return;
-    TimingRec r{n, nullptr, nullptr};
-    cudaEventCreate(&r.start);
-    cudaEventCreate(&r.stop);
+    TimingRec r{n, pooled_event(), pooled_event()};
     cudaEventRecord(r.start, s);
     g_timing_recs.push_back(r);
     slot = reinterpret_cast<void*>(g_timing_recs.size());
@@ -103,8 +114,8 @@ int medusa_timing_read(const char** names, float* ms, int max) {
             if (ms) ms[n] = t;
             ++n;
         }
-        cudaEventDestroy(r.start);
-        cudaEventDestroy(r.stop);
+        g_event_pool.push_back(r.start);
+        g_event_pool.push_back(r.stop);
     }
     g_timing_recs.clear();
     return n;
