@@ -4,41 +4,39 @@
 // [base_i, base_i + size_i) holds w ("identical or within the range");
 // emit the indirect index pointer table in word order.
 //
-// Structure of a well-formed trace that the GPU design exploits (DESIGN.md §3):
+// Structure of a well-formed trace that the GPU design exploits (DESIGN.md §5):
 //  * I = allocations live at the LAST launch T_last.  All of them are live at
 //    the same instant, so they are pairwise address-disjoint: one list sorted by
 //    base answers "which I-allocation holds w" with one search; it is live at
 //    t <= T_last iff t_alloc < t.  (Weights, KV cache, static inputs, permanent
 //    buffers: ~27k entries for the ten-model set.)
 //  * M = every other allocation ("mortal": capture temporaries, warm-up and
-//    profiling scratch).  A mortal is registered in exactly the word chunks that
-//    hold words of nodes launched during its lifetime; a chunk's window (~60
-//    entries for the ten-model set) sits in shared memory in list order with a
-//    per-node live bit mask; a word is looked up among the entries live at its
-//    node (about four in the BASELINE sets) by a range test.
+//    profiling scratch).  The mortals live at one launch are pairwise disjoint;
+//    a chunk's window (~60 entries for the ten-model set) holds exactly the
+//    mortals live at one of its launches, found by a descent of the MORTAL TREE
+//    (a 32-ary max tree over ordinals: leaf = t_free of a mortal, node = max
+//    over its ordinals + the first ordinal's t_alloc); a word is looked up among
+//    the entries live at its node (about four) by a range test.
 //  * Well-formedness (no two simultaneously-live allocations overlap) is checked
 //    exactly: I-I by adjacency of the sorted list, M-I with per-32-entry
 //    min(t_alloc) / max(t_free) summaries over the address run a mortal meets,
-//    M-M inside blocks of 32 allocation ordinals against the mortals registered
-//    as live there.
+//    M-M per block of 32 ordinals against the mortals the tree reports live when
+//    they are allocated.
 // Pipeline (the synchronous entry adds one host read at the end):
-//   memset (counters) -> k_trace -> k_prepare -> k_classify ............ (join) [-> k_result]
-//   side (high priority):  k_rank -> (after k_classify) k_iresolve -> k_emit ---^
-//   low (default priority): (after k_rank) k_check ----------------------------^
-//   k_trace      [nodes] CSR / launch-order checks, first/last node per chunk;
-//                [allocs] trace checks, I/M split, registration ranges, two-level
-//                registration counts, I compaction
-//   k_prepare    [sort] I keys sorted in tiles of 1024 (register bitonic per warp
-//                + shared-memory merges); [scatter] registration lists.  Triggers
-//                its dependents at once: k_classify's setup overlaps it
-//   k_rank       global rank of every I key -> the sorted I arrays, the fences and
-//                the per-32 summaries
-//   k_classify   one CTA per 2048-word chunk: before griddepcontrol.wait the TMA
-//                copy of the chunk's words, node starts, candidate compaction;
-//                after it the mortal window, per-node live masks, the lookups;
-//                mask words, records at their word index, I-list candidates into
-//                a per-warp queue, the chunk's slot count
-//   k_check      M-M, M-I and I-I overlap checks
+//   memset -> k_trace -> k_classify .......................................(join) [-> k_result]
+//   side (high priority):  k_isort -> k_rank -> (after k_classify) k_iresolve -> k_emit --^
+//   low (default priority): k_check_mm ... (after k_rank) k_check_mi ---------------------^
+//   k_trace      [nodes] CSR / launch-order checks, first/last node of each chunk and
+//                their launch positions; [allocs] trace checks, I/M split, the
+//                mortal tree, prefilter bounds, I compaction (ordinal order)
+//   k_isort      I keys sorted in tiles of 1024 (register bitonic per warp + merges)
+//   k_rank       global rank of every I key -> the sorted I arrays, fences, summaries
+//   k_classify   one CTA per 2048-word chunk: TMA copy of the words (before the
+//                wait), node starts, the window by a tree query, candidate
+//                compaction, live masks, lookups; per warp: records and I-list
+//                queue entries into its regions, mask words, slot count
+//   k_check_mm   M-M overlap check (tree descent per warp)
+//   k_check_mi   M-I and I-I overlap checks
 //   k_iresolve   queued candidates against the sorted I list
 //   k_emit       chunk_base (two-level prefix) and the records compacted into the
 //                slot table
