@@ -23,9 +23,9 @@
 //    M-M per block of 32 ordinals against the mortals the tree reports live when
 //    they are allocated.
 // Pipeline (the synchronous entry adds one host read at the end):
-//   memset -> k_trace -> k_classify .......................................(join) [-> k_result]
-//   side (high priority):  k_isort -> k_rank -> (after k_classify) k_iresolve -> k_emit --^
-//   low (default priority): k_check_mm ... (after k_rank) k_check_mi ---------------------^
+//   memset -> k_trace -> k_classify -> (after k_rank) k_iresolve -> k_emit ....(join) [-> k_result]
+//   side (high priority):  k_isort -> k_rank --^
+//   low (default priority): k_check_mm ... (after k_rank) k_check_mi ------------------^
 //   k_trace      [nodes] CSR / launch-order checks, first/last node of each chunk and
 //                their launch positions; [allocs] trace checks, I/M split, the
 //                mortal tree, prefilter bounds, I compaction (ordinal order)
@@ -1649,9 +1649,9 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
 }
 
 // the whole analysis on `stream` (no synchronization):
-//   stream:            memset -> k_trace [traced] -> k_classify [classified] .............. [emitted][join]
-//   side (high prio):             [traced] k_isort -> k_rank [ranked] [classified] k_iresolve -> k_emit [emitted]
-//   low (default):                    [traced] k_check_mm ... [ranked] k_check_mi [join]
+//   stream:            memset -> k_trace [traced] -> k_classify -> [ranked] k_iresolve -> k_emit [join]
+//   side (high prio):             [traced] k_isort -> k_rank [ranked]
+//   low (default):                [traced] k_check_mm ... [ranked] k_check_mi [join]
 // The high-priority stream gets the sort / rank CTAs dispatched ahead of the
 // classify CTAs and the queue resolution / emission ahead of the trace checks,
 // which fill in around them and complete the call.
@@ -1703,20 +1703,39 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         TimedLaunch tl("mat_classify", stream);
         if ((e = launch_pdl(k_classify, C, kThreads, kClsSmem, stream, p))) return e;
     }
+#ifndef MEDUSA_MAIN_TAIL
+#define MEDUSA_MAIN_TAIL 1  // (0: on the side stream, joined: ALL10 +1.5 us, C5 +1.2 us)
+#endif
     if (n) {
-        if ((e = cudaEventRecord(s.classified, stream))) return e;
-        // high priority after the classify: queue resolution and emission (the
-        // rank is already on this stream)
-        if ((e = cudaStreamWaitEvent(side, s.classified, 0))) return e;
-        if (C) {
-            {
-                TimedLaunch tl("mat_iresolve", side);
-                k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
+        if (MEDUSA_MAIN_TAIL) {
+            // the caller's stream after the classify and the rank: queue resolution and
+            // emission, so k_result and a following restore are their programmatic successors
+            if ((e = cudaStreamWaitEvent(stream, s.ranked, 0))) return e;
+            if (C) {
+                {
+                    TimedLaunch tl("mat_iresolve", stream);
+                    if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0,
+                                        stream, p)))
+                        return e;
+                }
+                TimedLaunch tl("mat_emit", stream);
+                if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
             }
-            TimedLaunch tl("mat_emit", side);
-            if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
+        } else {
+            if ((e = cudaEventRecord(s.classified, stream))) return e;
+            // high priority after the classify: queue resolution and emission (the
+            // rank is already on this stream)
+            if ((e = cudaStreamWaitEvent(side, s.classified, 0))) return e;
+            if (C) {
+                {
+                    TimedLaunch tl("mat_iresolve", side);
+                    k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
+                }
+                TimedLaunch tl("mat_emit", side);
+                if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
+            }
+            if ((e = cudaEventRecord(s.emitted, side))) return e;
         }
-        if ((e = cudaEventRecord(s.emitted, side))) return e;
         // default priority: the trace checks fill in around them (M-M needs the
         // mortal tree only, M-I and I-I the sorted I list)
         if ((e = cudaStreamWaitEvent(low, s.traced, 0))) return e;
@@ -1730,7 +1749,8 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             k_check_mi<<<check_ctas, kThreads, 0, low>>>(p);
         }
         if ((e = cudaEventRecord(s.join, low))) return e;
-        if ((e = cudaStreamWaitEvent(stream, s.emitted, 0)) || (e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
+        if (!MEDUSA_MAIN_TAIL && (e = cudaStreamWaitEvent(stream, s.emitted, 0))) return e;
+        if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
         TimedLaunch tl("mat_emit", stream);
         if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
