@@ -1714,8 +1714,11 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
             if (C) {
                 {
                     TimedLaunch tl("mat_iresolve", stream);
-                    if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0,
-                                        stream, p)))
+#ifndef MEDUSA_IRES_PER_SM
+#define MEDUSA_IRES_PER_SM 6
+#endif
+                    if ((e = launch_pdl(k_iresolve, std::min<unsigned>(C, (unsigned)s.sm_count * MEDUSA_IRES_PER_SM),
+                                        kThreads, 0, stream, p)))
                         return e;
                 }
                 TimedLaunch tl("mat_emit", stream);
