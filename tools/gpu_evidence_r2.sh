@@ -6,7 +6,12 @@ TAG=${TAG:-r2}
 python -c "import __graft_entry__ as g; g.build()" || exit 1
 nvidia-smi --query-gpu=name,driver_version,clocks.max.sm,memory.total --format=csv > gpurun_out/gpu_$TAG.txt
 lscpu | grep -E "Model name|^CPU\(s\)" >> gpurun_out/gpu_$TAG.txt
-for W in all10 llama2-13b qwen1.5-4b llama2-7b; do
+timeout 900 python bench.py --steps 50 --warmup 5 > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TAG.err
+: > gpurun_out/configs_$TAG.jsonl
+for W in qwen1.5-4b llama2-7b llama2-13b all10-inband; do
+  timeout 600 python bench.py --workload $W --steps 50 --warmup 5 --cpu-seconds 4 --no-buffers --sustained 8 --c5-sustained 0 >> gpurun_out/configs_$TAG.jsonl 2> gpurun_out/configs_${TAG}_$W.err
+done
+for W in all10 llama2-13b qwen1.5-4b llama2-7b all10-inband; do
   timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum --clock-control none --csv --log-file gpurun_out/launches_${TAG}_$W.csv python bench.py --workload $W --steps 2 --warmup 3 --sustained 0 --no-cpu-baseline --no-c5 --no-buffers > /dev/null 2>&1
   python tools/make_traffic.py gpurun_out/launches_${TAG}_$W.csv gpurun_out/ncu_traffic_$TAG.json $W > /dev/null
   echo "launch list $W: $(wc -l < gpurun_out/launches_${TAG}_$W.csv) lines"
@@ -23,11 +28,15 @@ timeout 300 python tools/timeline.py --workload llama2-13b --steps 5 > gpurun_ou
 timeout 300 python tools/timeline.py --serial --steps 3 > gpurun_out/timeline_${TAG}_serial.txt 2>&1
 # sanitizers: every GPU test for memcheck; the full-size and special paths for the others
 : > gpurun_out/sanitizer_summary_$TAG.txt
-timeout 2400 compute-sanitizer --tool memcheck --error-exitcode 9 python -m pytest tests -m gpu -x -q > gpurun_out/sanitizer_memcheck_$TAG.log 2>&1
+timeout 2400 compute-sanitizer --tool memcheck --report-api-errors no --error-exitcode 9 python -m pytest tests -m gpu -x -q > gpurun_out/sanitizer_memcheck_$TAG.log 2>&1
 echo "memcheck (all -m gpu tests) exit=$?" >> gpurun_out/sanitizer_summary_$TAG.txt; tail -3 gpurun_out/sanitizer_memcheck_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
-for tool in racecheck synccheck initcheck; do
-  timeout 2400 compute-sanitizer --tool $tool --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py tests/test_gpu_buffers.py tests/test_real_capture.py -m gpu -x -q -k "all10 or in_place or overflow or real or table or malformed or toy or tiny or edge or capacity or fault or async" > gpurun_out/sanitizer_${tool}_$TAG.log 2>&1
+for tool in racecheck synccheck; do
+  timeout 1800 compute-sanitizer --tool $tool --report-api-errors no --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py tests/test_gpu_buffers.py tests/test_real_capture.py tests/test_gpu_multi.py -m gpu -x -q -k "all10 or in_place or overflow or real or table or malformed or toy or tiny or edge or capacity or fault or async or every_gpu" > gpurun_out/sanitizer_${tool}_$TAG.log 2>&1
   echo "$tool (full-size + special paths) exit=$?" >> gpurun_out/sanitizer_summary_$TAG.txt
   tail -3 gpurun_out/sanitizer_${tool}_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
 done
+# initcheck tracks every byte: the small sets, one ALL10 full path, in place, the table cases
+timeout 1800 compute-sanitizer --tool initcheck --report-api-errors no --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py -m gpu -x -q -k "full_path_parity and (toy or llama2) or in_place_full_path or fault or edge or capacity or hand_derived or overflow" > gpurun_out/sanitizer_initcheck_$TAG.log 2>&1
+echo "initcheck (small sets, ALL10 full path, in place, faults, tables, overflow) exit=$?" >> gpurun_out/sanitizer_summary_$TAG.txt
+tail -3 gpurun_out/sanitizer_initcheck_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
 cat gpurun_out/sanitizer_summary_$TAG.txt
