@@ -551,7 +551,7 @@ def oracle_parity(gs, slots, n_slots, dst, fout, rep):
         "n_slots": n_slots == m["n_slots"],
         "mask": np.array_equal(h(slots.mask).view(np.uint32), mask),
         "chunk_base": np.array_equal(h(slots.chunk_base).view(np.uint32), cb),
-        "records": np.array_equal(h(slots.slot)[:m["n_slots"]].view(np.uint64), rec),
+        "records": np.array_equal(h(slots.slot[:m["n_slots"]]).view(np.uint64), rec),
         "words": np.array_equal(medusa.to_numpy_u64(dst), odst),
         "func_out": np.array_equal(medusa.to_numpy_u64(fout), ofout),
         "report": np.array_equal(medusa.report_numpy(rep), orep),

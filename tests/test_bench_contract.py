@@ -1,4 +1,4 @@
-"""The committed bench line (profiles/r1_bench.json, written by bench.py on a B200)
+"""The committed bench line (profiles/r2_bench.json, written by bench.py on a B200)
 keeps the driver's JSON contract: every required key, the timing rules it can
 show (warm-up >= 3, clocks sampled inside the timed region, no throttle reason
 that rejects a run), and self-consistent derived numbers."""
@@ -8,7 +8,7 @@ import os
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-LINE = os.path.join(ROOT, "profiles", "r1_bench.json")
+LINE = os.path.join(ROOT, "profiles", "r2_bench.json")
 
 
 @pytest.fixture(scope="module")
@@ -48,3 +48,22 @@ def test_derived_numbers(line):
     e2e = line["e2e"]
     assert e2e["unit"] == line["unit"] and e2e["h2d_bytes_per_step"] > 0 and e2e["d2h_bytes_per_step"] > 0
     assert e2e["value"] < line["value"]  # the end-to-end number is not the device-timed one
+
+
+def test_multi_gpu_block(line):
+    mg = line["multi_gpu"]
+    assert mg["collective"].startswith("none")
+    assert len(mg["headline_per_rank"]) == line["n_gpus"]
+    assert all(r["parity"]["ok"] for r in mg["headline_per_rank"])
+    c5 = mg["c5"]
+    assert len(c5["per_gpu"]) == line["n_gpus"]
+    for g in c5["per_gpu"]:
+        assert g["seed"] == 100 + g["rank"] and g["parity"]["ok"]
+    nodes = sum(g["nodes"] for g in c5["per_gpu"])
+    assert c5["aggregate_nodes_per_s"] == pytest.approx(nodes / (c5["ms_per_step"] / 1e3), rel=1e-6)
+
+
+def test_whole_step_fraction(line):
+    ws = line["roofline"]["whole_step"]
+    assert ws["ms_per_step"] == pytest.approx(line["ms_per_step"], rel=1e-9)
+    assert ws["achieved"] == pytest.approx(ws["alg_bytes"] / (ws["ms_per_step"] / 1e3) / 1e9, rel=1e-6)

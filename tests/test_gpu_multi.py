@@ -57,7 +57,7 @@ def test_every_gpu_restores_its_own_instance_concurrently():
                 s.synchronize()
                 h = lambda t: t.detach().cpu().numpy()
                 out[seed] = (slots.n_slots, h(slots.mask).view(np.uint32), h(slots.chunk_base).view(np.uint32),
-                             h(slots.slot)[: slots.n_slots].view(np.uint64), medusa.to_numpy_u64(dst),
+                             h(slots.slot[:slots.n_slots]).view(np.uint64), medusa.to_numpy_u64(dst),
                              medusa.to_numpy_u64(fout) if gather else None, medusa.report_numpy(rep))
         except Exception as e:  # pragma: no cover - reported below
             errs.append((seed, repr(e)))

@@ -42,7 +42,7 @@ def _check_materialize(slots, m, packed, n_words):
     assert slots.n_slots == m["n_slots"]
     assert np.array_equal(_h(slots.mask).view(np.uint32), mask)
     assert np.array_equal(_h(slots.chunk_base).view(np.uint32), cb)
-    assert np.array_equal(_h(slots.slot)[: slots.n_slots].view(np.uint64), rec)
+    assert np.array_equal(_h(slots.slot[:slots.n_slots]).view(np.uint64), rec)
 
 
 @pytest.mark.parametrize("name", ["toy", "qwen1.5-4b", "llama2-7b", "llama2-13b", "all10", "all10-inband"])
@@ -186,7 +186,7 @@ def test_tiny_traces_status_and_slots(overlap_p):
             assert s.n_slots == m["n_slots"]
             assert np.array_equal(_h(s.mask).view(np.uint32), mask), seed
             assert np.array_equal(_h(s.chunk_base).view(np.uint32), cb), seed
-            assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec), seed
+            assert np.array_equal(_h(s.slot[:s.n_slots]).view(np.uint64), rec), seed
 
 
 @pytest.mark.parametrize("seed", range(6))
@@ -205,7 +205,7 @@ def test_long_chunks_many_nodes_and_window_batches(seed):
         assert s.n_slots == m["n_slots"]
         assert np.array_equal(_h(s.mask).view(np.uint32), mask)
         assert np.array_equal(_h(s.chunk_base).view(np.uint32), cb)
-        assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec)
+        assert np.array_equal(_h(s.slot[:s.n_slots]).view(np.uint64), rec)
 
 
 def test_edge_cases():
@@ -227,7 +227,7 @@ def test_edge_cases():
     st, s = _run_tiny(w, np.array([0, 1, 4096, 5000], np.uint64), np.array([2, 3, 4], np.uint32),
                       A([(b, 8 * 5000, 1, T_NEVER)]))
     assert st == 0 and s.n_slots == 5000
-    assert (_h(s.slot)[:5000] == np.arange(5000) * 8).all()
+    assert (_h(s.slot[:5000]) == np.arange(5000) * 8).all()
     # a single node spanning many chunks with its allocation freed before it launches
     st, s = _run_tiny(w, np.array([0, 5000], np.uint64), np.array([9], np.uint32), A([(b, 8 * 5000, 1, 9)]))
     assert st == 0 and s.n_slots == 0
@@ -431,13 +431,13 @@ def test_overflow_retry_many_batches_wide_chunks(seed):
     assert s.n_slots == m["n_slots"]
     assert np.array_equal(_h(s.mask).view(np.uint32), mask)
     assert np.array_equal(_h(s.chunk_base).view(np.uint32), cb)
-    assert np.array_equal(_h(s.slot)[: s.n_slots].view(np.uint64), rec)
+    assert np.array_equal(_h(s.slot[:s.n_slots]).view(np.uint64), rec)
     # the async entry now runs with the grown scratch
     res = torch.zeros(2, dtype=torch.int64, device=DEV)
     out = medusa.alloc_slots(words.size, DEV)
     medusa.materialize_async(**inp, out=out, result=res)
     assert medusa.mat_result(res) == (0, m["n_slots"])
-    assert np.array_equal(_h(out.slot)[: m["n_slots"]].view(np.uint64), rec)
+    assert np.array_equal(_h(out.slot[:m["n_slots"]]).view(np.uint64), rec)
 
 
 def test_malformed_csr_across_chunks_is_rejected_safely(graph_sets):

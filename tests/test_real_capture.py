@@ -32,7 +32,7 @@ def test_real_graph_materialize_restore_replay():
     mask, cb, rec = oracle.pack(m, r["words"].size)
     s = r["slots"]
     assert s.n_slots == m["n_slots"] > 0
-    assert np.array_equal(medusa.to_numpy_u64(s.slot)[: s.n_slots], rec)
+    assert np.array_equal(medusa.to_numpy_u64(s.slot[: s.n_slots]), rec)
     assert np.array_equal(s.mask.cpu().numpy().view(np.uint32), mask)
     # restore: every slot valid; the oracle restores the same bytes
     assert int(r["report"][0]) == 0

@@ -36,7 +36,7 @@ for tool in racecheck synccheck; do
   tail -3 gpurun_out/sanitizer_${tool}_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
 done
 # initcheck tracks every byte: the small sets, one ALL10 full path, in place, the table cases
-timeout 1800 compute-sanitizer --tool initcheck --report-api-errors no --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py -m gpu -x -q -k "full_path_parity and (toy or llama2) or in_place_full_path or fault or edge or capacity or hand_derived or overflow" > gpurun_out/sanitizer_initcheck_$TAG.log 2>&1
+timeout 1800 compute-sanitizer --tool initcheck --report-api-errors no --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py -m gpu -x -q -k "full_path_parity and (toy or llama2-13b) or in_place_full_path or fault or edge or capacity or hand_derived or overflow" > gpurun_out/sanitizer_initcheck_$TAG.log 2>&1
 echo "initcheck (small sets, ALL10 full path, in place, faults, tables, overflow) exit=$?" >> gpurun_out/sanitizer_summary_$TAG.txt
 tail -3 gpurun_out/sanitizer_initcheck_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
 cat gpurun_out/sanitizer_summary_$TAG.txt
