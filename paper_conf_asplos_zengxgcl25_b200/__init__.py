@@ -15,7 +15,8 @@ import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmedusa.so")
+# MEDUSA_LIB: a diagnostic build variant of the same library (tools/, A/B runs)
+LIB_PATH = os.environ.get("MEDUSA_LIB") or os.path.join(_HERE, "libmedusa.so")
 
 OK, ERR_INVALID_ARG, ERR_TRACE, ERR_CAPACITY, ERR_NO_TABLE, ERR_CUDA, ERR_RETRY = 0, -1, -2, -3, -4, -5, -6
 N_SLOTS_FROM_TABLE = (1 << 64) - 1

@@ -112,7 +112,6 @@ struct Dev {  // scratch of one call (device pointers)
     uint64_t *sk0, *sk;                          // [n] I keys (base): compacted by k_trace / sorted tiles
     uint32_t *sv0, *sv;                          // [n] their allocation ordinals
     uint32_t* icnt;                              // [n/256+1] I keys of each k_trace alloc CTA (ordered mode)
-    uint32_t* tcnt;                              // [n/8192+1] I keys of each ordinal-range tile (early mode)
     uint64_t* tmax_k;                            // [n/1024+1] greatest key of each sorted tile
     uint32_t* tmax_v;
     uint64_t* samp_k;                            // [n/64+1] every 64th key of each sorted tile
@@ -141,8 +140,6 @@ struct P {  // kernel parameters
     uint32_t alloc_ctas;         // k_trace: CTAs with the allocation role
     uint32_t ordered;            // I keys compacted in ordinal order (k_isort gathers them by the
                                  //  CTA prefix of icnt); else in atomic order (very large traces)
-    uint32_t early;              // the I list sorted beside k_trace over ordinal-range tiles
-                                 //  (k_isort_early); k_trace then neither compacts nor counts I
 };
 
 __device__ __forceinline__ void flag(Ctl* c, unsigned int bit) { atomicOr(&c->status, bit); }
@@ -293,7 +290,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         // ordered: the CTA's keys at its own region, k_isort finds them by the CTA
         // prefix of icnt; else one atomic hands out positions
         if (p.ordered) { s_base = cta * kThreads; p.d.icnt[cta] = ni; }
-        if (ni && !p.early) {
+        if (ni) {
             const uint32_t b = atomicAdd(&p.d.ctl->nI, ni);
             if (!p.ordered) s_base = b;
         }
@@ -308,7 +305,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
             for (uint32_t l = 2; l <= T.top; ++l) atomicMax(&T.node[T.off[l] + (i0 >> (5 * l))].x, cmax);
     }
     __syncthreads();
-    if (isI && !p.early) {
+    if (isI) {
         const uint32_t pos = s_base + wpos + __popc(bal & lanemask_lt());
         p.d.sk0[pos] = x.base;
         p.d.sv0[pos] = i;
@@ -513,150 +510,6 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
     pdl_trigger();
 }
 
-// 2a'. k_isort_early (side stream, beside k_trace: it reads only the inputs):
-//     tile t = allocation ordinals [t S, t S + S), S = kEarlySpan.  The tile's I
-//     allocations (non-empty, t_alloc < T_last < t_free) are compacted into
-//     shared memory (kEarlyLoads record loads in flight per thread) and sorted by
-//     (base, ordinal): up to kEarlyCap keys by a register bitonic sort of 128
-//     keys per warp and merge-path rounds through shared memory, more (an
-//     I-dense tile) by a plain bitonic sort in shared memory.  Output at the
-//     tile's fixed offset t S: the sorted keys, every 32nd key as a sample, the
-//     tile's greatest key and count; a single tile writes the I list itself.
-constexpr int kEarlyThreads = 512;
-constexpr int kEarlySpan = 8192;
-constexpr int kEarlyCap = kEarlyThreads * kSortPer;  // 2048
-constexpr int kEarlyLoads = 4;
-struct EarlyShared {
-    uint64_t k[kEarlySpan];
-    uint32_t v[kEarlySpan];
-    uint32_t m;
-};
-constexpr size_t kEarlySmem = sizeof(EarlyShared);
-
-__global__ void __launch_bounds__(kEarlyThreads) k_isort_early(P p) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    EarlyShared& S = *reinterpret_cast<EarlyShared*>(smem_raw);
-    const unsigned long long tl0 = TL_NOW();
-    unsigned long long tl_p = tl0;
-    const MaterializeArgs& a = p.a;
-    const uint32_t tid = threadIdx.x, lane = tid & 31;
-    const uint32_t tile = blockIdx.x;
-    const uint32_t i0 = tile * kEarlySpan;
-    const uint32_t nt = (uint32_t)min((uint64_t)kEarlySpan, (uint64_t)a.n_alloc - i0);
-    const uint32_t N = a.n_nodes;
-    const uint32_t t_last = N ? __ldg(a.node_t + N - 1) : 0;
-    if (tid == 0) S.m = 0;
-    __syncthreads();
-    for (uint32_t k0 = 0; k0 < nt; k0 += kEarlyThreads * kEarlyLoads) {
-        medusa_alloc x[kEarlyLoads];
-#pragma unroll
-        for (int r = 0; r < kEarlyLoads; ++r) {
-            const uint32_t q = k0 + r * kEarlyThreads + tid;
-            x[r] = q < nt ? ld_alloc(a.alloc + i0 + q) : medusa_alloc{};
-        }
-#pragma unroll
-        for (int r = 0; r < kEarlyLoads; ++r) {
-            const uint32_t q = k0 + r * kEarlyThreads + tid;
-            const bool isI = x[r].size != 0 && N && x[r].t_alloc < t_last && t_last < x[r].t_free;
-            const uint32_t b = __ballot_sync(0xffffffffu, isI);
-            uint32_t base = 0;
-            if (lane == 0 && b) base = atomicAdd(&S.m, (uint32_t)__popc(b));
-            base = __shfl_sync(0xffffffffu, base, 0);
-            if (isI) {
-                const uint32_t pos = base + __popc(b & lanemask_lt());
-                S.k[pos] = x[r].base;
-                S.v[pos] = i0 + q;
-            }
-        }
-    }
-    __syncthreads();
-    const uint32_t m = S.m;
-    TL_PHASE(2, 30, tl_p);  // load + compaction
-    if (m <= (uint32_t)kEarlyCap) {
-        const uint32_t o = tid * kSortPer;
-        uint64_t k[kSortPer];
-        uint32_t v[kSortPer];
-#pragma unroll
-        for (int r = 0; r < kSortPer; ++r) {
-            k[r] = o + r < m ? S.k[o + r] : ~0ull;
-            v[r] = o + r < m ? S.v[o + r] : 0xFFFFFFFFu;
-        }
-        warp_bitonic_kv<kSortPer>(k, v);
-#pragma unroll 1
-        for (uint32_t run = 32 * kSortPer; run < kEarlyCap; run <<= 1) {
-            __syncthreads();  // (the first round: every thread has read its input)
-#pragma unroll
-            for (int r = 0; r < kSortPer; ++r) { S.k[o + r] = k[r]; S.v[o + r] = v[r]; }
-            __syncthreads();
-            const uint32_t a0 = o / (2 * run) * (2 * run), b0 = a0 + run;
-            const uint32_t d = o - a0;
-            uint32_t lo = d > run ? d - run : 0, hi = min(d, run);
-            while (lo < hi) {
-                const uint32_t mid = (lo + hi) >> 1;
-                const uint32_t pb = b0 + d - 1 - mid, pa = a0 + mid;
-                const uint64_t xx = S.k[pa], yy = S.k[pb];
-                if (xx < yy || (xx == yy && S.v[pa] < S.v[pb])) lo = mid + 1; else hi = mid;
-            }
-            uint32_t ia = lo, ib = d - lo;
-#pragma unroll
-            for (int r = 0; r < kSortPer; ++r) {
-                const uint32_t pa = a0 + min(ia, run - 1), pb = b0 + min(ib, run - 1);
-                const uint64_t ka = S.k[pa], kb = S.k[pb];
-                const uint32_t va = S.v[pa], vb = S.v[pb];
-                const bool takeA = ib >= run || (ia < run && kv_less(ka, va, kb, vb));
-                k[r] = takeA ? ka : kb;
-                v[r] = takeA ? va : vb;
-                if (takeA) ++ia; else ++ib;
-            }
-        }
-        __syncthreads();
-#pragma unroll
-        for (int r = 0; r < kSortPer; ++r) { S.k[o + r] = k[r]; S.v[o + r] = v[r]; }
-    } else {  // an I-dense tile: bitonic sort of the next power of two in shared memory
-        uint32_t P2 = kEarlyCap;
-        while (P2 < m) P2 <<= 1;
-        for (uint32_t q = m + tid; q < P2; q += kEarlyThreads) { S.k[q] = ~0ull; S.v[q] = 0xFFFFFFFFu; }
-        for (uint32_t size = 2; size <= P2; size <<= 1) {
-            for (uint32_t j = size >> 1; j > 0; j >>= 1) {
-                __syncthreads();
-                for (uint32_t t = tid; t < P2 / 2; t += kEarlyThreads) {
-                    const uint32_t e = 2 * j * (t / j) + (t % j), f = e + j;
-                    const bool up = (e & size) == 0;
-                    if (kv_less(S.k[f], S.v[f], S.k[e], S.v[e]) == up) {
-                        const uint64_t tk = S.k[e]; S.k[e] = S.k[f]; S.k[f] = tk;
-                        const uint32_t tv = S.v[e]; S.v[e] = S.v[f]; S.v[f] = tv;
-                    }
-                }
-            }
-        }
-    }
-    __syncthreads();
-    TL_PHASE(2, 31, tl_p);  // sort
-    const bool single = a.n_alloc <= (uint32_t)kEarlySpan;  // one tile: its order is final (nI = m)
-    for (uint32_t q = tid; q < m; q += kEarlyThreads) {
-        if (single) {
-            write_i_entry(p, q, m, S.v[q], ld_alloc(a.alloc + S.v[q]));
-        } else {
-            p.d.sk[i0 + q] = S.k[q];
-            p.d.sv[i0 + q] = S.v[q];
-            if ((q & 31) == 0) {
-                p.d.samp_k[i0 / 32 + q / 32] = S.k[q];
-                p.d.samp_v[i0 / 32 + q / 32] = S.v[q];
-            }
-            if (q + 1 == m) {
-                p.d.tmax_k[tile] = S.k[q];
-                p.d.tmax_v[tile] = S.v[q];
-            }
-        }
-    }
-    if (tid == 0) {
-        p.d.tcnt[tile] = m;
-        if (m) atomicAdd(&p.d.ctl->nI, m);
-    }
-    TL_REC(2, 0, tl0);
-    pdl_trigger();
-}
-
 // ----------------------------------------------------------------------------
 // 2b. k_rank (after k_isort, only with more than one tile): global rank of every
 //     I key = its index in its sorted tile + the count of smaller keys in every
@@ -701,28 +554,20 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
     const uint32_t nI = p.d.ctl->nI;
-    // tiles: compacted (tile t = keys [1024 t, 1024 t + 1024)) or, early, ordinal
-    // ranges of kEarlySpan allocations with their own counts (stored at t kEarlySpan)
-    const uint32_t span = p.early ? (uint32_t)kEarlySpan : (uint32_t)kIsortTile;
-    const uint32_t T = p.early ? (p.a.n_alloc + span - 1) / span : (nI + span - 1) / span;
-    auto tcount = [&](uint32_t t) { return p.early ? __ldcg(p.d.tcnt + t) : min(span, nI - t * span); };
+    const uint32_t T = (nI + kIsortTile - 1) / kIsortTile;
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    // blocks of 32 keys of one tile, grid-stride over every tile's span / 32 slots
-    // (slots past a tile's count exit at once; the grid is sized by the allocation count)
-    for (uint32_t sb = blockIdx.x; T > 1 && sb < T * (span / 32); sb += gridDim.x) {
-        const uint32_t ta = sb / (span / 32), k0 = (sb % (span / 32)) * 32;
-        const uint32_t na = tcount(ta);
-        if (k0 >= na) continue;  // (uniform over the CTA)
-        const uint32_t g = ta * span + k0 + lane;
-        const bool has = k0 + lane < na;
+    // ranges of 32 keys, grid-stride (the grid is sized by the allocation count)
+    for (uint32_t g0 = blockIdx.x * 32; T > 1 && g0 < nI; g0 += gridDim.x * 32) {
+        const uint32_t ta = g0 / kIsortTile;
+        const uint32_t g = g0 + lane;
+        const bool has = g < nI;
         const uint64_t xk = has ? __ldcg(p.d.sk + g) : ~0ull;
         const uint32_t xv = has ? __ldcg(p.d.sv + g) : 0xFFFFFFFFu;
         uint32_t cnt = 0;
         for (uint32_t tb = warp; tb < T; tb += kWarps) {
             if (tb == ta) continue;
-            const uint32_t b0 = tb * span, nb = tcount(tb);
-            if (nb == 0) continue;
-            const uint32_t ns = (nb + kSampleStride - 1) / kSampleStride;  // samples of tile tb
+            const uint32_t b0 = tb * kIsortTile, nb = min((uint32_t)kIsortTile, nI - b0);
+            const uint32_t ns = (nb + kSampleStride - 1) / kSampleStride;  // samples of tile tb (<= 64)
             const uint32_t s0 = b0 / kSampleStride;
             {  // the tile's key range: lanes below its least key count 0, above its greatest nb
                 const uint64_t mnk = __ldcg(p.d.samp_k + s0), mxk = __ldcg(p.d.tmax_k + tb);
@@ -733,17 +578,6 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
                     cnt += above ? nb : 0u;
                     continue;
                 }
-            }
-            if (ns > 64) {  // (an I-dense early tile) every lane searches the tile in memory
-                uint32_t lo = 0, hi = has ? nb : 0;
-                while (lo < hi) {
-                    const uint32_t mid = (lo + hi) >> 1;
-                    const uint64_t bk = __ldcg(p.d.sk + b0 + mid);
-                    const bool lt = bk < xk || (bk == xk && __ldcg(p.d.sv + b0 + mid) < xv);
-                    if (lt) lo = mid + 1; else hi = mid;
-                }
-                cnt += lo;
-                continue;
             }
             uint64_t sk0 = ~0ull, sk1 = ~0ull;
             uint32_t sv0 = 0xFFFFFFFFu, sv1 = 0xFFFFFFFFu;
@@ -791,7 +625,7 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
         s_cnt[warp][lane] = cnt;
         __syncthreads();
         if (warp == 0 && has) {
-            uint32_t rank = k0 + lane;  // index inside its own tile
+            uint32_t rank = g - ta * kIsortTile;  // index inside its own tile
 #pragma unroll
             for (int w = 0; w < kWarps; ++w) rank += s_cnt[w][lane];
             write_i_entry(p, rank, nI, xv, ld_alloc(p.a.alloc + xv));
@@ -1761,8 +1595,8 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
     s.d.tree.node = (uint2*)(z + o);
     if ((e = grow(s, s.d.jf, CC)) || (e = grow(s, s.d.jl, CC)) || (e = grow(s, s.d.tree.leaf, N)) || (e = grow(s, s.d.tree.leaf_be, N)) ||
         (e = grow(s, s.d.sk0, N + kThreads)) || (e = grow(s, s.d.sv0, N + kThreads)) || (e = grow(s, s.d.sk, N)) ||
-        (e = grow(s, s.d.sv, N)) || (e = grow(s, s.d.icnt, N / kThreads + 2)) || (e = grow(s, s.d.tcnt, N / kEarlySpan + 2)) ||
-        (e = grow(s, s.d.tmax_k, N / 1024 + 2)) || (e = grow(s, s.d.tmax_v, N / 1024 + 2)) ||
+        (e = grow(s, s.d.sv, N)) || (e = grow(s, s.d.icnt, N / kThreads + 2)) ||
+        (e = grow(s, s.d.tmax_k, N / kIsortTile + 2)) || (e = grow(s, s.d.tmax_v, N / kIsortTile + 2)) ||
         (e = grow(s, s.d.samp_k, N / kSampleStride + 64)) || (e = grow(s, s.d.samp_v, N / kSampleStride + 64)) ||
         (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
         (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
@@ -1798,7 +1632,6 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
         cudaFuncSetAttribute(k_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kClsSmem);
         cudaFuncSetAttribute(k_isort, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)(kIsortSmem + (kOrderedCtas + 1) * 4));
-        cudaFuncSetAttribute(k_isort_early, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kEarlySmem);
         int prio_lo = 0, prio_hi = 0;
         cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
         if ((*e = cudaStreamCreateWithPriority(&s.side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
@@ -1837,12 +1670,8 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     // ordinal-ordered I compaction pays when the set spans several address regions
     // (several models: most rank tiles then hold another model's keys); a single
     // model's set (<= 128 k_trace CTAs, ~4 tiles) skips the gather it costs k_isort
-#ifndef MEDUSA_EARLY_ISORT
-#define MEDUSA_EARLY_ISORT 0
-#endif
-    const uint32_t early = MEDUSA_EARLY_ISORT ? 1u : 0u;
-    const uint32_t ordered = (!early && alloc_ctas > 128 && alloc_ctas <= kOrderedCtas) ? 1u : 0u;
-    P p{a, d, C, nb, node_ctas, alloc_ctas, ordered, early};
+    const uint32_t ordered = (alloc_ctas > 128 && alloc_ctas <= kOrderedCtas) ? 1u : 0u;
+    P p{a, d, C, nb, node_ctas, alloc_ctas, ordered};
     *out = p;
     cudaError_t e;
     // branches (serialized on the caller's stream while per-launch timing is on)
@@ -1850,23 +1679,17 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     cudaStream_t side = serial ? stream : s.side, low = serial ? stream : s.low;
     if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) return e;
     if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) return e;
-    if (n && early) {  // the I-list sort reads only the inputs: beside k_trace
-        if ((e = cudaEventRecord(s.fork, stream)) || (e = cudaStreamWaitEvent(side, s.fork, 0))) return e;
-        TimedLaunch tl("mat_isort", side);
-        k_isort_early<<<(unsigned)((n + kEarlySpan - 1) / kEarlySpan), kEarlyThreads, kEarlySmem, side>>>(p);
-    }
     {
         TimedLaunch tl("mat_trace", stream);
         k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
     }
     if (n) {
-        if ((e = cudaEventRecord(s.traced, stream))) return e;
-        if (!early) {
-            if ((e = cudaStreamWaitEvent(side, s.traced, 0))) return e;
+        if ((e = cudaEventRecord(s.traced, stream)) || (e = cudaStreamWaitEvent(side, s.traced, 0))) return e;
+        {
             TimedLaunch tl("mat_isort", side);
             k_isort<<<sort_ctas, kIsortThreads, kIsortSmem + (ordered ? (alloc_ctas + 1) * 4 : 0), side>>>(p);
         }
-        if (n > (uint64_t)(early ? kEarlySpan : kIsortTile)) {  // (with one tile the sort writes the I list itself)
+        if (n > (uint64_t)kIsortTile) {  // (with one tile k_isort writes the I list itself)
             TimedLaunch tl("mat_rank", side);
             // one CTA per 32 I keys (the list's size is known on the device only: bound
             // by the allocation count; surplus CTAs exit at once)
