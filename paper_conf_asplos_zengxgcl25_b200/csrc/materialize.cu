@@ -1310,12 +1310,13 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 // ----------------------------------------------------------------------------
 // 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
 //     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
-//     CTA; warp w takes the queue range classify's warp w filled.  Per candidate
-//     one group of bases and one entry (two dependent loads); a hit writes its
-//     record over its queue entry's word and sets its bit in the mask and in the
-//     I-resolved mask; the chunk's count grows by
-//     one atomic per warp (no CTA barrier: the warps run through the chunks
-//     independently).
+//     CTA; the chunk's eight queue ranges (one per classify warp) are spread over
+//     the whole CTA (entry i of their concatenation -> thread i mod 256: a long
+//     range no longer sets the chunk's time; per-warp ranges measured ALL10
+//     iresolve 16.0 vs 13.8 us span).  Per candidate one group of bases and one
+//     entry (two dependent loads); a hit writes its record over its queue
+//     entry's word and sets its bit in the mask and in the I-resolved mask; the
+//     chunk's count grows by one atomic per warp.
 __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
     const unsigned long long tl0 = TL_NOW();
@@ -1323,18 +1324,39 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
     const uint32_t nI = p.d.ctl->nI;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (nI) {
+        // the chunk's queue ranges (one per classify warp) taken by the whole CTA:
+        // entry i of the chunk's concatenated ranges -> thread i mod 256, so a warp
+        // whose range is long (up to cap_pw entries) does not set the chunk's time
+        __shared__ uint32_t s_pre[kWarps + 1];
         const uint32_t stride = fence_stride(nI);
         const uint32_t nf = (nI + stride - 1) / stride;
+        const uint32_t cap = p.d.cap_pw;
         for (uint32_t f = tid; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
-        __syncthreads();
+        uint32_t my_cnt = (blockIdx.x < p.C && tid < kWarps) ? min(__ldcg(p.d.qcnt + blockIdx.x * kWarps + tid), cap) : 0u;
         for (uint32_t c = blockIdx.x; c < p.C; c += gridDim.x) {
-            const uint32_t nq = __ldcg(p.d.qcnt + c * kWarps + warp);
-            const uint32_t q0 = (c * kWarps + warp) * p.d.cap_pw;
+            if (warp == 0) {  // exclusive prefix of the 8 range lengths
+                uint32_t incl = lane < kWarps ? my_cnt : 0u;
+#pragma unroll
+                for (int d = 1; d < kWarps; d <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+                    if (lane >= (uint32_t)d) incl += y;
+                }
+                if (lane < kWarps) s_pre[lane + 1] = incl;
+                if (lane == 0) s_pre[0] = 0;
+            }
+            __syncthreads();  // (also: the fences, on the first chunk)
+            const uint32_t cn = c + gridDim.x;  // the next chunk's counts, loaded early
+            if (tid < kWarps) my_cnt = cn < p.C ? min(__ldcg(p.d.qcnt + cn * kWarps + tid), cap) : 0u;
+            const uint32_t total = s_pre[kWarps];
             uint32_t cnt = 0;
-            for (uint32_t i0 = 0; i0 < nq; i0 += 32) {
-                const uint32_t k = q0 + i0 + lane;
+            for (uint32_t i0 = 0; i0 < total; i0 += kThreads) {
+                const uint32_t i = i0 + tid;
                 bool hit = false;
-                if (i0 + lane < nq) {
+                if (i < total) {
+                    uint32_t w = 0;  // the range holding entry i
+#pragma unroll
+                    for (int r = 1; r < kWarps; ++r) w += s_pre[r] <= i ? 1u : 0u;
+                    const uint64_t k = (uint64_t)(c * kWarps + w) * cap + (i - s_pre[w]);
                     const IQ q = p.d.queue[k];
                     const uint32_t le = i_count_le(s_fence, nf, stride, nI, p.d.i_base, q.x);
                     if (le) {
@@ -1350,11 +1372,11 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                 }
                 cnt += __popc(__ballot_sync(0xffffffffu, hit));
             }
-            // per-warp counts (no CTA barrier: the warps run ahead independently)
             if (lane == 0 && cnt) {
                 atomicAdd(p.d.chunk_cnt + c, cnt);
                 atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)cnt);
             }
+            __syncthreads();  // s_pre is rewritten for the next chunk
         }
     }
     pdl_trigger();
@@ -1376,6 +1398,7 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     __shared__ uint32_t s_pre[kEmitChunks][65], s_prm[kEmitChunks][65], s_prq[kEmitChunks][65];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
+    if (MEDUSA_EARLY_TRIGGER) pdl_trigger();  // k_result waits for this grid's completion
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t c0 = blockIdx.x * kEmitChunks;
@@ -1475,15 +1498,16 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
         for (uint32_t r = tid + kRecPerThread * kThreads; r < total[h]; r += kThreads)
             if (pf + r < a.capacity) a.slot[pf + r] = source(h, r);
     }
-    pdl_trigger();
+    if (!MEDUSA_EARLY_TRIGGER) pdl_trigger();
     TL_REC(5, 0, tl0);
 }
 
 // ----------------------------------------------------------------------------
 // 6. k_result (async entry): the outcome as a medusa_mat_result
 __global__ void k_result(P p, medusa_mat_result* r) {
+    if (MEDUSA_EARLY_TRIGGER) pdl_trigger();
     pdl_wait();
-    pdl_trigger();
+    if (!MEDUSA_EARLY_TRIGGER) pdl_trigger();
     const Ctl& c = *p.d.ctl;
     int32_t st = MEDUSA_OK;
     if (c.status & ST_INVALID) st = MEDUSA_ERR_INVALID_ARG;

@@ -46,8 +46,9 @@ MEDUSA_TL_DEFINE
 
 __global__ void report_init(medusa_report* r) {
     const unsigned long long tl0 = TL_NOW();
+    if (MEDUSA_EARLY_TRIGGER) pdl_trigger();  // (the restore waits before it reads the table)
     pdl_wait();  // the previous user of the report may still read it
-    pdl_trigger();
+    if (!MEDUSA_EARLY_TRIGGER) pdl_trigger();
     r->n_bad_slot = 0;
     r->first_bad_word = ~0ull;
     r->n_bad_id = 0;
@@ -290,6 +291,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         }
         if (!tma)
             for (uint32_t q = tid; q < n; q += kThreads) s_words[q] = ld_stream(gsrc + q);
+        pdl_wait();  // the table (the previous kernels' output) and the report are ready
         table_load<CPB>(a, task, T);
         TL_PHASE(7, 10, tl_p);  // mask + record range loaded
         // 2. popcount prefix and consistency (warp 0) while the other warps load the
@@ -390,7 +392,6 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
             for (uint32_t q = tid; q < n; q += kThreads) st_stream(gdst + q, s_words[q]);
         }
         TL_PHASE(7, 13, tl_p);  // bulk store issued and read out of shared memory
-        pdl_wait();  // report_init (this launch's PDL predecessor) has run
         pdl_trigger();
         report_add(rep, n_id, n_rg, n_st, first, tid == 0 ? __popc(kAllOk & ~T.ok) : 0u);
         TL_REC(7, 0, tl0);
@@ -422,6 +423,7 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     const unsigned long long tl0 = TL_NOW();
     if (task < n_word_tasks) {
         const uint64_t ws = (uint64_t)task * kWords;
+        pdl_wait();  // the table (the previous kernels' output) and the report are ready
         table_load<CPB>(a, task, T);
         if (tid < 32) table_prefix<CPB>(T);
         const uint32_t cb0 = T.cb[0];
@@ -483,7 +485,6 @@ restore_inplace_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 if (bad) first = min(first, ws + q);
             }
         }
-        pdl_wait();
         pdl_trigger();
         report_add(rep, n_id, n_rg, n_st, first, tid == 0 ? __popc(kAllOk & ~T.ok) : 0u);
         TL_REC(7, 2, tl0);
