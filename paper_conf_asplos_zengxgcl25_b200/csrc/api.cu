@@ -1,5 +1,6 @@
 // C-ABI entry points of libmedusa.so (include/medusa.h): argument checks,
 // per-device kernel-address tables, status / error plumbing, instrumentation.
+#include <algorithm>
 #include <mutex>
 #include <vector>
 
@@ -166,6 +167,21 @@ medusa_status medusa_materialize_async(const uint64_t* d_words, uint64_t n_words
     return st;
 }
 
+#ifndef MEDUSA_TABLE_KERNEL
+#define MEDUSA_TABLE_KERNEL 1
+#endif
+namespace medusa {
+// the kernel-address table copy as a kernel: in a captured step a kernel node
+// starts sooner than a copy-engine memcpy node, and the analysis that follows
+// may start beside it (it triggers at once; the restore, two launches on, is
+// the first kernel that reads the table)
+static __global__ void k_table_copy(uint64_t* dst, const uint64_t* src, uint32_t n) {
+    medusa::pdl_wait();  // the previous user of the table
+    medusa::pdl_trigger();
+    for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += gridDim.x * blockDim.x) dst[k] = src[k];
+}
+}  // namespace medusa
+
 medusa_status medusa_kernel_table_set(const uint64_t* d_func_addr, uint32_t n_func, cudaStream_t stream) {
     if (n_func > 0 && (!d_func_addr || !aligned8(d_func_addr))) return MEDUSA_ERR_INVALID_ARG;
     int dev = 0;
@@ -186,8 +202,14 @@ medusa_status medusa_kernel_table_set(const uint64_t* d_func_addr, uint32_t n_fu
         t.capacity = cap;
     }
     if (n_func > 0) {
-        e = cudaMemcpyAsync(t.d_table, d_func_addr, (size_t)n_func * sizeof(uint64_t), cudaMemcpyDeviceToDevice,
-                            stream);
+        if (MEDUSA_TABLE_KERNEL) {
+            medusa::TimedLaunch tl("table_copy", stream);
+            e = medusa::launch_pdl(medusa::k_table_copy, std::min<uint32_t>((n_func + 255) / 256, 148u), 256, 0, stream, t.d_table,
+                                   d_func_addr, n_func);
+        } else {
+            e = cudaMemcpyAsync(t.d_table, d_func_addr, (size_t)n_func * sizeof(uint64_t), cudaMemcpyDeviceToDevice,
+                                stream);
+        }
         if (e != cudaSuccess) return cuda_fail(e);
     }
     t.n_func = n_func;

@@ -199,6 +199,18 @@ __device__ __forceinline__ medusa_alloc ld_alloc(const medusa_alloc* q) {
 
 
 // ----------------------------------------------------------------------------
+// 0. k_zero: the call's zeroed scratch (counters, check summaries, tree nodes) as
+//    the first kernel, so that k_trace is its programmatic successor: k_trace's
+//    CTAs load their records while it runs (a memset node measured ~2 us more
+//    in front of the first CTA)
+__global__ void __launch_bounds__(kThreads) k_zero(uint4* z, size_t n16) {
+    pdl_trigger();
+    pdl_wait();  // (launched programmatically: the previous call's last kernels may still read the scratch)
+    for (size_t k = (size_t)blockIdx.x * kThreads + threadIdx.x; k < n16; k += (size_t)gridDim.x * kThreads)
+        z[k] = make_uint4(0u, 0u, 0u, 0u);
+}
+
+// ----------------------------------------------------------------------------
 // 1. k_trace
 __device__ void nodes_role(const P& p, uint64_t i) {
     const MaterializeArgs& a = p.a;
@@ -242,6 +254,7 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
     const uint32_t t_last = N ? __ldg(a.node_t + N - 1) : 0;
     uint32_t ta_next = __shfl_down_sync(0xffffffffu, x.t_alloc, 1);  // the next ordinal's t_alloc
     if (lane == 31 && i + 1 < a.n_alloc) ta_next = (uint32_t)__ldg(reinterpret_cast<const unsigned long long*>(a.alloc + i + 1) + 2);
+    pdl_wait();  // (k_zero: the counters and tree nodes below are zero)
     bool isI = false;
     uint32_t v = 0;  // leaf value: t_free of a mortal, else 0
     if (valid) {
@@ -315,11 +328,11 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
 
 __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
     const unsigned long long tl0 = TL_NOW();
-    pdl_wait();
     // k_classify's CTAs may start in the slots this grid leaves free and issue
     // their word copies; they read nothing of this grid before griddepcontrol.wait
     pdl_trigger();
     if (blockIdx.x < p.node_ctas) {  // kNodesPerThread nodes per thread, CTA-strided
+        pdl_wait();  // (k_zero)
 #pragma unroll
         for (int k = 0; k < kNodesPerThread; ++k)
             nodes_role(p, ((uint64_t)blockIdx.x * kNodesPerThread + k) * blockDim.x + threadIdx.x);
@@ -1404,17 +1417,21 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     const uint32_t c0 = blockIdx.x * kEmitChunks;
     const uint32_t nch = min((uint32_t)kEmitChunks, p.C - c0);
     const uint64_t n_mask = (a.n_words + 31) / 32;
-    // the first chunk's first slot: the sum of the slot counts of all earlier chunks
-    uint64_t prefix = block_prefix(p.d.chunk_cnt, p.d.chunk_sup, c0);
+    // the mask words (warps 0-3, one per lane), the chunks' counts and (in the same
+    // load round) the first chunk's first slot: the sum of the slot counts of all
+    // earlier chunks
+    const uint32_t h_m = warp >> 1;
+    const uint64_t mw_m = (uint64_t)(c0 + h_m) * (kChunkWords / 32) + (warp & 1) * 32 + lane;
+    const bool in_m = warp < 2 * kEmitChunks && h_m < nch && mw_m < n_mask;
+    const uint32_t mv_m = in_m ? __ldcg(a.mask + mw_m) : 0u, iv_m = in_m ? __ldcg(p.d.imask + mw_m) : 0u;
+    const uint32_t qv_m = in_m ? __ldcg(p.d.qmask + mw_m) : 0u;
     uint32_t total[kEmitChunks];
 #pragma unroll
     for (int h = 0; h < kEmitChunks; ++h) total[h] = (uint32_t)h < nch ? __ldcg(p.d.chunk_cnt + c0 + h) : 0u;
+    uint64_t prefix = block_prefix(p.d.chunk_cnt, p.d.chunk_sup, c0);
     if (warp < 2 * kEmitChunks) {  // popcount prefixes of each half of each chunk's 64 mask words
-        const uint32_t h = warp >> 1, half = warp & 1;
-        const uint64_t mw = (uint64_t)(c0 + h) * (kChunkWords / 32) + half * 32 + lane;
-        const bool in = h < nch && mw < n_mask;
-        const uint32_t mv = in ? __ldcg(a.mask + mw) : 0u, iv = in ? __ldcg(p.d.imask + mw) : 0u;
-        const uint32_t qv = in ? __ldcg(p.d.qmask + mw) : 0u;
+        const uint32_t h = h_m, half = warp & 1;
+        const uint32_t mv = mv_m, iv = iv_m, qv = qv_m;
         const uint32_t x = half * 32 + lane;
         s_m[h][x] = mv;
         s_i[h][x] = iv;
@@ -1605,7 +1622,7 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
     // zero region: Ctl | chunk_sup [CC/256+1] (u64) | blk_min_ta_c blk_max_tf [NS] | chunk_cnt [CC] |
     //              tree nodes [NT] (uint2)
     const size_t GC = CC / 256 + 1;
-    s.zero_bytes = 256 + GC * 8 + 2 * NS * 4 + CC * 4 + 64 + NT * 8;
+    s.zero_bytes = (256 + GC * 8 + 2 * NS * 4 + CC * 4 + 64 + NT * 8 + 15) & ~(size_t)15;
     if ((e = cudaMalloc(&s.zero_region, s.zero_bytes)) != cudaSuccess) return e;
     s.bytes += s.zero_bytes;
     char* z = (char*)s.zero_region;
@@ -1701,9 +1718,22 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     // branches (serialized on the caller's stream while per-launch timing is on)
     const bool serial = timing_enabled();
     cudaStream_t side = serial ? stream : s.side, low = serial ? stream : s.low;
-    if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) return e;
+#ifndef MEDUSA_ZERO_KERNEL
+#define MEDUSA_ZERO_KERNEL 1
+#endif
     if (C == 0 && (e = cudaMemsetAsync(a.chunk_base, 0, sizeof(uint32_t), stream)) != cudaSuccess) return e;
-    {
+    if (MEDUSA_ZERO_KERNEL) {
+        const size_t n16 = s.zero_bytes / 16;  // (zero_bytes: a multiple of 16)
+        {
+            TimedLaunch tl("mat_zero", stream);
+            if ((e = launch_pdl(k_zero, (unsigned)std::min<size_t>((n16 + kThreads - 1) / kThreads, (size_t)s.sm_count * 2),
+                                kThreads, 0, stream, reinterpret_cast<uint4*>(s.zero_region), n16)))
+                return e;
+        }
+        TimedLaunch tl("mat_trace", stream);
+        if ((e = launch_pdl(k_trace, node_ctas + alloc_ctas, kThreads, 0, stream, p))) return e;
+    } else {
+        if ((e = cudaMemsetAsync(s.zero_region, 0, s.zero_bytes, stream)) != cudaSuccess) return e;
         TimedLaunch tl("mat_trace", stream);
         k_trace<<<node_ctas + alloc_ctas, kThreads, 0, stream>>>(p);
     }

@@ -11,7 +11,7 @@ import sys
 NAMES = {"k_classify": "mat_classify", "restore_kernel": "restore", "k_trace": "mat_trace", "k_isort": "mat_isort",
          "report_init": "restore_report_init", "k_result": "mat_result",
          "k_prepare": "mat_prepare", "k_rank": "mat_rank", "k_check_mi": "mat_check_mi",
-         "k_check_mm": "mat_check_mm", "k_check": "mat_check", "k_iresolve": "mat_iresolve", "k_emit": "mat_emit",
+         "k_check_mm": "mat_check_mm", "k_check": "mat_check", "k_iresolve": "mat_iresolve", "k_emit": "mat_emit", "k_zero": "mat_zero",
          "restore_inplace_kernel": "restore_inplace", "k_buf_copy<true>": "buf_save", "k_buf_copy<false>": "buf_restore"}
 rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 10]
 h = rows[0]
