@@ -44,14 +44,13 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 // it touches anything the predecessor writes.  Most kernels call pdl_trigger()
 // only after their own pdl_wait(), so "my predecessor has triggered" implies
 // "everything before my predecessor is complete" and a kernel may read the
-// outputs of kernels two or more launches back before it waits (k_buf_copy,
-// restore's gather role, classify's word copy).  With MEDUSA_EARLY_TRIGGER the
+// outputs of kernels two or more launches back before it waits (k_buf_copy).  With MEDUSA_EARLY_TRIGGER the
 // tail of a call -- k_emit, k_result, report_init -- triggers at its start, so
 // each successor is resident and waiting when its predecessor completes; the
 // restore then reads nothing a kernel of the stream wrote before its own
-// pdl_wait() (it reads the table after it; before it only its inputs: the
-// image words, the kernel ids and the kernel table).  (ALL10 / C5 step -0.2 /
-// -0.4 us: measured, kept.)
+// pdl_wait() (the slot table and the kernel table after it; before it only its
+// inputs: the image words and the kernel ids).  (ALL10 / C5 step -0.2 / -0.4
+// us: measured, kept.)
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 #ifndef MEDUSA_EARLY_TRIGGER
 #define MEDUSA_EARLY_TRIGGER 1

@@ -204,8 +204,11 @@ __device__ __forceinline__ medusa_alloc ld_alloc(const medusa_alloc* q) {
 //    CTAs load their records while it runs (a memset node measured ~2 us more
 //    in front of the first CTA)
 __global__ void __launch_bounds__(kThreads) k_zero(uint4* z, size_t n16) {
+    // launched programmatically: the previous kernels (the last of an earlier call
+    // may still read this scratch; one may have written the image) complete first,
+    // then k_trace and k_classify may start and read the inputs
+    pdl_wait();
     pdl_trigger();
-    pdl_wait();  // (launched programmatically: the previous call's last kernels may still read the scratch)
     for (size_t k = (size_t)blockIdx.x * kThreads + threadIdx.x; k < n16; k += (size_t)gridDim.x * kThreads)
         z[k] = make_uint4(0u, 0u, 0u, 0u);
 }

@@ -71,13 +71,23 @@ __device__ __forceinline__ void gather_role(const RestoreArgs& a, uint32_t gt, u
     const uint64_t j0 = (uint64_t)gt * kNodesPerTask;
     uint32_t n_bad = 0;
     uint64_t first = ~0ull;
+    constexpr int kPer = kNodesPerTask / kThreads;
+    uint32_t f[kPer];
 #pragma unroll
-    for (int k = 0; k < kNodesPerTask / kThreads; ++k) {
+    for (int k = 0; k < kPer; ++k) {  // the kernel ids (an input) before the wait
+        const uint64_t j = j0 + tid + k * kThreads;
+        f[k] = j < a.n_nodes ? a.func_id[j] : 0u;
+    }
+    // the kernel table may have been written by a kernel two or more launches back
+    // (k_table_copy; the tail of a call triggers its successors early: common.cuh)
+    pdl_wait();
+    pdl_trigger();
+#pragma unroll
+    for (int k = 0; k < kPer; ++k) {
         const uint64_t j = j0 + tid + k * kThreads;
         if (j < a.n_nodes) {
-            const uint32_t f = a.func_id[j];
             uint64_t addr = 0;
-            if (f < a.n_func) addr = __ldg(a.table + f);
+            if (f[k] < a.n_func) addr = __ldg(a.table + f[k]);
             if (addr == 0) {
                 ++n_bad;
                 first = min(first, j);
@@ -85,8 +95,6 @@ __device__ __forceinline__ void gather_role(const RestoreArgs& a, uint32_t gt, u
             a.func_out[j] = addr;
         }
     }
-    pdl_wait();
-    pdl_trigger();
     if (n_bad) {
         atomicAdd(rep + 5, (unsigned long long)n_bad);
         atomicMin(rep + 6, (unsigned long long)first);
