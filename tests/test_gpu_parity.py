@@ -365,6 +365,61 @@ def test_async_graph_path_parity(graph_sets, name):
         assert np.array_equal(medusa.report_numpy(rep), packed[5])
 
 
+@pytest.mark.parametrize("name", ["toy", "llama2-13b"])
+def test_stream_ordered_chain_without_host_sync(graph_sets, name):
+    """In-place restore -> materialize_async of the restored image against the
+    replayed trace -> kernel_table_set -> restore of that table, enqueued on one
+    stream with no host synchronisation, five rounds: every programmatic launch
+    (k_table_copy, k_zero, the early-triggering tail of each call) must order a
+    read after the write it depends on.  Against the oracle run on the same chain."""
+    gs = graph_sets(name)
+    inp = medusa.upload(gs, DEV)
+    slots = medusa.materialize(inp["words"], inp["node_off"], inp["node_t"], inp["allocs"])
+    m1, p1 = _oracle_full(gs.words, gs.node_word_off, gs.node_t, gs.allocs, gs.new_base, gs.new_size,
+                          gs.func_id, gs.table)
+    allocs2 = gs.allocs.copy()
+    allocs2["base"] = gs.new_base  # the replayed trace: the restored image's pointers live here
+    new_base2 = gs.new_base + np.uint64(1 << 36)
+    table2 = gs.table.copy()
+    table2[table2 != 0] += np.uint64(4096)
+    m2, p2 = _oracle_full(p1[3], gs.node_word_off, gs.node_t, allocs2, new_base2, gs.new_size, gs.func_id, table2)
+    assert m2["status"] == 0
+    t64 = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int64)).to(DEV)  # noqa: E731
+    allocs2_t = torch.from_numpy(np.ascontiguousarray(allocs2).view(np.int64).reshape(-1, 3)).to(DEV)
+    nb2, tab2 = t64(new_base2), t64(table2)
+    buf = torch.empty_like(inp["words"])
+    dst2 = torch.empty_like(inp["words"])
+    f1 = torch.empty(gs.n_nodes, dtype=torch.int64, device=DEV)
+    f2 = torch.empty_like(f1)
+    rep1 = torch.empty(8, dtype=torch.int64, device=DEV)
+    rep2 = torch.empty_like(rep1)
+    res = torch.empty(2, dtype=torch.int64, device=DEV)
+    slots2 = medusa.alloc_slots(gs.n_words, DEV)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for _ in range(5):
+            buf.copy_(inp["words"])
+            dst2.fill_(-1)
+            medusa.kernel_table_set(inp["table"])
+            medusa.restore(buf, slots, inp["old_base"], inp["new_base"], inp["new_size"], inp["func_id"], dst=buf,
+                           func_out=f1, report=rep1)
+            medusa.materialize_async(buf, inp["node_off"], inp["node_t"], allocs2_t, out=slots2, result=res)
+            medusa.kernel_table_set(tab2)
+            medusa.restore(buf, slots2, inp["new_base"], nb2, inp["new_size"], inp["func_id"], dst=dst2, func_out=f2,
+                           report=rep2, from_table=True)
+    torch.cuda.synchronize()
+    assert np.array_equal(medusa.to_numpy_u64(buf), p1[3])
+    assert np.array_equal(medusa.to_numpy_u64(f1), p1[4])
+    assert np.array_equal(medusa.report_numpy(rep1), p1[5])
+    assert medusa.mat_result(res) == (0, m2["n_slots"])
+    slots2.n_slots = m2["n_slots"]
+    _check_materialize(slots2, m2, p2, gs.n_words)
+    assert np.array_equal(medusa.to_numpy_u64(dst2), p2[3])
+    assert np.array_equal(medusa.to_numpy_u64(f2), p2[4])
+    assert np.array_equal(medusa.report_numpy(rep2), p2[5])
+
+
 def test_async_reports_trace_error_and_capacity():
     """The async entry point reports what the synchronous one raises, in the result word."""
     t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a).view(dt)).to(DEV)
