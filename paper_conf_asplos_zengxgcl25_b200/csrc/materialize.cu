@@ -215,26 +215,27 @@ __global__ void __launch_bounds__(kThreads) k_zero(uint4* z, size_t n16) {
 
 // ----------------------------------------------------------------------------
 // 1. k_trace
-__device__ void nodes_role(const P& p, uint64_t i) {
+// node i of the CSR (o0 = node_off[i], o1 = node_off[i + 1], t0 / t1 = the launch
+// positions of nodes i and i + 1): the CSR / launch-order checks and the chunks
+// whose first or last word it holds
+__device__ __forceinline__ void nodes_role(const P& p, uint64_t i, uint64_t o0, uint64_t o1, uint32_t t0, uint32_t t1) {
     const MaterializeArgs& a = p.a;
     const uint32_t N = a.n_nodes;
     if (i > N) return;
-    const uint64_t o0 = a.node_off[i];
     if (i == 0 && o0 != 0) flag(p.d.ctl, ST_INVALID);
     if (i == N) {
         if (o0 != a.n_words) flag(p.d.ctl, ST_INVALID);
         return;
     }
-    const uint64_t o1 = a.node_off[i + 1];
     if (o1 < o0) { flag(p.d.ctl, ST_INVALID); return; }
-    if (i + 1 < N && !(a.node_t[i] < a.node_t[i + 1])) flag(p.d.ctl, ST_INVALID);
+    if (i + 1 < N && !(t0 < t1)) flag(p.d.ctl, ST_INVALID);
     if (o1 == o0 || o1 > a.n_words) return;
     // node i writes the chunks whose first or last word it holds
     for (uint64_t c = o0 / kChunkWords; c <= (o1 - 1) / kChunkWords; ++c) {
         const uint64_t cs = c * kChunkWords;
         const uint64_t ce = min(cs + kChunkWords, a.n_words) - 1;
-        if (o0 <= cs) p.d.jf[c] = make_uint2((uint32_t)i, a.node_t[i]);
-        if (ce < o1) p.d.jl[c] = make_uint2((uint32_t)i, a.node_t[i]);
+        if (o0 <= cs) p.d.jf[c] = make_uint2((uint32_t)i, t0);
+        if (ce < o1) p.d.jl[c] = make_uint2((uint32_t)i, t0);
     }
 }
 
@@ -335,10 +336,23 @@ __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
     // their word copies; they read nothing of this grid before griddepcontrol.wait
     pdl_trigger();
     if (blockIdx.x < p.node_ctas) {  // kNodesPerThread nodes per thread, CTA-strided
+        // every node's offsets and launch positions loaded in one round, then the checks
+        const uint32_t N = p.a.n_nodes;
+        uint64_t o0[kNodesPerThread], o1[kNodesPerThread];
+        uint32_t t0[kNodesPerThread], t1[kNodesPerThread];
+#pragma unroll
+        for (int k = 0; k < kNodesPerThread; ++k) {
+            const uint64_t i = ((uint64_t)blockIdx.x * kNodesPerThread + k) * blockDim.x + threadIdx.x;
+            o0[k] = i <= N ? __ldg(p.a.node_off + i) : 0ull;
+            o1[k] = i < N ? __ldg(p.a.node_off + i + 1) : 0ull;
+            t0[k] = i < N ? __ldg(p.a.node_t + i) : 0u;
+            t1[k] = i + 1 < N ? __ldg(p.a.node_t + i + 1) : 0u;
+        }
         pdl_wait();  // (k_zero)
 #pragma unroll
         for (int k = 0; k < kNodesPerThread; ++k)
-            nodes_role(p, ((uint64_t)blockIdx.x * kNodesPerThread + k) * blockDim.x + threadIdx.x);
+            nodes_role(p, ((uint64_t)blockIdx.x * kNodesPerThread + k) * blockDim.x + threadIdx.x, o0[k], o1[k], t0[k],
+                       t1[k]);
         TL_REC(1, 0, tl0);
     } else {
         allocs_role(p, blockIdx.x - p.node_ctas);
