@@ -36,7 +36,10 @@ for tool in racecheck synccheck; do
   tail -3 gpurun_out/sanitizer_${tool}_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
 done
 # initcheck tracks every byte: the small sets, one ALL10 full path, in place, the table cases
-timeout 1800 compute-sanitizer --tool initcheck --report-api-errors no --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py -m gpu -x -q -k "full_path_parity and (toy or llama2-13b) or in_place_full_path or fault or edge or capacity or hand_derived or overflow" > gpurun_out/sanitizer_initcheck_$TAG.log 2>&1
-echo "initcheck (small sets, ALL10 full path, in place, faults, tables, overflow) exit=$?" >> gpurun_out/sanitizer_summary_$TAG.txt
+# (--check-api-memory-access no: restore writes its output with TMA bulk stores, which initcheck does not
+#  track, so every host copy of a restored image would be reported; tests/test_gpu_parity.py
+#  test_restore_writes_every_word shows with sentinel-filled destinations that every word is written)
+timeout 1800 compute-sanitizer --tool initcheck --check-api-memory-access no --report-api-errors no --error-exitcode 9 python -m pytest tests/test_gpu_parity.py tests/test_gpu_table.py -m gpu -x -q -p no:cacheprovider -k "(full_path_parity and toy) or (in_place_full_path and toy) or fault or edge_cases or capacity or hand or (chain and toy)" > gpurun_out/sanitizer_initcheck_$TAG.log 2>&1
+echo "initcheck (small sets: toy full path, in place, faults, edge cases, capacity, tables, tiny traces, the stream chain) exit=$?" >> gpurun_out/sanitizer_summary_$TAG.txt
 tail -3 gpurun_out/sanitizer_initcheck_$TAG.log >> gpurun_out/sanitizer_summary_$TAG.txt
 cat gpurun_out/sanitizer_summary_$TAG.txt
