@@ -31,7 +31,9 @@ NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan
          (4, 10): " cls:A setup", (4, 11): " cls:B starts+cand", (4, 12): " cls:D query", (4, 13): " cls:D live+search",
          (4, 14): " cls:E queue", (4, 15): " cls:E records+queue", (4, 16): " cls:win-load", (4, 17): " cls:sort",
          (7, 2): "restore/in-place", (7, 10): " res:mask+range", (7, 11): " res:records+gathers",
-         (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store"}
+         (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store",
+         (10, 50): " ires:fences+prefix", (10, 51): " ires:queue entry", (10, 52): " ires:fence search+group",
+         (10, 53): " ires:entry+mask"}
 REC = np.dtype([("t0", "<u8"), ("t1", "<u8"), ("kernel", "<u4"), ("cta", "<u4"), ("sm", "<u4"), ("tag", "<u4")])
 
 

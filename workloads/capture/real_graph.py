@@ -629,7 +629,11 @@ def online(torch, medusa, in_dir, arena_bytes=1 << 30):
     if L.ta_init(arena_bytes) != 0:
         raise RuntimeError("tracing allocator: cudaMalloc of the arenas failed")
     alloc = torch.cuda.memory.CUDAPluggableAllocator(build(), "ta_malloc", "ta_free")
-    L.ta_select(0)
+    # the second arena: a fresh process on the same box may receive the very same
+    # virtual addresses for its first cudaMalloc as the offline process did, so the
+    # first arena would hand out the offline addresses again (nothing to relocate);
+    # the second one lies elsewhere by construction
+    L.ta_select(1)
     L.ta_clear()
     L.ta_log(1)
     pool = torch.cuda.MemPool(alloc.allocator())
