@@ -37,6 +37,23 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
     return m;
 }
 
+// Position of the k-th (0-based) set bit of w; requires k < popc(w).  Five
+// popcount halvings, branch-free (the __fns library sequence is ~3x as many
+// instructions, with branches).
+__device__ __forceinline__ uint32_t nth_set_bit(uint32_t w, uint32_t k) {
+    uint32_t pos = 0, c;
+    c = __popc(w & 0xFFFFu);
+    if (k >= c) { k -= c; pos = 16; }
+    c = __popc((w >> pos) & 0xFFu);
+    if (k >= c) { k -= c; pos += 8; }
+    c = __popc((w >> pos) & 0xFu);
+    if (k >= c) { k -= c; pos += 4; }
+    c = __popc((w >> pos) & 0x3u);
+    if (k >= c) { k -= c; pos += 2; }
+    c = (w >> pos) & 1u;
+    return k >= c ? pos + 1 : pos;
+}
+
 // ---- programmatic dependent launch (PDL) --------------------------------------
 // Kernels after the first of a call are launched with programmatic stream
 // serialization: a grid may start while its predecessor drains.  Every kernel

@@ -1427,8 +1427,10 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     __shared__ uint32_t s_m[kEmitChunks][64], s_i[kEmitChunks][64], s_q[kEmitChunks][64];
     __shared__ uint32_t s_pre[kEmitChunks][65], s_prm[kEmitChunks][65], s_prq[kEmitChunks][65];
     const unsigned long long tl0 = TL_NOW();
+    unsigned long long tl_p = tl0;
     pdl_wait();
     if (MEDUSA_EARLY_TRIGGER) pdl_trigger();  // k_result waits for this grid's completion
+    TL_PHASE(5, 60, tl_p);  // wait
     const MaterializeArgs& a = p.a;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t c0 = blockIdx.x * kEmitChunks;
@@ -1446,6 +1448,7 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
 #pragma unroll
     for (int h = 0; h < kEmitChunks; ++h) total[h] = (uint32_t)h < nch ? __ldcg(p.d.chunk_cnt + c0 + h) : 0u;
     uint64_t prefix = block_prefix(p.d.chunk_cnt, p.d.chunk_sup, c0);
+    TL_PHASE(5, 61, tl_p);  // mask words, counts, chunk prefix
     if (warp < 2 * kEmitChunks) {  // popcount prefixes of each half of each chunk's 64 mask words
         const uint32_t h = h_m, half = warp & 1;
         const uint32_t mv = mv_m, iv = iv_m, qv = qv_m;
@@ -1489,13 +1492,14 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
             }
         }
     }
+    TL_PHASE(5, 62, tl_p);  // popcount prefixes, chunk_base
     // records: every load of the CTA's (up to kRecPerThread per chunk per thread)
     // issued before the first store -- the loads do not wait for each other
     constexpr int kRecPerThread = 2;
     auto source = [&](int h, uint32_t r) -> uint64_t {  // the record of the chunk's r-th slot
         uint32_t lo = 0, hi = 64;  // last mask word m with s_pre[m] <= r
         while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
-        const uint32_t bit = __fns(s_m[h][lo], 0, (int)(r - s_pre[h][lo]) + 1);  // the (r - s_pre[lo])-th set bit
+        const uint32_t bit = nth_set_bit(s_m[h][lo], r - s_pre[h][lo]);  // the (r - s_pre[lo])-th set bit
         const uint32_t below = (1u << bit) - 1u;
         const uint32_t w = lo / 8;  // the classify warp that owned the word
         const uint64_t region = (uint64_t)((c0 + h) * kWarps + w) * p.d.cap_pw;
@@ -1532,6 +1536,7 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
         for (uint32_t r = tid + kRecPerThread * kThreads; r < total[h]; r += kThreads)
             if (pf + r < a.capacity) a.slot[pf + r] = source(h, r);
     }
+    TL_PHASE(5, 63, tl_p);  // records
     if (!MEDUSA_EARLY_TRIGGER) pdl_trigger();
     TL_REC(5, 0, tl0);
 }

@@ -25,7 +25,7 @@
 //     chunk_base[c+1]), known after one load.  Work is per record, not per
 //     word: thread r loads record r (coalesced), gathers old_base / new_base /
 //     new_size of its allocation (L2-resident, 24 B per allocation), finds its
-//     word as the (r - prefix)-th set bit of one mask word (__fns over a 64-entry
+//     word as the (r - prefix)-th set bit of one mask word (nth_set_bit over a 64-entry
 //     shared popcount prefix), validates and rewrites the word in shared memory;
 //   * gather tasks (2048 nodes each) are appended to the same grid;
 //   * validation failures (rare) go to the report with atomics; a one-thread
@@ -183,7 +183,7 @@ template <int CPB>
 __device__ __forceinline__ uint32_t table_word(const TableView<CPB>& T, uint32_t r) {
     uint32_t lo = 0, hi = TableView<CPB>::kMask;
     while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (T.pre[mid] <= r) lo = mid; else hi = mid; }
-    return lo * 32 + __fns(T.mask[lo], 0, (int)(r - T.pre[lo]) + 1);
+    return lo * 32 + nth_set_bit(T.mask[lo], r - T.pre[lo]);
 }
 
 // record k -> kind (0 ok, 1 bad id / missing record, 2 bad range), expected source

@@ -33,7 +33,8 @@ NAMES = {(1, 0): "trace/nodes", (1, 1): "trace/allocs", (1, 2): "trace/last-scan
          (7, 2): "restore/in-place", (7, 10): " res:mask+range", (7, 11): " res:records+gathers",
          (7, 12): " res:apply (+word wait)", (7, 13): " res:bulk store",
          (10, 50): " ires:fences+prefix", (10, 51): " ires:queue entry", (10, 52): " ires:fence search+group",
-         (10, 53): " ires:entry+mask"}
+         (10, 53): " ires:entry+mask", (5, 60): " emit:wait", (5, 61): " emit:masks+prefix",
+         (5, 62): " emit:popc prefixes", (5, 63): " emit:records"}
 REC = np.dtype([("t0", "<u8"), ("t1", "<u8"), ("kernel", "<u4"), ("cta", "<u4"), ("sm", "<u4"), ("tag", "<u4")])
 
 
