@@ -1818,15 +1818,19 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         // default priority: the trace checks fill in around them (M-M needs the
         // mortal tree only, M-I and I-I the sorted I list)
         if ((e = cudaStreamWaitEvent(low, s.traced, 0))) return e;
+#ifndef MEDUSA_DIAG_NO_CHECKS  // (diagnostic builds only: the step without the R-Q7 checks)
         {
             TimedLaunch tl("mat_check_mm", low);
             k_check_mm<<<check_ctas, kThreads, 0, low>>>(p);
         }
+#endif
         if ((e = cudaStreamWaitEvent(low, s.ranked, 0))) return e;
+#ifndef MEDUSA_DIAG_NO_CHECKS
         {
             TimedLaunch tl("mat_check_mi", low);
             k_check_mi<<<check_ctas, kThreads, 0, low>>>(p);
         }
+#endif
         if ((e = cudaEventRecord(s.join, low))) return e;
         if (!MEDUSA_MAIN_TAIL && (e = cudaStreamWaitEvent(stream, s.emitted, 0))) return e;
         if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;

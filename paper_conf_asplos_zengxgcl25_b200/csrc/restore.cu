@@ -237,12 +237,19 @@ __device__ __forceinline__ void report_add(unsigned long long* rep, uint32_t n_i
     if (n_chunk) atomicAdd(rep + 7, (unsigned long long)n_chunk);
 }
 
+#ifndef MEDUSA_RESTORE_PER
+#define MEDUSA_RESTORE_PER 2
+#endif
+constexpr int kRestorePer2 = MEDUSA_RESTORE_PER;  // records per thread in flight per round, two-chunk CTAs (3 and 4:
+                                                  //  a shorter apply phase, a longer first round: ALL10 restore
+                                                  //  span +1.3 / +1.9 us, measured)
 template <int CPB>
 __global__ void __launch_bounds__(kThreads, (CPB == 1 ? 8 : 6))
 restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
     constexpr uint32_t kWords = CPB * kTaskWords;   // words of this CTA (CPB consecutive chunks)
     constexpr uint32_t kMask = CPB * kMaskPerTask;  // their mask words
     constexpr uint32_t kAllOk = (1u << CPB) - 1u;
+    constexpr int kRestorePer = CPB == 2 ? kRestorePer2 : 2;
     __shared__ __align__(128) uint64_t s_words[kWords];
     __shared__ TableView<CPB> T;
     __shared__ __align__(8) unsigned long long s_mbar[CPB];
@@ -308,17 +315,17 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
         if (tid < 32) table_prefix<CPB>(T);
         const uint32_t cb0 = T.cb[0];
         uint32_t n_bits = T.cb[CPB] >= cb0 ? min(T.cb[CPB] - cb0, kWords) : 0u;  // exact once verified
-        // 3. records, two per thread per round: load, gather, (after the prefix is
+        // 3. records, kRestorePer per thread per round: load, gather, (after the prefix is
         //    ready) locate the word, validate and rewrite it in shared memory
         uint32_t n_id = 0, n_rg = 0, n_st = 0;
         uint64_t first = ~0ull;
         uint32_t ready_mask = tma ? 0u : ~0u;  // chunks whose words have landed
         bool fast = true;
-        for (uint32_t rb = 0; rb < max(n_bits, 1u); rb += 2 * kThreads) {
-            uint64_t exp[2], nv[2];
-            uint32_t kind[2];  // 0 ok, 1 bad id, 2 bad range, 3 none
+        for (uint32_t rb = 0; rb < max(n_bits, 1u); rb += kRestorePer * kThreads) {
+            uint64_t exp[kRestorePer], nv[kRestorePer];
+            uint32_t kind[kRestorePer];  // 0 ok, 1 bad id, 2 bad range, 3 none
 #pragma unroll
-            for (int u = 0; u < 2; ++u) {
+            for (int u = 0; u < kRestorePer; ++u) {
                 const uint32_t r = rb + tid + u * kThreads;
                 kind[u] = 3;
                 exp[u] = nv[u] = 0;
@@ -332,7 +339,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 if (T.ok != kAllOk) {  // (rare) an inconsistent chunk: round 0 again, chunk by chunk
                     fast = false;
 #pragma unroll
-                    for (int u = 0; u < 2; ++u) {
+                    for (int u = 0; u < kRestorePer; ++u) {
                         const uint32_t r = tid + u * kThreads;
                         uint64_t k;
                         kind[u] = (r < n_bits && table_rec<CPB>(T, r, k)) ? load_rec(a, k, exp[u], nv[u]) : 3u;
@@ -340,7 +347,7 @@ restore_kernel(RestoreArgs a, uint32_t n_word_tasks, uint32_t n_tasks) {
                 }
             }
 #pragma unroll
-            for (int u = 0; u < 2; ++u) {
+            for (int u = 0; u < kRestorePer; ++u) {
                 if (kind[u] == 3) continue;
                 const uint32_t r = rb + tid + u * kThreads;
                 const uint32_t q = table_word<CPB>(T, r);
