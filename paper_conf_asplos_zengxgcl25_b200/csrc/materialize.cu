@@ -1421,8 +1421,10 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
 //    window hits below q), else from its queue entry, where k_iresolve left it (rank among the
 //    warp's queued words below q).  Regions are read in order: no word-indexed
 //    staging.
-constexpr int kEmitChunks = 2;  // chunks per k_emit CTA (the grid fits one wave)
-
+// chunks per k_emit CTA: 2 (the grid of a large set fits one wave); 1 for a set of
+// fewer than two chunks per SM (a single model's), whose CTAs then spread over
+// more SMs with half the records each
+template <int kEmitChunks>
 __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     __shared__ uint32_t s_m[kEmitChunks][64], s_i[kEmitChunks][64], s_q[kEmitChunks][64];
     __shared__ uint32_t s_pre[kEmitChunks][65], s_prm[kEmitChunks][65], s_prq[kEmitChunks][65];
@@ -1711,6 +1713,14 @@ Scratch* device_scratch(cudaError_t* e, std::unique_lock<std::mutex>* lk) {
     return &s;
 }
 
+cudaError_t launch_emit(const Scratch& s, uint32_t C, cudaStream_t st, const P& p) {
+#ifndef MEDUSA_EMIT_SMALL
+#define MEDUSA_EMIT_SMALL 1
+#endif
+    if (MEDUSA_EMIT_SMALL && C < 2u * (uint32_t)s.sm_count) return launch_pdl(k_emit<1>, C, kThreads, 0, st, p);
+    return launch_pdl(k_emit<2>, (C + 1) / 2, kThreads, 0, st, p);
+}
+
 // the whole analysis on `stream` (no synchronization):
 //   stream:            memset -> k_trace [traced] -> k_classify -> [ranked] k_iresolve -> k_emit [join]
 //   side (high prio):             [traced] k_isort -> k_rank [ranked]
@@ -1798,7 +1808,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
                         return e;
                 }
                 TimedLaunch tl("mat_emit", stream);
-                if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
+                if ((e = launch_emit(s, C, stream, p))) return e;
             }
         } else {
             if ((e = cudaEventRecord(s.classified, stream))) return e;
@@ -1811,7 +1821,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
                     k_iresolve<<<std::min<unsigned>(C, (unsigned)s.sm_count * 6), kThreads, 0, side>>>(p);  // one wave (6 per SM)
                 }
                 TimedLaunch tl("mat_emit", side);
-                if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, side, p))) return e;
+                if ((e = launch_emit(s, C, side, p))) return e;
             }
             if ((e = cudaEventRecord(s.emitted, side))) return e;
         }
@@ -1836,7 +1846,7 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
         if ((e = cudaStreamWaitEvent(stream, s.join, 0))) return e;
     } else if (C) {
         TimedLaunch tl("mat_emit", stream);
-        if ((e = launch_pdl(k_emit, (C + kEmitChunks - 1) / kEmitChunks, kThreads, 0, stream, p))) return e;
+        if ((e = launch_emit(s, C, stream, p))) return e;
     }
     return cudaGetLastError();
 }
