@@ -159,7 +159,12 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
     return v;
 }
 
-__device__ __forceinline__ uint32_t fence_stride(uint32_t nI) { return nI ? (nI + kFenceCap - 1) / kFenceCap : 1; }
+// every stride-th sorted I base is a fence; the stride is a multiple of 4 so a
+// group [j stride, (j + 1) stride) of the sorted bases is whole 32-byte blocks
+// (the i_base array is 256-byte aligned and padded)
+__device__ __forceinline__ uint32_t fence_stride(uint32_t nI) {
+    return 4u * ((nI + 4u * kFenceCap - 1) / (4u * kFenceCap));
+}
 
 // Sum of cnt[0, k) of a two-level counter (sup[g] = sum of cnt[256g, 256g + 256)):
 // at most k/256 + 255 loads, spread over the CTA, and one reduction; every thread
@@ -666,21 +671,29 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
     TL_REC(3, 0, tl0);
 }
 
-// count of sorted I bases <= x (fences in shared memory, then one group of <= stride
-// bases read with independent loads)
+// four sorted I bases (one 32-byte block, one L2 sector) in one load
+__device__ __forceinline__ void ld_base4(const uint64_t* q, uint64_t& b0, uint64_t& b1, uint64_t& b2, uint64_t& b3) {
+    asm volatile("ld.global.v4.u64 {%0, %1, %2, %3}, [%4];" : "=l"(b0), "=l"(b1), "=l"(b2), "=l"(b3) : "l"(q));
+}
+
+// count of sorted I bases <= x: the fences in shared memory, then the group of
+// stride bases after the last fence <= x in 32-byte blocks (one sector each; 8-byte
+// loads cost one sector per base: 2.5 us of k_iresolve's 7 us per CTA, measured)
+// (fence: shared memory in k_iresolve, global in k_check_mi)
 __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t nf, uint32_t stride, uint32_t nI,
                                                const uint64_t* i_base, uint64_t x) {
-    uint32_t lo = 0, hi = nf;  // (fence: shared memory in k_iresolve, global in k_check_mi)
+    uint32_t lo = 0, hi = nf;
     while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (fence[mid] <= x) lo = mid + 1; else hi = mid; }
     if (lo == 0) return 0;
     const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
-    uint32_t c = g0 + 1;
-    for (uint32_t k = g0 + 1; k < g1; k += 8) {
+    uint32_t c = g0 + 1;  // base g0 (the fence) <= x
+    for (uint32_t k = g0; k < g1; k += 8) {  // two blocks per round (a group of 4: one)
         uint64_t b[8];
+        ld_base4(i_base + k, b[0], b[1], b[2], b[3]);
+        if (k + 4 < g1) ld_base4(i_base + k + 4, b[4], b[5], b[6], b[7]);
+        else b[4] = b[5] = b[6] = b[7] = ~0ull;
 #pragma unroll
-        for (int u = 0; u < 8; ++u) b[u] = (k + u < g1) ? i_base[k + u] : ~0ull;
-#pragma unroll
-        for (int u = 0; u < 8; ++u) c += (k + u < g1 && b[u] <= x) ? 1u : 0u;
+        for (int u = 0; u < 8; ++u) c += (k + u > g0 && k + u < g1 && b[u] <= x) ? 1u : 0u;
         if (b[7] > x) break;
     }
     return c;
@@ -1663,12 +1676,15 @@ cudaError_t ensure(Scratch& s, size_t n, size_t C, size_t W, size_t need_pw) {
         (e = grow(s, s.d.sv, N)) || (e = grow(s, s.d.icnt, N / kThreads + 2)) ||
         (e = grow(s, s.d.tmax_k, N / kIsortTile + 2)) || (e = grow(s, s.d.tmax_v, N / kIsortTile + 2)) ||
         (e = grow(s, s.d.samp_k, N / kSampleStride + 64)) || (e = grow(s, s.d.samp_v, N / kSampleStride + 64)) ||
-        (e = grow(s, s.d.i_base, N)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
+        (e = grow(s, s.d.i_base, N + 64)) || (e = grow(s, s.d.i_rest, N)) || (e = grow(s, s.d.i_tf, N)) ||
         (e = grow(s, s.d.fence, (size_t)kFenceCap)) ||
         (e = grow(s, s.d.rec, QQ)) || (e = grow(s, s.d.queue, QQ)) ||
         (e = grow(s, s.d.qcnt, CC * kWarps)) ||
         (e = grow(s, s.d.imask, WW / 32 + 1)) || (e = grow(s, s.d.qmask, WW / 32 + 1)))
         return e;
+    // (the group scan reads whole 32-byte blocks, up to 7 bases past the list's end:
+    // initialized once, their values are never used)
+    if ((e = cudaMemset(s.d.i_base, 0, (N + 64) * sizeof(uint64_t)))) return e;
     s.d.cap_pw = (uint32_t)RR;
     s.cap_n = N; s.cap_C = CC; s.cap_w = WW; s.cap_r = RR; s.cap_q = QQ;
     return cudaSuccess;
