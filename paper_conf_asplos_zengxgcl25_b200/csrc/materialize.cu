@@ -1353,7 +1353,7 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 // ----------------------------------------------------------------------------
 // 4b. k_iresolve (after k_rank and k_classify): the queued candidates against the
 //     sorted I list.  Persistent CTAs loop over chunks, fences loaded once per
-//     CTA; the chunk's eight queue ranges (one per classify warp) are spread over
+//     CTA before the wait for k_classify; the chunk's eight queue ranges (one per classify warp) are spread over
 //     the whole CTA (entry i of their concatenation -> thread i mod 256: a long
 //     range no longer sets the chunk's time; per-warp ranges measured ALL10
 //     iresolve 16.0 vs 13.8 us span).  Per candidate one group of bases and one
@@ -1363,9 +1363,17 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
     const unsigned long long tl0 = TL_NOW();
-    pdl_wait();
-    const uint32_t nI = p.d.ctl->nI;
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // the sorted I list is complete when this grid starts (k_isort / k_rank are a
+    // full dependency through the 'ranked' event, k_trace one before them): the
+    // fences come in before the wait for k_classify
+    const uint32_t nI = __ldcg(&p.d.ctl->nI);
+    {
+        const uint32_t stride = fence_stride(nI);
+        const uint32_t nf = nI ? (nI + stride - 1) / stride : 0u;
+        for (uint32_t f = tid; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
+    }
+    pdl_wait();  // k_classify: queue, counts, masks
     if (nI) {
         // the chunk's queue ranges (one per classify warp) taken by the whole CTA:
         // entry i of the chunk's concatenated ranges -> thread i mod 256, so a warp
@@ -1374,7 +1382,6 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
         const uint32_t stride = fence_stride(nI);
         const uint32_t nf = (nI + stride - 1) / stride;
         const uint32_t cap = p.d.cap_pw;
-        for (uint32_t f = tid; f < nf; f += kThreads) s_fence[f] = __ldcg(p.d.fence + f);
         uint32_t my_cnt = (blockIdx.x < p.C && tid < kWarps) ? min(__ldcg(p.d.qcnt + blockIdx.x * kWarps + tid), cap) : 0u;
         for (uint32_t c = blockIdx.x; c < p.C; c += gridDim.x) {
             if (warp == 0) {  // exclusive prefix of the 8 range lengths
@@ -1759,7 +1766,10 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     // ordinal-ordered I compaction pays when the set spans several address regions
     // (several models: most rank tiles then hold another model's keys); a single
     // model's set (<= 128 k_trace CTAs, ~4 tiles) skips the gather it costs k_isort
-    const uint32_t ordered = (alloc_ctas > 128 && alloc_ctas <= kOrderedCtas) ? 1u : 0u;
+#ifndef MEDUSA_ORDERED_MIN_CTAS
+#define MEDUSA_ORDERED_MIN_CTAS 128
+#endif
+    const uint32_t ordered = (alloc_ctas > MEDUSA_ORDERED_MIN_CTAS && alloc_ctas <= kOrderedCtas) ? 1u : 0u;
     P p{a, d, C, nb, node_ctas, alloc_ctas, ordered};
     *out = p;
     cudaError_t e;
