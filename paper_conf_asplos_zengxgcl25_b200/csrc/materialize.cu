@@ -163,7 +163,7 @@ __device__ __forceinline__ uint64_t warp_max_u64(uint64_t v) {
 // group [j stride, (j + 1) stride) of the sorted bases is whole 32-byte blocks
 // (the i_base array is 256-byte aligned and padded)
 __device__ __forceinline__ uint32_t fence_stride(uint32_t nI) {
-    return 4u * ((nI + 4u * kFenceCap - 1) / (4u * kFenceCap));
+    return 4u * max(1u, (nI + 4u * kFenceCap - 1) / (4u * kFenceCap));  // (>= 4 also for an empty list)
 }
 
 // Sum of cnt[0, k) of a two-level counter (sup[g] = sum of cnt[256g, 256g + 256)):
