@@ -1360,6 +1360,9 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 //     entry (two dependent loads); a hit writes its record over its queue
 //     entry's word and sets its bit in the mask and in the I-resolved mask; the
 //     chunk's count grows by one atomic per warp.
+#ifndef MEDUSA_IRES_SMEM_MASK
+#define MEDUSA_IRES_SMEM_MASK 1  // a chunk's I-resolved bits gathered in shared memory, one atomic per mask word
+#endif
 __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
     __shared__ uint64_t s_fence[kFenceCap];
     const unsigned long long tl0 = TL_NOW();
@@ -1379,6 +1382,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
         // entry i of the chunk's concatenated ranges -> thread i mod 256, so a warp
         // whose range is long (up to cap_pw entries) does not set the chunk's time
         __shared__ uint32_t s_pre[kWarps + 1];
+        __shared__ uint32_t s_mb[kChunkWords / 32];  // the chunk's I-resolved bits (MEDUSA_IRES_SMEM_MASK)
         const uint32_t stride = fence_stride(nI);
         const uint32_t nf = (nI + stride - 1) / stride;
         const uint32_t cap = p.d.cap_pw;
@@ -1394,6 +1398,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                 if (lane < kWarps) s_pre[lane + 1] = incl;
                 if (lane == 0) s_pre[0] = 0;
             }
+            if (MEDUSA_IRES_SMEM_MASK && tid < kChunkWords / 32) s_mb[tid] = 0;
             __syncthreads();  // (also: the fences, on the first chunk)
             const uint32_t cn = c + gridDim.x;  // the next chunk's counts, loaded early
             if (tid < kWarps) my_cnt = cn < p.C ? min(__ldcg(p.d.qcnt + cn * kWarps + tid), cap) : 0u;
@@ -1415,8 +1420,12 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                         if (q.x < e.end && e.t_alloc < q.t) {
                             hit = true;
                             p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
-                            atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
-                            atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
+                            if (MEDUSA_IRES_SMEM_MASK) {
+                                atomicOr(&s_mb[(q.g - c * kChunkWords) >> 5], 1u << (q.g & 31));
+                            } else {
+                                atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
+                                atomicOr(p.d.imask + (q.g >> 5), 1u << (q.g & 31));
+                            }
                         }
                     }
                 }
@@ -1426,7 +1435,15 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                 atomicAdd(p.d.chunk_cnt + c, cnt);
                 atomicAdd(p.d.chunk_sup + (c >> 8), (unsigned long long)cnt);
             }
-            __syncthreads();  // s_pre is rewritten for the next chunk
+            if (MEDUSA_IRES_SMEM_MASK) {  // the chunk's bits: one reduction per mask word (no return value)
+                __syncthreads();
+                const uint64_t mw = (uint64_t)c * (kChunkWords / 32) + tid;
+                if (tid < kChunkWords / 32 && s_mb[tid]) {
+                    atomicOr(p.a.mask + mw, s_mb[tid]);
+                    p.d.imask[mw] = s_mb[tid];  // (k_classify zeroed it; this CTA alone writes the chunk's words)
+                }
+            }
+            __syncthreads();  // s_pre / s_mb are rewritten for the next chunk
         }
     }
     pdl_trigger();
