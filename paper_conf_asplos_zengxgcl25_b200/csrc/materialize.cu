@@ -1536,8 +1536,9 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
     // issued before the first store -- the loads do not wait for each other
     constexpr int kRecPerThread = 2;
     auto source = [&](int h, uint32_t r) -> uint64_t {  // the record of the chunk's r-th slot
-        uint32_t lo = 0, hi = 64;  // last mask word m with s_pre[m] <= r
-        while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[h][mid] <= r) lo = mid; else hi = mid; }
+        uint32_t lo = 0;  // last mask word m with s_pre[m] <= r (s_pre[0] = 0): binary lifting, no branches
+#pragma unroll
+        for (uint32_t st = 32; st > 0; st >>= 1) lo += s_pre[h][lo + st] <= r ? st : 0u;
         const uint32_t bit = nth_set_bit(s_m[h][lo], r - s_pre[h][lo]);  // the (r - s_pre[lo])-th set bit
         const uint32_t below = (1u << bit) - 1u;
         const uint32_t w = lo / 8;  // the classify warp that owned the word

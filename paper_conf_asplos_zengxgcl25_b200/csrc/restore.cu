@@ -181,8 +181,9 @@ __device__ __forceinline__ bool table_rec(const TableView<CPB>& T, uint32_t r, u
 // word (in the CTA) of the r-th slot bit, r < pre[kMask]
 template <int CPB>
 __device__ __forceinline__ uint32_t table_word(const TableView<CPB>& T, uint32_t r) {
-    uint32_t lo = 0, hi = TableView<CPB>::kMask;
-    while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (T.pre[mid] <= r) lo = mid; else hi = mid; }
+    uint32_t lo = 0;  // last mask word m with pre[m] <= r (pre[0] = 0): binary lifting, no branches
+#pragma unroll
+    for (uint32_t st = TableView<CPB>::kMask / 2; st > 0; st >>= 1) lo += T.pre[lo + st] <= r ? st : 0u;
     return lo * 32 + nth_set_bit(T.mask[lo], r - T.pre[lo]);
 }
 
