@@ -682,8 +682,12 @@ __device__ __forceinline__ void ld_base4(const uint64_t* q, uint64_t& b0, uint64
 // (fence: shared memory in k_iresolve, global in k_check_mi)
 __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t nf, uint32_t stride, uint32_t nI,
                                                const uint64_t* i_base, uint64_t x) {
-    uint32_t lo = 0, hi = nf;
-    while (lo < hi) { uint32_t mid = (lo + hi) >> 1; if (fence[mid] <= x) lo = mid + 1; else hi = mid; }
+    uint32_t lo = 0;  // #{fences <= x}: binary lifting, no data-dependent branches
+#pragma unroll
+    for (uint32_t st = kFenceCap; st > 0; st >>= 1) {  // (reaches 2 kFenceCap - 1 >= nf)
+        const uint32_t k = lo + st;
+        if (k <= nf) lo = fence[k - 1] <= x ? k : lo;
+    }
     if (lo == 0) return 0;
     const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
     uint32_t c = g0 + 1;  // base g0 (the fence) <= x
@@ -789,6 +793,19 @@ __device__ __forceinline__ int q_start(const Tree& T) {
     return l;
 }
 
+// #{u < n : a[u] <= y} (kStrict: a[u] < y) of an ascending array of n < 2 kTop
+// entries in shared memory: binary lifting, no data-dependent branches
+template <uint32_t kTop, bool kStrict = false>
+__device__ __forceinline__ uint32_t count_upto(const uint32_t* a, uint32_t n, uint32_t y) {
+    uint32_t c = 0;
+#pragma unroll
+    for (uint32_t st = kTop; st > 0; st >>= 1) {
+        const uint32_t k = c + st;  // take a[c .. k) if it is in range and its last entry qualifies
+        if (k <= n) c = (kStrict ? a[k - 1] < y : a[k - 1] <= y) ? k : c;
+    }
+    return c;
+}
+
 __device__ __forceinline__ bool q_test(const Tree& T, const ClsShared& S, int l, uint32_t c, const QRange& q) {
     if (c >= T.cnt[l]) return false;
     const uint32_t sh = 5u * (uint32_t)l;  // a node of level l covers 2^sh ordinals
@@ -797,8 +814,7 @@ __device__ __forceinline__ bool q_test(const Tree& T, const ClsShared& S, int l,
     const uint2 nd = l > 0 ? __ldcg(T.node + T.off[l] + c) : __ldcg(T.leaf + c);
     bool keep = nd.x > q.T0 && nd.y < q.T1;
     if (keep && l == 0 && q.exact) {  // live at one of the chunk's launches
-        uint32_t lo = 0, hi = q.ng0;   // the first segment launched after t_alloc
-        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (S.nt0[mid] <= nd.y) lo = mid + 1; else hi = mid; }
+        const uint32_t lo = count_upto<kNodeGrp>(S.nt0, q.ng0, nd.y);  // the first segment launched after t_alloc
         keep = lo < q.ng0 && S.nt0[lo] < nd.x;
     }
     return keep;
@@ -871,12 +887,8 @@ __device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uin
     __syncthreads();
     for (uint32_t e = tid; e < m; e += kThreads) {
         const uint32_t ta = S.rta[e], tf = S.rtf[e];
-        uint32_t lo = 0, hi = ng;  // u0 = #{u : t_u <= t_alloc}
-        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] <= ta) lo = mid + 1; else hi = mid; }
-        const uint32_t u0 = lo;
-        hi = ng;  // u1 = #{u : t_u < t_free}
-        while (lo < hi) { const uint32_t mid = (lo + hi) >> 1; if (nt[mid] < tf) lo = mid + 1; else hi = mid; }
-        const uint32_t u1 = lo;
+        const uint32_t u0 = count_upto<kNodeGrp>(nt, ng, ta);        // #{u : t_u <= t_alloc}
+        const uint32_t u1 = count_upto<kNodeGrp, true>(nt, ng, tf);  // #{u : t_u < t_free}
         if (u0 < u1) {
             atomicXor(&S.live[u0][e >> 5], 1u << (e & 31));
             if (u1 < ng) atomicXor(&S.live[u1][e >> 5], 1u << (e & 31));
