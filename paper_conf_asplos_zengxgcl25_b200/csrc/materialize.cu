@@ -101,6 +101,7 @@ struct Tree {
     uint32_t off[kMaxLevels + 1]; // off[1] = 0
     uint32_t cnt[kMaxLevels + 1]; // nodes of level l (cnt[0] = n)
     uint32_t top;                 // the level with <= 32 nodes (0 if n <= 32)
+    int32_t l0;                   // a query's start level: the highest with <= kThreads nodes (set on the host)
 };
 
 struct Dev {  // scratch of one call (device pointers)
@@ -787,11 +788,7 @@ struct QRange {
     bool exact;
 };
 
-__device__ __forceinline__ int q_start(const Tree& T) {
-    int l = (int)T.top;
-    while (l > 0 && T.cnt[l - 1] <= (uint32_t)kThreads) --l;
-    return l;
-}
+__device__ __forceinline__ int q_start(const Tree& T) { return T.l0; }
 
 // #{u < n : a[u] <= y} (kStrict: a[u] < y) of an ascending array of n < 2 kTop
 // entries in shared memory: binary lifting, no data-dependent branches
@@ -1792,6 +1789,11 @@ cudaError_t enqueue(Scratch& s, const MaterializeArgs& a, cudaStream_t stream, P
     Dev d = s.d;
     const Tree shape = tree_shape(n);
     d.tree.top = shape.top;
+    {  // the query's start level (q_start)
+        int l = (int)shape.top;
+        while (l > 0 && shape.cnt[l - 1] <= (uint32_t)kThreads) --l;
+        d.tree.l0 = l;
+    }
     for (int l = 0; l <= kMaxLevels; ++l) { d.tree.cnt[l] = shape.cnt[l]; d.tree.off[l] = shape.off[l]; }
     // ordinal-ordered I compaction pays when the set spans several address regions
     // (several models: most rank tiles then hold another model's keys); a single
