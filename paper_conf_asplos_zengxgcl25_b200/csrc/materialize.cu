@@ -313,9 +313,9 @@ __device__ void allocs_role(const P& p, uint32_t cta) {
         // ordered: the CTA's keys at its own region, k_isort finds them by the CTA
         // prefix of icnt; else one atomic hands out positions
         if (p.ordered) { s_base = cta * kThreads; p.d.icnt[cta] = ni; }
-        if (ni) {
-            const uint32_t b = atomicAdd(&p.d.ctl->nI, ni);
-            if (!p.ordered) s_base = b;
+        if (ni) {  // (ordered: a reduction, nothing to wait for; else the CTA's positions)
+            if (p.ordered) atomicAdd(&p.d.ctl->nI, ni);
+            else s_base = atomicAdd(&p.d.ctl->nI, ni);
         }
         if (s_mx) {
             atomicMax(&p.d.ctl->gmin_c, ~s_mn);
