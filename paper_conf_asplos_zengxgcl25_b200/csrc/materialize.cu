@@ -495,13 +495,21 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
     const uint32_t o = tid * kSortPer;  // this thread's consecutive elements
     uint64_t k[kSortPer];
     uint32_t v[kSortPer];
+    // (ordered) the k_trace CTA holding compacted position g = last b with s_pre[b]
+    // <= g: one binary search for the thread's first position, then a forward step
+    // per following one (its kSortPer positions are consecutive)
+    uint32_t lo = 0;
+    if (p.ordered && t0 + o < n) {
+        uint32_t hi = p.alloc_ctas;
+        const uint32_t g = t0 + o;
+        while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= g) lo = mid; else hi = mid; }
+    }
 #pragma unroll
     for (int r = 0; r < kSortPer; ++r) {
         const uint32_t g = t0 + o + r;
         uint32_t q = g;
-        if (p.ordered && g < n) {  // the CTA holding compacted position g: last b with s_pre[b] <= g
-            uint32_t lo = 0, hi = p.alloc_ctas;
-            while (hi - lo > 1) { const uint32_t mid = (lo + hi) >> 1; if (s_pre[mid] <= g) lo = mid; else hi = mid; }
+        if (p.ordered && g < n) {
+            while (lo + 1 < p.alloc_ctas && s_pre[lo + 1] <= g) ++lo;  // (empty CTAs share a prefix value)
             q = lo * kThreads + (g - s_pre[lo]);
         }
         k[r] = g < n ? __ldcg(p.d.sk0 + q) : ~0ull;
