@@ -614,7 +614,7 @@ __device__ __forceinline__ uint32_t count_lt64(uint64_t k0, uint32_t v0, uint64_
     return c > ne ? ne : c;
 }
 
-__global__ void __launch_bounds__(kThreads) k_rank(P p) {
+__global__ void __launch_bounds__(kThreads, 8) k_rank(P p) {
     __shared__ uint32_t s_cnt[kWarps][32];
     const unsigned long long tl0 = TL_NOW();
     pdl_wait();
@@ -629,14 +629,29 @@ __global__ void __launch_bounds__(kThreads) k_rank(P p) {
         const uint64_t xk = has ? __ldcg(p.d.sk + g) : ~0ull;
         const uint32_t xv = has ? __ldcg(p.d.sv + g) : 0xFFFFFFFFu;
         uint32_t cnt = 0;
-        for (uint32_t tb = warp; tb < T; tb += kWarps) {
+        // the key ranges of this warp's tiles (warp, warp + 8, ...), lane t holding the
+        // t-th: one load round for all of them (up to 32 per pass)
+        uint64_t bmnk = 0, bmxk = 0;
+        uint32_t bmnv = 0, bmxv = 0;
+        uint32_t tpass = 0;  // the pass of 32 tiles whose bounds the lanes hold
+        auto load_bounds = [&](uint32_t pass) {
+            const uint32_t tl = warp + (pass * 32 + lane) * kWarps;
+            if (tl < T) {
+                const uint32_t sl = tl * kIsortTile / kSampleStride;
+                bmnk = __ldcg(p.d.samp_k + sl); bmnv = __ldcg(p.d.samp_v + sl);
+                bmxk = __ldcg(p.d.tmax_k + tl); bmxv = __ldcg(p.d.tmax_v + tl);
+            }
+        };
+        load_bounds(0);
+        for (uint32_t tb = warp, ti = 0; tb < T; tb += kWarps, ++ti) {
+            if (ti / 32 != tpass) load_bounds(tpass = ti / 32);  // (more than 256 tiles)
+            const uint64_t mnk = __shfl_sync(0xffffffffu, bmnk, ti % 32), mxk = __shfl_sync(0xffffffffu, bmxk, ti % 32);
+            const uint32_t mnv = __shfl_sync(0xffffffffu, bmnv, ti % 32), mxv = __shfl_sync(0xffffffffu, bmxv, ti % 32);
             if (tb == ta) continue;
             const uint32_t b0 = tb * kIsortTile, nb = min((uint32_t)kIsortTile, nI - b0);
             const uint32_t ns = (nb + kSampleStride - 1) / kSampleStride;  // samples of tile tb (<= 64)
             const uint32_t s0 = b0 / kSampleStride;
             {  // the tile's key range: lanes below its least key count 0, above its greatest nb
-                const uint64_t mnk = __ldcg(p.d.samp_k + s0), mxk = __ldcg(p.d.tmax_k + tb);
-                const uint32_t mnv = __ldcg(p.d.samp_v + s0), mxv = __ldcg(p.d.tmax_v + tb);
                 const bool above = has && kv_less(mxk, mxv, xk, xv);
                 const bool below = !has || kv_less(xk, xv, mnk, mnv);
                 if (__all_sync(0xffffffffu, above || below)) {  // (ordered I keys: most tiles of the ten-model set)
