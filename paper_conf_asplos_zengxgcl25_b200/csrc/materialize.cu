@@ -579,7 +579,8 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
 // 2b. k_rank (after k_isort, only with more than one tile): global rank of every
 //     I key = its index in its sorted tile + the count of smaller keys in every
 //     other tile.  One CTA per range of 32 consecutive keys of one tile (one key
-//     per lane); warp w counts against tiles b = w, w + 8, ...: the tile's <= 32
+//     per lane); warp w counts against tiles b = w, w + 8, ... (their key ranges
+//     come in with one load round, lane t holding tile w + 8t): the tile's <= 32
 //     samples (every 32nd key) come in with one coalesced load and locate, by a
 //     shuffle search, the 32-key block of the tile holding each lane's lower
 //     bound; the block comes in with one more coalesced load and a shuffle
@@ -587,7 +588,8 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
 //     below the 32 keys is counted from its least and greatest key alone (the I
 //     keys are compacted in ordinal order, so with several models in one set most
 //     tiles hold another model's disjoint address region).  The counts of the 8
-//     warps meet in shared memory; warp 0 writes the 32 I entries.
+//     warps meet in shared memory; warp 0 writes the 32 I entries (with ordered
+//     keys, their block summaries combined per block: write_i_entry_warp).
 __device__ __forceinline__ bool kv_lt_lane(uint64_t k, uint32_t v, uint32_t src, uint64_t xk, uint32_t xv) {
     const uint64_t sk = __shfl_sync(0xffffffffu, k, src);
     const uint32_t sv = __shfl_sync(0xffffffffu, v, src);
@@ -1417,8 +1419,10 @@ __global__ void __launch_bounds__(kThreads, MEDUSA_CLS_MINB) k_classify(P p) {
 //     range no longer sets the chunk's time; per-warp ranges measured ALL10
 //     iresolve 16.0 vs 13.8 us span).  Per candidate one group of bases and one
 //     entry (two dependent loads); a hit writes its record over its queue
-//     entry's word and sets its bit in the mask and in the I-resolved mask; the
-//     chunk's count grows by one atomic per warp.
+//     entry's word and sets its bit in a shared copy of the chunk's I-resolved
+//     bits, which go to the mask (one red.or per mask word) and the I-resolved
+//     mask (one store per word) at the chunk's end; the chunk's count grows by
+//     one atomic per warp.
 #ifndef MEDUSA_IRES_SMEM_MASK
 #define MEDUSA_IRES_SMEM_MASK 1  // a chunk's I-resolved bits gathered in shared memory, one atomic per mask word
 #endif
