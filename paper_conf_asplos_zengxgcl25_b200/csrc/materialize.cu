@@ -384,13 +384,14 @@ __device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t n
 // block first (k_rank: a warp's 32 keys mostly take consecutive ranks, so one
 // pair of atomics per block instead of one per key -- the per-key atomics on the
 // same block cost k_rank ~1.3 us of its span beside k_classify, measured)
-__device__ __forceinline__ void write_i_entry_warp(const P& p, uint32_t r, uint32_t nI, uint32_t id, const medusa_alloc& x) {
+// (act: the calling lanes, all of which make this call)
+__device__ __forceinline__ void write_i_entry_warp(const P& p, uint32_t r, uint32_t nI, uint32_t id, const medusa_alloc& x,
+                                                   uint32_t act) {
     p.d.i_base[r] = x.base;
     p.d.i_rest[r] = IRest{x.base + x.size, x.t_alloc, id};
     p.d.i_tf[r] = x.t_free;
     const uint32_t stride = fence_stride(nI);
     if (r % stride == 0) p.d.fence[r / stride] = x.base;
-    const uint32_t act = __activemask();
     const uint32_t b = r / kIBlk;
     const uint32_t grp = __match_any_sync(act, b);
     const uint32_t mn_c = __reduce_max_sync(grp, ~x.t_alloc);  // (min t_alloc kept as the max of its complement)
@@ -706,16 +707,17 @@ __global__ void __launch_bounds__(kThreads, 8) k_rank(P p) {
         }
         s_cnt[warp][lane] = cnt;
         __syncthreads();
+#ifndef MEDUSA_RANK_WARP_BLK
+#define MEDUSA_RANK_WARP_BLK 1
+#endif
+        const uint32_t has_lanes = __ballot_sync(0xffffffffu, has);  // (every warp; used by warp 0)
         if (warp == 0 && has) {
             uint32_t rank = g - ta * kIsortTile;  // index inside its own tile
 #pragma unroll
             for (int w = 0; w < kWarps; ++w) rank += s_cnt[w][lane];
-#ifndef MEDUSA_RANK_WARP_BLK
-#define MEDUSA_RANK_WARP_BLK 1
-#endif
             // (ordered compaction: a warp's keys take consecutive ranks, one or two
             // blocks; otherwise their ranks scatter and the combining only costs)
-            if (MEDUSA_RANK_WARP_BLK && p.ordered) write_i_entry_warp(p, rank, nI, xv, ld_alloc(p.a.alloc + xv));
+            if (MEDUSA_RANK_WARP_BLK && p.ordered) write_i_entry_warp(p, rank, nI, xv, ld_alloc(p.a.alloc + xv), has_lanes);
             else write_i_entry(p, rank, nI, xv, ld_alloc(p.a.alloc + xv));
         }
         __syncthreads();  // s_cnt is rewritten by the next range
