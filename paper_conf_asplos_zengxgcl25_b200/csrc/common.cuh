@@ -1,5 +1,6 @@
 // Shared device helpers and internal launch interfaces of libmedusa (sm_100a).
 #pragma once
+#include <cstdio>
 
 #include <cstdint>
 #include <utility>
@@ -106,6 +107,24 @@ struct TimedLaunch {
 // ---- timeline instrumentation (diagnostic builds only: -DMEDUSA_TIMELINE) ------
 // Thread 0 of a CTA appends {start, end, kernel, cta, sm, tag} to a per-TU device
 // buffer (tools/timeline.py builds libmedusa_tl.so and reads it back).
+// ---- checked builds (-DMEDUSA_CHECKED; diagnostic, tools/gpu_variant_tests.sh) ----
+// MCHECK(c): a device-side bounds / invariant check on the computed indices of
+// the shared- and global-memory accesses that depend on data (positions from
+// searches, counts, ranks); a failure traps the kernel, so the test that ran it
+// fails with a CUDA error.  Compiled out of the product build.
+#ifdef MEDUSA_CHECKED
+#define MCHECK(c)                                                                          \
+    do {                                                                                   \
+        if (!(c)) {                                                                        \
+            printf("MCHECK failed: %s at %s:%d (block %u thread %u)\n", #c, __FILE__, __LINE__, \
+                   blockIdx.x, threadIdx.x);                                               \
+            __trap();                                                                      \
+        }                                                                                  \
+    } while (0)
+#else
+#define MCHECK(c) ((void)0)
+#endif
+
 #ifdef MEDUSA_TIMELINE
 struct TlRec {
     unsigned long long t0, t1;

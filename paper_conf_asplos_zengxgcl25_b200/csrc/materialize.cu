@@ -371,6 +371,7 @@ __global__ void __launch_bounds__(kThreads, 8) k_trace(P p) {
 
 // the I entry of sorted position r: arrays, fence, block summaries
 __device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t nI, uint32_t id, const medusa_alloc& x) {
+    MCHECK(r < nI && id < p.a.n_alloc);
     p.d.i_base[r] = x.base;
     p.d.i_rest[r] = IRest{x.base + x.size, x.t_alloc, id};
     p.d.i_tf[r] = x.t_free;
@@ -387,6 +388,7 @@ __device__ __forceinline__ void write_i_entry(const P& p, uint32_t r, uint32_t n
 // (act: the calling lanes, all of which make this call)
 __device__ __forceinline__ void write_i_entry_warp(const P& p, uint32_t r, uint32_t nI, uint32_t id, const medusa_alloc& x,
                                                    uint32_t act) {
+    MCHECK(r < nI && id < p.a.n_alloc && ((act >> (threadIdx.x & 31)) & 1u));
     p.d.i_base[r] = x.base;
     p.d.i_rest[r] = IRest{x.base + x.size, x.t_alloc, id};
     p.d.i_tf[r] = x.t_free;
@@ -512,6 +514,7 @@ __global__ void __launch_bounds__(kIsortThreads) k_isort(P p) {
         if (p.ordered && g < n) {
             while (lo + 1 < p.alloc_ctas && s_pre[lo + 1] <= g) ++lo;  // (empty CTAs share a prefix value)
             q = lo * kThreads + (g - s_pre[lo]);
+            MCHECK(lo < p.alloc_ctas && g >= s_pre[lo] && g - s_pre[lo] < (uint32_t)kThreads && q < p.a.n_alloc);
         }
         k[r] = g < n ? __ldcg(p.d.sk0 + q) : ~0ull;
         v[r] = g < n ? __ldcg(p.d.sv0 + q) : 0xFFFFFFFFu;
@@ -745,6 +748,7 @@ __device__ __forceinline__ uint32_t i_count_le(const uint64_t* fence, uint32_t n
     }
     if (lo == 0) return 0;
     const uint32_t g0 = (lo - 1) * stride, g1 = min(g0 + stride, nI);
+    MCHECK(g0 < nI);
     uint32_t c = g0 + 1;  // base g0 (the fence) <= x
     for (uint32_t k = g0; k < g1; k += 8) {  // two blocks per round (a group of 4: one)
         uint64_t b[8];
@@ -866,6 +870,7 @@ __device__ __forceinline__ bool q_test(const Tree& T, const ClsShared& S, int l,
     bool keep = nd.x > q.T0 && nd.y < q.T1;
     if (keep && l == 0 && q.exact) {  // live at one of the chunk's launches
         const uint32_t lo = count_upto<kNodeGrp>(S.nt0, q.ng0, nd.y);  // the first segment launched after t_alloc
+        MCHECK(lo <= q.ng0 && q.ng0 <= (uint32_t)kNodeGrp);
         keep = lo < q.ng0 && S.nt0[lo] < nd.x;
     }
     return keep;
@@ -981,7 +986,7 @@ __device__ __forceinline__ int window_find(const ClsShared& S, uint32_t m, uint3
             bits &= bits - 1;
             uint64_t b, en;  // one 16-byte load of (base, end)
             asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(b), "=l"(en) : "r"(a_rbe + 16 * e));
-            if (b <= x && x < en) return (int)e;
+            if (b <= x && x < en) { MCHECK(e < m); return (int)e; }
         }
     }
     return -1;
@@ -1486,6 +1491,7 @@ __global__ void __launch_bounds__(kThreads, 6) k_iresolve(P p) {
                             hit = true;
                             p.d.queue[k].x = ((uint64_t)e.id << MEDUSA_OFF_BITS) | (q.x - base);
                             if (MEDUSA_IRES_SMEM_MASK) {
+                                MCHECK(q.g >= c * kChunkWords && q.g - c * kChunkWords < (uint32_t)kChunkWords);
                                 atomicOr(&s_mb[(q.g - c * kChunkWords) >> 5], 1u << (q.g & 31));
                             } else {
                                 atomicOr(p.a.mask + (q.g >> 5), 1u << (q.g & 31));
@@ -1604,7 +1610,9 @@ __global__ void __launch_bounds__(kThreads) k_emit(P p) {
         uint32_t lo = 0;  // last mask word m with s_pre[m] <= r (s_pre[0] = 0): binary lifting, no branches
 #pragma unroll
         for (uint32_t st = 32; st > 0; st >>= 1) lo += s_pre[h][lo + st] <= r ? st : 0u;
+        MCHECK(lo < 64 && r >= s_pre[h][lo] && r - s_pre[h][lo] < (uint32_t)__popc(s_m[h][lo]));
         const uint32_t bit = nth_set_bit(s_m[h][lo], r - s_pre[h][lo]);  // the (r - s_pre[lo])-th set bit
+        MCHECK(bit < 32 && ((s_m[h][lo] >> bit) & 1u));
         const uint32_t below = (1u << bit) - 1u;
         const uint32_t w = lo / 8;  // the classify warp that owned the word
         const uint64_t region = (uint64_t)((c0 + h) * kWarps + w) * p.d.cap_pw;

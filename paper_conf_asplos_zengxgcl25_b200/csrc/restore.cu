@@ -184,6 +184,7 @@ __device__ __forceinline__ uint32_t table_word(const TableView<CPB>& T, uint32_t
     uint32_t lo = 0;  // last mask word m with pre[m] <= r (pre[0] = 0): binary lifting, no branches
 #pragma unroll
     for (uint32_t st = TableView<CPB>::kMask / 2; st > 0; st >>= 1) lo += T.pre[lo + st] <= r ? st : 0u;
+    MCHECK(lo < TableView<CPB>::kMask && r >= T.pre[lo] && r - T.pre[lo] < (uint32_t)__popc(T.mask[lo]));
     return lo * 32 + nth_set_bit(T.mask[lo], r - T.pre[lo]);
 }
 
