@@ -1206,7 +1206,13 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                         atomicOr(&wh[(q & 255) >> 5], 1u << (q & 31));
                     }
                 }
-                __syncthreads();  // the live masks / window are rewritten by the next group / batch
+                // the live masks / window are rewritten by the next group / batch; after
+                // the last one each warp goes on to its own records (nothing it reads there
+                // is rewritten), so a warp with few lookups does not wait for the others
+#ifndef MEDUSA_CLS_LAST_BARRIER
+#define MEDUSA_CLS_LAST_BARRIER 0
+#endif
+                if (MEDUSA_CLS_LAST_BARRIER || !(g0 + kNodeGrp >= n_seg && o_hi >= n_alloc)) __syncthreads();
             }
         }
         TL_PHASE(4, 13, tl_p);  // D: live masks, window search
