@@ -931,7 +931,8 @@ __device__ bool tree_query(const Tree& T, ClsShared& S, const QRange& q) {
 // The live masks of nodes g0 .. g0+ng for the loaded batch of m entries (whole CTA;
 // nt = their launch positions).  Entry e is live at nodes u0 <= u < u1
 // (t_alloc < t_u < t_free): toggle bit e at u0 and u1, then a prefix XOR over u.
-__device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uint32_t ng, uint32_t m) {
+// (cleared: the live masks were zeroed before the caller's last barrier)
+__device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uint32_t ng, uint32_t m, bool cleared) {
     const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {  // the batch's address hull
         uint64_t lo = ~0ull, hi = 0;
@@ -939,8 +940,10 @@ __device__ __forceinline__ void build_live(ClsShared& S, const uint32_t* nt, uin
         S.hull_lo = lo;
         S.hull_hi = hi;
     }
-    for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
-    __syncthreads();
+    if (!cleared) {
+        for (uint32_t k = tid; k < kNodeGrp * (kWinCap / 32); k += kThreads) (&S.live[0][0])[k] = 0u;
+        __syncthreads();
+    }
     for (uint32_t e = tid; e < m; e += kThreads) {
         const uint32_t ta = S.rta[e], tf = S.rtf[e];
         const uint32_t u0 = count_upto<kNodeGrp>(nt, ng, ta);        // #{u : t_u <= t_alloc}
@@ -1185,6 +1188,9 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         TL_PHASE(4, 12, tl_p);  // D: tree query
         if (m) {
             if (tid < kWinCap) window_load(p, S, m);
+            else  // the other threads zero the live masks meanwhile (the first group's)
+                for (uint32_t k = tid - kWinCap; k < kNodeGrp * (kWinCap / 32); k += kThreads - kWinCap)
+                    (&S.live[0][0])[k] = 0u;
             __syncthreads();
             for (uint32_t g0 = 0; g0 < n_seg; g0 += kNodeGrp) {
                 const uint32_t ng = min((uint32_t)kNodeGrp, n_seg - g0);
@@ -1193,7 +1199,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
                     seg_times(p, S, S.nt, g0, ng, cs, jf, jl);
                     nt = S.nt;
                 }
-                build_live(S, nt, ng, m);
+                build_live(S, nt, ng, m, g0 == 0);
                 for (uint32_t i = lane; i < nc; i += 32) {
                     const uint32_t q = wl[i];
                     if ((wh[(q & 255) >> 5] >> (q & 31)) & 1u) continue;  // found in an earlier batch
