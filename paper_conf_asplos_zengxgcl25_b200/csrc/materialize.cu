@@ -187,8 +187,7 @@ __device__ __forceinline__ unsigned long long block_prefix(const uint32_t* cnt, 
     unsigned long long t = 0;
 #pragma unroll
     for (int w = 0; w < kWarps; ++w) t += s_r[w];
-    __syncthreads();
-    return t;
+    return t;  // (called once per CTA: s_r is not rewritten, no barrier after the reads)
 }
 
 // one allocation record through the read-only path
@@ -1184,7 +1183,7 @@ __device__ void classify_role(const P& p, uint32_t c, ClsShared& S) {
         }
         have = false;
         const uint32_t m = S.nres;
-        __syncthreads();  // every thread has read nres before a later query resets it
+        if (o_hi < n_alloc) __syncthreads();  // every thread has read nres before a later query resets it
         TL_PHASE(4, 12, tl_p);  // D: tree query
         if (m) {
             if (tid < kWinCap) window_load(p, S, m);
